@@ -1,0 +1,254 @@
+/*
+ * protean.h — C ABI of the B200-native PROTEAN placement scorer and trace replayer.
+ *
+ * What this library computes is the "PROTEAN epoch model" (PEM): the paper's slowdown model
+ * (Eq 1 / Eq 2), Job Distribution (Alg 1), the GPU Reconfigurator's decision step (Alg 2,
+ * hysteresis + ~30% cap) and cost-aware procurement, driven by an exhaustive per-epoch search
+ * over MIG geometries (the paper's "Oracle" scheme run online).  Paper citations are
+ * "P:L<n>" = line n of PAPER.md (Bhasi et al., "Towards SLO-Compliant and Cost-Effective
+ * Serverless Computing on Emerging GPU Architectures", MIDDLEWARE '24).  Every reading of a
+ * silent / ambiguous passage is listed in DESIGN.md §3 (Q1..Q39 follow SURVEY.md §8(c)).
+ *
+ * Units everywhere: time in integer microseconds (int64 inside, uint32 for stored arrivals and
+ * batch ready times), memory in MiB, fractional bandwidth (FBR) in ppm (10^6 == 1.0), prices
+ * in USD per node-hour.  No floating point enters any decision; cost and utilisation are
+ * converted to double once, from integer accumulators.
+ *
+ * Ownership: the caller owns every input and output buffer.  The library owns only the handle,
+ * its device copy of the tables, its scratch memory and (mode G) its NCCL communicator; all are
+ * released by protean_free().  The library never frees or reallocates caller memory.
+ *
+ * Pointers: every pointer inside protean_epoch_in / protean_epoch_out / protean_replay_cfg /
+ * protean_replay_out is a DEVICE pointer (cudaMalloc'd or torch CUDA tensor data) on the
+ * handle's device, unless the field comment says "host".  protean_profiles holds host pointers.
+ *
+ * Errors: every call returns an int code (PROTEAN_OK == 0 or a negative PROTEAN_E*).  There are
+ * no exceptions or aborts across the ABI.  On a non-OK return the outputs are undefined.
+ * PROTEAN_ECUDA / PROTEAN_ENCCL poison the handle: every later call returns PROTEAN_ESTATE until
+ * protean_free().  protean_last_error() gives a human-readable detail of the last failure.
+ *
+ * Threading: a handle is not thread-safe; distinct handles are independent.
+ */
+#ifndef PROTEAN_H_
+#define PROTEAN_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define PROTEAN_ABI_VERSION 1
+
+enum {
+  PROTEAN_OK = 0,
+  PROTEAN_EINVAL = -1,  /* bad pointer / size / ordering / value (e.g. unsorted arrivals,
+                           model id >= n_models, fbr > 10^6, solo <= 0, geometry violating T2) */
+  PROTEAN_ERANGE = -2,  /* a value does not fit its field: time >= 2^32 us in a uint32 field,
+                           n_gpus > 255, G > 254, live residents > max_live in a given state */
+  PROTEAN_ENOMEM = -3,  /* device / host allocation failed */
+  PROTEAN_ECUDA = -4,   /* a CUDA runtime call failed (handle poisoned) */
+  PROTEAN_ENCCL = -5,   /* an NCCL call failed (handle poisoned) */
+  PROTEAN_ESTATE = -6,  /* handle poisoned, or bad call order */
+  PROTEAN_EUNSUP = -7   /* valid request this build does not implement (e.g. policy = Alg 2) */
+};
+
+/* MIG slice profiles of the A100-40GB, T2, in ascending-resource order (the order
+ * Alg 1 walks; 3g < 4g by compute since both hold 20 GB, reading Q3).
+ *   compute (sevenths) 1,2,3,4,7;  memory MiB 5120,10240,20480,20480,40960;  max count 7,3,2,1,1 */
+enum { PROTEAN_P_1G = 0, PROTEAN_P_2G, PROTEAN_P_3G, PROTEAN_P_4G, PROTEAN_P_7G, PROTEAN_NPROF };
+
+#define PROTEAN_MAX_MODELS 64
+#define PROTEAN_MAX_SLICES 7      /* a geometry has at most 7 slices (T2: "maximum of 7") */
+#define PROTEAN_MAX_LIVE 64       /* max live batches per simulated GPU (reading Q39) */
+#define PROTEAN_NBUCKETS 3328     /* log-linear latency histogram buckets (O7, reading Q30) */
+#define PROTEAN_NCOUNTERS 10
+#define PROTEAN_NACCUM 4
+
+typedef struct protean_handle protean_handle;
+
+/* ---------------------------------------------------------------------------------------------
+ * 1. Profiles: per model x per slice profile tables + the candidate geometry set.
+ *    Solo/FBR per slice are the "prerequisites ... estimated through profiling";
+ *    FBR = bw*sm of Eq 1; RDF = solo[p]/solo[7g].
+ *    All pointers are HOST pointers; the library copies them.                                  */
+typedef struct {
+  int32_t abi_version;             /* must be PROTEAN_ABI_VERSION */
+  int32_t n_models;                /* M, 1..64 */
+  const int32_t *solo_us;          /* [M][5] solo (isolated) batch exec time per profile, > 0 */
+  const int32_t *fbr_ppm;          /* [M][5] fractional bandwidth requirement per profile, 0..10^6 */
+  const int32_t *mem_mib;          /* [M] memory footprint of one batch, 1..40960 */
+  const int32_t *batch_size;       /* [M] B_m, 1..65535 (128 vision, 4 language) */
+  const int32_t *slo_us;           /* [M] strict SLO, > 0 (paper: 3 x solo on 7g) */
+  const int32_t *batch_timeout_us; /* [M] T_m >= 0: a batch closes at B_m requests or first+T_m (Q14) */
+  int32_t geometry_set;            /* 0: the 12 multiset-maximal geometries (default)
+                                      1: all 37 feasible geometries
+                                      2: explicit list (geoms) */
+  int32_t n_geoms;                 /* explicit only: G, 1..254 */
+  const uint8_t *geoms;            /* explicit only: [G][8] profile ids ascending, 0xFF padded;
+                                      each validated against T2 (counts, compute <= 7/7, mem <= 40 GB) */
+  int32_t device;                  /* CUDA device ordinal */
+} protean_profiles;
+
+/* Validates the tables, enumerates the geometry set (canonical order: count vectors
+ * (c7g,c4g,c3g,c2g,c1g) descending lexicographically; index 0 = (7g), 1 = (4g,3g),
+ * 2 = (4g,2g,1g) in both built-in sets), uploads everything to the device and returns a handle.
+ * Synchronous.  Errors: EINVAL (bad table value / pointer / geometry), ERANGE (G > 254),
+ * ENOMEM, ECUDA. */
+int protean_load_profiles(const protean_profiles *p, protean_handle **out);
+void protean_free(protean_handle *h);
+const char *protean_strerror(int code);
+const char *protean_last_error(const protean_handle *h);
+
+/* Geometry table of the handle: *n_geoms = G; if geoms != NULL it receives [G][8] host bytes
+ * (profile ids ascending, 0xFF padded).  Host pointers. */
+int protean_get_geometries(const protean_handle *h, int32_t *n_geoms, uint8_t *geoms);
+
+/* Number of epochs of a replay: E = ceil(trace_len/W) + ceil(max_m T_m / W) (O4).  Host. */
+int protean_num_epochs(const protean_handle *h, int64_t trace_len_us, int64_t epoch_len_us,
+                       int64_t *n_epochs);
+
+/* ---------------------------------------------------------------------------------------------
+ * 2. One epoch of the search for R replicas x N simulated GPUs (§8(a) S4, S6, S7, S8).
+ *    For every GPU: the pending reconfiguration is installed if recfg_end <= T = (epoch+1)W;
+ *    its batches are placed on its CURRENT geometry with Alg 1 on the carried state (the actual
+ *    placement, which advances `state`); and if the GPU is decidable at T (has_vm and
+ *    recfg_end <= T) every candidate geometry j in [geom_lo, geom_hi) replays the same batch list
+ *    from an idle GPU and is scored by key = misses<<40 | BE_tail<<8 | tag, tag 0 = current
+ *    geometry, else j+1 (O8).  Asynchronous on `stream` (cudaStream_t; NULL = legacy default).  */
+typedef struct {           /* 16 B */
+  uint32_t ready_us;       /* batch ready time (O3): last member's arrival if full, else first + T_m */
+  uint32_t req_off;        /* index of the batch's first member in arrival_us */
+  uint16_t n_req;          /* members; they are arrival_us[req_off .. req_off + n_req), sorted */
+  uint8_t model;           /* model id < M */
+  uint8_t strict;          /* 1 = strict (SLO), 0 = best effort (BE) */
+  uint32_t gpu;            /* informational: the GPU it was dispatched to */
+} protean_batch;
+
+typedef struct {           /* 24 B: one batch resident on a simulated GPU */
+  int64_t start_us, end_us;/* [start, end) on its slice; end = start + exec (Eq 1, frozen at start) */
+  int32_t mem_mib;
+  uint8_t slice;           /* slice position within the geometry (ascending profile order) */
+  uint8_t model, strict, pad;
+} protean_resident;
+
+typedef struct {           /* one simulated GPU's carried state; caller-allocated */
+  uint8_t geom;            /* current geometry index */
+  uint8_t target;          /* pending reconfiguration target, 0xFF = none */
+  uint8_t wait_ctr;        /* Alg 2 wait_ctr — not modified by score_epoch */
+  uint8_t n_live;          /* residents in live[] (<= max_live) */
+  uint8_t has_vm;          /* 1 = the node holds a VM at the decision time */
+  uint8_t vm_type, pad[2];
+  int64_t recfg_start_us, recfg_end_us;  /* reconfiguration window [start, end), 0/0 = none */
+  int64_t last_start_us[PROTEAN_MAX_SLICES];   /* FIFO: latest start on each slice */
+  int64_t busy_until_us[PROTEAN_MAX_SLICES];   /* busy-time union bookkeeping (O6e) */
+  protean_resident live[PROTEAN_MAX_LIVE];
+} protean_gpu_state;
+
+typedef struct {           /* 24 B */
+  int64_t start_us, end_us;
+  uint8_t slice;           /* chosen slice position (valid when dropped == 0) */
+  uint8_t dropped;         /* 0 placed, 2 placement drop (no slice fits), 3 overflow (max_live) */
+  uint8_t pad[6];
+} protean_placement;
+
+typedef struct {
+  int32_t n_replicas, n_gpus, epoch;   /* R >= 1, 1 <= N <= 255, epoch >= 0 */
+  int32_t max_live;                    /* 1..64 (default 64) */
+  int64_t epoch_len_us;                /* W > 0 */
+  int64_t horizon_us;                  /* H: busy/memory accounting is clipped to [0, H) */
+  const protean_batch *batches;        /* ordered by (replica, gpu, batch id) */
+  const int32_t *batch_off;            /* [R*N+1] CSR offsets into batches */
+  const uint32_t *arrival_us;          /* member arrivals referenced by req_off */
+  protean_gpu_state *state;            /* [R*N] in/out */
+  int32_t geom_lo, geom_hi;            /* candidate range; [0, G) = all */
+} protean_epoch_in;
+
+typedef struct {
+  int64_t *best_key;          /* [R*N] min key over the range; -1 if the GPU is not decidable */
+  int64_t *cand_key;          /* [R*N*(hi-lo)] every candidate key (-1 if not decidable), or NULL */
+  protean_placement *placement; /* [n_batches] actual placement, same order as batches */
+  int64_t *counters;          /* [R][10] ACCUMULATED (+=): see protean_replay_out.counters */
+  int64_t *accum;             /* [R][4] ACCUMULATED, or NULL: busy_w, mem_num (see replay) */
+} protean_epoch_out;
+
+int protean_score_epoch(protean_handle *h, const protean_epoch_in *in, protean_epoch_out *out,
+                        void *stream);
+
+/* ---------------------------------------------------------------------------------------------
+ * 3. Trace replay, epoch by epoch, of many independent replicas (the north-star path, §8(a)
+ *    S2..S11 fused).  Per replica, for e = 0..E-1 (O5): VM events -> batch formation (O3) ->
+ *    round-robin dispatch (Q18) -> actual Alg-1 placement + per-request accounting (O6, O7) ->
+ *    candidate scoring of every geometry for every decidable GPU (O8) -> hysteresis + 30% cap +
+ *    reconfiguration windows (O9, O10).  Then percentiles, cost and utilisation (O12).
+ *    Synchronous (returns after the outputs are written).                                      */
+typedef struct {
+  int32_t n_replicas;          /* replicas in THIS call */
+  int32_t n_gpus;              /* N simulated GPUs per replica, 1..255 */
+  int64_t replica_base;        /* global id of the first replica (RNG stream of O11); mode R
+                                  sharding passes each rank its own slice of replicas */
+  int64_t trace_len_us;        /* arrivals lie in [0, trace_len) */
+  int64_t epoch_len_us;        /* W, Monitor_Interval of Alg 2; default 1'000'000 (Q1) */
+  const uint32_t *arrival_us;  /* device: per replica, sorted non-decreasing */
+  const uint8_t *meta;         /* device: bits 0..5 model id, bit 7 strict (user-annotated) */
+  const int64_t *replica_off;  /* device: [R+1] offsets into arrival_us / meta */
+  int32_t policy;              /* 0 = geometry search (default); 1 = fixed geometry (no search);
+                                  2 = Alg 2 heuristic (EUNSUP in this build) */
+  int32_t wait_limit;          /* Alg 2 wait_limit, default 3 (reading Q22) */
+  int32_t reconfig_cap_pct;    /* default 30 (reading Q23) */
+  int32_t init_geom;           /* default 2 = (4g,2g,1g) (reading Q25) */
+  int32_t max_live;            /* 1..64, default 64 */
+  int32_t vm_policy;           /* 0 on-demand only; 1 PROTEAN spot + on-demand fallback;
+                                  2 spot only */
+  int64_t reconfig_us;         /* MIG reconfiguration downtime, default 2'000'000 */
+  double p_rev;                /* revocation probability per interval, 0..1 */
+  double price_od_node_hr, price_spot_node_hr; /* default AWS T3 / 8: 4.096575, 1.228975 (Q27) */
+  int64_t rev_interval_us;     /* revocation interval T_rev (default 300 s, Q28); must be >= W */
+  int64_t notice_us;           /* eviction notice (default 30 s); must be < T_rev */
+  uint64_t seed;               /* VM RNG seed (O11) */
+  int32_t shard_mode;          /* 0 = replicas (mode R); 1 = geometry ranges (mode G, EUNSUP here) */
+  int32_t rank, nranks;        /* mode G only */
+  const uint8_t *nccl_id;      /* mode G only: host, 128-byte ncclUniqueId */
+} protean_replay_cfg;
+
+/* counters[10] per replica (O7/O8/O10):
+ *   0 strict_arr  1 strict_met  2 strict_missed  3 strict_drop
+ *   4 be_arr      5 be_served   6 be_drop        7 reconfigs
+ *   8 slot_evals (sum over candidate x batch of the geometry's slice count)
+ *   9 geom_candidates (replica x epoch x decidable GPU x geometry schedules)
+ * accum[4] per replica: 0 busy_w  = sum over slices of compute7 x busy us (clipped to [0,H))
+ *                       1 mem_num = sum over batches of mem_mib x |[start,end) ∩ [0,H)|
+ *                       2 vm_od_us, 3 vm_spot_us (billed node-us over [0,H))              */
+typedef struct {
+  uint32_t ready_us;
+  uint32_t epoch;
+  uint16_t n_req; uint8_t model, strict;
+  uint8_t gpu, slice, dropped, pad;  /* dropped: 0 placed, 1 dispatch, 2 placement, 3 overflow */
+  int64_t start_us, end_us;
+} protean_batch_rec;         /* 32 B, debug log of every batch in id order */
+
+typedef struct {             /* caller-allocated, one row per replica of this call */
+  int64_t *counters;         /* [R][10] */
+  int64_t *accum;            /* [R][4] */
+  uint32_t *hist;            /* [R][2][3328] latency histograms (0 strict, 1 BE) */
+  int64_t *p50_p99_us;       /* [R][2][2] nearest-rank P50/P99 (bucket lower edges, O12) */
+  double *cost_usd;          /* [R] */
+  double *util;              /* [R][2]: compute-weighted busy, memory-time */
+  uint8_t *decisions;        /* [R][E][N] best geometry per decidable GPU-epoch, 0xFF otherwise;
+                                or NULL */
+  int64_t *cand_keys;        /* [R][E][N][G] every candidate key (-1 when not scored), or NULL */
+  protean_batch_rec *batch_log; /* [R][batch_log_cap] or NULL */
+  int64_t batch_log_cap;
+  int64_t *n_batches;        /* [R] batches formed (also when batch_log is NULL), or NULL */
+} protean_replay_out;
+
+int protean_replay_traces(protean_handle *h, const protean_replay_cfg *cfg,
+                          protean_replay_out *out, void *stream);
+
+/* Fill a replay config with the defaults listed above (host). */
+void protean_replay_cfg_defaults(protean_replay_cfg *cfg);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PROTEAN_H_ */
