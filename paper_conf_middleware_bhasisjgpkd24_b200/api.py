@@ -1,0 +1,183 @@
+"""Thin Python binding of the C ABI (same names as include/protean.h).
+
+torch is used for device memory and streams only; every computation runs in libprotean.so.
+"""
+from __future__ import annotations
+
+import ctypes as C
+
+import numpy as np
+
+from . import _abi as A
+
+_REPLAY_DEFAULTS = dict(n_gpus=8, epoch_len_us=1_000_000, policy=0, wait_limit=3, reconfig_cap_pct=30,
+                        init_geom=2, max_live=64, vm_policy=0, reconfig_us=2_000_000, p_rev=0.0,
+                        price_od_node_hr=32.7726 / 8, price_spot_node_hr=9.8318 / 8,
+                        rev_interval_us=300_000_000, notice_us=30_000_000, seed=0, shard_mode=0,
+                        replica_base=0)
+
+
+def _torch():
+    import torch
+    if not torch.cuda.is_available():
+        raise RuntimeError("paper_conf_middleware_bhasisjgpkd24_b200 needs a CUDA device (no CPU fallback)")
+    return torch
+
+
+def _check(h, rc):
+    if rc != A.OK:
+        detail = A.load().protean_last_error(h).decode() if h else ""
+        raise A.ProteanError(rc, detail)
+
+
+class Handle:
+    """protean_load_profiles(): validated tables + geometry set resident on `device`."""
+
+    def __init__(self, profiles, device: int = 0):
+        self._lib = A.load()
+        self.device = device
+        arrs = [np.ascontiguousarray(x, np.int32) for x in
+                (profiles.solo_us, profiles.fbr_ppm, profiles.mem_mib, profiles.batch_size,
+                 profiles.slo_us, profiles.timeout_us)]
+        geoms = None if profiles.geoms is None else np.ascontiguousarray(profiles.geoms, np.uint8)
+        p = A.Profiles(A.ABI_VERSION, int(arrs[0].shape[0]), *[a.ctypes.data for a in arrs],
+                       int(profiles.geometry_set), 0 if geoms is None else int(geoms.shape[0]),
+                       None if geoms is None else geoms.ctypes.data, int(device))
+        self._h = C.c_void_p()
+        rc = self._lib.protean_load_profiles(C.byref(p), C.byref(self._h))
+        if rc != A.OK:
+            raise A.ProteanError(rc, "protean_load_profiles")
+        n = C.c_int32()
+        self._lib.protean_get_geometries(self._h, C.byref(n), None)
+        self.n_geoms = n.value
+
+    def close(self):
+        if getattr(self, "_h", None):
+            self._lib.protean_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def geometries(self) -> np.ndarray:
+        n = C.c_int32()
+        out = np.zeros((self.n_geoms, 8), np.uint8)
+        _check(self._h, self._lib.protean_get_geometries(self._h, C.byref(n), out.ctypes.data))
+        return out
+
+    def num_epochs(self, trace_len_us: int, epoch_len_us: int = 1_000_000) -> int:
+        E = C.c_int64()
+        _check(self._h, self._lib.protean_num_epochs(self._h, int(trace_len_us), int(epoch_len_us), C.byref(E)))
+        return E.value
+
+    # -------------------------------------------------------------------------------- replay
+    def alloc_replay_out(self, R: int, E: int, N: int, *, decisions=True, cand_keys=False, log_cap=0):
+        torch = _torch()
+        dev = torch.device("cuda", self.device)
+        out = dict(counters=torch.zeros((R, 10), dtype=torch.int64, device=dev),
+                   accum=torch.zeros((R, 4), dtype=torch.int64, device=dev),
+                   hist=torch.zeros((R, 2, A.NBUCKETS), dtype=torch.int32, device=dev),
+                   p50_p99=torch.zeros((R, 2, 2), dtype=torch.int64, device=dev),
+                   cost=torch.zeros(R, dtype=torch.float64, device=dev),
+                   util=torch.zeros((R, 2), dtype=torch.float64, device=dev),
+                   n_batches=torch.zeros(R, dtype=torch.int64, device=dev))
+        if decisions:
+            out["decisions"] = torch.zeros((R, E, N), dtype=torch.uint8, device=dev)
+        if cand_keys:
+            out["cand_keys"] = torch.zeros((R, E, N, self.n_geoms), dtype=torch.int64, device=dev)
+        if log_cap:
+            out["log"] = torch.zeros((R, log_cap, C.sizeof(A.BatchRec)), dtype=torch.uint8, device=dev)
+        out["log_cap"] = int(log_cap)
+        return out
+
+    def replay_traces(self, arrival_us, meta, replica_off, *, trace_len_us: int, out=None,
+                      want_decisions=True, want_cand_keys=False, log_cap=0, stream=None, **cfg):
+        """protean_replay_traces on device tensors (arrival uint32/int32, meta uint8, off int64)."""
+        torch = _torch()
+        c = dict(_REPLAY_DEFAULTS)
+        c.update(cfg)
+        R = int(replica_off.shape[0]) - 1
+        N = int(c["n_gpus"])
+        E = self.num_epochs(trace_len_us, c["epoch_len_us"])
+        if out is None:
+            out = self.alloc_replay_out(R, E, N, decisions=want_decisions, cand_keys=want_cand_keys,
+                                        log_cap=log_cap)
+        assert arrival_us.element_size() == 4 and meta.element_size() == 1 and replica_off.element_size() == 8
+        for t in (arrival_us, meta, replica_off):
+            assert t.is_cuda and t.is_contiguous()
+        cf = A.ReplayCfg()
+        self._lib.protean_replay_cfg_defaults(C.byref(cf))
+        cf.n_replicas, cf.n_gpus = R, N
+        cf.replica_base = int(c["replica_base"])
+        cf.trace_len_us = int(trace_len_us)
+        cf.epoch_len_us = int(c["epoch_len_us"])
+        cf.arrival_us = arrival_us.data_ptr() if arrival_us.numel() else replica_off.data_ptr()
+        cf.meta = meta.data_ptr() if meta.numel() else replica_off.data_ptr()
+        cf.replica_off = replica_off.data_ptr()
+        for k in ("policy", "wait_limit", "reconfig_cap_pct", "init_geom", "max_live", "vm_policy",
+                  "reconfig_us", "rev_interval_us", "notice_us", "seed", "shard_mode"):
+            setattr(cf, k, int(c[k]))
+        for k in ("p_rev", "price_od_node_hr", "price_spot_node_hr"):
+            setattr(cf, k, float(c[k]))
+        o = A.ReplayOut(out["counters"].data_ptr(), out["accum"].data_ptr(), out["hist"].data_ptr(),
+                        out["p50_p99"].data_ptr(), out["cost"].data_ptr(), out["util"].data_ptr(),
+                        out["decisions"].data_ptr() if "decisions" in out else None,
+                        out["cand_keys"].data_ptr() if "cand_keys" in out else None,
+                        out["log"].data_ptr() if "log" in out else None, out.get("log_cap", 0),
+                        out["n_batches"].data_ptr())
+        st = stream if stream is not None else torch.cuda.current_stream(self.device)
+        _check(self._h, self._lib.protean_replay_traces(self._h, C.byref(cf), C.byref(o),
+                                                        C.c_void_p(st.cuda_stream)))
+        out["E"] = E
+        return out
+
+    def replay_traces_host(self, trace, *, pinned=None, stream=None, **cfg):
+        """End-to-end public call on HOST buffers: H2D of the trace, the replay, D2H of results."""
+        torch = _torch()
+        dev = torch.device("cuda", self.device)
+        arr = torch.from_numpy(np.ascontiguousarray(trace.arrival_us).view(np.int32))
+        meta = torch.from_numpy(np.ascontiguousarray(trace.meta))
+        off = torch.from_numpy(np.ascontiguousarray(trace.replica_off, np.int64))
+        if pinned is not None:
+            arr, meta, off = pinned
+        d = [x.to(dev, non_blocking=True) for x in (arr, meta, off)]
+        cfg.setdefault("replica_base", trace.replica_base)
+        out = self.replay_traces(d[0], d[1], d[2], trace_len_us=trace.trace_len_us, stream=stream, **cfg)
+        return {k: (v.cpu().numpy() if hasattr(v, "cpu") else v) for k, v in out.items()}
+
+    # -------------------------------------------------------------------------------- score_epoch
+    def score_epoch(self, *, n_replicas, n_gpus, epoch, batches, batch_off, arrival_us, state,
+                    geom_lo=0, geom_hi=None, epoch_len_us=1_000_000, horizon_us=1 << 62, max_live=64,
+                    counters=None, accum=None, want_cand_keys=True, stream=None):
+        """protean_score_epoch.  batches: uint8 device tensor of protean_batch rows (16 B each);
+        state: uint8 device tensor of protean_gpu_state rows (modified in place)."""
+        torch = _torch()
+        dev = torch.device("cuda", self.device)
+        geom_hi = self.n_geoms if geom_hi is None else geom_hi
+        R, N = int(n_replicas), int(n_gpus)
+        nb = batches.numel() // 16
+        nc = geom_hi - geom_lo
+        out = dict(best_key=torch.zeros(R * N, dtype=torch.int64, device=dev),
+                   placement=torch.zeros((max(nb, 1), 24), dtype=torch.uint8, device=dev),
+                   counters=counters if counters is not None else torch.zeros((R, 10), dtype=torch.int64, device=dev),
+                   accum=accum if accum is not None else torch.zeros((R, 4), dtype=torch.int64, device=dev))
+        if want_cand_keys:
+            out["cand_key"] = torch.zeros(R * N * max(nc, 1), dtype=torch.int64, device=dev)
+        ei = A.EpochIn(R, N, int(epoch), int(max_live), int(epoch_len_us), int(horizon_us),
+                       batches.data_ptr() if nb else out["placement"].data_ptr(), batch_off.data_ptr(),
+                       arrival_us.data_ptr() if arrival_us.numel() else batch_off.data_ptr(),
+                       state.data_ptr(), int(geom_lo), int(geom_hi))
+        eo = A.EpochOut(out["best_key"].data_ptr(), out["cand_key"].data_ptr() if want_cand_keys else None,
+                        out["placement"].data_ptr(), out["counters"].data_ptr(), out["accum"].data_ptr())
+        st = stream if stream is not None else torch.cuda.current_stream(self.device)
+        _check(self._h, self._lib.protean_score_epoch(self._h, C.byref(ei), C.byref(eo),
+                                                      C.c_void_p(st.cuda_stream)))
+        out["placement"] = out["placement"][:nb]
+        return out
+
+
+def load_profiles(profiles, device: int = 0) -> Handle:
+    return Handle(profiles, device)

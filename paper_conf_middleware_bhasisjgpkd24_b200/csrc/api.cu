@@ -1,0 +1,496 @@
+// api.cu — host side of the C ABI (include/protean.h): validation, the geometry set by T2 sum
+// constraints (reading Q2), device tables, scratch, launches.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <array>
+#include <cmath>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "replay.cuh"
+
+using namespace pemgpu;
+
+struct protean_handle {
+  int device = 0;
+  int M = 0, G = 0, maxT = 0;
+  TabLayout tl;
+  std::vector<int32_t> words;
+  std::vector<uint8_t> geoms;  // [G][8]
+  int32_t* d_tab = nullptr;
+  std::string err;
+  bool poisoned = false;
+  int nsm = 148;
+  void* d_scratch = nullptr;
+  size_t scratch_bytes = 0;
+  int64_t* d_eoff = nullptr;
+  size_t eoff_bytes = 0;
+  void* d_small = nullptr;  // wmax (8 B) + err (16 B)
+};
+
+namespace {
+
+int fail(protean_handle* h, int code, const std::string& what) {
+  if (h) h->err = what;
+  return code;
+}
+
+int cuda_fail(protean_handle* h, cudaError_t e, const char* where) {
+  if (h) {
+    h->poisoned = true;
+    h->err = std::string(where) + ": " + cudaGetErrorString(e);
+  }
+  return PROTEAN_ECUDA;
+}
+
+#define CK(h, call)                                    \
+  do {                                                 \
+    cudaError_t e_ = (call);                           \
+    if (e_ != cudaSuccess) return cuda_fail(h, e_, #call); \
+  } while (0)
+
+const int kCompute[5] = {1, 2, 3, 4, 7};
+const int kMem[5] = {5120, 10240, 20480, 20480, 40960};
+const int kMaxCnt[5] = {7, 3, 2, 1, 1};
+
+// O2 by T2 sum constraints: count vectors with at most the T2 max counts, <= 7/7 compute and
+// <= 40 GB.  Default set = multiset-maximal ones.  Order: (c7g,c4g,c3g,c2g,c1g) descending.
+std::vector<std::vector<uint8_t>> geometry_set(bool all) {
+  std::vector<std::array<int, 5>> feas;
+  for (int a = 0; a <= kMaxCnt[0]; ++a)
+    for (int b = 0; b <= kMaxCnt[1]; ++b)
+      for (int c = 0; c <= kMaxCnt[2]; ++c)
+        for (int d = 0; d <= kMaxCnt[3]; ++d)
+          for (int f = 0; f <= kMaxCnt[4]; ++f) {
+            const int cnt[5] = {a, b, c, d, f};
+            int comp = 0, mem = 0, tot = 0;
+            for (int p = 0; p < 5; ++p) {
+              comp += cnt[p] * kCompute[p];
+              mem += cnt[p] * kMem[p];
+              tot += cnt[p];
+            }
+            if (tot >= 1 && comp <= 7 && mem <= 40960) feas.push_back({a, b, c, d, f});
+          }
+  std::vector<std::array<int, 5>> keep;
+  for (const auto& x : feas) {
+    bool dominated = false;
+    for (const auto& y : feas) {
+      if (y == x) continue;
+      bool ge = true;
+      for (int p = 0; p < 5; ++p) ge = ge && y[p] >= x[p];
+      if (ge) dominated = true;
+    }
+    if (all || !dominated) keep.push_back(x);
+  }
+  std::sort(keep.begin(), keep.end(), [](const std::array<int, 5>& x, const std::array<int, 5>& y) {
+    for (int p = 4; p >= 0; --p)
+      if (x[p] != y[p]) return x[p] > y[p];
+    return false;
+  });
+  std::vector<std::vector<uint8_t>> out;
+  for (const auto& x : keep) {
+    std::vector<uint8_t> g;
+    for (int p = 0; p < 5; ++p)
+      for (int i = 0; i < x[p]; ++i) g.push_back((uint8_t)p);
+    out.push_back(g);
+  }
+  return out;
+}
+
+int validate_row(const uint8_t* row, std::vector<uint8_t>* g) {
+  int cnt[5] = {0, 0, 0, 0, 0}, comp = 0, mem = 0, k = 0;
+  bool ended = false;
+  for (int i = 0; i < 8; ++i) {
+    if (row[i] == 0xFF) { ended = true; continue; }
+    if (ended || row[i] >= 5 || i >= 7 || (k > 0 && row[i] < (*g)[k - 1])) return PROTEAN_EINVAL;
+    cnt[row[i]]++;
+    comp += kCompute[row[i]];
+    mem += kMem[row[i]];
+    g->push_back(row[i]);
+    ++k;
+  }
+  if (k == 0) return PROTEAN_EINVAL;
+  for (int p = 0; p < 5; ++p)
+    if (cnt[p] > kMaxCnt[p]) return PROTEAN_EINVAL;
+  if (comp > 7 || mem > 40960) return PROTEAN_EINVAL;
+  return PROTEAN_OK;
+}
+
+int ensure(protean_handle* h, void** p, size_t* have, size_t need) {
+  if (*have >= need && *p) return PROTEAN_OK;
+  if (*p) cudaFree(*p);
+  *p = nullptr;
+  *have = 0;
+  cudaError_t e = cudaMalloc(p, need);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return fail(h, PROTEAN_ENOMEM, "cudaMalloc scratch failed");
+  }
+  *have = need;
+  return PROTEAN_OK;
+}
+
+size_t al(size_t x) { return (x + 255) & ~(size_t)255; }
+
+}  // namespace
+
+extern "C" {
+
+const char* protean_strerror(int code) {
+  switch (code) {
+    case PROTEAN_OK: return "ok";
+    case PROTEAN_EINVAL: return "invalid argument";
+    case PROTEAN_ERANGE: return "value out of range";
+    case PROTEAN_ENOMEM: return "out of memory";
+    case PROTEAN_ECUDA: return "CUDA error";
+    case PROTEAN_ENCCL: return "NCCL error";
+    case PROTEAN_ESTATE: return "bad state (poisoned handle or call order)";
+    case PROTEAN_EUNSUP: return "unsupported in this build";
+    default: return "unknown error";
+  }
+}
+
+const char* protean_last_error(const protean_handle* h) { return h ? h->err.c_str() : ""; }
+
+void protean_replay_cfg_defaults(protean_replay_cfg* c) {
+  std::memset(c, 0, sizeof(*c));
+  c->n_gpus = 8;
+  c->epoch_len_us = 1000000;
+  c->policy = 0;
+  c->wait_limit = 3;
+  c->reconfig_cap_pct = 30;
+  c->init_geom = 2;
+  c->max_live = 64;
+  c->vm_policy = 0;
+  c->reconfig_us = 2000000;
+  c->p_rev = 0.0;
+  c->price_od_node_hr = 32.7726 / 8.0;
+  c->price_spot_node_hr = 9.8318 / 8.0;
+  c->rev_interval_us = 300000000;
+  c->notice_us = 30000000;
+}
+
+int protean_load_profiles(const protean_profiles* p, protean_handle** out) {
+  if (!out) return PROTEAN_EINVAL;
+  *out = nullptr;
+  if (!p || p->abi_version != PROTEAN_ABI_VERSION) return PROTEAN_EINVAL;
+  const int M = p->n_models;
+  if (M < 1 || M > PROTEAN_MAX_MODELS) return PROTEAN_EINVAL;
+  if (!p->solo_us || !p->fbr_ppm || !p->mem_mib || !p->batch_size || !p->slo_us || !p->batch_timeout_us)
+    return PROTEAN_EINVAL;
+  for (int i = 0; i < 5 * M; ++i) {
+    if (p->solo_us[i] <= 0) return PROTEAN_EINVAL;
+    if (p->fbr_ppm[i] < 0 || p->fbr_ppm[i] > 1000000) return PROTEAN_EINVAL;
+  }
+  int maxT = 0;
+  for (int m = 0; m < M; ++m) {
+    if (p->mem_mib[m] < 1 || p->mem_mib[m] > 40960) return PROTEAN_EINVAL;
+    if (p->batch_size[m] < 1 || p->batch_size[m] > 65535) return PROTEAN_EINVAL;
+    if (p->slo_us[m] <= 0 || p->batch_timeout_us[m] < 0) return PROTEAN_EINVAL;
+    maxT = std::max(maxT, p->batch_timeout_us[m]);
+  }
+  std::vector<std::vector<uint8_t>> gs;
+  if (p->geometry_set == 0 || p->geometry_set == 1) {
+    gs = geometry_set(p->geometry_set == 1);
+  } else if (p->geometry_set == 2) {
+    if (p->n_geoms < 1) return PROTEAN_EINVAL;
+    if (p->n_geoms > 254) return PROTEAN_ERANGE;
+    if (!p->geoms) return PROTEAN_EINVAL;
+    for (int j = 0; j < p->n_geoms; ++j) {
+      std::vector<uint8_t> g;
+      int rc = validate_row(p->geoms + 8 * j, &g);
+      if (rc) return rc;
+      gs.push_back(g);
+    }
+  } else {
+    return PROTEAN_EINVAL;
+  }
+  protean_handle* h = new protean_handle();
+  h->device = p->device;
+  h->M = M;
+  h->G = (int)gs.size();
+  h->maxT = maxT;
+  h->tl.init(M, h->G);
+  h->words.assign(h->tl.words, 0);
+  int32_t* w = h->words.data();
+  std::memcpy(w + h->tl.o_solo, p->solo_us, sizeof(int32_t) * 5 * M);
+  std::memcpy(w + h->tl.o_fbr, p->fbr_ppm, sizeof(int32_t) * 5 * M);
+  std::memcpy(w + h->tl.o_mem, p->mem_mib, sizeof(int32_t) * M);
+  std::memcpy(w + h->tl.o_bsz, p->batch_size, sizeof(int32_t) * M);
+  std::memcpy(w + h->tl.o_slo, p->slo_us, sizeof(int32_t) * M);
+  std::memcpy(w + h->tl.o_tmo, p->batch_timeout_us, sizeof(int32_t) * M);
+  uint8_t* gp = reinterpret_cast<uint8_t*>(w + h->tl.o_gprof);
+  h->geoms.assign((size_t)h->G * 8, 0xFF);
+  for (int j = 0; j < h->G; ++j) {
+    int pref = 0;
+    for (int s = 0; s < 8; ++s) {
+      const uint8_t v = s < (int)gs[j].size() ? gs[j][s] : 0xFF;
+      gp[j * 8 + s] = v;
+      h->geoms[j * 8 + s] = v;
+      if (v != 0xFF) pref += kMem[v];
+      w[h->tl.o_gpref + j * 8 + s] = pref;  // capacity of slices 0..s (Alg 1 tag walk)
+    }
+    w[h->tl.o_gn + j] = (int32_t)gs[j].size();
+  }
+  cudaError_t e = cudaSetDevice(h->device);
+  if (e == cudaSuccess) e = cudaDeviceGetAttribute(&h->nsm, cudaDevAttrMultiProcessorCount, h->device);
+  if (e == cudaSuccess) e = cudaMalloc(&h->d_tab, sizeof(int32_t) * h->words.size());
+  if (e == cudaSuccess)
+    e = cudaMemcpy(h->d_tab, h->words.data(), sizeof(int32_t) * h->words.size(), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMalloc(&h->d_small, 256);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    protean_free(h);
+    return e == cudaErrorMemoryAllocation ? PROTEAN_ENOMEM : PROTEAN_ECUDA;
+  }
+  *out = h;
+  return PROTEAN_OK;
+}
+
+void protean_free(protean_handle* h) {
+  if (!h) return;
+  cudaSetDevice(h->device);
+  if (h->d_tab) cudaFree(h->d_tab);
+  if (h->d_scratch) cudaFree(h->d_scratch);
+  if (h->d_eoff) cudaFree(h->d_eoff);
+  if (h->d_small) cudaFree(h->d_small);
+  delete h;
+}
+
+int protean_get_geometries(const protean_handle* h, int32_t* n, uint8_t* geoms) {
+  if (!h || !n) return PROTEAN_EINVAL;
+  *n = h->G;
+  if (geoms) std::memcpy(geoms, h->geoms.data(), h->geoms.size());
+  return PROTEAN_OK;
+}
+
+int protean_num_epochs(const protean_handle* h, int64_t trace_len, int64_t W, int64_t* E) {
+  if (!h || !E || W <= 0 || trace_len <= 0) return PROTEAN_EINVAL;
+  *E = (trace_len + W - 1) / W + ((int64_t)h->maxT + W - 1) / W;
+  return PROTEAN_OK;
+}
+
+int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, protean_replay_out* out,
+                          void* stream) {
+  if (!h) return PROTEAN_EINVAL;
+  if (h->poisoned) return PROTEAN_ESTATE;
+  if (!cfg || !out) return fail(h, PROTEAN_EINVAL, "null cfg/out");
+  const protean_replay_cfg& c = *cfg;
+  if (c.n_replicas < 1) return fail(h, PROTEAN_EINVAL, "n_replicas < 1");
+  if (c.n_gpus < 1) return fail(h, PROTEAN_EINVAL, "n_gpus < 1");
+  if (c.n_gpus > 255) return fail(h, PROTEAN_ERANGE, "n_gpus > 255");
+  if (c.epoch_len_us <= 0 || c.trace_len_us <= 0) return fail(h, PROTEAN_EINVAL, "W / trace_len");
+  if (c.trace_len_us - 1 + h->maxT > (int64_t)0xFFFFFFFFLL)
+    return fail(h, PROTEAN_ERANGE, "ready times exceed uint32 us");
+  if (c.policy == 2) return fail(h, PROTEAN_EUNSUP, "policy 2 (Alg 2 heuristic) not built");
+  if (c.policy != 0 && c.policy != 1) return fail(h, PROTEAN_EINVAL, "policy");
+  if (c.shard_mode == 1) return fail(h, PROTEAN_EUNSUP, "shard mode G not built");
+  if (c.shard_mode != 0) return fail(h, PROTEAN_EINVAL, "shard_mode");
+  if (c.wait_limit < 0 || c.wait_limit > 255) return fail(h, PROTEAN_EINVAL, "wait_limit");
+  if (c.reconfig_cap_pct < 0 || c.reconfig_cap_pct > 100) return fail(h, PROTEAN_EINVAL, "cap pct");
+  if (c.init_geom < 0 || c.init_geom >= h->G) return fail(h, PROTEAN_EINVAL, "init_geom");
+  if (c.max_live < 1 || c.max_live > PROTEAN_MAX_LIVE) return fail(h, PROTEAN_EINVAL, "max_live");
+  if (c.vm_policy < 0 || c.vm_policy > 2) return fail(h, PROTEAN_EINVAL, "vm_policy");
+  if (c.reconfig_us < 0) return fail(h, PROTEAN_EINVAL, "reconfig_us");
+  if (!(c.price_od_node_hr >= 0) || !(c.price_spot_node_hr >= 0)) return fail(h, PROTEAN_EINVAL, "price");
+  if (c.vm_policy != 0) {
+    if (!(c.p_rev >= 0 && c.p_rev <= 1)) return fail(h, PROTEAN_EINVAL, "p_rev");
+    if (c.rev_interval_us < c.epoch_len_us) return fail(h, PROTEAN_EINVAL, "rev_interval < W");
+    if (c.notice_us < 0 || c.notice_us >= c.rev_interval_us) return fail(h, PROTEAN_EINVAL, "notice");
+  }
+  if (!c.arrival_us || !c.meta || !c.replica_off) return fail(h, PROTEAN_EINVAL, "null trace");
+  if (!out->counters || !out->accum || !out->hist || !out->p50_p99_us || !out->cost_usd || !out->util)
+    return fail(h, PROTEAN_EINVAL, "null output");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  CK(h, cudaSetDevice(h->device));
+  const int R = c.n_replicas, N = c.n_gpus;
+  std::vector<int64_t> roff(R + 1);
+  CK(h, cudaMemcpyAsync(roff.data(), c.replica_off, sizeof(int64_t) * (R + 1), cudaMemcpyDeviceToHost, st));
+  CK(h, cudaStreamSynchronize(st));
+  if (roff[0] != 0) return fail(h, PROTEAN_EINVAL, "replica_off[0] != 0");
+  for (int r = 0; r < R; ++r)
+    if (roff[r + 1] < roff[r]) return fail(h, PROTEAN_EINVAL, "replica_off not monotone");
+
+  const int64_t W = c.epoch_len_us;
+  const int64_t E = (c.trace_len_us + W - 1) / W + ((int64_t)h->maxT + W - 1) / W;
+  const int64_t H = E * W;
+
+  // prepass: per (replica, epoch) request offsets, largest epoch window
+  const size_t eoff_need = sizeof(int64_t) * (size_t)R * (size_t)(E + 1);
+  {
+    void* p = h->d_eoff;
+    int rc = ensure(h, &p, &h->eoff_bytes, eoff_need);
+    h->d_eoff = static_cast<int64_t*>(p);
+    if (rc) return rc;
+  }
+  unsigned long long* d_wmax = static_cast<unsigned long long*>(h->d_small);
+  int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 64);
+  CK(h, cudaMemsetAsync(h->d_small, 0, 256, st));
+  CK(h, launch_prepass(c.arrival_us, c.replica_off, R, E, W, h->maxT, h->d_eoff, d_wmax, d_err, st));
+  unsigned long long wmax = 0;
+  int herr = 0;
+  CK(h, cudaMemcpyAsync(&wmax, d_wmax, 8, cudaMemcpyDeviceToHost, st));
+  CK(h, cudaMemcpyAsync(&herr, d_err, 4, cudaMemcpyDeviceToHost, st));
+  CK(h, cudaStreamSynchronize(st));
+  if (herr) return fail(h, PROTEAN_EINVAL, "arrivals not sorted or beyond the trace");
+  const int WCAP = (int)std::max<unsigned long long>(wmax, 1);
+  if (wmax >= (1ull << 25)) return fail(h, PROTEAN_ERANGE, "epoch window >= 2^25 requests");
+
+  // launch geometry
+  const int Gc = h->G;
+  const int nl = N * (1 + Gc);
+  int block = ((nl + 31) / 32) * 32;
+  block = std::max(128, std::min(1024, block));
+  SmemLayout sl;
+  sl.init(h->tl.words, h->M, N, Gc, 0, 0);
+  const size_t fixed = sl.total;
+  size_t budget = 72 * 1024;
+  int BS = std::min(WCAP, 256);
+  if (const char* ev = std::getenv("PROTEAN_SMEM_BUDGET_KB")) {  // test knob: force spill paths
+    budget = (size_t)std::atoi(ev) * 1024;
+    BS = std::min(BS, std::max(1, std::atoi(ev)));
+  }
+  budget = std::max<size_t>(budget, fixed + (size_t)BS * (sizeof(Bat) + 8) + 64);
+  size_t rem = budget > fixed + (size_t)BS * (sizeof(Bat) + 8) ? budget - fixed - (size_t)BS * (sizeof(Bat) + 8) : 0;
+  int WS = (int)std::min<size_t>((size_t)WCAP, rem / 4);
+  sl.init(h->tl.words, h->M, N, Gc, BS, WS);
+  if (sl.total > 227 * 1024) return fail(h, PROTEAN_ERANGE, "shared memory layout too large");
+  int per_sm = 0;
+  CK(h, replay_occupancy(block, sl.total, &per_sm));
+  if (per_sm < 1) return fail(h, PROTEAN_ERANGE, "replay kernel does not fit an SM");
+  const int grid = std::min<int64_t>(R, (int64_t)h->nsm * per_sm);
+
+  ReplayParams P;
+  std::memset(&P, 0, sizeof(P));
+  P.tab = h->d_tab;
+  P.tl = h->tl;
+  P.maxT = h->maxT;
+  P.arr = c.arrival_us;
+  P.meta = c.meta;
+  P.roff = c.replica_off;
+  P.eoff = h->d_eoff;
+  P.R = R;
+  P.N = N;
+  P.base = c.replica_base;
+  P.trace_len = c.trace_len_us;
+  P.W = W;
+  P.E = E;
+  P.H = H;
+  P.policy = c.policy;
+  P.wait_limit = c.wait_limit;
+  P.cap_pct = c.reconfig_cap_pct;
+  P.init_geom = c.init_geom;
+  P.max_live = c.max_live;
+  P.vm_policy = c.vm_policy;
+  P.reconfig_us = c.reconfig_us;
+  P.rev = c.vm_policy ? c.rev_interval_us : 1;
+  P.notice = c.notice_us;
+  P.thr = (uint64_t)(c.p_rev * 9007199254740992.0);
+  P.seed = c.seed;
+  P.price_od = c.price_od_node_hr;
+  P.price_spot = c.price_spot_node_hr;
+  P.geom_lo = 0;
+  P.geom_hi = Gc;
+  P.counters = out->counters;
+  P.accum = out->accum;
+  P.hist = out->hist;
+  P.pct = out->p50_p99_us;
+  P.cost = out->cost_usd;
+  P.util = out->util;
+  P.decisions = out->decisions;
+  P.cand_keys = out->cand_keys;
+  P.log = out->batch_log;
+  P.log_cap = out->batch_log ? out->batch_log_cap : 0;
+  P.n_batches = out->n_batches;
+  P.sl = sl;
+  P.WCAP = WCAP;
+  size_t o = 0;
+  P.o_lists = o; o += al((size_t)nl * c.max_live * sizeof(protean_resident));
+  P.o_lane_n = o; o += al((size_t)N * 4);
+  P.o_ls = o; o += al((size_t)N * kMaxSl * 8);
+  P.o_bu = o; o += al((size_t)N * kMaxSl * 8);
+  const size_t gb = WCAP > BS ? (size_t)(WCAP - BS) : 0;
+  P.o_gbat = o; o += al(gb * sizeof(Bat));
+  P.o_gord = o; o += al(gb * 4);
+  P.o_gglist = o; o += al(gb * 4);
+  P.o_gsarr = o; o += al((size_t)(WCAP > WS ? WCAP - WS : 0) * 4);
+  P.slot_bytes = al(o);
+  {
+    int rc = ensure(h, &h->d_scratch, &h->scratch_bytes, P.slot_bytes * (size_t)grid);
+    if (rc) return rc;
+  }
+  P.scratch = static_cast<char*>(h->d_scratch);
+  P.err = d_err;
+  CK(h, launch_replay(P, grid, block, st));
+  CK(h, cudaMemcpyAsync(&herr, d_err, 4, cudaMemcpyDeviceToHost, st));
+  CK(h, cudaStreamSynchronize(st));
+  if (herr) return fail(h, PROTEAN_EINVAL, "invalid request (unsorted, model id, or arrival >= trace_len)");
+  return PROTEAN_OK;
+}
+
+int protean_score_epoch(protean_handle* h, const protean_epoch_in* in, protean_epoch_out* out,
+                        void* stream) {
+  if (!h) return PROTEAN_EINVAL;
+  if (h->poisoned) return PROTEAN_ESTATE;
+  if (!in || !out) return fail(h, PROTEAN_EINVAL, "null in/out");
+  if (in->n_replicas < 1 || in->n_gpus < 1 || in->epoch < 0 || in->epoch_len_us <= 0 || in->horizon_us < 0)
+    return fail(h, PROTEAN_EINVAL, "sizes");
+  if (in->n_gpus > 255) return fail(h, PROTEAN_ERANGE, "n_gpus > 255");
+  if (in->max_live < 1 || in->max_live > PROTEAN_MAX_LIVE) return fail(h, PROTEAN_EINVAL, "max_live");
+  if (in->geom_lo < 0 || in->geom_hi > h->G || in->geom_lo >= in->geom_hi)
+    return fail(h, PROTEAN_EINVAL, "geometry range");
+  if (!in->batch_off || !in->state || !out->best_key || !out->counters || !out->placement)
+    return fail(h, PROTEAN_EINVAL, "null pointer");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  CK(h, cudaSetDevice(h->device));
+  const int R = in->n_replicas, N = in->n_gpus, Gc = in->geom_hi - in->geom_lo;
+  int32_t b0 = 0;
+  CK(h, cudaMemcpyAsync(&b0, in->batch_off, 4, cudaMemcpyDeviceToHost, st));
+  CK(h, cudaStreamSynchronize(st));
+  if (b0 != 0) return fail(h, PROTEAN_EINVAL, "batch_off[0] != 0");
+  const size_t need = sizeof(protean_resident) * (size_t)R * N * Gc * in->max_live;
+  {
+    int rc = ensure(h, &h->d_scratch, &h->scratch_bytes, std::max<size_t>(need, 256));
+    if (rc) return rc;
+  }
+  int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 64);
+  CK(h, cudaMemsetAsync(d_err, 0, 16, st));
+  ScoreParams P;
+  std::memset(&P, 0, sizeof(P));
+  P.tab = h->d_tab;
+  P.tl = h->tl;
+  P.R = R;
+  P.N = N;
+  P.epoch = in->epoch;
+  P.max_live = in->max_live;
+  P.geom_lo = in->geom_lo;
+  P.geom_hi = in->geom_hi;
+  P.W = in->epoch_len_us;
+  P.H = in->horizon_us;
+  P.batches = in->batches;
+  P.batch_off = in->batch_off;
+  P.arrival = in->arrival_us;
+  P.state = in->state;
+  P.best_key = out->best_key;
+  P.cand_key = out->cand_key;
+  P.placement = out->placement;
+  P.counters = out->counters;
+  P.accum = out->accum;
+  P.scratch = static_cast<protean_resident*>(h->d_scratch);
+  P.err = d_err;
+  const int nl = N * (1 + Gc);
+  int block = std::max(128, std::min(1024, ((nl + 31) / 32) * 32));
+  CK(h, launch_score(P, block, st));
+  int errs[2] = {0, 0};
+  CK(h, cudaMemcpyAsync(errs, d_err, 8, cudaMemcpyDeviceToHost, st));
+  CK(h, cudaStreamSynchronize(st));
+  if (errs[0]) return fail(h, PROTEAN_EINVAL, "invalid state / batch");
+  if (errs[1]) return fail(h, PROTEAN_ERANGE, "n_live > max_live");
+  return PROTEAN_OK;
+}
+
+}  // extern "C"

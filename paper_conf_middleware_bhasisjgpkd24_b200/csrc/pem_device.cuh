@@ -1,0 +1,219 @@
+// pem_device.cuh — device-side building blocks of the B200 PROTEAN epoch engine (sm_100a).
+//
+// The lane-level Place() is Alg 1 under the slowdown model Eq 1 / Eq 2 (P:L191,
+// P:L208) in exact integers; every reading it relies on is listed in DESIGN.md §3.  One lane
+// owns one resident list (the actual GPU state, or one candidate geometry replayed from idle)
+// and walks the GPU-epoch's batches; lanes of the same simulated GPU walk the same batch list in
+// lock-step, so batch descriptors are warp-broadcast loads.
+#pragma once
+#include <stdint.h>
+#include "../../include/protean.h"
+
+namespace pemgpu {
+
+constexpr int kNProf = 5;
+constexpr int kMaxSl = 7;
+constexpr int64_t kPpm = 1000000;
+constexpr uint32_t kNoGeom = 0xFF;
+constexpr int kNB = PROTEAN_NBUCKETS;
+
+// T2 — slice memory in MiB and compute sevenths per profile (1g,2g,3g,4g,7g).
+__host__ __device__ __forceinline__ int32_t prof_cap(int p) {
+  return p == 0 ? 5120 : p == 1 ? 10240 : p == 4 ? 40960 : 20480;
+}
+__host__ __device__ __forceinline__ int32_t prof_compute(int p) {
+  return p == 0 ? 1 : p == 1 ? 2 : p == 2 ? 3 : p == 3 ? 4 : 7;
+}
+
+// Table block layout (int32 words), identical on host and device; staged into smem per CTA.
+struct TabLayout {
+  int M, G;
+  int o_solo, o_fbr, o_mem, o_bsz, o_slo, o_tmo;  // [M*5],[M*5],[M],[M],[M],[M]
+  int o_gprof;   // G*8 bytes packed into G*2 words: profile ids ascending, 0xFF padded
+  int o_gn;      // G words: slice count
+  int o_gpref;   // G*8 words: prefix capacity including slice s (tag walk, Alg 1 lines 1-8)
+  int words;
+  __host__ __device__ void init(int m, int g) {
+    M = m; G = g;
+    o_solo = 0; o_fbr = o_solo + 5 * M; o_mem = o_fbr + 5 * M; o_bsz = o_mem + M;
+    o_slo = o_bsz + M; o_tmo = o_slo + M; o_gprof = o_tmo + M; o_gn = o_gprof + 2 * G;
+    o_gpref = o_gn + G; words = o_gpref + 8 * G;
+  }
+};
+
+struct Tab {  // smem views
+  int M, G;
+  const int32_t *solo, *fbr, *mem, *bsz, *slo, *tmo, *gn, *gpref;
+  const uint8_t *gprof;
+  __device__ void bind(const int32_t* w, const TabLayout& L) {
+    M = L.M; G = L.G;
+    solo = w + L.o_solo; fbr = w + L.o_fbr; mem = w + L.o_mem; bsz = w + L.o_bsz;
+    slo = w + L.o_slo; tmo = w + L.o_tmo; gn = w + L.o_gn; gpref = w + L.o_gpref;
+    gprof = reinterpret_cast<const uint8_t*>(w + L.o_gprof);
+  }
+};
+
+// A resident list: protean_resident rows (24 B), contiguous per lane.
+// meta word at byte 20 = slice | model << 8 | strict << 16.
+struct Rows {
+  protean_resident* r;
+  __device__ __forceinline__ int64_t st(int i) const { return r[i].start_us; }
+  __device__ __forceinline__ int64_t en(int i) const { return r[i].end_us; }
+  __device__ __forceinline__ int32_t mem(int i) const { return r[i].mem_mib; }
+  __device__ __forceinline__ uint32_t meta(int i) const {
+    return *reinterpret_cast<const uint32_t*>(&r[i].slice);
+  }
+};
+
+struct PlaceRes {
+  int64_t start, end;
+  int slice;
+  int dropped;  // 0 placed, 2 no slice holds the footprint, 3 max_live overflow
+};
+
+// Eq 1 in integers: exec = floor(solo * max(F, 10^6) / 10^6) (reading Q10).
+__device__ __forceinline__ int64_t exec_time(int32_t solo, int64_t F) {
+  int64_t f = F < kPpm ? kPpm : F;
+  return ((int64_t)solo * f) / kPpm;
+}
+
+// Place one batch (model m, class strict, ready t) on geometry `geom` over list L (n rows).
+// ls[] = last start per slice position (FIFO).  Returns the chosen slice and [start, end).
+__device__ __forceinline__ PlaceRes place_lane(const Tab& T, int geom, Rows L, int& n,
+                                               int64_t (&ls)[kMaxSl], int64_t t, int m,
+                                               bool strict, int max_live) {
+  PlaceRes o;
+  o.dropped = 0;
+  o.slice = -1;
+  o.start = o.end = 0;
+  // residents that ended by t can never matter again: stable compaction
+  int k = 0;
+  for (int i = 0; i < n; ++i) {
+    if (L.en(i) > t) {
+      if (k != i) L.r[k] = L.r[i];
+      ++k;
+    }
+  }
+  n = k;
+  if (n >= max_live) {  // reading Q39
+    o.dropped = 3;
+    return o;
+  }
+  const int32_t q = T.mem[m];
+  const int ns = T.gn[geom];
+  int64_t be_mem = 0;  // Alg 1 line 1: BE memory on this GPU (reading Q5)
+  for (int i = 0; i < n; ++i)
+    if (!((L.meta(i) >> 16) & 1)) be_mem += L.mem(i);
+
+  uint64_t best = ~0ull;
+  int64_t bstart = 0, bend = 0;
+#pragma unroll
+  for (int s = 0; s < kMaxSl; ++s) {
+    if (s < ns) {
+      const int p = T.gprof[geom * 8 + s];
+      const int32_t Ms = prof_cap(p);
+      if (q <= Ms) {
+        const int64_t t0 = t > ls[s] ? t : ls[s];
+        int64_t used = 0;
+        for (int i = 0; i < n; ++i)
+          if ((int)(L.meta(i) & 0xFF) == s && L.en(i) > t0) used += L.mem(i);
+        int64_t start = t0;
+        if (used + q > Ms) {  // memory wait: earliest release that makes the batch fit
+          start = INT64_MAX;
+          for (int i = 0; i < n; ++i) {
+            if ((int)(L.meta(i) & 0xFF) != s || L.en(i) <= t0) continue;
+            const int64_t ei = L.en(i);
+            int64_t rem = 0;
+            for (int j = 0; j < n; ++j)
+              if ((int)(L.meta(j) & 0xFF) == s && L.en(j) > ei) rem += L.mem(j);
+            if (rem + q <= Ms && ei < start) start = ei;
+          }
+        }
+        int64_t F = T.fbr[m * kNProf + p];  // Eq 1's co-located sum at the start instant
+        for (int i = 0; i < n; ++i) {
+          const uint32_t mt = L.meta(i);
+          if ((int)(mt & 0xFF) == s && L.st(i) <= start && start < L.en(i))
+            F += T.fbr[((mt >> 8) & 0xFF) * kNProf + p];
+        }
+        const int64_t c = start + exec_time(T.solo[m * kNProf + p], F);
+        uint64_t key;
+        if (strict) {  // choose_strict_slice: tag < 1, least eta == least completion (Q11)
+          const uint64_t inelig = (be_mem >= T.gpref[geom * 8 + s]) ? (1ull << 62) : 0ull;
+          key = inelig | ((uint64_t)c << 6) | ((uint64_t)(4 - p) << 3) | (uint64_t)s;
+        } else {       // choose_best_effort_slice: first fit, else earliest start (Q12)
+          key = ((uint64_t)start << 3) | (uint64_t)s;
+        }
+        if (key < best) {
+          best = key;
+          bstart = start;
+          bend = c;
+        }
+      }
+    }
+  }
+  if (best == ~0ull) {
+    o.dropped = 2;
+    return o;
+  }
+  const int s = (int)(best & 7);
+  protean_resident nr;
+  nr.start_us = bstart;
+  nr.end_us = bend;
+  nr.mem_mib = q;
+  nr.slice = (uint8_t)s;
+  nr.model = (uint8_t)m;
+  nr.strict = strict ? 1 : 0;
+  nr.pad = 0;
+  L.r[n] = nr;
+  ++n;
+#pragma unroll
+  for (int x = 0; x < kMaxSl; ++x)
+    if (x == s) ls[x] = bstart;
+  o.slice = s;
+  o.start = bstart;
+  o.end = bend;
+  return o;
+}
+
+// O7 log-linear latency bucket (reading Q30).
+__device__ __forceinline__ int lat_bucket(int64_t x) {
+  uint64_t v = x < 0 ? 0 : (uint64_t)x;
+  if (v > 0xFFFFFFFFull) v = 0xFFFFFFFFull;
+  if (v < 128) return (int)v;
+  const int k = 31 - __clz((unsigned)v);
+  return 128 + (k - 7) * 128 + (int)((v >> (k - 7)) & 127);
+}
+
+__host__ __device__ __forceinline__ uint64_t bucket_lower_edge(int b) {
+  if (b < 128) return (uint64_t)b;
+  const int k = 7 + (b - 128) / 128;
+  return (uint64_t)(128 + (b - 128) % 128) << (k - 7);
+}
+
+// O8 key (reading Q20)
+__device__ __forceinline__ int64_t make_key(int64_t misses, int64_t tail, int tag) {
+  const int64_t mm = (1LL << 23) - 1;
+  if (misses > mm) misses = mm;
+  if (tail > 0xFFFFFFFFLL) tail = 0xFFFFFFFFLL;
+  return (misses << 40) | (tail << 8) | (int64_t)tag;
+}
+
+__device__ __forceinline__ uint64_t smix(uint64_t x) {
+  x += 0x9E3779B97F4A7C15ull;
+  x = (x ^ (x >> 30)) * 0xBF58476D1CE4E5B9ull;
+  x = (x ^ (x >> 27)) * 0x94D049BB133111EBull;
+  return x ^ (x >> 31);
+}
+
+// #{members a with c - a <= slo} over a sorted ascending member list (binary search).
+__device__ __forceinline__ int hits_sorted(const uint32_t* a, int n, int64_t c, int64_t slo) {
+  const int64_t lo_a = c - slo;  // need a >= c - slo
+  int lo = 0, hi = n;
+  while (lo < hi) {
+    int mid = (lo + hi) >> 1;
+    if ((int64_t)a[mid] >= lo_a) hi = mid; else lo = mid + 1;
+  }
+  return n - lo;
+}
+
+}  // namespace pemgpu

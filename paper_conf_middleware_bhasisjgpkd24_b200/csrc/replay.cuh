@@ -1,0 +1,117 @@
+// replay.cuh — host/device shared launch structures of the fused epoch engine.
+#pragma once
+#include <stddef.h>
+#include <stdint.h>
+#include <cuda_runtime.h>
+#include "pem_device.cuh"
+
+namespace pemgpu {
+
+constexpr int kNSeg = 4;          // warps that stream-partition the request window
+constexpr int64_t kForever = INT64_MAX;
+
+// One batch of the current epoch (40 B).  info = n | model << 16 | strict << 24.
+struct Bat {
+  uint64_t key;       // id-order key: ready(32) | class(1) | model(6) | stream position(25)
+  uint32_t ready, info, pos;
+  uint8_t gpu, slice, drop, pad;
+  int64_t start, end;
+};
+
+// Dynamic shared-memory layout (byte offsets), computed on the host.
+struct SmemLayout {
+  int S;            // streams = 2 * M
+  int N, Gc;        // simulated GPUs, candidate geometries in range
+  int BS, WS;       // batches / window entries held in smem (rest spills to global scratch)
+  size_t tab, hist, s_cnt, s_run, s_base, s_tot, s_skip, s_pend;
+  size_t g_u8, g_i64, g_i32, keys, bats, ord, glist, sarr, total;
+  __host__ void init(int words, int M, int n_gpus, int gc, int bs, int ws) {
+    S = 2 * M; N = n_gpus; Gc = gc; BS = bs; WS = ws;
+    size_t o = 0;
+    auto take = [&](size_t bytes) { size_t r = o; o += (bytes + 15) & ~(size_t)15; return r; };
+    tab = take((size_t)words * 4);
+    hist = take((size_t)kNB * 4);               // 2 classes x 3328 buckets as packed u16 pairs
+    s_cnt = take((size_t)kNSeg * S * 4);
+    s_run = take((size_t)kNSeg * S * 4);
+    s_base = take((size_t)S * 4);
+    s_tot = take((size_t)S * 4);
+    s_skip = take((size_t)S * 4);
+    s_pend = take((size_t)S * 4);
+    g_u8 = take((size_t)N * 8);                 // geom, target, ctr, vm, bill, dec, best, want
+    g_i64 = take((size_t)N * 12 * 8);           // rs, re, from, until, since, maxend, kbest, kcur, od, spot, busy, mem
+    g_i32 = take((size_t)(2 * N + 2) * 4);      // gcnt[N], goff[N+1]
+    keys = take((size_t)N * Gc * 8);
+    bats = take((size_t)BS * sizeof(Bat));
+    ord = take((size_t)BS * 4);
+    glist = take((size_t)BS * 4);
+    sarr = take((size_t)WS * 4);
+    total = o;
+  }
+};
+
+struct ReplayParams {
+  // tables
+  const int32_t* tab;
+  TabLayout tl;
+  int maxT;
+  // trace (device)
+  const uint32_t* arr;
+  const uint8_t* meta;
+  const int64_t* roff;
+  const int64_t* eoff;     // [R][E+1] first request index with arrival >= e*W
+  int R, N;
+  int64_t base, trace_len, W, E, H;
+  // policy
+  int policy, wait_limit, cap_pct, init_geom, max_live, vm_policy;
+  int64_t reconfig_us, rev, notice;
+  uint64_t thr, seed;
+  double price_od, price_spot;
+  int geom_lo, geom_hi;
+  // outputs (device)
+  int64_t* counters;
+  int64_t* accum;
+  uint32_t* hist;
+  int64_t* pct;
+  double* cost;
+  double* util;
+  uint8_t* decisions;
+  int64_t* cand_keys;
+  protean_batch_rec* log;
+  int64_t log_cap;
+  int64_t* n_batches;
+  // scratch
+  SmemLayout sl;
+  int WCAP;                // max window entries of any epoch (prepass)
+  char* scratch;
+  size_t slot_bytes, o_lists, o_lane_n, o_ls, o_bu, o_gbat, o_gord, o_gglist, o_gsarr;
+  int* err;
+};
+
+struct ScoreParams {
+  const int32_t* tab;
+  TabLayout tl;
+  int R, N, epoch, max_live, geom_lo, geom_hi;
+  int64_t W, H;
+  const protean_batch* batches;
+  const int32_t* batch_off;
+  const uint32_t* arrival;
+  protean_gpu_state* state;
+  int64_t* best_key;
+  int64_t* cand_key;
+  protean_placement* placement;
+  int64_t* counters;
+  int64_t* accum;
+  protean_resident* scratch;  // [R][N*(Gc)][max_live]
+  int* err;                   // err[0] EINVAL, err[1] ERANGE
+};
+
+// launchers (replay.cu / score.cu)
+cudaError_t launch_prepass(const uint32_t* arr, const int64_t* roff, int R, int64_t E, int64_t W,
+                           int64_t maxT, int64_t* eoff, unsigned long long* wmax, int* err,
+                           cudaStream_t st);
+cudaError_t launch_replay(const ReplayParams& P, int grid, int block, cudaStream_t st);
+cudaError_t replay_occupancy(int block, size_t smem, int* blocks_per_sm);
+cudaError_t launch_score(const ScoreParams& P, int block, cudaStream_t st);
+size_t score_smem_bytes(const TabLayout& tl, int N, int Gc);
+
+}  // namespace pemgpu

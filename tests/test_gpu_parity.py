@@ -1,0 +1,247 @@
+"""GPU (CUDA, sm_100a) vs CPU oracle parity through the C ABI.  -m gpu."""
+import json
+import os
+
+import numpy as np
+import pytest
+
+from gpu_common import compare, gpu_replay, oracle_replay
+from helpers import GOLDEN, tables, trace_from, w1
+from protean_inputs import (c1_profiles, c1_trace, concat, mix_a_params, mix_b_params, pack_meta,
+                            random_profiles, synth_profiles, tick_trace, uniform_trace)
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.mark.parametrize("gset", [0, 1])
+def test_config1_exact(oracle, gset):
+    """Config 1: 1 sim-GPU, 3 models, 200-request 1 s Poisson trace; G = 12 and 37."""
+    prof = c1_profiles().with_geometry_set(gset)
+    tr = c1_trace()
+    g = gpu_replay(prof, tr, n_gpus=1)
+    o = oracle_replay(oracle, prof, tr, n_gpus=1)
+    compare(g, o, 1)
+    assert o["counters"][0, 9] > 0
+
+
+def test_w1_golden_gpu(oracle):
+    gold, P, tr = w1()
+    ex = gold["expected"]
+    g = gpu_replay(P, tr, n_gpus=1, init_geom=2)
+    assert g["cand_keys"][0, 0, 0].tolist() == ex["cand_keys_epoch0"]
+    assert g["decisions"][0, 0, 0] == ex["best_epoch0"]
+    assert g["p50_p99"][0].tolist() == ex["p50_p99_us"]
+    log = g["log"][0][: g["n_batches"][0]]
+    assert [[int(b["slice"]), int(b["start"]), int(b["end"])] for b in log] == ex["actual_placement_j2"]
+    compare(g, oracle_replay(oracle, P, tr, n_gpus=1, init_geom=2), 1)
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_fuzz_replay(oracle, seed):
+    rng = np.random.default_rng(100 + seed)
+    M = int(rng.integers(1, 7))
+    prof = random_profiles(rng, M).with_geometry_set(int(rng.integers(0, 2)))
+    N = int(rng.choice([1, 2, 3, 8]))
+    R = int(rng.integers(1, 6))
+    tr = uniform_trace(rng, R, M, int(rng.integers(2, 12)) * 1_000_000, int(rng.integers(5, 600)))
+    cfg = dict(n_gpus=N, policy=int(rng.integers(0, 2)) if seed % 3 == 0 else 0,
+               init_geom=int(rng.integers(0, 12)), max_live=int(rng.choice([2, 8, 64])),
+               wait_limit=int(rng.integers(0, 4)), reconfig_us=int(rng.integers(0, 3_000_000)),
+               vm_policy=int(seed % 3), p_rev=float(rng.choice([0.0, 0.354, 0.708, 1.0])),
+               rev_interval_us=2_000_000, notice_us=300_000, seed=seed, replica_base=int(rng.integers(0, 100)))
+    tr.replica_base = cfg.pop("replica_base")
+    g = gpu_replay(prof, tr, **cfg)
+    o = oracle_replay(oracle, prof, tr, **cfg)
+    compare(g, o, R)
+
+
+@pytest.mark.parametrize("budget_kb", ["1", "24"])
+def test_spill_paths(oracle, monkeypatch, budget_kb):
+    """Force batch / window arrays to spill from shared memory to global scratch."""
+    monkeypatch.setenv("PROTEAN_SMEM_BUDGET_KB", budget_kb)
+    rng = np.random.default_rng(7)
+    prof = random_profiles(rng, 5)
+    tr = uniform_trace(rng, 3, 5, 6_000_000, 900)
+    g = gpu_replay(prof, tr, n_gpus=4)
+    o = oracle_replay(oracle, prof, tr, n_gpus=4)
+    compare(g, o, 3)
+
+
+def test_mix_a_sample(oracle):
+    """Config-5 shaped replicas (Mix A, 22-model table, 8 sim-GPUs), shortened to 40 s."""
+    prof = synth_profiles()
+    tr = tick_trace(mix_a_params(3, seed=1, seconds=40))
+    g = gpu_replay(prof, tr, n_gpus=8)
+    o = oracle_replay(oracle, prof, tr, n_gpus=8)
+    compare(g, o, 3)
+    c = o["counters"]
+    assert c[:, 8].sum() > 0 and (o["decisions"] != 255).any()
+
+
+def test_mix_b_vm_sample(oracle):
+    """Config-2/3 shaped (Mix B, bursty vision + language, 22 models) with spot/on-demand."""
+    prof = synth_profiles()
+    tr = tick_trace(mix_b_params(2, seed=3, seconds=30))
+    for vm_policy, p_rev in [(0, 0.0), (1, 0.708), (2, 0.354)]:
+        cfg = dict(n_gpus=8, vm_policy=vm_policy, p_rev=p_rev, rev_interval_us=5_000_000,
+                   notice_us=1_000_000, seed=11)
+        compare(gpu_replay(prof, tr, **cfg), oracle_replay(oracle, prof, tr, **cfg), 2)
+
+
+def test_reconfig_scenarios_gpu(oracle):
+    """T6/T7: hysteresis fires on the 4th mismatch; at most 2 of 8 GPUs reconfigure at once."""
+    from test_oracle_pins import _w1_repeated
+    _, P, _ = w1()
+    P8, tr8 = _w1_repeated(P, 5, copies=8)
+    g = gpu_replay(P8, tr8, n_gpus=8, init_geom=2)
+    compare(g, oracle_replay(oracle, P8, tr8, n_gpus=8, init_geom=2), 1)
+    assert g["counters"][0, 7] == 2
+    P1, tr1 = _w1_repeated(P, 8)
+    g = gpu_replay(P1, tr1, n_gpus=1, init_geom=2)
+    compare(g, oracle_replay(oracle, P1, tr1, n_gpus=1, init_geom=2), 1)
+
+
+def test_edge_cases(oracle):
+    # empty replica, a single request, all ties, footprint larger than every slice but 7g
+    P = tables([[1000, 900, 800, 700, 600], [500] * 5], [[900_000] * 5, [300_000] * 5], [30_000, 100],
+               bsz=[3, 2], tmo=[50, 0])
+    parts = [(np.zeros(0, np.uint32), np.zeros(0, np.uint8)),
+             (np.array([5], np.uint32), pack_meta([0], [1])),
+             (np.full(50, 777, np.uint32), pack_meta(np.arange(50) % 2, (np.arange(50) // 2) % 2)),
+             (np.sort(np.random.default_rng(1).integers(0, 3_000_000, 400)).astype(np.uint32),
+              pack_meta(np.zeros(400), np.ones(400)))]
+    tr = concat(parts, 3_000_000)
+    for init in (0, 2, 11):
+        g = gpu_replay(P, tr, n_gpus=2, init_geom=init)
+        compare(g, oracle_replay(oracle, P, tr, n_gpus=2, init_geom=init), 4)
+
+
+def test_determinism():
+    rng = np.random.default_rng(3)
+    prof = random_profiles(rng, 4)
+    tr = uniform_trace(rng, 6, 4, 5_000_000, 500)
+    a = gpu_replay(prof, tr, n_gpus=3)
+    b = gpu_replay(prof, tr, n_gpus=3)
+    for k in ("counters", "accum", "hist", "decisions", "cand_keys", "log", "cost", "util"):
+        assert np.array_equal(a[k], b[k]), k
+
+
+def test_error_codes_match_oracle(oracle):
+    import paper_conf_middleware_bhasisjgpkd24_b200 as pkg
+    P = tables([[1000] * 5], [[0] * 5], [100])
+    good = trace_from([(5, 0, 1), (7, 0, 0)], 1_000_000)
+
+    def gcode(prof, tr, **cfg):
+        try:
+            h = pkg.load_profiles(prof)
+            h.replay_traces_host(tr, **cfg)
+        except pkg.ProteanError as e:
+            return e.code
+        return 0
+
+    def ocode(prof, tr, **cfg):
+        try:
+            oracle_replay(oracle, prof, tr, want_keys=False, want_log=False, **cfg)
+        except oracle.OracleError as e:
+            return e.code
+        return 0
+    cases = [
+        (P, concat([(np.array([7, 5], np.uint32), pack_meta([0, 0], [1, 1]))], 10**6), {}),
+        (P, concat([(np.array([5], np.uint32), pack_meta([3], [1]))], 10**6), {}),
+        (P, concat([(np.array([5], np.uint32), pack_meta([0], [1]) | 64)], 10**6), {}),
+        (P, concat([(np.array([2_000_000], np.uint32), pack_meta([0], [1]))], 10**6), {}),
+        (tables([[1000] * 5], [[1_000_001] * 5], [100]), good, {}),
+        (tables([[0] * 5], [[0] * 5], [100]), good, {}),
+        (P, good, dict(n_gpus=256)),
+        (tables([[1000] * 5], [[0] * 5], [100], geoms=[[4]] * 255), good, {}),
+        (tables([[1000] * 5], [[0] * 5], [100], geoms=[[3, 4]]), good, {}),
+        (P, concat([(np.array([5], np.uint32), pack_meta([0], [1]))], 2**32 + 5), {}),
+        (P, good, dict(policy=2)),
+        (P, good, dict(max_live=0)),
+        (P, good, dict(init_geom=12)),
+        (P, good, {}),
+    ]
+    for prof, tr, cfg in cases:
+        assert gcode(prof, tr, **cfg) == ocode(prof, tr, **cfg), cfg
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_score_epoch_fuzz(oracle, seed):
+    """protean_score_epoch vs the oracle on realistic carried states (built by the oracle's own
+    Place on a previous epoch), pending reconfigurations and undecidable GPUs."""
+    import ctypes as C
+    import torch
+    import paper_conf_middleware_bhasisjgpkd24_b200 as pkg
+    from paper_conf_middleware_bhasisjgpkd24_b200 import _abi as A
+    rng = np.random.default_rng(500 + seed)
+    M = 4
+    prof = random_profiles(rng, M, max_batch=6)
+    R, N, epoch, W = int(rng.integers(1, 4)), int(rng.integers(1, 5)), 3, 1_000_000
+    G = 12
+    eW = epoch * W
+    ostates = (oracle.State * (R * N))()
+    gstates = (A.GpuState * (R * N))()
+    b_ready, b_off, b_n, b_model, b_strict, batch_off, arrival = [], [], [], [], [], [0], []
+    for x in range(R * N):
+        geom = int(rng.integers(0, G))
+        s = oracle.new_state(geom)
+        for t in np.sort(rng.integers(eW - 400_000, eW, size=int(rng.integers(0, 5)))):
+            oracle.place(prof, s, int(t), int(rng.integers(0, M)), int(rng.integers(0, 2)))
+        s.has_vm = int(rng.random() < 0.85)
+        if rng.random() < 0.3:
+            s.target = int(rng.integers(0, G))
+            s.recfg_start = eW - 500_000
+            s.recfg_end = eW + int(rng.integers(-200_000, 2_500_000))
+        ostates[x] = s
+        gs = gstates[x]
+        gs.geom, gs.target, gs.n_live, gs.has_vm = s.geom, 255 if s.target < 0 else s.target, s.n_res, s.has_vm
+        gs.recfg_start_us, gs.recfg_end_us = s.recfg_start, s.recfg_end
+        for i in range(7):
+            gs.last_start_us[i], gs.busy_until_us[i] = s.last_start[i], s.busy_until[i]
+        for i in range(s.n_res):
+            rr = s.res[i]
+            gs.live[i] = A.Resident(rr.start, rr.end, rr.mem, rr.slice, rr.model, rr.strict, 0)
+        nb = int(rng.integers(0, 9))
+        for t in np.sort(rng.integers(eW, eW + W, size=nb)):
+            n = int(rng.integers(1, 7))
+            arr = np.sort(rng.integers(max(0, t - 300_000), t + 1, size=n))
+            b_off.append(len(arrival))
+            arrival.extend(arr.tolist())
+            b_ready.append(int(t)); b_n.append(n); b_model.append(int(rng.integers(0, M)))
+            b_strict.append(int(rng.integers(0, 2)))
+        batch_off.append(len(b_ready))
+    batches = dict(ready=b_ready, req_off=b_off, n=b_n, model=b_model, strict=b_strict)
+    H = 50 * W
+    o = oracle.score_epoch(prof, R=R, N=N, epoch=epoch, batches=batches, batch_off=batch_off,
+                           arrival=np.array(arrival, np.uint32), states=ostates, W=W, H=H)
+    nb = len(b_ready)
+    rows = np.zeros((max(nb, 1), 16), np.uint8)
+    for i in range(nb):
+        rows[i] = np.frombuffer(bytes(A.Batch(b_ready[i], b_off[i], b_n[i], b_model[i], b_strict[i], 0)), np.uint8)
+    dev = torch.device("cuda", 0)
+    t_rows = torch.from_numpy(rows[:nb].reshape(-1)).to(dev) if nb else torch.zeros(16, dtype=torch.uint8, device=dev)[:0]
+    t_off = torch.tensor(batch_off, dtype=torch.int32, device=dev)
+    t_arr = torch.tensor(np.array(arrival, np.uint32).view(np.int32), device=dev) if arrival else torch.zeros(1, dtype=torch.int32, device=dev)
+    t_state = torch.from_numpy(np.frombuffer(bytes(gstates), np.uint8).copy()).to(dev)
+    h = pkg.load_profiles(prof)
+    g = h.score_epoch(n_replicas=R, n_gpus=N, epoch=epoch, batches=t_rows, batch_off=t_off,
+                      arrival_us=t_arr, state=t_state, epoch_len_us=W, horizon_us=H)
+    assert g["best_key"].cpu().tolist() == o["best_key"].tolist()
+    assert g["cand_key"].cpu().tolist() == o["cand_key"].tolist()
+    assert g["counters"].cpu().numpy().tolist() == o["counters"].tolist()
+    assert g["accum"].cpu().numpy()[:, :2].tolist() == o["accum"][:, :2].tolist()
+    pl = g["placement"].cpu().numpy()
+    for i in range(nb):
+        p = A.Placement.from_buffer_copy(pl[i].tobytes())
+        assert (p.start_us, p.end_us, p.dropped) == (o["start"][i], o["end"][i], o["dropped"][i])
+        if not p.dropped:
+            assert p.slice == o["slice"][i]
+    st = (A.GpuState * (R * N)).from_buffer_copy(t_state.cpu().numpy().tobytes())
+    for x in range(R * N):
+        assert st[x].geom == ostates[x].geom and st[x].n_live == ostates[x].n_res
+        for i in range(st[x].n_live):
+            a, b = st[x].live[i], ostates[x].res[i]
+            assert (a.start_us, a.end_us, a.mem_mib, a.slice, a.model, a.strict) == \
+                (b.start, b.end, b.mem, b.slice, b.model, b.strict)
+        assert list(st[x].last_start_us) == list(ostates[x].last_start)
+        assert list(st[x].busy_until_us) == list(ostates[x].busy_until)
