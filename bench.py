@@ -1,0 +1,339 @@
+#!/usr/bin/env python3
+"""bench.py — placement candidates scored/s (slot-evals/s) of the fused B200 epoch engine.
+
+Workload (BASELINE.json configs[4], "C5"): 4096 trace-seed replicas x 8 simulated GPUs x 600 s of
+Mix A (Wiki-shaped 5000 rps vision trace, 50/50 strict/BE, 22-model synthetic profile table),
+12 candidate geometries, geometry search policy, on-demand VMs.  One step = one full
+protean_replay_traces over all replicas of this rank (every epoch of every replica: batch
+formation, dispatch, actual placement, per-request accounting, candidate scoring, argmin,
+hysteresis/cap, finalize).  Weak scaling: each rank replays its own 4096 replicas (global replica
+ids rank*4096 + i), no data-path collective.  Inputs are generated in HBM before timing (61 GB per
+rank, far larger than the 126 MB L2, so no L2 flush is needed between steps).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--replicas R]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from protean_inputs import mix_a_params, synth_profiles, tick_trace  # noqa: E402
+
+METRIC = "placement candidates scored/s (slot-evals/s)"
+UNIT = "slot-evals/s"
+HBM_PEAK_FALLBACK = 6650.0
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured"
+    except Exception:
+        return HBM_PEAK_FALLBACK, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    Q = ("index,clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.15)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=2)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 8:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = float(f[2])
+            except ValueError:
+                continue
+            for n, v in zip(names, f[4:8]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        load = [x for x in sm if mx and x > 0.3 * mx] or sm
+        return {"sm_mhz": statistics.median(load) if load else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def dist_setup():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+# ------------------------------------------------------------------------------------------------
+# CPU oracle legs (the reference arm and the cpu_baseline of our arm)
+# ------------------------------------------------------------------------------------------------
+def _gen_one(args):
+    n, seed, seconds, base = args
+    gp = mix_a_params(1, seed=seed, seconds=seconds, replica_base=base)
+    t = tick_trace(gp)
+    return t.arrival_us, t.meta
+
+
+def oracle_sample(n_rep: int, seconds: int, seed: int = 1, base: int = 0):
+    from concurrent.futures import ProcessPoolExecutor
+    from protean_inputs import concat
+    with ProcessPoolExecutor(max_workers=min(n_rep, os.cpu_count() or 1)) as ex:
+        parts = list(ex.map(_gen_one, [(1, seed, seconds, base + i) for i in range(n_rep)]))
+    tr = concat(parts, seconds * 1_000_000, base)
+    return tr
+
+
+def time_oracle(prof, tr, cores: int):
+    from oracle import oracle as O
+    O.build()
+    t0 = time.perf_counter()
+    out = O.replay(prof, tr, N=8, nthreads=cores)
+    dt = time.perf_counter() - t0
+    c = out["counters"]
+    return dt, int(c[:, 8].sum()), int((c[:, 0] + c[:, 4]).sum()), int(c[:, 9].sum())
+
+
+def run_reference(args):
+    world, rank, _ = dist_setup()
+    if rank != 0:
+        return 0
+    prof = synth_profiles()
+    cores = os.cpu_count() or 1
+    n_rep = max(1, min(args.replicas, 2 * cores))
+    tr = oracle_sample(n_rep, args.seconds)
+    for _ in range(args.warmup):
+        time_oracle(prof, tr, cores)
+    dts, slots, reqs = [], 0, 0
+    for _ in range(args.steps):
+        dt, s, q, _g = time_oracle(prof, tr, cores)
+        dts.append(dt)
+        slots, reqs = s, q
+    tot = sum(dts)
+    val = slots * args.steps / tot
+    sample = f"{n_rep} replicas x {args.seconds} s of the config-5 workload (Mix A, 8 sim-GPUs, G=12)"
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
+            "data": "synthetic",
+            "config": {"workload": "C5 (configs[4]) sample: Mix A, 8 sim-GPUs, 600 s, G=12, search policy",
+                       "replicas": n_rep, "seconds": args.seconds},
+            "simulated_requests_per_s": reqs * args.steps / tot,
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------------------------------------
+# our arm
+# ------------------------------------------------------------------------------------------------
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_middleware_bhasisjgpkd24_b200 as pkg
+    from tools import tracegen
+
+    world, rank, local = dist_setup()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    prof = synth_profiles()
+    R, S, N = args.replicas, args.seconds, 8
+    gp = mix_a_params(R, seed=1, seconds=S, replica_base=rank * R)
+    arr, meta, roff = tracegen.generate_on_device(gp, local)
+    n_req = int(arr.shape[0])
+    h = pkg.load_profiles(prof, device=local)
+    E = h.num_epochs(gp.trace_len_us)
+    out = h.alloc_replay_out(R, E, N, decisions=True)
+    stream = torch.cuda.current_stream(dev)
+    cfg = dict(n_gpus=N, replica_base=rank * R)
+
+    def step():
+        h.replay_traces(arr, meta, roff, trace_len_us=gp.trace_len_us, out=out, stream=stream, **cfg)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    clk = ClockSampler(local)
+    clk.start()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    kern_ms, pre_ms = [], []
+    for i in range(args.steps):
+        evs[i][0].record(stream)
+        step()
+        evs[i][1].record(stream)
+        p, k, launch = h.last_timings()
+        kern_ms.append(k)
+        pre_ms.append(p)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks = clk.stop()
+    step_ms = [a.elapsed_time(b) for a, b in evs]
+    tot_ms = sum(step_ms)
+    c = out["counters"].sum(0).cpu().numpy()
+    slot, geom_c, reqs = int(c[8]), int(c[9]), int(c[0] + c[4])
+    if world > 1:
+        t = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        tot_ms = float(t.item())
+        s = torch.tensor([slot, geom_c, reqs, n_req], dtype=torch.int64, device=dev)
+        dist.all_reduce(s)
+        slot, geom_c, reqs, n_req_all = [int(x) for x in s.tolist()]
+    else:
+        n_req_all = n_req
+    sec = tot_ms / 1e3
+    value = slot * args.steps / sec
+
+    # e2e: the public call on HOST buffers (pinned), H2D + replay + D2H inside the timed region
+    e2e = None
+    if rank == 0 and args.e2e_replicas > 0:
+        Re = min(args.e2e_replicas, R)
+        hi = int(roff[Re].item())
+        h_arr = torch.empty(hi, dtype=torch.int32, pin_memory=True)
+        h_meta = torch.empty(hi, dtype=torch.uint8, pin_memory=True)
+        h_off = torch.empty(Re + 1, dtype=torch.int64, pin_memory=True)
+        h_arr.copy_(arr[:hi])
+        h_meta.copy_(meta[:hi])
+        h_off.copy_(roff[:Re + 1])
+        eo = h.alloc_replay_out(Re, E, N, decisions=True)
+        d_arr = torch.empty_like(h_arr, device=dev)
+        d_meta = torch.empty_like(h_meta, device=dev)
+        d_off = torch.empty_like(h_off, device=dev)
+        res_bytes = sum(t.numel() * t.element_size() for k, t in eo.items() if hasattr(t, "numel"))
+        pinned_out = {k: torch.empty(t.shape, dtype=t.dtype, pin_memory=True)
+                      for k, t in eo.items() if hasattr(t, "numel")}
+
+        def e2e_step():
+            d_arr.copy_(h_arr, non_blocking=True)
+            d_meta.copy_(h_meta, non_blocking=True)
+            d_off.copy_(h_off, non_blocking=True)
+            h.replay_traces(d_arr, d_meta, d_off, trace_len_us=gp.trace_len_us, out=eo, stream=stream, **cfg)
+            for k, t in pinned_out.items():
+                t.copy_(eo[k], non_blocking=True)
+        e2e_step()
+        torch.cuda.synchronize()
+        ea, eb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ea.record(stream)
+        ks = max(1, min(args.steps, 3))
+        for _ in range(ks):
+            e2e_step()
+        eb.record(stream)
+        torch.cuda.synchronize()
+        ems = ea.elapsed_time(eb)
+        es = int(pinned_out["counters"][:, 8].sum())
+        e2e = {"value": es * ks / (ems / 1e3), "unit": UNIT,
+               "h2d_bytes_per_step": int(hi * 5 + (Re + 1) * 8), "d2h_bytes_per_step": int(res_bytes),
+               "sample": f"{Re} of {R} replicas through Handle.replay_traces from pinned host memory"}
+
+    cpu = None
+    if rank == 0 and world == 1 and args.cpu_sample > 0:
+        cores = os.cpu_count() or 1
+        n_rep = min(args.cpu_sample, R)
+        tr = oracle_sample(n_rep, S, base=0)
+        dt, s_cpu, q_cpu, _ = time_oracle(prof, tr, cores)
+        cpu = {"value": s_cpu / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
+               "sample": f"{n_rep} replicas x {S} s of this workload (numpy-generated), "
+                         f"{dt:.1f} s wall on {cores} threads",
+               "simulated_requests_per_s": q_cpu / dt}
+
+    if rank == 0:
+        peak, peak_kind = peaks()
+        k_ms = statistics.mean(kern_ms)
+        alg_bytes = 5.0 * n_req                      # 4 B arrival + 1 B meta per request, read once
+        achieved = alg_bytes / (k_ms / 1e3) / 1e9
+        traffic = None
+        prof_path = os.path.join(ROOT, "profiles", "ncu_summary.json")
+        if os.path.exists(prof_path):
+            try:
+                ps = json.load(open(prof_path))
+                traffic = ps["dram_bytes_per_request"] * n_req
+            except Exception:
+                traffic = None
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+            "config": {"workload": "C5 (configs[4]): Mix A Wiki-shaped 5000 rps, 22-model table, "
+                                   "8 sim-GPUs, 600 s, 12 geometries, search policy, on-demand VMs",
+                       "replicas_per_rank": R, "seconds": S, "sim_gpus": N, "geometries": h.n_geoms,
+                       "requests_per_rank": n_req, "l2_flush": "inputs (5 B/request, "
+                       f"{alg_bytes / 1e9:.1f} GB per rank) exceed the 126 MB L2"},
+            "simulated_requests_per_s": reqs * args.steps / sec,
+            "geom_candidates_per_s": geom_c * args.steps / sec,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
+                         "kernel": "replay_kernel", "kernel_ms": k_ms, "prepass_ms": statistics.mean(pre_ms),
+                         "launch": launch},
+            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": 2 * args.steps * world, "clocks": clocks,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--replicas", type=int, default=4096, help="replicas per rank")
+    ap.add_argument("--seconds", type=int, default=600)
+    ap.add_argument("--e2e-replicas", type=int, default=512)
+    ap.add_argument("--cpu-sample", type=int, default=64, help="replicas timed on the CPU oracle")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

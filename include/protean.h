@@ -115,7 +115,8 @@ int protean_num_epochs(const protean_handle *h, int64_t trace_len_us, int64_t ep
  *    placement, which advances `state`); and if the GPU is decidable at T (has_vm and
  *    recfg_end <= T) every candidate geometry j in [geom_lo, geom_hi) replays the same batch list
  *    from an idle GPU and is scored by key = misses<<40 | BE_tail<<8 | tag, tag 0 = current
- *    geometry, else j+1 (O8).  Asynchronous on `stream` (cudaStream_t; NULL = legacy default).  */
+ *    geometry, else j+1 (O8).  Enqueued on `stream` (cudaStream_t; NULL = legacy default); returns
+ *    after the stream completes, because the in-kernel validation verdict is read back.         */
 typedef struct {           /* 16 B */
   uint32_t ready_us;       /* batch ready time (O3): last member's arrival if full, else first + T_m */
   uint32_t req_off;        /* index of the batch's first member in arrival_us */
@@ -244,6 +245,12 @@ typedef struct {             /* caller-allocated, one row per replica of this ca
 
 int protean_replay_traces(protean_handle *h, const protean_replay_cfg *cfg,
                           protean_replay_out *out, void *stream);
+
+/* Device time (CUDA events on the launching stream) of the last protean_replay_traces call:
+ * the prepass kernel and the fused replay kernel, in ms; launch = {grid, block, dynamic smem
+ * bytes, resident CTAs per SM} of the replay kernel (any pointer may be NULL).  Host. */
+int protean_last_timings(const protean_handle *h, float *prepass_ms, float *replay_ms,
+                         int32_t *launch);
 
 /* Fill a replay config with the defaults listed above (host). */
 void protean_replay_cfg_defaults(protean_replay_cfg *cfg);

@@ -95,7 +95,7 @@ assert C.sizeof(BatchRec) == 32
 
 EXPORTS = ["protean_load_profiles", "protean_free", "protean_strerror", "protean_last_error",
            "protean_get_geometries", "protean_num_epochs", "protean_score_epoch",
-           "protean_replay_traces", "protean_replay_cfg_defaults"]
+           "protean_replay_traces", "protean_replay_cfg_defaults", "protean_last_timings"]
 
 _lib = None
 
@@ -121,6 +121,7 @@ def load(path: str = LIB_PATH, require_cuda: bool = True):
     L.protean_replay_traces.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
     L.protean_replay_cfg_defaults.argtypes = [C.c_void_p]
     L.protean_replay_cfg_defaults.restype = None
+    L.protean_last_timings.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
     _lib = L
     return L
 

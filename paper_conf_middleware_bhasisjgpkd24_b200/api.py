@@ -73,6 +73,13 @@ class Handle:
         _check(self._h, self._lib.protean_num_epochs(self._h, int(trace_len_us), int(epoch_len_us), C.byref(E)))
         return E.value
 
+    def last_timings(self):
+        """(prepass_ms, replay_kernel_ms, {grid, block, smem, per_sm}) of the last replay call."""
+        a, b = C.c_float(), C.c_float()
+        launch = (C.c_int32 * 4)()
+        _check(self._h, self._lib.protean_last_timings(self._h, C.byref(a), C.byref(b), launch))
+        return a.value, b.value, dict(zip(("grid", "block", "smem", "per_sm"), list(launch)))
+
     # -------------------------------------------------------------------------------- replay
     def alloc_replay_out(self, R: int, E: int, N: int, *, decisions=True, cand_keys=False, log_cap=0):
         torch = _torch()

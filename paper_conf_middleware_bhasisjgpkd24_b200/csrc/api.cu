@@ -30,6 +30,9 @@ struct protean_handle {
   int64_t* d_eoff = nullptr;
   size_t eoff_bytes = 0;
   void* d_small = nullptr;  // wmax (8 B) + err (16 B)
+  cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};  // prepass / replay kernel bracket
+  float t_prepass = 0.f, t_replay = 0.f;
+  int last_grid = 0, last_block = 0, last_smem = 0, last_per_sm = 0;
 };
 
 namespace {
@@ -242,6 +245,7 @@ int protean_load_profiles(const protean_profiles* p, protean_handle** out) {
   if (e == cudaSuccess)
     e = cudaMemcpy(h->d_tab, h->words.data(), sizeof(int32_t) * h->words.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMalloc(&h->d_small, 256);
+  for (int i = 0; i < 4 && e == cudaSuccess; ++i) e = cudaEventCreate(&h->ev[i]);
   if (e != cudaSuccess) {
     cudaGetLastError();
     protean_free(h);
@@ -258,7 +262,23 @@ void protean_free(protean_handle* h) {
   if (h->d_scratch) cudaFree(h->d_scratch);
   if (h->d_eoff) cudaFree(h->d_eoff);
   if (h->d_small) cudaFree(h->d_small);
+  for (int i = 0; i < 4; ++i)
+    if (h->ev[i]) cudaEventDestroy(h->ev[i]);
   delete h;
+}
+
+int protean_last_timings(const protean_handle* h, float* prepass_ms, float* replay_ms,
+                          int32_t* launch) {
+  if (!h) return PROTEAN_EINVAL;
+  if (prepass_ms) *prepass_ms = h->t_prepass;
+  if (replay_ms) *replay_ms = h->t_replay;
+  if (launch) {
+    launch[0] = h->last_grid;
+    launch[1] = h->last_block;
+    launch[2] = h->last_smem;
+    launch[3] = h->last_per_sm;
+  }
+  return PROTEAN_OK;
 }
 
 int protean_get_geometries(const protean_handle* h, int32_t* n, uint8_t* geoms) {
@@ -330,7 +350,9 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   unsigned long long* d_wmax = static_cast<unsigned long long*>(h->d_small);
   int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 64);
   CK(h, cudaMemsetAsync(h->d_small, 0, 256, st));
+  CK(h, cudaEventRecord(h->ev[0], st));
   CK(h, launch_prepass(c.arrival_us, c.replica_off, R, E, W, h->maxT, h->d_eoff, d_wmax, d_err, st));
+  CK(h, cudaEventRecord(h->ev[1], st));
   unsigned long long wmax = 0;
   int herr = 0;
   CK(h, cudaMemcpyAsync(&wmax, d_wmax, 8, cudaMemcpyDeviceToHost, st));
@@ -425,9 +447,17 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   }
   P.scratch = static_cast<char*>(h->d_scratch);
   P.err = d_err;
+  CK(h, cudaEventRecord(h->ev[2], st));
   CK(h, launch_replay(P, grid, block, st));
+  CK(h, cudaEventRecord(h->ev[3], st));
   CK(h, cudaMemcpyAsync(&herr, d_err, 4, cudaMemcpyDeviceToHost, st));
   CK(h, cudaStreamSynchronize(st));
+  CK(h, cudaEventElapsedTime(&h->t_prepass, h->ev[0], h->ev[1]));
+  CK(h, cudaEventElapsedTime(&h->t_replay, h->ev[2], h->ev[3]));
+  h->last_grid = grid;
+  h->last_block = block;
+  h->last_smem = (int)sl.total;
+  h->last_per_sm = per_sm;
   if (herr) return fail(h, PROTEAN_EINVAL, "invalid request (unsorted, model id, or arrival >= trace_len)");
   return PROTEAN_OK;
 }

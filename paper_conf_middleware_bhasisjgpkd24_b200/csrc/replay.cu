@@ -138,8 +138,6 @@ __device__ __forceinline__ int hits_in(const Ctx& c, int pos, int n, int64_t end
   return n - lo;
 }
 
-__device__ __forceinline__ unsigned lane_id() { return threadIdx.x & 31; }
-
 }  // namespace
 
 __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
@@ -193,7 +191,7 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
 
   for (int r = blockIdx.x; r < P.R; r += gridDim.x) {
     const uint64_t replica = (uint64_t)(P.base + r);
-    const int64_t r_lo = P.roff[r], r_hi = P.roff[r + 1];
+    const int64_t r_lo = P.roff[r];
     const int64_t* eoff = P.eoff + (size_t)r * (P.E + 1);
     uint32_t* ghist = P.hist + (size_t)r * 2 * kNB;
     int64_t cnt[10];
