@@ -364,14 +364,15 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
 
   // launch geometry
   const int Gc = h->G;
-  const int nl = N * (1 + Gc);
+  const int LPG = (1 + Gc) <= 16 ? 16 : ((1 + Gc + 31) / 32) * 32;  // lanes per simulated GPU
+  const int nl = N * LPG;
   int block = ((nl + 31) / 32) * 32;
-  block = std::max(128, std::min(1024, block));
+  block = std::max(128, std::min(256, block));
   SmemLayout sl;
   sl.init(h->tl.words, h->M, N, Gc, 0, 0);
   const size_t fixed = sl.total;
   size_t budget = 72 * 1024;
-  int BS = std::min(WCAP, 256);
+  int BS = std::min(WCAP, 64);
   if (const char* ev = std::getenv("PROTEAN_SMEM_BUDGET_KB")) {  // test knob: force spill paths
     budget = (size_t)std::atoi(ev) * 1024;
     BS = std::min(BS, std::max(1, std::atoi(ev)));
@@ -513,7 +514,7 @@ int protean_score_epoch(protean_handle* h, const protean_epoch_in* in, protean_e
   P.scratch = static_cast<protean_resident*>(h->d_scratch);
   P.err = d_err;
   const int nl = N * (1 + Gc);
-  int block = std::max(128, std::min(1024, ((nl + 31) / 32) * 32));
+  int block = std::max(128, std::min(256, ((nl + 31) / 32) * 32));
   CK(h, launch_score(P, block, st));
   int errs[2] = {0, 0};
   CK(h, cudaMemcpyAsync(errs, d_err, 8, cudaMemcpyDeviceToHost, st));

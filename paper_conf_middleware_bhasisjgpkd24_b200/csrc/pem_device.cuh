@@ -77,8 +77,42 @@ __device__ __forceinline__ int64_t exec_time(int32_t solo, int64_t F) {
   return ((int64_t)solo * f) / kPpm;
 }
 
+// Rare path of Place for one slice (memory wait, or a resident starting after t0): the plain
+// definition of O6(a)/(b) by explicit scans.  Kept out of line to keep the hot loop small.
+static __device__ __noinline__ void place_slow_slice(const Tab& T, const uint8_t* gp, Rows L, int n, int s,
+                                              int p, int64_t t0, int32_t q, int m, int64_t* start_out,
+                                              int64_t* F_out) {
+  const int32_t Ms = prof_cap(p);
+  int64_t used = 0;
+  for (int i = 0; i < n; ++i)
+    if ((int)(L.meta(i) & 0xFF) == s && L.en(i) > t0) used += L.mem(i);
+  int64_t start = t0;
+  if (used + q > Ms) {  // earliest release that makes the batch fit
+    start = INT64_MAX;
+    for (int i = 0; i < n; ++i) {
+      if ((int)(L.meta(i) & 0xFF) != s || L.en(i) <= t0) continue;
+      const int64_t ei = L.en(i);
+      int64_t rem = 0;
+      for (int j = 0; j < n; ++j)
+        if ((int)(L.meta(j) & 0xFF) == s && L.en(j) > ei) rem += L.mem(j);
+      if (rem + q <= Ms && ei < start) start = ei;
+    }
+  }
+  int64_t F = T.fbr[m * kNProf + p];
+  for (int i = 0; i < n; ++i) {
+    const uint32_t mt = L.meta(i);
+    if ((int)(mt & 0xFF) == s && L.st(i) <= start && start < L.en(i))
+      F += T.fbr[((mt >> 8) & 0xFF) * kNProf + gp[s]];
+  }
+  *start_out = start;
+  *F_out = F;
+}
+
 // Place one batch (model m, class strict, ready t) on geometry `geom` over list L (n rows).
-// ls[] = last start per slice position (FIFO).  Returns the chosen slice and [start, end).
+// ls[] = last start per slice position (FIFO).  One pass over the residents accumulates, per
+// slice, the memory still held after t0_s = max(t, last_start_s) and the FBR of those residents;
+// since every resident of a slice started at or before its last start (FIFO), they are exactly
+// Eq 1's co-runners at t0_s.  The rare memory-wait case takes place_slow_slice().
 __device__ __forceinline__ PlaceRes place_lane(const Tab& T, int geom, Rows L, int& n,
                                                int64_t (&ls)[kMaxSl], int64_t t, int m,
                                                bool strict, int max_live) {
@@ -86,12 +120,33 @@ __device__ __forceinline__ PlaceRes place_lane(const Tab& T, int geom, Rows L, i
   o.dropped = 0;
   o.slice = -1;
   o.start = o.end = 0;
-  // residents that ended by t can never matter again: stable compaction
+  const uint8_t* gp = T.gprof + geom * 8;
+  int64_t t0[kMaxSl];
+  int32_t used[kMaxSl], fs[kMaxSl];
+  uint32_t fut = 0;
+#pragma unroll
+  for (int x = 0; x < kMaxSl; ++x) {
+    t0[x] = t > ls[x] ? t : ls[x];
+    used[x] = 0;
+    fs[x] = 0;
+  }
+  int32_t be_mem = 0;
   int k = 0;
   for (int i = 0; i < n; ++i) {
-    if (L.en(i) > t) {
-      if (k != i) L.r[k] = L.r[i];
-      ++k;
+    const protean_resident r = L.r[i];
+    if (r.end_us <= t) continue;  // ended: can never matter again (stable compaction)
+    if (k != i) L.r[k] = r;
+    ++k;
+    const int s = r.slice;
+    if (!r.strict) be_mem += r.mem_mib;
+    const int32_t f = T.fbr[r.model * kNProf + gp[s]];
+#pragma unroll
+    for (int x = 0; x < kMaxSl; ++x) {
+      if (x == s && r.end_us > t0[x]) {
+        used[x] += r.mem_mib;
+        fs[x] += f;
+        if (r.start_us > t0[x]) fut |= 1u << x;
+      }
     }
   }
   n = k;
@@ -101,47 +156,28 @@ __device__ __forceinline__ PlaceRes place_lane(const Tab& T, int geom, Rows L, i
   }
   const int32_t q = T.mem[m];
   const int ns = T.gn[geom];
-  int64_t be_mem = 0;  // Alg 1 line 1: BE memory on this GPU (reading Q5)
-  for (int i = 0; i < n; ++i)
-    if (!((L.meta(i) >> 16) & 1)) be_mem += L.mem(i);
-
   uint64_t best = ~0ull;
   int64_t bstart = 0, bend = 0;
 #pragma unroll
-  for (int s = 0; s < kMaxSl; ++s) {
-    if (s < ns) {
-      const int p = T.gprof[geom * 8 + s];
+  for (int x = 0; x < kMaxSl; ++x) {
+    if (x < ns) {
+      const int p = gp[x];
       const int32_t Ms = prof_cap(p);
       if (q <= Ms) {
-        const int64_t t0 = t > ls[s] ? t : ls[s];
-        int64_t used = 0;
-        for (int i = 0; i < n; ++i)
-          if ((int)(L.meta(i) & 0xFF) == s && L.en(i) > t0) used += L.mem(i);
-        int64_t start = t0;
-        if (used + q > Ms) {  // memory wait: earliest release that makes the batch fit
-          start = INT64_MAX;
-          for (int i = 0; i < n; ++i) {
-            if ((int)(L.meta(i) & 0xFF) != s || L.en(i) <= t0) continue;
-            const int64_t ei = L.en(i);
-            int64_t rem = 0;
-            for (int j = 0; j < n; ++j)
-              if ((int)(L.meta(j) & 0xFF) == s && L.en(j) > ei) rem += L.mem(j);
-            if (rem + q <= Ms && ei < start) start = ei;
-          }
-        }
-        int64_t F = T.fbr[m * kNProf + p];  // Eq 1's co-located sum at the start instant
-        for (int i = 0; i < n; ++i) {
-          const uint32_t mt = L.meta(i);
-          if ((int)(mt & 0xFF) == s && L.st(i) <= start && start < L.en(i))
-            F += T.fbr[((mt >> 8) & 0xFF) * kNProf + p];
+        int64_t start, F;
+        if (used[x] + q <= Ms && !((fut >> x) & 1)) {
+          start = t0[x];
+          F = (int64_t)T.fbr[m * kNProf + p] + fs[x];
+        } else {
+          place_slow_slice(T, gp, L, n, x, p, t0[x], q, m, &start, &F);
         }
         const int64_t c = start + exec_time(T.solo[m * kNProf + p], F);
         uint64_t key;
         if (strict) {  // choose_strict_slice: tag < 1, least eta == least completion (Q11)
-          const uint64_t inelig = (be_mem >= T.gpref[geom * 8 + s]) ? (1ull << 62) : 0ull;
-          key = inelig | ((uint64_t)c << 6) | ((uint64_t)(4 - p) << 3) | (uint64_t)s;
+          const uint64_t inelig = (be_mem >= T.gpref[geom * 8 + x]) ? (1ull << 62) : 0ull;
+          key = inelig | ((uint64_t)c << 6) | ((uint64_t)(4 - p) << 3) | (uint64_t)x;
         } else {       // choose_best_effort_slice: first fit, else earliest start (Q12)
-          key = ((uint64_t)start << 3) | (uint64_t)s;
+          key = ((uint64_t)start << 3) | (uint64_t)x;
         }
         if (key < best) {
           best = key;

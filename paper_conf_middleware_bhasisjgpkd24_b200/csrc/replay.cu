@@ -119,10 +119,12 @@ __device__ void vm_event(const ReplayParams& P, const Ctx& c, uint64_t replica, 
 
 __device__ __forceinline__ void install(const Ctx& c, int g) { reset_gpu_state(c, g, c.g_target[g]); }
 
-__device__ __forceinline__ void hist_add(const Ctx& c, uint32_t* ghist, int idx) {
+// Packed u16 smem histogram; a half crossing 2^15 moves 2^15 counts to the HBM histogram
+// (cnt <= 32 per call, so a half never exceeds 0xFFFF before the move).
+__device__ __forceinline__ void hist_add(const Ctx& c, uint32_t* ghist, int idx, uint32_t cnt) {
   const int w = idx >> 1, sh = (idx & 1) * 16;
-  const uint32_t old = atomicAdd(&c.hist[w], 1u << sh);
-  if (((old >> sh) & 0xFFFFu) == 0x7FFFu) {  // packed u16 half reached 2^15: move it to HBM
+  const uint32_t old = (atomicAdd(&c.hist[w], cnt << sh) >> sh) & 0xFFFFu;
+  if (old < 0x8000u && old + cnt >= 0x8000u) {
     atomicSub(&c.hist[w], 0x8000u << sh);
     atomicAdd(&ghist[idx], 0x8000u);
   }
@@ -140,7 +142,7 @@ __device__ __forceinline__ int hits_in(const Ctx& c, int pos, int n, int64_t end
 
 }  // namespace
 
-__global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
+__global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ CtaState cs;
   const SmemLayout& SL = P.sl;
@@ -149,6 +151,7 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
 
   Ctx c;
   int32_t* tabw = reinterpret_cast<int32_t*>(smem + SL.tab);
+#pragma unroll 1
   for (int i = tid; i < P.tl.words; i += NT) tabw[i] = P.tab[i];
   c.T.bind(tabw, P.tl);
   c.hist = reinterpret_cast<uint32_t*>(smem + SL.hist);
@@ -186,9 +189,12 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
   const Tab& T = c.T;
   int sum_slots = 0;  // sum of slice counts over the candidate range (slot-evals per batch)
   __syncthreads();
+#pragma unroll 1
   for (int j = P.geom_lo; j < P.geom_hi; ++j) sum_slots += T.gn[j];
-  const int nl = N * (1 + Gc);
+  const int LPG = (1 + Gc) <= 16 ? 16 : ((1 + Gc + 31) / 32) * 32;  // lanes per simulated GPU
+  const int nlp = N * LPG;
 
+#pragma unroll 1
   for (int r = blockIdx.x; r < P.R; r += gridDim.x) {
     const uint64_t replica = (uint64_t)(P.base + r);
     const int64_t r_lo = P.roff[r];
@@ -199,9 +205,13 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
     for (int i = 0; i < 10; ++i) cnt[i] = 0;
 
     // ---------------------------------------------------------------- replica init
+#pragma unroll 1
     for (int i = tid; i < kNB; i += NT) c.hist[i] = 0;          // kNB words = 2*3328 halves
+#pragma unroll 1
     for (int i = tid; i < 2 * kNB; i += NT) ghist[i] = 0;
+#pragma unroll 1
     for (int k = tid; k < S; k += NT) c.s_skip[k] = 0;
+#pragma unroll 1
     for (int g = tid; g < N; g += NT) {
       reset_gpu_state(c, g, P.init_geom);
       c.g_vm[g] = c.g_bill[g] = (P.vm_policy == 0) ? VM_OD : VM_SPOT;
@@ -221,12 +231,16 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
     }
     __syncthreads();
 
+#pragma unroll 1
     for (int64_t e = 0; e < P.E; ++e) {
       const int64_t eW = e * P.W, Tend = eW + P.W;
       // ---------------------------------------------------------------- A: VM events, installs
+#pragma unroll 1
       for (int i = tid; i < kNSeg * S; i += NT) c.s_cnt[i] = 0;
+#pragma unroll 1
       for (int g = tid; g < N; g += NT) {
         if (P.vm_policy != 0) {
+#pragma unroll 1
           for (int64_t k = (eW + P.rev - 1) / P.rev; k * P.rev < Tend; ++k) {
             const int64_t tau = k * P.rev;
             if (k < 1 || tau >= P.H) continue;
@@ -249,6 +263,7 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
       const int64_t w_beg = eoff[e], w_end = eoff[e + 1];
       const int64_t w_lo = cs.w_lo;
       __syncthreads();
+#pragma unroll 1
       for (int g = tid; g < N; g += NT) {
         const bool whole = c.g_from[g] <= eW && c.g_until[g] >= Tend &&
                            !(c.g_rs[g] < Tend && c.g_re[g] > eW);
@@ -260,29 +275,37 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
         if (tid == 0) atomicOr(P.err, 1);
       }
       // ---------------------------------------------------------------- B: stream partition
-      if (!bad_window && warp < kNSeg) {
+      if (!bad_window && warp < kNSeg) {  // count per (segment, stream); 4 loads in flight per lane
         const int64_t a = w_lo + len * warp / kNSeg, b = w_lo + len * (warp + 1) / kNSeg;
         int* cntw = c.s_cnt + warp * S;
-        for (int64_t i = a + lane; i < b; i += 32) {
-          const uint8_t mt = P.meta[i];
-          int m = mt & 63;
-          if (i >= w_beg) {  // validate each request once (when it is new)
-            const uint32_t ai = P.arr[i];
-            if ((mt & 0x40) || m >= T.M || (int64_t)ai >= P.trace_len ||
-                (i > r_lo && ai < P.arr[i - 1]))
-              atomicOr(P.err, 1);
+#pragma unroll 1
+        for (int64_t i0 = a; i0 < b; i0 += 128) {
+          uint8_t mt[4];
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const int64_t i = i0 + u * 32 + lane;
+            mt[u] = i < b ? P.meta[i] : (uint8_t)0xFF;
           }
-          if (m >= T.M) m = 0;
-          atomicAdd(&cntw[2 * m + ((mt >> 7) ? 0 : 1)], 1);
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const bool valid = i0 + u * 32 + lane < b;
+            int m = mt[u] & 63;
+            if (m >= T.M) m = 0;
+            const int key = valid ? 2 * m + ((mt[u] >> 7) ? 0 : 1) : 1024 + lane;
+            const unsigned peers = __match_any_sync(0xffffffffu, key);
+            if (valid && (peers & ((1u << lane) - 1u)) == 0) cntw[key] += __popc(peers);
+          }
         }
       }
       __syncthreads();
       if (warp == 0) {  // stream offsets: per-stream totals, exclusive scan over streams
         int carry = 0;
+#pragma unroll 1
         for (int k0 = 0; k0 < S; k0 += 32) {
           const int k = k0 + lane;
           int tot = 0;
           if (k < S) {
+#pragma unroll 1
             for (int w = 0; w < kNSeg; ++w) {
               const int cv = c.s_cnt[w * S + k];
               c.s_run[w * S + k] = tot;
@@ -299,38 +322,53 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
           if (k < S) {
             c.s_base[k] = base;
             c.s_tot[k] = tot;
+#pragma unroll 1
             for (int w = 0; w < kNSeg; ++w) c.s_run[w * S + k] += base;
           }
           carry += __shfl_sync(0xffffffffu, x, 31);
         }
       }
       __syncthreads();
-      if (!bad_window && warp < kNSeg) {  // stable scatter into stream-sorted order
+      if (!bad_window && warp < kNSeg) {  // stable scatter into stream-sorted order + validation
         const int64_t a = w_lo + len * warp / kNSeg, b = w_lo + len * (warp + 1) / kNSeg;
         int* runw = c.s_run + warp * S;
-        for (int64_t i0 = a; i0 < b; i0 += 32) {
-          const int64_t i = i0 + lane;
-          const bool valid = i < b;
-          int key = 1024 + lane;
-          uint32_t ai = 0;
-          if (valid) {
-            const uint8_t mt = P.meta[i];
-            int m = mt & 63;
-            if (m >= T.M) m = 0;
-            key = 2 * m + ((mt >> 7) ? 0 : 1);
-            ai = P.arr[i];
+#pragma unroll 1
+        for (int64_t i0 = a; i0 < b; i0 += 128) {
+          uint8_t mt[4];
+          uint32_t ai[4], ap[4];
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const int64_t i = i0 + u * 32 + lane;
+            const bool valid = i < b;
+            mt[u] = valid ? P.meta[i] : (uint8_t)0;
+            ai[u] = valid ? P.arr[i] : 0u;
+            ap[u] = (valid && i >= w_beg && i > r_lo) ? P.arr[i - 1] : 0u;
           }
-          const unsigned peers = __match_any_sync(0xffffffffu, key);
-          const unsigned rank = __popc(peers & ((1u << lane) - 1u));
-          if (valid) c.sa(runw[key] + (int)rank) = ai;
-          __syncwarp();
-          if (valid && rank == 0) runw[key] += __popc(peers);
-          __syncwarp();
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const int64_t i = i0 + u * 32 + lane;
+            const bool valid = i < b;
+            int m = mt[u] & 63;
+            if (valid && i >= w_beg &&  // validate each request once (when it is new)
+                ((mt[u] & 0x40) || m >= T.M || (int64_t)ai[u] >= P.trace_len || ai[u] < ap[u]))
+              atomicOr(P.err, 1);
+            if (m >= T.M) m = 0;
+            const int key = valid ? 2 * m + ((mt[u] >> 7) ? 0 : 1) : 1024 + lane;
+            const unsigned peers = __match_any_sync(0xffffffffu, key);
+            const unsigned rank = __popc(peers & ((1u << lane) - 1u));
+            if (valid) c.sa(runw[key] + (int)rank) = ai[u];
+            __syncwarp();
+            if (valid && rank == 0) runw[key] += __popc(peers);
+            __syncwarp();
+          }
         }
       }
       __syncthreads();
       // ---------------------------------------------------------------- C: batch formation
-      for (int k = tid; k < S; k += NT) {
+      // warp per stream: lanes test 32 consecutive B-sized batches at once (full batches are the
+      // common case); a batch closed by the timeout, or still open, is resolved by lane 0.
+#pragma unroll 1
+      for (int k = warp; k < S; k += NW) {
         if (bad_window) break;
         const int m = k >> 1;
         const bool strict = (k & 1) == 0;
@@ -341,49 +379,77 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
         int pend = 0;
         uint32_t a0p = 0xFFFFFFFFu;
         while (i < end) {
-          const int64_t a0 = c.sa(i);
-          const int64_t deadline = a0 + Tm;
-          const int lim = (end - i > B) ? i + B : end;
-          int j;
-          if ((int64_t)c.sa(lim - 1) <= deadline) {
-            j = lim;
-          } else {  // first member beyond the timeout
-            int lo = i + 1, hi = lim - 1;
+          const int64_t st = (int64_t)i + (int64_t)lane * B;
+          bool full = false;
+          if (st + B <= end) full = (int64_t)c.sa((int)(st + B - 1)) <= (int64_t)c.sa((int)st) + Tm;
+          const unsigned fm = __ballot_sync(0xffffffffu, full);
+          const int nfull = __ffs(~fm) ? __ffs(~fm) - 1 : 32;
+          int slot0 = 0;
+          if (lane == 0 && nfull) slot0 = atomicAdd(&cs.nb, nfull);
+          slot0 = __shfl_sync(0xffffffffu, slot0, 0);
+          if (lane < nfull) {
+            const int ii = (int)st;
+            const uint32_t ready = c.sa(ii + B - 1);
+            Bat& bt = c.bat(slot0 + lane);
+            bt.key = ((uint64_t)ready << 32) | ((uint64_t)(strict ? 0 : 1) << 31) |
+                     ((uint64_t)m << 25) | (uint64_t)(ii & 0x1FFFFFF);
+            bt.ready = ready;
+            bt.info = (uint32_t)B | ((uint32_t)m << 16) | ((uint32_t)(strict ? 1 : 0) << 24);
+            bt.pos = (uint32_t)ii;
+            bt.gpu = 0xFF;
+            bt.slice = 0xFF;
+            bt.drop = 0;
+            bt.start = bt.end = 0;
+          }
+          i += nfull * B;
+          if (nfull == 32) continue;
+          if (i >= end) break;
+          // batch starting at i is not full within this window: lane 0 resolves it
+          int j = 0, state = 0;  // state 0 emit, 1 pending
+          int64_t ready = 0;
+          if (lane == 0) {
+            const int64_t a0 = c.sa(i);
+            const int64_t deadline = a0 + Tm;
+            const int lim = (end - i > B) ? i + B : end;
+            int lo = i + 1, hi = lim;  // first member beyond the timeout, else lim
             while (lo < hi) {
               const int mid = (lo + hi) >> 1;
               if ((int64_t)c.sa(mid) > deadline) hi = mid; else lo = mid + 1;
             }
             j = lo;
+            if (j - i == B) ready = c.sa(j - 1);        // full (only possible at the window end)
+            else if (j < end) ready = deadline;         // a later arrival missed the timeout
+            else if (deadline < Tend) ready = deadline; // timed out inside this epoch
+            else { state = 1; pend = end - i; a0p = (uint32_t)a0; }
+            if (state == 0) {
+              const int slot = atomicAdd(&cs.nb, 1);
+              Bat& bt = c.bat(slot);
+              bt.key = ((uint64_t)ready << 32) | ((uint64_t)(strict ? 0 : 1) << 31) |
+                       ((uint64_t)m << 25) | (uint64_t)(i & 0x1FFFFFF);
+              bt.ready = (uint32_t)ready;
+              bt.info = (uint32_t)(j - i) | ((uint32_t)m << 16) | ((uint32_t)(strict ? 1 : 0) << 24);
+              bt.pos = (uint32_t)i;
+              bt.gpu = 0xFF;
+              bt.slice = 0xFF;
+              bt.drop = 0;
+              bt.start = bt.end = 0;
+            }
           }
-          int64_t ready;
-          if (j - i == B) ready = c.sa(j - 1);          // full
-          else if (j < end) ready = deadline;           // a later arrival missed the timeout
-          else if (deadline < Tend) ready = deadline;   // timed out inside this epoch
-          else {                                        // still open: carried to the next epoch
-            pend = end - i;
-            a0p = (uint32_t)a0;
-            break;
-          }
-          const int slot = atomicAdd(&cs.nb, 1);
-          Bat& bt = c.bat(slot);
-          bt.key = ((uint64_t)ready << 32) | ((uint64_t)(strict ? 0 : 1) << 31) |
-                   ((uint64_t)m << 25) | (uint64_t)(i & 0x1FFFFFF);
-          bt.ready = (uint32_t)ready;
-          bt.info = (uint32_t)(j - i) | ((uint32_t)m << 16) | ((uint32_t)(strict ? 1 : 0) << 24);
-          bt.pos = (uint32_t)i;
-          bt.gpu = 0xFF;
-          bt.slice = 0xFF;
-          bt.drop = 0;
-          bt.start = bt.end = 0;
+          state = __shfl_sync(0xffffffffu, state, 0);
+          j = __shfl_sync(0xffffffffu, j, 0);
+          if (state) break;
           i = j;
         }
-        c.s_pend[k] = pend;
-        if (pend) atomicMin(&cs.amin, a0p);
+        if (lane == 0) {
+          c.s_pend[k] = pend;
+          if (pend) atomicMin(&cs.amin, a0p);
+        }
       }
       __syncthreads();
       const int nb = cs.nb;
       const unsigned amin = cs.amin;
       // next window: stream entries at/after the earliest open batch's first arrival are re-read
+#pragma unroll 1
       for (int k = tid; k < S; k += NT) {
         if (bad_window) break;
         const int b0 = c.s_base[k], tot = c.s_tot[k];
@@ -396,9 +462,11 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
         if (lo) atomicAdd(reinterpret_cast<unsigned long long*>(&cs.lt_total), (unsigned long long)lo);
         c.s_skip[k] = ge - c.s_pend[k];
       }
+#pragma unroll 1
       for (int b = tid; b < nb; b += NT) {  // id order (O3): rank by key
         const uint64_t kb = c.bat(b).key;
         int rank = 0;
+#pragma unroll 1
         for (int x = 0; x < nb; ++x) rank += (c.bat(x).key < kb) ? 1 : 0;
         c.ord(rank) = (uint32_t)b;
       }
@@ -407,13 +475,16 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
       // ---------------------------------------------------------------- D: dispatch
       if (cs.all_avail) {
         const int cursor = cs.cursor;
+#pragma unroll 1
         for (int rk = tid; rk < nb; rk += NT) c.bat(c.ord(rk)).gpu = (uint8_t)((cursor + rk) % N);
+#pragma unroll 1
         for (int g = tid; g < N; g += NT) {
           const int d = (g - cursor % N + N) % N;
           const int cntg = d < nb ? (nb - d + N - 1) / N : 0;
           c.g_cnt[g] = cntg;
           // offset = sum of counts of GPUs before g
           int off = 0;
+#pragma unroll 1
           for (int h = 0; h < g; ++h) {
             const int dh = (h - cursor % N + N) % N;
             off += dh < nb ? (nb - dh + N - 1) / N : 0;
@@ -422,24 +493,69 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
           if (g == N - 1) c.g_off[N] = off + cntg;
         }
         __syncthreads();
+#pragma unroll 1
         for (int rk = tid; rk < nb; rk += NT) {
           const int g = (cursor + rk) % N;
           c.gl(c.g_off[g] + rk / N) = c.ord(rk);
         }
         if (tid == 0) cs.cursor = (int)((cursor + nb) % N);
+      } else if (N <= 32) {
+        if (warp == 0) {  // lanes = simulated GPUs; availability masks + cursor chase
+          int64_t fr = 0, un = 0, rs = 0, re = 0;
+          if (lane < N) { fr = c.g_from[lane]; un = c.g_until[lane]; rs = c.g_rs[lane]; re = c.g_re[lane]; }
+          int cur = cs.cursor, mycnt = 0;
+#pragma unroll 1
+          for (int rk = 0; rk < nb; ++rk) {
+            Bat& bt = c.bat(c.ord(rk));
+            const int64_t t = bt.ready;
+            const bool av = lane < N && fr <= t && t < un && !(rs <= t && t < re);
+            const unsigned am = __ballot_sync(0xffffffffu, av);
+            int chosen = -1;
+            if (am) {
+              const unsigned hi = am & ~((1u << cur) - 1u);
+              chosen = hi ? __ffs(hi) - 1 : __ffs(am) - 1;
+              cur = (chosen + 1) % N;
+              if (lane == chosen) ++mycnt;
+            }
+            if (lane == 0) {
+              bt.gpu = chosen < 0 ? (uint8_t)0xFF : (uint8_t)chosen;
+              if (chosen < 0) bt.drop = 1;  // dispatch drop
+            }
+          }
+          int x = mycnt;
+#pragma unroll
+          for (int d = 1; d < 32; d <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, x, d);
+            if (lane >= d) x += y;
+          }
+          if (lane < N) c.g_off[lane] = x - mycnt;
+          if (lane == N - 1) c.g_off[N] = x;
+          __syncwarp();
+          int fill = 0;
+#pragma unroll 1
+          for (int rk = 0; rk < nb; ++rk) {
+            const uint32_t b = c.ord(rk);
+            const int g = c.bat(b).gpu;
+            if (lane == g) c.gl(c.g_off[lane] + fill++) = b;
+          }
+          if (lane == 0) cs.cursor = cur;
+        }
       } else {
         if (tid == 0) {
           int cur = cs.cursor;
+#pragma unroll 1
           for (int g = 0; g < N; ++g) c.g_cnt[g] = 0;
+#pragma unroll 1
           for (int rk = 0; rk < nb; ++rk) {
             Bat& bt = c.bat(c.ord(rk));
             int chosen = -1;
+#pragma unroll 1
             for (int i = 0; i < N; ++i) {
               const int g = (cur + i) % N;
               if (available(c, g, bt.ready)) { chosen = g; break; }
             }
             if (chosen < 0) {
-              bt.drop = 1;  // dispatch drop
+              bt.drop = 1;
               bt.gpu = 0xFF;
             } else {
               bt.gpu = (uint8_t)chosen;
@@ -448,12 +564,14 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
             }
           }
           int off = 0;
+#pragma unroll 1
           for (int g = 0; g < N; ++g) {
             c.g_off[g] = off;
             off += c.g_cnt[g];
             c.g_cnt[g] = 0;
           }
           c.g_off[N] = off;
+#pragma unroll 1
           for (int rk = 0; rk < nb; ++rk) {
             const uint32_t b = c.ord(rk);
             const Bat& bt = c.bat(b);
@@ -465,87 +583,75 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
       }
       __syncthreads();
       // ---------------------------------------------------------------- E: placement lanes
-      for (int L = tid; L < nl; L += NT) {
-        const int g = L / (1 + Gc), v = L - g * (1 + Gc);
+      // lane = (GPU g, v): v = 0 the actual placement on the current geometry (carried state),
+      // v = 1..Gc candidate geometry v-1 replayed from idle on the same batch list (O8).
+#pragma unroll 1
+      for (int L = tid; L < nlp; L += NT) {
+        const int g = L / LPG, v = L - g * LPG;
+        if (g >= N || v > Gc) continue;
+        const bool actual = v == 0;
+        const int j = actual ? (int)c.g_geom[g] : P.geom_lo + v - 1;
+        if (!actual && !(P.policy == 0 && c.g_dec[g])) {
+          c.keys[g * Gc + v - 1] = -1;
+          if (P.cand_keys) P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = -1;
+          continue;
+        }
         const int x0 = c.g_off[g], x1 = c.g_off[g + 1];
         Rows rows{c.lists + (size_t)L * P.max_live};
-        if (v == 0) {  // the actual placement on the current geometry, carried state
-          const int geom = c.g_geom[g];
-          int n = c.lane_n[g];
-          int64_t ls[kMaxSl], bu[kMaxSl];
+        int n = actual ? c.lane_n[g] : 0;
+        int64_t ls[kMaxSl];
 #pragma unroll
-          for (int s = 0; s < kMaxSl; ++s) {
-            ls[s] = c.ls[g * kMaxSl + s];
-            bu[s] = c.bu[g * kMaxSl + s];
-          }
-          int64_t busy = 0, memt = 0;
-          for (int x = x0; x < x1; ++x) {
-            Bat& bt = c.bat(c.gl(x));
-            const int m = (bt.info >> 16) & 0xFF;
-            const bool strict = (bt.info >> 24) & 1;
-            const PlaceRes pr = place_lane(T, geom, rows, n, ls, bt.ready, m, strict, P.max_live);
+        for (int s = 0; s < kMaxSl; ++s) ls[s] = actual ? c.ls[g * kMaxSl + s] : 0;
+        int64_t acc0 = 0, acc1 = 0;  // actual: busy, mem-time;  candidate: misses, BE tail
+#pragma unroll 1
+        for (int x = x0; x < x1; ++x) {
+          Bat& bt = c.bat(c.gl(x));
+          const uint32_t info = bt.info;
+          const int m = (info >> 16) & 0xFF, nreq = info & 0xFFFF;
+          const bool strict = (info >> 24) & 1;
+          const PlaceRes pr = place_lane(T, j, rows, n, ls, bt.ready, m, strict, P.max_live);
+          if (actual) {
             bt.drop = (uint8_t)pr.dropped;
             bt.slice = pr.dropped ? 0xFF : (uint8_t)pr.slice;
             bt.start = pr.dropped ? 0 : pr.start;
             bt.end = pr.dropped ? 0 : pr.end;
             if (!pr.dropped) {  // busy union + memory-time, clipped to [0, H) (reading Q29)
-              const int p = T.gprof[geom * 8 + pr.slice];
-#pragma unroll
-              for (int s = 0; s < kMaxSl; ++s) {
-                if (s == pr.slice) {
-                  const int64_t lo = pr.start > bu[s] ? pr.start : bu[s];
-                  const int64_t hi = pr.end < P.H ? pr.end : P.H;
-                  if (hi > lo) busy += (int64_t)prof_compute(p) * (hi - lo);
-                  if (pr.end > bu[s]) bu[s] = pr.end;
-                }
-              }
-              const int64_t mhi = pr.end < P.H ? pr.end : P.H;
-              if (mhi > pr.start) memt += (int64_t)T.mem[m] * (mhi - pr.start);
+              int64_t& b_until = c.bu[g * kMaxSl + pr.slice];
+              const int64_t b_old = b_until;
+              const int p = T.gprof[j * 8 + pr.slice];
+              const int64_t lo = pr.start > b_old ? pr.start : b_old;
+              const int64_t hi = pr.end < P.H ? pr.end : P.H;
+              if (hi > lo) acc0 += (int64_t)prof_compute(p) * (hi - lo);
+              if (pr.end > b_old) b_until = pr.end;
+              if (hi > pr.start) acc1 += (int64_t)T.mem[m] * (hi - pr.start);
             }
+          } else if (strict) {
+            acc0 += pr.dropped ? nreq : nreq - hits_in(c, bt.pos, nreq, pr.end, T.slo[m]);
+          } else {
+            const int64_t tb = pr.dropped ? (int64_t)0xFFFFFFFFLL : pr.end - (int64_t)c.sa(bt.pos);
+            acc1 = tb > acc1 ? tb : acc1;
           }
+        }
+        if (actual) {
           c.lane_n[g] = n;
           int64_t mx = 0;
+#pragma unroll 1
           for (int i = 0; i < n; ++i) mx = rows.en(i) > mx ? rows.en(i) : mx;
           c.g_maxend[g] = mx;
 #pragma unroll
-          for (int s = 0; s < kMaxSl; ++s) {
-            c.ls[g * kMaxSl + s] = ls[s];
-            c.bu[g * kMaxSl + s] = bu[s];
-          }
-          c.g_busy[g] += busy;
-          c.g_mem[g] += memt;
-        } else {  // candidate geometry j replayed from idle on the same batch list (O8)
-          const int j = P.geom_lo + v - 1;
-          int64_t key = -1;
-          if (P.policy == 0 && c.g_dec[g]) {
-            int n = 0;
-            int64_t ls[kMaxSl];
-#pragma unroll
-            for (int s = 0; s < kMaxSl; ++s) ls[s] = 0;
-            int64_t misses = 0, tail = 0;
-            for (int x = x0; x < x1; ++x) {
-              const Bat& bt = c.bat(c.gl(x));
-              const int m = (bt.info >> 16) & 0xFF;
-              const bool strict = (bt.info >> 24) & 1;
-              const int nreq = bt.info & 0xFFFF;
-              const PlaceRes pr = place_lane(T, j, rows, n, ls, bt.ready, m, strict, P.max_live);
-              if (strict) {
-                misses += pr.dropped ? nreq : nreq - hits_in(c, bt.pos, nreq, pr.end, T.slo[m]);
-              } else {
-                const int64_t tb = pr.dropped ? (int64_t)0xFFFFFFFFLL : pr.end - (int64_t)c.sa(bt.pos);
-                tail = tb > tail ? tb : tail;
-              }
-            }
-            key = make_key(misses, tail, j == c.g_geom[g] ? 0 : j + 1);
-            if (j == c.g_geom[g]) c.g_kcur[g] = key;
-          }
+          for (int s = 0; s < kMaxSl; ++s) c.ls[g * kMaxSl + s] = ls[s];
+          c.g_busy[g] += acc0;
+          c.g_mem[g] += acc1;
+        } else {
+          const int64_t key = make_key(acc0, acc1, j == c.g_geom[g] ? 0 : j + 1);
+          if (j == c.g_geom[g]) c.g_kcur[g] = key;
           c.keys[g * Gc + v - 1] = key;
-          if (P.cand_keys)
-            P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = key;
+          if (P.cand_keys) P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = key;
         }
       }
       __syncthreads();
       // ---------------------------------------------------------------- F: accounting (O7)
+#pragma unroll 1
       for (int rk = warp; rk < nb; rk += NW) {
         const Bat& bt = c.bat(c.ord(rk));
         const int nreq = bt.info & 0xFFFF, m = (bt.info >> 16) & 0xFF;
@@ -575,25 +681,43 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
             P.log[(size_t)r * P.log_cap + row] = rec;
           }
         }
-        if (!bt.drop) {
-          const int64_t slo = T.slo[m];
-          for (int i = lane; i < nreq; i += 32) {
-            const int64_t lat = bt.end - (int64_t)c.sa(bt.pos + i);
-            if (strict) {
-              if (lat <= slo) cnt[1]++; else cnt[2]++;
-              hist_add(c, ghist, lat_bucket(lat));
-            } else {
-              cnt[5]++;
-              hist_add(c, ghist, kNB + lat_bucket(lat));
+        if (!bt.drop) {  // latencies are non-increasing along the sorted members: runs of equal
+          const int64_t slo = T.slo[m];  // buckets become one histogram update
+          const int cls = strict ? 0 : kNB;
+#pragma unroll 1
+          for (int i0 = 0; i0 < nreq; i0 += 32) {
+            const int i = i0 + lane;
+            const bool valid = i < nreq;
+            const int64_t lat = valid ? bt.end - (int64_t)c.sa(bt.pos + i) : 0;
+            const int bk = valid ? lat_bucket(lat) : -1;
+            const int prev = __shfl_up_sync(0xffffffffu, bk, 1);
+            const bool head = valid && (lane == 0 || prev != bk);
+            const unsigned heads = __ballot_sync(0xffffffffu, head);
+            const unsigned vmask = __ballot_sync(0xffffffffu, valid);
+            const unsigned met = __ballot_sync(0xffffffffu, valid && lat <= slo);
+            if (head) {
+              const unsigned after = heads & ~((2u << lane) - 1u);
+              const int stop = after ? __ffs(after) - 1 : 32 - __clz(vmask);
+              hist_add(c, ghist, cls + bk, (uint32_t)(stop - lane));
+            }
+            if (lane == 0) {
+              if (strict) {
+                cnt[1] += __popc(met);
+                cnt[2] += __popc(vmask) - __popc(met);
+              } else {
+                cnt[5] += __popc(vmask);
+              }
             }
           }
         }
       }
       // ---------------------------------------------------------------- G: decisions (O9, O10)
+#pragma unroll 1
       for (int g = tid; g < N; g += NT) {
         uint8_t dec_out = kNoGeom;
         if (P.policy == 0 && c.g_dec[g]) {
           int64_t kb = c.keys[g * Gc];
+#pragma unroll 1
           for (int v = 1; v < Gc; ++v) kb = c.keys[g * Gc + v] < kb ? c.keys[g * Gc + v] : kb;
           const int cur = c.g_geom[g];
           const int tag = (int)(kb & 255);
@@ -616,6 +740,7 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
       if (tid == 0) {
         if (P.policy == 0) {
           int alive = 0, open = 0;
+#pragma unroll 1
           for (int g = 0; g < N; ++g) {
             alive += has_vm(c, g, Tend) ? 1 : 0;
             open += c.g_re[g] > Tend ? 1 : 0;
@@ -626,6 +751,7 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
           while (free_slots > 0) {  // wants by (delta misses desc, gpu asc)
             int pick = -1;
             int64_t pd = 0;
+#pragma unroll 1
             for (int g = 0; g < N; ++g) {
               if (!c.g_want[g]) continue;
               const int64_t d = (c.g_kcur[g] >> 40) - (c.g_kbest[g] >> 40);
@@ -647,14 +773,12 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
     }
 
     // ---------------------------------------------------------------- finalize (O12)
+#pragma unroll 1
     for (int g = tid; g < N; g += NT) bill_switch(c, g, VM_NONE, P.H, P.H);
 #pragma unroll
-    for (int i = 0; i < 10; ++i) {
-      int64_t v = cnt[i];
-#pragma unroll
-      for (int d = 16; d > 0; d >>= 1) v += __shfl_xor_sync(0xffffffffu, v, d);
-      if (lane == 0 && v) atomicAdd(&cs.cnt[i], (unsigned long long)v);
-    }
+    for (int i = 0; i < 10; ++i)
+      if (cnt[i]) atomicAdd(&cs.cnt[i], (unsigned long long)cnt[i]);
+#pragma unroll 1
     for (int w = tid; w < kNB; w += NT) {  // fold the packed smem halves into the HBM histogram
       const uint32_t v = c.hist[w];
       if (v & 0xFFFFu) atomicAdd(&ghist[2 * w], v & 0xFFFFu);
@@ -664,6 +788,7 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
     if (warp < 2) {  // nearest-rank P50 / P99 per class
       const uint32_t* h = ghist + warp * kNB;
       uint64_t n = 0;
+#pragma unroll 1
       for (int b = lane; b < kNB; b += 32) n += h[b];
 #pragma unroll
       for (int d = 16; d > 0; d >>= 1) n += __shfl_xor_sync(0xffffffffu, n, d);
@@ -672,6 +797,7 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
         const uint64_t r50 = (50 * n + 99) / 100, r99 = (99 * n + 99) / 100;
         uint64_t cum = 0;
         int f50 = -1, f99 = -1;
+#pragma unroll 1
         for (int b0 = 0; b0 < kNB && f99 < 0; b0 += 32) {
           uint64_t x = h[b0 + lane];
 #pragma unroll
@@ -695,6 +821,7 @@ __global__ void __launch_bounds__(1024) replay_kernel(ReplayParams P) {
     }
     if (tid == 0) {
       int64_t od = 0, spot = 0, busy = 0, memt = 0;
+#pragma unroll 1
       for (int g = 0; g < N; ++g) {
         od += c.g_od[g];
         spot += c.g_spot[g];

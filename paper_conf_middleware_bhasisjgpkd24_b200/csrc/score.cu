@@ -7,7 +7,7 @@
 namespace pemgpu {
 
 
-__global__ void __launch_bounds__(1024) score_kernel(ScoreParams P) {
+__global__ void __launch_bounds__(256) score_kernel(ScoreParams P) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ int bad;
   const int tid = threadIdx.x, NT = blockDim.x;
