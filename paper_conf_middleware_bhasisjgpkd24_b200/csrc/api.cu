@@ -30,6 +30,8 @@ struct protean_handle {
   int64_t* d_eoff = nullptr;
   size_t eoff_bytes = 0;
   void* d_small = nullptr;  // wmax (8 B) + err (16 B)
+  uint32_t* d_pack = nullptr;  // candidate lane packing for the full geometry range
+  int CW = 0;
   cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};  // prepass / replay kernel bracket
   float t_prepass = 0.f, t_replay = 0.f;
   int last_grid = 0, last_block = 0, last_smem = 0, last_per_sm = 0;
@@ -239,6 +241,31 @@ int protean_load_profiles(const protean_profiles* p, protean_handle** out) {
     }
     w[h->tl.o_gn + j] = (int32_t)gs[j].size();
   }
+  // candidate lane packing: geometries in power-of-two lane groups, largest first, per warp
+  std::vector<uint32_t> pack;
+  {
+    std::vector<std::pair<int, int>> order;  // (Z, j)
+    for (int j = 0; j < h->G; ++j) {
+      int Z = 1;
+      while (Z < (int)gs[j].size()) Z <<= 1;
+      order.push_back({Z, j});
+    }
+    std::stable_sort(order.begin(), order.end(),
+                     [](const std::pair<int, int>& a, const std::pair<int, int>& b) { return a.first > b.first; });
+    int fill = 32;
+    for (const auto& zj : order) {
+      const int Z = zj.first, j = zj.second;
+      if (fill + Z > 32) {
+        pack.insert(pack.end(), 32, 0xFFu);
+        fill = 0;
+      }
+      const size_t w0 = pack.size() - 32;
+      for (int s = 0; s < Z; ++s)
+        pack[w0 + fill + s] = (uint32_t)j | ((uint32_t)s << 8) | ((uint32_t)Z << 16) | ((uint32_t)fill << 24);
+      fill += Z;
+    }
+    h->CW = (int)(pack.size() / 32);
+  }
   cudaError_t e = cudaSetDevice(h->device);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&h->nsm, cudaDevAttrMultiProcessorCount, h->device);
   if (e == cudaSuccess) e = cudaMalloc(&h->d_tab, sizeof(int32_t) * h->words.size());
@@ -246,6 +273,8 @@ int protean_load_profiles(const protean_profiles* p, protean_handle** out) {
     e = cudaMemcpy(h->d_tab, h->words.data(), sizeof(int32_t) * h->words.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMalloc(&h->d_small, 256);
   for (int i = 0; i < 4 && e == cudaSuccess; ++i) e = cudaEventCreate(&h->ev[i]);
+  if (e == cudaSuccess) e = cudaMalloc(&h->d_pack, pack.size() * 4);
+  if (e == cudaSuccess) e = cudaMemcpy(h->d_pack, pack.data(), pack.size() * 4, cudaMemcpyHostToDevice);
   if (e != cudaSuccess) {
     cudaGetLastError();
     protean_free(h);
@@ -262,6 +291,7 @@ void protean_free(protean_handle* h) {
   if (h->d_scratch) cudaFree(h->d_scratch);
   if (h->d_eoff) cudaFree(h->d_eoff);
   if (h->d_small) cudaFree(h->d_small);
+  if (h->d_pack) cudaFree(h->d_pack);
   for (int i = 0; i < 4; ++i)
     if (h->ev[i]) cudaEventDestroy(h->ev[i]);
   delete h;
@@ -362,25 +392,21 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   const int WCAP = (int)std::max<unsigned long long>(wmax, 1);
   if (wmax >= (1ull << 25)) return fail(h, PROTEAN_ERANGE, "epoch window >= 2^25 requests");
 
-  // launch geometry
+  // launch geometry: 8 warps; units = actual-placement warps + candidate warps per GPU
   const int Gc = h->G;
-  const int LPG = (1 + Gc) <= 16 ? 16 : ((1 + Gc + 31) / 32) * 32;  // lanes per simulated GPU
-  const int nl = N * LPG;
-  int block = ((nl + 31) / 32) * 32;
-  block = std::max(128, std::min(256, block));
+  const int block = 256;
   SmemLayout sl;
-  sl.init(h->tl.words, h->M, N, Gc, 0, 0);
+  sl.init(h->tl.words, h->M, N, Gc, h->CW, 0, 0);
   const size_t fixed = sl.total;
-  size_t budget = 72 * 1024;
   int BS = std::min(WCAP, 64);
+  size_t budget = 72 * 1024;
   if (const char* ev = std::getenv("PROTEAN_SMEM_BUDGET_KB")) {  // test knob: force spill paths
     budget = (size_t)std::atoi(ev) * 1024;
     BS = std::min(BS, std::max(1, std::atoi(ev)));
   }
-  budget = std::max<size_t>(budget, fixed + (size_t)BS * (sizeof(Bat) + 8) + 64);
-  size_t rem = budget > fixed + (size_t)BS * (sizeof(Bat) + 8) ? budget - fixed - (size_t)BS * (sizeof(Bat) + 8) : 0;
-  int WS = (int)std::min<size_t>((size_t)WCAP, rem / 4);
-  sl.init(h->tl.words, h->M, N, Gc, BS, WS);
+  const size_t with_bats = fixed + (size_t)BS * (sizeof(Bat) + 8) + 64;
+  const int WS = (with_bats + (size_t)WCAP * 4 <= budget) ? WCAP : 0;  // window all in smem or all in HBM
+  sl.init(h->tl.words, h->M, N, Gc, h->CW, BS, WS);
   if (sl.total > 227 * 1024) return fail(h, PROTEAN_ERANGE, "shared memory layout too large");
   int per_sm = 0;
   CK(h, replay_occupancy(block, sl.total, &per_sm));
@@ -391,6 +417,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   std::memset(&P, 0, sizeof(P));
   P.tab = h->d_tab;
   P.tl = h->tl;
+  P.pack = h->d_pack;
   P.maxT = h->maxT;
   P.arr = c.arrival_us;
   P.meta = c.meta;
@@ -432,15 +459,12 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   P.sl = sl;
   P.WCAP = WCAP;
   size_t o = 0;
-  P.o_lists = o; o += al((size_t)nl * c.max_live * sizeof(protean_resident));
-  P.o_lane_n = o; o += al((size_t)N * 4);
-  P.o_ls = o; o += al((size_t)N * kMaxSl * 8);
-  P.o_bu = o; o += al((size_t)N * kMaxSl * 8);
-  const size_t gb = WCAP > BS ? (size_t)(WCAP - BS) : 0;
-  P.o_gbat = o; o += al(gb * sizeof(Bat));
-  P.o_gord = o; o += al(gb * 4);
-  P.o_gglist = o; o += al(gb * 4);
-  P.o_gsarr = o; o += al((size_t)(WCAP > WS ? WCAP - WS : 0) * 4);
+  P.o_alist = o; o += al((size_t)N * kZA * c.max_live * 20);
+  P.o_clist = o; o += al((size_t)block * c.max_live * 20);
+  P.o_gbat = o; o += al((size_t)WCAP * sizeof(Bat));
+  P.o_gord = o; o += al((size_t)WCAP * 4);
+  P.o_gglist = o; o += al((size_t)WCAP * 4);
+  P.o_gsarr = o; o += al((size_t)(WS >= WCAP ? 0 : WCAP) * 4);
   P.slot_bytes = al(o);
   {
     int rc = ensure(h, &h->d_scratch, &h->scratch_bytes, P.slot_bytes * (size_t)grid);

@@ -2,14 +2,15 @@
 // over its E epochs.  Per epoch (O5):
 //   A  VM events + pending installs (thread per simulated GPU)            O11, O5.3
 //   B  stream partition of the epoch's request window in shared memory   O3
-//   C  batch formation per (model, class) stream, id-order rank sort     O3
+//   C  batch formation, warp per (model, class) stream; id-order ranks   O3
 //   D  round-robin dispatch (closed form when every GPU is available)    Q18
-//   E  placement lanes: lane = (sim-GPU, actual | candidate geometry);   O6 + O8 (Alg 1, Eq 1/2,
-//      candidates replay the GPU-epoch from idle and pack an int64 key    the "Oracle" P:L485)
-//   F  per-request accounting: SLO hits, log-linear histogram (smem)     O7
+//   E  placement units, lane per MIG slice: a lane group = one geometry  O6 + O8 (Alg 1, Eq 1/2,
+//      (actual state, or a candidate replayed from idle); group shuffles  the "Oracle" P:L485)
+//      give BE memory, live count and the min-loc of the slice keys
+//   F  per-request accounting: SLO hits, run-length histogram updates    O7
 //   G  argmin + Alg 2 hysteresis + ~30% cap                              O9, O10
-// The request stream (5 B/request) is read from HBM once, with coalesced loads; everything else
-// lives in shared memory, registers and L1/L2-resident per-CTA scratch.
+// The request stream (5 B/request) is read from HBM once with coalesced loads (a second, L2-hot
+// read scatters it); everything else lives in shared memory, registers and L1-resident scratch.
 #include <cuda_runtime.h>
 #include "replay.cuh"
 
@@ -17,25 +18,42 @@ namespace pemgpu {
 
 namespace {
 
+// Per-lane resident list, interleaved across lanes (entry i of lane l at i*stride + l) so that a
+// warp walking its lists in lock-step issues coalesced loads.  mm = mem | model << 16 | strict << 22.
+struct LaneList {
+  int64_t* st;
+  int64_t* en;
+  uint32_t* mm;
+  int stride;
+  __device__ __forceinline__ int64_t S(int i) const { return st[i * stride]; }
+  __device__ __forceinline__ int64_t E(int i) const { return en[i * stride]; }
+  __device__ __forceinline__ uint32_t M(int i) const { return mm[i * stride]; }
+  __device__ __forceinline__ void put(int i, int64_t s, int64_t e, uint32_t m) const {
+    st[i * stride] = s;
+    en[i * stride] = e;
+    mm[i * stride] = m;
+  }
+};
+
 struct Ctx {
   Tab T;
+  const uint32_t* pack;
   uint32_t* hist;
   int *s_cnt, *s_run, *s_base, *s_tot, *s_skip, *s_pend;
   uint8_t *g_geom, *g_target, *g_ctr, *g_vm, *g_bill, *g_dec, *g_best, *g_want;
   int64_t *g_rs, *g_re, *g_from, *g_until, *g_since, *g_maxend, *g_kbest, *g_kcur, *g_od,
       *g_spot, *g_busy, *g_mem;
   int *g_cnt, *g_off;
+  int* a_n;
+  int64_t *a_ls, *a_bu;
   int64_t* keys;
   Bat *sb, *gb;
-  uint32_t *sord, *gord, *sgl, *ggl, *ssarr, *gsarr;
-  int BS, WS;
-  protean_resident* lists;
-  int* lane_n;
-  int64_t *ls, *bu;  // [N][7]
-  __device__ __forceinline__ Bat& bat(int i) const { return i < BS ? sb[i] : gb[i - BS]; }
-  __device__ __forceinline__ uint32_t& ord(int i) const { return i < BS ? sord[i] : gord[i - BS]; }
-  __device__ __forceinline__ uint32_t& gl(int i) const { return i < BS ? sgl[i] : ggl[i - BS]; }
-  __device__ __forceinline__ uint32_t& sa(int i) const { return i < WS ? ssarr[i] : gsarr[i - WS]; }
+  uint32_t *sord, *gord, *sgl, *ggl, *sarr;
+  int BS;
+  // per-epoch generic views (shared or global memory)
+  Bat* bats;
+  uint32_t *ord, *gl;
+  __device__ __forceinline__ Bat& bat_w(int i) const { return i < BS ? sb[i] : gb[i]; }
 };
 
 struct CtaState {
@@ -61,11 +79,11 @@ __device__ void reset_gpu_state(const Ctx& c, int g, int geom) {
   c.g_geom[g] = (uint8_t)geom;
   c.g_target[g] = kNoGeom;
   c.g_ctr[g] = 0;
-  c.lane_n[g] = 0;
-#pragma unroll
-  for (int s = 0; s < kMaxSl; ++s) {
-    c.ls[g * kMaxSl + s] = 0;
-    c.bu[g * kMaxSl + s] = 0;
+#pragma unroll 1
+  for (int s = 0; s < kZA; ++s) {
+    c.a_n[g * kZA + s] = 0;
+    c.a_ls[g * kZA + s] = 0;
+    c.a_bu[g * kZA + s] = 0;
   }
 }
 
@@ -77,13 +95,13 @@ __device__ __forceinline__ bool available(const Ctx& c, int g, int64_t t) {
 }
 
 // O11: one revocation boundary tau = k * T_rev for node g (draws specified in DESIGN.md §3).
-__device__ void vm_event(const ReplayParams& P, const Ctx& c, uint64_t replica, int g, int64_t k,
-                         int64_t tau) {
+__device__ __forceinline__ void vm_event(const ReplayParams& P, const Ctx& c, uint64_t replica, int g,
+                                      int64_t k, int64_t tau) {
   const uint64_t x = (replica << 32) ^ ((uint64_t)g << 20) ^ ((uint64_t)k << 2);
   const uint64_t d0 = smix(P.seed ^ smix(x ^ 0ull)) >> 11;
   const uint64_t d1 = smix(P.seed ^ smix(x ^ 1ull)) >> 11;
   const bool revoked = d0 < P.thr, spot_ok = d1 >= P.thr;
-  if (P.vm_policy == 1) {
+  if (P.vm_policy == 1) {  // PROTEAN: retry spot, else on-demand; seamless redirect
     if (c.g_vm[g] == VM_SPOT) {
       if (revoked && !spot_ok) {
         c.g_vm[g] = VM_OD;
@@ -95,7 +113,7 @@ __device__ void vm_event(const ReplayParams& P, const Ctx& c, uint64_t replica, 
         bill_switch(c, g, VM_SPOT, tau, P.H);
       }
     }
-  } else if (P.vm_policy == 2) {
+  } else if (P.vm_policy == 2) {  // Spot Only
     if (c.g_vm[g] == VM_SPOT) {
       if (revoked && !spot_ok) {
         c.g_vm[g] = VM_NONE;
@@ -117,8 +135,6 @@ __device__ void vm_event(const ReplayParams& P, const Ctx& c, uint64_t replica, 
   }
 }
 
-__device__ __forceinline__ void install(const Ctx& c, int g) { reset_gpu_state(c, g, c.g_target[g]); }
-
 // Packed u16 smem histogram; a half crossing 2^15 moves 2^15 counts to the HBM histogram
 // (cnt <= 32 per call, so a half never exceeds 0xFFFF before the move).
 __device__ __forceinline__ void hist_add(const Ctx& c, uint32_t* ghist, int idx, uint32_t cnt) {
@@ -130,30 +146,164 @@ __device__ __forceinline__ void hist_add(const Ctx& c, uint32_t* ghist, int idx,
   }
 }
 
-__device__ __forceinline__ int hits_in(const Ctx& c, int pos, int n, int64_t end, int64_t slo) {
+__device__ __forceinline__ int hits_in(const uint32_t* a, int n, int64_t end, int64_t slo) {
   const int64_t need = end - slo;  // c - a <= slo  <=>  a >= c - slo
   int lo = 0, hi = n;
+#pragma unroll 1
   while (lo < hi) {
     const int mid = (lo + hi) >> 1;
-    if ((int64_t)c.sa(pos + mid) >= need) hi = mid; else lo = mid + 1;
+    if ((int64_t)a[mid] >= need) hi = mid; else lo = mid + 1;
   }
   return n - lo;
 }
 
+// Sum / min over the aligned lane group of size Z (1..8) containing this lane.
+__device__ __forceinline__ int group_sum32(int v, int Z) {
+#pragma unroll
+  for (int d = 1; d < 8; d <<= 1) {
+    const int o = __shfl_xor_sync(0xffffffffu, v, d);
+    if (d < Z) v += o;
+  }
+  return v;
+}
+__device__ __forceinline__ int64_t group_sum(int64_t v, int Z) {
+#pragma unroll
+  for (int d = 1; d < 8; d <<= 1) {
+    const int64_t o = __shfl_xor_sync(0xffffffffu, v, d);
+    if (d < Z) v += o;
+  }
+  return v;
+}
+__device__ __forceinline__ uint64_t group_min(uint64_t v, int Z) {
+#pragma unroll
+  for (int d = 1; d < 8; d <<= 1) {
+    const uint64_t o = __shfl_xor_sync(0xffffffffu, v, d);
+    if (d < Z && o < v) v = o;
+  }
+  return v;
+}
+
+// The slice lane's own list: memory wait and Eq 1 co-runner sum by their plain definitions
+// (rare: only when the batch does not fit the slice at t0, or a resident starts after t0).
+__device__ __noinline__ void slice_slow(const LaneList& L, int n, int64_t t0, int32_t q, int32_t Ms,
+                                        const int32_t* fbr_p, int64_t own_f, int64_t* start_out,
+                                        int64_t* F_out) {
+  int64_t used = 0;
+#pragma unroll 1
+  for (int i = 0; i < n; ++i)
+    if (L.E(i) > t0) used += L.M(i) & 0xFFFF;
+  int64_t start = t0;
+  if (used + q > Ms) {
+    start = INT64_MAX;
+  #pragma unroll 1
+  for (int i = 0; i < n; ++i) {
+      const int64_t ei = L.E(i);
+      if (ei <= t0) continue;
+      int64_t rem = 0;
+#pragma unroll 1
+      for (int k = 0; k < n; ++k)
+        if (L.E(k) > ei) rem += L.M(k) & 0xFFFF;
+      if (rem + q <= Ms && ei < start) start = ei;
+    }
+  }
+  int64_t F = own_f;
+#pragma unroll 1
+  for (int i = 0; i < n; ++i)
+    if (L.S(i) <= start && start < L.E(i)) F += fbr_p[((L.M(i) >> 16) & 63) * kNProf];
+  *start_out = start;
+  *F_out = F;
+}
+
+struct SliceOut {
+  uint64_t kmin;     // group min key (~0 = no feasible slice or overflow)
+  bool drop_overflow;
+};
+
+// One Place() (Alg 1) of a batch on one lane group: each lane is one slice position s of
+// geometry j; the lane keeps its own slice's resident list.  Returns the group outcome; this
+// lane's own [start, end) candidate in *my_start / *my_end.
+__device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, int j, int s, int p,
+                                                int Z, const LaneList& L, int& n, int64_t& ls,
+                                                int64_t t, int m, bool strict, int max_live,
+                                                int64_t* my_start, int64_t* my_end) {
+  const int64_t t0 = t > ls ? t : ls;
+  const int32_t* fbr_p = T.fbr + p;  // fbr[model][p] = fbr_p[model * 5]
+  int32_t used = 0, be = 0;
+  int64_t fs = 0;
+  bool fut = false;
+  if (active) {
+    int k = 0;
+#pragma unroll 1
+    for (int i = 0; i < n; ++i) {
+      const int64_t ei = L.E(i);
+      if (ei <= t) continue;  // ended: can never matter again (stable compaction)
+      const int64_t si = L.S(i);
+      const uint32_t mi = L.M(i);
+      if (k != i) L.put(k, si, ei, mi);
+      ++k;
+      if (!((mi >> 22) & 1)) be += mi & 0xFFFF;
+      if (ei > t0) {
+        used += mi & 0xFFFF;
+        fs += fbr_p[((mi >> 16) & 63) * kNProf];
+        fut |= si > t0;
+      }
+    }
+    n = k;
+  }
+  const int live = group_sum32(active ? n : 0, Z);
+  const int be_mem = group_sum32(be, Z);
+  SliceOut o;
+  o.drop_overflow = live >= max_live;
+  uint64_t key = ~0ull;
+  int64_t start = 0, c = 0;
+  const int32_t q = T.mem[m];
+  const int32_t Ms = prof_cap(p);
+  if (active && !o.drop_overflow && q <= Ms) {
+    int64_t F;
+    const int64_t own_f = fbr_p[m * kNProf];
+    if (used + q <= Ms && !fut) {
+      start = t0;
+      F = own_f + fs;
+    } else {
+      slice_slow(L, n, t0, q, Ms, fbr_p, own_f, &start, &F);
+    }
+    c = start + exec_time(T.solo[m * kNProf + p], F);
+    if (strict) {  // choose_strict_slice: tag < 1 (Alg 1 lines 1-8), least eta == least completion
+      const uint64_t inelig = (be_mem >= T.gpref[j * 8 + s]) ? (1ull << 62) : 0ull;
+      key = inelig | ((uint64_t)c << 6) | ((uint64_t)(4 - p) << 3) | (uint64_t)s;
+    } else {       // choose_best_effort_slice: first fit, else earliest start (reading Q12)
+      key = ((uint64_t)start << 3) | (uint64_t)s;
+    }
+  }
+  o.kmin = group_min(key, Z);
+  *my_start = start;
+  *my_end = c;
+  if (o.kmin != ~0ull && key == o.kmin) {  // schedule(batch, chosen_slice)
+    L.put(n, start, c, (uint32_t)q | ((uint32_t)m << 16) | ((uint32_t)(strict ? 1 : 0) << 22));
+    ++n;
+    ls = start;
+  }
+  return o;
+}
+
 }  // namespace
 
-__global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
+__global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ CtaState cs;
   const SmemLayout& SL = P.sl;
   const int tid = threadIdx.x, NT = blockDim.x, lane = tid & 31, warp = tid >> 5, NW = NT >> 5;
-  const int N = P.N, S = SL.S, Gc = SL.Gc;
+  const int N = P.N, S = SL.S, Gc = SL.Gc, CW = SL.CW;
 
   Ctx c;
   int32_t* tabw = reinterpret_cast<int32_t*>(smem + SL.tab);
 #pragma unroll 1
   for (int i = tid; i < P.tl.words; i += NT) tabw[i] = P.tab[i];
+  uint32_t* packs = reinterpret_cast<uint32_t*>(smem + SL.pack);
+#pragma unroll 1
+  for (int i = tid; i < CW * 32; i += NT) packs[i] = P.pack[i];
   c.T.bind(tabw, P.tl);
+  c.pack = packs;
   c.hist = reinterpret_cast<uint32_t*>(smem + SL.hist);
   c.s_cnt = reinterpret_cast<int*>(smem + SL.s_cnt);
   c.s_run = reinterpret_cast<int*>(smem + SL.s_run);
@@ -170,29 +320,39 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
   c.g_od = gi + 8 * N; c.g_spot = gi + 9 * N; c.g_busy = gi + 10 * N; c.g_mem = gi + 11 * N;
   c.g_cnt = reinterpret_cast<int*>(smem + SL.g_i32);
   c.g_off = c.g_cnt + N;
+  c.a_n = reinterpret_cast<int*>(smem + SL.a_n);
+  c.a_ls = reinterpret_cast<int64_t*>(smem + SL.a_ls);
+  c.a_bu = reinterpret_cast<int64_t*>(smem + SL.a_bu);
   c.keys = reinterpret_cast<int64_t*>(smem + SL.keys);
   c.BS = SL.BS;
-  c.WS = SL.WS;
   c.sb = reinterpret_cast<Bat*>(smem + SL.bats);
   c.sord = reinterpret_cast<uint32_t*>(smem + SL.ord);
   c.sgl = reinterpret_cast<uint32_t*>(smem + SL.glist);
-  c.ssarr = reinterpret_cast<uint32_t*>(smem + SL.sarr);
   char* slot = P.scratch + (size_t)blockIdx.x * P.slot_bytes;
-  c.lists = reinterpret_cast<protean_resident*>(slot + P.o_lists);
-  c.lane_n = reinterpret_cast<int*>(slot + P.o_lane_n);
-  c.ls = reinterpret_cast<int64_t*>(slot + P.o_ls);
-  c.bu = reinterpret_cast<int64_t*>(slot + P.o_bu);
   c.gb = reinterpret_cast<Bat*>(slot + P.o_gbat);
   c.gord = reinterpret_cast<uint32_t*>(slot + P.o_gord);
   c.ggl = reinterpret_cast<uint32_t*>(slot + P.o_gglist);
-  c.gsarr = reinterpret_cast<uint32_t*>(slot + P.o_gsarr);
+  c.sarr = SL.WS >= P.WCAP ? reinterpret_cast<uint32_t*>(smem + SL.sarr)
+                           : reinterpret_cast<uint32_t*>(slot + P.o_gsarr);
+  // resident lists: actual lanes [N*8 lanes][max_live], candidate lanes [NT lanes][max_live]
+  const int NA = N * kZA;
+  LaneList AL;
+  AL.stride = NA;
+  AL.st = reinterpret_cast<int64_t*>(slot + P.o_alist);
+  AL.en = AL.st + (size_t)NA * P.max_live;
+  AL.mm = reinterpret_cast<uint32_t*>(AL.en + (size_t)NA * P.max_live);
+  LaneList CL;
+  CL.stride = NT;
+  CL.st = reinterpret_cast<int64_t*>(slot + P.o_clist) + tid;
+  CL.en = CL.st + (size_t)NT * P.max_live;
+  CL.mm = reinterpret_cast<uint32_t*>(reinterpret_cast<int64_t*>(slot + P.o_clist) + 2 * (size_t)NT * P.max_live) + tid;
   const Tab& T = c.T;
-  int sum_slots = 0;  // sum of slice counts over the candidate range (slot-evals per batch)
   __syncthreads();
+  int sum_slots = 0;  // slot-evals per batch per decidable GPU
 #pragma unroll 1
   for (int j = P.geom_lo; j < P.geom_hi; ++j) sum_slots += T.gn[j];
-  const int LPG = (1 + Gc) <= 16 ? 16 : ((1 + Gc + 31) / 32) * 32;  // lanes per simulated GPU
-  const int nlp = N * LPG;
+  const int n_aunits = (N + 3) / 4;  // actual-placement warp units: 4 GPUs x 8 slice lanes
+  const uint32_t* sarr = c.sarr;
 
 #pragma unroll 1
   for (int r = blockIdx.x; r < P.R; r += gridDim.x) {
@@ -244,11 +404,11 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
           for (int64_t k = (eW + P.rev - 1) / P.rev; k * P.rev < Tend; ++k) {
             const int64_t tau = k * P.rev;
             if (k < 1 || tau >= P.H) continue;
-            if (c.g_target[g] != kNoGeom && c.g_re[g] <= tau) install(c, g);
+            if (c.g_target[g] != kNoGeom && c.g_re[g] <= tau) reset_gpu_state(c, g, c.g_target[g]);
             vm_event(P, c, replica, g, k, tau);
           }
         }
-        if (c.g_target[g] != kNoGeom && c.g_re[g] <= Tend) install(c, g);
+        if (c.g_target[g] != kNoGeom && c.g_re[g] <= Tend) reset_gpu_state(c, g, c.g_target[g]);
         c.g_dec[g] = (has_vm(c, g, Tend) && c.g_re[g] <= Tend) ? 1 : 0;
         c.g_want[g] = 0;
         c.g_best[g] = kNoGeom;
@@ -269,31 +429,30 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
                            !(c.g_rs[g] < Tend && c.g_re[g] > eW);
         if (!whole) cs.all_avail = 0;
       }
-      const int64_t len = w_end - w_lo;
-      const bool bad_window = len < 0 || len > P.WCAP || w_beg < w_lo;
-      if (bad_window) {
-        if (tid == 0) atomicOr(P.err, 1);
-      }
+      const int64_t len64 = w_end - w_lo;
+      const bool bad_window = len64 < 0 || len64 > P.WCAP || w_beg < w_lo;
+      if (bad_window && tid == 0) atomicOr(P.err, 1);
+      const int len = bad_window ? 0 : (int)len64;
+      const uint32_t* warr = P.arr + w_lo;
+      const uint8_t* wmeta = P.meta + w_lo;
+      const int nbeg = (int)(w_beg - w_lo);  // window offset of the first new request
       // ---------------------------------------------------------------- B: stream partition
-      if (!bad_window && warp < kNSeg) {  // count per (segment, stream); 4 loads in flight per lane
-        const int64_t a = w_lo + len * warp / kNSeg, b = w_lo + len * (warp + 1) / kNSeg;
+      if (warp < kNSeg) {  // count per (segment, stream): warp-aggregated by match_any
+        const int a = (int)((int64_t)len * warp / kNSeg), b = (int)((int64_t)len * (warp + 1) / kNSeg);
         int* cntw = c.s_cnt + warp * S;
 #pragma unroll 1
-        for (int64_t i0 = a; i0 < b; i0 += 128) {
+        for (int i0 = a; i0 < b; i0 += 128) {
           uint8_t mt[4];
 #pragma unroll
           for (int u = 0; u < 4; ++u) {
-            const int64_t i = i0 + u * 32 + lane;
-            mt[u] = i < b ? P.meta[i] : (uint8_t)0xFF;
+            const int i = i0 + u * 32 + lane;
+            mt[u] = i < b ? wmeta[i] : (uint8_t)0xFF;
           }
 #pragma unroll
           for (int u = 0; u < 4; ++u) {
-            const bool valid = i0 + u * 32 + lane < b;
-            int m = mt[u] & 63;
-            if (m >= T.M) m = 0;
-            const int key = valid ? 2 * m + ((mt[u] >> 7) ? 0 : 1) : 1024 + lane;
+            const int key = mt[u] == 0xFF ? 1024 + lane : 2 * ((mt[u] & 63) < T.M ? (mt[u] & 63) : 0) + ((mt[u] >> 7) ? 0 : 1);
             const unsigned peers = __match_any_sync(0xffffffffu, key);
-            if (valid && (peers & ((1u << lane) - 1u)) == 0) cntw[key] += __popc(peers);
+            if (key < 1024 && (peers & ((1u << lane) - 1u)) == 0) cntw[key] += __popc(peers);
           }
         }
       }
@@ -305,7 +464,7 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
           const int k = k0 + lane;
           int tot = 0;
           if (k < S) {
-#pragma unroll 1
+#pragma unroll
             for (int w = 0; w < kNSeg; ++w) {
               const int cv = c.s_cnt[w * S + k];
               c.s_run[w * S + k] = tot;
@@ -322,41 +481,44 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
           if (k < S) {
             c.s_base[k] = base;
             c.s_tot[k] = tot;
-#pragma unroll 1
+#pragma unroll
             for (int w = 0; w < kNSeg; ++w) c.s_run[w * S + k] += base;
           }
           carry += __shfl_sync(0xffffffffu, x, 31);
         }
       }
       __syncthreads();
-      if (!bad_window && warp < kNSeg) {  // stable scatter into stream-sorted order + validation
-        const int64_t a = w_lo + len * warp / kNSeg, b = w_lo + len * (warp + 1) / kNSeg;
+      if (warp < kNSeg) {  // stable scatter into stream-sorted order + validation of new requests
+        const int a = (int)((int64_t)len * warp / kNSeg), b = (int)((int64_t)len * (warp + 1) / kNSeg);
         int* runw = c.s_run + warp * S;
+        uint32_t* sa = c.sarr;
+        uint32_t prev_last = (a > 0) ? warr[a - 1] : (w_lo > r_lo ? P.arr[w_lo - 1] : 0u);
 #pragma unroll 1
-        for (int64_t i0 = a; i0 < b; i0 += 128) {
+        for (int i0 = a; i0 < b; i0 += 128) {
           uint8_t mt[4];
-          uint32_t ai[4], ap[4];
+          uint32_t ai[4];
 #pragma unroll
           for (int u = 0; u < 4; ++u) {
-            const int64_t i = i0 + u * 32 + lane;
+            const int i = i0 + u * 32 + lane;
             const bool valid = i < b;
-            mt[u] = valid ? P.meta[i] : (uint8_t)0;
-            ai[u] = valid ? P.arr[i] : 0u;
-            ap[u] = (valid && i >= w_beg && i > r_lo) ? P.arr[i - 1] : 0u;
+            mt[u] = valid ? wmeta[i] : (uint8_t)0xFF;
+            ai[u] = valid ? warr[i] : 0xFFFFFFFFu;
           }
 #pragma unroll
           for (int u = 0; u < 4; ++u) {
-            const int64_t i = i0 + u * 32 + lane;
+            const int i = i0 + u * 32 + lane;
             const bool valid = i < b;
-            int m = mt[u] & 63;
-            if (valid && i >= w_beg &&  // validate each request once (when it is new)
-                ((mt[u] & 0x40) || m >= T.M || (int64_t)ai[u] >= P.trace_len || ai[u] < ap[u]))
+            uint32_t ap = __shfl_up_sync(0xffffffffu, ai[u], 1);
+            if (lane == 0) ap = prev_last;
+            prev_last = __shfl_sync(0xffffffffu, ai[u], 31);
+            const int m = mt[u] & 63;
+            if (valid && i >= nbeg &&  // validate each request once (when it is new)
+                ((mt[u] & 0x40) || m >= T.M || (int64_t)ai[u] >= P.trace_len || ai[u] < ap))
               atomicOr(P.err, 1);
-            if (m >= T.M) m = 0;
-            const int key = valid ? 2 * m + ((mt[u] >> 7) ? 0 : 1) : 1024 + lane;
+            const int key = valid ? 2 * (m < T.M ? m : 0) + ((mt[u] >> 7) ? 0 : 1) : 1024 + lane;
             const unsigned peers = __match_any_sync(0xffffffffu, key);
             const unsigned rank = __popc(peers & ((1u << lane) - 1u));
-            if (valid) c.sa(runw[key] + (int)rank) = ai[u];
+            if (valid) sa[runw[key] + (int)rank] = ai[u];
             __syncwarp();
             if (valid && rank == 0) runw[key] += __popc(peers);
             __syncwarp();
@@ -378,10 +540,11 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
         const int end = c.s_base[k] + c.s_tot[k];
         int pend = 0;
         uint32_t a0p = 0xFFFFFFFFu;
+#pragma unroll 1
         while (i < end) {
           const int64_t st = (int64_t)i + (int64_t)lane * B;
           bool full = false;
-          if (st + B <= end) full = (int64_t)c.sa((int)(st + B - 1)) <= (int64_t)c.sa((int)st) + Tm;
+          if (st + B <= end) full = (int64_t)sarr[st + B - 1] <= (int64_t)sarr[st] + Tm;
           const unsigned fm = __ballot_sync(0xffffffffu, full);
           const int nfull = __ffs(~fm) ? __ffs(~fm) - 1 : 32;
           int slot0 = 0;
@@ -389,8 +552,8 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
           slot0 = __shfl_sync(0xffffffffu, slot0, 0);
           if (lane < nfull) {
             const int ii = (int)st;
-            const uint32_t ready = c.sa(ii + B - 1);
-            Bat& bt = c.bat(slot0 + lane);
+            const uint32_t ready = sarr[ii + B - 1];
+            Bat& bt = c.bat_w(slot0 + lane);
             bt.key = ((uint64_t)ready << 32) | ((uint64_t)(strict ? 0 : 1) << 31) |
                      ((uint64_t)m << 25) | (uint64_t)(ii & 0x1FFFFFF);
             bt.ready = ready;
@@ -404,26 +567,26 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
           i += nfull * B;
           if (nfull == 32) continue;
           if (i >= end) break;
-          // batch starting at i is not full within this window: lane 0 resolves it
           int j = 0, state = 0;  // state 0 emit, 1 pending
-          int64_t ready = 0;
           if (lane == 0) {
-            const int64_t a0 = c.sa(i);
+            const int64_t a0 = sarr[i];
             const int64_t deadline = a0 + Tm;
             const int lim = (end - i > B) ? i + B : end;
             int lo = i + 1, hi = lim;  // first member beyond the timeout, else lim
+#pragma unroll 1
             while (lo < hi) {
               const int mid = (lo + hi) >> 1;
-              if ((int64_t)c.sa(mid) > deadline) hi = mid; else lo = mid + 1;
+              if ((int64_t)sarr[mid] > deadline) hi = mid; else lo = mid + 1;
             }
             j = lo;
-            if (j - i == B) ready = c.sa(j - 1);        // full (only possible at the window end)
+            int64_t ready = 0;
+            if (j - i == B) ready = sarr[j - 1];        // full (only at the window end)
             else if (j < end) ready = deadline;         // a later arrival missed the timeout
             else if (deadline < Tend) ready = deadline; // timed out inside this epoch
             else { state = 1; pend = end - i; a0p = (uint32_t)a0; }
             if (state == 0) {
               const int slot = atomicAdd(&cs.nb, 1);
-              Bat& bt = c.bat(slot);
+              Bat& bt = c.bat_w(slot);
               bt.key = ((uint64_t)ready << 32) | ((uint64_t)(strict ? 0 : 1) << 31) |
                        ((uint64_t)m << 25) | (uint64_t)(i & 0x1FFFFFF);
               bt.ready = (uint32_t)ready;
@@ -448,27 +611,42 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
       __syncthreads();
       const int nb = cs.nb;
       const unsigned amin = cs.amin;
+      if (nb > c.BS) {  // rare: more batches than the smem arrays hold -> all in global scratch
+#pragma unroll 1
+        for (int b = tid; b < c.BS; b += NT) c.gb[b] = c.sb[b];
+        c.bats = c.gb;
+        c.ord = c.gord;
+        c.gl = c.ggl;
+      } else {
+        c.bats = c.sb;
+        c.ord = c.sord;
+        c.gl = c.sgl;
+      }
+      __syncthreads();
       // next window: stream entries at/after the earliest open batch's first arrival are re-read
 #pragma unroll 1
       for (int k = tid; k < S; k += NT) {
         if (bad_window) break;
         const int b0 = c.s_base[k], tot = c.s_tot[k];
         int lo = 0, hi = tot;
+#pragma unroll 1
         while (lo < hi) {
           const int mid = (lo + hi) >> 1;
-          if (c.sa(b0 + mid) >= amin) hi = mid; else lo = mid + 1;
+          if (sarr[b0 + mid] >= amin) hi = mid; else lo = mid + 1;
         }
-        const int ge = tot - lo;
         if (lo) atomicAdd(reinterpret_cast<unsigned long long*>(&cs.lt_total), (unsigned long long)lo);
-        c.s_skip[k] = ge - c.s_pend[k];
+        c.s_skip[k] = tot - lo - c.s_pend[k];
       }
+      Bat* bats = c.bats;
+      uint32_t* ord = c.ord;
+      uint32_t* gl = c.gl;
 #pragma unroll 1
       for (int b = tid; b < nb; b += NT) {  // id order (O3): rank by key
-        const uint64_t kb = c.bat(b).key;
+        const uint64_t kb = bats[b].key;
         int rank = 0;
-#pragma unroll 1
-        for (int x = 0; x < nb; ++x) rank += (c.bat(x).key < kb) ? 1 : 0;
-        c.ord(rank) = (uint32_t)b;
+#pragma unroll 4
+        for (int x = 0; x < nb; ++x) rank += (bats[x].key < kb) ? 1 : 0;
+        ord[rank] = (uint32_t)b;
       }
       __syncthreads();
       if (tid == 0) cs.w_lo = bad_window ? w_end : w_lo + cs.lt_total;
@@ -476,13 +654,12 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
       if (cs.all_avail) {
         const int cursor = cs.cursor;
 #pragma unroll 1
-        for (int rk = tid; rk < nb; rk += NT) c.bat(c.ord(rk)).gpu = (uint8_t)((cursor + rk) % N);
+        for (int rk = tid; rk < nb; rk += NT) bats[ord[rk]].gpu = (uint8_t)((cursor + rk) % N);
 #pragma unroll 1
         for (int g = tid; g < N; g += NT) {
           const int d = (g - cursor % N + N) % N;
           const int cntg = d < nb ? (nb - d + N - 1) / N : 0;
           c.g_cnt[g] = cntg;
-          // offset = sum of counts of GPUs before g
           int off = 0;
 #pragma unroll 1
           for (int h = 0; h < g; ++h) {
@@ -496,7 +673,7 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
 #pragma unroll 1
         for (int rk = tid; rk < nb; rk += NT) {
           const int g = (cursor + rk) % N;
-          c.gl(c.g_off[g] + rk / N) = c.ord(rk);
+          gl[c.g_off[g] + rk / N] = ord[rk];
         }
         if (tid == 0) cs.cursor = (int)((cursor + nb) % N);
       } else if (N <= 32) {
@@ -506,7 +683,7 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
           int cur = cs.cursor, mycnt = 0;
 #pragma unroll 1
           for (int rk = 0; rk < nb; ++rk) {
-            Bat& bt = c.bat(c.ord(rk));
+            Bat& bt = bats[ord[rk]];
             const int64_t t = bt.ready;
             const bool av = lane < N && fr <= t && t < un && !(rs <= t && t < re);
             const unsigned am = __ballot_sync(0xffffffffu, av);
@@ -534,118 +711,180 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
           int fill = 0;
 #pragma unroll 1
           for (int rk = 0; rk < nb; ++rk) {
-            const uint32_t b = c.ord(rk);
-            const int g = c.bat(b).gpu;
-            if (lane == g) c.gl(c.g_off[lane] + fill++) = b;
+            const uint32_t b = ord[rk];
+            const int g = bats[b].gpu;
+            if (lane == g) gl[c.g_off[lane] + fill++] = b;
           }
           if (lane == 0) cs.cursor = cur;
         }
-      } else {
-        if (tid == 0) {
-          int cur = cs.cursor;
+      } else if (tid == 0) {
+        int cur = cs.cursor;
 #pragma unroll 1
-          for (int g = 0; g < N; ++g) c.g_cnt[g] = 0;
+        for (int g = 0; g < N; ++g) c.g_cnt[g] = 0;
 #pragma unroll 1
-          for (int rk = 0; rk < nb; ++rk) {
-            Bat& bt = c.bat(c.ord(rk));
-            int chosen = -1;
+        for (int rk = 0; rk < nb; ++rk) {
+          Bat& bt = bats[ord[rk]];
+          int chosen = -1;
 #pragma unroll 1
-            for (int i = 0; i < N; ++i) {
-              const int g = (cur + i) % N;
-              if (available(c, g, bt.ready)) { chosen = g; break; }
-            }
-            if (chosen < 0) {
-              bt.drop = 1;
-              bt.gpu = 0xFF;
-            } else {
-              bt.gpu = (uint8_t)chosen;
-              c.g_cnt[chosen]++;
-              cur = (chosen + 1) % N;
-            }
+          for (int i = 0; i < N; ++i) {
+            const int g = (cur + i) % N;
+            if (available(c, g, bt.ready)) { chosen = g; break; }
           }
-          int off = 0;
-#pragma unroll 1
-          for (int g = 0; g < N; ++g) {
-            c.g_off[g] = off;
-            off += c.g_cnt[g];
-            c.g_cnt[g] = 0;
+          if (chosen < 0) {
+            bt.drop = 1;
+            bt.gpu = 0xFF;
+          } else {
+            bt.gpu = (uint8_t)chosen;
+            c.g_cnt[chosen]++;
+            cur = (chosen + 1) % N;
           }
-          c.g_off[N] = off;
-#pragma unroll 1
-          for (int rk = 0; rk < nb; ++rk) {
-            const uint32_t b = c.ord(rk);
-            const Bat& bt = c.bat(b);
-            if (bt.drop) continue;
-            c.gl(c.g_off[bt.gpu] + c.g_cnt[bt.gpu]++) = b;
-          }
-          cs.cursor = cur;
         }
+        int off = 0;
+#pragma unroll 1
+        for (int g = 0; g < N; ++g) {
+          c.g_off[g] = off;
+          off += c.g_cnt[g];
+          c.g_cnt[g] = 0;
+        }
+        c.g_off[N] = off;
+#pragma unroll 1
+        for (int rk = 0; rk < nb; ++rk) {
+          const uint32_t b = ord[rk];
+          const Bat& bt = bats[b];
+          if (bt.drop) continue;
+          gl[c.g_off[bt.gpu] + c.g_cnt[bt.gpu]++] = b;
+        }
+        cs.cursor = cur;
       }
       __syncthreads();
-      // ---------------------------------------------------------------- E: placement lanes
-      // lane = (GPU g, v): v = 0 the actual placement on the current geometry (carried state),
-      // v = 1..Gc candidate geometry v-1 replayed from idle on the same batch list (O8).
+      // ---------------------------------------------------------------- E: placement units
+      // unit < n_aunits: actual placement of GPUs 4u..4u+3 (8 slice lanes each, carried state);
+      // otherwise candidate warp w of GPU g: lane groups = candidate geometries from idle (O8).
+      // One loop body serves both kinds (a single inlined copy of Place).
+      const int n_units = n_aunits + (P.policy == 0 ? N * CW : 0);
 #pragma unroll 1
-      for (int L = tid; L < nlp; L += NT) {
-        const int g = L / LPG, v = L - g * LPG;
-        if (g >= N || v > Gc) continue;
-        const bool actual = v == 0;
-        const int j = actual ? (int)c.g_geom[g] : P.geom_lo + v - 1;
-        if (!actual && !(P.policy == 0 && c.g_dec[g])) {
-          c.keys[g * Gc + v - 1] = -1;
-          if (P.cand_keys) P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = -1;
-          continue;
+      for (int u = warp; u < n_units; u += NW) {
+        const bool actual = u < n_aunits;
+        int g, s, Z, gbase, j;
+        bool valid;
+        if (actual) {
+          g = u * 4 + (lane >> 3);
+          s = lane & 7;
+          Z = kZA;
+          gbase = lane & ~7;
+          valid = g < N;
+          j = valid ? c.g_geom[g] : 0;
+        } else {
+          const int cu = u - n_aunits, w = cu % CW;
+          g = cu / CW;
+          const uint32_t pk = c.pack[w * 32 + lane];
+          const int jr = pk & 0xFF;
+          s = (pk >> 8) & 0xFF;
+          Z = (pk >> 16) & 0xFF;
+          gbase = pk >> 24;
+          valid = jr != 0xFF;
+          j = valid ? jr : 0;
+          if (!c.g_dec[g]) {  // undecidable at T: no candidates scored (O5.4)
+            if (valid && lane == gbase) {
+              c.keys[g * Gc + (j - P.geom_lo)] = -1;
+              if (P.cand_keys) P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = -1;
+            }
+            continue;  // warp-uniform: the whole unit belongs to g
+          }
         }
-        const int x0 = c.g_off[g], x1 = c.g_off[g + 1];
-        Rows rows{c.lists + (size_t)L * P.max_live};
-        int n = actual ? c.lane_n[g] : 0;
-        int64_t ls[kMaxSl];
+        const bool active = valid && s < T.gn[j];
+        const int p = active ? T.gprof[j * 8 + s] : 0;
+        const int al = actual && valid ? g * kZA + s : 0;  // actual lane id
+        LaneList L;
+        if (actual) {
+          L = AL;
+          L.st += al; L.en += al; L.mm += al;
+        } else {
+          L = CL;
+        }
+        int n = actual && valid ? c.a_n[al] : 0;
+        int64_t ls = actual && valid ? c.a_ls[al] : 0;
+        int64_t bu = actual && valid ? c.a_bu[al] : 0;
+        const int x0 = valid ? c.g_off[g] : 0, x1 = valid ? c.g_off[g + 1] : 0;
+        int len_max = x1 - x0;
 #pragma unroll
-        for (int s = 0; s < kMaxSl; ++s) ls[s] = actual ? c.ls[g * kMaxSl + s] : 0;
-        int64_t acc0 = 0, acc1 = 0;  // actual: busy, mem-time;  candidate: misses, BE tail
+        for (int d = 1; d < 32; d <<= 1) {
+          const int o = __shfl_xor_sync(0xffffffffu, len_max, d);
+          len_max = o > len_max ? o : len_max;
+        }
+        int64_t acc0 = 0, acc1 = 0;  // actual: busy, mem-time; candidate: misses, BE tail
 #pragma unroll 1
-        for (int x = x0; x < x1; ++x) {
-          Bat& bt = c.bat(c.gl(x));
-          const uint32_t info = bt.info;
+        for (int xi = 0; xi < len_max; ++xi) {
+          const bool has = xi < x1 - x0;
+          Bat* bt = &bats[has ? gl[x0 + xi] : 0];
+          const uint32_t info = has ? bt->info : 0u;
           const int m = (info >> 16) & 0xFF, nreq = info & 0xFFFF;
           const bool strict = (info >> 24) & 1;
-          const PlaceRes pr = place_lane(T, j, rows, n, ls, bt.ready, m, strict, P.max_live);
+          const int64_t t = has ? (int64_t)bt->ready : 0;
+          int64_t st, en;
+          const SliceOut so = place_group(T, active && has, j, s, p, Z, L, n, ls, t, m, strict,
+                                          P.max_live, &st, &en);
+          const bool placed = !so.drop_overflow && so.kmin != ~0ull;
+          const int wl = (gbase + (int)(so.kmin & 7)) & 31;
+          const int64_t cwin = __shfl_sync(0xffffffffu, en, wl);
+          if (!has) continue;
           if (actual) {
-            bt.drop = (uint8_t)pr.dropped;
-            bt.slice = pr.dropped ? 0xFF : (uint8_t)pr.slice;
-            bt.start = pr.dropped ? 0 : pr.start;
-            bt.end = pr.dropped ? 0 : pr.end;
-            if (!pr.dropped) {  // busy union + memory-time, clipped to [0, H) (reading Q29)
-              int64_t& b_until = c.bu[g * kMaxSl + pr.slice];
-              const int64_t b_old = b_until;
-              const int p = T.gprof[j * 8 + pr.slice];
-              const int64_t lo = pr.start > b_old ? pr.start : b_old;
-              const int64_t hi = pr.end < P.H ? pr.end : P.H;
+            if (placed && lane == wl) {  // winner: busy union + memory-time, clipped to [0, H)
+              const int64_t lo = st > bu ? st : bu;
+              const int64_t hi = en < P.H ? en : P.H;
               if (hi > lo) acc0 += (int64_t)prof_compute(p) * (hi - lo);
-              if (pr.end > b_old) b_until = pr.end;
-              if (hi > pr.start) acc1 += (int64_t)T.mem[m] * (hi - pr.start);
+              if (en > bu) bu = en;
+              if (hi > st) acc1 += (int64_t)T.mem[m] * (hi - st);
+              bt->slice = (uint8_t)s;
+              bt->start = st;
+              bt->end = en;
+              bt->drop = 0;
             }
-          } else if (strict) {
-            acc0 += pr.dropped ? nreq : nreq - hits_in(c, bt.pos, nreq, pr.end, T.slo[m]);
-          } else {
-            const int64_t tb = pr.dropped ? (int64_t)0xFFFFFFFFLL : pr.end - (int64_t)c.sa(bt.pos);
-            acc1 = tb > acc1 ? tb : acc1;
+            if (!placed && lane == gbase) {
+              bt->drop = so.drop_overflow ? 3 : 2;
+              bt->slice = 0xFF;
+              bt->start = bt->end = 0;
+            }
+          } else if (lane == gbase && valid) {  // group leader keeps the candidate's score
+            if (strict) {
+              if (!placed) {
+                acc0 += nreq;
+              } else {  // latencies fall along the sorted members: test the ends first
+                const uint32_t* ma = sarr + bt->pos;
+                const int64_t slo = T.slo[m];
+                if (cwin - (int64_t)ma[0] > slo)
+                  acc0 += (cwin - (int64_t)ma[nreq - 1] > slo) ? nreq : nreq - hits_in(ma, nreq, cwin, slo);
+              }
+            } else {
+              const int64_t tb = placed ? cwin - (int64_t)sarr[bt->pos] : (int64_t)0xFFFFFFFFLL;
+              acc1 = tb > acc1 ? tb : acc1;
+            }
           }
         }
         if (actual) {
-          c.lane_n[g] = n;
           int64_t mx = 0;
+          if (valid) {
+            c.a_n[al] = n;
+            c.a_ls[al] = ls;
+            c.a_bu[al] = bu;
 #pragma unroll 1
-          for (int i = 0; i < n; ++i) mx = rows.en(i) > mx ? rows.en(i) : mx;
-          c.g_maxend[g] = mx;
+            for (int i = 0; i < n; ++i) mx = L.E(i) > mx ? L.E(i) : mx;
+          }
 #pragma unroll
-          for (int s = 0; s < kMaxSl; ++s) c.ls[g * kMaxSl + s] = ls[s];
-          c.g_busy[g] += acc0;
-          c.g_mem[g] += acc1;
-        } else {
+          for (int d = 1; d < 8; d <<= 1) {
+            const int64_t o = __shfl_xor_sync(0xffffffffu, mx, d);
+            mx = o > mx ? o : mx;
+          }
+          const int64_t bsum = group_sum(acc0, 8), msum = group_sum(acc1, 8);
+          if (valid && s == 0) {
+            c.g_maxend[g] = mx;
+            c.g_busy[g] += bsum;
+            c.g_mem[g] += msum;
+          }
+        } else if (valid && lane == gbase) {
           const int64_t key = make_key(acc0, acc1, j == c.g_geom[g] ? 0 : j + 1);
           if (j == c.g_geom[g]) c.g_kcur[g] = key;
-          c.keys[g * Gc + v - 1] = key;
+          c.keys[g * Gc + (j - P.geom_lo)] = key;
           if (P.cand_keys) P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = key;
         }
       }
@@ -653,7 +892,7 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
       // ---------------------------------------------------------------- F: accounting (O7)
 #pragma unroll 1
       for (int rk = warp; rk < nb; rk += NW) {
-        const Bat& bt = c.bat(c.ord(rk));
+        const Bat& bt = bats[ord[rk]];
         const int nreq = bt.info & 0xFFFF, m = (bt.info >> 16) & 0xFF;
         const bool strict = (bt.info >> 24) & 1;
         if (lane == 0) {
@@ -684,11 +923,13 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
         if (!bt.drop) {  // latencies are non-increasing along the sorted members: runs of equal
           const int64_t slo = T.slo[m];  // buckets become one histogram update
           const int cls = strict ? 0 : kNB;
+          const uint32_t* ma = sarr + bt.pos;
+          const int64_t bend = bt.end;
 #pragma unroll 1
           for (int i0 = 0; i0 < nreq; i0 += 32) {
             const int i = i0 + lane;
             const bool valid = i < nreq;
-            const int64_t lat = valid ? bt.end - (int64_t)c.sa(bt.pos + i) : 0;
+            const int64_t lat = valid ? bend - (int64_t)ma[i] : 0;
             const int bk = valid ? lat_bucket(lat) : -1;
             const int prev = __shfl_up_sync(0xffffffffu, bk, 1);
             const bool head = valid && (lane == 0 || prev != bk);
@@ -735,6 +976,11 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
           cnt[9] += Gc;
         }
         if (P.decisions) P.decisions[((size_t)r * P.E + e) * N + g] = dec_out;
+        if (P.policy != 0 && P.cand_keys) {
+#pragma unroll 1
+          for (int j = P.geom_lo; j < P.geom_hi; ++j)
+            P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = -1;
+        }
       }
       __syncthreads();
       if (tid == 0) {
@@ -748,6 +994,7 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
           int cap = P.cap_pct * alive / 100;
           if (cap < 1) cap = 1;
           int free_slots = cap - open;
+#pragma unroll 1
           while (free_slots > 0) {  // wants by (delta misses desc, gpu asc)
             int pick = -1;
             int64_t pd = 0;
@@ -787,22 +1034,22 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
     __syncthreads();
     if (warp < 2) {  // nearest-rank P50 / P99 per class
       const uint32_t* h = ghist + warp * kNB;
-      uint64_t n = 0;
+      uint32_t n = 0;  // requests per class per replica < 2^32
 #pragma unroll 1
       for (int b = lane; b < kNB; b += 32) n += h[b];
 #pragma unroll
       for (int d = 16; d > 0; d >>= 1) n += __shfl_xor_sync(0xffffffffu, n, d);
       int64_t p50 = 0, p99 = 0;
       if (n) {
-        const uint64_t r50 = (50 * n + 99) / 100, r99 = (99 * n + 99) / 100;
+        const uint64_t r50 = (50 * (uint64_t)n + 99) / 100, r99 = (99 * (uint64_t)n + 99) / 100;
         uint64_t cum = 0;
         int f50 = -1, f99 = -1;
 #pragma unroll 1
         for (int b0 = 0; b0 < kNB && f99 < 0; b0 += 32) {
-          uint64_t x = h[b0 + lane];
+          uint32_t x = h[b0 + lane];
 #pragma unroll
           for (int d = 1; d < 32; d <<= 1) {
-            const uint64_t y = __shfl_up_sync(0xffffffffu, x, d);
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, d);
             if (lane >= d) x += y;
           }
           const unsigned m50 = __ballot_sync(0xffffffffu, cum + x >= r50);
@@ -828,6 +1075,7 @@ __global__ void __launch_bounds__(256, 2) replay_kernel(ReplayParams P) {
         busy += c.g_busy[g];
         memt += c.g_mem[g];
       }
+#pragma unroll 1
       for (int i = 0; i < 10; ++i) P.counters[(size_t)r * 10 + i] = (int64_t)cs.cnt[i];
       P.accum[(size_t)r * 4 + 0] = busy;
       P.accum[(size_t)r * 4 + 1] = memt;

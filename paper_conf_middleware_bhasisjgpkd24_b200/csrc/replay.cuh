@@ -8,6 +8,7 @@
 namespace pemgpu {
 
 constexpr int kNSeg = 4;          // warps that stream-partition the request window
+constexpr int kZA = 8;            // lanes per actual-placement group (one per slice position)
 constexpr int64_t kForever = INT64_MAX;
 
 // One batch of the current epoch (40 B).  info = n | model << 16 | strict << 24.
@@ -18,18 +19,23 @@ struct Bat {
   int64_t start, end;
 };
 
+// Candidate lane packing (host-built, P.pack): per candidate warp w of a GPU and lane l, the
+// geometry (0xFF idle), the slice position, the group size Z (power of two >= slice count) and the
+// lane of the group's slice 0, packed as j | s << 8 | Z << 16 | base << 24.
+
 // Dynamic shared-memory layout (byte offsets), computed on the host.
 struct SmemLayout {
   int S;            // streams = 2 * M
-  int N, Gc;        // simulated GPUs, candidate geometries in range
-  int BS, WS;       // batches / window entries held in smem (rest spills to global scratch)
-  size_t tab, hist, s_cnt, s_run, s_base, s_tot, s_skip, s_pend;
-  size_t g_u8, g_i64, g_i32, keys, bats, ord, glist, sarr, total;
-  __host__ void init(int words, int M, int n_gpus, int gc, int bs, int ws) {
-    S = 2 * M; N = n_gpus; Gc = gc; BS = bs; WS = ws;
+  int N, Gc, CW;    // simulated GPUs, candidate geometries in range, candidate warps per GPU
+  int BS, WS;       // batches / window entries held in smem
+  size_t tab, pack, hist, s_cnt, s_run, s_base, s_tot, s_skip, s_pend;
+  size_t g_u8, g_i64, g_i32, a_n, a_ls, a_bu, keys, bats, ord, glist, sarr, total;
+  __host__ void init(int words, int M, int n_gpus, int gc, int cw, int bs, int ws) {
+    S = 2 * M; N = n_gpus; Gc = gc; CW = cw; BS = bs; WS = ws;
     size_t o = 0;
     auto take = [&](size_t bytes) { size_t r = o; o += (bytes + 15) & ~(size_t)15; return r; };
     tab = take((size_t)words * 4);
+    pack = take((size_t)CW * 32 * 4);
     hist = take((size_t)kNB * 4);               // 2 classes x 3328 buckets as packed u16 pairs
     s_cnt = take((size_t)kNSeg * S * 4);
     s_run = take((size_t)kNSeg * S * 4);
@@ -40,6 +46,9 @@ struct SmemLayout {
     g_u8 = take((size_t)N * 8);                 // geom, target, ctr, vm, bill, dec, best, want
     g_i64 = take((size_t)N * 12 * 8);           // rs, re, from, until, since, maxend, kbest, kcur, od, spot, busy, mem
     g_i32 = take((size_t)(2 * N + 2) * 4);      // gcnt[N], goff[N+1]
+    a_n = take((size_t)N * kZA * 4);            // actual lanes: list length, last start, busy-until
+    a_ls = take((size_t)N * kZA * 8);
+    a_bu = take((size_t)N * kZA * 8);
     keys = take((size_t)N * Gc * 8);
     bats = take((size_t)BS * sizeof(Bat));
     ord = take((size_t)BS * 4);
@@ -53,6 +62,7 @@ struct ReplayParams {
   // tables
   const int32_t* tab;
   TabLayout tl;
+  const uint32_t* pack;    // [CW*32] candidate lane packing
   int maxT;
   // trace (device)
   const uint32_t* arr;
@@ -83,7 +93,7 @@ struct ReplayParams {
   SmemLayout sl;
   int WCAP;                // max window entries of any epoch (prepass)
   char* scratch;
-  size_t slot_bytes, o_lists, o_lane_n, o_ls, o_bu, o_gbat, o_gord, o_gglist, o_gsarr;
+  size_t slot_bytes, o_alist, o_clist, o_gbat, o_gord, o_gglist, o_gsarr;
   int* err;
 };
 
