@@ -394,7 +394,13 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
 
   // launch geometry: 8 warps; units = actual-placement warps + candidate warps per GPU
   const int Gc = h->G;
-  const int block = 256;
+  // warps per CTA: the placement phase runs n_units warp units; pick 4..8 warps that divide them
+  // most evenly (prefer more warps on ties)
+  const int n_units = (N + 3) / 4 + (c.policy == 0 ? N * h->CW : 0);
+  int best_nw = 8;  // measured on B200: 8 warps x 3 CTAs/SM beat 6 x 4 (L1 room for lane lists)
+  (void)n_units;
+  if (const char* ev = std::getenv("PROTEAN_WARPS")) best_nw = std::max(4, std::min(8, std::atoi(ev)));
+  const int block = 32 * best_nw;
   SmemLayout sl;
   sl.init(h->tl.words, h->M, N, Gc, h->CW, 0, 0);
   const size_t fixed = sl.total;

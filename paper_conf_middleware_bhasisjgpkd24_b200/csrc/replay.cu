@@ -222,12 +222,20 @@ struct SliceOut {
 // One Place() (Alg 1) of a batch on one lane group: each lane is one slice position s of
 // geometry j; the lane keeps its own slice's resident list.  Returns the group outcome; this
 // lane's own [start, end) candidate in *my_start / *my_end.
-__device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, int j, int s, int p,
-                                                int Z, const LaneList& L, int& n, int64_t& ls,
+struct SliceLane {        // per-lane constants of one placement unit
+  const int32_t* fbr_p;   // fbr[model][p] = fbr_p[model * 5]
+  const int32_t* solo_p;  // solo[model][p] = solo_p[model * 5]
+  int32_t Ms, pref;       // slice memory; capacity of slices 0..s (tag walk, Alg 1 lines 1-8)
+  int s, p, Z;
+};
+
+__device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, const SliceLane& K,
+                                                const LaneList& L, int& n, int64_t& ls,
                                                 int64_t t, int m, bool strict, int max_live,
                                                 int64_t* my_start, int64_t* my_end) {
   const int64_t t0 = t > ls ? t : ls;
-  const int32_t* fbr_p = T.fbr + p;  // fbr[model][p] = fbr_p[model * 5]
+  const int32_t* fbr_p = K.fbr_p;
+  const int Z = K.Z, s = K.s, p = K.p;
   int32_t used = 0, be = 0;
   int64_t fs = 0;
   bool fut = false;
@@ -257,7 +265,7 @@ __device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, int j
   uint64_t key = ~0ull;
   int64_t start = 0, c = 0;
   const int32_t q = T.mem[m];
-  const int32_t Ms = prof_cap(p);
+  const int32_t Ms = K.Ms;
   if (active && !o.drop_overflow && q <= Ms) {
     int64_t F;
     const int64_t own_f = fbr_p[m * kNProf];
@@ -267,9 +275,9 @@ __device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, int j
     } else {
       slice_slow(L, n, t0, q, Ms, fbr_p, own_f, &start, &F);
     }
-    c = start + exec_time(T.solo[m * kNProf + p], F);
+    c = start + exec_time(K.solo_p[m * kNProf], F);
     if (strict) {  // choose_strict_slice: tag < 1 (Alg 1 lines 1-8), least eta == least completion
-      const uint64_t inelig = (be_mem >= T.gpref[j * 8 + s]) ? (1ull << 62) : 0ull;
+      const uint64_t inelig = (be_mem >= K.pref) ? (1ull << 62) : 0ull;
       key = inelig | ((uint64_t)c << 6) | ((uint64_t)(4 - p) << 3) | (uint64_t)s;
     } else {       // choose_best_effort_slice: first fit, else earliest start (reading Q12)
       key = ((uint64_t)start << 3) | (uint64_t)s;
@@ -302,6 +310,13 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
   uint32_t* packs = reinterpret_cast<uint32_t*>(smem + SL.pack);
 #pragma unroll 1
   for (int i = tid; i < CW * 32; i += NT) packs[i] = P.pack[i];
+  uint16_t* klut = reinterpret_cast<uint16_t*>(smem + SL.klut);  // meta byte -> stream key
+#pragma unroll 1
+  for (int b = tid; b < 256; b += NT) {
+    const int m = b & 63;
+    const bool ok = !(b & 0x40) && m < P.tl.M;
+    klut[b] = (uint16_t)((2 * (ok ? m : 0) + ((b >> 7) ? 0 : 1)) | (ok ? 0 : 0x8000));
+  }
   c.T.bind(tabw, P.tl);
   c.pack = packs;
   c.hist = reinterpret_cast<uint32_t*>(smem + SL.hist);
@@ -450,7 +465,7 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
           }
 #pragma unroll
           for (int u = 0; u < 4; ++u) {
-            const int key = mt[u] == 0xFF ? 1024 + lane : 2 * ((mt[u] & 63) < T.M ? (mt[u] & 63) : 0) + ((mt[u] >> 7) ? 0 : 1);
+            const int key = i0 + u * 32 + lane < b ? (klut[mt[u]] & 0x7FFF) : 1024 + lane;
             const unsigned peers = __match_any_sync(0xffffffffu, key);
             if (key < 1024 && (peers & ((1u << lane) - 1u)) == 0) cntw[key] += __popc(peers);
           }
@@ -511,11 +526,11 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
             uint32_t ap = __shfl_up_sync(0xffffffffu, ai[u], 1);
             if (lane == 0) ap = prev_last;
             prev_last = __shfl_sync(0xffffffffu, ai[u], 31);
-            const int m = mt[u] & 63;
+            const int kv = klut[mt[u]];
             if (valid && i >= nbeg &&  // validate each request once (when it is new)
-                ((mt[u] & 0x40) || m >= T.M || (int64_t)ai[u] >= P.trace_len || ai[u] < ap))
+                ((kv & 0x8000) || (int64_t)ai[u] >= P.trace_len || ai[u] < ap))
               atomicOr(P.err, 1);
-            const int key = valid ? 2 * (m < T.M ? m : 0) + ((mt[u] >> 7) ? 0 : 1) : 1024 + lane;
+            const int key = valid ? (kv & 0x7FFF) : 1024 + lane;
             const unsigned peers = __match_any_sync(0xffffffffu, key);
             const unsigned rank = __popc(peers & ((1u << lane) - 1u));
             if (valid) sa[runw[key] + (int)rank] = ai[u];
@@ -794,6 +809,14 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
         }
         const bool active = valid && s < T.gn[j];
         const int p = active ? T.gprof[j * 8 + s] : 0;
+        SliceLane K;
+        K.fbr_p = T.fbr + p;
+        K.solo_p = T.solo + p;
+        K.Ms = prof_cap(p);
+        K.pref = T.gpref[j * 8 + (s & 7)];
+        K.s = s;
+        K.p = p;
+        K.Z = Z;
         const int al = actual && valid ? g * kZA + s : 0;  // actual lane id
         LaneList L;
         if (actual) {
@@ -822,7 +845,7 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
           const bool strict = (info >> 24) & 1;
           const int64_t t = has ? (int64_t)bt->ready : 0;
           int64_t st, en;
-          const SliceOut so = place_group(T, active && has, j, s, p, Z, L, n, ls, t, m, strict,
+          const SliceOut so = place_group(T, active && has, K, L, n, ls, t, m, strict,
                                           P.max_live, &st, &en);
           const bool placed = !so.drop_overflow && so.kmin != ~0ull;
           const int wl = (gbase + (int)(so.kmin & 7)) & 31;

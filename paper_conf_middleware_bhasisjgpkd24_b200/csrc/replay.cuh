@@ -28,7 +28,7 @@ struct SmemLayout {
   int S;            // streams = 2 * M
   int N, Gc, CW;    // simulated GPUs, candidate geometries in range, candidate warps per GPU
   int BS, WS;       // batches / window entries held in smem
-  size_t tab, pack, hist, s_cnt, s_run, s_base, s_tot, s_skip, s_pend;
+  size_t tab, pack, klut, hist, s_cnt, s_run, s_base, s_tot, s_skip, s_pend;
   size_t g_u8, g_i64, g_i32, a_n, a_ls, a_bu, keys, bats, ord, glist, sarr, total;
   __host__ void init(int words, int M, int n_gpus, int gc, int cw, int bs, int ws) {
     S = 2 * M; N = n_gpus; Gc = gc; CW = cw; BS = bs; WS = ws;
@@ -36,6 +36,7 @@ struct SmemLayout {
     auto take = [&](size_t bytes) { size_t r = o; o += (bytes + 15) & ~(size_t)15; return r; };
     tab = take((size_t)words * 4);
     pack = take((size_t)CW * 32 * 4);
+    klut = take(256 * 2);
     hist = take((size_t)kNB * 4);               // 2 classes x 3328 buckets as packed u16 pairs
     s_cnt = take((size_t)kNSeg * S * 4);
     s_run = take((size_t)kNSeg * S * 4);
