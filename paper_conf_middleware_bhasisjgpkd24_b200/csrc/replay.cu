@@ -13,6 +13,22 @@
 // read scatters it); everything else lives in shared memory, registers and L1-resident scratch.
 #include <cuda_runtime.h>
 #include "replay.cuh"
+#ifndef PROTEAN_MINB
+#define PROTEAN_MINB 3
+#endif
+#ifdef PROTEAN_PHASE_TIMING  // debug build only: per-phase wall cycles between CTA barriers
+__device__ unsigned long long g_phase_cycles[16];
+#define PH(k)                                   \
+  do {                                          \
+    if (threadIdx.x == 0) {                     \
+      const long long t_ = clock64();           \
+      ph_acc[k] += (unsigned long long)(t_ - ph_last); \
+      ph_last = t_;                             \
+    }                                           \
+  } while (0)
+#else
+#define PH(k) do {} while (0)
+#endif
 
 namespace pemgpu {
 
@@ -59,6 +75,7 @@ struct Ctx {
 struct CtaState {
   int64_t w_lo, lt_total, nlog;
   int nb, cursor, all_avail, bad;
+  int task, adone;
   unsigned amin;
   unsigned long long cnt[10];
 };
@@ -132,6 +149,18 @@ __device__ __forceinline__ void vm_event(const ReplayParams& P, const Ctx& c, ui
         c.g_rs[g] = c.g_re[g] = 0;
       }
     }
+  }
+}
+
+// Bulk L2 prefetch (TMA engine, sm_90+): [p, p + bytes) rounded out to 16-byte boundaries.
+__device__ __forceinline__ void prefetch_l2(const void* p, int64_t bytes) {
+  if (bytes <= 0) return;
+  uintptr_t a = reinterpret_cast<uintptr_t>(p) & ~(uintptr_t)15;
+  uintptr_t e = (reinterpret_cast<uintptr_t>(p) + (uintptr_t)bytes + 15) & ~(uintptr_t)15;
+  while (a < e) {
+    const uint32_t n = (uint32_t)((e - a) > (1u << 20) ? (1u << 20) : (e - a));
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a), "r"(n) : "memory");
+    a += n;
   }
 }
 
@@ -294,11 +323,120 @@ __device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, const
   return o;
 }
 
+// Candidate unit with register-resident slice lists (the GPU-epoch has <= kKR batches, so no lane
+// ever holds more residents).  Replay states are FIFO-consistent, so every resident started at or
+// before the slice's last start: Eq 1's co-runners at an instant x >= t0 are exactly the residents
+// with end > x, and start times need not be kept.  Ended residents (end <= t) are simply ignored.
+constexpr int kKR = 6;
+__device__ __forceinline__ void candidate_unit_regs(const Tab& T, const SliceLane& K, bool active,
+                                                    bool leader, const Bat* bats, const uint32_t* gl,
+                                                    int x0, int x1, const uint32_t* sarr, int max_live,
+                                                    int64_t* misses_out, int64_t* tail_out) {
+  int64_t en_r[kKR];
+  uint32_t mm_r[kKR];
+#pragma unroll
+  for (int i = 0; i < kKR; ++i) { en_r[i] = 0; mm_r[i] = 0; }
+  int n = 0;
+  int64_t ls = 0, misses = 0, tail = 0;
+  const int lane = threadIdx.x & 31;
+  const int gbase = lane & ~(K.Z - 1);
+#pragma unroll 1
+  for (int x = x0; x < x1; ++x) {
+    const Bat& bt = bats[gl[x]];
+    const uint32_t info = bt.info;
+    const int m = (info >> 16) & 0xFF, nreq = info & 0xFFFF;
+    const bool strict = (info >> 24) & 1;
+    const int64_t t = bt.ready;
+    const int64_t t0 = t > ls ? t : ls;
+    int32_t used = 0, be = 0, live = 0;
+    int64_t fs = 0;
+#pragma unroll
+    for (int i = 0; i < kKR; ++i) {
+      if (i < n && en_r[i] > t) {
+        const int32_t mem = mm_r[i] & 0xFFFF;
+        ++live;
+        if (!((mm_r[i] >> 22) & 1)) be += mem;
+        if (en_r[i] > t0) {
+          used += mem;
+          fs += K.fbr_p[((mm_r[i] >> 16) & 63) * kNProf];
+        }
+      }
+    }
+    const int live_g = group_sum32(active ? live : 0, K.Z);
+    const int be_mem = group_sum32(active ? be : 0, K.Z);
+    const bool overflow = live_g >= max_live;
+    const int32_t q = T.mem[m];
+    uint64_t key = ~0ull;
+    int64_t start = 0, c = 0;
+    if (active && !overflow && q <= K.Ms) {
+      int64_t F = K.fbr_p[m * kNProf];
+      if (used + q <= K.Ms) {
+        start = t0;
+        F += fs;
+      } else {  // memory wait: the earliest release after which the batch fits
+        start = INT64_MAX;
+#pragma unroll
+        for (int jj = 0; jj < kKR; ++jj) {
+          if (jj < n && en_r[jj] > t0) {
+            int32_t rem = 0;
+#pragma unroll
+            for (int i = 0; i < kKR; ++i)
+              if (i < n && en_r[i] > en_r[jj]) rem += mm_r[i] & 0xFFFF;
+            if (rem + q <= K.Ms && en_r[jj] < start) start = en_r[jj];
+          }
+        }
+#pragma unroll
+        for (int i = 0; i < kKR; ++i)
+          if (i < n && en_r[i] > start) F += K.fbr_p[((mm_r[i] >> 16) & 63) * kNProf];
+      }
+      c = start + exec_time(K.solo_p[m * kNProf], F);
+      if (strict) {
+        const uint64_t inelig = (be_mem >= K.pref) ? (1ull << 62) : 0ull;
+        key = inelig | ((uint64_t)c << 6) | ((uint64_t)(4 - K.p) << 3) | (uint64_t)K.s;
+      } else {
+        key = ((uint64_t)start << 3) | (uint64_t)K.s;
+      }
+    }
+    const uint64_t kmin = group_min(key, K.Z);
+    const bool placed = !overflow && kmin != ~0ull;
+    if (placed && key == kmin) {  // schedule(batch, chosen_slice)
+      const uint32_t mw = (uint32_t)q | ((uint32_t)m << 16) | ((uint32_t)(strict ? 1 : 0) << 22);
+#pragma unroll
+      for (int i = 0; i < kKR; ++i)
+        if (i == n) { en_r[i] = c; mm_r[i] = mw; }
+      ++n;
+      ls = start;
+    }
+    const int64_t cwin = __shfl_sync(0xffffffffu, c, (gbase + (int)(kmin & 7)) & 31);
+    if (leader) {
+      if (strict) {
+        if (!placed) {
+          misses += nreq;
+        } else {  // latencies fall along the sorted members: test the ends first
+          const uint32_t* ma = sarr + bt.pos;
+          const int64_t slo = T.slo[m];
+          if (cwin - (int64_t)ma[0] > slo)
+            misses += (cwin - (int64_t)ma[nreq - 1] > slo) ? nreq : nreq - hits_in(ma, nreq, cwin, slo);
+        }
+      } else {
+        const int64_t tb = placed ? cwin - (int64_t)sarr[bt.pos] : (int64_t)0xFFFFFFFFLL;
+        tail = tb > tail ? tb : tail;
+      }
+    }
+  }
+  *misses_out = misses;
+  *tail_out = tail;
+}
+
 }  // namespace
 
-__global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
+__global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams P) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ CtaState cs;
+#ifdef PROTEAN_PHASE_TIMING
+  unsigned long long ph_acc[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
+  long long ph_last = clock64();
+#endif
   const SmemLayout& SL = P.sl;
   const int tid = threadIdx.x, NT = blockDim.x, lane = tid & 31, warp = tid >> 5, NW = NT >> 5;
   const int N = P.N, S = SL.S, Gc = SL.Gc, CW = SL.CW;
@@ -411,7 +549,7 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
       const int64_t eW = e * P.W, Tend = eW + P.W;
       // ---------------------------------------------------------------- A: VM events, installs
 #pragma unroll 1
-      for (int i = tid; i < kNSeg * S; i += NT) c.s_cnt[i] = 0;
+      for (int i = tid; i < NW * S; i += NT) c.s_cnt[i] = 0;
 #pragma unroll 1
       for (int g = tid; g < N; g += NT) {
         if (P.vm_policy != 0) {
@@ -430,6 +568,8 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
         c.g_kcur[g] = -1;
       }
       if (tid == 0) {
+        cs.task = 0;
+        cs.adone = 0;
         cs.nb = 0;
         cs.amin = 0xFFFFFFFFu;
         cs.lt_total = 0;
@@ -437,7 +577,13 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
       }
       const int64_t w_beg = eoff[e], w_end = eoff[e + 1];
       const int64_t w_lo = cs.w_lo;
+      if (tid == 32 && e + 1 < P.E) {  // the next epoch's new requests: into L2 during this one
+        const int64_t nb0 = w_end, nb1 = eoff[e + 2];
+        prefetch_l2(P.meta + nb0, nb1 - nb0);
+        prefetch_l2(P.arr + nb0, (nb1 - nb0) * 4);
+      }
       __syncthreads();
+      PH(0);
 #pragma unroll 1
       for (int g = tid; g < N; g += NT) {
         const bool whole = c.g_from[g] <= eW && c.g_until[g] >= Tend &&
@@ -452,37 +598,56 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
       const uint8_t* wmeta = P.meta + w_lo;
       const int nbeg = (int)(w_beg - w_lo);  // window offset of the first new request
       // ---------------------------------------------------------------- B: stream partition
-      if (warp < kNSeg) {  // count per (segment, stream): warp-aggregated by match_any
-        const int a = (int)((int64_t)len * warp / kNSeg), b = (int)((int64_t)len * (warp + 1) / kNSeg);
+      // every warp owns one contiguous segment of the window: (1) count per (segment, stream) with
+      // 16-byte meta loads, (2) after one barrier each warp derives its own per-stream write
+      // offsets (redundant scan over streams), (3) stable scatter of its segment with 8 loads in
+      // flight per lane, validating every request once (when it is new).
+      const int sa_lo = (int)((int64_t)len * warp / NW), sa_hi = (int)((int64_t)len * (warp + 1) / NW);
+      {
         int* cntw = c.s_cnt + warp * S;
+        const int h = min(sa_hi, sa_lo + (int)((16u - ((uint32_t)(uintptr_t)(wmeta + sa_lo) & 15u)) & 15u));
+        {  // unaligned head (< 16 elements)
+          const int i = sa_lo + lane;
+          const int key = i < h ? (klut[wmeta[i]] & 0x7FFF) : 1024 + lane;
+          const unsigned peers = __match_any_sync(0xffffffffu, key);
+          if (key < 1024 && (peers & ((1u << lane) - 1u)) == 0) cntw[key] += __popc(peers);
+        }
+        const int nch = (sa_hi - h) >> 4;
+        const uint4* gv = reinterpret_cast<const uint4*>(wmeta + h);
 #pragma unroll 1
-        for (int i0 = a; i0 < b; i0 += 128) {
-          uint8_t mt[4];
+        for (int c0 = 0; c0 < nch; c0 += 32) {
+          const int ch = c0 + lane;
+          const bool valid = ch < nch;
+          const uint4 v = valid ? gv[ch] : make_uint4(0u, 0u, 0u, 0u);
+          const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
-          for (int u = 0; u < 4; ++u) {
-            const int i = i0 + u * 32 + lane;
-            mt[u] = i < b ? wmeta[i] : (uint8_t)0xFF;
-          }
-#pragma unroll
-          for (int u = 0; u < 4; ++u) {
-            const int key = i0 + u * 32 + lane < b ? (klut[mt[u]] & 0x7FFF) : 1024 + lane;
+          for (int q = 0; q < 16; ++q) {
+            const int key = valid ? (klut[(w4[q >> 2] >> (8 * (q & 3))) & 0xFF] & 0x7FFF) : 1024 + lane;
             const unsigned peers = __match_any_sync(0xffffffffu, key);
             if (key < 1024 && (peers & ((1u << lane) - 1u)) == 0) cntw[key] += __popc(peers);
           }
         }
+        {  // tail (< 16 elements)
+          const int i = h + nch * 16 + lane;
+          const int key = i < sa_hi ? (klut[wmeta[i]] & 0x7FFF) : 1024 + lane;
+          const unsigned peers = __match_any_sync(0xffffffffu, key);
+          if (key < 1024 && (peers & ((1u << lane) - 1u)) == 0) cntw[key] += __popc(peers);
+        }
       }
       __syncthreads();
-      if (warp == 0) {  // stream offsets: per-stream totals, exclusive scan over streams
+      PH(1);
+      {  // this warp's write offsets: base_k (exclusive scan of stream totals) + earlier segments
+        int* runw = c.s_run + warp * S;
         int carry = 0;
 #pragma unroll 1
         for (int k0 = 0; k0 < S; k0 += 32) {
           const int k = k0 + lane;
-          int tot = 0;
+          int tot = 0, part = 0;
           if (k < S) {
-#pragma unroll
-            for (int w = 0; w < kNSeg; ++w) {
+#pragma unroll 1
+            for (int w = 0; w < NW; ++w) {
               const int cv = c.s_cnt[w * S + k];
-              c.s_run[w * S + k] = tot;
+              if (w < warp) part += cv;
               tot += cv;
             }
           }
@@ -494,35 +659,32 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
           }
           const int base = carry + x - tot;
           if (k < S) {
-            c.s_base[k] = base;
-            c.s_tot[k] = tot;
-#pragma unroll
-            for (int w = 0; w < kNSeg; ++w) c.s_run[w * S + k] += base;
+            runw[k] = base + part;
+            if (warp == 0) {
+              c.s_base[k] = base;
+              c.s_tot[k] = tot;
+            }
           }
           carry += __shfl_sync(0xffffffffu, x, 31);
         }
-      }
-      __syncthreads();
-      if (warp < kNSeg) {  // stable scatter into stream-sorted order + validation of new requests
-        const int a = (int)((int64_t)len * warp / kNSeg), b = (int)((int64_t)len * (warp + 1) / kNSeg);
-        int* runw = c.s_run + warp * S;
+        __syncwarp();
         uint32_t* sa = c.sarr;
-        uint32_t prev_last = (a > 0) ? warr[a - 1] : (w_lo > r_lo ? P.arr[w_lo - 1] : 0u);
+        uint32_t prev_last = (sa_lo > 0) ? warr[sa_lo - 1] : (w_lo > r_lo ? P.arr[w_lo - 1] : 0u);
 #pragma unroll 1
-        for (int i0 = a; i0 < b; i0 += 128) {
-          uint8_t mt[4];
-          uint32_t ai[4];
+        for (int i0 = sa_lo; i0 < sa_hi; i0 += 256) {
+          uint8_t mt[8];
+          uint32_t ai[8];
 #pragma unroll
-          for (int u = 0; u < 4; ++u) {
+          for (int u = 0; u < 8; ++u) {
             const int i = i0 + u * 32 + lane;
-            const bool valid = i < b;
-            mt[u] = valid ? wmeta[i] : (uint8_t)0xFF;
+            const bool valid = i < sa_hi;
+            mt[u] = valid ? wmeta[i] : (uint8_t)0;
             ai[u] = valid ? warr[i] : 0xFFFFFFFFu;
           }
 #pragma unroll
-          for (int u = 0; u < 4; ++u) {
+          for (int u = 0; u < 8; ++u) {
             const int i = i0 + u * 32 + lane;
-            const bool valid = i < b;
+            const bool valid = i < sa_hi;
             uint32_t ap = __shfl_up_sync(0xffffffffu, ai[u], 1);
             if (lane == 0) ap = prev_last;
             prev_last = __shfl_sync(0xffffffffu, ai[u], 31);
@@ -541,6 +703,7 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
         }
       }
       __syncthreads();
+      PH(3);
       // ---------------------------------------------------------------- C: batch formation
       // warp per stream: lanes test 32 consecutive B-sized batches at once (full batches are the
       // common case); a batch closed by the timeout, or still open, is resolved by lane 0.
@@ -624,6 +787,7 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
         }
       }
       __syncthreads();
+      PH(4);
       const int nb = cs.nb;
       const unsigned amin = cs.amin;
       if (nb > c.BS) {  // rare: more batches than the smem arrays hold -> all in global scratch
@@ -664,6 +828,7 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
         ord[rank] = (uint32_t)b;
       }
       __syncthreads();
+      PH(5);
       if (tid == 0) cs.w_lo = bad_window ? w_end : w_lo + cs.lt_total;
       // ---------------------------------------------------------------- D: dispatch
       if (cs.all_avail) {
@@ -772,13 +937,97 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
         cs.cursor = cur;
       }
       __syncthreads();
+      PH(6);
       // ---------------------------------------------------------------- E: placement units
       // unit < n_aunits: actual placement of GPUs 4u..4u+3 (8 slice lanes each, carried state);
       // otherwise candidate warp w of GPU g: lane groups = candidate geometries from idle (O8).
       // One loop body serves both kinds (a single inlined copy of Place).
+      // dynamic task queue: [actual units][candidate units][accounting of batch rank rk];
+      // accounting waits (rarely) for the actual units, whose warps publish via cs.adone
       const int n_units = n_aunits + (P.policy == 0 ? N * CW : 0);
+      const int n_tasks = n_units + nb;
+      for (;;) {
+        int u = 0;
+        if (lane == 0) u = atomicAdd(&cs.task, 1);
+        u = __shfl_sync(0xffffffffu, u, 0);
+        if (u >= n_tasks) break;
+#ifdef PROTEAN_PHASE_TIMING
+        const long long tk0 = clock64();
+        const int tkind = u >= n_units ? 2 : (u < n_aunits ? 0 : 1);
+        struct TaskClock {
+          long long t0; int kind; int lane; unsigned long long* acc;
+          __device__ ~TaskClock() { if (lane == 0) atomicAdd(&acc[kind], (unsigned long long)(clock64() - t0)); }
+        } tclock{tk0, tkind, lane, g_phase_cycles + 10};
+#endif
+        if (u >= n_units) {  // ---- F: accounting (O7) of batch rank u - n_units
+          if (lane == 0) {
+            while (*(volatile int*)&cs.adone < n_aunits) __nanosleep(64);
+          }
+          __syncwarp();
+          __threadfence_block();
+          const int rk = u - n_units;
+          const Bat& bt = bats[ord[rk]];
+          const int nreq = bt.info & 0xFFFF, m = (bt.info >> 16) & 0xFF;
+          const bool strict = (bt.info >> 24) & 1;
+          if (lane == 0) {
+            if (strict) {
+              cnt[0] += nreq;
+              if (bt.drop) cnt[3] += nreq;
+            } else {
+              cnt[4] += nreq;
+              if (bt.drop) cnt[6] += nreq;
+            }
+            const int64_t row = cs.nlog + rk;
+            if (P.log && row < P.log_cap) {
+              protean_batch_rec rec;
+              rec.ready_us = bt.ready;
+              rec.epoch = (uint32_t)e;
+              rec.n_req = (uint16_t)nreq;
+              rec.model = (uint8_t)m;
+              rec.strict = strict ? 1 : 0;
+              rec.gpu = bt.gpu;
+              rec.slice = bt.slice;
+              rec.dropped = bt.drop;
+              rec.pad = 0;
+              rec.start_us = bt.start;
+              rec.end_us = bt.end;
+              P.log[(size_t)r * P.log_cap + row] = rec;
+            }
+          }
+          if (!bt.drop) {  // latencies are non-increasing along the sorted members: runs of equal
+            const int64_t slo = T.slo[m];  // buckets become one histogram update
+            const int cls = strict ? 0 : kNB;
+            const uint32_t* ma = sarr + bt.pos;
+            const int64_t bend = bt.end;
 #pragma unroll 1
-      for (int u = warp; u < n_units; u += NW) {
+            for (int i0 = 0; i0 < nreq; i0 += 32) {
+              const int i = i0 + lane;
+              const bool valid = i < nreq;
+              const int64_t lat = valid ? bend - (int64_t)ma[i] : 0;
+              const int bk = valid ? lat_bucket(lat) : -1;
+              const int prev = __shfl_up_sync(0xffffffffu, bk, 1);
+              const bool head = valid && (lane == 0 || prev != bk);
+              const unsigned heads = __ballot_sync(0xffffffffu, head);
+              const unsigned vmask = __ballot_sync(0xffffffffu, valid);
+              const unsigned met = __ballot_sync(0xffffffffu, valid && lat <= slo);
+              if (head) {
+                const unsigned after = heads & ~((2u << lane) - 1u);
+                const int stop = after ? __ffs(after) - 1 : 32 - __clz(vmask);
+                hist_add(c, ghist, cls + bk, (uint32_t)(stop - lane));
+              }
+              if (lane == 0) {
+                if (strict) {
+                  cnt[1] += __popc(met);
+                  cnt[2] += __popc(vmask) - __popc(met);
+                } else {
+                  cnt[5] += __popc(vmask);
+                }
+              }
+            }
+          }
+      
+          continue;
+        }
         const bool actual = u < n_aunits;
         int g, s, Z, gbase, j;
         bool valid;
@@ -834,6 +1083,19 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
         for (int d = 1; d < 32; d <<= 1) {
           const int o = __shfl_xor_sync(0xffffffffu, len_max, d);
           len_max = o > len_max ? o : len_max;
+        }
+        if (!actual && len_max <= kKR) {  // register-resident candidate lists
+          int64_t misses, tail;
+          // warp-uniform batch range (idle lanes must still take part in the group shuffles)
+          candidate_unit_regs(T, K, active, lane == gbase && valid, bats, gl, c.g_off[g],
+                              c.g_off[g + 1], sarr, P.max_live, &misses, &tail);
+          if (valid && lane == gbase) {
+            const int64_t key = make_key(misses, tail, j == c.g_geom[g] ? 0 : j + 1);
+            if (j == c.g_geom[g]) c.g_kcur[g] = key;
+            c.keys[g * Gc + (j - P.geom_lo)] = key;
+            if (P.cand_keys) P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = key;
+          }
+          continue;
         }
         int64_t acc0 = 0, acc1 = 0;  // actual: busy, mem-time; candidate: misses, BE tail
 #pragma unroll 1
@@ -904,6 +1166,11 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
             c.g_busy[g] += bsum;
             c.g_mem[g] += msum;
           }
+          __syncwarp();
+          if (lane == 0) {
+            __threadfence_block();
+            atomicAdd(&cs.adone, 1);
+          }
         } else if (valid && lane == gbase) {
           const int64_t key = make_key(acc0, acc1, j == c.g_geom[g] ? 0 : j + 1);
           if (j == c.g_geom[g]) c.g_kcur[g] = key;
@@ -912,69 +1179,7 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
         }
       }
       __syncthreads();
-      // ---------------------------------------------------------------- F: accounting (O7)
-#pragma unroll 1
-      for (int rk = warp; rk < nb; rk += NW) {
-        const Bat& bt = bats[ord[rk]];
-        const int nreq = bt.info & 0xFFFF, m = (bt.info >> 16) & 0xFF;
-        const bool strict = (bt.info >> 24) & 1;
-        if (lane == 0) {
-          if (strict) {
-            cnt[0] += nreq;
-            if (bt.drop) cnt[3] += nreq;
-          } else {
-            cnt[4] += nreq;
-            if (bt.drop) cnt[6] += nreq;
-          }
-          const int64_t row = cs.nlog + rk;
-          if (P.log && row < P.log_cap) {
-            protean_batch_rec rec;
-            rec.ready_us = bt.ready;
-            rec.epoch = (uint32_t)e;
-            rec.n_req = (uint16_t)nreq;
-            rec.model = (uint8_t)m;
-            rec.strict = strict ? 1 : 0;
-            rec.gpu = bt.gpu;
-            rec.slice = bt.slice;
-            rec.dropped = bt.drop;
-            rec.pad = 0;
-            rec.start_us = bt.start;
-            rec.end_us = bt.end;
-            P.log[(size_t)r * P.log_cap + row] = rec;
-          }
-        }
-        if (!bt.drop) {  // latencies are non-increasing along the sorted members: runs of equal
-          const int64_t slo = T.slo[m];  // buckets become one histogram update
-          const int cls = strict ? 0 : kNB;
-          const uint32_t* ma = sarr + bt.pos;
-          const int64_t bend = bt.end;
-#pragma unroll 1
-          for (int i0 = 0; i0 < nreq; i0 += 32) {
-            const int i = i0 + lane;
-            const bool valid = i < nreq;
-            const int64_t lat = valid ? bend - (int64_t)ma[i] : 0;
-            const int bk = valid ? lat_bucket(lat) : -1;
-            const int prev = __shfl_up_sync(0xffffffffu, bk, 1);
-            const bool head = valid && (lane == 0 || prev != bk);
-            const unsigned heads = __ballot_sync(0xffffffffu, head);
-            const unsigned vmask = __ballot_sync(0xffffffffu, valid);
-            const unsigned met = __ballot_sync(0xffffffffu, valid && lat <= slo);
-            if (head) {
-              const unsigned after = heads & ~((2u << lane) - 1u);
-              const int stop = after ? __ffs(after) - 1 : 32 - __clz(vmask);
-              hist_add(c, ghist, cls + bk, (uint32_t)(stop - lane));
-            }
-            if (lane == 0) {
-              if (strict) {
-                cnt[1] += __popc(met);
-                cnt[2] += __popc(vmask) - __popc(met);
-              } else {
-                cnt[5] += __popc(vmask);
-              }
-            }
-          }
-        }
-      }
+      PH(7);
       // ---------------------------------------------------------------- G: decisions (O9, O10)
 #pragma unroll 1
       for (int g = tid; g < N; g += NT) {
@@ -1006,6 +1211,7 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
         }
       }
       __syncthreads();
+      PH(8);
       if (tid == 0) {
         if (P.policy == 0) {
           int alive = 0, open = 0;
@@ -1040,6 +1246,7 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
         cs.nlog += nb;
       }
       __syncthreads();
+      PH(9);
     }
 
     // ---------------------------------------------------------------- finalize (O12)
@@ -1113,7 +1320,17 @@ __global__ void __launch_bounds__(256, 3) replay_kernel(ReplayParams P) {
     }
     __syncthreads();
   }
+#ifdef PROTEAN_PHASE_TIMING
+  if (threadIdx.x == 0)
+    for (int k = 0; k < 10; ++k) atomicAdd(&g_phase_cycles[k], ph_acc[k]);
+#endif
 }
+
+#ifdef PROTEAN_PHASE_TIMING
+extern "C" int protean_debug_phase_cycles(unsigned long long* out) {
+  return (int)cudaMemcpyFromSymbol(out, g_phase_cycles, sizeof(unsigned long long) * 13);
+}
+#endif
 
 // Prepass: eoff[r][e] = first request of replica r with arrival >= e*W (e = 0..E), and the
 // largest request window any epoch needs: [lower_bound(eW - maxT), eoff[e+1]).

@@ -7,7 +7,7 @@
 
 namespace pemgpu {
 
-constexpr int kNSeg = 4;          // warps that stream-partition the request window
+constexpr int kNSeg = 8;          // max warps per CTA (stream-partition segments)
 constexpr int kZA = 8;            // lanes per actual-placement group (one per slice position)
 constexpr int64_t kForever = INT64_MAX;
 

@@ -1,0 +1,39 @@
+"""Run one replay with the phase-timing debug build (libprotean_phase.so) and print the share of
+CTA wall cycles per epoch phase (thread 0 clock64 between barriers)."""
+import ctypes as C
+import os
+import shutil
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+PKG = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "paper_conf_middleware_bhasisjgpkd24_b200")
+import paper_conf_middleware_bhasisjgpkd24_b200._abi as A  # noqa: E402
+
+A.LIB_PATH = os.path.join(PKG, "libprotean_phase.so")
+import torch  # noqa: E402
+
+import paper_conf_middleware_bhasisjgpkd24_b200 as pkg  # noqa: E402
+from protean_inputs import mix_a_params, synth_profiles  # noqa: E402
+from tools import tracegen  # noqa: E402
+
+R = int(sys.argv[1]) if len(sys.argv) > 1 else 444
+S = int(sys.argv[2]) if len(sys.argv) > 2 else 60
+gp = mix_a_params(R, seed=1, seconds=S)
+arr, meta, roff = tracegen.generate_on_device(gp, 0)
+A._lib = None
+L = A.load(A.LIB_PATH)
+h = pkg.load_profiles(synth_profiles())
+out = h.replay_traces(arr, meta, roff, trace_len_us=gp.trace_len_us, n_gpus=8)
+torch.cuda.synchronize()
+buf = (C.c_ulonglong * 13)()
+L.protean_debug_phase_cycles(buf)
+names = ["A vm/install", "B count", "B offsets", "B scatter", "C formation", "C rank+window",
+         "D dispatch", "E placement", "F accounting+G decide", "G cap"]
+tot = sum(buf[:10]) or 1
+print("kernel ms", h.last_timings()[1])
+for n, v in zip(names, buf):
+    print(f"{100 * v / tot:5.1f}%  {n}")
+tt = sum(buf[10:13]) or 1
+ntask = (R * (gp.seconds + 1))
+for n, v in zip(["actual units", "candidate units", "accounting tasks"], buf[10:13]):
+    print(f"task time {100 * v / tt:5.1f}%  {n}  ({v / ntask:.0f} warp-cycles per replica-epoch)")
