@@ -54,11 +54,9 @@ struct LaneList {
 struct Ctx {
   Tab T;
   const uint32_t* pack;
-  uint32_t* hist;
-  int *s_cnt, *s_run, *s_base, *s_tot, *s_skip, *s_pend;
-  uint8_t *g_geom, *g_target, *g_ctr, *g_vm, *g_bill, *g_dec, *g_best, *g_want;
-  int64_t *g_rs, *g_re, *g_from, *g_until, *g_since, *g_maxend, *g_kbest, *g_kcur, *g_od,
-      *g_spot, *g_busy, *g_mem;
+  int N;
+  uint8_t* gu8;   // [8][N]: geom, target, ctr, vm, bill, dec, best, want
+  int64_t* gi;    // [12][N]: rs, re, from, until, since, maxend, kbest, kcur, od, spot, busy, mem
   int *g_cnt, *g_off;
   int* a_n;
   int64_t *a_ls, *a_bu;
@@ -85,17 +83,17 @@ enum { VM_NONE = 0, VM_OD = 1, VM_SPOT = 2 };
 __device__ __forceinline__ int64_t clip_h(int64_t x, int64_t H) { return x < H ? x : H; }
 
 __device__ void bill_switch(const Ctx& c, int g, int type, int64_t at, int64_t H) {
-  const int64_t d = clip_h(at, H) - clip_h(c.g_since[g], H);
-  if (c.g_bill[g] == VM_OD) c.g_od[g] += d;
-  if (c.g_bill[g] == VM_SPOT) c.g_spot[g] += d;
-  c.g_bill[g] = (uint8_t)type;
-  c.g_since[g] = at;
+  const int64_t d = clip_h(at, H) - clip_h(c.gi[4 * c.N + g], H);
+  if (c.gu8[4 * c.N + g] == VM_OD) c.gi[8 * c.N + g] += d;
+  if (c.gu8[4 * c.N + g] == VM_SPOT) c.gi[9 * c.N + g] += d;
+  c.gu8[4 * c.N + g] = (uint8_t)type;
+  c.gi[4 * c.N + g] = at;
 }
 
 __device__ void reset_gpu_state(const Ctx& c, int g, int geom) {
-  c.g_geom[g] = (uint8_t)geom;
-  c.g_target[g] = kNoGeom;
-  c.g_ctr[g] = 0;
+  c.gu8[0 * c.N + g] = (uint8_t)geom;
+  c.gu8[1 * c.N + g] = kNoGeom;
+  c.gu8[2 * c.N + g] = 0;
 #pragma unroll 1
   for (int s = 0; s < kZA; ++s) {
     c.a_n[g * kZA + s] = 0;
@@ -105,10 +103,10 @@ __device__ void reset_gpu_state(const Ctx& c, int g, int geom) {
 }
 
 __device__ __forceinline__ bool has_vm(const Ctx& c, int g, int64_t t) {
-  return c.g_from[g] <= t && t < c.g_until[g];
+  return c.gi[2 * c.N + g] <= t && t < c.gi[3 * c.N + g];
 }
 __device__ __forceinline__ bool available(const Ctx& c, int g, int64_t t) {
-  return has_vm(c, g, t) && !(c.g_rs[g] <= t && t < c.g_re[g]);
+  return has_vm(c, g, t) && !(c.gi[0 * c.N + g] <= t && t < c.gi[1 * c.N + g]);
 }
 
 // O11: one revocation boundary tau = k * T_rev for node g (draws specified in DESIGN.md §3).
@@ -119,34 +117,34 @@ __device__ __forceinline__ void vm_event(const ReplayParams& P, const Ctx& c, ui
   const uint64_t d1 = smix(P.seed ^ smix(x ^ 1ull)) >> 11;
   const bool revoked = d0 < P.thr, spot_ok = d1 >= P.thr;
   if (P.vm_policy == 1) {  // PROTEAN: retry spot, else on-demand; seamless redirect
-    if (c.g_vm[g] == VM_SPOT) {
+    if (c.gu8[3 * c.N + g] == VM_SPOT) {
       if (revoked && !spot_ok) {
-        c.g_vm[g] = VM_OD;
+        c.gu8[3 * c.N + g] = VM_OD;
         bill_switch(c, g, VM_OD, tau + P.notice, P.H);
       }
-    } else if (c.g_vm[g] == VM_OD) {
+    } else if (c.gu8[3 * c.N + g] == VM_OD) {
       if (spot_ok) {
-        c.g_vm[g] = VM_SPOT;
+        c.gu8[3 * c.N + g] = VM_SPOT;
         bill_switch(c, g, VM_SPOT, tau, P.H);
       }
     }
   } else if (P.vm_policy == 2) {  // Spot Only
-    if (c.g_vm[g] == VM_SPOT) {
+    if (c.gu8[3 * c.N + g] == VM_SPOT) {
       if (revoked && !spot_ok) {
-        c.g_vm[g] = VM_NONE;
-        c.g_until[g] = tau;
+        c.gu8[3 * c.N + g] = VM_NONE;
+        c.gi[3 * c.N + g] = tau;
         bill_switch(c, g, VM_NONE, tau + P.notice, P.H);
-        c.g_target[g] = kNoGeom;
-        c.g_rs[g] = c.g_re[g] = 0;
+        c.gu8[1 * c.N + g] = kNoGeom;
+        c.gi[0 * c.N + g] = c.gi[1 * c.N + g] = 0;
       }
-    } else if (c.g_vm[g] == VM_NONE) {
+    } else if (c.gu8[3 * c.N + g] == VM_NONE) {
       if (spot_ok) {
-        c.g_vm[g] = VM_SPOT;
-        c.g_from[g] = tau;
-        c.g_until[g] = kForever;
+        c.gu8[3 * c.N + g] = VM_SPOT;
+        c.gi[2 * c.N + g] = tau;
+        c.gi[3 * c.N + g] = kForever;
         bill_switch(c, g, VM_SPOT, tau, P.H);
         reset_gpu_state(c, g, P.init_geom);
-        c.g_rs[g] = c.g_re[g] = 0;
+        c.gi[0 * c.N + g] = c.gi[1 * c.N + g] = 0;
       }
     }
   }
@@ -166,11 +164,11 @@ __device__ __forceinline__ void prefetch_l2(const void* p, int64_t bytes) {
 
 // Packed u16 smem histogram; a half crossing 2^15 moves 2^15 counts to the HBM histogram
 // (cnt <= 32 per call, so a half never exceeds 0xFFFF before the move).
-__device__ __forceinline__ void hist_add(const Ctx& c, uint32_t* ghist, int idx, uint32_t cnt) {
+__device__ __forceinline__ void hist_add(uint32_t* hist, uint32_t* ghist, int idx, uint32_t cnt) {
   const int w = idx >> 1, sh = (idx & 1) * 16;
-  const uint32_t old = (atomicAdd(&c.hist[w], cnt << sh) >> sh) & 0xFFFFu;
+  const uint32_t old = (atomicAdd(&hist[w], cnt << sh) >> sh) & 0xFFFFu;
   if (old < 0x8000u && old + cnt >= 0x8000u) {
-    atomicSub(&c.hist[w], 0x8000u << sh);
+    atomicSub(&hist[w], 0x8000u << sh);
     atomicAdd(&ghist[idx], 0x8000u);
   }
 }
@@ -433,6 +431,10 @@ __device__ __forceinline__ void candidate_unit_regs(const Tab& T, const SliceLan
 __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams P) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ CtaState cs;
+  __shared__ uint32_t s_hist[2 * kNB];  // 2 classes x 3328 buckets (u32 < 2^32 per replica)
+  __shared__ uint16_t klut[256];        // meta byte -> stream key (| 0x8000 if invalid)
+  __shared__ int s_cnt[kNSeg * kMaxStreams], s_run[kNSeg * kMaxStreams];
+  __shared__ int s_base[kMaxStreams], s_tot[kMaxStreams], s_skip[kMaxStreams], s_pend[kMaxStreams];
 #ifdef PROTEAN_PHASE_TIMING
   unsigned long long ph_acc[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
   long long ph_last = clock64();
@@ -448,7 +450,6 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
   uint32_t* packs = reinterpret_cast<uint32_t*>(smem + SL.pack);
 #pragma unroll 1
   for (int i = tid; i < CW * 32; i += NT) packs[i] = P.pack[i];
-  uint16_t* klut = reinterpret_cast<uint16_t*>(smem + SL.klut);  // meta byte -> stream key
 #pragma unroll 1
   for (int b = tid; b < 256; b += NT) {
     const int m = b & 63;
@@ -457,20 +458,9 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
   }
   c.T.bind(tabw, P.tl);
   c.pack = packs;
-  c.hist = reinterpret_cast<uint32_t*>(smem + SL.hist);
-  c.s_cnt = reinterpret_cast<int*>(smem + SL.s_cnt);
-  c.s_run = reinterpret_cast<int*>(smem + SL.s_run);
-  c.s_base = reinterpret_cast<int*>(smem + SL.s_base);
-  c.s_tot = reinterpret_cast<int*>(smem + SL.s_tot);
-  c.s_skip = reinterpret_cast<int*>(smem + SL.s_skip);
-  c.s_pend = reinterpret_cast<int*>(smem + SL.s_pend);
-  uint8_t* gu8 = smem + SL.g_u8;
-  c.g_geom = gu8; c.g_target = gu8 + N; c.g_ctr = gu8 + 2 * N; c.g_vm = gu8 + 3 * N;
-  c.g_bill = gu8 + 4 * N; c.g_dec = gu8 + 5 * N; c.g_best = gu8 + 6 * N; c.g_want = gu8 + 7 * N;
-  int64_t* gi = reinterpret_cast<int64_t*>(smem + SL.g_i64);
-  c.g_rs = gi; c.g_re = gi + N; c.g_from = gi + 2 * N; c.g_until = gi + 3 * N;
-  c.g_since = gi + 4 * N; c.g_maxend = gi + 5 * N; c.g_kbest = gi + 6 * N; c.g_kcur = gi + 7 * N;
-  c.g_od = gi + 8 * N; c.g_spot = gi + 9 * N; c.g_busy = gi + 10 * N; c.g_mem = gi + 11 * N;
+  c.N = N;
+  c.gu8 = smem + SL.g_u8;
+  c.gi = reinterpret_cast<int64_t*>(smem + SL.g_i64);
   c.g_cnt = reinterpret_cast<int*>(smem + SL.g_i32);
   c.g_off = c.g_cnt + N;
   c.a_n = reinterpret_cast<int*>(smem + SL.a_n);
@@ -519,20 +509,18 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
 
     // ---------------------------------------------------------------- replica init
 #pragma unroll 1
-    for (int i = tid; i < kNB; i += NT) c.hist[i] = 0;          // kNB words = 2*3328 halves
+    for (int i = tid; i < 2 * kNB; i += NT) s_hist[i] = 0;
 #pragma unroll 1
-    for (int i = tid; i < 2 * kNB; i += NT) ghist[i] = 0;
-#pragma unroll 1
-    for (int k = tid; k < S; k += NT) c.s_skip[k] = 0;
+    for (int k = tid; k < S; k += NT) s_skip[k] = 0;
 #pragma unroll 1
     for (int g = tid; g < N; g += NT) {
       reset_gpu_state(c, g, P.init_geom);
-      c.g_vm[g] = c.g_bill[g] = (P.vm_policy == 0) ? VM_OD : VM_SPOT;
-      c.g_rs[g] = c.g_re[g] = 0;
-      c.g_from[g] = 0;
-      c.g_until[g] = kForever;
-      c.g_since[g] = 0;
-      c.g_od[g] = c.g_spot[g] = c.g_busy[g] = c.g_mem[g] = 0;
+      c.gu8[3 * c.N + g] = c.gu8[4 * c.N + g] = (P.vm_policy == 0) ? VM_OD : VM_SPOT;
+      c.gi[0 * c.N + g] = c.gi[1 * c.N + g] = 0;
+      c.gi[2 * c.N + g] = 0;
+      c.gi[3 * c.N + g] = kForever;
+      c.gi[4 * c.N + g] = 0;
+      c.gi[8 * c.N + g] = c.gi[9 * c.N + g] = c.gi[10 * c.N + g] = c.gi[11 * c.N + g] = 0;
     }
     if (tid == 0) {
       cs.w_lo = r_lo;
@@ -549,7 +537,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       const int64_t eW = e * P.W, Tend = eW + P.W;
       // ---------------------------------------------------------------- A: VM events, installs
 #pragma unroll 1
-      for (int i = tid; i < NW * S; i += NT) c.s_cnt[i] = 0;
+      for (int i = tid; i < NW * S; i += NT) s_cnt[i] = 0;
 #pragma unroll 1
       for (int g = tid; g < N; g += NT) {
         if (P.vm_policy != 0) {
@@ -557,15 +545,15 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           for (int64_t k = (eW + P.rev - 1) / P.rev; k * P.rev < Tend; ++k) {
             const int64_t tau = k * P.rev;
             if (k < 1 || tau >= P.H) continue;
-            if (c.g_target[g] != kNoGeom && c.g_re[g] <= tau) reset_gpu_state(c, g, c.g_target[g]);
+            if (c.gu8[1 * c.N + g] != kNoGeom && c.gi[1 * c.N + g] <= tau) reset_gpu_state(c, g, c.gu8[1 * c.N + g]);
             vm_event(P, c, replica, g, k, tau);
           }
         }
-        if (c.g_target[g] != kNoGeom && c.g_re[g] <= Tend) reset_gpu_state(c, g, c.g_target[g]);
-        c.g_dec[g] = (has_vm(c, g, Tend) && c.g_re[g] <= Tend) ? 1 : 0;
-        c.g_want[g] = 0;
-        c.g_best[g] = kNoGeom;
-        c.g_kcur[g] = -1;
+        if (c.gu8[1 * c.N + g] != kNoGeom && c.gi[1 * c.N + g] <= Tend) reset_gpu_state(c, g, c.gu8[1 * c.N + g]);
+        c.gu8[5 * c.N + g] = (has_vm(c, g, Tend) && c.gi[1 * c.N + g] <= Tend) ? 1 : 0;
+        c.gu8[7 * c.N + g] = 0;
+        c.gu8[6 * c.N + g] = kNoGeom;
+        c.gi[7 * c.N + g] = -1;
       }
       if (tid == 0) {
         cs.task = 0;
@@ -586,8 +574,8 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       PH(0);
 #pragma unroll 1
       for (int g = tid; g < N; g += NT) {
-        const bool whole = c.g_from[g] <= eW && c.g_until[g] >= Tend &&
-                           !(c.g_rs[g] < Tend && c.g_re[g] > eW);
+        const bool whole = c.gi[2 * c.N + g] <= eW && c.gi[3 * c.N + g] >= Tend &&
+                           !(c.gi[0 * c.N + g] < Tend && c.gi[1 * c.N + g] > eW);
         if (!whole) cs.all_avail = 0;
       }
       const int64_t len64 = w_end - w_lo;
@@ -604,7 +592,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       // flight per lane, validating every request once (when it is new).
       const int sa_lo = (int)((int64_t)len * warp / NW), sa_hi = (int)((int64_t)len * (warp + 1) / NW);
       {
-        int* cntw = c.s_cnt + warp * S;
+        int* cntw = s_cnt + warp * S;
         const int h = min(sa_hi, sa_lo + (int)((16u - ((uint32_t)(uintptr_t)(wmeta + sa_lo) & 15u)) & 15u));
         {  // unaligned head (< 16 elements)
           const int i = sa_lo + lane;
@@ -620,11 +608,14 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           const bool valid = ch < nch;
           const uint4 v = valid ? gv[ch] : make_uint4(0u, 0u, 0u, 0u);
           const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
+          int keys[16];
+#pragma unroll
+          for (int q = 0; q < 16; ++q)
+            keys[q] = valid ? (klut[(w4[q >> 2] >> (8 * (q & 3))) & 0xFF] & 0x7FFF) : 1024 + lane;
 #pragma unroll
           for (int q = 0; q < 16; ++q) {
-            const int key = valid ? (klut[(w4[q >> 2] >> (8 * (q & 3))) & 0xFF] & 0x7FFF) : 1024 + lane;
-            const unsigned peers = __match_any_sync(0xffffffffu, key);
-            if (key < 1024 && (peers & ((1u << lane) - 1u)) == 0) cntw[key] += __popc(peers);
+            const unsigned peers = __match_any_sync(0xffffffffu, keys[q]);
+            if (keys[q] < 1024 && (peers & ((1u << lane) - 1u)) == 0) atomicAdd(&cntw[keys[q]], __popc(peers));
           }
         }
         {  // tail (< 16 elements)
@@ -637,7 +628,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       __syncthreads();
       PH(1);
       {  // this warp's write offsets: base_k (exclusive scan of stream totals) + earlier segments
-        int* runw = c.s_run + warp * S;
+        int* runw = s_run + warp * S;
         int carry = 0;
 #pragma unroll 1
         for (int k0 = 0; k0 < S; k0 += 32) {
@@ -646,7 +637,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           if (k < S) {
 #pragma unroll 1
             for (int w = 0; w < NW; ++w) {
-              const int cv = c.s_cnt[w * S + k];
+              const int cv = s_cnt[w * S + k];
               if (w < warp) part += cv;
               tot += cv;
             }
@@ -661,8 +652,8 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           if (k < S) {
             runw[k] = base + part;
             if (warp == 0) {
-              c.s_base[k] = base;
-              c.s_tot[k] = tot;
+              s_base[k] = base;
+              s_tot[k] = tot;
             }
           }
           carry += __shfl_sync(0xffffffffu, x, 31);
@@ -714,8 +705,8 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
         const bool strict = (k & 1) == 0;
         const int B = T.bsz[m];
         const int64_t Tm = T.tmo[m];
-        int i = c.s_base[k] + c.s_skip[k];
-        const int end = c.s_base[k] + c.s_tot[k];
+        int i = s_base[k] + s_skip[k];
+        const int end = s_base[k] + s_tot[k];
         int pend = 0;
         uint32_t a0p = 0xFFFFFFFFu;
 #pragma unroll 1
@@ -782,7 +773,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           i = j;
         }
         if (lane == 0) {
-          c.s_pend[k] = pend;
+          s_pend[k] = pend;
           if (pend) atomicMin(&cs.amin, a0p);
         }
       }
@@ -806,7 +797,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
 #pragma unroll 1
       for (int k = tid; k < S; k += NT) {
         if (bad_window) break;
-        const int b0 = c.s_base[k], tot = c.s_tot[k];
+        const int b0 = s_base[k], tot = s_tot[k];
         int lo = 0, hi = tot;
 #pragma unroll 1
         while (lo < hi) {
@@ -814,7 +805,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           if (sarr[b0 + mid] >= amin) hi = mid; else lo = mid + 1;
         }
         if (lo) atomicAdd(reinterpret_cast<unsigned long long*>(&cs.lt_total), (unsigned long long)lo);
-        c.s_skip[k] = tot - lo - c.s_pend[k];
+        s_skip[k] = tot - lo - s_pend[k];
       }
       Bat* bats = c.bats;
       uint32_t* ord = c.ord;
@@ -859,7 +850,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       } else if (N <= 32) {
         if (warp == 0) {  // lanes = simulated GPUs; availability masks + cursor chase
           int64_t fr = 0, un = 0, rs = 0, re = 0;
-          if (lane < N) { fr = c.g_from[lane]; un = c.g_until[lane]; rs = c.g_rs[lane]; re = c.g_re[lane]; }
+          if (lane < N) { fr = c.gi[2 * c.N + lane]; un = c.gi[3 * c.N + lane]; rs = c.gi[0 * c.N + lane]; re = c.gi[1 * c.N + lane]; }
           int cur = cs.cursor, mycnt = 0;
 #pragma unroll 1
           for (int rk = 0; rk < nb; ++rk) {
@@ -1013,7 +1004,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
               if (head) {
                 const unsigned after = heads & ~((2u << lane) - 1u);
                 const int stop = after ? __ffs(after) - 1 : 32 - __clz(vmask);
-                hist_add(c, ghist, cls + bk, (uint32_t)(stop - lane));
+                atomicAdd(&s_hist[cls + bk], (uint32_t)(stop - lane));
               }
               if (lane == 0) {
                 if (strict) {
@@ -1037,7 +1028,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           Z = kZA;
           gbase = lane & ~7;
           valid = g < N;
-          j = valid ? c.g_geom[g] : 0;
+          j = valid ? c.gu8[0 * c.N + g] : 0;
         } else {
           const int cu = u - n_aunits, w = cu % CW;
           g = cu / CW;
@@ -1048,7 +1039,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           gbase = pk >> 24;
           valid = jr != 0xFF;
           j = valid ? jr : 0;
-          if (!c.g_dec[g]) {  // undecidable at T: no candidates scored (O5.4)
+          if (!c.gu8[5 * c.N + g]) {  // undecidable at T: no candidates scored (O5.4)
             if (valid && lane == gbase) {
               c.keys[g * Gc + (j - P.geom_lo)] = -1;
               if (P.cand_keys) P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = -1;
@@ -1090,8 +1081,8 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           candidate_unit_regs(T, K, active, lane == gbase && valid, bats, gl, c.g_off[g],
                               c.g_off[g + 1], sarr, P.max_live, &misses, &tail);
           if (valid && lane == gbase) {
-            const int64_t key = make_key(misses, tail, j == c.g_geom[g] ? 0 : j + 1);
-            if (j == c.g_geom[g]) c.g_kcur[g] = key;
+            const int64_t key = make_key(misses, tail, j == c.gu8[0 * c.N + g] ? 0 : j + 1);
+            if (j == c.gu8[0 * c.N + g]) c.gi[7 * c.N + g] = key;
             c.keys[g * Gc + (j - P.geom_lo)] = key;
             if (P.cand_keys) P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = key;
           }
@@ -1162,9 +1153,9 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           }
           const int64_t bsum = group_sum(acc0, 8), msum = group_sum(acc1, 8);
           if (valid && s == 0) {
-            c.g_maxend[g] = mx;
-            c.g_busy[g] += bsum;
-            c.g_mem[g] += msum;
+            c.gi[5 * c.N + g] = mx;
+            c.gi[10 * c.N + g] += bsum;
+            c.gi[11 * c.N + g] += msum;
           }
           __syncwarp();
           if (lane == 0) {
@@ -1172,8 +1163,8 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
             atomicAdd(&cs.adone, 1);
           }
         } else if (valid && lane == gbase) {
-          const int64_t key = make_key(acc0, acc1, j == c.g_geom[g] ? 0 : j + 1);
-          if (j == c.g_geom[g]) c.g_kcur[g] = key;
+          const int64_t key = make_key(acc0, acc1, j == c.gu8[0 * c.N + g] ? 0 : j + 1);
+          if (j == c.gu8[0 * c.N + g]) c.gi[7 * c.N + g] = key;
           c.keys[g * Gc + (j - P.geom_lo)] = key;
           if (P.cand_keys) P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = key;
         }
@@ -1184,21 +1175,21 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
 #pragma unroll 1
       for (int g = tid; g < N; g += NT) {
         uint8_t dec_out = kNoGeom;
-        if (P.policy == 0 && c.g_dec[g]) {
+        if (P.policy == 0 && c.gu8[5 * c.N + g]) {
           int64_t kb = c.keys[g * Gc];
 #pragma unroll 1
           for (int v = 1; v < Gc; ++v) kb = c.keys[g * Gc + v] < kb ? c.keys[g * Gc + v] : kb;
-          const int cur = c.g_geom[g];
+          const int cur = c.gu8[0 * c.N + g];
           const int tag = (int)(kb & 255);
           const int best = tag == 0 ? cur : tag - 1;
           dec_out = (uint8_t)best;
-          c.g_best[g] = (uint8_t)best;
-          c.g_kbest[g] = kb;
+          c.gu8[6 * c.N + g] = (uint8_t)best;
+          c.gi[6 * c.N + g] = kb;
           if (best != cur) {
-            if (c.g_ctr[g] >= P.wait_limit) c.g_want[g] = 1;
-            else c.g_ctr[g]++;
+            if (c.gu8[2 * c.N + g] >= P.wait_limit) c.gu8[7 * c.N + g] = 1;
+            else c.gu8[2 * c.N + g]++;
           } else {
-            c.g_ctr[g] = 0;
+            c.gu8[2 * c.N + g] = 0;
           }
           cnt[8] += (int64_t)(c.g_off[g + 1] - c.g_off[g]) * sum_slots;
           cnt[9] += Gc;
@@ -1218,7 +1209,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
 #pragma unroll 1
           for (int g = 0; g < N; ++g) {
             alive += has_vm(c, g, Tend) ? 1 : 0;
-            open += c.g_re[g] > Tend ? 1 : 0;
+            open += c.gi[1 * c.N + g] > Tend ? 1 : 0;
           }
           int cap = P.cap_pct * alive / 100;
           if (cap < 1) cap = 1;
@@ -1229,16 +1220,16 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
             int64_t pd = 0;
 #pragma unroll 1
             for (int g = 0; g < N; ++g) {
-              if (!c.g_want[g]) continue;
-              const int64_t d = (c.g_kcur[g] >> 40) - (c.g_kbest[g] >> 40);
+              if (!c.gu8[7 * c.N + g]) continue;
+              const int64_t d = (c.gi[7 * c.N + g] >> 40) - (c.gi[6 * c.N + g] >> 40);
               if (pick < 0 || d > pd) { pick = g; pd = d; }
             }
             if (pick < 0) break;
-            c.g_want[pick] = 0;
-            const int64_t drain_end = c.g_maxend[pick] > Tend ? c.g_maxend[pick] : Tend;
-            c.g_rs[pick] = Tend;
-            c.g_re[pick] = drain_end + P.reconfig_us;
-            c.g_target[pick] = c.g_best[pick];
+            c.gu8[7 * c.N + pick] = 0;
+            const int64_t drain_end = c.gi[5 * c.N + pick] > Tend ? c.gi[5 * c.N + pick] : Tend;
+            c.gi[0 * c.N + pick] = Tend;
+            c.gi[1 * c.N + pick] = drain_end + P.reconfig_us;
+            c.gu8[1 * c.N + pick] = c.gu8[6 * c.N + pick];
             cnt[7] += 1;
             --free_slots;
           }
@@ -1256,11 +1247,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
     for (int i = 0; i < 10; ++i)
       if (cnt[i]) atomicAdd(&cs.cnt[i], (unsigned long long)cnt[i]);
 #pragma unroll 1
-    for (int w = tid; w < kNB; w += NT) {  // fold the packed smem halves into the HBM histogram
-      const uint32_t v = c.hist[w];
-      if (v & 0xFFFFu) atomicAdd(&ghist[2 * w], v & 0xFFFFu);
-      if (v >> 16) atomicAdd(&ghist[2 * w + 1], v >> 16);
-    }
+    for (int w = tid; w < 2 * kNB; w += NT) ghist[w] = s_hist[w];  // histogram to HBM
     __syncthreads();
     if (warp < 2) {  // nearest-rank P50 / P99 per class
       const uint32_t* h = ghist + warp * kNB;
@@ -1300,10 +1287,10 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       int64_t od = 0, spot = 0, busy = 0, memt = 0;
 #pragma unroll 1
       for (int g = 0; g < N; ++g) {
-        od += c.g_od[g];
-        spot += c.g_spot[g];
-        busy += c.g_busy[g];
-        memt += c.g_mem[g];
+        od += c.gi[8 * c.N + g];
+        spot += c.gi[9 * c.N + g];
+        busy += c.gi[10 * c.N + g];
+        memt += c.gi[11 * c.N + g];
       }
 #pragma unroll 1
       for (int i = 0; i < 10; ++i) P.counters[(size_t)r * 10 + i] = (int64_t)cs.cnt[i];

@@ -9,6 +9,7 @@ namespace pemgpu {
 
 constexpr int kNSeg = 8;          // max warps per CTA (stream-partition segments)
 constexpr int kZA = 8;            // lanes per actual-placement group (one per slice position)
+constexpr int kMaxStreams = 2 * PROTEAN_MAX_MODELS;
 constexpr int64_t kForever = INT64_MAX;
 
 // One batch of the current epoch (40 B).  info = n | model << 16 | strict << 24.
@@ -28,7 +29,7 @@ struct SmemLayout {
   int S;            // streams = 2 * M
   int N, Gc, CW;    // simulated GPUs, candidate geometries in range, candidate warps per GPU
   int BS, WS;       // batches / window entries held in smem
-  size_t tab, pack, klut, hist, s_cnt, s_run, s_base, s_tot, s_skip, s_pend;
+  size_t tab, pack;
   size_t g_u8, g_i64, g_i32, a_n, a_ls, a_bu, keys, bats, ord, glist, sarr, total;
   __host__ void init(int words, int M, int n_gpus, int gc, int cw, int bs, int ws) {
     S = 2 * M; N = n_gpus; Gc = gc; CW = cw; BS = bs; WS = ws;
@@ -36,14 +37,6 @@ struct SmemLayout {
     auto take = [&](size_t bytes) { size_t r = o; o += (bytes + 15) & ~(size_t)15; return r; };
     tab = take((size_t)words * 4);
     pack = take((size_t)CW * 32 * 4);
-    klut = take(256 * 2);
-    hist = take((size_t)kNB * 4);               // 2 classes x 3328 buckets as packed u16 pairs
-    s_cnt = take((size_t)kNSeg * S * 4);
-    s_run = take((size_t)kNSeg * S * 4);
-    s_base = take((size_t)S * 4);
-    s_tot = take((size_t)S * 4);
-    s_skip = take((size_t)S * 4);
-    s_pend = take((size_t)S * 4);
     g_u8 = take((size_t)N * 8);                 // geom, target, ctr, vm, bill, dec, best, want
     g_i64 = take((size_t)N * 12 * 8);           // rs, re, from, until, since, maxend, kbest, kcur, od, spot, busy, mem
     g_i32 = take((size_t)(2 * N + 2) * 4);      // gcnt[N], goff[N+1]

@@ -22,4 +22,11 @@ h = pkg.load_profiles(synth_profiles())
 for _ in range(a.repeat):
     out = h.replay_traces(arr, meta, roff, trace_len_us=gp.trace_len_us, n_gpus=8)
 torch.cuda.synchronize()
-print("requests", arr.shape[0], "timings", h.last_timings(), "slot_evals", int(out["counters"][:, 8].sum()))
+import json
+c = out["counters"].sum(0).cpu().tolist()
+info = {"replicas": a.replicas, "seconds": a.seconds, "requests": int(arr.shape[0]),
+        "slot_evals": int(c[8]), "geom_candidates": int(c[9]), "timings": h.last_timings()[:2],
+        "launch": h.last_timings()[2]}
+print(json.dumps(info))
+os.makedirs("gpurun_out", exist_ok=True)
+json.dump(info, open("gpurun_out/profile_run_info.json", "w"))
