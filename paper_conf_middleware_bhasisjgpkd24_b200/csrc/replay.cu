@@ -162,17 +162,6 @@ __device__ __forceinline__ void prefetch_l2(const void* p, int64_t bytes) {
   }
 }
 
-// Packed u16 smem histogram; a half crossing 2^15 moves 2^15 counts to the HBM histogram
-// (cnt <= 32 per call, so a half never exceeds 0xFFFF before the move).
-__device__ __forceinline__ void hist_add(uint32_t* hist, uint32_t* ghist, int idx, uint32_t cnt) {
-  const int w = idx >> 1, sh = (idx & 1) * 16;
-  const uint32_t old = (atomicAdd(&hist[w], cnt << sh) >> sh) & 0xFFFFu;
-  if (old < 0x8000u && old + cnt >= 0x8000u) {
-    atomicSub(&hist[w], 0x8000u << sh);
-    atomicAdd(&ghist[idx], 0x8000u);
-  }
-}
-
 __device__ __forceinline__ int hits_in(const uint32_t* a, int n, int64_t end, int64_t slo) {
   const int64_t need = end - slo;  // c - a <= slo  <=>  a >= c - slo
   int lo = 0, hi = n;
@@ -348,8 +337,10 @@ __device__ __forceinline__ void candidate_unit_regs(const Tab& T, const SliceLan
     const int64_t t0 = t > ls ? t : ls;
     int32_t used = 0, be = 0, live = 0;
     int64_t fs = 0;
+    const int nw = __reduce_max_sync(0xffffffffu, (unsigned)n);  // warp-uniform loop bound
 #pragma unroll
     for (int i = 0; i < kKR; ++i) {
+      if (i >= nw) break;
       if (i < n && en_r[i] > t) {
         const int32_t mem = mm_r[i] & 0xFFFF;
         ++live;
@@ -375,17 +366,22 @@ __device__ __forceinline__ void candidate_unit_regs(const Tab& T, const SliceLan
         start = INT64_MAX;
 #pragma unroll
         for (int jj = 0; jj < kKR; ++jj) {
-          if (jj < n && en_r[jj] > t0) {
+          if (jj >= n) break;
+          if (en_r[jj] > t0) {
             int32_t rem = 0;
 #pragma unroll
-            for (int i = 0; i < kKR; ++i)
-              if (i < n && en_r[i] > en_r[jj]) rem += mm_r[i] & 0xFFFF;
+            for (int i = 0; i < kKR; ++i) {
+              if (i >= n) break;
+              if (en_r[i] > en_r[jj]) rem += mm_r[i] & 0xFFFF;
+            }
             if (rem + q <= K.Ms && en_r[jj] < start) start = en_r[jj];
           }
         }
 #pragma unroll
-        for (int i = 0; i < kKR; ++i)
-          if (i < n && en_r[i] > start) F += K.fbr_p[((mm_r[i] >> 16) & 63) * kNProf];
+        for (int i = 0; i < kKR; ++i) {
+          if (i >= n) break;
+          if (en_r[i] > start) F += K.fbr_p[((mm_r[i] >> 16) & 63) * kNProf];
+        }
       }
       c = start + exec_time(K.solo_p[m * kNProf], F);
       if (strict) {
@@ -686,10 +682,10 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
             const int key = valid ? (kv & 0x7FFF) : 1024 + lane;
             const unsigned peers = __match_any_sync(0xffffffffu, key);
             const unsigned rank = __popc(peers & ((1u << lane) - 1u));
-            if (valid) sa[runw[key] + (int)rank] = ai[u];
-            __syncwarp();
-            if (valid && rank == 0) runw[key] += __popc(peers);
-            __syncwarp();
+            int base = 0;  // the group leader reserves the group's run of slots in stream order
+            if (valid && rank == 0) base = atomicAdd(&runw[key], __popc(peers));
+            base = __shfl_sync(0xffffffffu, base, __ffs(peers) - 1);
+            if (valid) sa[base + (int)rank] = ai[u];
           }
         }
       }
@@ -848,28 +844,52 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
         }
         if (tid == 0) cs.cursor = (int)((cursor + nb) % N);
       } else if (N <= 32) {
-        if (warp == 0) {  // lanes = simulated GPUs; availability masks + cursor chase
-          int64_t fr = 0, un = 0, rs = 0, re = 0;
-          if (lane < N) { fr = c.gi[2 * c.N + lane]; un = c.gi[3 * c.N + lane]; rs = c.gi[0 * c.N + lane]; re = c.gi[1 * c.N + lane]; }
-          int cur = cs.cursor, mycnt = 0;
+        // availability mask per batch (parallel); then runs of equal masks are dispatched in
+        // closed form: inside a run the k-th batch goes to the (i0 + k) mod |A|-th available GPU
 #pragma unroll 1
-          for (int rk = 0; rk < nb; ++rk) {
-            Bat& bt = bats[ord[rk]];
-            const int64_t t = bt.ready;
-            const bool av = lane < N && fr <= t && t < un && !(rs <= t && t < re);
-            const unsigned am = __ballot_sync(0xffffffffu, av);
-            int chosen = -1;
-            if (am) {
-              const unsigned hi = am & ~((1u << cur) - 1u);
-              chosen = hi ? __ffs(hi) - 1 : __ffs(am) - 1;
-              cur = (chosen + 1) % N;
-              if (lane == chosen) ++mycnt;
+        for (int rk = tid; rk < nb; rk += NT) {
+          Bat& bt = bats[ord[rk]];
+          const int64_t t = bt.ready;
+          uint32_t m = 0;
+#pragma unroll 1
+          for (int g = 0; g < N; ++g)
+            if (available(c, g, t)) m |= 1u << g;
+          bt.key = m;  // the id-order key is no longer needed
+        }
+        __syncthreads();
+        if (warp == 0) {
+          int cur = cs.cursor;
+#pragma unroll 1
+          for (int r0 = 0; r0 < nb;) {
+            const uint32_t m = (uint32_t)bats[ord[r0]].key;
+            int r1 = r0 + 1;
+#pragma unroll 1
+            for (;;) {  // end of the run of equal masks
+              const int rk = r1 + lane;
+              const unsigned dm = __ballot_sync(0xffffffffu, rk >= nb || (uint32_t)bats[ord[rk]].key != m);
+              if (dm) { r1 += __ffs(dm) - 1; break; }
+              r1 += 32;
             }
-            if (lane == 0) {
-              bt.gpu = chosen < 0 ? (uint8_t)0xFF : (uint8_t)chosen;
-              if (chosen < 0) bt.drop = 1;  // dispatch drop
+            const int A = __popc(m);
+            const int i0 = A ? __popc(m & ((1u << cur) - 1u)) % A : 0;  // first available >= cur
+#pragma unroll 1
+            for (int rk = r0 + lane; rk < r1; rk += 32) {
+              Bat& bt = bats[ord[rk]];
+              if (A == 0) {
+                bt.gpu = 0xFF;
+                bt.drop = 1;  // dispatch drop
+              } else {
+                bt.gpu = (uint8_t)__fns(m, 0, (i0 + (rk - r0)) % A + 1);
+              }
             }
+            if (A) cur = ((int)__fns(m, 0, (i0 + (r1 - 1 - r0)) % A + 1) + 1) % N;
+            r0 = r1;
           }
+          __syncwarp();
+          // lanes = GPUs: per-GPU counts, offsets, and the id-ordered per-GPU lists
+          int mycnt = 0;
+#pragma unroll 1
+          for (int rk = 0; rk < nb; ++rk) mycnt += (bats[ord[rk]].gpu == lane) ? 1 : 0;
           int x = mycnt;
 #pragma unroll
           for (int d = 1; d < 32; d <<= 1) {
@@ -883,8 +903,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
 #pragma unroll 1
           for (int rk = 0; rk < nb; ++rk) {
             const uint32_t b = ord[rk];
-            const int g = bats[b].gpu;
-            if (lane == g) gl[c.g_off[lane] + fill++] = b;
+            if (bats[b].gpu == lane) gl[c.g_off[lane] + fill++] = b;
           }
           if (lane == 0) cs.cursor = cur;
         }
