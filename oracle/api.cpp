@@ -321,7 +321,7 @@ int orc_replay(const orc_tables* t, const orc_replay_in* in, orc_replay_out* out
         std::copy(ro.decisions.begin(), ro.decisions.end(), out->decisions + (int64_t)r * E * N);
       if (out->cand_keys)
         std::copy(ro.cand_keys.begin(), ro.cand_keys.end(), out->cand_keys + (int64_t)r * E * N * G);
-      if (out->n_batches) out->n_batches[r] = (int64_t)ro.log.size();
+      if (out->n_batches) out->n_batches[r] = ro.n_batches;
       if (out->log) {
         for (size_t i = 0; i < ro.log.size() && (int64_t)i < out->log_cap; ++i) {
           const BatchRec& b = ro.log[i];

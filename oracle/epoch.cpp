@@ -301,6 +301,7 @@ void replay_replica(const Tables& tb, const ReplayCfg& cfg, uint64_t replica_id,
   std::vector<Batch> batches = form_batches(tb, arrival, meta, n);
   Replay rp(tb, cfg, replica_id, E * cfg.W, out);
   rp.run(batches, E, want_keys, want_log);
+  out->n_batches = (int64_t)batches.size();
 }
 
 }  // namespace pem

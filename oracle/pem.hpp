@@ -126,6 +126,7 @@ struct ReplayOut {
   std::vector<uint8_t> decisions;       // [E][N]
   std::vector<int64_t> cand_keys;       // [E][N][G]
   std::vector<BatchRec> log;
+  int64_t n_batches = 0;
 };
 int64_t num_epochs(const Tables& tb, int64_t trace_len, int64_t W);
 void replay_replica(const Tables& tb, const ReplayCfg& cfg, uint64_t replica_id,
