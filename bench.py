@@ -310,7 +310,7 @@ def run_ours(args):
                          "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
                          "kernel": "replay_kernel", "kernel_ms": k_ms, "prepass_ms": statistics.mean(pre_ms),
                          "launch": launch},
-            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": 2 * args.steps * world, "clocks": clocks,
+            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": 3 * args.steps * world, "clocks": clocks,
         }
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -48,7 +48,7 @@ enum {
                            n_gpus > 255, G > 254, live residents > max_live in a given state */
   PROTEAN_ENOMEM = -3,  /* device / host allocation failed */
   PROTEAN_ECUDA = -4,   /* a CUDA runtime call failed (handle poisoned) */
-  PROTEAN_ENCCL = -5,   /* an NCCL call failed (handle poisoned) */
+  PROTEAN_ENCCL = -5,   /* a cross-rank exchange failed or timed out (handle poisoned) */
   PROTEAN_ESTATE = -6,  /* handle poisoned, or bad call order */
   PROTEAN_EUNSUP = -7   /* valid request this build does not implement (e.g. policy = Alg 2) */
 };
@@ -207,9 +207,11 @@ typedef struct {
   int64_t rev_interval_us;     /* revocation interval T_rev (default 300 s, Q28); must be >= W */
   int64_t notice_us;           /* eviction notice (default 30 s); must be < T_rev */
   uint64_t seed;               /* VM RNG seed (O11) */
-  int32_t shard_mode;          /* 0 = replicas (mode R); 1 = geometry ranges (mode G, EUNSUP here) */
-  int32_t rank, nranks;        /* mode G only */
-  const uint8_t *nccl_id;      /* mode G only: host, 128-byte ncclUniqueId */
+  int32_t shard_mode;          /* 0 = replicas (mode R); 1 = geometry ranges (mode G, section 4) */
+  int32_t rank, nranks;        /* mode G only: must match the handle's exchange set-up */
+  int32_t max_ctas;            /* 0 = the resident capacity of the device; else caps the replay
+                                  grid (lets several mode-G ranks share one GPU) */
+  int32_t reserved;            /* must be 0 */
 } protean_replay_cfg;
 
 /* counters[10] per replica (O7/O8/O10):
@@ -247,13 +249,58 @@ int protean_replay_traces(protean_handle *h, const protean_replay_cfg *cfg,
                           protean_replay_out *out, void *stream);
 
 /* Device time (CUDA events on the launching stream) of the last protean_replay_traces call:
- * the prepass kernel and the fused replay kernel, in ms; launch = {grid, block, dynamic smem
+ * the prepass kernels (epoch offsets; per-epoch, per-segment stream counts) and the fused replay
+ * kernel, in ms; launch = {grid, block, dynamic smem
  * bytes, resident CTAs per SM} of the replay kernel (any pointer may be NULL).  Host. */
 int protean_last_timings(const protean_handle *h, float *prepass_ms, float *replay_ms,
                          int32_t *launch);
 
 /* Fill a replay config with the defaults listed above (host). */
 void protean_replay_cfg_defaults(protean_replay_cfg *cfg);
+
+/* ---------------------------------------------------------------------------------------------
+ * 4. Mode G: geometry-range sharding with one min-loc exchange per replica-epoch (SURVEY §8(e),
+ *    S8 "argmin over geometries + cross-rank min-loc"; the search is the Oracle's sweep).
+ *
+ * Rank k of n scores only geometries [bounds[k], bounds[k+1]) of protean_geometry_split and
+ * redundantly runs everything else (dispatch, actual placement, accounting, decisions), so no
+ * state is exchanged: per (replica, epoch, sim-GPU) each rank contributes its best key and the
+ * current geometry's key (INT64_MAX when not in its range), and every rank takes the min of each.
+ * The packed key (O8) makes min-loc a plain min, so every rank reaches the decision a 1-rank run
+ * reaches: decisions, histograms, counters 0..7 and accumulators are identical to mode R / one
+ * rank; counters 8 and 9 count the rank's own candidates (their sum over ranks is the 1-rank
+ * value) and cand_keys is written for the rank's range only.
+ *
+ * The exchange is fused into the replay kernel (no host round trip, no NCCL launch per epoch):
+ * every CTA stores its 16-byte (best, current) pairs straight into every rank's exchange buffer
+ * (peer stores over NVLink through CUDA IPC mappings), publishes a per-(source rank, replica)
+ * sequence number with release semantics at system scope, and reduces after acquiring every
+ * source's flag.  Keys are double-buffered by sequence parity; sequence numbers continue across
+ * calls, so all ranks must issue the same sequence of mode-G replay calls (same R, N and E), and
+ * the kernels of one call must run concurrently (one GPU per rank, or grids that fit together on
+ * one GPU: cfg.max_ctas; ranks sharing a process must use non-default streams, since the legacy
+ * default stream serialises; the library grows its scratch with the stream-ordered allocator and
+ * sets kernel attributes once, so it adds no implicit device-wide synchronisation itself).  A source whose flag does not arrive within 30 s makes the call return
+ * PROTEAN_ENCCL (the handle is poisoned).                                                        */
+
+/* Balanced geometry ranges: bounds[0] = 0, bounds[nranks] = G, every range non-empty, cut where
+ * the running slice count first reaches k/nranks of the total (slot-balanced; host only, no
+ * device needed).  EINVAL for nranks < 1 or nranks > G; geometry set as protean_load_profiles. */
+int protean_geometry_split(const protean_profiles *p, int32_t nranks, int32_t *bounds);
+
+/* Allocate (zeroed) this rank's exchange buffer for up to max_replicas replicas per call and
+ * max_gpus sim-GPUs, and write its 64-byte cudaIpcMemHandle_t to ipc_handle (host). */
+int protean_xchg_export(protean_handle *h, int32_t nranks, int32_t rank, int32_t max_replicas,
+                        int32_t max_gpus, void *ipc_handle);
+
+/* Map every rank's buffer: ipc_handles = [nranks][64] bytes gathered from every rank's
+ * protean_xchg_export (this rank's own entry is not opened).  Host; synchronous. */
+int protean_xchg_import(protean_handle *h, const void *ipc_handles);
+
+/* Single-process set-up: handles[k] is rank k (one handle per rank, any devices that can access
+ * each other's memory); allocates and cross-wires all buffers.  Host; synchronous. */
+int protean_xchg_attach(protean_handle *const *handles, int32_t nranks, int32_t max_replicas,
+                        int32_t max_gpus);
 
 #ifdef __cplusplus
 }

@@ -74,7 +74,7 @@ class ReplayCfg(C.Structure):
                 ("p_rev", C.c_double), ("price_od_node_hr", C.c_double), ("price_spot_node_hr", C.c_double),
                 ("rev_interval_us", C.c_int64), ("notice_us", C.c_int64), ("seed", C.c_uint64),
                 ("shard_mode", C.c_int32), ("rank", C.c_int32), ("nranks", C.c_int32),
-                ("nccl_id", C.c_void_p)]
+                ("max_ctas", C.c_int32), ("reserved", C.c_int32)]
 
 
 class BatchRec(C.Structure):     # protean_batch_rec, 32 B
@@ -95,7 +95,9 @@ assert C.sizeof(BatchRec) == 32
 
 EXPORTS = ["protean_load_profiles", "protean_free", "protean_strerror", "protean_last_error",
            "protean_get_geometries", "protean_num_epochs", "protean_score_epoch",
-           "protean_replay_traces", "protean_replay_cfg_defaults", "protean_last_timings"]
+           "protean_replay_traces", "protean_replay_cfg_defaults", "protean_last_timings",
+           "protean_geometry_split", "protean_xchg_export", "protean_xchg_import", "protean_xchg_attach"]
+IPC_HANDLE_BYTES = 64
 
 _lib = None
 
@@ -122,6 +124,10 @@ def load(path: str = LIB_PATH, require_cuda: bool = True):
     L.protean_replay_cfg_defaults.argtypes = [C.c_void_p]
     L.protean_replay_cfg_defaults.restype = None
     L.protean_last_timings.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
+    L.protean_geometry_split.argtypes = [C.c_void_p, C.c_int32, C.c_void_p]
+    L.protean_xchg_export.argtypes = [C.c_void_p, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_void_p]
+    L.protean_xchg_import.argtypes = [C.c_void_p, C.c_void_p]
+    L.protean_xchg_attach.argtypes = [C.c_void_p, C.c_int32, C.c_int32, C.c_int32]
     _lib = L
     return L
 

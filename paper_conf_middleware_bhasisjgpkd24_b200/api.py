@@ -14,7 +14,7 @@ _REPLAY_DEFAULTS = dict(n_gpus=8, epoch_len_us=1_000_000, policy=0, wait_limit=3
                         init_geom=2, max_live=64, vm_policy=0, reconfig_us=2_000_000, p_rev=0.0,
                         price_od_node_hr=32.7726 / 8, price_spot_node_hr=9.8318 / 8,
                         rev_interval_us=300_000_000, notice_us=30_000_000, seed=0, shard_mode=0,
-                        replica_base=0)
+                        rank=0, nranks=1, max_ctas=0, replica_base=0)
 
 
 def _torch():
@@ -30,26 +30,70 @@ def _check(h, rc):
         raise A.ProteanError(rc, detail)
 
 
+def _profiles_struct(profiles, device: int = 0):
+    """protean_profiles for `profiles` (+ the numpy arrays it points into, to keep alive)."""
+    arrs = [np.ascontiguousarray(x, np.int32) for x in
+            (profiles.solo_us, profiles.fbr_ppm, profiles.mem_mib, profiles.batch_size,
+             profiles.slo_us, profiles.timeout_us)]
+    geoms = None if profiles.geoms is None else np.ascontiguousarray(profiles.geoms, np.uint8)
+    p = A.Profiles(A.ABI_VERSION, int(arrs[0].shape[0]), *[a.ctypes.data for a in arrs],
+                   int(profiles.geometry_set), 0 if geoms is None else int(geoms.shape[0]),
+                   None if geoms is None else geoms.ctypes.data, int(device))
+    return p, (arrs, geoms)
+
+
+def geometry_split(profiles, nranks: int) -> list[int]:
+    """protean_geometry_split: slot-balanced geometry range bounds [nranks + 1] (host only)."""
+    lib = A.load(require_cuda=False)
+    p, keep = _profiles_struct(profiles)
+    b = (C.c_int32 * (nranks + 1))()
+    rc = lib.protean_geometry_split(C.byref(p), int(nranks), b)
+    if rc != A.OK:
+        raise A.ProteanError(rc, "protean_geometry_split")
+    del keep
+    return list(b)
+
+
 class Handle:
     """protean_load_profiles(): validated tables + geometry set resident on `device`."""
 
     def __init__(self, profiles, device: int = 0):
         self._lib = A.load()
         self.device = device
-        arrs = [np.ascontiguousarray(x, np.int32) for x in
-                (profiles.solo_us, profiles.fbr_ppm, profiles.mem_mib, profiles.batch_size,
-                 profiles.slo_us, profiles.timeout_us)]
-        geoms = None if profiles.geoms is None else np.ascontiguousarray(profiles.geoms, np.uint8)
-        p = A.Profiles(A.ABI_VERSION, int(arrs[0].shape[0]), *[a.ctypes.data for a in arrs],
-                       int(profiles.geometry_set), 0 if geoms is None else int(geoms.shape[0]),
-                       None if geoms is None else geoms.ctypes.data, int(device))
+        p, keep = _profiles_struct(profiles, device)
         self._h = C.c_void_p()
         rc = self._lib.protean_load_profiles(C.byref(p), C.byref(self._h))
         if rc != A.OK:
             raise A.ProteanError(rc, "protean_load_profiles")
+        del keep
         n = C.c_int32()
         self._lib.protean_get_geometries(self._h, C.byref(n), None)
         self.n_geoms = n.value
+
+    # ------------------------------------------------------------------ mode G exchange set-up
+    def xchg_export(self, nranks: int, rank: int, max_replicas: int, max_gpus: int) -> bytes:
+        """protean_xchg_export: allocate this rank's exchange buffer; returns its IPC handle."""
+        buf = (C.c_char * A.IPC_HANDLE_BYTES)()
+        _check(self._h, self._lib.protean_xchg_export(self._h, int(nranks), int(rank), int(max_replicas),
+                                                      int(max_gpus), buf))
+        return bytes(buf)
+
+    def xchg_import(self, handles: list[bytes]):
+        """protean_xchg_import: map every rank's buffer (handles in rank order)."""
+        blob = b"".join(handles)
+        assert len(blob) == A.IPC_HANDLE_BYTES * len(handles)
+        buf = (C.c_char * len(blob)).from_buffer_copy(blob)
+        _check(self._h, self._lib.protean_xchg_import(self._h, buf))
+
+    @staticmethod
+    def xchg_attach(handles: list["Handle"], max_replicas: int, max_gpus: int):
+        """protean_xchg_attach: every rank in this process, handles[k] = rank k."""
+        lib = A.load()
+        arr = (C.c_void_p * len(handles))(*[h._h.value for h in handles])
+        rc = lib.protean_xchg_attach(arr, len(handles), int(max_replicas), int(max_gpus))
+        if rc != A.OK:
+            raise A.ProteanError(rc, "protean_xchg_attach: "
+                                 + " | ".join(lib.protean_last_error(h._h).decode() for h in handles))
 
     def close(self):
         if getattr(self, "_h", None):
@@ -125,7 +169,8 @@ class Handle:
         cf.meta = meta.data_ptr() if meta.numel() else replica_off.data_ptr()
         cf.replica_off = replica_off.data_ptr()
         for k in ("policy", "wait_limit", "reconfig_cap_pct", "init_geom", "max_live", "vm_policy",
-                  "reconfig_us", "rev_interval_us", "notice_us", "seed", "shard_mode"):
+                  "reconfig_us", "rev_interval_us", "notice_us", "seed", "shard_mode", "rank", "nranks",
+                  "max_ctas"):
             setattr(cf, k, int(c[k]))
         for k in ("p_rev", "price_od_node_hr", "price_spot_node_hr"):
             setattr(cf, k, float(c[k]))

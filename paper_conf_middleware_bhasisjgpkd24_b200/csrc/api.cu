@@ -29,12 +29,27 @@ struct protean_handle {
   size_t scratch_bytes = 0;
   int64_t* d_eoff = nullptr;
   size_t eoff_bytes = 0;
+  void* d_ecnt = nullptr;
+  size_t ecnt_bytes = 0;
   void* d_small = nullptr;  // wmax (8 B) + err (16 B)
   uint32_t* d_pack = nullptr;  // candidate lane packing for the full geometry range
   int CW = 0;
   cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};  // prepass / replay kernel bracket
   float t_prepass = 0.f, t_replay = 0.f;
   int last_grid = 0, last_block = 0, last_smem = 0, last_per_sm = 0;
+  std::vector<int> gn;  // slice count per geometry
+  // mode G: candidate lane packing of the rank's geometry range
+  uint32_t* d_pack_g = nullptr;
+  int CW_g = 0, pack_lo = -1, pack_hi = -1;
+  // mode G exchange (protean_xchg_*)
+  XLayout xl{0, 0, 0};
+  int xrank = 0;
+  bool x_ready = false;
+  uint32_t xseq = 0;
+  void* d_xbuf = nullptr;                // this rank's buffer (owned)
+  std::vector<char*> xpeer;              // every rank's buffer in this process
+  std::vector<char> x_opened;            // 1 = opened through cudaIpcOpenMemHandle
+  char** d_xpeer = nullptr;              // device copy of xpeer
 };
 
 namespace {
@@ -125,21 +140,160 @@ int validate_row(const uint8_t* row, std::vector<uint8_t>* g) {
   return PROTEAN_OK;
 }
 
-int ensure(protean_handle* h, void** p, size_t* have, size_t need) {
+// Grow a scratch buffer with the stream-ordered allocator: cudaMalloc / cudaFree are implicit
+// device-wide synchronisation points, which would serialise (and, with the mode-G exchange,
+// stall) replay kernels that other handles of this process run concurrently.
+int ensure(protean_handle* h, void** p, size_t* have, size_t need, cudaStream_t st) {
   if (*have >= need && *p) return PROTEAN_OK;
-  if (*p) cudaFree(*p);
+  if (*p) cudaFreeAsync(*p, st);
   *p = nullptr;
   *have = 0;
-  cudaError_t e = cudaMalloc(p, need);
+  cudaError_t e = cudaMallocAsync(p, need, st);
   if (e != cudaSuccess) {
     cudaGetLastError();
-    return fail(h, PROTEAN_ENOMEM, "cudaMalloc scratch failed");
+    *p = nullptr;
+    return fail(h, PROTEAN_ENOMEM, "cudaMallocAsync scratch failed");
   }
   *have = need;
   return PROTEAN_OK;
 }
 
 size_t al(size_t x) { return (x + 255) & ~(size_t)255; }
+
+// Candidate lane packing of geometries [lo, hi): power-of-two lane groups (>= the slice count),
+// largest first, filled into 32-lane warps; entry = j | slice << 8 | Z << 16 | group base << 24.
+std::vector<uint32_t> build_pack(const std::vector<int>& gn, int lo, int hi, int* CW) {
+  std::vector<uint32_t> pack;
+  std::vector<std::pair<int, int>> order;  // (Z, j)
+  for (int j = lo; j < hi; ++j) {
+    int Z = 1;
+    while (Z < gn[j]) Z <<= 1;
+    order.push_back({Z, j});
+  }
+  std::stable_sort(order.begin(), order.end(),
+                   [](const std::pair<int, int>& a, const std::pair<int, int>& b) { return a.first > b.first; });
+  int fill = 32;
+  for (const auto& zj : order) {
+    const int Z = zj.first, j = zj.second;
+    if (fill + Z > 32) {
+      pack.insert(pack.end(), 32, 0xFFu);
+      fill = 0;
+    }
+    const size_t w0 = pack.size() - 32;
+    for (int s = 0; s < Z; ++s)
+      pack[w0 + fill + s] = (uint32_t)j | ((uint32_t)s << 8) | ((uint32_t)Z << 16) | ((uint32_t)fill << 24);
+    fill += Z;
+  }
+  *CW = (int)(pack.size() / 32);
+  return pack;
+}
+
+// Slot-balanced split of G geometries (slice counts gn) into nranks non-empty ranges: cut k sits
+// at the geometry boundary whose running slice count is nearest k/nranks of the total (ties to
+// the earlier boundary), kept strictly increasing.
+void split_ranges(const std::vector<int>& gn, int nranks, int32_t* b) {
+  const int G = (int)gn.size();
+  std::vector<int64_t> pre(G + 1, 0);
+  for (int j = 0; j < G; ++j) pre[j + 1] = pre[j] + gn[j];
+  const int64_t total = pre[G];
+  b[0] = 0;
+  for (int k = 1; k < nranks; ++k) {
+    int best = 0;
+    int64_t bd = -1;
+    for (int j = 0; j <= G; ++j) {
+      const int64_t d = std::llabs(pre[j] * nranks - (int64_t)k * total);
+      if (bd < 0 || d < bd) { bd = d; best = j; }
+    }
+    best = std::max(best, b[k - 1] + 1);
+    best = std::min(best, G - (nranks - k));
+    b[k] = best;
+  }
+  b[nranks] = G;
+}
+
+// Geometry lists of a profile set (protean_load_profiles' rules), host only.
+int profile_geometries(const protean_profiles* p, std::vector<std::vector<uint8_t>>* gs) {
+  if (!p || p->abi_version != PROTEAN_ABI_VERSION) return PROTEAN_EINVAL;
+  if (p->geometry_set == 0 || p->geometry_set == 1) {
+    *gs = geometry_set(p->geometry_set == 1);
+    return PROTEAN_OK;
+  }
+  if (p->geometry_set != 2) return PROTEAN_EINVAL;
+  if (p->n_geoms < 1) return PROTEAN_EINVAL;
+  if (p->n_geoms > 254) return PROTEAN_ERANGE;
+  if (!p->geoms) return PROTEAN_EINVAL;
+  for (int j = 0; j < p->n_geoms; ++j) {
+    std::vector<uint8_t> g;
+    int rc = validate_row(p->geoms + 8 * j, &g);
+    if (rc) return rc;
+    gs->push_back(g);
+  }
+  return PROTEAN_OK;
+}
+
+void xchg_release(protean_handle* h) {
+  for (size_t i = 0; i < h->xpeer.size(); ++i)
+    if (h->x_opened[i] && h->xpeer[i]) cudaIpcCloseMemHandle(h->xpeer[i]);
+  if (h->d_xbuf) cudaFree(h->d_xbuf);
+  if (h->d_xpeer) cudaFree(h->d_xpeer);
+  h->d_xbuf = nullptr;
+  h->d_xpeer = nullptr;
+  h->xpeer.clear();
+  h->x_opened.clear();
+  h->x_ready = false;
+  h->xl = XLayout{0, 0, 0};
+  h->xseq = 0;
+}
+
+int xchg_alloc(protean_handle* h, int nranks, int rank, int max_replicas, int max_gpus) {
+  if (nranks < 2 || nranks > 64 || rank < 0 || rank >= nranks) return fail(h, PROTEAN_EINVAL, "nranks/rank");
+  if (max_replicas < 1 || max_gpus < 1) return fail(h, PROTEAN_EINVAL, "exchange capacity");
+  if (max_gpus > 255) return fail(h, PROTEAN_ERANGE, "max_gpus > 255");
+  if (nranks > h->G) return fail(h, PROTEAN_EINVAL, "more ranks than geometries");
+  CK(h, cudaSetDevice(h->device));
+  xchg_release(h);
+  h->xl = XLayout{nranks, max_replicas, max_gpus};
+  h->xrank = rank;
+  const size_t bytes = h->xl.bytes();
+  cudaError_t e = cudaMalloc(&h->d_xbuf, bytes);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    h->d_xbuf = nullptr;
+    h->xl = XLayout{0, 0, 0};
+    return fail(h, PROTEAN_ENOMEM, "exchange buffer");
+  }
+  CK(h, cudaMemset(h->d_xbuf, 0, bytes));
+  CK(h, cudaDeviceSynchronize());
+  h->xpeer.assign(nranks, nullptr);
+  h->x_opened.assign(nranks, 0);
+  h->xpeer[rank] = static_cast<char*>(h->d_xbuf);
+  return PROTEAN_OK;
+}
+
+int xchg_finish(protean_handle* h) {
+  CK(h, cudaSetDevice(h->device));
+  {  // candidate lane packing of this rank's geometry range
+    std::vector<int32_t> b(h->xl.n + 1);
+    split_ranges(h->gn, h->xl.n, b.data());
+    int cw = 0;
+    std::vector<uint32_t> pk = build_pack(h->gn, b[h->xrank], b[h->xrank + 1], &cw);
+    if (h->d_pack_g) cudaFree(h->d_pack_g);
+    h->d_pack_g = nullptr;
+    CK(h, cudaMalloc(&h->d_pack_g, pk.size() * 4));
+    CK(h, cudaMemcpy(h->d_pack_g, pk.data(), pk.size() * 4, cudaMemcpyHostToDevice));
+    h->CW_g = cw;
+    h->pack_lo = b[h->xrank];
+    h->pack_hi = b[h->xrank + 1];
+  }
+  // load every kernel now: lazy module loading at first launch must not run while a peer rank's
+  // replay kernel in this process spins on the exchange
+  CK(h, preload_kernels());
+  CK(h, cudaMalloc(&h->d_xpeer, sizeof(char*) * h->xpeer.size()));
+  CK(h, cudaMemcpy(h->d_xpeer, h->xpeer.data(), sizeof(char*) * h->xpeer.size(), cudaMemcpyHostToDevice));
+  h->x_ready = true;
+  h->xseq = 0;
+  return PROTEAN_OK;
+}
 
 }  // namespace
 
@@ -199,20 +353,9 @@ int protean_load_profiles(const protean_profiles* p, protean_handle** out) {
     maxT = std::max(maxT, p->batch_timeout_us[m]);
   }
   std::vector<std::vector<uint8_t>> gs;
-  if (p->geometry_set == 0 || p->geometry_set == 1) {
-    gs = geometry_set(p->geometry_set == 1);
-  } else if (p->geometry_set == 2) {
-    if (p->n_geoms < 1) return PROTEAN_EINVAL;
-    if (p->n_geoms > 254) return PROTEAN_ERANGE;
-    if (!p->geoms) return PROTEAN_EINVAL;
-    for (int j = 0; j < p->n_geoms; ++j) {
-      std::vector<uint8_t> g;
-      int rc = validate_row(p->geoms + 8 * j, &g);
-      if (rc) return rc;
-      gs.push_back(g);
-    }
-  } else {
-    return PROTEAN_EINVAL;
+  {
+    int rc = profile_geometries(p, &gs);
+    if (rc) return rc;
   }
   protean_handle* h = new protean_handle();
   h->device = p->device;
@@ -241,31 +384,10 @@ int protean_load_profiles(const protean_profiles* p, protean_handle** out) {
     }
     w[h->tl.o_gn + j] = (int32_t)gs[j].size();
   }
-  // candidate lane packing: geometries in power-of-two lane groups, largest first, per warp
-  std::vector<uint32_t> pack;
-  {
-    std::vector<std::pair<int, int>> order;  // (Z, j)
-    for (int j = 0; j < h->G; ++j) {
-      int Z = 1;
-      while (Z < (int)gs[j].size()) Z <<= 1;
-      order.push_back({Z, j});
-    }
-    std::stable_sort(order.begin(), order.end(),
-                     [](const std::pair<int, int>& a, const std::pair<int, int>& b) { return a.first > b.first; });
-    int fill = 32;
-    for (const auto& zj : order) {
-      const int Z = zj.first, j = zj.second;
-      if (fill + Z > 32) {
-        pack.insert(pack.end(), 32, 0xFFu);
-        fill = 0;
-      }
-      const size_t w0 = pack.size() - 32;
-      for (int s = 0; s < Z; ++s)
-        pack[w0 + fill + s] = (uint32_t)j | ((uint32_t)s << 8) | ((uint32_t)Z << 16) | ((uint32_t)fill << 24);
-      fill += Z;
-    }
-    h->CW = (int)(pack.size() / 32);
-  }
+  for (int j = 0; j < h->G; ++j) h->gn.push_back((int)gs[j].size());
+  int cw = 0;
+  std::vector<uint32_t> pack = build_pack(h->gn, 0, h->G, &cw);
+  h->CW = cw;
   cudaError_t e = cudaSetDevice(h->device);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&h->nsm, cudaDevAttrMultiProcessorCount, h->device);
   if (e == cudaSuccess) e = cudaMalloc(&h->d_tab, sizeof(int32_t) * h->words.size());
@@ -290,11 +412,88 @@ void protean_free(protean_handle* h) {
   if (h->d_tab) cudaFree(h->d_tab);
   if (h->d_scratch) cudaFree(h->d_scratch);
   if (h->d_eoff) cudaFree(h->d_eoff);
+  if (h->d_ecnt) cudaFree(h->d_ecnt);
   if (h->d_small) cudaFree(h->d_small);
   if (h->d_pack) cudaFree(h->d_pack);
+  if (h->d_pack_g) cudaFree(h->d_pack_g);
+  xchg_release(h);
   for (int i = 0; i < 4; ++i)
     if (h->ev[i]) cudaEventDestroy(h->ev[i]);
   delete h;
+}
+
+int protean_geometry_split(const protean_profiles* p, int32_t nranks, int32_t* bounds) {
+  if (!bounds) return PROTEAN_EINVAL;
+  std::vector<std::vector<uint8_t>> gs;
+  int rc = profile_geometries(p, &gs);
+  if (rc) return rc;
+  if (nranks < 1 || nranks > (int)gs.size()) return PROTEAN_EINVAL;
+  std::vector<int> gn;
+  for (const auto& g : gs) gn.push_back((int)g.size());
+  split_ranges(gn, nranks, bounds);
+  return PROTEAN_OK;
+}
+
+int protean_xchg_export(protean_handle* h, int32_t nranks, int32_t rank, int32_t max_replicas,
+                        int32_t max_gpus, void* ipc_handle) {
+  if (!h) return PROTEAN_EINVAL;
+  if (h->poisoned) return PROTEAN_ESTATE;
+  if (!ipc_handle) return fail(h, PROTEAN_EINVAL, "null ipc_handle");
+  int rc = xchg_alloc(h, nranks, rank, max_replicas, max_gpus);
+  if (rc) return rc;
+  cudaIpcMemHandle_t ih;
+  CK(h, cudaIpcGetMemHandle(&ih, h->d_xbuf));
+  static_assert(sizeof(cudaIpcMemHandle_t) == 64, "ipc handle size");
+  std::memcpy(ipc_handle, &ih, 64);
+  return PROTEAN_OK;
+}
+
+int protean_xchg_import(protean_handle* h, const void* ipc_handles) {
+  if (!h) return PROTEAN_EINVAL;
+  if (h->poisoned) return PROTEAN_ESTATE;
+  if (!ipc_handles) return fail(h, PROTEAN_EINVAL, "null ipc_handles");
+  if (!h->d_xbuf || h->x_ready) return fail(h, PROTEAN_ESTATE, "import needs a fresh export");
+  CK(h, cudaSetDevice(h->device));
+  for (int k = 0; k < h->xl.n; ++k) {
+    if (k == h->xrank) continue;
+    cudaIpcMemHandle_t ih;
+    std::memcpy(&ih, static_cast<const char*>(ipc_handles) + 64 * k, 64);
+    void* ptr = nullptr;
+    CK(h, cudaIpcOpenMemHandle(&ptr, ih, cudaIpcMemLazyEnablePeerAccess));
+    h->xpeer[k] = static_cast<char*>(ptr);
+    h->x_opened[k] = 1;
+  }
+  return xchg_finish(h);
+}
+
+int protean_xchg_attach(protean_handle* const* hs, int32_t nranks, int32_t max_replicas,
+                        int32_t max_gpus) {
+  if (!hs || nranks < 2 || nranks > 64) return PROTEAN_EINVAL;
+  for (int k = 0; k < nranks; ++k) {
+    if (!hs[k]) return PROTEAN_EINVAL;
+    if (hs[k]->poisoned) return PROTEAN_ESTATE;
+    for (int q = 0; q < k; ++q)
+      if (hs[q] == hs[k]) return fail(hs[k], PROTEAN_EINVAL, "one handle per rank");
+  }
+  for (int k = 0; k < nranks; ++k) {
+    int rc = xchg_alloc(hs[k], nranks, k, max_replicas, max_gpus);
+    if (rc) return rc;
+  }
+  for (int k = 0; k < nranks; ++k) {  // peer access between distinct devices
+    for (int q = 0; q < nranks; ++q) {
+      if (hs[q]->device == hs[k]->device) continue;
+      CK(hs[k], cudaSetDevice(hs[k]->device));
+      cudaError_t e = cudaDeviceEnablePeerAccess(hs[q]->device, 0);
+      if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) return cuda_fail(hs[k], e, "peer access");
+      cudaGetLastError();
+    }
+    for (int q = 0; q < nranks; ++q) hs[k]->xpeer[q] = static_cast<char*>(hs[q]->d_xbuf);
+  }
+  for (int k = 0; k < nranks; ++k) {
+    int rc = xchg_finish(hs[k]);
+    if (rc) return rc;
+  }
+  return PROTEAN_OK;
 }
 
 int protean_last_timings(const protean_handle* h, float* prepass_ms, float* replay_ms,
@@ -338,8 +537,15 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
     return fail(h, PROTEAN_ERANGE, "ready times exceed uint32 us");
   if (c.policy == 2) return fail(h, PROTEAN_EUNSUP, "policy 2 (Alg 2 heuristic) not built");
   if (c.policy != 0 && c.policy != 1) return fail(h, PROTEAN_EINVAL, "policy");
-  if (c.shard_mode == 1) return fail(h, PROTEAN_EUNSUP, "shard mode G not built");
-  if (c.shard_mode != 0) return fail(h, PROTEAN_EINVAL, "shard_mode");
+  if (c.shard_mode != 0 && c.shard_mode != 1) return fail(h, PROTEAN_EINVAL, "shard_mode");
+  if (c.max_ctas < 0 || c.reserved != 0) return fail(h, PROTEAN_EINVAL, "max_ctas / reserved");
+  const bool modeG = c.shard_mode == 1;
+  if (modeG) {
+    if (!h->x_ready) return fail(h, PROTEAN_ESTATE, "mode G without an exchange set-up");
+    if (c.nranks != h->xl.n || c.rank != h->xrank) return fail(h, PROTEAN_EINVAL, "rank/nranks vs exchange");
+    if (c.n_replicas > h->xl.Rcap || c.n_gpus > h->xl.Ncap)
+      return fail(h, PROTEAN_ERANGE, "replicas/gpus exceed the exchange capacity");
+  }
   if (c.wait_limit < 0 || c.wait_limit > 255) return fail(h, PROTEAN_EINVAL, "wait_limit");
   if (c.reconfig_cap_pct < 0 || c.reconfig_cap_pct > 100) return fail(h, PROTEAN_EINVAL, "cap pct");
   if (c.init_geom < 0 || c.init_geom >= h->G) return fail(h, PROTEAN_EINVAL, "init_geom");
@@ -373,7 +579,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   const size_t eoff_need = sizeof(int64_t) * (size_t)R * (size_t)(E + 1);
   {
     void* p = h->d_eoff;
-    int rc = ensure(h, &p, &h->eoff_bytes, eoff_need);
+    int rc = ensure(h, &p, &h->eoff_bytes, eoff_need, st);
     h->d_eoff = static_cast<int64_t*>(p);
     if (rc) return rc;
   }
@@ -382,6 +588,14 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   CK(h, cudaMemsetAsync(h->d_small, 0, 256, st));
   CK(h, cudaEventRecord(h->ev[0], st));
   CK(h, launch_prepass(c.arrival_us, c.replica_off, R, E, W, h->maxT, h->d_eoff, d_wmax, d_err, st));
+  const int kWarps = 8;  // replay CTA = 8 warps; the partition uses kWarps - 1 new-request segments
+  {  // per-(replica, epoch, segment, stream) counts of each epoch's new requests
+    const size_t need = sizeof(uint32_t) * (size_t)R * (size_t)E * (kWarps - 1) * (size_t)(2 * h->M);
+    int rc = ensure(h, &h->d_ecnt, &h->ecnt_bytes, need, st);
+    if (rc) return rc;
+    CK(h, launch_epoch_count(c.meta, h->d_eoff, R, E, kWarps - 1, 2 * h->M, h->M,
+                             static_cast<uint32_t*>(h->d_ecnt), st));
+  }
   CK(h, cudaEventRecord(h->ev[1], st));
   unsigned long long wmax = 0;
   int herr = 0;
@@ -392,17 +606,28 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   const int WCAP = (int)std::max<unsigned long long>(wmax, 1);
   if (wmax >= (1ull << 25)) return fail(h, PROTEAN_ERANGE, "epoch window >= 2^25 requests");
 
+  // candidate range: all geometries, or this rank's slot-balanced range (mode G)
+  int geom_lo = 0, geom_hi = h->G;
+  const uint32_t* d_pack = h->d_pack;
+  int CW = h->CW;
+  if (modeG) {
+    std::vector<int32_t> b(h->xl.n + 1);
+    split_ranges(h->gn, h->xl.n, b.data());
+    geom_lo = b[h->xrank];
+    geom_hi = b[h->xrank + 1];
+    if (h->pack_lo != geom_lo || h->pack_hi != geom_hi) return fail(h, PROTEAN_ESTATE, "range packing");
+    d_pack = h->d_pack_g;
+    CW = h->CW_g;
+  }
   // launch geometry: 8 warps; units = actual-placement warps + candidate warps per GPU
-  const int Gc = h->G;
+  const int Gc = geom_hi - geom_lo;
   // warps per CTA: the placement phase runs n_units warp units; pick 4..8 warps that divide them
   // most evenly (prefer more warps on ties)
-  const int n_units = (N + 3) / 4 + (c.policy == 0 ? N * h->CW : 0);
-  int best_nw = 8;  // measured on B200: 8 warps x 3 CTAs/SM beat 6 x 4 (L1 room for lane lists)
+  const int n_units = (N + 3) / 4 + (c.policy == 0 ? N * CW : 0);
   (void)n_units;
-  if (const char* ev = std::getenv("PROTEAN_WARPS")) best_nw = std::max(4, std::min(8, std::atoi(ev)));
-  const int block = 32 * best_nw;
+  const int block = 32 * kWarps;  // measured on B200: 8 warps x 3 CTAs/SM beat 6 x 4
   SmemLayout sl;
-  sl.init(h->tl.words, h->M, N, Gc, h->CW, 0, 0);
+  sl.init(h->tl.words, h->M, N, Gc, CW, 0, 0);
   const size_t fixed = sl.total;
   int BS = std::min(WCAP, 64);
   size_t budget = 72 * 1024;
@@ -412,23 +637,25 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   }
   const size_t with_bats = fixed + (size_t)BS * (sizeof(Bat) + 8) + 64;
   const int WS = (with_bats + (size_t)WCAP * 4 <= budget) ? WCAP : 0;  // window all in smem or all in HBM
-  sl.init(h->tl.words, h->M, N, Gc, h->CW, BS, WS);
+  sl.init(h->tl.words, h->M, N, Gc, CW, BS, WS);
   if (sl.total > 227 * 1024) return fail(h, PROTEAN_ERANGE, "shared memory layout too large");
   int per_sm = 0;
   CK(h, replay_occupancy(block, sl.total, &per_sm));
   if (per_sm < 1) return fail(h, PROTEAN_ERANGE, "replay kernel does not fit an SM");
-  const int grid = std::min<int64_t>(R, (int64_t)h->nsm * per_sm);
+  int grid = (int)std::min<int64_t>(R, (int64_t)h->nsm * per_sm);
+  if (c.max_ctas > 0) grid = std::min(grid, c.max_ctas);
 
   ReplayParams P;
   std::memset(&P, 0, sizeof(P));
   P.tab = h->d_tab;
   P.tl = h->tl;
-  P.pack = h->d_pack;
+  P.pack = d_pack;
   P.maxT = h->maxT;
   P.arr = c.arrival_us;
   P.meta = c.meta;
   P.roff = c.replica_off;
   P.eoff = h->d_eoff;
+  P.ecnt = static_cast<const uint32_t*>(h->d_ecnt);
   P.R = R;
   P.N = N;
   P.base = c.replica_base;
@@ -449,8 +676,17 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   P.seed = c.seed;
   P.price_od = c.price_od_node_hr;
   P.price_spot = c.price_spot_node_hr;
-  P.geom_lo = 0;
-  P.geom_hi = Gc;
+  P.geom_lo = geom_lo;
+  P.geom_hi = geom_hi;
+  if (modeG && !std::getenv("PROTEAN_XCHG_OFF")) {  // debug knob: score the range, no exchange
+    P.xl = h->xl;
+    P.xpeer = h->d_xpeer;
+    P.xrank = h->xrank;
+    P.xseq = h->xseq;
+    P.xtimeout_ns = 30ull * 1000000000ull;
+    if (const char* ev = std::getenv("PROTEAN_XCHG_TIMEOUT_S"))
+      P.xtimeout_ns = (uint64_t)std::max(1, std::atoi(ev)) * 1000000000ull;
+  }
   P.counters = out->counters;
   P.accum = out->accum;
   P.hist = out->hist;
@@ -473,7 +709,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   P.o_gsarr = o; o += al((size_t)(WS >= WCAP ? 0 : WCAP) * 4);
   P.slot_bytes = al(o);
   {
-    int rc = ensure(h, &h->d_scratch, &h->scratch_bytes, P.slot_bytes * (size_t)grid);
+    int rc = ensure(h, &h->d_scratch, &h->scratch_bytes, P.slot_bytes * (size_t)grid, st);
     if (rc) return rc;
   }
   P.scratch = static_cast<char*>(h->d_scratch);
@@ -481,8 +717,15 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   CK(h, cudaEventRecord(h->ev[2], st));
   CK(h, launch_replay(P, grid, block, st));
   CK(h, cudaEventRecord(h->ev[3], st));
-  CK(h, cudaMemcpyAsync(&herr, d_err, 4, cudaMemcpyDeviceToHost, st));
+  int herr2[2] = {0, 0};
+  CK(h, cudaMemcpyAsync(herr2, d_err, 8, cudaMemcpyDeviceToHost, st));
   CK(h, cudaStreamSynchronize(st));
+  herr = herr2[0];
+  if (modeG) h->xseq += (uint32_t)E;
+  if (herr2[1]) {
+    h->poisoned = true;
+    return fail(h, PROTEAN_ENCCL, "mode G exchange: a peer rank did not publish within 30 s");
+  }
   CK(h, cudaEventElapsedTime(&h->t_prepass, h->ev[0], h->ev[1]));
   CK(h, cudaEventElapsedTime(&h->t_replay, h->ev[2], h->ev[3]));
   h->last_grid = grid;
@@ -515,7 +758,7 @@ int protean_score_epoch(protean_handle* h, const protean_epoch_in* in, protean_e
   if (b0 != 0) return fail(h, PROTEAN_EINVAL, "batch_off[0] != 0");
   const size_t need = sizeof(protean_resident) * (size_t)R * N * Gc * in->max_live;
   {
-    int rc = ensure(h, &h->d_scratch, &h->scratch_bytes, std::max<size_t>(need, 256));
+    int rc = ensure(h, &h->d_scratch, &h->scratch_bytes, std::max<size_t>(need, 256), st);
     if (rc) return rc;
   }
   int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 64);

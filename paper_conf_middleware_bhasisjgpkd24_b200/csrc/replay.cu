@@ -12,6 +12,8 @@
 // The request stream (5 B/request) is read from HBM once with coalesced loads (a second, L2-hot
 // read scatters it); everything else lives in shared memory, registers and L1-resident scratch.
 #include <cuda_runtime.h>
+#include <mutex>
+
 #include "replay.cuh"
 #ifndef PROTEAN_MINB
 #define PROTEAN_MINB 3
@@ -79,6 +81,65 @@ struct CtaState {
 };
 
 enum { VM_NONE = 0, VM_OD = 1, VM_SPOT = 2 };
+
+// ------------------------------------------------------------------ mode G exchange (S8, §8(e))
+__device__ __forceinline__ uint64_t global_ns() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+// Per (replica r, sequence seq): publish this rank's {best, current} key pairs of every sim-GPU
+// into every rank's buffer (peer stores over NVLink), release a flag per destination, acquire
+// every source's flag, then take the min of each pair over sources into gi rows 6 (best) and 7
+// (current geometry's key).  Called by the whole CTA (contains barriers).
+static __device__ __noinline__ void exchange_keys(XLayout X, char* const* xpeer, int xrank,
+                                                   int* err, uint64_t timeout_ns, int64_t* gi,
+                                                   int N, int r, uint32_t seq, int tid, int NT) {
+  const int par = (int)(seq & 1u);
+  __syncthreads();  // gi row 6 of every sim-GPU is final
+  for (int i = tid; i < N * X.n; i += NT) {  // (gpu, destination) pairs
+    const int g = i % N, dst = i / N;
+    const int64_t kb = gi[6 * N + g], kc0 = gi[7 * N + g];
+    const int64_t kc = kc0 >= 0 ? kc0 : kForever;
+    longlong2* d = reinterpret_cast<longlong2*>(xpeer[dst] + X.key_off(par, xrank, r, g));
+    *d = make_longlong2(kb, kc);
+  }
+  __threadfence_system();
+  __syncthreads();
+  if (tid < X.n) {  // release: the pairs above are visible before the flag
+    uint32_t* f = reinterpret_cast<uint32_t*>(xpeer[tid] + X.flag_off(xrank, r));
+    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(f), "r"(seq + 1u) : "memory");
+  }
+  if (tid < X.n && *(volatile int*)(err + 1) == 0) {  // acquire every source's flag (fail fast
+    // once any wait of this call timed out)
+    const uint32_t* f = reinterpret_cast<const uint32_t*>(xpeer[xrank] + X.flag_off(tid, r));
+    const uint64_t t0 = global_ns();
+    for (;;) {
+      uint32_t v;
+      asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(f) : "memory");
+      if ((int32_t)(v - (seq + 1u)) >= 0) break;
+      if (global_ns() - t0 > timeout_ns) {
+        atomicOr(err + 1, 1);
+        break;
+      }
+      __nanosleep(256);
+    }
+  }
+  __syncthreads();
+  const char* mine = xpeer[xrank];
+  for (int g = tid; g < N; g += NT) {
+    int64_t kb = kForever, kc = kForever;
+    for (int src = 0; src < X.n; ++src) {
+      const longlong2 v = __ldcv(reinterpret_cast<const longlong2*>(mine + X.key_off(par, src, r, g)));
+      kb = v.x < kb ? v.x : kb;
+      kc = v.y < kc ? v.y : kc;
+    }
+    gi[6 * N + g] = kb;
+    gi[7 * N + g] = kc;
+  }
+  __syncthreads();
+}
 
 __device__ __forceinline__ int64_t clip_h(int64_t x, int64_t H) { return x < H ? x : H; }
 
@@ -310,6 +371,56 @@ __device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, const
   return o;
 }
 
+// Per-stream request counts of meta[lo, hi) (one warp; 16-byte loads; match_any aggregation).
+__device__ __forceinline__ void count_segment(const uint8_t* meta, int64_t lo, int64_t hi, int* cntw,
+                                              const uint16_t* klut) {
+  const int lane = threadIdx.x & 31;
+  const int64_t h = min(hi, lo + (int64_t)((16u - ((uint32_t)(uintptr_t)(meta + lo) & 15u)) & 15u));
+  {  // unaligned head (< 16 elements)
+    const int64_t i = lo + lane;
+    const int key = i < h ? (klut[meta[i]] & 0x7FFF) : 1024 + lane;
+    const unsigned peers = __match_any_sync(0xffffffffu, key);
+    if (key < 1024 && (peers & ((1u << lane) - 1u)) == 0) atomicAdd(&cntw[key], __popc(peers));
+  }
+  const int nch = (int)((hi - h) >> 4);
+  const uint4* gv = reinterpret_cast<const uint4*>(meta + h);
+#pragma unroll 1
+  for (int c0 = 0; c0 < nch; c0 += 32) {
+    const int ch = c0 + lane;
+    const bool valid = ch < nch;
+    const uint4 v = valid ? gv[ch] : make_uint4(0u, 0u, 0u, 0u);
+    const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
+    int keys[16];
+#pragma unroll
+    for (int q = 0; q < 16; ++q)
+      keys[q] = valid ? (klut[(w4[q >> 2] >> (8 * (q & 3))) & 0xFF] & 0x7FFF) : 1024 + lane;
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      const unsigned peers = __match_any_sync(0xffffffffu, keys[q]);
+      if (keys[q] < 1024 && (peers & ((1u << lane) - 1u)) == 0) atomicAdd(&cntw[keys[q]], __popc(peers));
+    }
+  }
+  {  // tail (< 16 elements)
+    const int64_t i = h + (int64_t)nch * 16 + lane;
+    const int key = i < hi ? (klut[meta[i]] & 0x7FFF) : 1024 + lane;
+    const unsigned peers = __match_any_sync(0xffffffffu, key);
+    if (key < 1024 && (peers & ((1u << lane) - 1u)) == 0) atomicAdd(&cntw[key], __popc(peers));
+  }
+}
+
+// Segment s of a window whose first nbeg entries are carried from the previous epoch:
+// segment 0 = the carried part, segments 1..nw-1 split the new requests evenly.
+__device__ __forceinline__ void seg_bounds(int64_t nbeg, int64_t len, int s, int nw, int64_t* lo,
+                                           int64_t* hi) {
+  if (s == 0) {
+    *lo = 0;
+    *hi = nbeg;
+  } else {
+    *lo = nbeg + (len - nbeg) * (s - 1) / (nw - 1);
+    *hi = nbeg + (len - nbeg) * s / (nw - 1);
+  }
+}
+
 // Candidate unit with register-resident slice lists (the GPU-epoch has <= kKR batches, so no lane
 // ever holds more residents).  Replay states are FIFO-consistent, so every resident started at or
 // before the slice's last start: Eq 1's co-runners at an instant x >= t0 are exactly the residents
@@ -431,6 +542,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
   __shared__ uint16_t klut[256];        // meta byte -> stream key (| 0x8000 if invalid)
   __shared__ int s_cnt[kNSeg * kMaxStreams], s_run[kNSeg * kMaxStreams];
   __shared__ int s_base[kMaxStreams], s_tot[kMaxStreams], s_skip[kMaxStreams], s_pend[kMaxStreams];
+  __shared__ int s_ge[kMaxStreams];      // carried entries per stream (previous epoch's bookkeeping)
 #ifdef PROTEAN_PHASE_TIMING
   unsigned long long ph_acc[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
   long long ph_last = clock64();
@@ -507,7 +619,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
 #pragma unroll 1
     for (int i = tid; i < 2 * kNB; i += NT) s_hist[i] = 0;
 #pragma unroll 1
-    for (int k = tid; k < S; k += NT) s_skip[k] = 0;
+    for (int k = tid; k < S; k += NT) s_skip[k] = s_ge[k] = 0;
 #pragma unroll 1
     for (int g = tid; g < N; g += NT) {
       reset_gpu_state(c, g, P.init_geom);
@@ -532,8 +644,6 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
     for (int64_t e = 0; e < P.E; ++e) {
       const int64_t eW = e * P.W, Tend = eW + P.W;
       // ---------------------------------------------------------------- A: VM events, installs
-#pragma unroll 1
-      for (int i = tid; i < NW * S; i += NT) s_cnt[i] = 0;
 #pragma unroll 1
       for (int g = tid; g < N; g += NT) {
         if (P.vm_policy != 0) {
@@ -586,40 +696,20 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       // 16-byte meta loads, (2) after one barrier each warp derives its own per-stream write
       // offsets (redundant scan over streams), (3) stable scatter of its segment with 8 loads in
       // flight per lane, validating every request once (when it is new).
-      const int sa_lo = (int)((int64_t)len * warp / NW), sa_hi = (int)((int64_t)len * (warp + 1) / NW);
+      int sa_lo, sa_hi;
       {
-        int* cntw = s_cnt + warp * S;
-        const int h = min(sa_hi, sa_lo + (int)((16u - ((uint32_t)(uintptr_t)(wmeta + sa_lo) & 15u)) & 15u));
-        {  // unaligned head (< 16 elements)
-          const int i = sa_lo + lane;
-          const int key = i < h ? (klut[wmeta[i]] & 0x7FFF) : 1024 + lane;
-          const unsigned peers = __match_any_sync(0xffffffffu, key);
-          if (key < 1024 && (peers & ((1u << lane) - 1u)) == 0) cntw[key] += __popc(peers);
-        }
-        const int nch = (sa_hi - h) >> 4;
-        const uint4* gv = reinterpret_cast<const uint4*>(wmeta + h);
+        int64_t lo64, hi64;
+        seg_bounds(nbeg, len, warp, NW, &lo64, &hi64);
+        sa_lo = (int)lo64;
+        sa_hi = (int)hi64;
+      }
+      // per (segment, stream) counts: segment 0 = carried (previous epoch), 1..NW-1 = new requests
+      // counted ahead by epoch_count_kernel
+      {
+        const uint32_t* tb = P.ecnt + (((size_t)r * P.E + e) * (NW - 1)) * S;
 #pragma unroll 1
-        for (int c0 = 0; c0 < nch; c0 += 32) {
-          const int ch = c0 + lane;
-          const bool valid = ch < nch;
-          const uint4 v = valid ? gv[ch] : make_uint4(0u, 0u, 0u, 0u);
-          const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
-          int keys[16];
-#pragma unroll
-          for (int q = 0; q < 16; ++q)
-            keys[q] = valid ? (klut[(w4[q >> 2] >> (8 * (q & 3))) & 0xFF] & 0x7FFF) : 1024 + lane;
-#pragma unroll
-          for (int q = 0; q < 16; ++q) {
-            const unsigned peers = __match_any_sync(0xffffffffu, keys[q]);
-            if (keys[q] < 1024 && (peers & ((1u << lane) - 1u)) == 0) atomicAdd(&cntw[keys[q]], __popc(peers));
-          }
-        }
-        {  // tail (< 16 elements)
-          const int i = h + nch * 16 + lane;
-          const int key = i < sa_hi ? (klut[wmeta[i]] & 0x7FFF) : 1024 + lane;
-          const unsigned peers = __match_any_sync(0xffffffffu, key);
-          if (key < 1024 && (peers & ((1u << lane) - 1u)) == 0) cntw[key] += __popc(peers);
-        }
+        for (int i = tid; i < NW * S; i += NT)
+          s_cnt[i] = bad_window ? 0 : (i < S ? s_ge[i] : (int)tb[i - S]);
       }
       __syncthreads();
       PH(1);
@@ -792,7 +882,10 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       // next window: stream entries at/after the earliest open batch's first arrival are re-read
 #pragma unroll 1
       for (int k = tid; k < S; k += NT) {
-        if (bad_window) break;
+        if (bad_window) {  // the next window starts at w_end: nothing carried
+          s_ge[k] = 0;
+          continue;
+        }
         const int b0 = s_base[k], tot = s_tot[k];
         int lo = 0, hi = tot;
 #pragma unroll 1
@@ -802,6 +895,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
         }
         if (lo) atomicAdd(reinterpret_cast<unsigned long long*>(&cs.lt_total), (unsigned long long)lo);
         s_skip[k] = tot - lo - s_pend[k];
+        s_ge[k] = tot - lo;  // the next window re-reads these (arrival >= amin): its segment 0
       }
       Bat* bats = c.bats;
       uint32_t* ord = c.ord;
@@ -1191,19 +1285,30 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       __syncthreads();
       PH(7);
       // ---------------------------------------------------------------- G: decisions (O9, O10)
+      if (P.policy == 0) {  // S8: min over this rank's geometry range
+#pragma unroll 1
+        for (int g = tid; g < N; g += NT) {
+          int64_t kb = kForever;
+          if (c.gu8[5 * c.N + g]) {
+#pragma unroll 1
+            for (int v = 0; v < Gc; ++v) kb = c.keys[g * Gc + v] < kb ? c.keys[g * Gc + v] : kb;
+          }
+          c.gi[6 * c.N + g] = kb;
+        }
+        if (P.xl.n > 1)
+          exchange_keys(P.xl, P.xpeer, P.xrank, P.err, P.xtimeout_ns, c.gi, N, r,
+                        (uint32_t)(P.xseq + (uint32_t)e), tid, NT);
+      }
 #pragma unroll 1
       for (int g = tid; g < N; g += NT) {
         uint8_t dec_out = kNoGeom;
         if (P.policy == 0 && c.gu8[5 * c.N + g]) {
-          int64_t kb = c.keys[g * Gc];
-#pragma unroll 1
-          for (int v = 1; v < Gc; ++v) kb = c.keys[g * Gc + v] < kb ? c.keys[g * Gc + v] : kb;
+          const int64_t kb = c.gi[6 * c.N + g];
           const int cur = c.gu8[0 * c.N + g];
           const int tag = (int)(kb & 255);
           const int best = tag == 0 ? cur : tag - 1;
           dec_out = (uint8_t)best;
           c.gu8[6 * c.N + g] = (uint8_t)best;
-          c.gi[6 * c.N + g] = kb;
           if (best != cur) {
             if (c.gu8[2 * c.N + g] >= P.wait_limit) c.gu8[7 * c.N + g] = 1;
             else c.gu8[2 * c.N + g]++;
@@ -1338,6 +1443,43 @@ extern "C" int protean_debug_phase_cycles(unsigned long long* out) {
 }
 #endif
 
+// Per-(replica, epoch, segment, stream) counts of each epoch's new requests, segments as in
+// seg_bounds (nbeg = 0): warp per (replica, epoch, segment).  Consumed by the replay's stable
+// stream partition, which therefore needs no count pass of its own.
+__global__ void __launch_bounds__(256) epoch_count_kernel(const uint8_t* meta, const int64_t* eoff,
+                                                          int R, int64_t E, int nseg, int S, int M,
+                                                          uint32_t* table) {
+  __shared__ uint16_t klut[256];
+  __shared__ int cnt[8][kMaxStreams];
+  for (int b = threadIdx.x; b < 256; b += blockDim.x) {
+    const int m = b & 63;
+    const bool ok = !(b & 0x40) && m < M;
+    klut[b] = (uint16_t)((2 * (ok ? m : 0) + ((b >> 7) ? 0 : 1)) | (ok ? 0 : 0x8000));
+  }
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (int k = lane; k < S; k += 32) cnt[warp][k] = 0;
+  __syncthreads();
+  const int64_t idx = (int64_t)blockIdx.x * 8 + warp;  // (r, e, seg)
+  if (idx >= (int64_t)R * E * nseg) return;
+  const int64_t re = idx / nseg;
+  const int sg = (int)(idx - re * nseg) + 1;
+  const int r = (int)(re / E);
+  const int64_t e = re - (int64_t)r * E;
+  const int64_t A = eoff[(size_t)r * (E + 1) + e], B = eoff[(size_t)r * (E + 1) + e + 1];
+  int64_t lo, hi;
+  seg_bounds(0, B - A, sg, nseg + 1, &lo, &hi);
+  if (hi > lo) count_segment(meta + A, lo, hi, cnt[warp], klut);
+  __syncwarp();
+  for (int k = lane; k < S; k += 32) table[(size_t)idx * S + k] = (uint32_t)cnt[warp][k];
+}
+
+cudaError_t launch_epoch_count(const uint8_t* meta, const int64_t* eoff, int R, int64_t E, int nseg,
+                               int S, int M, uint32_t* table, cudaStream_t st) {
+  const int64_t warps = (int64_t)R * E * nseg;
+  epoch_count_kernel<<<(unsigned)((warps + 7) / 8), 256, 0, st>>>(meta, eoff, R, E, nseg, S, M, table);
+  return cudaGetLastError();
+}
+
 // Prepass: eoff[r][e] = first request of replica r with arrival >= e*W (e = 0..E), and the
 // largest request window any epoch needs: [lower_bound(eW - maxT), eoff[e+1]).
 __global__ void prepass_kernel(const uint32_t* arr, const int64_t* roff, int R, int64_t E,
@@ -1378,17 +1520,47 @@ cudaError_t launch_prepass(const uint32_t* arr, const int64_t* roff, int R, int6
   return cudaGetLastError();
 }
 
+// The replay kernel's dynamic shared-memory limit is raised once per device, to the opt-in
+// maximum: changing a function attribute while an instance of the function runs can wait for it,
+// which would serialise concurrently running mode-G ranks of one process.
+static cudaError_t raise_dyn_smem_once() {
+  static std::mutex mu;
+  static bool done[256] = {};
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  std::lock_guard<std::mutex> lk(mu);
+  if (dev < 256 && done[dev]) return cudaSuccess;
+  int optin = 0;
+  e = cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+  if (e != cudaSuccess) return e;
+  cudaFuncAttributes a;
+  e = cudaFuncGetAttributes(&a, replay_kernel);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(replay_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           optin - (int)a.sharedSizeBytes);
+  if (e == cudaSuccess && dev < 256) done[dev] = true;
+  return e;
+}
+
+cudaError_t preload_kernels() {
+  cudaFuncAttributes a;
+  cudaError_t e = cudaFuncGetAttributes(&a, replay_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, prepass_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, epoch_count_kernel);
+  if (e == cudaSuccess) e = raise_dyn_smem_once();
+  return e;
+}
+
 cudaError_t launch_replay(const ReplayParams& P, int grid, int block, cudaStream_t st) {
-  cudaError_t e = cudaFuncSetAttribute(replay_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)P.sl.total);
+  cudaError_t e = raise_dyn_smem_once();
   if (e != cudaSuccess) return e;
   replay_kernel<<<grid, block, P.sl.total, st>>>(P);
   return cudaGetLastError();
 }
 
 cudaError_t replay_occupancy(int block, size_t smem, int* blocks_per_sm) {
-  cudaError_t e = cudaFuncSetAttribute(replay_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)smem);
+  cudaError_t e = raise_dyn_smem_once();
   if (e != cudaSuccess) return e;
   return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, replay_kernel, block, smem);
 }

@@ -52,6 +52,19 @@ struct SmemLayout {
   }
 };
 
+// Mode G exchange buffer of one rank (byte offsets): keys [2 parity][n src][Rcap][Ncap] x
+// {best, current} int64, then flags [n src][Rcap] uint32 (the source's sequence number + 1).
+struct XLayout {
+  int n, Rcap, Ncap;  // n = 0: no exchange
+  __host__ __device__ size_t key_off(int par, int src, int r, int g) const {
+    return ((((size_t)par * n + src) * Rcap + r) * Ncap + g) * 16;
+  }
+  __host__ __device__ size_t flag_off(int src, int r) const {
+    return (size_t)2 * n * Rcap * Ncap * 16 + ((size_t)src * Rcap + r) * 4;
+  }
+  __host__ __device__ size_t bytes() const { return flag_off(n, 0); }
+};
+
 struct ReplayParams {
   // tables
   const int32_t* tab;
@@ -63,6 +76,7 @@ struct ReplayParams {
   const uint8_t* meta;
   const int64_t* roff;
   const int64_t* eoff;     // [R][E+1] first request index with arrival >= e*W
+  const uint32_t* ecnt;    // [R][E][NW-1][S] per-segment stream counts of each epoch's new requests
   int R, N;
   int64_t base, trace_len, W, E, H;
   // policy
@@ -88,7 +102,13 @@ struct ReplayParams {
   int WCAP;                // max window entries of any epoch (prepass)
   char* scratch;
   size_t slot_bytes, o_alist, o_clist, o_gbat, o_gord, o_gglist, o_gsarr;
-  int* err;
+  int* err;                // err[0]: invalid request, err[1]: exchange timeout
+  // mode G exchange (xl.n == 0: off)
+  XLayout xl;
+  char* const* xpeer;      // [n] every rank's exchange buffer, mapped in this process
+  int xrank;
+  uint32_t xseq;           // sequence number of epoch 0 of this call
+  uint64_t xtimeout_ns;    // a source flag not seen within this time fails the call (ENCCL)
 };
 
 struct ScoreParams {
@@ -113,8 +133,11 @@ struct ScoreParams {
 cudaError_t launch_prepass(const uint32_t* arr, const int64_t* roff, int R, int64_t E, int64_t W,
                            int64_t maxT, int64_t* eoff, unsigned long long* wmax, int* err,
                            cudaStream_t st);
+cudaError_t launch_epoch_count(const uint8_t* meta, const int64_t* eoff, int R, int64_t E, int nseg,
+                               int S, int M, uint32_t* table, cudaStream_t st);
 cudaError_t launch_replay(const ReplayParams& P, int grid, int block, cudaStream_t st);
 cudaError_t replay_occupancy(int block, size_t smem, int* blocks_per_sm);
+cudaError_t preload_kernels();
 cudaError_t launch_score(const ScoreParams& P, int block, cudaStream_t st);
 size_t score_smem_bytes(const TabLayout& tl, int N, int Gc);
 

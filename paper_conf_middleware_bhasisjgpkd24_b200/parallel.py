@@ -55,3 +55,35 @@ def max_over_ranks(value: float) -> float:
     t = torch.tensor([float(value)], dtype=torch.float64)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
+
+
+# ------------------------------------------------------------------------------------------------
+# Mode G (geometry-range sharding): rank k scores geometries [b[k], b[k+1]) of
+# protean_geometry_split and every rank runs the rest redundantly; the per-epoch min-loc exchange
+# is fused into the replay kernel over peer memory (include/protean.h section 4).  The host side
+# only wires the exchange buffers once: export -> all-gather of the 64-byte IPC handles -> import.
+
+def setup_geometry_sharding(handle, world: int, rank: int, max_replicas: int, max_gpus: int):
+    """Export this rank's exchange buffer, all-gather the IPC handles, map every peer's buffer."""
+    import torch.distributed as dist
+    mine = handle.xchg_export(world, rank, max_replicas, max_gpus)
+    parts = [None] * world
+    dist.all_gather_object(parts, (rank, mine))
+    ordered = [h for _, h in sorted(parts)]
+    assert [k for k, _ in sorted(parts)] == list(range(world))
+    handle.xchg_import(ordered)
+    return ordered
+
+
+def merge_geometry_shards(outs: list, bounds: list[int]) -> dict:
+    """Combine the per-rank outputs of one mode-G replay: every field is identical across ranks
+    except counters 8/9 (each rank's own candidates: summed) and cand_keys (each rank's range)."""
+    base = {k: (np.array(v, copy=True) if isinstance(v, np.ndarray) else v) for k, v in outs[0].items()}
+    if "counters" in base:
+        base["counters"][:, 8] = sum(np.asarray(o["counters"])[:, 8] for o in outs)
+        base["counters"][:, 9] = sum(np.asarray(o["counters"])[:, 9] for o in outs)
+    if "cand_keys" in base:
+        for k, o in enumerate(outs):
+            lo, hi = bounds[k], bounds[k + 1]
+            base["cand_keys"][..., lo:hi] = np.asarray(o["cand_keys"])[..., lo:hi]
+    return base
