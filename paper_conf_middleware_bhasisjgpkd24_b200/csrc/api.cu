@@ -29,8 +29,6 @@ struct protean_handle {
   size_t scratch_bytes = 0;
   int64_t* d_eoff = nullptr;
   size_t eoff_bytes = 0;
-  void* d_ecnt = nullptr;
-  size_t ecnt_bytes = 0;
   void* d_small = nullptr;  // wmax (8 B) + err (16 B)
   uint32_t* d_pack = nullptr;  // candidate lane packing for the full geometry range
   int CW = 0;
@@ -412,7 +410,6 @@ void protean_free(protean_handle* h) {
   if (h->d_tab) cudaFree(h->d_tab);
   if (h->d_scratch) cudaFree(h->d_scratch);
   if (h->d_eoff) cudaFree(h->d_eoff);
-  if (h->d_ecnt) cudaFree(h->d_ecnt);
   if (h->d_small) cudaFree(h->d_small);
   if (h->d_pack) cudaFree(h->d_pack);
   if (h->d_pack_g) cudaFree(h->d_pack_g);
@@ -588,14 +585,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   CK(h, cudaMemsetAsync(h->d_small, 0, 256, st));
   CK(h, cudaEventRecord(h->ev[0], st));
   CK(h, launch_prepass(c.arrival_us, c.replica_off, R, E, W, h->maxT, h->d_eoff, d_wmax, d_err, st));
-  const int kWarps = 8;  // replay CTA = 8 warps; the partition uses kWarps - 1 new-request segments
-  {  // per-(replica, epoch, segment, stream) counts of each epoch's new requests
-    const size_t need = sizeof(uint32_t) * (size_t)R * (size_t)E * (kWarps - 1) * (size_t)(2 * h->M);
-    int rc = ensure(h, &h->d_ecnt, &h->ecnt_bytes, need, st);
-    if (rc) return rc;
-    CK(h, launch_epoch_count(c.meta, h->d_eoff, R, E, kWarps - 1, 2 * h->M, h->M,
-                             static_cast<uint32_t*>(h->d_ecnt), st));
-  }
+  const int kWarps = 8;  // replay CTA = 8 warps
   CK(h, cudaEventRecord(h->ev[1], st));
   unsigned long long wmax = 0;
   int herr = 0;
@@ -652,10 +642,11 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   P.pack = d_pack;
   P.maxT = h->maxT;
   P.arr = c.arrival_us;
+  P.vec_ok = ((reinterpret_cast<uintptr_t>(c.arrival_us) & 15u) == 0) &&
+             ((reinterpret_cast<uintptr_t>(c.meta) & 15u) == 0);
   P.meta = c.meta;
   P.roff = c.replica_off;
   P.eoff = h->d_eoff;
-  P.ecnt = static_cast<const uint32_t*>(h->d_ecnt);
   P.R = R;
   P.N = N;
   P.base = c.replica_base;

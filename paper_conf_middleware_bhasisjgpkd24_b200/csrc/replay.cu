@@ -371,53 +371,125 @@ __device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, const
   return o;
 }
 
-// Per-stream request counts of meta[lo, hi) (one warp; 16-byte loads; match_any aggregation).
-__device__ __forceinline__ void count_segment(const uint8_t* meta, int64_t lo, int64_t hi, int* cntw,
-                                              const uint16_t* klut) {
-  const int lane = threadIdx.x & 31;
-  const int64_t h = min(hi, lo + (int64_t)((16u - ((uint32_t)(uintptr_t)(meta + lo) & 15u)) & 15u));
-  {  // unaligned head (< 16 elements)
-    const int64_t i = lo + lane;
-    const int key = i < h ? (klut[meta[i]] & 0x7FFF) : 1024 + lane;
-    const unsigned peers = __match_any_sync(0xffffffffu, key);
-    if (key < 1024 && (peers & ((1u << lane) - 1u)) == 0) atomicAdd(&cntw[key], __popc(peers));
-  }
-  const int nch = (int)((hi - h) >> 4);
-  const uint4* gv = reinterpret_cast<const uint4*>(meta + h);
-#pragma unroll 1
-  for (int c0 = 0; c0 < nch; c0 += 32) {
-    const int ch = c0 + lane;
-    const bool valid = ch < nch;
-    const uint4 v = valid ? gv[ch] : make_uint4(0u, 0u, 0u, 0u);
-    const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
-    int keys[16];
-#pragma unroll
-    for (int q = 0; q < 16; ++q)
-      keys[q] = valid ? (klut[(w4[q >> 2] >> (8 * (q & 3))) & 0xFF] & 0x7FFF) : 1024 + lane;
-#pragma unroll
-    for (int q = 0; q < 16; ++q) {
-      const unsigned peers = __match_any_sync(0xffffffffu, keys[q]);
-      if (keys[q] < 1024 && (peers & ((1u << lane) - 1u)) == 0) atomicAdd(&cntw[keys[q]], __popc(peers));
-    }
-  }
-  {  // tail (< 16 elements)
-    const int64_t i = h + (int64_t)nch * 16 + lane;
-    const int key = i < hi ? (klut[meta[i]] & 0x7FFF) : 1024 + lane;
-    const unsigned peers = __match_any_sync(0xffffffffu, key);
-    if (key < 1024 && (peers & ((1u << lane) - 1u)) == 0) atomicAdd(&cntw[key], __popc(peers));
-  }
+// Predicated shared-memory reduction (keeps the per-element loops free of branches).
+__device__ __forceinline__ void red_shared_if(bool p, uint32_t saddr, uint32_t v) {
+  asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.shared.add.u32 [%0], %1;\n\t}"
+               ::"r"(saddr), "r"(v), "r"((uint32_t)p) : "memory");
 }
 
-// Segment s of a window whose first nbeg entries are carried from the previous epoch:
-// segment 0 = the carried part, segments 1..nw-1 split the new requests evenly.
-__device__ __forceinline__ void seg_bounds(int64_t nbeg, int64_t len, int s, int nw, int64_t* lo,
-                                           int64_t* hi) {
-  if (s == 0) {
-    *lo = 0;
-    *hi = nbeg;
-  } else {
-    *lo = nbeg + (len - nbeg) * (s - 1) / (nw - 1);
-    *hi = nbeg + (len - nbeg) * s / (nw - 1);
+// Count pass of one warp over window entries [lo, hi): per-stream counts into the warp-private
+// cntw (one predicated shared reduction per request; same-address reductions of a warp are
+// combined by the hardware), and validation of every entry: model id, arrival < trace_len, and
+// arrival >= its predecessor (window entry 0 against prev0, the entry before the window, if any).
+// Every adjacent pair of a replica's trace lies inside some window, so this validates sortedness.
+// vec: meta and arrivals are 16-byte aligned at the same element index, so the body takes 16
+// consecutive requests per lane (one 16-byte meta load, four 16-byte arrival loads).
+__device__ __forceinline__ void count_check_one(const uint8_t* meta, const uint32_t* arr, int64_t i,
+                                                bool valid, bool has_prev0, uint32_t prev0,
+                                                uint32_t tlm1, uint32_t cb, const uint16_t* klut,
+                                                bool& bad) {
+  const int kv = klut[valid ? meta[i] : 0];
+  const uint32_t a = valid ? arr[i] : 0u;
+  const uint32_t ap = (valid && i > 0) ? arr[i - 1] : (has_prev0 ? prev0 : 0u);
+  bad |= valid && ((kv & 0x8000) != 0 || a > tlm1 || a < ap);
+  red_shared_if(valid, cb + 4u * (uint32_t)(kv & 0x7FFF), 1u);
+}
+
+__device__ __forceinline__ bool count_segment(const uint8_t* meta, const uint32_t* arr, int64_t lo,
+                                              int64_t hi, bool vec, bool has_prev0, uint32_t prev0,
+                                              uint32_t tlm1, int* cntw, const uint16_t* klut) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t cb = (uint32_t)__cvta_generic_to_shared(cntw);
+  bool bad = false;
+  const int64_t h = vec ? min(hi, lo + (int64_t)((16u - ((uint32_t)(uintptr_t)(meta + lo) & 15u)) & 15u)) : hi;
+#pragma unroll 1
+  for (int64_t i0 = lo; i0 < h; i0 += 32)  // unaligned head (< 16 entries), or everything (!vec)
+    count_check_one(meta, arr, i0 + lane, i0 + lane < h, has_prev0, prev0, tlm1, cb, klut, bad);
+  if (vec) {
+    const int nch = (int)((hi - h) >> 4);
+    const uint4* gv = reinterpret_cast<const uint4*>(meta + h);
+    const uint4* ga = reinterpret_cast<const uint4*>(arr + h);
+#pragma unroll 1
+    for (int c0 = 0; c0 < nch; c0 += 32) {
+      const int ch = c0 + lane;
+      const bool valid = ch < nch;
+      uint4 v = make_uint4(0u, 0u, 0u, 0u), a0 = v, a1 = v, a2 = v, a3 = v;
+      uint32_t ap = 0u;
+      if (valid) {
+        v = gv[ch];
+        a0 = ga[4 * ch];
+        a1 = ga[4 * ch + 1];
+        a2 = ga[4 * ch + 2];
+        a3 = ga[4 * ch + 3];
+        const int64_t i = h + 16 * (int64_t)ch;
+        ap = i > 0 ? arr[i - 1] : (has_prev0 ? prev0 : 0u);
+      }
+      const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
+      const uint32_t av[16] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w,
+                               a2.x, a2.y, a2.z, a2.w, a3.x, a3.y, a3.z, a3.w};
+      uint32_t flags = 0;  // model-id flags; sortedness pairwise; the last entry is the maximum
+      bool uns = av[0] < ap;
+#pragma unroll
+      for (int q = 0; q < 16; ++q) {
+        const int kv = klut[(w4[q >> 2] >> (8 * (q & 3))) & 0xFF];
+        flags |= (uint32_t)kv;
+        if (q > 0) uns |= av[q] < av[q - 1];
+        red_shared_if(valid, cb + 4u * (uint32_t)(kv & 0x7FFF), 1u);
+      }
+      bad |= valid && ((flags & 0x8000u) != 0 || av[15] > tlm1 || uns);
+    }
+#pragma unroll 1
+    for (int64_t i0 = h + 16 * (int64_t)nch; i0 < hi; i0 += 32)  // tail (< 16 entries)
+      count_check_one(meta, arr, i0 + lane, i0 + lane < hi, has_prev0, prev0, tlm1, cb, klut, bad);
+  }
+  return bad;
+}
+
+// Stable scatter of window entries [lo, hi) (one warp) into their streams' runs of sa (entries
+// were validated by the count pass).  K = 1..4: the segment holds exactly the streams ak[0..K),
+// whose running offsets run[] live in registers and whose in-warp ranks come from one ballot each;
+// K = 0: any number of streams, ranks from match_any and warp-private running offsets in runw.
+template <int K>
+__device__ __forceinline__ void scatter_segment(const uint32_t* warr, const uint8_t* wmeta, int lo, int hi,
+                                                const uint16_t* klut, int* runw, uint32_t* sa,
+                                                const int (&ak)[4], int (&run)[4]) {
+  const int lane = threadIdx.x & 31;
+  const unsigned lt = (1u << lane) - 1u;
+#pragma unroll 1
+  for (int i0 = lo; i0 < hi; i0 += 256) {
+    uint8_t mt[8];
+    uint32_t ai[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int i = i0 + u * 32 + lane;
+      const bool valid = i < hi;
+      mt[u] = valid ? wmeta[i] : (uint8_t)0;
+      ai[u] = valid ? warr[i] : 0u;
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const bool valid = i0 + u * 32 + lane < hi;
+      const int key = klut[mt[u]] & 0x7FFF;
+      if (K > 0) {
+        int pos = 0;
+#pragma unroll
+        for (int t = 0; t < K; ++t) {
+          const bool mine = valid && key == ak[t];
+          const unsigned b = __ballot_sync(0xffffffffu, mine);
+          if (mine) pos = run[t] + __popc(b & lt);
+          run[t] += __popc(b);
+        }
+        if (valid) sa[pos] = ai[u];
+      } else {
+        const unsigned peers = __match_any_sync(0xffffffffu, valid ? key : 1024 + lane);
+        const int rank = __popc(peers & lt);
+        // the group's run of slots in stream order; its last lane advances the offset
+        const int base = runw[valid ? key : 0];
+        if (valid) sa[base + rank] = ai[u];
+        if (valid && (peers >> lane) == 1u) runw[key] = base + rank + 1;
+        __syncwarp();
+      }
+    }
   }
 }
 
@@ -542,7 +614,6 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
   __shared__ uint16_t klut[256];        // meta byte -> stream key (| 0x8000 if invalid)
   __shared__ int s_cnt[kNSeg * kMaxStreams], s_run[kNSeg * kMaxStreams];
   __shared__ int s_base[kMaxStreams], s_tot[kMaxStreams], s_skip[kMaxStreams], s_pend[kMaxStreams];
-  __shared__ int s_ge[kMaxStreams];      // carried entries per stream (previous epoch's bookkeeping)
 #ifdef PROTEAN_PHASE_TIMING
   unsigned long long ph_acc[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
   long long ph_last = clock64();
@@ -611,15 +682,12 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
     const int64_t r_lo = P.roff[r];
     const int64_t* eoff = P.eoff + (size_t)r * (P.E + 1);
     uint32_t* ghist = P.hist + (size_t)r * 2 * kNB;
-    int64_t cnt[10];
-#pragma unroll
-    for (int i = 0; i < 10; ++i) cnt[i] = 0;
 
     // ---------------------------------------------------------------- replica init
 #pragma unroll 1
     for (int i = tid; i < 2 * kNB; i += NT) s_hist[i] = 0;
 #pragma unroll 1
-    for (int k = tid; k < S; k += NT) s_skip[k] = s_ge[k] = 0;
+    for (int k = tid; k < S; k += NT) s_skip[k] = 0;
 #pragma unroll 1
     for (int g = tid; g < N; g += NT) {
       reset_gpu_state(c, g, P.init_geom);
@@ -690,26 +758,23 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       const int len = bad_window ? 0 : (int)len64;
       const uint32_t* warr = P.arr + w_lo;
       const uint8_t* wmeta = P.meta + w_lo;
-      const int nbeg = (int)(w_beg - w_lo);  // window offset of the first new request
       // ---------------------------------------------------------------- B: stream partition
-      // every warp owns one contiguous segment of the window: (1) count per (segment, stream) with
-      // 16-byte meta loads, (2) after one barrier each warp derives its own per-stream write
-      // offsets (redundant scan over streams), (3) stable scatter of its segment with 8 loads in
-      // flight per lane, validating every request once (when it is new).
-      int sa_lo, sa_hi;
+      // every warp owns one contiguous 1/NW of the window: (1) it counts its segment per stream
+      // (16-byte meta loads, match_any aggregation), (2) after one barrier derives its own
+      // per-stream write offsets (redundant scan over streams), (3) scatters its segment stably with
+      // 8 loads in flight per lane, validating every request once (when it is new).  The window is
+      // L2-resident (prefetched during the previous epoch); offsets are warp-private, so the
+      // scatter needs no atomics.
+      const int sa_lo = (int)((int64_t)len * warp / NW), sa_hi = (int)((int64_t)len * (warp + 1) / NW);
       {
-        int64_t lo64, hi64;
-        seg_bounds(nbeg, len, warp, NW, &lo64, &hi64);
-        sa_lo = (int)lo64;
-        sa_hi = (int)hi64;
-      }
-      // per (segment, stream) counts: segment 0 = carried (previous epoch), 1..NW-1 = new requests
-      // counted ahead by epoch_count_kernel
-      {
-        const uint32_t* tb = P.ecnt + (((size_t)r * P.E + e) * (NW - 1)) * S;
+        int* cntw = s_cnt + warp * S;
 #pragma unroll 1
-        for (int i = tid; i < NW * S; i += NT)
-          s_cnt[i] = bad_window ? 0 : (i < S ? s_ge[i] : (int)tb[i - S]);
+        for (int k = lane; k < S; k += 32) cntw[k] = 0;
+        __syncwarp();
+        if (sa_hi > sa_lo &&
+            count_segment(wmeta, warr, sa_lo, sa_hi, P.vec_ok, w_lo > r_lo, w_lo > r_lo ? P.arr[w_lo - 1] : 0u,
+                          (uint32_t)(P.trace_len - 1), cntw, klut))  // arrivals < trace_len <= 2^32 (host check)
+          atomicOr(P.err, 1);
       }
       __syncthreads();
       PH(1);
@@ -745,38 +810,28 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           carry += __shfl_sync(0xffffffffu, x, 31);
         }
         __syncwarp();
-        uint32_t* sa = c.sarr;
-        uint32_t prev_last = (sa_lo > 0) ? warr[sa_lo - 1] : (w_lo > r_lo ? P.arr[w_lo - 1] : 0u);
+        // the streams present in this warp's segment: <= 4 take the ballot path
+        int K = 0, ak[4] = {0, 0, 0, 0}, run[4] = {0, 0, 0, 0};
 #pragma unroll 1
-        for (int i0 = sa_lo; i0 < sa_hi; i0 += 256) {
-          uint8_t mt[8];
-          uint32_t ai[8];
+        for (int k0 = 0; k0 < S; k0 += 32) {
+          unsigned pres = __ballot_sync(0xffffffffu, k0 + lane < S && s_cnt[warp * S + k0 + lane] > 0);
+#pragma unroll 1
+          while (pres) {
+            const int k = k0 + __ffs(pres) - 1;
+            pres &= pres - 1;
 #pragma unroll
-          for (int u = 0; u < 8; ++u) {
-            const int i = i0 + u * 32 + lane;
-            const bool valid = i < sa_hi;
-            mt[u] = valid ? wmeta[i] : (uint8_t)0;
-            ai[u] = valid ? warr[i] : 0xFFFFFFFFu;
+            for (int t = 0; t < 4; ++t)
+              if (K == t) { ak[t] = k; run[t] = runw[k]; }
+            ++K;
           }
-#pragma unroll
-          for (int u = 0; u < 8; ++u) {
-            const int i = i0 + u * 32 + lane;
-            const bool valid = i < sa_hi;
-            uint32_t ap = __shfl_up_sync(0xffffffffu, ai[u], 1);
-            if (lane == 0) ap = prev_last;
-            prev_last = __shfl_sync(0xffffffffu, ai[u], 31);
-            const int kv = klut[mt[u]];
-            if (valid && i >= nbeg &&  // validate each request once (when it is new)
-                ((kv & 0x8000) || (int64_t)ai[u] >= P.trace_len || ai[u] < ap))
-              atomicOr(P.err, 1);
-            const int key = valid ? (kv & 0x7FFF) : 1024 + lane;
-            const unsigned peers = __match_any_sync(0xffffffffu, key);
-            const unsigned rank = __popc(peers & ((1u << lane) - 1u));
-            int base = 0;  // the group leader reserves the group's run of slots in stream order
-            if (valid && rank == 0) base = atomicAdd(&runw[key], __popc(peers));
-            base = __shfl_sync(0xffffffffu, base, __ffs(peers) - 1);
-            if (valid) sa[base + (int)rank] = ai[u];
-          }
+        }
+        switch (K) {
+          case 0: break;
+          case 1: scatter_segment<1>(warr, wmeta, sa_lo, sa_hi, klut, runw, c.sarr, ak, run); break;
+          case 2: scatter_segment<2>(warr, wmeta, sa_lo, sa_hi, klut, runw, c.sarr, ak, run); break;
+          case 3: scatter_segment<3>(warr, wmeta, sa_lo, sa_hi, klut, runw, c.sarr, ak, run); break;
+          case 4: scatter_segment<4>(warr, wmeta, sa_lo, sa_hi, klut, runw, c.sarr, ak, run); break;
+          default: scatter_segment<0>(warr, wmeta, sa_lo, sa_hi, klut, runw, c.sarr, ak, run); break;
         }
       }
       __syncthreads();
@@ -882,10 +937,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       // next window: stream entries at/after the earliest open batch's first arrival are re-read
 #pragma unroll 1
       for (int k = tid; k < S; k += NT) {
-        if (bad_window) {  // the next window starts at w_end: nothing carried
-          s_ge[k] = 0;
-          continue;
-        }
+        if (bad_window) continue;  // the next window starts at w_end: nothing carried
         const int b0 = s_base[k], tot = s_tot[k];
         int lo = 0, hi = tot;
 #pragma unroll 1
@@ -894,8 +946,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           if (sarr[b0 + mid] >= amin) hi = mid; else lo = mid + 1;
         }
         if (lo) atomicAdd(reinterpret_cast<unsigned long long*>(&cs.lt_total), (unsigned long long)lo);
-        s_skip[k] = tot - lo - s_pend[k];
-        s_ge[k] = tot - lo;  // the next window re-reads these (arrival >= amin): its segment 0
+        s_skip[k] = tot - lo - s_pend[k];  // the next window re-reads entries with arrival >= amin
       }
       Bat* bats = c.bats;
       uint32_t* ord = c.ord;
@@ -1074,13 +1125,6 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           const int nreq = bt.info & 0xFFFF, m = (bt.info >> 16) & 0xFF;
           const bool strict = (bt.info >> 24) & 1;
           if (lane == 0) {
-            if (strict) {
-              cnt[0] += nreq;
-              if (bt.drop) cnt[3] += nreq;
-            } else {
-              cnt[4] += nreq;
-              if (bt.drop) cnt[6] += nreq;
-            }
             const int64_t row = cs.nlog + rk;
             if (P.log && row < P.log_cap) {
               protean_batch_rec rec;
@@ -1098,38 +1142,51 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
               P.log[(size_t)r * P.log_cap + row] = rec;
             }
           }
-          if (!bt.drop) {  // latencies are non-increasing along the sorted members: runs of equal
-            const int64_t slo = T.slo[m];  // buckets become one histogram update
+          int met = 0;  // strict members within the SLO (lane 0's count)
+          if (!bt.drop) {
+            const int64_t slo = T.slo[m];
             const int cls = strict ? 0 : kNB;
             const uint32_t* ma = sarr + bt.pos;
             const int64_t bend = bt.end;
+            const uint32_t hb = (uint32_t)__cvta_generic_to_shared(s_hist + cls);
+            if (bend - (int64_t)ma[0] <= (int64_t)0xFFFFFFFFLL) {
+              // every latency end - a (>= 0, <= end - a_first) fits 32 bits: lat = end - a mod 2^32;
+              // bucket = 128 s + (lat >> s), s = max(0, floor(log2 lat) - 7) (O7, reading Q30)
+              const uint32_t e32 = (uint32_t)bend;
+              const uint32_t slo32 = slo > (int64_t)0xFFFFFFFFLL ? 0xFFFFFFFFu : (uint32_t)slo;
 #pragma unroll 1
-            for (int i0 = 0; i0 < nreq; i0 += 32) {
-              const int i = i0 + lane;
-              const bool valid = i < nreq;
-              const int64_t lat = valid ? bend - (int64_t)ma[i] : 0;
-              const int bk = valid ? lat_bucket(lat) : -1;
-              const int prev = __shfl_up_sync(0xffffffffu, bk, 1);
-              const bool head = valid && (lane == 0 || prev != bk);
-              const unsigned heads = __ballot_sync(0xffffffffu, head);
-              const unsigned vmask = __ballot_sync(0xffffffffu, valid);
-              const unsigned met = __ballot_sync(0xffffffffu, valid && lat <= slo);
-              if (head) {
-                const unsigned after = heads & ~((2u << lane) - 1u);
-                const int stop = after ? __ffs(after) - 1 : 32 - __clz(vmask);
-                atomicAdd(&s_hist[cls + bk], (uint32_t)(stop - lane));
+              for (int i0 = 0; i0 < nreq; i0 += 32) {
+                const int i = i0 + lane;
+                const bool valid = i < nreq;
+                const uint32_t lat = e32 - ma[valid ? i : 0];
+                const int sh = max(24 - __clz(lat), 0);
+                red_shared_if(valid, hb + 4u * (uint32_t)((sh << 7) + (int)(lat >> sh)), 1u);
+                met += __popc(__ballot_sync(0xffffffffu, valid && lat <= slo32));
               }
-              if (lane == 0) {
-                if (strict) {
-                  cnt[1] += __popc(met);
-                  cnt[2] += __popc(vmask) - __popc(met);
-                } else {
-                  cnt[5] += __popc(vmask);
-                }
+            } else {  // some latency >= 2^32 us: the saturating 64-bit bucket
+#pragma unroll 1
+              for (int i0 = 0; i0 < nreq; i0 += 32) {
+                const int i = i0 + lane;
+                const bool valid = i < nreq;
+                const int64_t lat = bend - (int64_t)ma[valid ? i : 0];
+                red_shared_if(valid, hb + 4u * (uint32_t)lat_bucket(lat), 1u);
+                met += __popc(__ballot_sync(0xffffffffu, valid && lat <= slo));
               }
             }
           }
-      
+          if (lane == 0) {
+            if (strict) {
+              atomicAdd(&cs.cnt[0], (unsigned long long)nreq);
+              if (bt.drop) atomicAdd(&cs.cnt[3], (unsigned long long)nreq);
+              else {
+                atomicAdd(&cs.cnt[1], (unsigned long long)met);
+                atomicAdd(&cs.cnt[2], (unsigned long long)(nreq - met));
+              }
+            } else {
+              atomicAdd(&cs.cnt[4], (unsigned long long)nreq);
+              atomicAdd(&cs.cnt[bt.drop ? 6 : 5], (unsigned long long)nreq);
+            }
+          }
           continue;
         }
         const bool actual = u < n_aunits;
@@ -1315,8 +1372,8 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           } else {
             c.gu8[2 * c.N + g] = 0;
           }
-          cnt[8] += (int64_t)(c.g_off[g + 1] - c.g_off[g]) * sum_slots;
-          cnt[9] += Gc;
+          atomicAdd(&cs.cnt[8], (unsigned long long)(c.g_off[g + 1] - c.g_off[g]) * (unsigned long long)sum_slots);
+          atomicAdd(&cs.cnt[9], (unsigned long long)Gc);
         }
         if (P.decisions) P.decisions[((size_t)r * P.E + e) * N + g] = dec_out;
         if (P.policy != 0 && P.cand_keys) {
@@ -1354,7 +1411,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
             c.gi[0 * c.N + pick] = Tend;
             c.gi[1 * c.N + pick] = drain_end + P.reconfig_us;
             c.gu8[1 * c.N + pick] = c.gu8[6 * c.N + pick];
-            cnt[7] += 1;
+            cs.cnt[7] += 1;
             --free_slots;
           }
         }
@@ -1367,9 +1424,6 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
     // ---------------------------------------------------------------- finalize (O12)
 #pragma unroll 1
     for (int g = tid; g < N; g += NT) bill_switch(c, g, VM_NONE, P.H, P.H);
-#pragma unroll
-    for (int i = 0; i < 10; ++i)
-      if (cnt[i]) atomicAdd(&cs.cnt[i], (unsigned long long)cnt[i]);
 #pragma unroll 1
     for (int w = tid; w < 2 * kNB; w += NT) ghist[w] = s_hist[w];  // histogram to HBM
     __syncthreads();
@@ -1443,43 +1497,6 @@ extern "C" int protean_debug_phase_cycles(unsigned long long* out) {
 }
 #endif
 
-// Per-(replica, epoch, segment, stream) counts of each epoch's new requests, segments as in
-// seg_bounds (nbeg = 0): warp per (replica, epoch, segment).  Consumed by the replay's stable
-// stream partition, which therefore needs no count pass of its own.
-__global__ void __launch_bounds__(256) epoch_count_kernel(const uint8_t* meta, const int64_t* eoff,
-                                                          int R, int64_t E, int nseg, int S, int M,
-                                                          uint32_t* table) {
-  __shared__ uint16_t klut[256];
-  __shared__ int cnt[8][kMaxStreams];
-  for (int b = threadIdx.x; b < 256; b += blockDim.x) {
-    const int m = b & 63;
-    const bool ok = !(b & 0x40) && m < M;
-    klut[b] = (uint16_t)((2 * (ok ? m : 0) + ((b >> 7) ? 0 : 1)) | (ok ? 0 : 0x8000));
-  }
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  for (int k = lane; k < S; k += 32) cnt[warp][k] = 0;
-  __syncthreads();
-  const int64_t idx = (int64_t)blockIdx.x * 8 + warp;  // (r, e, seg)
-  if (idx >= (int64_t)R * E * nseg) return;
-  const int64_t re = idx / nseg;
-  const int sg = (int)(idx - re * nseg) + 1;
-  const int r = (int)(re / E);
-  const int64_t e = re - (int64_t)r * E;
-  const int64_t A = eoff[(size_t)r * (E + 1) + e], B = eoff[(size_t)r * (E + 1) + e + 1];
-  int64_t lo, hi;
-  seg_bounds(0, B - A, sg, nseg + 1, &lo, &hi);
-  if (hi > lo) count_segment(meta + A, lo, hi, cnt[warp], klut);
-  __syncwarp();
-  for (int k = lane; k < S; k += 32) table[(size_t)idx * S + k] = (uint32_t)cnt[warp][k];
-}
-
-cudaError_t launch_epoch_count(const uint8_t* meta, const int64_t* eoff, int R, int64_t E, int nseg,
-                               int S, int M, uint32_t* table, cudaStream_t st) {
-  const int64_t warps = (int64_t)R * E * nseg;
-  epoch_count_kernel<<<(unsigned)((warps + 7) / 8), 256, 0, st>>>(meta, eoff, R, E, nseg, S, M, table);
-  return cudaGetLastError();
-}
-
 // Prepass: eoff[r][e] = first request of replica r with arrival >= e*W (e = 0..E), and the
 // largest request window any epoch needs: [lower_bound(eW - maxT), eoff[e+1]).
 __global__ void prepass_kernel(const uint32_t* arr, const int64_t* roff, int R, int64_t E,
@@ -1547,7 +1564,6 @@ cudaError_t preload_kernels() {
   cudaFuncAttributes a;
   cudaError_t e = cudaFuncGetAttributes(&a, replay_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, prepass_kernel);
-  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, epoch_count_kernel);
   if (e == cudaSuccess) e = raise_dyn_smem_once();
   return e;
 }

@@ -76,8 +76,8 @@ struct ReplayParams {
   const uint8_t* meta;
   const int64_t* roff;
   const int64_t* eoff;     // [R][E+1] first request index with arrival >= e*W
-  const uint32_t* ecnt;    // [R][E][NW-1][S] per-segment stream counts of each epoch's new requests
   int R, N;
+  bool vec_ok;             // arr and meta 16-byte aligned at equal element indices
   int64_t base, trace_len, W, E, H;
   // policy
   int policy, wait_limit, cap_pct, init_geom, max_live, vm_policy;
@@ -133,8 +133,6 @@ struct ScoreParams {
 cudaError_t launch_prepass(const uint32_t* arr, const int64_t* roff, int R, int64_t E, int64_t W,
                            int64_t maxT, int64_t* eoff, unsigned long long* wmax, int* err,
                            cudaStream_t st);
-cudaError_t launch_epoch_count(const uint8_t* meta, const int64_t* eoff, int R, int64_t E, int nseg,
-                               int S, int M, uint32_t* table, cudaStream_t st);
 cudaError_t launch_replay(const ReplayParams& P, int grid, int block, cudaStream_t st);
 cudaError_t replay_occupancy(int block, size_t smem, int* blocks_per_sm);
 cudaError_t preload_kernels();

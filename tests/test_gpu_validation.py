@@ -1,0 +1,97 @@
+"""Request validation inside the fused replay (count pass) and unaligned trace buffers.  -m gpu.
+
+Every request is checked once per window it appears in: model id < M and no reserved bit, arrival <
+trace_len, arrival >= its predecessor (a malformed trace is PROTEAN_EINVAL, no
+partial result).  The body of the count pass reads 16 requests per lane with 16-byte loads, so the
+faults are planted at positions that cover the unaligned head, the vector body (inside a 16-entry
+group, across groups, across lanes) and the tail of several windows.  Unaligned device pointers take
+the scalar path and must give the oracle's result bit for bit."""
+import numpy as np
+import pytest
+
+from gpu_common import compare, gpu_replay, oracle_replay
+from protean_inputs import concat, pack_meta, random_profiles
+
+pytestmark = pytest.mark.gpu
+
+
+def _trace(rng, n=6000, M=4, T=3_000_000):
+    a = np.sort(rng.integers(0, T, n)).astype(np.uint32)
+    return a, pack_meta(rng.integers(0, M, n), rng.integers(0, 2, n)), T
+
+
+def _code(prof, tr):
+    import paper_conf_middleware_bhasisjgpkd24_b200 as pkg
+    try:
+        h = pkg.load_profiles(prof)
+        h.replay_traces_host(tr, n_gpus=2)
+    except pkg.ProteanError as e:
+        return e.code
+    return 0
+
+
+@pytest.mark.parametrize("kind", ["unsorted", "model", "reserved_bit", "beyond_trace"])
+def test_planted_faults(oracle, kind):
+    rng = np.random.default_rng({"unsorted": 1, "model": 2, "reserved_bit": 3, "beyond_trace": 4}[kind])
+    prof = random_profiles(rng, 4)
+    a0, m0, T = _trace(rng)
+    assert _code(prof, concat([(a0, m0)], T)) == 0
+    positions = sorted({1, 2, 15, 16, 17, 31, 32, 33, 511, 512, 513, 1999, 2000, 2001, 4095, 4096,
+                        len(a0) - 2, len(a0) - 1, *rng.integers(1, len(a0), 8).tolist()})
+    for p in positions:
+        a, m = a0.copy(), m0.copy()
+        if kind == "unsorted":
+            if a[p] == 0:
+                continue
+            a[p] = a[p - 1] - 1 if a[p - 1] > 0 else 0
+            if a[p] >= a[p - 1]:
+                continue
+        elif kind == "model":
+            m[p] = (m[p] & 0x80) | 9          # model 9 >= M = 4
+        elif kind == "reserved_bit":
+            m[p] |= 0x40
+        else:
+            if p != len(a) - 1:
+                continue
+            a[p] = T                          # arrival == trace_len
+        tr = concat([(a, m)], T)
+        g = _code(prof, tr)
+        o = 0
+        try:
+            oracle_replay(oracle, prof, tr, want_keys=False, want_log=False, n_gpus=2)
+        except oracle.OracleError as e:
+            o = e.code
+        assert o != 0 and g == o, (kind, p, g, o)
+
+
+@pytest.mark.parametrize("shift", [(1, 3), (2, 0), (0, 5)])
+def test_unaligned_device_buffers(oracle, shift):
+    """arrival/meta views at 4-byte / 1-byte offsets: the scalar count path, same results."""
+    import torch
+    import paper_conf_middleware_bhasisjgpkd24_b200 as pkg
+    rng = np.random.default_rng(11)
+    prof = random_profiles(rng, 3)
+    parts = []
+    for _ in range(3):
+        a, m, T = _trace(rng, n=int(rng.integers(2000, 5000)), M=3)
+        parts.append((a, m))
+    tr = concat(parts, T)
+    sa, sm = shift
+    n = tr.arrival_us.shape[0]
+    abuf = torch.zeros(n + 8, dtype=torch.int32, device="cuda")
+    mbuf = torch.zeros(n + 16, dtype=torch.uint8, device="cuda")
+    arr = abuf[sa:sa + n]
+    meta = mbuf[sm:sm + n]
+    arr.copy_(torch.from_numpy(tr.arrival_us.view(np.int32)))
+    meta.copy_(torch.from_numpy(tr.meta))
+    off = torch.from_numpy(tr.replica_off).cuda()
+    h = pkg.load_profiles(prof)
+    out = h.replay_traces(arr, meta, off, trace_len_us=T, n_gpus=3, want_cand_keys=True, log_cap=n)
+    g = {k: (v.cpu().numpy() if hasattr(v, "cpu") else v) for k, v in out.items()}
+    g["hist"] = g["hist"].view(np.uint32)
+    from gpu_common import GPU_LOG_DTYPE
+    g["log"] = g["log"].reshape(3, n, 32).view(GPU_LOG_DTYPE).reshape(3, n)
+    compare(g, oracle_replay(oracle, prof, tr, n_gpus=3), 3)
+    ref = gpu_replay(prof, tr, n_gpus=3)
+    for k in ("counters", "hist", "cand_keys"):
+        assert np.array_equal(g[k], ref[k]), k
