@@ -626,7 +626,9 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
     BS = std::min(BS, std::max(1, std::atoi(ev)));
   }
   const size_t with_bats = fixed + (size_t)BS * (sizeof(Bat) + 8) + 64;
-  const int WS = (with_bats + (size_t)WCAP * 4 <= budget) ? WCAP : 0;  // window all in smem or all in HBM
+  int WS = (with_bats + (size_t)WCAP * 4 <= budget) ? WCAP : 0;  // window all in smem or all in HBM
+  if (const char* ev = std::getenv("PROTEAN_WINDOW_SMEM"))  // experiment knob: 0 = window in global scratch
+    if (std::atoi(ev) == 0) WS = 0;
   sl.init(h->tl.words, h->M, N, Gc, CW, BS, WS);
   if (sl.total > 227 * 1024) return fail(h, PROTEAN_ERANGE, "shared memory layout too large");
   int per_sm = 0;

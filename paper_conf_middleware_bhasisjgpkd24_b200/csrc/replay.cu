@@ -605,6 +605,117 @@ __device__ __forceinline__ void candidate_unit_regs(const Tab& T, const SliceLan
   *tail_out = tail;
 }
 
+// Candidate unit, fast path: the GPU-epoch's <= kKR batches fully unrolled, times 32-bit relative to
+// the first batch's ready time tb.  Every lane of a geometry's group keeps the whole placement so
+// far (end en[x], footprint / BE flag mm[x], FBR on the lane's own profile fb[x], and the mask of
+// batches on its own slice), so the GPU-wide quantities of Alg 1 -- live residents (reading Q39)
+// and BE memory for the tag walk (lines 1-8) -- need no shuffles; only the slice min-loc does.
+// Returns false (warp-uniform) if a completion does not fit 25 bits; the caller then re-runs the
+// unit on the 64-bit path.  Same arithmetic as candidate_unit_regs (Eq 1 exact integers, Q10-Q12).
+__device__ __forceinline__ uint32_t group_min32(uint32_t v, int Z) {
+#pragma unroll
+  for (int d = 1; d < 8; d <<= 1) {
+    const uint32_t o = __shfl_xor_sync(0xffffffffu, v, d);
+    if (d < Z && o < v) v = o;
+  }
+  return v;
+}
+
+__device__ __forceinline__ bool candidate_unit_fast(const Tab& T, const SliceLane& K, bool active,
+                                                    bool leader, const Bat* bats, const uint32_t* gl,
+                                                    int x0, int len, const uint32_t* sarr, int max_live,
+                                                    int64_t* misses_out, int64_t* tail_out) {
+  uint32_t en[kKR], mm[kKR];
+  int32_t fb[kKR];
+  uint32_t mine = 0, rls = 0;
+  bool ok = true;
+  int64_t misses = 0, tail = 0;
+  const int lane = threadIdx.x & 31;
+  const int gbase = lane & ~(K.Z - 1);
+  const uint32_t tb = len > 0 ? bats[gl[x0]].ready : 0u;
+#pragma unroll
+  for (int x = 0; x < kKR; ++x) {
+    if (x >= len) break;
+    const Bat& bt = bats[gl[x0 + x]];
+    const uint32_t info = bt.info;
+    const int m = (info >> 16) & 0xFF, nreq = info & 0xFFFF;
+    const bool strict = (info >> 24) & 1;
+    const uint32_t rt = bt.ready - tb;
+    const uint32_t rt0 = rt > rls ? rt : rls;
+    int32_t used = 0, be = 0, live = 0, fs = 0;
+#pragma unroll
+    for (int i = 0; i < x; ++i) {
+      const bool alive = en[i] > rt;
+      live += alive ? 1 : 0;
+      if (alive && (mm[i] >> 16)) be += (int32_t)(mm[i] & 0xFFFF);
+      if (((mine >> i) & 1u) && en[i] > rt0) {
+        used += (int32_t)(mm[i] & 0xFFFF);
+        fs += fb[i];
+      }
+    }
+    const int32_t q = T.mem[m];
+    const int32_t fbm = K.fbr_p[m * kNProf];
+    const bool overflow = live >= max_live;
+    uint32_t key = 0xFFFFFFFFu, start = 0, c = 0;
+    if (active && !overflow && q <= K.Ms) {
+      int64_t F = fbm;
+      if (used + q <= K.Ms) {
+        start = rt0;
+        F += fs;
+      } else {  // memory wait: the earliest release on this slice after which the batch fits
+        start = 0xFFFFFFFFu;
+#pragma unroll
+        for (int jj = 0; jj < x; ++jj) {
+          if (((mine >> jj) & 1u) && en[jj] > rt0) {
+            int32_t rem = 0;
+#pragma unroll
+            for (int i = 0; i < x; ++i)
+              if (((mine >> i) & 1u) && en[i] > en[jj]) rem += (int32_t)(mm[i] & 0xFFFF);
+            if (rem + q <= K.Ms && en[jj] < start) start = en[jj];
+          }
+        }
+#pragma unroll
+        for (int i = 0; i < x; ++i)
+          if (((mine >> i) & 1u) && en[i] > start) F += fb[i];
+      }
+      const int64_t c64 = (int64_t)start + exec_time(K.solo_p[m * kNProf], F);
+      ok &= c64 < (int64_t)(1 << 25);
+      c = (uint32_t)c64;
+      key = strict ? (((be >= K.pref) ? 0x80000000u : 0u) | (c << 6) | ((uint32_t)(4 - K.p) << 3) | (uint32_t)K.s)
+                   : ((start << 3) | (uint32_t)K.s);
+    }
+    const uint32_t kmin = group_min32(key, K.Z);
+    const bool placed = !overflow && kmin != 0xFFFFFFFFu;
+    const uint32_t cwin = __shfl_sync(0xffffffffu, c, (gbase + (int)(kmin & 7)) & 31);
+    en[x] = placed ? cwin : 0u;
+    mm[x] = (uint32_t)q | (strict ? 0u : 0x10000u);
+    fb[x] = fbm;
+    if (placed && key == kmin) {  // schedule(batch, chosen_slice)
+      mine |= 1u << x;
+      rls = start;
+    }
+    if (leader) {
+      const int64_t cw = (int64_t)tb + (int64_t)cwin;
+      if (strict) {
+        if (!placed) {
+          misses += nreq;
+        } else {  // latencies fall along the sorted members: test the ends first
+          const uint32_t* ma = sarr + bt.pos;
+          const int64_t slo = T.slo[m];
+          if (cw - (int64_t)ma[0] > slo)
+            misses += (cw - (int64_t)ma[nreq - 1] > slo) ? nreq : nreq - hits_in(ma, nreq, cw, slo);
+        }
+      } else {
+        const int64_t tbv = placed ? cw - (int64_t)sarr[bt.pos] : (int64_t)0xFFFFFFFFLL;
+        tail = tbv > tail ? tbv : tail;
+      }
+    }
+  }
+  *misses_out = misses;
+  *tail_out = tail;
+  return __all_sync(0xffffffffu, ok);
+}
+
 }  // namespace
 
 __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams P) {
@@ -1248,8 +1359,10 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
         if (!actual && len_max <= kKR) {  // register-resident candidate lists
           int64_t misses, tail;
           // warp-uniform batch range (idle lanes must still take part in the group shuffles)
-          candidate_unit_regs(T, K, active, lane == gbase && valid, bats, gl, c.g_off[g],
-                              c.g_off[g + 1], sarr, P.max_live, &misses, &tail);
+          if (!candidate_unit_fast(T, K, active, lane == gbase && valid, bats, gl, c.g_off[g],
+                                   c.g_off[g + 1] - c.g_off[g], sarr, P.max_live, &misses, &tail))
+            candidate_unit_regs(T, K, active, lane == gbase && valid, bats, gl, c.g_off[g],
+                                c.g_off[g + 1], sarr, P.max_live, &misses, &tail);
           if (valid && lane == gbase) {
             const int64_t key = make_key(misses, tail, j == c.gu8[0 * c.N + g] ? 0 : j + 1);
             if (j == c.gu8[0 * c.N + g]) c.gi[7 * c.N + g] = key;

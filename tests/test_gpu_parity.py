@@ -245,3 +245,19 @@ def test_score_epoch_fuzz(oracle, seed):
                 (b.start, b.end, b.mem, b.slice, b.model, b.strict)
         assert list(st[x].last_start_us) == list(ostates[x].last_start)
         assert list(st[x].busy_until_us) == list(ostates[x].busy_until)
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_long_jobs_wide_times(oracle, seed):
+    """Solo times of tens of seconds: candidate completions beyond 2^25 us from the first ready
+    time of the GPU-epoch force the 64-bit candidate path on some units (the fast path is 32-bit
+    relative); overloaded slices also exercise the memory-wait branch.  Bit-exact vs the oracle."""
+    rng = np.random.default_rng(900 + seed)
+    M = 3
+    solo7 = rng.integers(5_000_000, 40_000_000, M)
+    prof = tables(np.stack([solo7 * f for f in (6, 4, 3, 2, 1)], 1), rng.integers(200_000, 1_000_000, (M, 5)),
+                  rng.integers(2_000, 12_000, M), bsz=[2, 3, 1], slo=3 * solo7, tmo=[0, 500_000, 0])
+    tr = uniform_trace(rng, 3, M, 120_000_000, 60)
+    for N in (1, 3):
+        g = gpu_replay(prof, tr, n_gpus=N)
+        compare(g, oracle_replay(oracle, prof, tr, n_gpus=N), 3)
