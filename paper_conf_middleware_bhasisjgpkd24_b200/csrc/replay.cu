@@ -371,10 +371,11 @@ __device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, const
   return o;
 }
 
-// Predicated shared-memory reduction (keeps the per-element loops free of branches).
-__device__ __forceinline__ void red_shared_if(bool p, uint32_t saddr, uint32_t v) {
-  asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.shared.add.u32 [%0], %1;\n\t}"
-               ::"r"(saddr), "r"(v), "r"((uint32_t)p) : "memory");
+// Shared-memory increment by exactly 1, unpredicated (ptxas aggregates a warp's same-address
+// increments, ATOMS.POPC.INC); lanes with nothing to count increment a sink word instead, which
+// keeps the per-element loops free of branches.
+__device__ __forceinline__ void inc_shared(uint32_t saddr) {
+  asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(saddr) : "memory");
 }
 
 // Count pass of one warp over window entries [lo, hi): per-stream counts into the warp-private
@@ -386,25 +387,25 @@ __device__ __forceinline__ void red_shared_if(bool p, uint32_t saddr, uint32_t v
 // consecutive requests per lane (one 16-byte meta load, four 16-byte arrival loads).
 __device__ __forceinline__ void count_check_one(const uint8_t* meta, const uint32_t* arr, int64_t i,
                                                 bool valid, bool has_prev0, uint32_t prev0,
-                                                uint32_t tlm1, uint32_t cb, const uint16_t* klut,
-                                                bool& bad) {
+                                                uint32_t tlm1, uint32_t cb, uint32_t sink,
+                                                const uint16_t* klut, bool& bad) {
   const int kv = klut[valid ? meta[i] : 0];
   const uint32_t a = valid ? arr[i] : 0u;
   const uint32_t ap = (valid && i > 0) ? arr[i - 1] : (has_prev0 ? prev0 : 0u);
   bad |= valid && ((kv & 0x8000) != 0 || a > tlm1 || a < ap);
-  red_shared_if(valid, cb + 4u * (uint32_t)(kv & 0x7FFF), 1u);
+  inc_shared(valid ? cb + 4u * (uint32_t)(kv & 0x7FFF) : sink);
 }
 
 __device__ __forceinline__ bool count_segment(const uint8_t* meta, const uint32_t* arr, int64_t lo,
                                               int64_t hi, bool vec, bool has_prev0, uint32_t prev0,
-                                              uint32_t tlm1, int* cntw, const uint16_t* klut) {
+                                              uint32_t tlm1, int* cntw, uint32_t sink, const uint16_t* klut) {
   const int lane = threadIdx.x & 31;
   const uint32_t cb = (uint32_t)__cvta_generic_to_shared(cntw);
   bool bad = false;
   const int64_t h = vec ? min(hi, lo + (int64_t)((16u - ((uint32_t)(uintptr_t)(meta + lo) & 15u)) & 15u)) : hi;
 #pragma unroll 1
   for (int64_t i0 = lo; i0 < h; i0 += 32)  // unaligned head (< 16 entries), or everything (!vec)
-    count_check_one(meta, arr, i0 + lane, i0 + lane < h, has_prev0, prev0, tlm1, cb, klut, bad);
+    count_check_one(meta, arr, i0 + lane, i0 + lane < h, has_prev0, prev0, tlm1, cb, sink, klut, bad);
   if (vec) {
     const int nch = (int)((hi - h) >> 4);
     const uint4* gv = reinterpret_cast<const uint4*>(meta + h);
@@ -434,13 +435,13 @@ __device__ __forceinline__ bool count_segment(const uint8_t* meta, const uint32_
         const int kv = klut[(w4[q >> 2] >> (8 * (q & 3))) & 0xFF];
         flags |= (uint32_t)kv;
         if (q > 0) uns |= av[q] < av[q - 1];
-        red_shared_if(valid, cb + 4u * (uint32_t)(kv & 0x7FFF), 1u);
+        inc_shared(valid ? cb + 4u * (uint32_t)(kv & 0x7FFF) : sink);
       }
       bad |= valid && ((flags & 0x8000u) != 0 || av[15] > tlm1 || uns);
     }
 #pragma unroll 1
     for (int64_t i0 = h + 16 * (int64_t)nch; i0 < hi; i0 += 32)  // tail (< 16 entries)
-      count_check_one(meta, arr, i0 + lane, i0 + lane < hi, has_prev0, prev0, tlm1, cb, klut, bad);
+      count_check_one(meta, arr, i0 + lane, i0 + lane < hi, has_prev0, prev0, tlm1, cb, sink, klut, bad);
   }
   return bad;
 }
@@ -722,6 +723,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ CtaState cs;
   __shared__ uint32_t s_hist[2 * kNB];  // 2 classes x 3328 buckets (u32 < 2^32 per replica)
+  __shared__ uint32_t s_sink;           // target of increments with nothing to count
   __shared__ uint16_t klut[256];        // meta byte -> stream key (| 0x8000 if invalid)
   __shared__ int s_cnt[kNSeg * kMaxStreams], s_run[kNSeg * kMaxStreams];
   __shared__ int s_base[kMaxStreams], s_tot[kMaxStreams], s_skip[kMaxStreams], s_pend[kMaxStreams];
@@ -731,6 +733,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
 #endif
   const SmemLayout& SL = P.sl;
   const int tid = threadIdx.x, NT = blockDim.x, lane = tid & 31, warp = tid >> 5, NW = NT >> 5;
+  const uint32_t sink = (uint32_t)__cvta_generic_to_shared(&s_sink);
   const int N = P.N, S = SL.S, Gc = SL.Gc, CW = SL.CW;
 
   Ctx c;
@@ -884,7 +887,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
         __syncwarp();
         if (sa_hi > sa_lo &&
             count_segment(wmeta, warr, sa_lo, sa_hi, P.vec_ok, w_lo > r_lo, w_lo > r_lo ? P.arr[w_lo - 1] : 0u,
-                          (uint32_t)(P.trace_len - 1), cntw, klut))  // arrivals < trace_len <= 2^32 (host check)
+                          (uint32_t)(P.trace_len - 1), cntw, sink, klut))  // arrivals < trace_len <= 2^32 (host check)
           atomicOr(P.err, 1);
       }
       __syncthreads();
@@ -1271,7 +1274,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
                 const bool valid = i < nreq;
                 const uint32_t lat = e32 - ma[valid ? i : 0];
                 const int sh = max(24 - __clz(lat), 0);
-                red_shared_if(valid, hb + 4u * (uint32_t)((sh << 7) + (int)(lat >> sh)), 1u);
+                inc_shared(valid ? hb + 4u * (uint32_t)((sh << 7) + (int)(lat >> sh)) : sink);
                 met += __popc(__ballot_sync(0xffffffffu, valid && lat <= slo32));
               }
             } else {  // some latency >= 2^32 us: the saturating 64-bit bucket
@@ -1280,7 +1283,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
                 const int i = i0 + lane;
                 const bool valid = i < nreq;
                 const int64_t lat = bend - (int64_t)ma[valid ? i : 0];
-                red_shared_if(valid, hb + 4u * (uint32_t)lat_bucket(lat), 1u);
+                inc_shared(valid ? hb + 4u * (uint32_t)lat_bucket(lat) : sink);
                 met += __popc(__ballot_sync(0xffffffffu, valid && lat <= slo));
               }
             }
