@@ -15,6 +15,15 @@
 #include <mutex>
 
 #include "replay.cuh"
+#ifndef PROTEAN_A_BARRIER
+#define PROTEAN_A_BARRIER 0
+#endif
+#ifndef PROTEAN_D_BARRIER
+#define PROTEAN_D_BARRIER 1
+#endif
+#ifndef PROTEAN_WARP_G
+#define PROTEAN_WARP_G 1
+#endif
 #ifndef PROTEAN_MINB
 #define PROTEAN_MINB 3
 #endif
@@ -817,6 +826,12 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       cs.nlog = 0;
       cs.cursor = 0;
       cs.bad = 0;
+      cs.task = 0;  // per-epoch scratch, re-armed at the end of every epoch
+      cs.adone = 0;
+      cs.nb = 0;
+      cs.amin = 0xFFFFFFFFu;
+      cs.lt_total = 0;
+      cs.all_avail = 1;
 #pragma unroll
       for (int i = 0; i < 10; ++i) cs.cnt[i] = 0;
     }
@@ -842,15 +857,13 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
         c.gu8[7 * c.N + g] = 0;
         c.gu8[6 * c.N + g] = kNoGeom;
         c.gi[7 * c.N + g] = -1;
+        const bool whole = c.gi[2 * c.N + g] <= eW && c.gi[3 * c.N + g] >= Tend &&
+                           !(c.gi[0 * c.N + g] < Tend && c.gi[1 * c.N + g] > eW);
+        if (!whole) cs.all_avail = 0;  // set to 1 before the previous epoch's last barrier
       }
-      if (tid == 0) {
-        cs.task = 0;
-        cs.adone = 0;
-        cs.nb = 0;
-        cs.amin = 0xFFFFFFFFu;
-        cs.lt_total = 0;
-        cs.all_avail = 1;
-      }
+#if PROTEAN_A_BARRIER
+      __syncthreads();
+#endif
       const int64_t w_beg = eoff[e], w_end = eoff[e + 1];
       const int64_t w_lo = cs.w_lo;
       if (tid == 32 && e + 1 < P.E) {  // the next epoch's new requests: into L2 during this one
@@ -858,14 +871,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
         prefetch_l2(P.meta + nb0, nb1 - nb0);
         prefetch_l2(P.arr + nb0, (nb1 - nb0) * 4);
       }
-      __syncthreads();
       PH(0);
-#pragma unroll 1
-      for (int g = tid; g < N; g += NT) {
-        const bool whole = c.gi[2 * c.N + g] <= eW && c.gi[3 * c.N + g] >= Tend &&
-                           !(c.gi[0 * c.N + g] < Tend && c.gi[1 * c.N + g] > eW);
-        if (!whole) cs.all_avail = 0;
-      }
       const int64_t len64 = w_end - w_lo;
       const bool bad_window = len64 < 0 || len64 > P.WCAP || w_beg < w_lo;
       if (bad_window && tid == 0) atomicOr(P.err, 1);
@@ -1042,12 +1048,12 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
         c.bats = c.gb;
         c.ord = c.gord;
         c.gl = c.ggl;
+        __syncthreads();
       } else {
         c.bats = c.sb;
         c.ord = c.sord;
         c.gl = c.sgl;
       }
-      __syncthreads();
       // next window: stream entries at/after the earliest open batch's first arrival are re-read
 #pragma unroll 1
       for (int k = tid; k < S; k += NT) {
@@ -1065,6 +1071,19 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       Bat* bats = c.bats;
       uint32_t* ord = c.ord;
       uint32_t* gl = c.gl;
+      // D (closed form, Q18) fused with the id-order ranking when every GPU is available all
+      // epoch: rank rk goes to GPU (cursor + rk) mod N, the rk / N-th of that GPU's list; GPU h
+      // receives q + [d_h < rem] batches (q, rem = nb div/mod N, d_h = (h - cursor) mod N)
+      const bool avail_all = cs.all_avail;
+      const int cursor = cs.cursor;
+      const int dq = nb / N, drem = nb - dq * N;
+      auto goff = [&](int g) {  // batches of GPUs 0..g-1
+        const int wrap = cursor + drem - N;
+        int x = g - cursor;
+        x = x < 0 ? 0 : (x > drem ? drem : x);
+        if (wrap > 0) x = min(max(g - cursor, 0), N - cursor) + min(g, wrap);
+        return g * dq + x;
+      };
 #pragma unroll 1
       for (int b = tid; b < nb; b += NT) {  // id order (O3): rank by key
         const uint64_t kb = bats[b].key;
@@ -1072,36 +1091,24 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
 #pragma unroll 4
         for (int x = 0; x < nb; ++x) rank += (bats[x].key < kb) ? 1 : 0;
         ord[rank] = (uint32_t)b;
+        if (avail_all) {
+          const int q = rank / N, g = cursor + (rank - q * N);
+          const int gg = g >= N ? g - N : g;
+          bats[b].gpu = (uint8_t)gg;
+          gl[goff(gg) + q] = (uint32_t)b;
+        }
       }
+      if (avail_all)
+        for (int g = tid; g <= N; g += NT) c.g_off[g] = goff(g);
       __syncthreads();
       PH(5);
-      if (tid == 0) cs.w_lo = bad_window ? w_end : w_lo + cs.lt_total;
+      if (tid == 0) {
+        cs.w_lo = bad_window ? w_end : w_lo + cs.lt_total;
+        if (avail_all) cs.cursor = (int)((cursor + nb) % N);
+      }
       // ---------------------------------------------------------------- D: dispatch
-      if (cs.all_avail) {
-        const int cursor = cs.cursor;
-#pragma unroll 1
-        for (int rk = tid; rk < nb; rk += NT) bats[ord[rk]].gpu = (uint8_t)((cursor + rk) % N);
-#pragma unroll 1
-        for (int g = tid; g < N; g += NT) {
-          const int d = (g - cursor % N + N) % N;
-          const int cntg = d < nb ? (nb - d + N - 1) / N : 0;
-          c.g_cnt[g] = cntg;
-          int off = 0;
-#pragma unroll 1
-          for (int h = 0; h < g; ++h) {
-            const int dh = (h - cursor % N + N) % N;
-            off += dh < nb ? (nb - dh + N - 1) / N : 0;
-          }
-          c.g_off[g] = off;
-          if (g == N - 1) c.g_off[N] = off + cntg;
-        }
-        __syncthreads();
-#pragma unroll 1
-        for (int rk = tid; rk < nb; rk += NT) {
-          const int g = (cursor + rk) % N;
-          gl[c.g_off[g] + rk / N] = ord[rk];
-        }
-        if (tid == 0) cs.cursor = (int)((cursor + nb) % N);
+      if (avail_all) {
+        // done above
       } else if (N <= 32) {
         // availability mask per batch (parallel); then runs of equal masks are dispatched in
         // closed form: inside a run the k-th batch goes to the (i0 + k) mod |A|-th available GPU
@@ -1205,7 +1212,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
         }
         cs.cursor = cur;
       }
-      __syncthreads();
+      if (PROTEAN_D_BARRIER || !avail_all) __syncthreads();  // (uniform)
       PH(6);
       // ---------------------------------------------------------------- E: placement units
       // unit < n_aunits: actual placement of GPUs 4u..4u+3 (8 slice lanes each, carried state);
@@ -1458,6 +1465,86 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       __syncthreads();
       PH(7);
       // ---------------------------------------------------------------- G: decisions (O9, O10)
+      if (PROTEAN_WARP_G && P.xl.n <= 1 && N <= 32) {
+        // one warp, lane = simulated GPU: argmin over the candidate keys, Alg 2 hysteresis, then
+        // the ~30% cap by (delta misses desc, GPU asc) as a warp argmax per pick; the other warps
+        // go straight to the epoch's last barrier
+        if (warp == 0) {
+          const int g = lane;
+          const bool gv = g < N;
+          bool want = false;
+          int64_t kb = kForever, kc = -1;
+          if (gv) {
+            uint8_t dec_out = kNoGeom;
+            if (P.policy == 0 && c.gu8[5 * c.N + g]) {
+#pragma unroll 1
+              for (int v = 0; v < Gc; ++v) kb = c.keys[g * Gc + v] < kb ? c.keys[g * Gc + v] : kb;
+              c.gi[6 * c.N + g] = kb;
+              kc = c.gi[7 * c.N + g];
+              const int cur = c.gu8[0 * c.N + g];
+              const int tag = (int)(kb & 255);
+              const int best = tag == 0 ? cur : tag - 1;
+              dec_out = (uint8_t)best;
+              c.gu8[6 * c.N + g] = (uint8_t)best;
+              if (best != cur) {
+                if (c.gu8[2 * c.N + g] >= P.wait_limit) want = true;
+                else c.gu8[2 * c.N + g]++;
+              } else {
+                c.gu8[2 * c.N + g] = 0;
+              }
+              atomicAdd(&cs.cnt[8], (unsigned long long)(c.g_off[g + 1] - c.g_off[g]) * (unsigned long long)sum_slots);
+              atomicAdd(&cs.cnt[9], (unsigned long long)Gc);
+            } else if (P.policy == 0) {
+              c.gi[6 * c.N + g] = kForever;
+            }
+            if (P.decisions) P.decisions[((size_t)r * P.E + e) * N + g] = dec_out;
+            if (P.policy != 0 && P.cand_keys) {
+#pragma unroll 1
+              for (int j = P.geom_lo; j < P.geom_hi; ++j)
+                P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = -1;
+            }
+          }
+          if (P.policy == 0) {
+            const unsigned alive = __ballot_sync(0xffffffffu, gv && has_vm(c, g, Tend));
+            const unsigned open = __ballot_sync(0xffffffffu, gv && c.gi[1 * c.N + g] > Tend);
+            int cap = P.cap_pct * __popc(alive) / 100;
+            if (cap < 1) cap = 1;
+            int free_slots = cap - __popc(open);
+            const int64_t d = want ? (kc >> 40) - (kb >> 40) : 0;
+#pragma unroll 1
+            while (free_slots > 0) {
+              const unsigned wm = __ballot_sync(0xffffffffu, want);
+              if (!wm) break;
+              int64_t best_d = want ? d : INT64_MIN;  // max d, then lowest GPU
+#pragma unroll
+              for (int o = 16; o > 0; o >>= 1) {
+                const int64_t od = __shfl_xor_sync(0xffffffffu, best_d, o);
+                best_d = od > best_d ? od : best_d;
+              }
+              const unsigned tie = __ballot_sync(0xffffffffu, want && d == best_d);
+              const int pick = __ffs(tie) - 1;
+              if (lane == pick) {
+                want = false;
+                const int64_t drain_end = c.gi[5 * c.N + g] > Tend ? c.gi[5 * c.N + g] : Tend;
+                c.gi[0 * c.N + g] = Tend;
+                c.gi[1 * c.N + g] = drain_end + P.reconfig_us;
+                c.gu8[1 * c.N + g] = c.gu8[6 * c.N + g];
+                cs.cnt[7] += 1;
+              }
+              --free_slots;
+            }
+          }
+          if (lane == 0) {
+            cs.nlog += nb;
+            cs.task = 0;  // re-arm the per-epoch scratch for the next epoch
+            cs.adone = 0;
+            cs.nb = 0;
+            cs.amin = 0xFFFFFFFFu;
+            cs.lt_total = 0;
+            cs.all_avail = 1;
+          }
+        }
+      } else {
       if (P.policy == 0) {  // S8: min over this rank's geometry range
 #pragma unroll 1
         for (int g = tid; g < N; g += NT) {
@@ -1532,6 +1619,13 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           }
         }
         cs.nlog += nb;
+        cs.task = 0;  // re-arm the per-epoch scratch for the next epoch
+        cs.adone = 0;
+        cs.nb = 0;
+        cs.amin = 0xFFFFFFFFu;
+        cs.lt_total = 0;
+        cs.all_avail = 1;
+      }
       }
       __syncthreads();
       PH(9);

@@ -1,5 +1,4 @@
 L=paper_conf_middleware_bhasisjgpkd24_b200
-python tools/variant_bench.py $L/libprotean.so
-PROTEAN_WINDOW_SMEM=0 python tools/variant_bench.py $L/libprotean.so
-python tools/variant_bench.py $L/libprotean_minb4.so
-PROTEAN_WINDOW_SMEM=0 python tools/variant_bench.py $L/libprotean_minb4.so
+for i in 1 2; do
+for v in libprotean libprotean_wg libprotean_ab; do python tools/variant_bench.py $L/$v.so 4096 120; done
+done
