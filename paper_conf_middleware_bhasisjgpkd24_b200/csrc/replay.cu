@@ -459,6 +459,7 @@ __device__ __forceinline__ bool count_segment(const uint8_t* meta, const uint32_
 // were validated by the count pass).  K = 1..4: the segment holds exactly the streams ak[0..K),
 // whose running offsets run[] live in registers and whose in-warp ranks come from one ballot each;
 // K = 0: any number of streams, ranks from match_any and warp-private running offsets in runw.
+constexpr int kSU = 4;  // requests per lane in flight per scatter step
 template <int K>
 __device__ __forceinline__ void scatter_segment(const uint32_t* warr, const uint8_t* wmeta, int lo, int hi,
                                                 const uint16_t* klut, int* runw, uint32_t* sa,
@@ -466,18 +467,18 @@ __device__ __forceinline__ void scatter_segment(const uint32_t* warr, const uint
   const int lane = threadIdx.x & 31;
   const unsigned lt = (1u << lane) - 1u;
 #pragma unroll 1
-  for (int i0 = lo; i0 < hi; i0 += 256) {
-    uint8_t mt[8];
-    uint32_t ai[8];
+  for (int i0 = lo; i0 < hi; i0 += 32 * kSU) {
+    uint8_t mt[kSU];
+    uint32_t ai[kSU];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
+    for (int u = 0; u < kSU; ++u) {
       const int i = i0 + u * 32 + lane;
       const bool valid = i < hi;
       mt[u] = valid ? wmeta[i] : (uint8_t)0;
       ai[u] = valid ? warr[i] : 0u;
     }
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
+    for (int u = 0; u < kSU; ++u) {
       const bool valid = i0 + u * 32 + lane < hi;
       const int key = klut[mt[u]] & 0x7FFF;
       if (K > 0) {
@@ -503,117 +504,7 @@ __device__ __forceinline__ void scatter_segment(const uint32_t* warr, const uint
   }
 }
 
-// Candidate unit with register-resident slice lists (the GPU-epoch has <= kKR batches, so no lane
-// ever holds more residents).  Replay states are FIFO-consistent, so every resident started at or
-// before the slice's last start: Eq 1's co-runners at an instant x >= t0 are exactly the residents
-// with end > x, and start times need not be kept.  Ended residents (end <= t) are simply ignored.
-constexpr int kKR = 6;
-__device__ __forceinline__ void candidate_unit_regs(const Tab& T, const SliceLane& K, bool active,
-                                                    bool leader, const Bat* bats, const uint32_t* gl,
-                                                    int x0, int x1, const uint32_t* sarr, int max_live,
-                                                    int64_t* misses_out, int64_t* tail_out) {
-  int64_t en_r[kKR];
-  uint32_t mm_r[kKR];
-#pragma unroll
-  for (int i = 0; i < kKR; ++i) { en_r[i] = 0; mm_r[i] = 0; }
-  int n = 0;
-  int64_t ls = 0, misses = 0, tail = 0;
-  const int lane = threadIdx.x & 31;
-  const int gbase = lane & ~(K.Z - 1);
-#pragma unroll 1
-  for (int x = x0; x < x1; ++x) {
-    const Bat& bt = bats[gl[x]];
-    const uint32_t info = bt.info;
-    const int m = (info >> 16) & 0xFF, nreq = info & 0xFFFF;
-    const bool strict = (info >> 24) & 1;
-    const int64_t t = bt.ready;
-    const int64_t t0 = t > ls ? t : ls;
-    int32_t used = 0, be = 0, live = 0;
-    int64_t fs = 0;
-    const int nw = __reduce_max_sync(0xffffffffu, (unsigned)n);  // warp-uniform loop bound
-#pragma unroll
-    for (int i = 0; i < kKR; ++i) {
-      if (i >= nw) break;
-      if (i < n && en_r[i] > t) {
-        const int32_t mem = mm_r[i] & 0xFFFF;
-        ++live;
-        if (!((mm_r[i] >> 22) & 1)) be += mem;
-        if (en_r[i] > t0) {
-          used += mem;
-          fs += K.fbr_p[((mm_r[i] >> 16) & 63) * kNProf];
-        }
-      }
-    }
-    const int live_g = group_sum32(active ? live : 0, K.Z);
-    const int be_mem = group_sum32(active ? be : 0, K.Z);
-    const bool overflow = live_g >= max_live;
-    const int32_t q = T.mem[m];
-    uint64_t key = ~0ull;
-    int64_t start = 0, c = 0;
-    if (active && !overflow && q <= K.Ms) {
-      int64_t F = K.fbr_p[m * kNProf];
-      if (used + q <= K.Ms) {
-        start = t0;
-        F += fs;
-      } else {  // memory wait: the earliest release after which the batch fits
-        start = INT64_MAX;
-#pragma unroll
-        for (int jj = 0; jj < kKR; ++jj) {
-          if (jj >= n) break;
-          if (en_r[jj] > t0) {
-            int32_t rem = 0;
-#pragma unroll
-            for (int i = 0; i < kKR; ++i) {
-              if (i >= n) break;
-              if (en_r[i] > en_r[jj]) rem += mm_r[i] & 0xFFFF;
-            }
-            if (rem + q <= K.Ms && en_r[jj] < start) start = en_r[jj];
-          }
-        }
-#pragma unroll
-        for (int i = 0; i < kKR; ++i) {
-          if (i >= n) break;
-          if (en_r[i] > start) F += K.fbr_p[((mm_r[i] >> 16) & 63) * kNProf];
-        }
-      }
-      c = start + exec_time(K.solo_p[m * kNProf], F);
-      if (strict) {
-        const uint64_t inelig = (be_mem >= K.pref) ? (1ull << 62) : 0ull;
-        key = inelig | ((uint64_t)c << 6) | ((uint64_t)(4 - K.p) << 3) | (uint64_t)K.s;
-      } else {
-        key = ((uint64_t)start << 3) | (uint64_t)K.s;
-      }
-    }
-    const uint64_t kmin = group_min(key, K.Z);
-    const bool placed = !overflow && kmin != ~0ull;
-    if (placed && key == kmin) {  // schedule(batch, chosen_slice)
-      const uint32_t mw = (uint32_t)q | ((uint32_t)m << 16) | ((uint32_t)(strict ? 1 : 0) << 22);
-#pragma unroll
-      for (int i = 0; i < kKR; ++i)
-        if (i == n) { en_r[i] = c; mm_r[i] = mw; }
-      ++n;
-      ls = start;
-    }
-    const int64_t cwin = __shfl_sync(0xffffffffu, c, (gbase + (int)(kmin & 7)) & 31);
-    if (leader) {
-      if (strict) {
-        if (!placed) {
-          misses += nreq;
-        } else {  // latencies fall along the sorted members: test the ends first
-          const uint32_t* ma = sarr + bt.pos;
-          const int64_t slo = T.slo[m];
-          if (cwin - (int64_t)ma[0] > slo)
-            misses += (cwin - (int64_t)ma[nreq - 1] > slo) ? nreq : nreq - hits_in(ma, nreq, cwin, slo);
-        }
-      } else {
-        const int64_t tb = placed ? cwin - (int64_t)sarr[bt.pos] : (int64_t)0xFFFFFFFFLL;
-        tail = tb > tail ? tb : tail;
-      }
-    }
-  }
-  *misses_out = misses;
-  *tail_out = tail;
-}
+constexpr int kKR = 6;  // batches per GPU-epoch handled by the register fast path
 
 // Candidate unit, fast path: the GPU-epoch's <= kKR batches fully unrolled, times 32-bit relative to
 // the first batch's ready time tb.  Every lane of a geometry's group keeps the whole placement so
@@ -930,7 +821,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           carry += __shfl_sync(0xffffffffu, x, 31);
         }
         __syncwarp();
-        // the streams present in this warp's segment: <= 4 take the ballot path
+        // the streams present in this warp's segment: <= 2 take the ballot path
         int K = 0, ak[4] = {0, 0, 0, 0}, run[4] = {0, 0, 0, 0};
 #pragma unroll 1
         for (int k0 = 0; k0 < S; k0 += 32) {
@@ -949,8 +840,6 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           case 0: break;
           case 1: scatter_segment<1>(warr, wmeta, sa_lo, sa_hi, klut, runw, c.sarr, ak, run); break;
           case 2: scatter_segment<2>(warr, wmeta, sa_lo, sa_hi, klut, runw, c.sarr, ak, run); break;
-          case 3: scatter_segment<3>(warr, wmeta, sa_lo, sa_hi, klut, runw, c.sarr, ak, run); break;
-          case 4: scatter_segment<4>(warr, wmeta, sa_lo, sa_hi, klut, runw, c.sarr, ak, run); break;
           default: scatter_segment<0>(warr, wmeta, sa_lo, sa_hi, klut, runw, c.sarr, ak, run); break;
         }
       }
@@ -1366,13 +1255,12 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           const int o = __shfl_xor_sync(0xffffffffu, len_max, d);
           len_max = o > len_max ? o : len_max;
         }
-        if (!actual && len_max <= kKR) {  // register-resident candidate lists
-          int64_t misses, tail;
-          // warp-uniform batch range (idle lanes must still take part in the group shuffles)
-          if (!candidate_unit_fast(T, K, active, lane == gbase && valid, bats, gl, c.g_off[g],
-                                   c.g_off[g + 1] - c.g_off[g], sarr, P.max_live, &misses, &tail))
-            candidate_unit_regs(T, K, active, lane == gbase && valid, bats, gl, c.g_off[g],
-                                c.g_off[g + 1], sarr, P.max_live, &misses, &tail);
+        int64_t misses, tail;
+        // register fast path (warp-uniform batch range: idle lanes still take part in the shuffles);
+        // if a completion does not fit its 32-bit frame, the unit re-runs on the generic path below
+        if (!actual && len_max <= kKR &&
+            candidate_unit_fast(T, K, active, lane == gbase && valid, bats, gl, c.g_off[g],
+                                c.g_off[g + 1] - c.g_off[g], sarr, P.max_live, &misses, &tail)) {
           if (valid && lane == gbase) {
             const int64_t key = make_key(misses, tail, j == c.gu8[0 * c.N + g] ? 0 : j + 1);
             if (j == c.gu8[0 * c.N + g]) c.gi[7 * c.N + g] = key;
