@@ -276,10 +276,13 @@ def run_ours(args):
         cores = os.cpu_count() or 1
         n_rep = min(args.cpu_sample, R)
         tr = oracle_sample(n_rep, S, base=0)
-        dt, s_cpu, q_cpu, _ = time_oracle(prof, tr, cores)
+        dt, s_cpu, q_cpu, passes = 0.0, 0, 0, 0
+        while passes < 1 or (dt < 10.0 and passes < 40):  # ~10 s of oracle work on the host cores
+            d, s1, q1, _ = time_oracle(prof, tr, cores)
+            dt, s_cpu, q_cpu, passes = dt + d, s_cpu + s1, q_cpu + q1, passes + 1
         cpu = {"value": s_cpu / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
-               "sample": f"{n_rep} replicas x {S} s of this workload (numpy-generated), "
-                         f"{dt:.1f} s wall on {cores} threads",
+               "sample": f"{n_rep} replicas x {S} s of this workload (numpy-generated), replayed "
+                         f"{passes}x: {dt:.1f} s wall on {cores} threads",
                "simulated_requests_per_s": q_cpu / dt}
 
     if rank == 0:
@@ -310,7 +313,7 @@ def run_ours(args):
                          "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
                          "kernel": "replay_kernel", "kernel_ms": k_ms, "prepass_ms": statistics.mean(pre_ms),
                          "launch": launch},
-            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": 3 * args.steps * world, "clocks": clocks,
+            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": 2 * args.steps * world, "clocks": clocks,
         }
         print(json.dumps(line), flush=True)
     if world > 1:
