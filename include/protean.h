@@ -249,9 +249,13 @@ int protean_replay_traces(protean_handle *h, const protean_replay_cfg *cfg,
                           protean_replay_out *out, void *stream);
 
 /* Device time (CUDA events on the launching stream) of the last protean_replay_traces call:
- * the prepass kernels (epoch offsets; per-epoch, per-segment stream counts) and the fused replay
- * kernel, in ms; launch = {grid, block, dynamic smem
- * bytes, resident CTAs per SM} of the replay kernel (any pointer may be NULL).  Host. */
+ * prepass_ms = the prepass (epoch offsets) + the trace-level stream partition (per-(replica, epoch,
+ * stream) counts, run indices, stable scatter into a stream-sorted copy of the arrivals, request
+ * validation); replay_ms = the fused replay kernel; launch = {grid, block, dynamic smem bytes,
+ * resident CTAs per SM} of the replay kernel (any pointer may be NULL).  Host.
+ * Device memory: besides its scratch, a call holds a stream-sorted copy of the arrivals
+ * (4 B/request) and two [R][E(+1)][2M] uint32 index tables, grown with the stream-ordered allocator
+ * and kept by the handle for the next call. */
 int protean_last_timings(const protean_handle *h, float *prepass_ms, float *replay_ms,
                          int32_t *launch);
 

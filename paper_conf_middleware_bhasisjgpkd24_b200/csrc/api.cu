@@ -29,10 +29,20 @@ struct protean_handle {
   size_t scratch_bytes = 0;
   int64_t* d_eoff = nullptr;
   size_t eoff_bytes = 0;
+  // trace-level stream partition (partition.cu): counts, run indices, stream-sorted arrivals
+  void* d_cnt = nullptr;
+  size_t cnt_bytes = 0;
+  void* d_sidx = nullptr;
+  size_t sidx_bytes = 0;
+  void* d_sa = nullptr;
+  size_t sa_bytes = 0;
+  void* d_saoff = nullptr;
+  size_t saoff_bytes = 0;
   void* d_small = nullptr;  // wmax (8 B) + err (16 B)
   uint32_t* d_pack = nullptr;  // candidate lane packing for the full geometry range
   int CW = 0;
-  cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};  // prepass / replay kernel bracket
+  // [0,1] prepass + partition count, [4,5] partition scan + scatter, [2,3] replay kernel
+  cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
   float t_prepass = 0.f, t_replay = 0.f;
   int last_grid = 0, last_block = 0, last_smem = 0, last_per_sm = 0;
   std::vector<int> gn;  // slice count per geometry
@@ -392,7 +402,7 @@ int protean_load_profiles(const protean_profiles* p, protean_handle** out) {
   if (e == cudaSuccess)
     e = cudaMemcpy(h->d_tab, h->words.data(), sizeof(int32_t) * h->words.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMalloc(&h->d_small, 256);
-  for (int i = 0; i < 4 && e == cudaSuccess; ++i) e = cudaEventCreate(&h->ev[i]);
+  for (int i = 0; i < 6 && e == cudaSuccess; ++i) e = cudaEventCreate(&h->ev[i]);
   if (e == cudaSuccess) e = cudaMalloc(&h->d_pack, pack.size() * 4);
   if (e == cudaSuccess) e = cudaMemcpy(h->d_pack, pack.data(), pack.size() * 4, cudaMemcpyHostToDevice);
   if (e != cudaSuccess) {
@@ -410,11 +420,13 @@ void protean_free(protean_handle* h) {
   if (h->d_tab) cudaFree(h->d_tab);
   if (h->d_scratch) cudaFree(h->d_scratch);
   if (h->d_eoff) cudaFree(h->d_eoff);
+  for (void* q : {h->d_cnt, h->d_sidx, h->d_sa, h->d_saoff})
+    if (q) cudaFree(q);
   if (h->d_small) cudaFree(h->d_small);
   if (h->d_pack) cudaFree(h->d_pack);
   if (h->d_pack_g) cudaFree(h->d_pack_g);
   xchg_release(h);
-  for (int i = 0; i < 4; ++i)
+  for (int i = 0; i < 6; ++i)
     if (h->ev[i]) cudaEventDestroy(h->ev[i]);
   delete h;
 }
@@ -585,16 +597,54 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   CK(h, cudaMemsetAsync(h->d_small, 0, 256, st));
   CK(h, cudaEventRecord(h->ev[0], st));
   CK(h, launch_prepass(c.arrival_us, c.replica_off, R, E, W, h->maxT, h->d_eoff, d_wmax, d_err, st));
-  const int kWarps = 8;  // replay CTA = 8 warps
+  const int kWarps = PROTEAN_WARPS;  // replay CTA warps (replay.cuh)
+  // stream partition, P1 (count + validate every request)
+  const int S = 2 * h->M;
+  std::vector<int64_t> saoff(R + 1);
+  saoff[0] = 0;
+  for (int r = 0; r < R; ++r) saoff[r + 1] = saoff[r] + ((roff[r + 1] - roff[r] + 3) & ~(int64_t)3);
+  {
+    int rc = ensure(h, &h->d_cnt, &h->cnt_bytes, std::max<size_t>(4, sizeof(uint32_t) * (size_t)R * E * S), st);
+    if (!rc) rc = ensure(h, &h->d_sidx, &h->sidx_bytes, std::max<size_t>(4, sizeof(uint32_t) * (size_t)R * (E + 1) * S), st);
+    if (!rc) rc = ensure(h, &h->d_sa, &h->sa_bytes, std::max<size_t>(16, sizeof(uint32_t) * (size_t)saoff[R]), st);
+    if (!rc) rc = ensure(h, &h->d_saoff, &h->saoff_bytes, sizeof(int64_t) * (size_t)(R + 1), st);
+    if (rc) return rc;
+  }
+  CK(h, cudaMemcpyAsync(h->d_saoff, saoff.data(), sizeof(int64_t) * (R + 1), cudaMemcpyHostToDevice, st));
+  PartitionArgs PA;
+  PA.arr = c.arrival_us;
+  PA.meta = c.meta;
+  PA.roff = c.replica_off;
+  PA.eoff = h->d_eoff;
+  PA.saoff = static_cast<const int64_t*>(h->d_saoff);
+  PA.R = R;
+  PA.S = S;
+  PA.M = h->M;
+  PA.E = E;
+  PA.tlm1 = (uint32_t)(c.trace_len_us - 1);  // trace_len - 1 + maxT <= 2^32 - 1 (checked above)
+  PA.vec = ((reinterpret_cast<uintptr_t>(c.arrival_us) & 15u) == 0) &&
+           ((reinterpret_cast<uintptr_t>(c.meta) & 15u) == 0);
+  PA.cnt = static_cast<uint32_t*>(h->d_cnt);
+  PA.sidx = static_cast<uint32_t*>(h->d_sidx);
+  PA.sa = static_cast<uint32_t*>(h->d_sa);
+  PA.err = d_err;
+  CK(h, launch_partition_count(PA, st));
   CK(h, cudaEventRecord(h->ev[1], st));
   unsigned long long wmax = 0;
   int herr = 0;
   CK(h, cudaMemcpyAsync(&wmax, d_wmax, 8, cudaMemcpyDeviceToHost, st));
   CK(h, cudaMemcpyAsync(&herr, d_err, 4, cudaMemcpyDeviceToHost, st));
   CK(h, cudaStreamSynchronize(st));
+  // the prepass guarantees that the epoch ranges tile every replica (else the scatter could leave
+  // it); request-level validation happens in the scatter pass and is reported after the replay
   if (herr) return fail(h, PROTEAN_EINVAL, "arrivals not sorted or beyond the trace");
-  const int WCAP = (int)std::max<unsigned long long>(wmax, 1);
   if (wmax >= (1ull << 25)) return fail(h, PROTEAN_ERANGE, "epoch window >= 2^25 requests");
+  // P2 + P3: run indices and the stable scatter (only on a validated trace)
+  CK(h, cudaEventRecord(h->ev[4], st));
+  CK(h, launch_partition_rest(PA, st));
+  CK(h, cudaEventRecord(h->ev[5], st));
+  // window capacity: the largest window (requests in [eW - maxT, (e+1)W)) + per-stream alignment
+  const int WCAP = (int)std::max<unsigned long long>(wmax, 1) + 8 * S;
 
   // candidate range: all geometries, or this rank's slot-balanced range (mode G)
   int geom_lo = 0, geom_hi = h->G;
@@ -643,12 +693,9 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   P.tl = h->tl;
   P.pack = d_pack;
   P.maxT = h->maxT;
-  P.arr = c.arrival_us;
-  P.vec_ok = ((reinterpret_cast<uintptr_t>(c.arrival_us) & 15u) == 0) &&
-             ((reinterpret_cast<uintptr_t>(c.meta) & 15u) == 0);
-  P.meta = c.meta;
-  P.roff = c.replica_off;
-  P.eoff = h->d_eoff;
+  P.sa = PA.sa;
+  P.saoff = PA.saoff;
+  P.sidx = PA.sidx;
   P.R = R;
   P.N = N;
   P.base = c.replica_base;
@@ -699,7 +746,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   P.o_gbat = o; o += al((size_t)WCAP * sizeof(Bat));
   P.o_gord = o; o += al((size_t)WCAP * 4);
   P.o_gglist = o; o += al((size_t)WCAP * 4);
-  P.o_gsarr = o; o += al((size_t)(WS >= WCAP ? 0 : WCAP) * 4);
+  P.o_gsarr = o; o += al((size_t)(WS > 0 ? 0 : WCAP) * 4);
   P.slot_bytes = al(o);
   {
     int rc = ensure(h, &h->d_scratch, &h->scratch_bytes, P.slot_bytes * (size_t)grid, st);
@@ -719,7 +766,12 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
     h->poisoned = true;
     return fail(h, PROTEAN_ENCCL, "mode G exchange: a peer rank did not publish within 30 s");
   }
-  CK(h, cudaEventElapsedTime(&h->t_prepass, h->ev[0], h->ev[1]));
+  {
+    float a = 0.f, b = 0.f;
+    CK(h, cudaEventElapsedTime(&a, h->ev[0], h->ev[1]));
+    CK(h, cudaEventElapsedTime(&b, h->ev[4], h->ev[5]));
+    h->t_prepass = a + b;  // device time of the prepass and the three partition passes
+  }
   CK(h, cudaEventElapsedTime(&h->t_replay, h->ev[2], h->ev[3]));
   h->last_grid = grid;
   h->last_block = block;

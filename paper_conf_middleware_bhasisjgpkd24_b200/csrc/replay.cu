@@ -82,10 +82,10 @@ struct Ctx {
 };
 
 struct CtaState {
-  int64_t w_lo, lt_total, nlog;
+  int64_t nlog;
   int nb, cursor, all_avail, bad;
   int task, adone;
-  unsigned amin;
+  int wtot;          // window entries copied this epoch (incl. alignment padding)
   unsigned long long cnt[10];
 };
 
@@ -380,130 +380,6 @@ __device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, const
   return o;
 }
 
-// Shared-memory increment by exactly 1, unpredicated (ptxas aggregates a warp's same-address
-// increments, ATOMS.POPC.INC); lanes with nothing to count increment a sink word instead, which
-// keeps the per-element loops free of branches.
-__device__ __forceinline__ void inc_shared(uint32_t saddr) {
-  asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(saddr) : "memory");
-}
-
-// Count pass of one warp over window entries [lo, hi): per-stream counts into the warp-private
-// cntw (one predicated shared reduction per request; same-address reductions of a warp are
-// combined by the hardware), and validation of every entry: model id, arrival < trace_len, and
-// arrival >= its predecessor (window entry 0 against prev0, the entry before the window, if any).
-// Every adjacent pair of a replica's trace lies inside some window, so this validates sortedness.
-// vec: meta and arrivals are 16-byte aligned at the same element index, so the body takes 16
-// consecutive requests per lane (one 16-byte meta load, four 16-byte arrival loads).
-__device__ __forceinline__ void count_check_one(const uint8_t* meta, const uint32_t* arr, int64_t i,
-                                                bool valid, bool has_prev0, uint32_t prev0,
-                                                uint32_t tlm1, uint32_t cb, uint32_t sink,
-                                                const uint16_t* klut, bool& bad) {
-  const int kv = klut[valid ? meta[i] : 0];
-  const uint32_t a = valid ? arr[i] : 0u;
-  const uint32_t ap = (valid && i > 0) ? arr[i - 1] : (has_prev0 ? prev0 : 0u);
-  bad |= valid && ((kv & 0x8000) != 0 || a > tlm1 || a < ap);
-  inc_shared(valid ? cb + 4u * (uint32_t)(kv & 0x7FFF) : sink);
-}
-
-__device__ __forceinline__ bool count_segment(const uint8_t* meta, const uint32_t* arr, int64_t lo,
-                                              int64_t hi, bool vec, bool has_prev0, uint32_t prev0,
-                                              uint32_t tlm1, int* cntw, uint32_t sink, const uint16_t* klut) {
-  const int lane = threadIdx.x & 31;
-  const uint32_t cb = (uint32_t)__cvta_generic_to_shared(cntw);
-  bool bad = false;
-  const int64_t h = vec ? min(hi, lo + (int64_t)((16u - ((uint32_t)(uintptr_t)(meta + lo) & 15u)) & 15u)) : hi;
-#pragma unroll 1
-  for (int64_t i0 = lo; i0 < h; i0 += 32)  // unaligned head (< 16 entries), or everything (!vec)
-    count_check_one(meta, arr, i0 + lane, i0 + lane < h, has_prev0, prev0, tlm1, cb, sink, klut, bad);
-  if (vec) {
-    const int nch = (int)((hi - h) >> 4);
-    const uint4* gv = reinterpret_cast<const uint4*>(meta + h);
-    const uint4* ga = reinterpret_cast<const uint4*>(arr + h);
-#pragma unroll 1
-    for (int c0 = 0; c0 < nch; c0 += 32) {
-      const int ch = c0 + lane;
-      const bool valid = ch < nch;
-      uint4 v = make_uint4(0u, 0u, 0u, 0u), a0 = v, a1 = v, a2 = v, a3 = v;
-      uint32_t ap = 0u;
-      if (valid) {
-        v = gv[ch];
-        a0 = ga[4 * ch];
-        a1 = ga[4 * ch + 1];
-        a2 = ga[4 * ch + 2];
-        a3 = ga[4 * ch + 3];
-        const int64_t i = h + 16 * (int64_t)ch;
-        ap = i > 0 ? arr[i - 1] : (has_prev0 ? prev0 : 0u);
-      }
-      const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
-      const uint32_t av[16] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w,
-                               a2.x, a2.y, a2.z, a2.w, a3.x, a3.y, a3.z, a3.w};
-      uint32_t flags = 0;  // model-id flags; sortedness pairwise; the last entry is the maximum
-      bool uns = av[0] < ap;
-#pragma unroll
-      for (int q = 0; q < 16; ++q) {
-        const int kv = klut[(w4[q >> 2] >> (8 * (q & 3))) & 0xFF];
-        flags |= (uint32_t)kv;
-        if (q > 0) uns |= av[q] < av[q - 1];
-        inc_shared(valid ? cb + 4u * (uint32_t)(kv & 0x7FFF) : sink);
-      }
-      bad |= valid && ((flags & 0x8000u) != 0 || av[15] > tlm1 || uns);
-    }
-#pragma unroll 1
-    for (int64_t i0 = h + 16 * (int64_t)nch; i0 < hi; i0 += 32)  // tail (< 16 entries)
-      count_check_one(meta, arr, i0 + lane, i0 + lane < hi, has_prev0, prev0, tlm1, cb, sink, klut, bad);
-  }
-  return bad;
-}
-
-// Stable scatter of window entries [lo, hi) (one warp) into their streams' runs of sa (entries
-// were validated by the count pass).  K = 1..4: the segment holds exactly the streams ak[0..K),
-// whose running offsets run[] live in registers and whose in-warp ranks come from one ballot each;
-// K = 0: any number of streams, ranks from match_any and warp-private running offsets in runw.
-constexpr int kSU = 4;  // requests per lane in flight per scatter step
-template <int K>
-__device__ __forceinline__ void scatter_segment(const uint32_t* warr, const uint8_t* wmeta, int lo, int hi,
-                                                const uint16_t* klut, int* runw, uint32_t* sa,
-                                                const int (&ak)[4], int (&run)[4]) {
-  const int lane = threadIdx.x & 31;
-  const unsigned lt = (1u << lane) - 1u;
-#pragma unroll 1
-  for (int i0 = lo; i0 < hi; i0 += 32 * kSU) {
-    uint8_t mt[kSU];
-    uint32_t ai[kSU];
-#pragma unroll
-    for (int u = 0; u < kSU; ++u) {
-      const int i = i0 + u * 32 + lane;
-      const bool valid = i < hi;
-      mt[u] = valid ? wmeta[i] : (uint8_t)0;
-      ai[u] = valid ? warr[i] : 0u;
-    }
-#pragma unroll
-    for (int u = 0; u < kSU; ++u) {
-      const bool valid = i0 + u * 32 + lane < hi;
-      const int key = klut[mt[u]] & 0x7FFF;
-      if (K > 0) {
-        int pos = 0;
-#pragma unroll
-        for (int t = 0; t < K; ++t) {
-          const bool mine = valid && key == ak[t];
-          const unsigned b = __ballot_sync(0xffffffffu, mine);
-          if (mine) pos = run[t] + __popc(b & lt);
-          run[t] += __popc(b);
-        }
-        if (valid) sa[pos] = ai[u];
-      } else {
-        const unsigned peers = __match_any_sync(0xffffffffu, valid ? key : 1024 + lane);
-        const int rank = __popc(peers & lt);
-        // the group's run of slots in stream order; its last lane advances the offset
-        const int base = runw[valid ? key : 0];
-        if (valid) sa[base + rank] = ai[u];
-        if (valid && (peers >> lane) == 1u) runw[key] = base + rank + 1;
-        __syncwarp();
-      }
-    }
-  }
-}
-
 constexpr int kKR = 6;  // batches per GPU-epoch handled by the register fast path
 
 // Candidate unit, fast path: the GPU-epoch's <= kKR batches fully unrolled, times 32-bit relative to
@@ -619,21 +495,21 @@ __device__ __forceinline__ bool candidate_unit_fast(const Tab& T, const SliceLan
 
 }  // namespace
 
-__global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams P) {
+__global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kernel(ReplayParams P) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ CtaState cs;
   __shared__ uint32_t s_hist[2 * kNB];  // 2 classes x 3328 buckets (u32 < 2^32 per replica)
   __shared__ uint32_t s_sink;           // target of increments with nothing to count
-  __shared__ uint16_t klut[256];        // meta byte -> stream key (| 0x8000 if invalid)
-  __shared__ int s_cnt[kNSeg * kMaxStreams], s_run[kNSeg * kMaxStreams];
-  __shared__ int s_base[kMaxStreams], s_tot[kMaxStreams], s_skip[kMaxStreams], s_pend[kMaxStreams];
+  const uint32_t sink = (uint32_t)__cvta_generic_to_shared(&s_sink);
+  __shared__ __align__(8) uint64_t s_mbar;  // TMA bulk-copy completion of the epoch's window
+  __shared__ int s_base[kMaxStreams], s_tot[kMaxStreams], s_cur[kMaxStreams], s_pend[kMaxStreams];
+  __shared__ int s_dst[kMaxStreams], s_alo[kMaxStreams], s_asz[kMaxStreams];
 #ifdef PROTEAN_PHASE_TIMING
   unsigned long long ph_acc[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
   long long ph_last = clock64();
 #endif
   const SmemLayout& SL = P.sl;
   const int tid = threadIdx.x, NT = blockDim.x, lane = tid & 31, warp = tid >> 5, NW = NT >> 5;
-  const uint32_t sink = (uint32_t)__cvta_generic_to_shared(&s_sink);
   const int N = P.N, S = SL.S, Gc = SL.Gc, CW = SL.CW;
 
   Ctx c;
@@ -643,12 +519,12 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
   uint32_t* packs = reinterpret_cast<uint32_t*>(smem + SL.pack);
 #pragma unroll 1
   for (int i = tid; i < CW * 32; i += NT) packs[i] = P.pack[i];
-#pragma unroll 1
-  for (int b = tid; b < 256; b += NT) {
-    const int m = b & 63;
-    const bool ok = !(b & 0x40) && m < P.tl.M;
-    klut[b] = (uint16_t)((2 * (ok ? m : 0) + ((b >> 7) ? 0 : 1)) | (ok ? 0 : 0x8000));
+  const uint32_t mbar = (uint32_t)__cvta_generic_to_shared(&s_mbar);
+  if (tid == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mbar) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
+  uint32_t mphase = 0;  // parity of the window barrier's next phase (uniform)
   c.T.bind(tabw, P.tl);
   c.pack = packs;
   c.N = N;
@@ -668,8 +544,8 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
   c.gb = reinterpret_cast<Bat*>(slot + P.o_gbat);
   c.gord = reinterpret_cast<uint32_t*>(slot + P.o_gord);
   c.ggl = reinterpret_cast<uint32_t*>(slot + P.o_gglist);
-  c.sarr = SL.WS >= P.WCAP ? reinterpret_cast<uint32_t*>(smem + SL.sarr)
-                           : reinterpret_cast<uint32_t*>(slot + P.o_gsarr);
+  const bool win_smem = SL.WS > 0;  // the epoch window in shared memory (else global scratch)
+  c.sarr = win_smem ? reinterpret_cast<uint32_t*>(smem + SL.sarr) : reinterpret_cast<uint32_t*>(slot + P.o_gsarr);
   // resident lists: actual lanes [N*8 lanes][max_live], candidate lanes [NT lanes][max_live]
   const int NA = N * kZA;
   LaneList AL;
@@ -693,15 +569,13 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
 #pragma unroll 1
   for (int r = blockIdx.x; r < P.R; r += gridDim.x) {
     const uint64_t replica = (uint64_t)(P.base + r);
-    const int64_t r_lo = P.roff[r];
-    const int64_t* eoff = P.eoff + (size_t)r * (P.E + 1);
     uint32_t* ghist = P.hist + (size_t)r * 2 * kNB;
 
     // ---------------------------------------------------------------- replica init
 #pragma unroll 1
     for (int i = tid; i < 2 * kNB; i += NT) s_hist[i] = 0;
 #pragma unroll 1
-    for (int k = tid; k < S; k += NT) s_skip[k] = 0;
+    for (int k = tid; k < S; k += NT) s_cur[k] = (int)P.sidx[(size_t)r * (P.E + 1) * S + k];
 #pragma unroll 1
     for (int g = tid; g < N; g += NT) {
       reset_gpu_state(c, g, P.init_geom);
@@ -713,15 +587,12 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       c.gi[8 * c.N + g] = c.gi[9 * c.N + g] = c.gi[10 * c.N + g] = c.gi[11 * c.N + g] = 0;
     }
     if (tid == 0) {
-      cs.w_lo = r_lo;
       cs.nlog = 0;
       cs.cursor = 0;
       cs.bad = 0;
       cs.task = 0;  // per-epoch scratch, re-armed at the end of every epoch
       cs.adone = 0;
       cs.nb = 0;
-      cs.amin = 0xFFFFFFFFu;
-      cs.lt_total = 0;
       cs.all_avail = 1;
 #pragma unroll
       for (int i = 0; i < 10; ++i) cs.cnt[i] = 0;
@@ -755,110 +626,107 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
 #if PROTEAN_A_BARRIER
       __syncthreads();
 #endif
-      const int64_t w_beg = eoff[e], w_end = eoff[e + 1];
-      const int64_t w_lo = cs.w_lo;
-      if (tid == 32 && e + 1 < P.E) {  // the next epoch's new requests: into L2 during this one
-        const int64_t nb0 = w_end, nb1 = eoff[e + 2];
-        prefetch_l2(P.meta + nb0, nb1 - nb0);
-        prefetch_l2(P.arr + nb0, (nb1 - nb0) * 4);
-      }
-      PH(0);
-      const int64_t len64 = w_end - w_lo;
-      const bool bad_window = len64 < 0 || len64 > P.WCAP || w_beg < w_lo;
-      if (bad_window && tid == 0) atomicOr(P.err, 1);
-      const int len = bad_window ? 0 : (int)len64;
-      const uint32_t* warr = P.arr + w_lo;
-      const uint8_t* wmeta = P.meta + w_lo;
-      // ---------------------------------------------------------------- B: stream partition
-      // every warp owns one contiguous 1/NW of the window: (1) it counts its segment per stream
-      // (16-byte meta loads, match_any aggregation), (2) after one barrier derives its own
-      // per-stream write offsets (redundant scan over streams), (3) scatters its segment stably with
-      // 8 loads in flight per lane, validating every request once (when it is new).  The window is
-      // L2-resident (prefetched during the previous epoch); offsets are warp-private, so the
-      // scatter needs no atomics.
-      const int sa_lo = (int)((int64_t)len * warp / NW), sa_hi = (int)((int64_t)len * (warp + 1) / NW);
-      {
-        int* cntw = s_cnt + warp * S;
-#pragma unroll 1
-        for (int k = lane; k < S; k += 32) cntw[k] = 0;
-        __syncwarp();
-        if (sa_hi > sa_lo &&
-            count_segment(wmeta, warr, sa_lo, sa_hi, P.vec_ok, w_lo > r_lo, w_lo > r_lo ? P.arr[w_lo - 1] : 0u,
-                          (uint32_t)(P.trace_len - 1), cntw, sink, klut))  // arrivals < trace_len <= 2^32 (host check)
-          atomicOr(P.err, 1);
-      }
-      __syncthreads();
-      PH(1);
-      {  // this warp's write offsets: base_k (exclusive scan of stream totals) + earlier segments
-        int* runw = s_run + warp * S;
+      // ---------------------------------------------------------------- B: stream windows
+      // Stream k's unbatched requests are [s_cur[k], sidx[r][e+1][k]) of the stream-sorted copy
+      // (partition.cu).  Warp 0 lays the streams out contiguously in the window (each as its
+      // 16-byte aligned superset) and, for a shared-memory window, every lane issues its streams'
+      // TMA bulk copies (cp.async.bulk global -> shared, completion on one mbarrier); the next
+      // epoch's new requests are prefetched into L2 meanwhile.  A global-scratch window (too large
+      // for shared memory) is filled by a cooperative 16-byte copy instead.
+      const uint32_t* sa_r = P.sa + P.saoff[r];
+      if (warp == 0) {
+        const uint32_t* s1 = P.sidx + ((size_t)r * (P.E + 1) + e + 1) * S;
         int carry = 0;
 #pragma unroll 1
         for (int k0 = 0; k0 < S; k0 += 32) {
           const int k = k0 + lane;
-          int tot = 0, part = 0;
+          int cur = 0, len = 0, alo = 0, asz = 0;
           if (k < S) {
-#pragma unroll 1
-            for (int w = 0; w < NW; ++w) {
-              const int cv = s_cnt[w * S + k];
-              if (w < warp) part += cv;
-              tot += cv;
+            cur = s_cur[k];
+            const int hi = (int)s1[k];
+            len = hi - cur;
+            alo = cur & ~3;
+            asz = len > 0 ? ((hi + 3) & ~3) - alo : 0;
+            if (e + 1 < P.E && tid < 32) {  // the next epoch's new requests: into L2 during this one
+              const int h2 = (int)s1[S + k];
+              if (h2 > hi) prefetch_l2(sa_r + hi, (int64_t)(h2 - hi) * 4);
             }
           }
-          int x = tot;
+          int x = asz;
 #pragma unroll
           for (int d = 1; d < 32; d <<= 1) {
             const int y = __shfl_up_sync(0xffffffffu, x, d);
             if (lane >= d) x += y;
           }
-          const int base = carry + x - tot;
+          const int dst = carry + x - asz;
           if (k < S) {
-            runw[k] = base + part;
-            if (warp == 0) {
-              s_base[k] = base;
-              s_tot[k] = tot;
-            }
+            s_base[k] = dst + (cur - alo);
+            s_tot[k] = len > 0 ? len : 0;
+            s_dst[k] = dst;
+            s_alo[k] = alo;
+            s_asz[k] = asz;
           }
           carry += __shfl_sync(0xffffffffu, x, 31);
         }
-        __syncwarp();
-        // the streams present in this warp's segment: <= 2 take the ballot path
-        int K = 0, ak[4] = {0, 0, 0, 0}, run[4] = {0, 0, 0, 0};
-#pragma unroll 1
-        for (int k0 = 0; k0 < S; k0 += 32) {
-          unsigned pres = __ballot_sync(0xffffffffu, k0 + lane < S && s_cnt[warp * S + k0 + lane] > 0);
-#pragma unroll 1
-          while (pres) {
-            const int k = k0 + __ffs(pres) - 1;
-            pres &= pres - 1;
-#pragma unroll
-            for (int t = 0; t < 4; ++t)
-              if (K == t) { ak[t] = k; run[t] = runw[k]; }
-            ++K;
-          }
+        const bool overflow = carry > P.WCAP;  // cannot happen for a valid trace (host bound)
+        if (overflow) {
+          for (int k = lane; k < S; k += 32) s_tot[k] = 0;
+          if (lane == 0) atomicOr(P.err, 1);
         }
-        switch (K) {
-          case 0: break;
-          case 1: scatter_segment<1>(warr, wmeta, sa_lo, sa_hi, klut, runw, c.sarr, ak, run); break;
-          case 2: scatter_segment<2>(warr, wmeta, sa_lo, sa_hi, klut, runw, c.sarr, ak, run); break;
-          default: scatter_segment<0>(warr, wmeta, sa_lo, sa_hi, klut, runw, c.sarr, ak, run); break;
+        const int tot = overflow ? 0 : carry;
+        if (lane == 0) cs.wtot = tot;
+        if (win_smem && tot > 0) {
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // prior generic accesses
+          __syncwarp();
+#pragma unroll 1
+          for (int k = lane; k < S; k += 32) {
+            const int asz = s_asz[k];
+            if (asz > 0) {
+              const uint32_t dsts = (uint32_t)__cvta_generic_to_shared(c.sarr + s_dst[k]);
+              asm volatile(
+                  "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                  ::"r"(dsts), "l"(sa_r + s_alo[k]), "r"(asz * 4), "r"(mbar) : "memory");
+            }
+          }
+          if (lane == 0)
+            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mbar), "r"(tot * 4) : "memory");
         }
       }
       __syncthreads();
+      PH(1);
+      if (win_smem) {
+        if (cs.wtot > 0) {  // uniform: wait for this epoch's bulk copies
+          uint32_t done = 0;
+          while (!done)
+            asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+                         "selp.u32 %0, 1, 0, p;\n\t}"
+                         : "=r"(done) : "r"(mbar), "r"(mphase) : "memory");
+          mphase ^= 1u;
+        }
+      } else {
+#pragma unroll 1
+        for (int k = 0; k < S; ++k) {
+          const int asz = s_asz[k];
+          if (asz <= 0 || cs.wtot == 0) continue;
+          const uint4* src = reinterpret_cast<const uint4*>(sa_r + s_alo[k]);
+          uint4* dst = reinterpret_cast<uint4*>(c.sarr + s_dst[k]);
+          for (int i = tid; i < asz / 4; i += NT) dst[i] = src[i];
+        }
+        __syncthreads();
+      }
       PH(3);
       // ---------------------------------------------------------------- C: batch formation
       // warp per stream: lanes test 32 consecutive B-sized batches at once (full batches are the
       // common case); a batch closed by the timeout, or still open, is resolved by lane 0.
 #pragma unroll 1
       for (int k = warp; k < S; k += NW) {
-        if (bad_window) break;
         const int m = k >> 1;
         const bool strict = (k & 1) == 0;
         const int B = T.bsz[m];
         const int64_t Tm = T.tmo[m];
-        int i = s_base[k] + s_skip[k];
+        int i = s_base[k];
         const int end = s_base[k] + s_tot[k];
         int pend = 0;
-        uint32_t a0p = 0xFFFFFFFFu;
 #pragma unroll 1
         while (i < end) {
           const int64_t st = (int64_t)i + (int64_t)lane * B;
@@ -902,7 +770,7 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
             if (j - i == B) ready = sarr[j - 1];        // full (only at the window end)
             else if (j < end) ready = deadline;         // a later arrival missed the timeout
             else if (deadline < Tend) ready = deadline; // timed out inside this epoch
-            else { state = 1; pend = end - i; a0p = (uint32_t)a0; }
+            else { state = 1; pend = end - i; }
             if (state == 0) {
               const int slot = atomicAdd(&cs.nb, 1);
               Bat& bt = c.bat_w(slot);
@@ -922,15 +790,11 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
           if (state) break;
           i = j;
         }
-        if (lane == 0) {
-          s_pend[k] = pend;
-          if (pend) atomicMin(&cs.amin, a0p);
-        }
+        if (lane == 0) s_pend[k] = pend;
       }
       __syncthreads();
       PH(4);
       const int nb = cs.nb;
-      const unsigned amin = cs.amin;
       if (nb > c.BS) {  // rare: more batches than the smem arrays hold -> all in global scratch
 #pragma unroll 1
         for (int b = tid; b < c.BS; b += NT) c.gb[b] = c.sb[b];
@@ -943,20 +807,9 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
         c.ord = c.sord;
         c.gl = c.sgl;
       }
-      // next window: stream entries at/after the earliest open batch's first arrival are re-read
+      // the open batch's requests (if any) stay unbatched: the next epoch's window starts there
 #pragma unroll 1
-      for (int k = tid; k < S; k += NT) {
-        if (bad_window) continue;  // the next window starts at w_end: nothing carried
-        const int b0 = s_base[k], tot = s_tot[k];
-        int lo = 0, hi = tot;
-#pragma unroll 1
-        while (lo < hi) {
-          const int mid = (lo + hi) >> 1;
-          if (sarr[b0 + mid] >= amin) hi = mid; else lo = mid + 1;
-        }
-        if (lo) atomicAdd(reinterpret_cast<unsigned long long*>(&cs.lt_total), (unsigned long long)lo);
-        s_skip[k] = tot - lo - s_pend[k];  // the next window re-reads entries with arrival >= amin
-      }
+      for (int k = tid; k < S; k += NT) s_cur[k] += s_tot[k] - s_pend[k];
       Bat* bats = c.bats;
       uint32_t* ord = c.ord;
       uint32_t* gl = c.gl;
@@ -992,7 +845,6 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
       __syncthreads();
       PH(5);
       if (tid == 0) {
-        cs.w_lo = bad_window ? w_end : w_lo + cs.lt_total;
         if (avail_all) cs.cursor = (int)((cursor + nb) % N);
       }
       // ---------------------------------------------------------------- D: dispatch
@@ -1427,8 +1279,6 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
             cs.task = 0;  // re-arm the per-epoch scratch for the next epoch
             cs.adone = 0;
             cs.nb = 0;
-            cs.amin = 0xFFFFFFFFu;
-            cs.lt_total = 0;
             cs.all_avail = 1;
           }
         }
@@ -1510,8 +1360,6 @@ __global__ void __launch_bounds__(256, PROTEAN_MINB) replay_kernel(ReplayParams 
         cs.task = 0;  // re-arm the per-epoch scratch for the next epoch
         cs.adone = 0;
         cs.nb = 0;
-        cs.amin = 0xFFFFFFFFu;
-        cs.lt_total = 0;
         cs.all_avail = 1;
       }
       }
@@ -1662,6 +1510,7 @@ cudaError_t preload_kernels() {
   cudaFuncAttributes a;
   cudaError_t e = cudaFuncGetAttributes(&a, replay_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, prepass_kernel);
+  if (e == cudaSuccess) e = preload_partition_kernels();
   if (e == cudaSuccess) e = raise_dyn_smem_once();
   return e;
 }

@@ -7,7 +7,17 @@
 
 namespace pemgpu {
 
-constexpr int kNSeg = 8;          // max warps per CTA (stream-partition segments)
+// Shared-memory increment by exactly 1, unpredicated (ptxas aggregates a warp's same-address
+// increments, ATOMS.POPC.INC); lanes with nothing to count increment a sink word instead, which
+// keeps the per-element loops free of branches.
+__device__ __forceinline__ void inc_shared(uint32_t saddr) {
+  asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(saddr) : "memory");
+}
+
+#ifndef PROTEAN_WARPS
+#define PROTEAN_WARPS 8  // warps per replay CTA
+#endif
+constexpr int kNSeg = PROTEAN_WARPS;  // warps per CTA (stream-partition segments)
 constexpr int kZA = 8;            // lanes per actual-placement group (one per slice position)
 constexpr int kMaxStreams = 2 * PROTEAN_MAX_MODELS;
 constexpr int64_t kForever = INT64_MAX;
@@ -71,13 +81,11 @@ struct ReplayParams {
   TabLayout tl;
   const uint32_t* pack;    // [CW*32] candidate lane packing
   int maxT;
-  // trace (device)
-  const uint32_t* arr;
-  const uint8_t* meta;
-  const int64_t* roff;
-  const int64_t* eoff;     // [R][E+1] first request index with arrival >= e*W
+  // trace (device): the stream-sorted copy built by the partition passes (partition.cu)
+  const uint32_t* sa;      // arrivals, per replica stream-major, replica r at sa + saoff[r]
+  const int64_t* saoff;    // [R+1] 16-byte aligned replica offsets into sa
+  const uint32_t* sidx;    // [R][E+1][S] first request of stream k with arrival >= e*W (replica-relative)
   int R, N;
-  bool vec_ok;             // arr and meta 16-byte aligned at equal element indices
   int64_t base, trace_len, W, E, H;
   // policy
   int policy, wait_limit, cap_pct, init_geom, max_live, vm_policy;
@@ -128,6 +136,26 @@ struct ScoreParams {
   protean_resident* scratch;  // [R][N*(Gc)][max_live]
   int* err;                   // err[0] EINVAL, err[1] ERANGE
 };
+
+// Trace-level stream partition (partition.cu): P1 count + validate, P2 scan, P3 stable scatter.
+struct PartitionArgs {
+  const uint32_t* arr;
+  const uint8_t* meta;
+  const int64_t* roff;
+  const int64_t* eoff;     // [R][E+1]
+  const int64_t* saoff;    // [R+1]
+  int R, S, M;
+  int64_t E;
+  uint32_t tlm1;           // trace_len - 1 (arrivals fit 32 bits, host check)
+  bool vec;                // arr and meta 16-byte aligned
+  uint32_t* cnt;           // [R][E][S] scratch
+  uint32_t* sidx;          // [R][E+1][S]
+  uint32_t* sa;            // stream-sorted arrivals
+  int* err;                // err[0] |= invalid request
+};
+cudaError_t launch_partition_count(const PartitionArgs& A, cudaStream_t st);
+cudaError_t launch_partition_rest(const PartitionArgs& A, cudaStream_t st);
+cudaError_t preload_partition_kernels();
 
 // launchers (replay.cu / score.cu)
 cudaError_t launch_prepass(const uint32_t* arr, const int64_t* roff, int R, int64_t E, int64_t W,

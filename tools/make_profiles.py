@@ -39,10 +39,11 @@ def main(tag):
             f.write(f"\"{k[:80]}\",{ms:.4f}\n")
     rep = [ms for k, ms in rows if "replay_kernel" in k]
     pre = [ms for k, ms in rows if "prepass_kernel" in k]
-    step = [a + b for a, b in zip(pre, rep)]
+    parts = {n: [ms for k, ms in rows if n in k] for n in ("part_count", "part_scan", "part_scatter")}
+    step = [a + b + sum(parts[n][i] for n in parts) for i, (a, b) in enumerate(zip(pre, rep))]
     json.dump({"command": "ncu --metrics gpu__time_duration.sum --clock-control none python bench.py "
                           "--steps 2 --warmup 1 --cpu-sample 0 --e2e-replicas 0",
-               "replay_kernel_ms": rep, "prepass_ms": pre,
+               "replay_kernel_ms": rep, "prepass_ms": pre, **{f"{n}_ms": v for n, v in parts.items()},
                "replay_share_of_step": sum(rep) / sum(step) if step else None,
                "note": "cold-cache, serialised per-launch times; compare shares, not absolutes"},
               open(os.path.join(PROF, f"{tag}_launch_summary.json"), "w"), indent=1)
@@ -71,7 +72,7 @@ def main(tag):
     s = {"report": f"{tag} replay_kernel ncu --set full", "workload": f"tools/profile_run.py --replicas "
          f"{info['replicas']} --seconds {info['seconds']} (config-5 shape)", "requests": info["requests"],
          "dram_bytes_read": rd, "dram_bytes_write": wr,
-         "dram_bytes_per_request": (rd + wr) / info["requests"], "algorithmic_bytes_per_request": 5.0,
+         "dram_bytes_per_request": (rd + wr) / info["requests"], "algorithmic_bytes_per_request": 4.0,
          "duration_ms_under_ncu": dur / 1e6 if dur > 1e4 else dur,
          "issue_active_pct": get("smsp__issue_active.avg.pct_of_peak_sustained_active"),
          "warp_instructions": get("smsp__inst_executed.sum")}
