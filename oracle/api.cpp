@@ -251,8 +251,18 @@ int orc_replay(const orc_tables* t, const orc_replay_in* in, orc_replay_out* out
   int64_t maxT = 0;
   for (int m = 0; m < tb.M; ++m) maxT = std::max<int64_t>(maxT, tb.tmo[m]);
   if (in->trace_len - 1 + maxT > (int64_t)0xFFFFFFFFLL) return ORC_ERANGE;
-  if (in->policy == 2) return ORC_EUNSUP;
-  if (in->policy != 0 && in->policy != 1) return ORC_EINVAL;
+  if (in->policy < 0 || in->policy > 2) return ORC_EINVAL;
+  if (in->policy == 2) {  // Alg 2 heuristic (N1): its knobs, and both of its geometries in the set
+    if (in->ewma_alpha_pm < 1 || in->ewma_alpha_pm > 1000) return ORC_EINVAL;
+    if (in->t_low < 0 || in->t_high < in->t_low) return ORC_EINVAL;
+    const std::vector<int> g421 = {0, 1, 3}, g43 = {2, 3};  // (4g,2g,1g), (4g,3g)
+    bool h421 = false, h43 = false;
+    for (const std::vector<int>& g : tb.geoms) {
+      h421 = h421 || g == g421;
+      h43 = h43 || g == g43;
+    }
+    if (!h421 || !h43) return ORC_EINVAL;
+  }
   if (in->shard_mode != 0 && in->shard_mode != 1) return ORC_EINVAL;
   if (in->wait_limit < 0 || in->wait_limit > 255) return ORC_EINVAL;
   if (in->cap_pct < 0 || in->cap_pct > 100) return ORC_EINVAL;
@@ -295,6 +305,9 @@ int orc_replay(const orc_tables* t, const orc_replay_in* in, orc_replay_out* out
   cfg.rev_interval = in->rev_interval;
   cfg.notice = in->notice;
   cfg.seed = in->seed;
+  cfg.ewma_alpha_pm = in->ewma_alpha_pm;
+  cfg.t_low = in->t_low;
+  cfg.t_high = in->t_high;
   const int64_t E = num_epochs(tb, in->trace_len, in->W);
   const int G = (int)tb.geoms.size();
   const int N = in->N;

@@ -4,6 +4,8 @@
 // placement + request accounting (O6, O7) -> scoring of every candidate geometry for every
 // decidable GPU, from idle, on that GPU's epoch batches (O8, readings Q19-Q21, the paper's
 // "Oracle" scheme P:L485) -> Alg 2 hysteresis + ~30% cap (O9, O10).
+// policy 2 (N1) replaces the scoring by Alg 2's own heuristic (lines 1-23, readings
+// R10-R17 of DESIGN.md): EWMA of the observed BE load -> small-slice set -> thresholds -> geometry.
 #include "pem.hpp"
 #include <algorithm>
 #include <climits>
@@ -33,6 +35,8 @@ struct Gpu {
   int ctr = 0;              // Alg 2 wait_ctr
   int64_t rs = 0, re = 0;   // reconfiguration window [rs, re)
   Node node;
+  int64_t pred_num = 0;     // Alg 2 history_info (N1): EWMA of BE batches, milli-batches
+  int64_t pred_mem = 0;     //   and of their total footprint, milli-MiB (R11)
 };
 
 struct Replay {
@@ -205,10 +209,65 @@ struct Replay {
       if (want_log) out->log.insert(out->log.end(), erec.begin(), erec.end());
 
       // 4. candidate scoring for every decidable GPU (has a VM at T, no open window)
+      std::vector<int> wants;
+      std::vector<int64_t> key_best(N, -1), key_cur(N, -1);
+      std::vector<int> best(N, -1);
+      if (cfg.policy == 2) {
+        // Alg 2 GPU_Reconfigurator, one decidable GPU at a time
+        for (int n = 0; n < N; ++n) {
+          Gpu& g = gpu[n];
+          if (!(has_vm(g, T) && g.re <= T)) continue;
+          const int cur = g.S.geom;
+          // line 2: curr_queue_info = the BE batches dispatched to this GPU in the epoch (R10)
+          int64_t be_num = 0, be_mem = 0;
+          for (size_t x : list[n]) {
+            if (batches[x].strict) continue;
+            be_num += 1;
+            be_mem += tb.mem[batches[x].model];  // footprint per batch (Q36)
+          }
+          // lines 8-9: pred_BE_num, pred_BE_mem by a light-weight EWMA [95] (R11)
+          const int64_t a = cfg.ewma_alpha_pm;
+          g.pred_num = (a * 1000 * be_num + (1000 - a) * g.pred_num) / 1000;
+          g.pred_mem = (a * 1000 * be_mem + (1000 - a) * g.pred_mem) / 1000;
+          // lines 5-7, 10-18: first small-slice set whose summed capacity holds pred_BE_mem (R12)
+          const std::vector<std::vector<int>> small_slice_set = {{0, 1}, {2}};  // [[1g,2g],[3g]]
+          bool found = false;
+          std::vector<int> chosen;
+          for (const std::vector<int>& ss : small_slice_set) {
+            int64_t sum_max_mem = 0;
+            for (int p : ss) sum_max_mem += kMemMiB[p];
+            if (sum_max_mem * 1000 >= g.pred_mem) {
+              chosen = ss;
+              found = true;
+              break;
+            }
+          }
+          const int64_t pot_occupancy = g.pred_num;  // line 13 (R13)
+          const int64_t T_low = cfg.t_low, T_high = cfg.t_high;  // lines 14-15 (R14)
+          // lines 19-23 (after the loop, reading Q26)
+          std::vector<int> final_geometry;
+          if (!found || pot_occupancy < T_low || pot_occupancy > T_high) {
+            final_geometry = {2, 3};  // (4g,3g)
+          } else {
+            final_geometry = chosen;
+            final_geometry.push_back(3);  // + 4g
+          }
+          std::sort(final_geometry.begin(), final_geometry.end());
+          int fin = -1;
+          for (int j = 0; j < G && fin < 0; ++j)
+            if (tb.geoms[j] == final_geometry) fin = j;  // present: checked by the API (R15)
+          best[n] = fin;
+          out->decisions[(size_t)e * N + n] = (uint8_t)fin;
+          // lines 24-30 (reading Q22)
+          if (fin != cur) {
+            if (g.ctr >= cfg.wait_limit) wants.push_back(n);
+            else g.ctr += 1;
+          } else {
+            g.ctr = 0;
+          }
+        }
+      }
       if (cfg.policy == 0) {
-        std::vector<int> wants;
-        std::vector<int64_t> key_best(N, -1), key_cur(N, -1);
-        std::vector<int> best(N, -1);
         for (int n = 0; n < N; ++n) {
           Gpu& g = gpu[n];
           if (!(has_vm(g, T) && g.re <= T)) continue;
@@ -253,7 +312,10 @@ struct Replay {
             g.ctr = 0;
           }
         }
-        // ~30% of GPUs may reconfigure simultaneously, reading Q23
+      }
+      if (cfg.policy != 1) {
+        // ~30% of GPUs may reconfigure simultaneously, reading Q23; under policy 2 there
+        // is no miss estimate, so the order is by GPU only (R16)
         int alive = 0, open = 0;
         for (int n = 0; n < N; ++n) {
           if (has_vm(gpu[n], T)) alive++;
@@ -262,8 +324,8 @@ struct Replay {
         int cap = std::max(1, cfg.cap_pct * alive / 100);
         int free_slots = std::max(0, cap - open);
         std::stable_sort(wants.begin(), wants.end(), [&](int a, int b) {
-          int64_t da = (key_cur[a] >> 40) - (key_best[a] >> 40);
-          int64_t db = (key_cur[b] >> 40) - (key_best[b] >> 40);
+          int64_t da = cfg.policy == 0 ? (key_cur[a] >> 40) - (key_best[a] >> 40) : 0;
+          int64_t db = cfg.policy == 0 ? (key_cur[b] >> 40) - (key_best[b] >> 40) : 0;
           if (da != db) return da > db;
           return a < b;
         });

@@ -72,6 +72,8 @@ typedef struct {
   int64_t rev_interval, notice;
   uint64_t seed;
   int32_t shard_mode, nthreads;
+  int32_t ewma_alpha_pm, pad;   /* policy 2 (N1): EWMA weight per mille, 1..1000 */
+  int64_t t_low, t_high;        /* policy 2: T_low <= T_high, milli-BE-batches per epoch */
 } orc_replay_in;
 
 typedef struct {

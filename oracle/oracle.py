@@ -50,7 +50,9 @@ class ReplayIn(C.Structure):
                 ("max_live", C.c_int32), ("vm_policy", C.c_int32), ("reconfig_us", C.c_int64),
                 ("p_rev", C.c_double), ("price_od", C.c_double), ("price_spot", C.c_double),
                 ("rev_interval", C.c_int64), ("notice", C.c_int64), ("seed", C.c_uint64),
-                ("shard_mode", C.c_int32), ("nthreads", C.c_int32)]
+                ("shard_mode", C.c_int32), ("nthreads", C.c_int32),
+                ("ewma_alpha_pm", C.c_int32), ("pad", C.c_int32), ("t_low", C.c_int64),
+                ("t_high", C.c_int64)]
 
 
 class BatchRec(C.Structure):
@@ -255,7 +257,7 @@ def tick_simulate(prof, geom, t, model, slice_):
 DEFAULT_CFG = dict(N=8, W=1_000_000, policy=0, wait_limit=3, cap_pct=30, init_geom=2, max_live=64,
                    vm_policy=0, reconfig_us=2_000_000, p_rev=0.0, price_od=32.7726 / 8,
                    price_spot=9.8318 / 8, rev_interval=300_000_000, notice=30_000_000, seed=0,
-                   shard_mode=0)
+                   shard_mode=0, ewma_alpha_pm=500, t_low=500, t_high=4000)
 
 
 def replay(prof, trace, *, nthreads=1, want_keys=False, want_log=False, log_cap=None, **cfg):
@@ -270,7 +272,8 @@ def replay(prof, trace, *, nthreads=1, want_keys=False, want_log=False, log_cap=
     rin = ReplayIn(R, N, int(trace.replica_base), int(trace.trace_len_us), int(c["W"]), _p(arr) or 0,
                    _p(meta) or 0, _p(off), c["policy"], c["wait_limit"], c["cap_pct"], c["init_geom"],
                    c["max_live"], c["vm_policy"], c["reconfig_us"], c["p_rev"], c["price_od"],
-                   c["price_spot"], c["rev_interval"], c["notice"], c["seed"], c["shard_mode"], nthreads)
+                   c["price_spot"], c["rev_interval"], c["notice"], c["seed"], c["shard_mode"], nthreads,
+                   c["ewma_alpha_pm"], 0, c["t_low"], c["t_high"])
     if arr.shape[0] == 0:  # keep pointers non-NULL for empty traces
         arr = np.zeros(1, np.uint32)
         meta = np.zeros(1, np.uint8)

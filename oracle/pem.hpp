@@ -2,7 +2,8 @@
 //
 // The CPU oracle of the PROTEAN epoch model (PEM): a plain, slow, step-by-step C++17 reading of
 // the paper's slowdown model (Eq 1/2), Job Distribution (Alg 1), GPU
-// Reconfigurator decision step (Alg 2 lines 24-30 + the ~30% cap) and
+// Reconfigurator (Alg 2: decision step lines 24-30 + the ~30% cap, and its own
+// heuristic, lines 1-23, as policy 2) and
 // cost-aware procurement, with the readings of DESIGN.md §3.
 //
 // Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / --impl reference leg may
@@ -112,6 +113,8 @@ struct ReplayCfg {
   double p_rev = 0, price_od = 4.096575, price_spot = 1.228975;
   int64_t rev_interval = 300000000, notice = 30000000;
   uint64_t seed = 0;
+  int ewma_alpha_pm = 500;                 // policy 2 (N1): EWMA weight of the newest epoch, per mille
+  int64_t t_low = 500, t_high = 4000;      //   T_low / T_high, milli-BE-batches per epoch (R14)
 };
 struct BatchRec {
   uint32_t ready; uint32_t epoch; int n, model; bool strict;

@@ -552,5 +552,5 @@ def test_error_codes(oracle):
     assert code(lambda: oracle.replay(tables([[1000] * 5], [[0] * 5], [100], geoms=[[4]] * 255), tr)) == -2
     assert code(lambda: oracle.replay(tables([[1000] * 5], [[0] * 5], [100], geoms=[[3, 4]]), tr)) == -1
     assert code(lambda: oracle.replay(P, concat([(np.array([5], np.uint32), pack_meta([0], [1]))], 2**32 + 5))) == -2
-    assert code(lambda: oracle.replay(P, tr, policy=2)) == -7
+    assert code(lambda: oracle.replay(P, tr, policy=3)) == -1
     assert code(lambda: oracle.replay(P, tr)) == 0
