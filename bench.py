@@ -35,6 +35,16 @@ UNIT = "slot-evals/s"
 HBM_PEAK_FALLBACK = 6650.0
 
 
+POLICIES = {"search": 0, "alg2": 2}
+
+
+def metric_of(policy: str):
+    """search: slot-evals/s (BASELINE metric); alg2 scores no candidates: simulated requests/s."""
+    if policy == "search":
+        return METRIC, UNIT
+    return "simulated requests/s (Alg 2 heuristic policy, N1)", "requests/s"
+
+
 def peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -123,11 +133,11 @@ def oracle_sample(n_rep: int, seconds: int, seed: int = 1, base: int = 0):
     return tr
 
 
-def time_oracle(prof, tr, cores: int):
+def time_oracle(prof, tr, cores: int, policy: int = 0):
     from oracle import oracle as O
     O.build()
     t0 = time.perf_counter()
-    out = O.replay(prof, tr, N=8, nthreads=cores)
+    out = O.replay(prof, tr, N=8, nthreads=cores, policy=policy)
     dt = time.perf_counter() - t0
     c = out["counters"]
     return dt, int(c[:, 8].sum()), int((c[:, 0] + c[:, 4]).sum()), int(c[:, 9].sum())
@@ -141,25 +151,27 @@ def run_reference(args):
     cores = os.cpu_count() or 1
     n_rep = max(1, min(args.replicas, 2 * cores))
     tr = oracle_sample(n_rep, args.seconds)
+    pol = POLICIES[args.policy]
     for _ in range(args.warmup):
-        time_oracle(prof, tr, cores)
+        time_oracle(prof, tr, cores, pol)
     dts, slots, reqs = [], 0, 0
     for _ in range(args.steps):
-        dt, s, q, _g = time_oracle(prof, tr, cores)
+        dt, s, q, _g = time_oracle(prof, tr, cores, pol)
         dts.append(dt)
         slots, reqs = s, q
     tot = sum(dts)
-    val = slots * args.steps / tot
+    metric, unit = metric_of(args.policy)
+    val = (slots if pol == 0 else reqs) * args.steps / tot
     sample = f"{n_rep} replicas x {args.seconds} s of the config-5 workload (Mix A, 8 sim-GPUs, G=12)"
-    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": world,
+    line = {"impl": "reference", "metric": metric, "value": val, "unit": unit, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
             "data": "synthetic",
-            "config": {"workload": "C5 (configs[4]) sample: Mix A, 8 sim-GPUs, 600 s, G=12, search policy",
+            "config": {"workload": f"C5 (configs[4]) sample: Mix A, 8 sim-GPUs, 600 s, G=12, {args.policy} policy",
                        "replicas": n_rep, "seconds": args.seconds},
             "simulated_requests_per_s": reqs * args.steps / tot,
-            "cpu_baseline": {"value": val, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
-            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+            "cpu_baseline": {"value": val, "unit": unit, "cores": cores, "kind": "oracle", "sample": sample},
+            "e2e": {"value": val, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
 
@@ -188,7 +200,9 @@ def run_ours(args):
     E = h.num_epochs(gp.trace_len_us)
     out = h.alloc_replay_out(R, E, N, decisions=True)
     stream = torch.cuda.current_stream(dev)
-    cfg = dict(n_gpus=N, replica_base=rank * R)
+    pol = POLICIES[args.policy]
+    metric, unit = metric_of(args.policy)
+    cfg = dict(n_gpus=N, replica_base=rank * R, policy=pol)
 
     def step():
         h.replay_traces(arr, meta, roff, trace_len_us=gp.trace_len_us, out=out, stream=stream, **cfg)
@@ -228,7 +242,7 @@ def run_ours(args):
     else:
         n_req_all = n_req
     sec = tot_ms / 1e3
-    value = slot * args.steps / sec
+    value = (slot if pol == 0 else reqs) * args.steps / sec
 
     # e2e: the public call on HOST buffers (pinned), H2D + replay + D2H inside the timed region
     e2e = None
@@ -266,8 +280,9 @@ def run_ours(args):
         eb.record(stream)
         torch.cuda.synchronize()
         ems = ea.elapsed_time(eb)
-        es = int(pinned_out["counters"][:, 8].sum())
-        e2e = {"value": es * ks / (ems / 1e3), "unit": UNIT,
+        pc = pinned_out["counters"]
+        es = int(pc[:, 8].sum()) if pol == 0 else int((pc[:, 0] + pc[:, 4]).sum())
+        e2e = {"value": es * ks / (ems / 1e3), "unit": unit,
                "h2d_bytes_per_step": int(hi * 5 + (Re + 1) * 8), "d2h_bytes_per_step": int(res_bytes),
                "sample": f"{Re} of {R} replicas through Handle.replay_traces from pinned host memory"}
 
@@ -278,9 +293,9 @@ def run_ours(args):
         tr = oracle_sample(n_rep, S, base=0)
         dt, s_cpu, q_cpu, passes = 0.0, 0, 0, 0
         while passes < 1 or (dt < 10.0 and passes < 40):  # ~10 s of oracle work on the host cores
-            d, s1, q1, _ = time_oracle(prof, tr, cores)
+            d, s1, q1, _ = time_oracle(prof, tr, cores, pol)
             dt, s_cpu, q_cpu, passes = dt + d, s_cpu + s1, q_cpu + q1, passes + 1
-        cpu = {"value": s_cpu / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
+        cpu = {"value": (s_cpu if pol == 0 else q_cpu) / dt, "unit": unit, "cores": cores, "kind": "oracle",
                "sample": f"{n_rep} replicas x {S} s of this workload (numpy-generated), replayed "
                          f"{passes}x: {dt:.1f} s wall on {cores} threads",
                "simulated_requests_per_s": q_cpu / dt}
@@ -304,11 +319,11 @@ def run_ours(args):
             except Exception:
                 traffic = None
         line = {
-            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "metric": metric, "value": value, "unit": unit, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
             "config": {"workload": "C5 (configs[4]): Mix A Wiki-shaped 5000 rps, 22-model table, "
-                                   "8 sim-GPUs, 600 s, 12 geometries, search policy, on-demand VMs",
+                                   f"8 sim-GPUs, 600 s, 12 geometries, {args.policy} policy, on-demand VMs",
                        "replicas_per_rank": R, "seconds": S, "sim_gpus": N, "geometries": h.n_geoms,
                        "requests_per_rank": n_req, "l2_flush": "inputs (5 B/request, "
                        f"{5.0 * n_req / 1e9:.1f} GB per rank) exceed the 126 MB L2"},
@@ -340,6 +355,8 @@ def main():
     ap.add_argument("--seconds", type=int, default=600)
     ap.add_argument("--e2e-replicas", type=int, default=512)
     ap.add_argument("--cpu-sample", type=int, default=64, help="replicas timed on the CPU oracle")
+    ap.add_argument("--policy", default="search", choices=sorted(POLICIES),
+                    help="search = the geometry search (headline); alg2 = Alg 2's own heuristic (N1)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)

@@ -194,7 +194,9 @@ typedef struct {
   const uint8_t *meta;         /* device: bits 0..5 model id, bit 7 strict (user-annotated) */
   const int64_t *replica_off;  /* device: [R+1] offsets into arrival_us / meta */
   int32_t policy;              /* 0 = geometry search (default); 1 = fixed geometry (no search);
-                                  2 = Alg 2 heuristic (EUNSUP in this build) */
+                                  2 = Alg 2 heuristic (N1, R10-R17): EWMA of
+                                  the observed BE load -> small-slice set -> T_low/T_high ->
+                                  (4g,2g,1g) or (4g,3g); EINVAL if the geometry set lacks either */
   int32_t wait_limit;          /* Alg 2 wait_limit, default 3 (reading Q22) */
   int32_t reconfig_cap_pct;    /* default 30 (reading Q23) */
   int32_t init_geom;           /* default 2 = (4g,2g,1g) (reading Q25) */
@@ -211,7 +213,10 @@ typedef struct {
   int32_t rank, nranks;        /* mode G only: must match the handle's exchange set-up */
   int32_t max_ctas;            /* 0 = the resident capacity of the device; else caps the replay
                                   grid (lets several mode-G ranks share one GPU) */
-  int32_t reserved;            /* must be 0 */
+  int32_t ewma_alpha_pm;       /* policy 2: EWMA weight of the newest epoch, per mille, 1..1000
+                                  (default 500; R11) */
+  int64_t t_low_milli;         /* policy 2: T_low, thousandths of a BE batch per epoch (default 500) */
+  int64_t t_high_milli;        /* policy 2: T_high >= T_low (default 4000; R14) */
 } protean_replay_cfg;
 
 /* counters[10] per replica (O7/O8/O10):

@@ -74,7 +74,8 @@ class ReplayCfg(C.Structure):
                 ("p_rev", C.c_double), ("price_od_node_hr", C.c_double), ("price_spot_node_hr", C.c_double),
                 ("rev_interval_us", C.c_int64), ("notice_us", C.c_int64), ("seed", C.c_uint64),
                 ("shard_mode", C.c_int32), ("rank", C.c_int32), ("nranks", C.c_int32),
-                ("max_ctas", C.c_int32), ("reserved", C.c_int32)]
+                ("max_ctas", C.c_int32), ("ewma_alpha_pm", C.c_int32), ("t_low_milli", C.c_int64),
+                ("t_high_milli", C.c_int64)]
 
 
 class BatchRec(C.Structure):     # protean_batch_rec, 32 B

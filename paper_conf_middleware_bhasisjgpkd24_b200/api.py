@@ -14,7 +14,8 @@ _REPLAY_DEFAULTS = dict(n_gpus=8, epoch_len_us=1_000_000, policy=0, wait_limit=3
                         init_geom=2, max_live=64, vm_policy=0, reconfig_us=2_000_000, p_rev=0.0,
                         price_od_node_hr=32.7726 / 8, price_spot_node_hr=9.8318 / 8,
                         rev_interval_us=300_000_000, notice_us=30_000_000, seed=0, shard_mode=0,
-                        rank=0, nranks=1, max_ctas=0, replica_base=0)
+                        rank=0, nranks=1, max_ctas=0, replica_base=0, ewma_alpha_pm=500, t_low_milli=500,
+                        t_high_milli=4000)
 
 
 def _torch():
@@ -170,7 +171,7 @@ class Handle:
         cf.replica_off = replica_off.data_ptr()
         for k in ("policy", "wait_limit", "reconfig_cap_pct", "init_geom", "max_live", "vm_policy",
                   "reconfig_us", "rev_interval_us", "notice_us", "seed", "shard_mode", "rank", "nranks",
-                  "max_ctas"):
+                  "max_ctas", "ewma_alpha_pm", "t_low_milli", "t_high_milli"):
             setattr(cf, k, int(c[k]))
         for k in ("p_rev", "price_od_node_hr", "price_spot_node_hr"):
             setattr(cf, k, float(c[k]))

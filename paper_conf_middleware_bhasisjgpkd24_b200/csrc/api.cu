@@ -339,6 +339,9 @@ void protean_replay_cfg_defaults(protean_replay_cfg* c) {
   c->price_spot_node_hr = 9.8318 / 8.0;
   c->rev_interval_us = 300000000;
   c->notice_us = 30000000;
+  c->ewma_alpha_pm = 500;
+  c->t_low_milli = 500;
+  c->t_high_milli = 4000;
 }
 
 int protean_load_profiles(const protean_profiles* p, protean_handle** out) {
@@ -544,10 +547,20 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   if (c.epoch_len_us <= 0 || c.trace_len_us <= 0) return fail(h, PROTEAN_EINVAL, "W / trace_len");
   if (c.trace_len_us - 1 + h->maxT > (int64_t)0xFFFFFFFFLL)
     return fail(h, PROTEAN_ERANGE, "ready times exceed uint32 us");
-  if (c.policy == 2) return fail(h, PROTEAN_EUNSUP, "policy 2 (Alg 2 heuristic) not built");
-  if (c.policy != 0 && c.policy != 1) return fail(h, PROTEAN_EINVAL, "policy");
+  if (c.policy < 0 || c.policy > 2) return fail(h, PROTEAN_EINVAL, "policy");
+  int g421 = -1, g43 = -1;  // Alg 2's two outcomes (R15): (4g,2g,1g) and (4g,3g) in the loaded set
+  if (c.policy == 2) {
+    if (c.ewma_alpha_pm < 1 || c.ewma_alpha_pm > 1000) return fail(h, PROTEAN_EINVAL, "ewma_alpha_pm");
+    if (c.t_low_milli < 0 || c.t_high_milli < c.t_low_milli) return fail(h, PROTEAN_EINVAL, "t_low / t_high");
+    for (int j = 0; j < h->G; ++j) {
+      const uint8_t* row = &h->geoms[(size_t)j * 8];
+      if (g421 < 0 && row[0] == 0 && row[1] == 1 && row[2] == 3 && row[3] == 0xFF) g421 = j;
+      if (g43 < 0 && row[0] == 2 && row[1] == 3 && row[2] == 0xFF) g43 = j;
+    }
+    if (g421 < 0 || g43 < 0) return fail(h, PROTEAN_EINVAL, "policy 2 needs (4g,2g,1g) and (4g,3g) in the set");
+  }
   if (c.shard_mode != 0 && c.shard_mode != 1) return fail(h, PROTEAN_EINVAL, "shard_mode");
-  if (c.max_ctas < 0 || c.reserved != 0) return fail(h, PROTEAN_EINVAL, "max_ctas / reserved");
+  if (c.max_ctas < 0) return fail(h, PROTEAN_EINVAL, "max_ctas");
   const bool modeG = c.shard_mode == 1;
   if (modeG) {
     if (!h->x_ready) return fail(h, PROTEAN_ESTATE, "mode G without an exchange set-up");
@@ -704,6 +717,11 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   P.E = E;
   P.H = H;
   P.policy = c.policy;
+  P.ewma_a = c.ewma_alpha_pm;
+  P.t_low = c.t_low_milli;
+  P.t_high = c.t_high_milli;
+  P.g421 = g421;
+  P.g43 = g43;
   P.wait_limit = c.wait_limit;
   P.cap_pct = c.reconfig_cap_pct;
   P.init_geom = c.init_geom;

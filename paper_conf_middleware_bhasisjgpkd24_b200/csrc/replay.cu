@@ -495,6 +495,32 @@ __device__ __forceinline__ bool candidate_unit_fast(const Tab& T, const SliceLan
 
 }  // namespace
 
+// Policy 2 (N1): Alg 2 GPU_Reconfigurator lines 1-23 for decidable GPU g, readings
+// R10-R15 of DESIGN.md.  Returns final_geometry; advances the GPU's EWMA history (gi rows 12, 13).
+__device__ __noinline__ int alg2_final_geometry(const ReplayParams& P, const Ctx& c, int g,
+                                                const Bat* bats, const uint32_t* gl) {
+  int64_t be_num = 0, be_mem = 0;  // line 2: the BE batches dispatched to g this epoch (R10)
+#pragma unroll 1
+  for (int x = c.g_off[g]; x < c.g_off[g + 1]; ++x) {
+    const uint32_t info = bats[gl[x]].info;
+    if ((info >> 24) & 1u) continue;
+    be_num += 1;
+    be_mem += c.T.mem[(info >> 16) & 0xFFu];  // footprint per batch (Q36)
+  }
+  // lines 8-9: EWMA in milli-units (R11)
+  const int64_t a = P.ewma_a;
+  const int64_t X = (a * 1000 * be_num + (1000 - a) * c.gi[12 * c.N + g]) / 1000;
+  const int64_t Y = (a * 1000 * be_mem + (1000 - a) * c.gi[13 * c.N + g]) / 1000;
+  c.gi[12 * c.N + g] = X;
+  c.gi[13 * c.N + g] = Y;
+  // lines 10-18: the first of [[1g,2g],[3g]] whose summed T2 capacity holds pred_BE_mem (R12)
+  const bool fits12 = (int64_t)(prof_cap(0) + prof_cap(1)) * 1000 >= Y;
+  const bool found = fits12 || (int64_t)prof_cap(2) * 1000 >= Y;
+  // lines 19-23: thresholds on pot_occupancy = pred_BE_num (R13, R14), (4g,3g) fallback, + 4g (R15)
+  if (!found || X < P.t_low || X > P.t_high) return P.g43;
+  return fits12 ? P.g421 : P.g43;
+}
+
 __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kernel(ReplayParams P) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ CtaState cs;
@@ -585,6 +611,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
       c.gi[3 * c.N + g] = kForever;
       c.gi[4 * c.N + g] = 0;
       c.gi[8 * c.N + g] = c.gi[9 * c.N + g] = c.gi[10 * c.N + g] = c.gi[11 * c.N + g] = 0;
+      c.gi[12 * c.N + g] = c.gi[13 * c.N + g] = 0;  // Alg 2 EWMA history (policy 2)
     }
     if (tid == 0) {
       cs.nlog = 0;
@@ -1234,6 +1261,17 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
               }
               atomicAdd(&cs.cnt[8], (unsigned long long)(c.g_off[g + 1] - c.g_off[g]) * (unsigned long long)sum_slots);
               atomicAdd(&cs.cnt[9], (unsigned long long)Gc);
+            } else if (P.policy == 2 && c.gu8[5 * c.N + g]) {  // Alg 2's own heuristic (N1)
+              const int cur = c.gu8[0 * c.N + g];
+              const int fin = alg2_final_geometry(P, c, g, c.bats, c.gl);
+              dec_out = (uint8_t)fin;
+              c.gu8[6 * c.N + g] = (uint8_t)fin;
+              if (fin != cur) {  // lines 24-30 (Q22)
+                if (c.gu8[2 * c.N + g] >= P.wait_limit) want = true;
+                else c.gu8[2 * c.N + g]++;
+              } else {
+                c.gu8[2 * c.N + g] = 0;
+              }
             } else if (P.policy == 0) {
               c.gi[6 * c.N + g] = kForever;
             }
@@ -1244,13 +1282,13 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
                 P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = -1;
             }
           }
-          if (P.policy == 0) {
+          if (P.policy != 1) {
             const unsigned alive = __ballot_sync(0xffffffffu, gv && has_vm(c, g, Tend));
             const unsigned open = __ballot_sync(0xffffffffu, gv && c.gi[1 * c.N + g] > Tend);
             int cap = P.cap_pct * __popc(alive) / 100;
             if (cap < 1) cap = 1;
             int free_slots = cap - __popc(open);
-            const int64_t d = want ? (kc >> 40) - (kb >> 40) : 0;
+            const int64_t d = (want && P.policy == 0) ? (kc >> 40) - (kb >> 40) : 0;  // policy 2: GPU order (R16)
 #pragma unroll 1
             while (free_slots > 0) {
               const unsigned wm = __ballot_sync(0xffffffffu, want);
@@ -1315,6 +1353,17 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
           }
           atomicAdd(&cs.cnt[8], (unsigned long long)(c.g_off[g + 1] - c.g_off[g]) * (unsigned long long)sum_slots);
           atomicAdd(&cs.cnt[9], (unsigned long long)Gc);
+        } else if (P.policy == 2 && c.gu8[5 * c.N + g]) {  // Alg 2's own heuristic (N1)
+          const int cur = c.gu8[0 * c.N + g];
+          const int fin = alg2_final_geometry(P, c, g, c.bats, c.gl);
+          dec_out = (uint8_t)fin;
+          c.gu8[6 * c.N + g] = (uint8_t)fin;
+          if (fin != cur) {
+            if (c.gu8[2 * c.N + g] >= P.wait_limit) c.gu8[7 * c.N + g] = 1;
+            else c.gu8[2 * c.N + g]++;
+          } else {
+            c.gu8[2 * c.N + g] = 0;
+          }
         }
         if (P.decisions) P.decisions[((size_t)r * P.E + e) * N + g] = dec_out;
         if (P.policy != 0 && P.cand_keys) {
@@ -1326,7 +1375,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
       __syncthreads();
       PH(8);
       if (tid == 0) {
-        if (P.policy == 0) {
+        if (P.policy != 1) {
           int alive = 0, open = 0;
 #pragma unroll 1
           for (int g = 0; g < N; ++g) {
@@ -1343,7 +1392,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
 #pragma unroll 1
             for (int g = 0; g < N; ++g) {
               if (!c.gu8[7 * c.N + g]) continue;
-              const int64_t d = (c.gi[7 * c.N + g] >> 40) - (c.gi[6 * c.N + g] >> 40);
+              const int64_t d = P.policy == 0 ? (c.gi[7 * c.N + g] >> 40) - (c.gi[6 * c.N + g] >> 40) : 0;
               if (pick < 0 || d > pd) { pick = g; pd = d; }
             }
             if (pick < 0) break;

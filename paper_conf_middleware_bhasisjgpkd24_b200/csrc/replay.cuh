@@ -48,7 +48,8 @@ struct SmemLayout {
     tab = take((size_t)words * 4);
     pack = take((size_t)CW * 32 * 4);
     g_u8 = take((size_t)N * 8);                 // geom, target, ctr, vm, bill, dec, best, want
-    g_i64 = take((size_t)N * 12 * 8);           // rs, re, from, until, since, maxend, kbest, kcur, od, spot, busy, mem
+    g_i64 = take((size_t)N * 14 * 8);           // rs, re, from, until, since, maxend, kbest, kcur, od, spot, busy, mem,
+                                                // Alg 2 EWMA pred_num, pred_mem (policy 2)
     g_i32 = take((size_t)(2 * N + 2) * 4);      // gcnt[N], goff[N+1]
     a_n = take((size_t)N * kZA * 4);            // actual lanes: list length, last start, busy-until
     a_ls = take((size_t)N * kZA * 8);
@@ -89,6 +90,8 @@ struct ReplayParams {
   int64_t base, trace_len, W, E, H;
   // policy
   int policy, wait_limit, cap_pct, init_geom, max_live, vm_policy;
+  int ewma_a, g421, g43;   // policy 2 (N1): EWMA weight per mille, indices of (4g,2g,1g), (4g,3g)
+  int64_t t_low, t_high;   //   T_low / T_high in milli-BE-batches per epoch
   int64_t reconfig_us, rev, notice;
   uint64_t thr, seed;
   double price_od, price_spot;

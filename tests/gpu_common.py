@@ -27,7 +27,8 @@ def gpu_replay(prof, trace, *, want_keys=True, want_log=True, **cfg):
 
 ORACLE_CFG_KEYS = {"n_gpus": "N", "epoch_len_us": "W", "reconfig_cap_pct": "cap_pct",
                    "price_od_node_hr": "price_od", "price_spot_node_hr": "price_spot",
-                   "rev_interval_us": "rev_interval", "notice_us": "notice"}
+                   "rev_interval_us": "rev_interval", "notice_us": "notice", "t_low_milli": "t_low",
+                   "t_high_milli": "t_high"}
 
 
 def oracle_replay(O, prof, trace, *, want_keys=True, want_log=True, nthreads=8, **cfg):

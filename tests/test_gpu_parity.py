@@ -44,7 +44,7 @@ def test_fuzz_replay(oracle, seed):
     N = int(rng.choice([1, 2, 3, 8]))
     R = int(rng.integers(1, 6))
     tr = uniform_trace(rng, R, M, int(rng.integers(2, 12)) * 1_000_000, int(rng.integers(5, 600)))
-    cfg = dict(n_gpus=N, policy=int(rng.integers(0, 2)) if seed % 3 == 0 else 0,
+    cfg = dict(n_gpus=N, policy=int(rng.integers(0, 3)) if seed % 3 == 0 else 0,
                init_geom=int(rng.integers(0, 12)), max_live=int(rng.choice([2, 8, 64])),
                wait_limit=int(rng.integers(0, 4)), reconfig_us=int(rng.integers(0, 3_000_000)),
                vm_policy=int(seed % 3), p_rev=float(rng.choice([0.0, 0.354, 0.708, 1.0])),
@@ -157,6 +157,11 @@ def test_error_codes_match_oracle(oracle):
         (tables([[1000] * 5], [[0] * 5], [100], geoms=[[3, 4]]), good, {}),
         (P, concat([(np.array([5], np.uint32), pack_meta([0], [1]))], 2**32 + 5), {}),
         (P, good, dict(policy=2)),
+        (P, good, dict(policy=3)),
+        (tables([[1000] * 5], [[0] * 5], [100], geoms=[[4], [0, 1, 3]]), good, dict(policy=2)),
+        (P, good, dict(policy=2, ewma_alpha_pm=0)),
+        (P, good, dict(policy=2, ewma_alpha_pm=1001)),
+        (P, good, dict(policy=2, t_low_milli=10, t_high_milli=5)),
         (P, good, dict(max_live=0)),
         (P, good, dict(init_geom=12)),
         (P, good, {}),
