@@ -23,12 +23,14 @@ arr, meta, roff = tracegen.generate_on_device(gp, 0)
 A._lib = None
 L = A.load(A.LIB_PATH)
 h = pkg.load_profiles(synth_profiles())
-out = h.replay_traces(arr, meta, roff, trace_len_us=gp.trace_len_us, n_gpus=8)
+POL = int(sys.argv[3]) if len(sys.argv) > 3 else 0
+out = h.replay_traces(arr, meta, roff, trace_len_us=gp.trace_len_us, n_gpus=8, policy=POL)
 torch.cuda.synchronize()
 buf = (C.c_ulonglong * 13)()
 L.protean_debug_phase_cycles(buf)
-names = ["A vm/install", "B count", "B offsets", "B scatter", "C formation", "C rank+window",
-         "D dispatch", "E placement", "F accounting+G decide", "G cap"]
+names = ["-", "A vm/install + B window layout", "-", "B window TMA wait", "C formation",
+         "C rank (+ closed-form dispatch)", "D dispatch", "E units + F accounting", "G decide",
+         "G cap + epoch barrier"]
 tot = sum(buf[:10]) or 1
 print("kernel ms", h.last_timings()[1])
 for n, v in zip(names, buf):

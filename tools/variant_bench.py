@@ -22,7 +22,7 @@ arr, meta, roff = tracegen.generate_on_device(gp, 0)
 h = pkg.load_profiles(synth_profiles())
 ts = []
 for _ in range(4):
-    out = h.replay_traces(arr, meta, roff, trace_len_us=gp.trace_len_us, n_gpus=8)
+    out = h.replay_traces(arr, meta, roff, trace_len_us=gp.trace_len_us, n_gpus=8, ewma_alpha_pm=0)  # 0: also the reserved word of pre-N1 builds
     torch.cuda.synchronize()
     ts.append(h.last_timings()[1])
 c = out["counters"].sum(0).cpu().tolist()
