@@ -676,7 +676,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   const int Gc = geom_hi - geom_lo;
   // warps per CTA: the placement phase runs n_units warp units; pick 4..8 warps that divide them
   // most evenly (prefer more warps on ties)
-  const int n_units = (N + 3) / 4 + (c.policy == 0 ? N * CW : 0);
+  const int n_units = (N + kAG - 1) / kAG + (c.policy == 0 ? N * CW : 0);
   (void)n_units;
   const int block = 32 * kWarps;  // measured on B200: 8 warps x 3 CTAs/SM beat 6 x 4
   SmemLayout sl;

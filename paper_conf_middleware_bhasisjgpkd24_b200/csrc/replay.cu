@@ -592,7 +592,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
   int sum_slots = 0;  // slot-evals per batch per decidable GPU
 #pragma unroll 1
   for (int j = P.geom_lo; j < P.geom_hi; ++j) sum_slots += T.gn[j];
-  const int n_aunits = (N + 3) / 4;  // actual-placement warp units: 4 GPUs x 8 slice lanes
+  const int n_aunits = (N + kAG - 1) / kAG;  // actual-placement warp units: kAG GPUs x 8 slice lanes
   const uint32_t* sarr = c.sarr;
 
 #pragma unroll 1
@@ -1085,11 +1085,11 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
         int g, s, Z, gbase, j;
         bool valid;
         if (actual) {
-          g = u * 4 + (lane >> 3);
+          g = u * kAG + (lane >> 3);
           s = lane & 7;
           Z = kZA;
           gbase = lane & ~7;
-          valid = g < N;
+          valid = (lane >> 3) < kAG && g < N;
           j = valid ? c.gu8[0 * c.N + g] : 0;
         } else {
           const int cu = u - n_aunits, w = cu % CW;

@@ -19,6 +19,10 @@ __device__ __forceinline__ void inc_shared(uint32_t saddr) {
 #endif
 constexpr int kNSeg = PROTEAN_WARPS;  // warps per CTA (stream-partition segments)
 constexpr int kZA = 8;            // lanes per actual-placement group (one per slice position)
+#ifndef PROTEAN_AGPU
+#define PROTEAN_AGPU 4
+#endif
+constexpr int kAG = PROTEAN_AGPU;  // simulated GPUs per actual-placement warp unit (1, 2 or 4)
 constexpr int kMaxStreams = 2 * PROTEAN_MAX_MODELS;
 constexpr int64_t kForever = INT64_MAX;
 

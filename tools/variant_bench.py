@@ -17,12 +17,13 @@ from tools import tracegen  # noqa: E402
 
 R = int(sys.argv[2]) if len(sys.argv) > 2 else 4096
 S = int(sys.argv[3]) if len(sys.argv) > 3 else 60
+POL = int(os.environ.get("PROTEAN_VB_POLICY", "0"))
 gp = mix_a_params(R, seed=1, seconds=S)
 arr, meta, roff = tracegen.generate_on_device(gp, 0)
 h = pkg.load_profiles(synth_profiles())
 ts = []
 for _ in range(4):
-    out = h.replay_traces(arr, meta, roff, trace_len_us=gp.trace_len_us, n_gpus=8, ewma_alpha_pm=0)  # 0: also the reserved word of pre-N1 builds
+    out = h.replay_traces(arr, meta, roff, trace_len_us=gp.trace_len_us, n_gpus=8, ewma_alpha_pm=0 if POL != 2 else 500, policy=POL)  # 0: also the reserved word of pre-N1 builds
     torch.cuda.synchronize()
     ts.append(h.last_timings()[1])
 c = out["counters"].sum(0).cpu().tolist()
