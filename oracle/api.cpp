@@ -479,4 +479,65 @@ int orc_score_epoch(const orc_tables* t, int32_t R, int32_t N, int32_t epoch, in
   return ORC_OK;
 }
 
+int orc_sweep(const orc_tables* t, int32_t R, int32_t N, int32_t max_live, int32_t max_batches,
+              const uint32_t* b_ready, const uint32_t* b_req_off, const int32_t* b_n,
+              const int32_t* b_model, const int32_t* b_strict, const int32_t* batch_off,
+              const uint32_t* arrival, const uint8_t* cur_geom, int32_t geom_lo, int32_t geom_hi,
+              int64_t* sweep_key, uint32_t* assign, int64_t* best_key, int64_t* n_assign) {
+  Tables tb;
+  int rc = build_tables(t, &tb);
+  if (rc) return rc;
+  const int G = (int)tb.geoms.size();
+  if (R < 1 || N < 1) return ORC_EINVAL;
+  if (N > 255) return ORC_ERANGE;
+  if (max_live < 1 || max_live > 64) return ORC_EINVAL;
+  if (max_batches < 1 || max_batches > 8) return ORC_EINVAL;
+  if (geom_lo < 0 || geom_hi > G || geom_lo >= geom_hi) return ORC_EINVAL;
+  if (!batch_off || !cur_geom || !best_key || !n_assign) return ORC_EINVAL;
+  if (batch_off[0] != 0) return ORC_EINVAL;
+  for (int x = 0; x < R * N; ++x) {
+    if (batch_off[x + 1] < batch_off[x]) return ORC_EINVAL;
+    if (cur_geom[x] != 0xFF && cur_geom[x] >= G) return ORC_EINVAL;
+    for (int32_t b = batch_off[x]; b < batch_off[x + 1]; ++b) {
+      if (b_model[b] < 0 || b_model[b] >= tb.M || b_n[b] < 1) return ORC_EINVAL;
+      if (b > batch_off[x] && b_ready[b] < b_ready[b - 1]) return ORC_EINVAL;
+      for (int i = 0; i < b_n[b]; ++i) {
+        uint32_t a = arrival[b_req_off[b] + i];
+        if (a > b_ready[b] || (i > 0 && a < arrival[b_req_off[b] + i - 1])) return ORC_EINVAL;
+      }
+    }
+    if (batch_off[x + 1] - batch_off[x] > max_batches) return ORC_ERANGE;
+  }
+  const int nc = geom_hi - geom_lo;
+  uint64_t total = 0;
+  for (int x = 0; x < R * N; ++x) {
+    std::vector<SweepBatch> bs;
+    for (int32_t b = batch_off[x]; b < batch_off[x + 1]; ++b) {
+      SweepBatch sb;
+      sb.ready = b_ready[b];
+      sb.model = b_model[b];
+      sb.strict = b_strict[b] != 0;
+      sb.arr.assign(arrival + b_req_off[b], arrival + b_req_off[b] + b_n[b]);
+      bs.push_back(sb);
+    }
+    best_key[x] = -1;
+    for (int j = geom_lo; j < geom_hi; ++j) {
+      int64_t key;
+      uint64_t idx;
+      sweep_gpu(tb, j, cur_geom[x] == j ? 0 : j + 1, bs, max_live, &key, &idx, &total);
+      const int S = (int)tb.geoms[j].size();
+      uint32_t code = 0;
+      for (size_t k = 0; k < bs.size(); ++k) {  // base-S digits -> 3-bit slice fields
+        code |= (uint32_t)(idx % (uint64_t)S) << (3 * k);
+        idx /= (uint64_t)S;
+      }
+      if (sweep_key) sweep_key[(int64_t)x * nc + (j - geom_lo)] = key;
+      if (assign) assign[(int64_t)x * nc + (j - geom_lo)] = code;
+      if (best_key[x] < 0 || key < best_key[x]) best_key[x] = key;
+    }
+  }
+  *n_assign += (int64_t)total;
+  return ORC_OK;
+}
+
 }  // extern "C"

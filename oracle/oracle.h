@@ -105,6 +105,16 @@ int orc_score_epoch(const orc_tables *t, int32_t R, int32_t N, int32_t epoch, in
                     int64_t *p_start, int64_t *p_end, int32_t *p_slice, int32_t *p_dropped,
                     int64_t *counters, int64_t *accum);
 
+/* N4a exhaustive assignment sweep (readings R18-R21): per (replica, gpu) and geometry j in
+ * [geom_lo, geom_hi) the min key over every assignment of the GPU's batches (<= max_batches <= 8)
+ * to j's slices, scheduled from idle with the slice forced; assign = slice of batch x in bits
+ * 3x..3x+2 of the lowest-index minimiser; best_key = min over the range, tag 0 when j == cur_geom. */
+int orc_sweep(const orc_tables *t, int32_t R, int32_t N, int32_t max_live, int32_t max_batches,
+              const uint32_t *b_ready, const uint32_t *b_req_off, const int32_t *b_n,
+              const int32_t *b_model, const int32_t *b_strict, const int32_t *batch_off,
+              const uint32_t *arrival, const uint8_t *cur_geom, int32_t geom_lo, int32_t geom_hi,
+              int64_t *sweep_key, uint32_t *assign, int64_t *best_key, int64_t *n_assign);
+
 #ifdef __cplusplus
 }
 #endif

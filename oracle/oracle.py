@@ -115,6 +115,8 @@ def lib():
         L.orc_replay.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p]
         L.orc_score_epoch.argtypes = ([C.c_void_p] + [C.c_int32] * 4 + [C.c_int64] * 2 +
                                       [C.c_void_p] * 8 + [C.c_int32] * 2 + [C.c_void_p] * 8)
+        L.orc_sweep.argtypes = ([C.c_void_p] + [C.c_int32] * 4 + [C.c_void_p] * 8 + [C.c_int32] * 2 +
+                                [C.c_void_p] * 4)
         _lib = L
     return _lib
 
@@ -329,4 +331,34 @@ def score_epoch(prof, *, R, N, epoch, batches, batch_off, arrival, states, geom_
         raise OracleError(rc)
     for k in ("start", "end", "slice", "dropped"):
         out[k] = out[k][:nb]
+    return out
+
+
+def sweep(prof, *, R, N, batches, batch_off, arrival, cur_geom, geom_lo=0, geom_hi=None, max_live=64,
+          max_batches=8):
+    """N4a exhaustive assignment sweep (orc_sweep); batches as for score_epoch."""
+    T = OTables(prof)
+    G = table_geometries(prof).shape[0]
+    if geom_hi is None:
+        geom_hi = G
+    arrs = {k: np.ascontiguousarray(batches[k], np.uint32 if k in ("ready", "req_off") else np.int32)
+            for k in ("ready", "req_off", "n", "model", "strict")}
+    for k in arrs:
+        if arrs[k].shape[0] == 0:
+            arrs[k] = np.zeros(1, arrs[k].dtype)
+    boff = np.ascontiguousarray(batch_off, np.int32)
+    arrival = np.ascontiguousarray(arrival, np.uint32)
+    if arrival.shape[0] == 0:
+        arrival = np.zeros(1, np.uint32)
+    cg = np.ascontiguousarray(cur_geom, np.uint8)
+    nc = geom_hi - geom_lo
+    out = dict(sweep_key=np.zeros(R * N * max(nc, 0), np.int64), assign=np.zeros(R * N * max(nc, 0), np.uint32),
+               best_key=np.zeros(R * N, np.int64), n_assign=np.zeros(1, np.int64))
+    rc = lib().orc_sweep(T.ref, R, N, max_live, max_batches, _p(arrs["ready"]), _p(arrs["req_off"]),
+                         _p(arrs["n"]), _p(arrs["model"]), _p(arrs["strict"]), _p(boff), _p(arrival),
+                         _p(cg), geom_lo, geom_hi, _p(out["sweep_key"]), _p(out["assign"]),
+                         _p(out["best_key"]), _p(out["n_assign"]))
+    if rc:
+        raise OracleError(rc)
+    out["n_assign"] = int(out["n_assign"][0])
     return out

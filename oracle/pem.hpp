@@ -143,4 +143,16 @@ void tick_simulate(const Tables& tb, const std::vector<int>& geom, std::vector<T
 // key of O8 (reading Q20)
 int64_t make_key(int64_t misses, int64_t tail, int tag);
 
+// ---- N4a: exhaustive assignment sweep (oracle/sweep.cpp, readings R18-R21) ---------------------
+struct SweepBatch {
+  int64_t ready = 0;
+  int model = 0;
+  bool strict = false;
+  std::vector<uint32_t> arr;  // member arrivals, ascending
+};
+PlaceOut place_forced(const Tables& tb, const std::vector<int>& geom, GpuState& S, int64_t t, int m,
+                      bool strict, int max_live, int slice);
+void sweep_gpu(const Tables& tb, int j, int tag, const std::vector<SweepBatch>& bs, int max_live,
+               int64_t* key_out, uint64_t* idx_out, uint64_t* n_assign);
+
 }  // namespace pem
