@@ -268,6 +268,40 @@ int protean_last_timings(const protean_handle *h, float *prepass_ms, float *repl
 void protean_replay_cfg_defaults(protean_replay_cfg *cfg);
 
 /* ---------------------------------------------------------------------------------------------
+ * 3b. Exhaustive assignment sweep (N4a): the paper's "Oracle" scheme, "ideal GPU configurations
+ *     ... obtained through multiple offline ... scheduling sweeps".  For every
+ *     (replica, sim-GPU) with b <= max_batches dispatched batches of one epoch and every geometry j
+ *     in [geom_lo, geom_hi), all S_j^b assignments of the batches to j's slices are scheduled from
+ *     idle with the slice forced (Place O6 restricted to that slice: live bound, footprint, FIFO +
+ *     memory wait, Eq 1 at the start instant over the slice's co-runners; R18-R21) and
+ *     scored with the O8 key; the minimum is kept.  Alg 1's greedy choice is one of the
+ *     assignments, so sweep_key[j] never exceeds protean_score_epoch's cand_key[j].
+ *     Synchronous (returns after the outputs are written).  Device pointers.                     */
+typedef struct {
+  int32_t n_replicas, n_gpus;      /* R >= 1, 1 <= N <= 255 */
+  int32_t max_live;                /* 1..64 (reading Q39) */
+  int32_t max_batches;             /* 1..8: a GPU with more batches -> PROTEAN_ERANGE */
+  const protean_batch *batches;    /* ordered by (replica, gpu, batch id); ready non-decreasing per GPU */
+  const int32_t *batch_off;        /* [R*N+1] CSR offsets into batches */
+  const uint32_t *arrival_us;      /* members referenced by req_off: sorted, each <= the batch's ready */
+  const uint8_t *cur_geom;         /* [R*N] current geometry (its key carries tag 0), 0xFF = none */
+  int32_t geom_lo, geom_hi;        /* geometry range; [0, G) = all */
+} protean_sweep_in;
+
+typedef struct {
+  int64_t *sweep_key;   /* [R*N*(hi-lo)] min key over the assignments (tag 0 if j == cur, else j+1), or NULL */
+  uint32_t *assign;     /* [R*N*(hi-lo)] the lowest-index minimiser: slice of batch x in bits 3x..3x+2, or NULL */
+  int64_t *best_key;    /* [R*N] min over the range */
+  int64_t *n_assign;    /* [1] ACCUMULATED (+=): assignments scored, sum over (GPU, j) of S_j^b */
+} protean_sweep_out;
+
+/* Errors: EINVAL (sizes, range, null pointers, batch_off[0] != 0 or decreasing, model id >= M,
+ * n_req < 1, ready not sorted per GPU, members unsorted or after ready, cur_geom >= G),
+ * ERANGE (a GPU with more than max_batches batches).  With several faults, the code of one. */
+int protean_sweep_assignments(protean_handle *h, const protean_sweep_in *in, protean_sweep_out *out,
+                              void *stream);
+
+/* ---------------------------------------------------------------------------------------------
  * 4. Mode G: geometry-range sharding with one min-loc exchange per replica-epoch (SURVEY §8(e),
  *    S8 "argmin over geometries + cross-rank min-loc"; the search is the Oracle's sweep).
  *

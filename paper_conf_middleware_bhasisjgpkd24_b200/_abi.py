@@ -78,6 +78,18 @@ class ReplayCfg(C.Structure):
                 ("t_high_milli", C.c_int64)]
 
 
+class SweepIn(C.Structure):      # protean_sweep_in
+    _fields_ = [("n_replicas", C.c_int32), ("n_gpus", C.c_int32), ("max_live", C.c_int32),
+                ("max_batches", C.c_int32), ("batches", C.c_void_p), ("batch_off", C.c_void_p),
+                ("arrival_us", C.c_void_p), ("cur_geom", C.c_void_p), ("geom_lo", C.c_int32),
+                ("geom_hi", C.c_int32)]
+
+
+class SweepOut(C.Structure):     # protean_sweep_out
+    _fields_ = [("sweep_key", C.c_void_p), ("assign", C.c_void_p), ("best_key", C.c_void_p),
+                ("n_assign", C.c_void_p)]
+
+
 class BatchRec(C.Structure):     # protean_batch_rec, 32 B
     _fields_ = [("ready_us", C.c_uint32), ("epoch", C.c_uint32), ("n_req", C.c_uint16), ("model", C.c_uint8),
                 ("strict", C.c_uint8), ("gpu", C.c_uint8), ("slice", C.c_uint8), ("dropped", C.c_uint8),
@@ -121,6 +133,7 @@ def load(path: str = LIB_PATH, require_cuda: bool = True):
     L.protean_get_geometries.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p]
     L.protean_num_epochs.argtypes = [C.c_void_p, C.c_int64, C.c_int64, C.c_void_p]
     L.protean_score_epoch.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
+    L.protean_sweep_assignments.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
     L.protean_replay_traces.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
     L.protean_replay_cfg_defaults.argtypes = [C.c_void_p]
     L.protean_replay_cfg_defaults.restype = None

@@ -231,6 +231,35 @@ class Handle:
         out["placement"] = out["placement"][:nb]
         return out
 
+    def sweep_assignments(self, *, n_replicas, n_gpus, batches, batch_off, arrival_us, cur_geom,
+                          geom_lo=0, geom_hi=None, max_live=64, max_batches=8, want_sweep_keys=True,
+                          out=None, stream=None):
+        """protean_sweep_assignments (N4a).  batches: uint8 device tensor of protean_batch rows
+        (16 B each); batch_off int32 [R*N+1]; arrival_us uint32/int32; cur_geom uint8 [R*N]."""
+        torch = _torch()
+        dev = torch.device("cuda", self.device)
+        geom_hi = self.n_geoms if geom_hi is None else geom_hi
+        R, N = int(n_replicas), int(n_gpus)
+        nc = geom_hi - geom_lo
+        if out is None:
+            out = dict(best_key=torch.zeros(R * N, dtype=torch.int64, device=dev),
+                       n_assign=torch.zeros(1, dtype=torch.int64, device=dev))
+            if want_sweep_keys:
+                out["sweep_key"] = torch.zeros(R * N * max(nc, 1), dtype=torch.int64, device=dev)
+                out["assign"] = torch.zeros(R * N * max(nc, 1), dtype=torch.int32, device=dev)
+        nb = batches.numel() // 16
+        si = A.SweepIn(R, N, int(max_live), int(max_batches),
+                       batches.data_ptr() if nb else batch_off.data_ptr(), batch_off.data_ptr(),
+                       arrival_us.data_ptr() if arrival_us.numel() else batch_off.data_ptr(),
+                       cur_geom.data_ptr(), int(geom_lo), int(geom_hi))
+        so = A.SweepOut(out["sweep_key"].data_ptr() if "sweep_key" in out else None,
+                        out["assign"].data_ptr() if "assign" in out else None,
+                        out["best_key"].data_ptr(), out["n_assign"].data_ptr())
+        st = stream if stream is not None else torch.cuda.current_stream(self.device)
+        _check(self._h, self._lib.protean_sweep_assignments(self._h, C.byref(si), C.byref(so),
+                                                            C.c_void_p(st.cuda_stream)))
+        return out
+
 
 def load_profiles(profiles, device: int = 0) -> Handle:
     return Handle(profiles, device)

@@ -296,6 +296,7 @@ int xchg_finish(protean_handle* h) {
   // load every kernel now: lazy module loading at first launch must not run while a peer rank's
   // replay kernel in this process spins on the exchange
   CK(h, preload_kernels());
+  CK(h, preload_sweep_kernel());
   CK(h, cudaMalloc(&h->d_xpeer, sizeof(char*) * h->xpeer.size()));
   CK(h, cudaMemcpy(h->d_xpeer, h->xpeer.data(), sizeof(char*) * h->xpeer.size(), cudaMemcpyHostToDevice));
   h->x_ready = true;
@@ -857,6 +858,58 @@ int protean_score_epoch(protean_handle* h, const protean_epoch_in* in, protean_e
   CK(h, cudaStreamSynchronize(st));
   if (errs[0]) return fail(h, PROTEAN_EINVAL, "invalid state / batch");
   if (errs[1]) return fail(h, PROTEAN_ERANGE, "n_live > max_live");
+  return PROTEAN_OK;
+}
+
+
+int protean_sweep_assignments(protean_handle* h, const protean_sweep_in* in, protean_sweep_out* out,
+                              void* stream) {
+  if (!h) return PROTEAN_EINVAL;
+  if (h->poisoned) return PROTEAN_ESTATE;
+  if (!in || !out) return fail(h, PROTEAN_EINVAL, "null in/out");
+  if (in->n_replicas < 1 || in->n_gpus < 1) return fail(h, PROTEAN_EINVAL, "sizes");
+  if (in->n_gpus > 255) return fail(h, PROTEAN_ERANGE, "n_gpus > 255");
+  if (in->max_live < 1 || in->max_live > PROTEAN_MAX_LIVE) return fail(h, PROTEAN_EINVAL, "max_live");
+  if (in->max_batches < 1 || in->max_batches > 8) return fail(h, PROTEAN_EINVAL, "max_batches");
+  if (in->geom_lo < 0 || in->geom_hi > h->G || in->geom_lo >= in->geom_hi)
+    return fail(h, PROTEAN_EINVAL, "geometry range");
+  if (!in->batch_off || !in->cur_geom || !out->best_key || !out->n_assign)
+    return fail(h, PROTEAN_EINVAL, "null pointer");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  CK(h, cudaSetDevice(h->device));
+  int32_t b0 = 0;
+  CK(h, cudaMemcpyAsync(&b0, in->batch_off, 4, cudaMemcpyDeviceToHost, st));
+  CK(h, cudaStreamSynchronize(st));
+  if (b0 != 0) return fail(h, PROTEAN_EINVAL, "batch_off[0] != 0");
+  int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 64);
+  CK(h, cudaMemsetAsync(d_err, 0, 16, st));
+  SweepParams P;
+  std::memset(&P, 0, sizeof(P));
+  P.tab = h->d_tab;
+  P.tl = h->tl;
+  P.R = in->n_replicas;
+  P.N = in->n_gpus;
+  P.max_live = in->max_live;
+  P.max_batches = in->max_batches;
+  P.geom_lo = in->geom_lo;
+  P.geom_hi = in->geom_hi;
+  P.batches = in->batches;
+  P.batch_off = in->batch_off;
+  P.arrival = in->arrival_us;
+  P.cur_geom = in->cur_geom;
+  P.sweep_key = out->sweep_key;
+  P.assign = out->assign;
+  P.best_key = out->best_key;
+  P.n_assign = out->n_assign;
+  P.err = d_err;
+  const int64_t units = (int64_t)in->n_replicas * in->n_gpus;
+  const int grid = (int)std::min<int64_t>(units, (int64_t)h->nsm * 8);
+  CK(h, launch_sweep(P, grid, st));
+  int errs[2] = {0, 0};
+  CK(h, cudaMemcpyAsync(errs, d_err, 8, cudaMemcpyDeviceToHost, st));
+  CK(h, cudaStreamSynchronize(st));
+  if (errs[0]) return fail(h, PROTEAN_EINVAL, "invalid batch / offsets / cur_geom");
+  if (errs[1]) return fail(h, PROTEAN_ERANGE, "more than max_batches batches on a GPU");
   return PROTEAN_OK;
 }
 

@@ -144,6 +144,24 @@ struct ScoreParams {
   int* err;                   // err[0] EINVAL, err[1] ERANGE
 };
 
+// N4a exhaustive assignment sweep (sweep.cu)
+struct SweepParams {
+  const int32_t* tab;
+  TabLayout tl;
+  int R, N, max_live, max_batches, geom_lo, geom_hi;
+  const protean_batch* batches;
+  const int32_t* batch_off;
+  const uint32_t* arrival;
+  const uint8_t* cur_geom;
+  int64_t* sweep_key;
+  uint32_t* assign;
+  int64_t* best_key;
+  int64_t* n_assign;
+  int* err;                   // err[0] EINVAL, err[1] ERANGE
+};
+cudaError_t launch_sweep(const SweepParams& P, int grid, cudaStream_t st);
+cudaError_t preload_sweep_kernel();
+
 // Trace-level stream partition (partition.cu): P1 count + validate, P2 scan, P3 stable scatter.
 struct PartitionArgs {
   const uint32_t* arr;
