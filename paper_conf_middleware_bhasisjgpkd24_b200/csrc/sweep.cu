@@ -21,6 +21,9 @@ namespace {
 
 constexpr int kSwMax = 8;      // batches per unit (max_batches cap)
 constexpr int kSwThreads = 256;
+#ifndef PROTEAN_SWEEP_MINB
+#define PROTEAN_SWEEP_MINB 3  // resident CTAs per SM the register budget is sized for
+#endif
 
 struct SwBatch {
   int64_t ready;
@@ -29,6 +32,7 @@ struct SwBatch {
   int32_t strict;
   int32_t slo;
   uint32_t moff;     // first member in the arrival array
+  int64_t a_first, a_last;  // first and last member arrivals (the both-ends SLO tests)
 };
 
 struct SwShared {
@@ -38,13 +42,16 @@ struct SwShared {
   int32_t cap[8];          // slice capacity MiB
   int64_t wkey[kSwThreads / 32];
   uint32_t widx[kSwThreads / 32];
+  int64_t tb;    // first ready time of the unit: schedule times are relative to it
+  bool narrow;   // every relative time of any assignment fits int32 (bound below)
   int nb;
 };
 
 // members of a placed strict batch that miss the SLO: #{a : end - a > slo} over sorted arrivals
-__device__ __forceinline__ int strict_misses(const uint32_t* arr, int n, int64_t end, int64_t slo) {
-  if (end - (int64_t)__ldg(arr) <= slo) return 0;             // the earliest member meets it
-  if (end - (int64_t)__ldg(arr + n - 1) > slo) return n;      // even the latest misses
+__device__ __forceinline__ int strict_misses(const SwBatch& b, const uint32_t* arr, int n, int64_t end,
+                                             int64_t slo) {
+  if (end - b.a_first <= slo) return 0;  // the earliest member meets it
+  if (end - b.a_last > slo) return n;    // even the latest misses
   int lo = 0, hi = n;  // first index with end - a <= slo  <=>  a >= end - slo
   const int64_t need = end - slo;
   while (lo < hi) {
@@ -58,88 +65,136 @@ __device__ __forceinline__ bool key_less(int64_t k1, uint32_t i1, int64_t k2, ui
   return k1 < k2 || (k1 == k2 && i1 < i2);
 }
 
-// Every assignment idx in [first, total) step `step` of a unit with exactly kB batches on a
-// geometry with S slices; returns the thread's best (key without tag, idx).
-template <int kB>
-__device__ __forceinline__ void sweep_range(const SwShared& sh, const uint32_t* arrival, int S, uint32_t total,
-                                            uint32_t first, uint32_t step, int max_live, int64_t* bk,
-                                            uint32_t* bi) {
+// Batch X of a unit placed on its forced slice sl[X] after batches 0..X-1 (R19): live bound,
+// footprint, FIFO after the slice's last start, memory wait, Eq 1 at the start instant over the
+// slice's co-runners; then its share of the key (strict misses / BE tail).  Times are relative to
+// the unit's first ready time tb, in TT (int32_t when the unit's bound fits, else int64_t).  X is a
+// constant after unrolling, so the schedule arrays stay in registers.
+template <int kB, typename TT>
+__device__ __forceinline__ void place_at(const int X, const SwShared& sh, const int (&sl)[kB], TT (&st)[kB],
+                                         TT (&en)[kB], bool (&ok)[kB], int max_live, int64_t tb,
+                                         const uint32_t* arrival, int64_t& misses, int64_t& tail) {
+  const SwBatch& b = sh.b[X];
+  const int s = sl[X];
+  const TT t = (TT)(b.ready - tb);
+  int live = 0;
+  TT ls = 0;
+#pragma unroll
+  for (int y = 0; y < kB; ++y) {
+    if (y >= X) break;
+    live += (ok[y] && en[y] > t) ? 1 : 0;
+    if (ok[y] && sl[y] == s && st[y] > ls) ls = st[y];  // FIFO: the slice's last start
+  }
+  const int32_t Ms = sh.cap[s];
+  ok[X] = live < max_live && b.q <= Ms;
+  st[X] = en[X] = 0;
+  if (ok[X]) {
+    const TT t0 = t > ls ? t : ls;
+    int32_t used = b.q;  // only batches that fit a slice are held: sums stay far below 2^31
+#pragma unroll
+    for (int y = 0; y < kB; ++y) {
+      if (y >= X) break;
+      if (ok[y] && sl[y] == s && en[y] > t0) used += sh.b[y].q;
+    }
+    TT start = t0;
+    if (used > Ms) {  // memory wait: the earliest release after which the batch fits
+      start = (TT)(sizeof(TT) == 4 ? INT32_MAX : INT64_MAX);
+#pragma unroll
+      for (int y = 0; y < kB; ++y) {
+        if (y >= X) break;
+        if (!(ok[y] && sl[y] == s && en[y] > t0)) continue;
+        int32_t rem = b.q;
+#pragma unroll
+        for (int z = 0; z < kB; ++z) {
+          if (z >= X) break;
+          if (ok[z] && sl[z] == s && en[z] > en[y]) rem += sh.b[z].q;
+        }
+        if (rem <= Ms && en[y] < start) start = en[y];
+      }
+    }
+    int64_t F = sh.fx[X][s];
+#pragma unroll
+    for (int y = 0; y < kB; ++y) {
+      if (y >= X) break;
+      if (ok[y] && sl[y] == s && st[y] <= start && start < en[y]) F += sh.fx[y][s];
+    }
+    st[X] = start;
+    en[X] = start + (TT)exec_time(sh.sx[X][s], F);
+  }
+  if (b.strict) {
+    misses += ok[X] ? strict_misses(b, arrival + b.moff, b.n, tb + (int64_t)en[X], b.slo) : b.n;
+  } else {
+    const int64_t tv = ok[X] ? tb + (int64_t)en[X] - b.a_first : (int64_t)0xFFFFFFFFLL;
+    tail = tv > tail ? tv : tail;
+  }
+}
+
+// The assignments of a unit with exactly kB batches on a geometry with S slices, shared-prefix
+// enumeration: a thread owns prefixes (slices of batches 0..kB-D-1, index p = sum s_x S^x), places
+// them once, then loops over the last D batches' slices re-placing only what changed -- about
+// S/(S-1) placements per assignment instead of kB.  Keeps the thread's min (key, index).
+template <int kB, int D, typename TT>
+__device__ __forceinline__ void sweep_range(const SwShared& sh, const uint32_t* arrival, int S, uint32_t first,
+                                            uint32_t step, int max_live, int64_t tb, int64_t* bk, uint32_t* bi) {
+  constexpr int K = kB - D;
+  uint32_t npre = 1;
+  for (int x = 0; x < K; ++x) npre *= (uint32_t)S;
+  const uint32_t wK = npre, wK1 = npre * (uint32_t)S;  // index weights of batches K and K+1
   int64_t best = INT64_MAX;
   uint32_t bidx = 0;
 #pragma unroll 1
-  for (uint32_t idx = first; idx < total; idx += step) {
+  for (uint32_t p = first; p < npre; p += step) {
     int sl[kB];
+    TT st[kB], en[kB];
+    bool ok[kB];
+    int64_t m0 = 0, t0 = 0;
     {
-      uint32_t rem = idx;
+      uint32_t rem = p;
 #pragma unroll
-      for (int x = 0; x < kB; ++x) {
+      for (int x = 0; x < K; ++x) {
         const uint32_t qd = rem / (uint32_t)S;
         sl[x] = (int)(rem - qd * (uint32_t)S);
         rem = qd;
       }
     }
-    int64_t st[kB], en[kB];
-    bool ok[kB];
-    int64_t misses = 0, tail = 0;
 #pragma unroll
-    for (int x = 0; x < kB; ++x) {
-      const SwBatch& b = sh.b[x];
-      const int s = sl[x];
-      const int64_t t = b.ready;
-      int live = 0;
-      int64_t ls = 0;
-#pragma unroll
-      for (int y = 0; y < x; ++y) {
-        live += (ok[y] && en[y] > t) ? 1 : 0;
-        if (ok[y] && sl[y] == s && st[y] > ls) ls = st[y];  // FIFO: the slice's last start
-      }
-      const int32_t Ms = sh.cap[s];
-      ok[x] = live < max_live && b.q <= Ms;
-      st[x] = en[x] = 0;
-      if (ok[x]) {
-        const int64_t t0 = t > ls ? t : ls;
-        int64_t used = b.q;
-#pragma unroll
-        for (int y = 0; y < x; ++y)
-          if (ok[y] && sl[y] == s && en[y] > t0) used += sh.b[y].q;
-        int64_t start = t0;
-        if (used > Ms) {  // memory wait: the earliest release after which the batch fits
-          start = INT64_MAX;
-#pragma unroll
-          for (int y = 0; y < x; ++y) {
-            if (!(ok[y] && sl[y] == s && en[y] > t0)) continue;
-            int64_t rem = b.q;
-#pragma unroll
-            for (int z = 0; z < x; ++z)
-              if (ok[z] && sl[z] == s && en[z] > en[y]) rem += sh.b[z].q;
-            if (rem <= Ms && en[y] < start) start = en[y];
-          }
-        }
-        int64_t F = sh.fx[x][s];
-#pragma unroll
-        for (int y = 0; y < x; ++y)
-          if (ok[y] && sl[y] == s && st[y] <= start && start < en[y]) F += sh.fx[y][s];
-        st[x] = start;
-        en[x] = start + exec_time(sh.sx[x][s], F);
-      }
-      if (b.strict) {
-        misses += ok[x] ? strict_misses(arrival + b.moff, b.n, en[x], b.slo) : b.n;
+    for (int x = 0; x < K; ++x) place_at<kB, TT>(x, sh, sl, st, en, ok, max_live, tb, arrival, m0, t0);
+#pragma unroll 1
+    for (int s1 = 0; s1 < S; ++s1) {
+      sl[K] = s1;
+      int64_t m1 = m0, t1 = t0;
+      place_at<kB, TT>(K, sh, sl, st, en, ok, max_live, tb, arrival, m1, t1);
+      if constexpr (D == 1) {
+        const int64_t key = make_key(m1, t1, 0);
+        const uint32_t idx = p + (uint32_t)s1 * wK;
+        if (key_less(key, idx, best, bidx)) { best = key; bidx = idx; }
       } else {
-        const int64_t tb = ok[x] ? en[x] - (int64_t)__ldg(arrival + b.moff) : (int64_t)0xFFFFFFFFLL;
-        tail = tb > tail ? tb : tail;
+#pragma unroll 1
+        for (int s2 = 0; s2 < S; ++s2) {
+          sl[K + 1] = s2;
+          int64_t m2 = m1, t2 = t1;
+          place_at<kB, TT>(K + 1, sh, sl, st, en, ok, max_live, tb, arrival, m2, t2);
+          const int64_t key = make_key(m2, t2, 0);
+          const uint32_t idx = p + (uint32_t)s1 * wK + (uint32_t)s2 * wK1;
+          if (key_less(key, idx, best, bidx)) { best = key; bidx = idx; }
+        }
       }
-    }
-    const int64_t key = make_key(misses, tail, 0);
-    if (key < best) {  // idx ascending per thread: keep the first minimiser
-      best = key;
-      bidx = idx;
     }
   }
   *bk = best;
   *bi = bidx;
 }
 
-__global__ void __launch_bounds__(kSwThreads) sweep_kernel(SweepParams P) {
+template <int kB>
+__device__ __forceinline__ void sweep_unit_geom(const SwShared& sh, const uint32_t* arrival, int S, uint32_t first,
+                                                uint32_t step, int max_live, int64_t tb, bool narrow,
+                                                int64_t* bk, uint32_t* bi) {
+  constexpr int D = kB >= 4 ? 2 : 1;
+  if (narrow) sweep_range<kB, D, int32_t>(sh, arrival, S, first, step, max_live, tb, bk, bi);
+  else sweep_range<kB, D, int64_t>(sh, arrival, S, first, step, max_live, tb, bk, bi);
+}
+
+__global__ void __launch_bounds__(kSwThreads, PROTEAN_SWEEP_MINB) sweep_kernel(SweepParams P) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ SwShared sh;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -173,6 +228,8 @@ __global__ void __launch_bounds__(kSwThreads) sweep_kernel(SweepParams P) {
         b.strict = pb.strict ? 1 : 0;
         b.slo = T.slo[m];
         b.moff = pb.req_off;
+        b.a_first = P.arrival[pb.req_off];
+        b.a_last = P.arrival[pb.req_off + pb.n_req - 1];
         for (int i = 0; i < pb.n_req; ++i) {  // members sorted and not after ready
           const uint32_t a = P.arrival[pb.req_off + i];
           if (a > pb.ready_us || (i > 0 && a < P.arrival[pb.req_off + i - 1])) { bad = true; break; }
@@ -182,6 +239,24 @@ __global__ void __launch_bounds__(kSwThreads) sweep_kernel(SweepParams P) {
     if (__syncthreads_or(bad)) {
       if (tid == 0) atomicOr(&P.err[0], 1);
       continue;
+    }
+    if (tid == 0) {  // relative-time bound: ends <= last ready + sum of the largest execution times
+      int64_t tb = nb ? sh.b[0].ready : 0, fsum = 0, span = 0;
+      for (int x = 0; x < nb; ++x) {
+        const int m = P.batches[b0 + x].model;
+        int32_t fm = 0;
+        for (int q = 0; q < kNProf; ++q) fm = max(fm, T.fbr[m * kNProf + q]);
+        fsum += fm;
+      }
+      for (int x = 0; x < nb; ++x) {
+        const int m = P.batches[b0 + x].model;
+        int32_t sm = 0;
+        for (int q = 0; q < kNProf; ++q) sm = max(sm, T.solo[m * kNProf + q]);
+        span += exec_time(sm, fsum);
+      }
+      if (nb) span += sh.b[nb - 1].ready - tb;
+      sh.tb = tb;
+      sh.narrow = span < (int64_t)INT32_MAX;
     }
     int64_t kbest = INT64_MAX;
     unsigned long long n_assign = 0;
@@ -201,19 +276,19 @@ __global__ void __launch_bounds__(kSwThreads) sweep_kernel(SweepParams P) {
       __syncthreads();
       uint32_t total = 1;
       for (int x = 0; x < nb; ++x) total *= (uint32_t)S;
-      n_assign += total;
+      n_assign += total;  // (sh.tb / sh.narrow are published by the barrier above)
       int64_t k = INT64_MAX;
       uint32_t ix = 0;
       switch (nb) {
         case 0: if (tid == 0) { k = make_key(0, 0, 0); ix = 0; } break;
-        case 1: sweep_range<1>(sh, P.arrival, S, total, tid, blockDim.x, P.max_live, &k, &ix); break;
-        case 2: sweep_range<2>(sh, P.arrival, S, total, tid, blockDim.x, P.max_live, &k, &ix); break;
-        case 3: sweep_range<3>(sh, P.arrival, S, total, tid, blockDim.x, P.max_live, &k, &ix); break;
-        case 4: sweep_range<4>(sh, P.arrival, S, total, tid, blockDim.x, P.max_live, &k, &ix); break;
-        case 5: sweep_range<5>(sh, P.arrival, S, total, tid, blockDim.x, P.max_live, &k, &ix); break;
-        case 6: sweep_range<6>(sh, P.arrival, S, total, tid, blockDim.x, P.max_live, &k, &ix); break;
-        case 7: sweep_range<7>(sh, P.arrival, S, total, tid, blockDim.x, P.max_live, &k, &ix); break;
-        default: sweep_range<8>(sh, P.arrival, S, total, tid, blockDim.x, P.max_live, &k, &ix); break;
+        case 1: sweep_unit_geom<1>(sh, P.arrival, S, tid, blockDim.x, P.max_live, sh.tb, sh.narrow, &k, &ix); break;
+        case 2: sweep_unit_geom<2>(sh, P.arrival, S, tid, blockDim.x, P.max_live, sh.tb, sh.narrow, &k, &ix); break;
+        case 3: sweep_unit_geom<3>(sh, P.arrival, S, tid, blockDim.x, P.max_live, sh.tb, sh.narrow, &k, &ix); break;
+        case 4: sweep_unit_geom<4>(sh, P.arrival, S, tid, blockDim.x, P.max_live, sh.tb, sh.narrow, &k, &ix); break;
+        case 5: sweep_unit_geom<5>(sh, P.arrival, S, tid, blockDim.x, P.max_live, sh.tb, sh.narrow, &k, &ix); break;
+        case 6: sweep_unit_geom<6>(sh, P.arrival, S, tid, blockDim.x, P.max_live, sh.tb, sh.narrow, &k, &ix); break;
+        case 7: sweep_unit_geom<7>(sh, P.arrival, S, tid, blockDim.x, P.max_live, sh.tb, sh.narrow, &k, &ix); break;
+        default: sweep_unit_geom<8>(sh, P.arrival, S, tid, blockDim.x, P.max_live, sh.tb, sh.narrow, &k, &ix); break;
       }
       // min (key, idx) over the CTA: lowest index among equal keys (R20)
 #pragma unroll
