@@ -71,9 +71,12 @@ __device__ __forceinline__ bool key_less(int64_t k1, uint32_t i1, int64_t k2, ui
 // the unit's first ready time tb, in TT (int32_t when the unit's bound fits, else int64_t).  X is a
 // constant after unrolling, so the schedule arrays stay in registers.
 template <int kB, typename TT>
-__device__ __forceinline__ void place_at(const int X, const SwShared& sh, const int (&sl)[kB], TT (&st)[kB],
-                                         TT (&en)[kB], bool (&ok)[kB], int max_live, int64_t tb,
+__device__ __forceinline__ void place_at(const int X, const SwShared& sh, const int32_t (&qv)[kB], int (&sl)[kB],
+                                         TT (&st)[kB], TT (&en)[kB], int max_live, int64_t tb,
                                          const uint32_t* arrival, int64_t& misses, int64_t& tail) {
+  // sl[y] of an earlier batch is its slice if it was placed, else kOff (matches no slice), and
+  // en[y] = 0 if it was not placed (never > t >= 0): one compare per test instead of two.
+  constexpr int kOff = 15;
   const SwBatch& b = sh.b[X];
   const int s = sl[X];
   const TT t = (TT)(b.ready - tb);
@@ -82,19 +85,19 @@ __device__ __forceinline__ void place_at(const int X, const SwShared& sh, const 
 #pragma unroll
   for (int y = 0; y < kB; ++y) {
     if (y >= X) break;
-    live += (ok[y] && en[y] > t) ? 1 : 0;
-    if (ok[y] && sl[y] == s && st[y] > ls) ls = st[y];  // FIFO: the slice's last start
+    live += en[y] > t ? 1 : 0;
+    if (sl[y] == s && st[y] > ls) ls = st[y];  // FIFO: the slice's last start
   }
   const int32_t Ms = sh.cap[s];
-  ok[X] = live < max_live && b.q <= Ms;
+  const bool ok = live < max_live && qv[X] <= Ms;
   st[X] = en[X] = 0;
-  if (ok[X]) {
+  if (ok) {
     const TT t0 = t > ls ? t : ls;
-    int32_t used = b.q;  // only batches that fit a slice are held: sums stay far below 2^31
+    int32_t used = qv[X];  // only batches that fit a slice are held: sums stay far below 2^31
 #pragma unroll
     for (int y = 0; y < kB; ++y) {
       if (y >= X) break;
-      if (ok[y] && sl[y] == s && en[y] > t0) used += sh.b[y].q;
+      if (sl[y] == s && en[y] > t0) used += qv[y];
     }
     TT start = t0;
     if (used > Ms) {  // memory wait: the earliest release after which the batch fits
@@ -102,12 +105,12 @@ __device__ __forceinline__ void place_at(const int X, const SwShared& sh, const 
 #pragma unroll
       for (int y = 0; y < kB; ++y) {
         if (y >= X) break;
-        if (!(ok[y] && sl[y] == s && en[y] > t0)) continue;
-        int32_t rem = b.q;
+        if (!(sl[y] == s && en[y] > t0)) continue;
+        int32_t rem = qv[X];
 #pragma unroll
         for (int z = 0; z < kB; ++z) {
           if (z >= X) break;
-          if (ok[z] && sl[z] == s && en[z] > en[y]) rem += sh.b[z].q;
+          if (sl[z] == s && en[z] > en[y]) rem += qv[z];
         }
         if (rem <= Ms && en[y] < start) start = en[y];
       }
@@ -116,15 +119,17 @@ __device__ __forceinline__ void place_at(const int X, const SwShared& sh, const 
 #pragma unroll
     for (int y = 0; y < kB; ++y) {
       if (y >= X) break;
-      if (ok[y] && sl[y] == s && st[y] <= start && start < en[y]) F += sh.fx[y][s];
+      if (sl[y] == s && st[y] <= start && start < en[y]) F += sh.fx[y][s];
     }
     st[X] = start;
     en[X] = start + (TT)exec_time(sh.sx[X][s], F);
+  } else {
+    sl[X] = kOff;
   }
   if (b.strict) {
-    misses += ok[X] ? strict_misses(b, arrival + b.moff, b.n, tb + (int64_t)en[X], b.slo) : b.n;
+    misses += ok ? strict_misses(b, arrival + b.moff, b.n, tb + (int64_t)en[X], b.slo) : b.n;
   } else {
-    const int64_t tv = ok[X] ? tb + (int64_t)en[X] - b.a_first : (int64_t)0xFFFFFFFFLL;
+    const int64_t tv = ok ? tb + (int64_t)en[X] - b.a_first : (int64_t)0xFFFFFFFFLL;
     tail = tv > tail ? tv : tail;
   }
 }
@@ -142,11 +147,13 @@ __device__ __forceinline__ void sweep_range(const SwShared& sh, const uint32_t* 
   const uint32_t wK = npre, wK1 = npre * (uint32_t)S;  // index weights of batches K and K+1
   int64_t best = INT64_MAX;
   uint32_t bidx = 0;
+  int32_t qv[kB];  // footprints, loop-invariant
+#pragma unroll
+  for (int x = 0; x < kB; ++x) qv[x] = sh.b[x].q;
 #pragma unroll 1
   for (uint32_t p = first; p < npre; p += step) {
     int sl[kB];
     TT st[kB], en[kB];
-    bool ok[kB];
     int64_t m0 = 0, t0 = 0;
     {
       uint32_t rem = p;
@@ -158,12 +165,12 @@ __device__ __forceinline__ void sweep_range(const SwShared& sh, const uint32_t* 
       }
     }
 #pragma unroll
-    for (int x = 0; x < K; ++x) place_at<kB, TT>(x, sh, sl, st, en, ok, max_live, tb, arrival, m0, t0);
+    for (int x = 0; x < K; ++x) place_at<kB, TT>(x, sh, qv, sl, st, en, max_live, tb, arrival, m0, t0);
 #pragma unroll 1
     for (int s1 = 0; s1 < S; ++s1) {
       sl[K] = s1;
       int64_t m1 = m0, t1 = t0;
-      place_at<kB, TT>(K, sh, sl, st, en, ok, max_live, tb, arrival, m1, t1);
+      place_at<kB, TT>(K, sh, qv, sl, st, en, max_live, tb, arrival, m1, t1);
       if constexpr (D == 1) {
         const int64_t key = make_key(m1, t1, 0);
         const uint32_t idx = p + (uint32_t)s1 * wK;
@@ -173,7 +180,7 @@ __device__ __forceinline__ void sweep_range(const SwShared& sh, const uint32_t* 
         for (int s2 = 0; s2 < S; ++s2) {
           sl[K + 1] = s2;
           int64_t m2 = m1, t2 = t1;
-          place_at<kB, TT>(K + 1, sh, sl, st, en, ok, max_live, tb, arrival, m2, t2);
+          place_at<kB, TT>(K + 1, sh, qv, sl, st, en, max_live, tb, arrival, m2, t2);
           const int64_t key = make_key(m2, t2, 0);
           const uint32_t idx = p + (uint32_t)s1 * wK + (uint32_t)s2 * wK1;
           if (key_less(key, idx, best, bidx)) { best = key; bidx = idx; }
