@@ -201,6 +201,72 @@ class Handle:
         out = self.replay_traces(d[0], d[1], d[2], trace_len_us=trace.trace_len_us, stream=stream, **cfg)
         return {k: (v.cpu().numpy() if hasattr(v, "cpu") else v) for k, v in out.items()}
 
+    def replay_traces_pinned(self, arrival_h, meta_h, off_h, *, trace_len_us: int, chunks: int = 4,
+                             out_host=None, stream=None, copy_stream=None, **cfg):
+        """End-to-end replay from PINNED host tensors with the PCIe transfers overlapped: the
+        replicas are cut into `chunks` contiguous ranges; chunk k+1's trace is copied host->device
+        on a copy stream while chunk k replays, and each chunk's results are copied back as soon as
+        it finishes.  Replicas are independent and keep their global ids (replica_base + r), so the
+        outputs equal one call over all replicas.  arrival_h int32/uint32 [n], meta_h uint8 [n],
+        off_h int64 [R+1] (host, pinned).  Returns pinned host output tensors."""
+        torch = _torch()
+        dev = torch.device("cuda", self.device)
+        c = dict(_REPLAY_DEFAULTS)
+        c.update(cfg)
+        R = int(off_h.shape[0]) - 1
+        N = int(c["n_gpus"])
+        E = self.num_epochs(trace_len_us, c["epoch_len_us"])
+        base = int(c.pop("replica_base", 0))
+        st = stream if stream is not None else torch.cuda.current_stream(self.device)
+        cs = copy_stream if copy_stream is not None else torch.cuda.Stream(self.device)
+        offs = off_h.numpy()
+        chunks = max(1, min(int(chunks), R))  # every chunk holds at least one replica
+        bounds = [round(k * R / chunks) for k in range(chunks + 1)]
+        cap = max(int(offs[bounds[k + 1]] - offs[bounds[k]]) for k in range(chunks))
+        rcap = max(bounds[k + 1] - bounds[k] for k in range(chunks))
+        bufs = [(torch.empty(max(cap, 1), dtype=torch.int32, device=dev),
+                 torch.empty(max(cap, 1), dtype=torch.uint8, device=dev),
+                 torch.empty(rcap + 1, dtype=torch.int64, device=dev)) for _ in range(2)]
+        off_rel = [torch.from_numpy(offs[bounds[k]:bounds[k + 1] + 1] - offs[bounds[k]]).pin_memory()
+                   for k in range(chunks)]
+        dout = self.alloc_replay_out(R, E, N, decisions=True)
+        if out_host is None:
+            out_host = {k: torch.empty(v.shape, dtype=v.dtype).pin_memory() for k, v in dout.items()
+                        if hasattr(v, "shape")}
+        ready = [torch.cuda.Event() for _ in range(chunks)]
+        freed = [torch.cuda.Event() for _ in range(chunks)]
+
+        def h2d(k):
+            b = bufs[k % 2]
+            if k >= 2:
+                cs.wait_event(freed[k - 2])  # the replay that used this buffer has finished
+            lo, hi = int(offs[bounds[k]]), int(offs[bounds[k + 1]])
+            with torch.cuda.stream(cs):
+                b[0][: hi - lo].copy_(arrival_h[lo:hi], non_blocking=True)
+                b[1][: hi - lo].copy_(meta_h[lo:hi], non_blocking=True)
+                b[2][: bounds[k + 1] - bounds[k] + 1].copy_(off_rel[k], non_blocking=True)
+            ready[k].record(cs)
+
+        h2d(0)
+        for k in range(chunks):
+            if k + 1 < chunks:
+                h2d(k + 1)  # overlaps chunk k's replay
+            st.wait_event(ready[k])
+            r0, r1 = bounds[k], bounds[k + 1]
+            b = bufs[k % 2]
+            n = int(offs[r1] - offs[r0])
+            view = {kk: v[r0:r1] for kk, v in dout.items() if hasattr(v, "shape")}
+            view["log_cap"] = 0
+            self.replay_traces(b[0][:max(n, 1)], b[1][:max(n, 1)], b[2][: r1 - r0 + 1], trace_len_us=trace_len_us,
+                               out=view, stream=st, replica_base=base + r0, **c)
+            freed[k].record(st)
+            with torch.cuda.stream(st):
+                for kk, v in view.items():
+                    if hasattr(v, "shape"):
+                        out_host[kk][r0:r1].copy_(v, non_blocking=True)
+        st.synchronize()
+        return out_host
+
     # -------------------------------------------------------------------------------- score_epoch
     def score_epoch(self, *, n_replicas, n_gpus, epoch, batches, batch_off, arrival_us, state,
                     geom_lo=0, geom_hi=None, epoch_len_us=1_000_000, horizon_us=1 << 62, max_live=64,
