@@ -117,3 +117,22 @@ def test_sweep_error_codes_match_oracle(oracle):
         assert gc == oc, (kw, gc, oc)
     gc, oc = codes(base, [0, 3], cur=(12,))
     assert gc == oc == -1
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_wide_times_64bit_path(oracle, seed):
+    """Solo times of minutes: a GPU-epoch's completion bound exceeds 2^31 us, so the sweep runs its
+    64-bit instance (the 32-bit one needs relative times below 2^31); heavy footprints exercise the
+    memory-wait branch.  Both instances meet in one call (units with and without wide models)."""
+    rng = np.random.default_rng(1700 + seed)
+    M = 3
+    solo7 = np.array([150_000_000, 300_000_000, 2_000])  # two very long models (x6 on 1g < 2^31), one short
+    prof = tables(np.stack([solo7 * f for f in (6, 4, 3, 2, 1)], 1), rng.integers(200_000, 1_000_000, (M, 5)),
+                  rng.integers(2_000, 18_000, M), bsz=[2, 3, 1], slo=3 * solo7, tmo=[0, 0, 0])
+    R, N = 2, 4
+    batches, off, arr, cur = epoch_batches(3000 + seed, R, N, models=range(M), mean_batches=3.0, max_batches=5,
+                                           batch_size=3, ragged=True)
+    g = _gpu_sweep(prof, R, N, batches, off, arr, cur, max_batches=5)
+    o = oracle.sweep(prof, R=R, N=N, batches=batches, batch_off=off, arrival=arr, cur_geom=cur, max_batches=5)
+    _compare(g, o, 12)
+    assert (o["sweep_key"] & 0xFFFFFFFFFF00 != 0).any()  # some BE tails are long
