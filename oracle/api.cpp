@@ -252,6 +252,8 @@ int orc_replay(const orc_tables* t, const orc_replay_in* in, orc_replay_out* out
   for (int m = 0; m < tb.M; ++m) maxT = std::max<int64_t>(maxT, tb.tmo[m]);
   if (in->trace_len - 1 + maxT > (int64_t)0xFFFFFFFFLL) return ORC_ERANGE;
   if (in->policy < 0 || in->policy > 2) return ORC_EINVAL;
+  if (in->cold_us < 0 || in->keepalive_epochs < 1 || in->prewarm < 0 || in->prewarm > kPoolCap)
+    return ORC_EINVAL;
   if (in->policy == 2) {  // Alg 2 heuristic (N1): its knobs, and both of its geometries in the set
     if (in->ewma_alpha_pm < 1 || in->ewma_alpha_pm > 1000) return ORC_EINVAL;
     if (in->t_low < 0 || in->t_high < in->t_low) return ORC_EINVAL;
@@ -305,6 +307,9 @@ int orc_replay(const orc_tables* t, const orc_replay_in* in, orc_replay_out* out
   cfg.rev_interval = in->rev_interval;
   cfg.notice = in->notice;
   cfg.seed = in->seed;
+  cfg.cold_us = in->cold_us;
+  cfg.keepalive_epochs = in->keepalive_epochs;
+  cfg.prewarm = in->prewarm;
   cfg.ewma_alpha_pm = in->ewma_alpha_pm;
   cfg.t_low = in->t_low;
   cfg.t_high = in->t_high;
@@ -313,6 +318,7 @@ int orc_replay(const orc_tables* t, const orc_replay_in* in, orc_replay_out* out
   const int N = in->N;
 
   std::atomic<int> next(0);
+  std::atomic<bool> overflow(false);
   auto worker = [&]() {
     for (;;) {
       int r = next.fetch_add(1);
@@ -335,6 +341,8 @@ int orc_replay(const orc_tables* t, const orc_replay_in* in, orc_replay_out* out
       if (out->cand_keys)
         std::copy(ro.cand_keys.begin(), ro.cand_keys.end(), out->cand_keys + (int64_t)r * E * N * G);
       if (out->n_batches) out->n_batches[r] = ro.n_batches;
+      if (out->cold_starts) out->cold_starts[r] = ro.cold_starts;
+      if (ro.pool_overflow) overflow = true;
       if (out->log) {
         for (size_t i = 0; i < ro.log.size() && (int64_t)i < out->log_cap; ++i) {
           const BatchRec& b = ro.log[i];
@@ -358,6 +366,7 @@ int orc_replay(const orc_tables* t, const orc_replay_in* in, orc_replay_out* out
   for (int i = 1; i < nt; ++i) th.emplace_back(worker);
   worker();
   for (auto& x : th) x.join();
+  if (overflow) return ORC_ERANGE;  // a container pool outgrew kPoolCap (N3, R22)
   return ORC_OK;
 }
 

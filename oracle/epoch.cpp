@@ -6,6 +6,8 @@
 // "Oracle" scheme P:L485) -> Alg 2 hysteresis + ~30% cap (O9, O10).
 // policy 2 (N1) replaces the scoring by Alg 2's own heuristic (lines 1-23, readings
 // R10-R17 of DESIGN.md): EWMA of the observed BE load -> small-slice set -> thresholds -> geometry.
+// N3 (cold_us > 0): the Autoscaler's container pools (readings R22-R27): one container
+// per batch, reactive scale-up with a cold start t_cold, delayed termination of surplus containers.
 #include "pem.hpp"
 #include <algorithm>
 #include <climits>
@@ -37,6 +39,8 @@ struct Gpu {
   Node node;
   int64_t pred_num = 0;     // Alg 2 history_info (N1): EWMA of BE batches, milli-batches
   int64_t pred_mem = 0;     //   and of their total footprint, milli-MiB (R11)
+  std::vector<std::vector<int64_t>> pool;  // N3: per model, busy-until of every container (R22)
+  std::vector<int> surplus_ctr;            // N3: consecutive epochs with surplus containers (R26)
 };
 
 struct Replay {
@@ -97,6 +101,7 @@ struct Replay {
           bill_switch(nd, VM_NONE, tau + cfg.notice);
           g.target = -1;
           g.rs = g.re = 0;
+          reset_pool(g);  // the node's containers go with it (R27)
         }
       } else if (nd.vm == VM_NONE) {
         if (spot_ok) {  // a new spot VM: initial geometry, idle, wait_ctr 0
@@ -110,9 +115,31 @@ struct Replay {
           g.target = -1;
           g.ctr = 0;
           g.rs = g.re = 0;
+          reset_pool(g);  // a new VM starts with the prewarmed pool only (R27)
         }
       }
     }
+  }
+
+  void reset_pool(Gpu& g) {  // R22: prewarm idle containers per model (busy-until 0)
+    g.pool.assign(tb.M, std::vector<int64_t>(cfg.prewarm, 0));
+    g.surplus_ctr.assign(tb.M, 0);
+  }
+
+  // R23: the container a batch of model m dispatched at t runs in: the first idle one (busy-until
+  // <= t), else a new one after a cold start.  Returns its index; *t_eff = t (+ cold_us if spawned).
+  size_t acquire(Gpu& g, int m, int64_t t, int64_t* t_eff) {
+    std::vector<int64_t>& P = g.pool[m];
+    for (size_t i = 0; i < P.size(); ++i)
+      if (P[i] <= t) {
+        *t_eff = t;
+        return i;
+      }
+    if ((int)P.size() >= kPoolCap) out->pool_overflow = true;  // R22 capacity (ERANGE)
+    P.push_back(t);  // reactive scale-up: one container per batch
+    out->cold_starts += 1;
+    *t_eff = t + cfg.cold_us;  // t = t_cold + t_queue + t_exec
+    return P.size() - 1;
   }
 
   void account(const Batch& b, const PlaceOut* po, int drop_kind) {
@@ -141,6 +168,7 @@ struct Replay {
       gpu[n].S.geom = cfg.init_geom;  // (4g,2g,1g) by default
       Node& nd = gpu[n].node;
       nd.vm = nd.bill = (cfg.vm_policy == 0) ? VM_OD : VM_SPOT;
+      reset_pool(gpu[n]);
     }
     out->hist.assign(2 * kBuckets, 0);
     out->decisions.assign((size_t)E * N, 0xFF);
@@ -193,8 +221,12 @@ struct Replay {
         Gpu& g = gpu[n];
         for (size_t x : list[n]) {
           const Batch& b = batches[x];
-          PlaceOut po = place(tb, tb.geoms[g.S.geom], g.S, b.ready, b.model, b.strict,
+          int64_t t_eff = b.ready;
+          size_t ci = 0;
+          if (cfg.cold_us > 0) ci = acquire(g, b.model, b.ready, &t_eff);  // N3 (R23)
+          PlaceOut po = place(tb, tb.geoms[g.S.geom], g.S, t_eff, b.model, b.strict,
                               cfg.max_live, &acc, H);
+          if (cfg.cold_us > 0) g.pool[b.model][ci] = po.dropped ? t_eff : po.end;  // R24
           account(b, &po, po.dropped);
           BatchRec& r = erec[x - first_bi];
           r.gpu = n;
@@ -207,6 +239,34 @@ struct Replay {
         }
       }
       if (want_log) out->log.insert(out->log.end(), erec.begin(), erec.end());
+
+      // N3 delayed termination (R26): n_c = batches of model m dispatched to the GPU in this
+      // epoch; a pool larger than n_c for keepalive_epochs consecutive epochs loses its
+      // surplus containers that are idle at T
+      if (cfg.cold_us > 0) {
+        for (int n = 0; n < N; ++n) {
+          Gpu& g = gpu[n];
+          std::vector<int64_t> need(tb.M, 0);
+          for (size_t x : list[n]) need[batches[x].model] += 1;
+          for (int m = 0; m < tb.M; ++m) {
+            std::vector<int64_t>& P = g.pool[m];
+            const int64_t surplus = (int64_t)P.size() - need[m];
+            if (surplus <= 0) {
+              g.surplus_ctr[m] = 0;
+              continue;
+            }
+            if (++g.surplus_ctr[m] < cfg.keepalive_epochs) continue;
+            int64_t drop = surplus;
+            std::vector<int64_t> kept;
+            for (int64_t bu : P) {
+              if (drop > 0 && bu <= T) { --drop; continue; }  // terminate an idle container
+              kept.push_back(bu);
+            }
+            P = kept;
+            g.surplus_ctr[m] = 0;
+          }
+        }
+      }
 
       // 4. candidate scoring for every decidable GPU (has a VM at T, no open window)
       std::vector<int> wants;
@@ -341,6 +401,7 @@ struct Replay {
       }
     }
 
+    // (delayed termination runs inside the epoch loop, see terminate_surplus)
     // close billing at H and finalize (O12)
     for (int n = 0; n < N; ++n) bill_switch(gpu[n].node, VM_NONE, H);
     out->accum[0] = acc.busy_w;

@@ -74,6 +74,9 @@ typedef struct {
   int32_t shard_mode, nthreads;
   int32_t ewma_alpha_pm, pad;   /* policy 2 (N1): EWMA weight per mille, 1..1000 */
   int64_t t_low, t_high;        /* policy 2: T_low <= T_high, milli-BE-batches per epoch */
+  int64_t cold_us;              /* N3: container cold start (0 = warm containers, Q15) */
+  int32_t keepalive_epochs;     /* N3: delayed termination after this many surplus epochs, >= 1 */
+  int32_t prewarm;              /* N3: idle containers per (sim-GPU, model) at t = 0, 0..128 */
 } orc_replay_in;
 
 typedef struct {
@@ -92,6 +95,7 @@ typedef struct {
   orc_batch_rec *log;  /* [R][log_cap] or NULL */
   int64_t log_cap;
   int64_t *n_batches;  /* [R] or NULL */
+  int64_t *cold_starts; /* [R] or NULL (N3) */
 } orc_replay_out;
 
 int orc_replay(const orc_tables *t, const orc_replay_in *in, orc_replay_out *out);

@@ -52,7 +52,8 @@ class ReplayIn(C.Structure):
                 ("rev_interval", C.c_int64), ("notice", C.c_int64), ("seed", C.c_uint64),
                 ("shard_mode", C.c_int32), ("nthreads", C.c_int32),
                 ("ewma_alpha_pm", C.c_int32), ("pad", C.c_int32), ("t_low", C.c_int64),
-                ("t_high", C.c_int64)]
+                ("t_high", C.c_int64), ("cold_us", C.c_int64), ("keepalive_epochs", C.c_int32),
+                ("prewarm", C.c_int32)]
 
 
 class BatchRec(C.Structure):
@@ -65,7 +66,7 @@ class ReplayOut(C.Structure):
     _fields_ = [("counters", C.c_void_p), ("accum", C.c_void_p), ("hist", C.c_void_p),
                 ("p50_p99", C.c_void_p), ("cost", C.c_void_p), ("util", C.c_void_p),
                 ("decisions", C.c_void_p), ("cand_keys", C.c_void_p), ("log", C.c_void_p),
-                ("log_cap", C.c_int64), ("n_batches", C.c_void_p)]
+                ("log_cap", C.c_int64), ("n_batches", C.c_void_p), ("cold_starts", C.c_void_p)]
 
 
 BATCH_REC_DTYPE = np.dtype([("ready", "<u4"), ("epoch", "<u4"), ("n", "<i4"), ("model", "<i4"),
@@ -259,7 +260,8 @@ def tick_simulate(prof, geom, t, model, slice_):
 DEFAULT_CFG = dict(N=8, W=1_000_000, policy=0, wait_limit=3, cap_pct=30, init_geom=2, max_live=64,
                    vm_policy=0, reconfig_us=2_000_000, p_rev=0.0, price_od=32.7726 / 8,
                    price_spot=9.8318 / 8, rev_interval=300_000_000, notice=30_000_000, seed=0,
-                   shard_mode=0, ewma_alpha_pm=500, t_low=500, t_high=4000)
+                   shard_mode=0, ewma_alpha_pm=500, t_low=500, t_high=4000, cold_us=0, keepalive_epochs=600,
+                   prewarm=0)
 
 
 def replay(prof, trace, *, nthreads=1, want_keys=False, want_log=False, log_cap=None, **cfg):
@@ -275,7 +277,8 @@ def replay(prof, trace, *, nthreads=1, want_keys=False, want_log=False, log_cap=
                    _p(meta) or 0, _p(off), c["policy"], c["wait_limit"], c["cap_pct"], c["init_geom"],
                    c["max_live"], c["vm_policy"], c["reconfig_us"], c["p_rev"], c["price_od"],
                    c["price_spot"], c["rev_interval"], c["notice"], c["seed"], c["shard_mode"], nthreads,
-                   c["ewma_alpha_pm"], 0, c["t_low"], c["t_high"])
+                   c["ewma_alpha_pm"], 0, c["t_low"], c["t_high"], c["cold_us"], c["keepalive_epochs"],
+                   c["prewarm"])
     if arr.shape[0] == 0:  # keep pointers non-NULL for empty traces
         arr = np.zeros(1, np.uint32)
         meta = np.zeros(1, np.uint8)
@@ -285,7 +288,8 @@ def replay(prof, trace, *, nthreads=1, want_keys=False, want_log=False, log_cap=
     out = dict(counters=np.zeros((R, 10), np.int64), accum=np.zeros((R, 4), np.int64),
                hist=np.zeros((R, 2, NB), np.uint32), p50_p99=np.zeros((R, 2, 2), np.int64),
                cost=np.zeros(R, np.float64), util=np.zeros((R, 2), np.float64),
-               decisions=np.zeros((R, E, N), np.uint8), n_batches=np.zeros(R, np.int64))
+               decisions=np.zeros((R, E, N), np.uint8), n_batches=np.zeros(R, np.int64),
+               cold_starts=np.zeros(R, np.int64))
     if want_keys:
         out["cand_keys"] = np.zeros((R, E, N, G), np.int64)
     if want_log:
@@ -294,7 +298,7 @@ def replay(prof, trace, *, nthreads=1, want_keys=False, want_log=False, log_cap=
         out["log"] = np.zeros((R, log_cap), BATCH_REC_DTYPE)
     ro = ReplayOut(_p(out["counters"]), _p(out["accum"]), _p(out["hist"]), _p(out["p50_p99"]),
                    _p(out["cost"]), _p(out["util"]), _p(out["decisions"]), _p(out.get("cand_keys")),
-                   _p(out.get("log")), int(log_cap or 0), _p(out["n_batches"]))
+                   _p(out.get("log")), int(log_cap or 0), _p(out["n_batches"]), _p(out["cold_starts"]))
     rc = lib().orc_replay(T.ref, C.byref(rin), C.byref(ro))
     if rc:
         raise OracleError(rc)

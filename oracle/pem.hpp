@@ -26,6 +26,7 @@ constexpr int kMaxSlices = 7;
 constexpr int64_t kPpm = 1000000;               // FBR 1.0 ("0.2 -> 20%")
 constexpr int kBuckets = 3328;
 constexpr uint64_t kSat32 = 0xFFFFFFFFull;
+constexpr int kPoolCap = 128;                   // N3: containers per (sim-GPU, model) (R22)
 
 enum Err { OK = 0, EINVAL_ = -1, ERANGE_ = -2, ENOMEM_ = -3, EUNSUP_ = -7 };
 
@@ -115,6 +116,9 @@ struct ReplayCfg {
   uint64_t seed = 0;
   int ewma_alpha_pm = 500;                 // policy 2 (N1): EWMA weight of the newest epoch, per mille
   int64_t t_low = 500, t_high = 4000;      //   T_low / T_high, milli-BE-batches per epoch (R14)
+  int64_t cold_us = 0;                     // N3: container cold start t_cold (0 = warm, reading Q15)
+  int keepalive_epochs = 600;              //   delayed termination (~10 min of surplus)
+  int prewarm = 0;                         //   idle containers per (sim-GPU, model) at t = 0
 };
 struct BatchRec {
   uint32_t ready; uint32_t epoch; int n, model; bool strict;
@@ -122,6 +126,8 @@ struct BatchRec {
 };
 struct ReplayOut {
   int64_t counters[10] = {0};
+  int64_t cold_starts = 0;              // N3: containers spawned for a batch (cold starts)
+  bool pool_overflow = false;           // N3: a pool outgrew kPoolCap containers (ERANGE)
   int64_t accum[4] = {0};
   std::vector<uint32_t> hist;           // [2][3328]
   int64_t p[2][2] = {{0, 0}, {0, 0}};
