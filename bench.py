@@ -133,11 +133,11 @@ def oracle_sample(n_rep: int, seconds: int, seed: int = 1, base: int = 0):
     return tr
 
 
-def time_oracle(prof, tr, cores: int, policy: int = 0):
+def time_oracle(prof, tr, cores: int, policy: int = 0, cold_us: int = 0, keepalive: int = 600):
     from oracle import oracle as O
     O.build()
     t0 = time.perf_counter()
-    out = O.replay(prof, tr, N=8, nthreads=cores, policy=policy)
+    out = O.replay(prof, tr, N=8, nthreads=cores, policy=policy, cold_us=cold_us, keepalive_epochs=keepalive)
     dt = time.perf_counter() - t0
     c = out["counters"]
     return dt, int(c[:, 8].sum()), int((c[:, 0] + c[:, 4]).sum()), int(c[:, 9].sum())
@@ -153,10 +153,10 @@ def run_reference(args):
     tr = oracle_sample(n_rep, args.seconds)
     pol = POLICIES[args.policy]
     for _ in range(args.warmup):
-        time_oracle(prof, tr, cores, pol)
+        time_oracle(prof, tr, cores, pol, args.cold_start_us, args.keepalive_epochs)
     dts, slots, reqs = [], 0, 0
     for _ in range(args.steps):
-        dt, s, q, _g = time_oracle(prof, tr, cores, pol)
+        dt, s, q, _g = time_oracle(prof, tr, cores, pol, args.cold_start_us, args.keepalive_epochs)
         dts.append(dt)
         slots, reqs = s, q
     tot = sum(dts)
@@ -202,7 +202,8 @@ def run_ours(args):
     stream = torch.cuda.current_stream(dev)
     pol = POLICIES[args.policy]
     metric, unit = metric_of(args.policy)
-    cfg = dict(n_gpus=N, replica_base=rank * R, policy=pol)
+    cfg = dict(n_gpus=N, replica_base=rank * R, policy=pol, cold_start_us=args.cold_start_us,
+               keepalive_epochs=args.keepalive_epochs)
 
     def step():
         h.replay_traces(arr, meta, roff, trace_len_us=gp.trace_len_us, out=out, stream=stream, **cfg)
@@ -278,7 +279,7 @@ def run_ours(args):
         tr = oracle_sample(n_rep, S, base=0)
         dt, s_cpu, q_cpu, passes = 0.0, 0, 0, 0
         while passes < 1 or (dt < 10.0 and passes < 40):  # ~10 s of oracle work on the host cores
-            d, s1, q1, _ = time_oracle(prof, tr, cores, pol)
+            d, s1, q1, _ = time_oracle(prof, tr, cores, pol, args.cold_start_us, args.keepalive_epochs)
             dt, s_cpu, q_cpu, passes = dt + d, s_cpu + s1, q_cpu + q1, passes + 1
         cpu = {"value": (s_cpu if pol == 0 else q_cpu) / dt, "unit": unit, "cores": cores, "kind": "oracle",
                "sample": f"{n_rep} replicas x {S} s of this workload (numpy-generated), replayed "
@@ -308,11 +309,14 @@ def run_ours(args):
             "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
             "config": {"workload": "C5 (configs[4]): Mix A Wiki-shaped 5000 rps, 22-model table, "
-                                   f"8 sim-GPUs, 600 s, 12 geometries, {args.policy} policy, on-demand VMs",
+                                   f"8 sim-GPUs, 600 s, 12 geometries, {args.policy} policy, on-demand VMs"
+                                   + (f", N3 cold starts {args.cold_start_us} us / keep-alive "
+                                      f"{args.keepalive_epochs} epochs" if args.cold_start_us else ""),
                        "replicas_per_rank": R, "seconds": S, "sim_gpus": N, "geometries": h.n_geoms,
                        "requests_per_rank": n_req, "l2_flush": "inputs (5 B/request, "
                        f"{5.0 * n_req / 1e9:.1f} GB per rank) exceed the 126 MB L2"},
             "simulated_requests_per_s": reqs * args.steps / sec,
+            "cold_starts_per_step": int(out["cold_starts"].sum().item()) * world if args.cold_start_us else None,
             "geom_candidates_per_s": geom_c * args.steps / sec,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
@@ -483,6 +487,9 @@ def main():
     ap.add_argument("--cpu-sample", type=int, default=64, help="replicas timed on the CPU oracle")
     ap.add_argument("--path", default="replay", choices=["replay", "sweep"],
                     help="replay = protean_replay_traces (headline); sweep = protean_sweep_assignments (N4a)")
+    ap.add_argument("--cold-start-us", type=int, default=0,
+                    help="N3 container cold start (0 = warm containers, the paper's headline setting)")
+    ap.add_argument("--keepalive-epochs", type=int, default=600, help="N3 delayed termination (epochs)")
     ap.add_argument("--policy", default="search", choices=sorted(POLICIES),
                     help="search = the geometry search (headline); alg2 = Alg 2's own heuristic (N1)")
     args = ap.parse_args()

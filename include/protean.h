@@ -217,6 +217,14 @@ typedef struct {
                                   (default 500; R11) */
   int64_t t_low_milli;         /* policy 2: T_low, thousandths of a BE batch per epoch (default 500) */
   int64_t t_high_milli;        /* policy 2: T_high >= T_low (default 4000; R14) */
+  int64_t cold_start_us;       /* N3 Autoscaler (R22-R27): container
+                                  cold start; 0 (default) = warm containers (reading Q15), no pools.
+                                  > 0: per (sim-GPU, model) pools of <= 128 containers, one per
+                                  batch; a batch finding none idle waits cold_start_us (PROTEAN_ERANGE
+                                  if a pool would exceed 128) */
+  int32_t keepalive_epochs;    /* N3: surplus containers terminated after this many consecutive
+                                  surplus epochs, >= 1 (default 600 = ~10 min at W = 1 s) */
+  int32_t prewarm;             /* N3: idle containers per (sim-GPU, model) at t = 0, 0..128 */
 } protean_replay_cfg;
 
 /* counters[10] per replica (O7/O8/O10):
@@ -248,6 +256,7 @@ typedef struct {             /* caller-allocated, one row per replica of this ca
   protean_batch_rec *batch_log; /* [R][batch_log_cap] or NULL */
   int64_t batch_log_cap;
   int64_t *n_batches;        /* [R] batches formed (also when batch_log is NULL), or NULL */
+  int64_t *cold_starts;      /* [R] N3 cold starts (containers spawned), or NULL */
 } protean_replay_out;
 
 int protean_replay_traces(protean_handle *h, const protean_replay_cfg *cfg,

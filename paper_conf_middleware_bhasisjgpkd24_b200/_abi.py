@@ -75,7 +75,8 @@ class ReplayCfg(C.Structure):
                 ("rev_interval_us", C.c_int64), ("notice_us", C.c_int64), ("seed", C.c_uint64),
                 ("shard_mode", C.c_int32), ("rank", C.c_int32), ("nranks", C.c_int32),
                 ("max_ctas", C.c_int32), ("ewma_alpha_pm", C.c_int32), ("t_low_milli", C.c_int64),
-                ("t_high_milli", C.c_int64)]
+                ("t_high_milli", C.c_int64), ("cold_start_us", C.c_int64), ("keepalive_epochs", C.c_int32),
+                ("prewarm", C.c_int32)]
 
 
 class SweepIn(C.Structure):      # protean_sweep_in
@@ -100,7 +101,7 @@ class ReplayOut(C.Structure):
     _fields_ = [("counters", C.c_void_p), ("accum", C.c_void_p), ("hist", C.c_void_p),
                 ("p50_p99_us", C.c_void_p), ("cost_usd", C.c_void_p), ("util", C.c_void_p),
                 ("decisions", C.c_void_p), ("cand_keys", C.c_void_p), ("batch_log", C.c_void_p),
-                ("batch_log_cap", C.c_int64), ("n_batches", C.c_void_p)]
+                ("batch_log_cap", C.c_int64), ("n_batches", C.c_void_p), ("cold_starts", C.c_void_p)]
 
 
 assert C.sizeof(Batch) == 16 and C.sizeof(Resident) == 24 and C.sizeof(Placement) == 24

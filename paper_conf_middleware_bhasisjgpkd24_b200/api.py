@@ -15,7 +15,7 @@ _REPLAY_DEFAULTS = dict(n_gpus=8, epoch_len_us=1_000_000, policy=0, wait_limit=3
                         price_od_node_hr=32.7726 / 8, price_spot_node_hr=9.8318 / 8,
                         rev_interval_us=300_000_000, notice_us=30_000_000, seed=0, shard_mode=0,
                         rank=0, nranks=1, max_ctas=0, replica_base=0, ewma_alpha_pm=500, t_low_milli=500,
-                        t_high_milli=4000)
+                        t_high_milli=4000, cold_start_us=0, keepalive_epochs=600, prewarm=0)
 
 
 def _torch():
@@ -135,7 +135,8 @@ class Handle:
                    p50_p99=torch.zeros((R, 2, 2), dtype=torch.int64, device=dev),
                    cost=torch.zeros(R, dtype=torch.float64, device=dev),
                    util=torch.zeros((R, 2), dtype=torch.float64, device=dev),
-                   n_batches=torch.zeros(R, dtype=torch.int64, device=dev))
+                   n_batches=torch.zeros(R, dtype=torch.int64, device=dev),
+                   cold_starts=torch.zeros(R, dtype=torch.int64, device=dev))
         if decisions:
             out["decisions"] = torch.zeros((R, E, N), dtype=torch.uint8, device=dev)
         if cand_keys:
@@ -171,7 +172,8 @@ class Handle:
         cf.replica_off = replica_off.data_ptr()
         for k in ("policy", "wait_limit", "reconfig_cap_pct", "init_geom", "max_live", "vm_policy",
                   "reconfig_us", "rev_interval_us", "notice_us", "seed", "shard_mode", "rank", "nranks",
-                  "max_ctas", "ewma_alpha_pm", "t_low_milli", "t_high_milli"):
+                  "max_ctas", "ewma_alpha_pm", "t_low_milli", "t_high_milli", "cold_start_us",
+                  "keepalive_epochs", "prewarm"):
             setattr(cf, k, int(c[k]))
         for k in ("p_rev", "price_od_node_hr", "price_spot_node_hr"):
             setattr(cf, k, float(c[k]))
@@ -180,7 +182,8 @@ class Handle:
                         out["decisions"].data_ptr() if "decisions" in out else None,
                         out["cand_keys"].data_ptr() if "cand_keys" in out else None,
                         out["log"].data_ptr() if "log" in out else None, out.get("log_cap", 0),
-                        out["n_batches"].data_ptr())
+                        out["n_batches"].data_ptr(),
+                        out["cold_starts"].data_ptr() if "cold_starts" in out else None)
         st = stream if stream is not None else torch.cuda.current_stream(self.device)
         _check(self._h, self._lib.protean_replay_traces(self._h, C.byref(cf), C.byref(o),
                                                         C.c_void_p(st.cuda_stream)))

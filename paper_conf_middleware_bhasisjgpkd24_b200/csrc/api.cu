@@ -343,6 +343,9 @@ void protean_replay_cfg_defaults(protean_replay_cfg* c) {
   c->ewma_alpha_pm = 500;
   c->t_low_milli = 500;
   c->t_high_milli = 4000;
+  c->cold_start_us = 0;
+  c->keepalive_epochs = 600;
+  c->prewarm = 0;
 }
 
 int protean_load_profiles(const protean_profiles* p, protean_handle** out) {
@@ -561,6 +564,8 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
     if (g421 < 0 || g43 < 0) return fail(h, PROTEAN_EINVAL, "policy 2 needs (4g,2g,1g) and (4g,3g) in the set");
   }
   if (c.shard_mode != 0 && c.shard_mode != 1) return fail(h, PROTEAN_EINVAL, "shard_mode");
+  if (c.cold_start_us < 0 || c.keepalive_epochs < 1 || c.prewarm < 0 || c.prewarm > kPoolCap)
+    return fail(h, PROTEAN_EINVAL, "cold_start_us / keepalive_epochs / prewarm");
   if (c.max_ctas < 0) return fail(h, PROTEAN_EINVAL, "max_ctas");
   const bool modeG = c.shard_mode == 1;
   if (modeG) {
@@ -718,6 +723,10 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   P.E = E;
   P.H = H;
   P.policy = c.policy;
+  P.cold_us = c.cold_start_us;
+  P.keepalive = c.keepalive_epochs;
+  P.prewarm = c.prewarm;
+  P.cold_starts = out->cold_starts;
   P.ewma_a = c.ewma_alpha_pm;
   P.t_low = c.t_low_milli;
   P.t_high = c.t_high_milli;
@@ -766,6 +775,8 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   P.o_gord = o; o += al((size_t)WCAP * 4);
   P.o_gglist = o; o += al((size_t)WCAP * 4);
   P.o_gsarr = o; o += al((size_t)(WS > 0 ? 0 : WCAP) * 4);
+  P.o_pool = o;  // N3 pools: busy-until [N][M][kPoolCap] int64, size + counter [N][M] int32
+  if (c.cold_start_us > 0) o += al((size_t)N * h->M * (kPoolCap * 8 + 8));
   P.slot_bytes = al(o);
   {
     int rc = ensure(h, &h->d_scratch, &h->scratch_bytes, P.slot_bytes * (size_t)grid, st);
@@ -776,8 +787,8 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   CK(h, cudaEventRecord(h->ev[2], st));
   CK(h, launch_replay(P, grid, block, st));
   CK(h, cudaEventRecord(h->ev[3], st));
-  int herr2[2] = {0, 0};
-  CK(h, cudaMemcpyAsync(herr2, d_err, 8, cudaMemcpyDeviceToHost, st));
+  int herr2[3] = {0, 0, 0};
+  CK(h, cudaMemcpyAsync(herr2, d_err, 12, cudaMemcpyDeviceToHost, st));
   CK(h, cudaStreamSynchronize(st));
   herr = herr2[0];
   if (modeG) h->xseq += (uint32_t)E;
@@ -797,6 +808,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   h->last_smem = (int)sl.total;
   h->last_per_sm = per_sm;
   if (herr) return fail(h, PROTEAN_EINVAL, "invalid request (unsorted, model id, or arrival >= trace_len)");
+  if (herr2[2]) return fail(h, PROTEAN_ERANGE, "a container pool outgrew 128 containers (N3)");
   return PROTEAN_OK;
 }
 

@@ -85,7 +85,8 @@ struct CtaState {
   int64_t nlog;
   int nb, cursor, all_avail, bad;
   int task, adone;
-  int wtot;          // window entries copied this epoch (incl. alignment padding)
+  int wtot;
+  unsigned long long cold;  // N3 cold starts of the replica          // window entries copied this epoch (incl. alignment padding)
   unsigned long long cnt[10];
 };
 
@@ -180,7 +181,8 @@ __device__ __forceinline__ bool available(const Ctx& c, int g, int64_t t) {
 }
 
 // O11: one revocation boundary tau = k * T_rev for node g (draws specified in DESIGN.md §3).
-__device__ __forceinline__ void vm_event(const ReplayParams& P, const Ctx& c, uint64_t replica, int g,
+// Returns true when the node changes VM under Spot Only (its containers go with it, reading R27).
+__device__ __forceinline__ bool vm_event(const ReplayParams& P, const Ctx& c, uint64_t replica, int g,
                                       int64_t k, int64_t tau) {
   const uint64_t x = (replica << 32) ^ ((uint64_t)g << 20) ^ ((uint64_t)k << 2);
   const uint64_t d0 = smix(P.seed ^ smix(x ^ 0ull)) >> 11;
@@ -206,6 +208,7 @@ __device__ __forceinline__ void vm_event(const ReplayParams& P, const Ctx& c, ui
         bill_switch(c, g, VM_NONE, tau + P.notice, P.H);
         c.gu8[1 * c.N + g] = kNoGeom;
         c.gi[0 * c.N + g] = c.gi[1 * c.N + g] = 0;
+        return true;
       }
     } else if (c.gu8[3 * c.N + g] == VM_NONE) {
       if (spot_ok) {
@@ -215,9 +218,89 @@ __device__ __forceinline__ void vm_event(const ReplayParams& P, const Ctx& c, ui
         bill_switch(c, g, VM_SPOT, tau, P.H);
         reset_gpu_state(c, g, P.init_geom);
         c.gi[0 * c.N + g] = c.gi[1 * c.N + g] = 0;
+        return true;
       }
     }
   }
+  return false;
+}
+
+// ---- N3: the Autoscaler's container pools (readings R22-R27).  Per CTA slot
+// in global scratch: busy-until [N][M][kPoolCap] int64, size [N][M] and surplus counter [N][M] int32.
+struct Pools {
+  int64_t* bu;
+  int32_t* sz;
+  int32_t* ctr;
+  int M;
+  __device__ __forceinline__ size_t pm(int g, int m) const { return (size_t)g * M + m; }
+};
+
+__device__ __forceinline__ void pool_reset(const ReplayParams& P, const Pools& pl, int g) {  // R22
+  for (int m = 0; m < pl.M; ++m) {
+    for (int i = 0; i < P.prewarm; ++i) pl.bu[pl.pm(g, m) * kPoolCap + i] = 0;
+    pl.sz[pl.pm(g, m)] = P.prewarm;
+    pl.ctr[pl.pm(g, m)] = 0;
+  }
+}
+
+// R23: the first container of (g, m) idle at t, else a new one after a cold start.  Called by every
+// lane of an actual-placement warp; the 8 lanes of a GPU's group scan its pool 8 entries at a time
+// (one coalesced 64-byte load), a ballot finds the first idle one.  `part`: this lane's group
+// places a batch now.  Returns the container index (-1: pool full, err[2]) and *t_eff = t or
+// t + cold_us, identical on every lane of the group; the group leader counts the cold start.
+__device__ __forceinline__ int pool_acquire(const ReplayParams& P, const Pools& pl, bool part, int g, int m,
+                                            int64_t t, int lane, int gbase, int64_t* t_eff,
+                                            unsigned long long* cold) {
+  const size_t k = part ? pl.pm(g, m) : 0;
+  const int64_t* b = pl.bu + k * kPoolCap;
+  const int n = part ? pl.sz[k] : 0;
+  int found = -1;
+#pragma unroll 1
+  for (int base = 0;; base += 8) {
+    const bool left = part && found < 0 && base < n;
+    if (!__any_sync(0xffffffffu, left)) break;
+    const int i = base + (lane & 7);
+    const bool hit = left && i < n && b[i] <= t;
+    const unsigned gm = (__ballot_sync(0xffffffffu, hit) >> gbase) & 0xFFu;
+    if (left && gm) found = base + __ffs(gm) - 1;
+  }
+  *t_eff = t;
+  if (!part || found >= 0) return found;
+  *t_eff = t + P.cold_us;  // a new container (reactive scale-up)
+  if (lane == gbase) *cold += 1;
+  if (n >= kPoolCap) {
+    if (lane == gbase) atomicOr(&P.err[2], 1);
+    return -1;
+  }
+  if (lane == gbase) {
+    pl.bu[k * kPoolCap + n] = t;
+    pl.sz[k] = n + 1;
+  }
+  return n;
+}
+
+// R26: at the epoch end, pools larger than the epoch's batch count n_c for keepalive_epochs
+// consecutive epochs terminate their surplus containers idle at T (stable compaction).
+__device__ __forceinline__ void pool_terminate(const ReplayParams& P, const Pools& pl, const Ctx& c, int g, int m,
+                                               const Bat* bats, const uint32_t* gl, int64_t T) {
+  int need = 0;
+  for (int x = c.g_off[g]; x < c.g_off[g + 1]; ++x) need += (((bats[gl[x]].info >> 16) & 0xFF) == (uint32_t)m) ? 1 : 0;
+  const size_t k = pl.pm(g, m);
+  const int n = pl.sz[k];
+  int surplus = n - need;
+  if (surplus <= 0) {
+    pl.ctr[k] = 0;
+    return;
+  }
+  if (++pl.ctr[k] < P.keepalive) return;
+  int64_t* b = pl.bu + k * kPoolCap;
+  int w = 0;
+  for (int i = 0; i < n; ++i) {
+    if (surplus > 0 && b[i] <= T) { --surplus; continue; }
+    b[w++] = b[i];
+  }
+  pl.sz[k] = w;
+  pl.ctr[k] = 0;
 }
 
 // Bulk L2 prefetch (TMA engine, sm_90+): [p, p + bytes) rounded out to 16-byte boundaries.
@@ -523,7 +606,7 @@ __device__ __forceinline__ int alg2_final_geometry(const ReplayParams& P, const 
 
 // kAlg2: the policy-2 instance (N1).  A separate instance keeps Alg 2's code out of the search
 // kernel's register allocation (measured: a shared instance costs the search path 1.5%).
-template <bool kAlg2>
+template <bool kAlg2, bool kN3>
 __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kernel(ReplayParams P) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ CtaState cs;
@@ -570,6 +653,11 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
   c.sord = reinterpret_cast<uint32_t*>(smem + SL.ord);
   c.sgl = reinterpret_cast<uint32_t*>(smem + SL.glist);
   char* slot = P.scratch + (size_t)blockIdx.x * P.slot_bytes;
+  Pools pl;  // N3 container pools (kN3 instance only)
+  pl.bu = reinterpret_cast<int64_t*>(slot + P.o_pool);
+  pl.sz = reinterpret_cast<int32_t*>(slot + P.o_pool + (size_t)N * P.tl.M * kPoolCap * 8);
+  pl.ctr = pl.sz + (size_t)N * P.tl.M;
+  pl.M = P.tl.M;
   c.gb = reinterpret_cast<Bat*>(slot + P.o_gbat);
   c.gord = reinterpret_cast<uint32_t*>(slot + P.o_gord);
   c.ggl = reinterpret_cast<uint32_t*>(slot + P.o_gglist);
@@ -615,6 +703,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
       c.gi[4 * c.N + g] = 0;
       c.gi[8 * c.N + g] = c.gi[9 * c.N + g] = c.gi[10 * c.N + g] = c.gi[11 * c.N + g] = 0;
       c.gi[12 * c.N + g] = c.gi[13 * c.N + g] = 0;  // Alg 2 EWMA history (policy 2)
+      if constexpr (kN3) pool_reset(P, pl, g);
     }
     if (tid == 0) {
       cs.nlog = 0;
@@ -624,6 +713,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
       cs.adone = 0;
       cs.nb = 0;
       cs.all_avail = 1;
+      cs.cold = 0;
 #pragma unroll
       for (int i = 0; i < 10; ++i) cs.cnt[i] = 0;
     }
@@ -641,7 +731,10 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
             const int64_t tau = k * P.rev;
             if (k < 1 || tau >= P.H) continue;
             if (c.gu8[1 * c.N + g] != kNoGeom && c.gi[1 * c.N + g] <= tau) reset_gpu_state(c, g, c.gu8[1 * c.N + g]);
-            vm_event(P, c, replica, g, k, tau);
+            const bool lost = vm_event(P, c, replica, g, k, tau);
+            if constexpr (kN3) {
+              if (lost) pool_reset(P, pl, g);
+            }
           }
         }
         if (c.gu8[1 * c.N + g] != kNoGeom && c.gi[1 * c.N + g] <= Tend) reset_gpu_state(c, g, c.gu8[1 * c.N + g]);
@@ -1159,13 +1252,30 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
           const uint32_t info = has ? bt->info : 0u;
           const int m = (info >> 16) & 0xFF, nreq = info & 0xFFFF;
           const bool strict = (info >> 24) & 1;
-          const int64_t t = has ? (int64_t)bt->ready : 0;
+          int64_t t = has ? (int64_t)bt->ready : 0;
+          int ci = -1;  // N3: the batch's container (group leader)
+          if constexpr (kN3) {  // R23: container acquisition on the actual placement only (R25)
+            if (actual) {
+              int64_t te = t;
+              unsigned long long cold = 0;
+              ci = pool_acquire(P, pl, has && valid, g, m, t, lane, gbase, &te, &cold);
+              if (cold) atomicAdd(&cs.cold, cold);
+              t = te;
+              if (lane != gbase) ci = -1;  // the leader releases it after the placement
+            }
+          }
           int64_t st, en;
           const SliceOut so = place_group(T, active && has, K, L, n, ls, t, m, strict,
                                           P.max_live, &st, &en);
           const bool placed = !so.drop_overflow && so.kmin != ~0ull;
           const int wl = (gbase + (int)(so.kmin & 7)) & 31;
           const int64_t cwin = __shfl_sync(0xffffffffu, en, wl);
+          if constexpr (kN3) {  // R24: busy until the batch ends (a drop releases it at once)
+            if (actual) {
+              if (ci >= 0) pl.bu[pl.pm(g, m) * kPoolCap + ci] = placed ? cwin : t;
+              __syncwarp();  // the group's next search reads the pool
+            }
+          }
           if (!has) continue;
           if (actual) {
             if (placed && lane == wl) {  // winner: busy union + memory-time, clipped to [0, H)
@@ -1234,6 +1344,10 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
       }
       __syncthreads();
       PH(7);
+      if constexpr (kN3) {  // R26: delayed termination (pools are next used in the next epoch's E)
+#pragma unroll 1
+        for (int k = tid; k < N * pl.M; k += NT) pool_terminate(P, pl, c, k / pl.M, k % pl.M, c.bats, c.gl, Tend);
+      }
       // ---------------------------------------------------------------- G: decisions (O9, O10)
       if (PROTEAN_WARP_G && P.xl.n <= 1 && N <= 32) {
         // one warp, lane = simulated GPU: argmin over the candidate keys, Alg 2 hysteresis, then
@@ -1260,7 +1374,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
                 atomicAdd(&cs.cnt[9], (unsigned long long)Gc);
               } else {  // policy 2: Alg 2's own heuristic (N1)
                 if constexpr (kAlg2) best = alg2_final_geometry(P, c, g, c.bats, c.gl);
-                else best = cur;  // unreachable: policy 2 launches replay_kernel<true>
+                else best = cur;  // unreachable: policy 2 launches replay_kernel<true, *>
               }
               dec_out = (uint8_t)best;
               c.gu8[6 * c.N + g] = (uint8_t)best;
@@ -1347,7 +1461,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
             atomicAdd(&cs.cnt[9], (unsigned long long)Gc);
           } else {  // policy 2: Alg 2's own heuristic (N1)
             if constexpr (kAlg2) best = alg2_final_geometry(P, c, g, c.bats, c.gl);
-            else best = cur;  // unreachable: policy 2 launches replay_kernel<true>
+            else best = cur;  // unreachable: policy 2 launches replay_kernel<true, *>
           }
           dec_out = (uint8_t)best;
           c.gu8[6 * c.N + g] = (uint8_t)best;
@@ -1470,6 +1584,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
       P.util[2 * (size_t)r] = __ddiv_rn((double)busy, __dmul_rn(__dmul_rn(7.0, dN), dH));
       P.util[2 * (size_t)r + 1] = __ddiv_rn((double)memt, __dmul_rn(__dmul_rn(40960.0, dN), dH));
       if (P.n_batches) P.n_batches[r] = cs.nlog;
+      if (P.cold_starts) P.cold_starts[r] = (int64_t)cs.cold;
     }
     __syncthreads();
   }
@@ -1539,7 +1654,8 @@ static cudaError_t raise_dyn_smem_once() {
   int optin = 0;
   e = cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
   if (e != cudaSuccess) return e;
-  for (auto k : {replay_kernel<false>, replay_kernel<true>}) {
+  for (auto k : {replay_kernel<false, false>, replay_kernel<true, false>, replay_kernel<false, true>,
+                 replay_kernel<true, true>}) {
     cudaFuncAttributes a;
     e = cudaFuncGetAttributes(&a, k);
     if (e != cudaSuccess) return e;
@@ -1552,8 +1668,10 @@ static cudaError_t raise_dyn_smem_once() {
 
 cudaError_t preload_kernels() {
   cudaFuncAttributes a;
-  cudaError_t e = cudaFuncGetAttributes(&a, replay_kernel<false>);
-  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, replay_kernel<true>);
+  cudaError_t e = cudaSuccess;
+  for (auto k : {replay_kernel<false, false>, replay_kernel<true, false>, replay_kernel<false, true>,
+                 replay_kernel<true, true>})
+    if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, k);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, prepass_kernel);
   if (e == cudaSuccess) e = preload_partition_kernels();
   if (e == cudaSuccess) e = raise_dyn_smem_once();
@@ -1563,10 +1681,14 @@ cudaError_t preload_kernels() {
 cudaError_t launch_replay(const ReplayParams& P, int grid, int block, cudaStream_t st) {
   cudaError_t e = raise_dyn_smem_once();
   if (e != cudaSuccess) return e;
-  if (P.policy == 2)
-    replay_kernel<true><<<grid, block, P.sl.total, st>>>(P);
-  else
-    replay_kernel<false><<<grid, block, P.sl.total, st>>>(P);
+  const bool n3 = P.cold_us > 0;  // cold_us = 0: warm containers, no pool work (reading Q15)
+  if (P.policy == 2) {
+    if (n3) replay_kernel<true, true><<<grid, block, P.sl.total, st>>>(P);
+    else replay_kernel<true, false><<<grid, block, P.sl.total, st>>>(P);
+  } else {
+    if (n3) replay_kernel<false, true><<<grid, block, P.sl.total, st>>>(P);
+    else replay_kernel<false, false><<<grid, block, P.sl.total, st>>>(P);
+  }
   return cudaGetLastError();
 }
 
@@ -1574,10 +1696,14 @@ cudaError_t launch_replay(const ReplayParams& P, int grid, int block, cudaStream
 cudaError_t replay_occupancy(int block, size_t smem, int* blocks_per_sm) {
   cudaError_t e = raise_dyn_smem_once();
   if (e != cudaSuccess) return e;
-  int a = 0, b = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, replay_kernel<false>, block, smem);
-  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, replay_kernel<true>, block, smem);
-  *blocks_per_sm = a < b ? a : b;
+  int lo = 1 << 30;
+  for (auto k : {replay_kernel<false, false>, replay_kernel<true, false>, replay_kernel<false, true>,
+                 replay_kernel<true, true>}) {
+    int a = 0;
+    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, k, block, smem);
+    lo = a < lo ? a : lo;
+  }
+  *blocks_per_sm = lo;
   return e;
 }
 

@@ -24,6 +24,7 @@ constexpr int kZA = 8;            // lanes per actual-placement group (one per s
 #endif
 constexpr int kAG = PROTEAN_AGPU;  // simulated GPUs per actual-placement warp unit (1, 2 or 4)
 constexpr int kMaxStreams = 2 * PROTEAN_MAX_MODELS;
+constexpr int kPoolCap = 128;     // N3: containers per (sim-GPU, model) (reading R22)
 constexpr int64_t kForever = INT64_MAX;
 
 // One batch of the current epoch (40 B).  info = n | model << 16 | strict << 24.
@@ -96,6 +97,8 @@ struct ReplayParams {
   int policy, wait_limit, cap_pct, init_geom, max_live, vm_policy;
   int ewma_a, g421, g43;   // policy 2 (N1): EWMA weight per mille, indices of (4g,2g,1g), (4g,3g)
   int64_t t_low, t_high;   //   T_low / T_high in milli-BE-batches per epoch
+  int64_t cold_us;         // N3: container cold start (0 = warm containers, no pool work)
+  int keepalive, prewarm;  //   delayed termination (epochs), idle containers at t = 0
   int64_t reconfig_us, rev, notice;
   uint64_t thr, seed;
   double price_od, price_spot;
@@ -112,12 +115,13 @@ struct ReplayParams {
   protean_batch_rec* log;
   int64_t log_cap;
   int64_t* n_batches;
+  int64_t* cold_starts;    // [R] N3 cold starts, or NULL
   // scratch
   SmemLayout sl;
   int WCAP;                // max window entries of any epoch (prepass)
   char* scratch;
-  size_t slot_bytes, o_alist, o_clist, o_gbat, o_gord, o_gglist, o_gsarr;
-  int* err;                // err[0]: invalid request, err[1]: exchange timeout
+  size_t slot_bytes, o_alist, o_clist, o_gbat, o_gord, o_gglist, o_gsarr, o_pool;
+  int* err;                // err[0]: invalid request, err[1]: exchange timeout, err[2]: pool overflow
   // mode G exchange (xl.n == 0: off)
   XLayout xl;
   char* const* xpeer;      // [n] every rank's exchange buffer, mapped in this process

@@ -28,7 +28,7 @@ def gpu_replay(prof, trace, *, want_keys=True, want_log=True, **cfg):
 ORACLE_CFG_KEYS = {"n_gpus": "N", "epoch_len_us": "W", "reconfig_cap_pct": "cap_pct",
                    "price_od_node_hr": "price_od", "price_spot_node_hr": "price_spot",
                    "rev_interval_us": "rev_interval", "notice_us": "notice", "t_low_milli": "t_low",
-                   "t_high_milli": "t_high"}
+                   "t_high_milli": "t_high", "cold_start_us": "cold_us"}
 
 
 def oracle_replay(O, prof, trace, *, want_keys=True, want_log=True, nthreads=8, **cfg):
@@ -45,6 +45,7 @@ def compare(g, o, R, *, keys=True, log=True):
             raise AssertionError(f"{k} mismatch at {bad.tolist()}: gpu {a[tuple(bad[0])]} oracle {b[tuple(bad[0])]}")
     assert np.array_equal(g["hist"], o["hist"]), "hist mismatch"
     assert np.array_equal(g["n_batches"], o["n_batches"]), "n_batches mismatch"
+    assert np.array_equal(g["cold_starts"], o["cold_starts"]), "cold_starts mismatch"
     np.testing.assert_allclose(g["cost"], o["cost"], rtol=1e-6, atol=0)
     np.testing.assert_allclose(g["util"], o["util"], rtol=1e-6, atol=0)
     assert np.array_equal(g["cost"], o["cost"]) and np.array_equal(g["util"], o["util"])
