@@ -3,6 +3,10 @@ import sys
 
 import pytest
 
+# hardware queues for the in-process mode-G ranks (see paper_conf_middleware_bhasisjgpkd24_b200/__init__.py);
+# must precede CUDA initialisation
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
+
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 if ROOT not in sys.path:
     sys.path.insert(0, ROOT)

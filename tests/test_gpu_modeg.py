@@ -82,7 +82,7 @@ def _check_ranks(host, merged, o, R, bounds):
         assert np.array_equal(h["cand_keys"][..., lo:hi], o["cand_keys"][..., lo:hi])
 
 
-@pytest.mark.parametrize("nranks", [2, 3])
+@pytest.mark.parametrize("nranks", [2, 3, 5, 8])
 def test_mode_g_mix_a(oracle, nranks):
     prof = synth_profiles()
     tr = tick_trace(mix_a_params(3, seed=21, seconds=20))
