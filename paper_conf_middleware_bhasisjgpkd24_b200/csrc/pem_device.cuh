@@ -83,20 +83,25 @@ static __device__ __noinline__ void place_slow_slice(const Tab& T, const uint8_t
                                               int p, int64_t t0, int32_t q, int m, int64_t* start_out,
                                               int64_t* F_out) {
   const int32_t Ms = prof_cap(p);
-  int64_t used = 0;
+  int64_t used = 0, e = INT64_MAX;
   for (int i = 0; i < n; ++i)
-    if ((int)(L.meta(i) & 0xFF) == s && L.en(i) > t0) used += L.mem(i);
-  int64_t start = t0;
-  if (used + q > Ms) {  // earliest release that makes the batch fit
-    start = INT64_MAX;
-    for (int i = 0; i < n; ++i) {
-      if ((int)(L.meta(i) & 0xFF) != s || L.en(i) <= t0) continue;
-      const int64_t ei = L.en(i);
-      int64_t rem = 0;
-      for (int j = 0; j < n; ++j)
-        if ((int)(L.meta(j) & 0xFF) == s && L.en(j) > ei) rem += L.mem(j);
-      if (rem + q <= Ms && ei < start) start = ei;
+    if ((int)(L.meta(i) & 0xFF) == s && L.en(i) > t0) {
+      used += L.mem(i);
+      e = L.en(i) < e ? L.en(i) : e;
     }
+  int64_t start = t0;
+  if (used + q > Ms) {  // earliest release that makes the batch fit, releases in ascending order
+    for (;;) {
+      int64_t rem = 0, nxt = INT64_MAX;
+      for (int j = 0; j < n; ++j)
+        if ((int)(L.meta(j) & 0xFF) == s && L.en(j) > e) {
+          rem += L.mem(j);
+          nxt = L.en(j) < nxt ? L.en(j) : nxt;
+        }
+      if (rem + q <= Ms) break;
+      e = nxt;
+    }
+    start = e;
   }
   int64_t F = T.fbr[m * kNProf + p];
   for (int i = 0; i < n; ++i) {

@@ -357,28 +357,45 @@ __device__ __forceinline__ uint64_t group_min(uint64_t v, int Z) {
 __device__ __noinline__ void slice_slow(const LaneList& L, int n, int64_t t0, int32_t q, int32_t Ms,
                                         const int32_t* fbr_p, int64_t own_f, int64_t* start_out,
                                         int64_t* F_out) {
-  int64_t used = 0;
+  // one pass per tried start time: memory still held, the next release, and Eq 1's co-runner sum
+  // at that time (residents with S <= start < E), so the accepted pass already holds F
+  int64_t used = 0, e = INT64_MAX, F = own_f;  // at t0: memory held after t0, earliest release
 #pragma unroll 1
-  for (int i = 0; i < n; ++i)
-    if (L.E(i) > t0) used += L.M(i) & 0xFFFF;
-  int64_t start = t0;
-  if (used + q > Ms) {
-    start = INT64_MAX;
-  #pragma unroll 1
   for (int i = 0; i < n; ++i) {
-      const int64_t ei = L.E(i);
-      if (ei <= t0) continue;
-      int64_t rem = 0;
-#pragma unroll 1
-      for (int k = 0; k < n; ++k)
-        if (L.E(k) > ei) rem += L.M(k) & 0xFFFF;
-      if (rem + q <= Ms && ei < start) start = ei;
+    const int64_t ei = L.E(i);
+    if (ei > t0) {
+      const uint32_t mi = L.M(i);
+      used += mi & 0xFFFF;
+      e = ei < e ? ei : e;
+      if (L.S(i) <= t0) F += fbr_p[((mi >> 16) & 63) * kNProf];
     }
   }
-  int64_t F = own_f;
+  int64_t start = t0;
+  if (used + q > Ms) {
+    // the earliest release e after which the footprints still held (ends > e) leave room: the
+    // held memory only shrinks as e grows, so releases are tried in ascending order and the first
+    // that fits is the minimum of the plain definition (each pass also finds the next release)
 #pragma unroll 1
-  for (int i = 0; i < n; ++i)
-    if (L.S(i) <= start && start < L.E(i)) F += fbr_p[((L.M(i) >> 16) & 63) * kNProf];
+    for (;;) {
+      int64_t rem = 0, nxt = INT64_MAX, Fe = own_f;
+#pragma unroll 1
+      for (int k = 0; k < n; ++k) {
+        const int64_t ek = L.E(k);
+        if (ek > e) {
+          const uint32_t mk = L.M(k);
+          rem += mk & 0xFFFF;
+          nxt = ek < nxt ? ek : nxt;
+          if (L.S(k) <= e) Fe += fbr_p[((mk >> 16) & 63) * kNProf];
+        }
+      }
+      if (rem + q <= Ms) {  // always by the last release (q <= Ms)
+        F = Fe;
+        break;
+      }
+      e = nxt;
+    }
+    start = e;
+  }
   *start_out = start;
   *F_out = F;
 }
