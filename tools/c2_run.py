@@ -16,6 +16,7 @@ arr = torch.from_numpy(np.ascontiguousarray(tr.arrival_us).view(np.int32)).to(de
 meta = torch.from_numpy(np.ascontiguousarray(tr.meta)).to(dev)
 off = torch.from_numpy(np.ascontiguousarray(tr.replica_off, np.int64)).to(dev)
 h = pkg.load_profiles(synth_profiles())
-out = h.replay_traces(arr, meta, off, trace_len_us=tr.trace_len_us, n_gpus=8)
+POL = int(sys.argv[2]) if len(sys.argv) > 2 else 0
+out = h.replay_traces(arr, meta, off, trace_len_us=tr.trace_len_us, n_gpus=8, policy=POL)
 torch.cuda.synchronize()
 print("replay ms", h.last_timings()[1], "launch", h.last_timings()[2])
