@@ -136,3 +136,24 @@ def test_wide_times_64bit_path(oracle, seed):
     o = oracle.sweep(prof, R=R, N=N, batches=batches, batch_off=off, arrival=arr, cur_geom=cur, max_batches=5)
     _compare(g, o, 12)
     assert (o["sweep_key"] & 0xFFFFFFFFFF00 != 0).any()  # some BE tails are long
+
+
+def test_bench_launch_sampled_units(oracle):
+    """The exact bench.py --path sweep launch (4096 replicas x 8 sim-GPUs, seed 1000, <= 8 batches):
+    sampled GPU-epochs (<= 6 batches, so the oracle's brute force stays in seconds) re-derived."""
+    P = synth_profiles()
+    R, N = 4096, 8
+    batches, off, arr, cur = epoch_batches(1000, R, N, max_batches=8)
+    g = _gpu_sweep(P, R, N, batches, off, arr, cur)
+    b = np.diff(off)
+    rng = np.random.default_rng(5)
+    picks = [u for u in rng.permutation(R * N)[:400] if b[u] <= 6][:12] + [0, R * N - 1]
+    for u in picks:
+        if b[u] > 6:
+            continue
+        lo, hi = int(off[u]), int(off[u + 1])
+        sb = {k: v[lo:hi] for k, v in batches.items()}
+        o = oracle.sweep(P, R=1, N=1, batches=sb, batch_off=[0, hi - lo], arrival=arr, cur_geom=cur[u:u + 1])
+        assert g["sweep_key"][u * 12:(u + 1) * 12].tolist() == o["sweep_key"].tolist()
+        assert g["assign"][u * 12:(u + 1) * 12].tolist() == o["assign"].tolist()
+        assert g["best_key"][u] == o["best_key"][0]
