@@ -225,6 +225,14 @@ typedef struct {
   int32_t keepalive_epochs;    /* N3: surplus containers terminated after this many consecutive
                                   surplus epochs, >= 1 (default 600 = ~10 min at W = 1 s) */
   int32_t prewarm;             /* N3: idle containers per (sim-GPU, model) at t = 0, 0..128 */
+  int32_t ctas_per_replica;    /* search policy, shard_mode 0: CTAs sharing one replica, each scoring
+                                  a slot-balanced geometry range and exchanging min-loc keys per
+                                  epoch in device memory (mode G inside one launch).  0 = auto
+                                  (min(16, G, SMs / replicas) when replicas < SMs, else 1); 1 = off;
+                                  k = min(k, 16, G).  Outputs are identical for every setting.  The
+                                  CTAs of a replica must run concurrently: a device shared with other
+                                  work can delay them past the exchange timeout (PROTEAN_ENCCL). */
+  int32_t reserved2;           /* must be 0 */
 } protean_replay_cfg;
 
 /* counters[10] per replica (O7/O8/O10):

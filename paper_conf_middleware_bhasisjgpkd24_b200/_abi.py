@@ -76,7 +76,7 @@ class ReplayCfg(C.Structure):
                 ("shard_mode", C.c_int32), ("rank", C.c_int32), ("nranks", C.c_int32),
                 ("max_ctas", C.c_int32), ("ewma_alpha_pm", C.c_int32), ("t_low_milli", C.c_int64),
                 ("t_high_milli", C.c_int64), ("cold_start_us", C.c_int64), ("keepalive_epochs", C.c_int32),
-                ("prewarm", C.c_int32)]
+                ("prewarm", C.c_int32), ("ctas_per_replica", C.c_int32), ("reserved2", C.c_int32)]
 
 
 class SweepIn(C.Structure):      # protean_sweep_in

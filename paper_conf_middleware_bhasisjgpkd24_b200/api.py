@@ -15,7 +15,8 @@ _REPLAY_DEFAULTS = dict(n_gpus=8, epoch_len_us=1_000_000, policy=0, wait_limit=3
                         price_od_node_hr=32.7726 / 8, price_spot_node_hr=9.8318 / 8,
                         rev_interval_us=300_000_000, notice_us=30_000_000, seed=0, shard_mode=0,
                         rank=0, nranks=1, max_ctas=0, replica_base=0, ewma_alpha_pm=500, t_low_milli=500,
-                        t_high_milli=4000, cold_start_us=0, keepalive_epochs=600, prewarm=0)
+                        t_high_milli=4000, cold_start_us=0, keepalive_epochs=600, prewarm=0,
+                        ctas_per_replica=0)
 
 
 def _torch():
@@ -173,7 +174,7 @@ class Handle:
         for k in ("policy", "wait_limit", "reconfig_cap_pct", "init_geom", "max_live", "vm_policy",
                   "reconfig_us", "rev_interval_us", "notice_us", "seed", "shard_mode", "rank", "nranks",
                   "max_ctas", "ewma_alpha_pm", "t_low_milli", "t_high_milli", "cold_start_us",
-                  "keepalive_epochs", "prewarm"):
+                  "keepalive_epochs", "prewarm", "ctas_per_replica"):
             setattr(cf, k, int(c[k]))
         for k in ("p_rev", "price_od_node_hr", "price_spot_node_hr"):
             setattr(cf, k, float(c[k]))

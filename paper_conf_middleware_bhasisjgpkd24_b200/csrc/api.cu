@@ -49,6 +49,15 @@ struct protean_handle {
   // mode G: candidate lane packing of the rank's geometry range
   uint32_t* d_pack_g = nullptr;
   int CW_g = 0, pack_lo = -1, pack_hi = -1;
+  // virtual ranks (several CTAs per replica inside one launch): packs, exchange buffers
+  int vr_n = 0;
+  std::vector<uint32_t*> vr_pack;
+  std::vector<int> vr_b, vr_cw;
+  void* d_vxbuf = nullptr;
+  size_t vx_bytes = 0;
+  char** d_vpeer = nullptr;
+  XLayout vxl{0, 0, 0};
+  uint32_t vseq = 0;
   // mode G exchange (protean_xchg_*)
   XLayout xl{0, 0, 0};
   int xrank = 0;
@@ -346,6 +355,7 @@ void protean_replay_cfg_defaults(protean_replay_cfg* c) {
   c->cold_start_us = 0;
   c->keepalive_epochs = 600;
   c->prewarm = 0;
+  c->ctas_per_replica = 0;
 }
 
 int protean_load_profiles(const protean_profiles* p, protean_handle** out) {
@@ -432,6 +442,9 @@ void protean_free(protean_handle* h) {
   if (h->d_small) cudaFree(h->d_small);
   if (h->d_pack) cudaFree(h->d_pack);
   if (h->d_pack_g) cudaFree(h->d_pack_g);
+  for (uint32_t* q : h->vr_pack) cudaFree(q);
+  if (h->d_vxbuf) cudaFree(h->d_vxbuf);
+  if (h->d_vpeer) cudaFree(h->d_vpeer);
   xchg_release(h);
   for (int i = 0; i < 6; ++i)
     if (h->ev[i]) cudaEventDestroy(h->ev[i]);
@@ -566,6 +579,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   if (c.shard_mode != 0 && c.shard_mode != 1) return fail(h, PROTEAN_EINVAL, "shard_mode");
   if (c.cold_start_us < 0 || c.keepalive_epochs < 1 || c.prewarm < 0 || c.prewarm > kPoolCap)
     return fail(h, PROTEAN_EINVAL, "cold_start_us / keepalive_epochs / prewarm");
+  if (c.ctas_per_replica < 0 || c.reserved2 != 0) return fail(h, PROTEAN_EINVAL, "ctas_per_replica / reserved2");
   if (c.max_ctas < 0) return fail(h, PROTEAN_EINVAL, "max_ctas");
   const bool modeG = c.shard_mode == 1;
   if (modeG) {
@@ -678,6 +692,37 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
     d_pack = h->d_pack_g;
     CW = h->CW_g;
   }
+  // virtual ranks: with fewer replicas than SMs, several CTAs share one replica, each scoring a
+  // slot-balanced geometry range and exchanging min-loc keys per epoch in device memory (the
+  // mode G exchange inside one launch); auto = min(16, G, SMs / R)
+  int vr_n = 1;
+  if (!modeG && c.policy == 0 && h->G >= 2 && c.ctas_per_replica != 1) {
+    vr_n = c.ctas_per_replica > 1 ? c.ctas_per_replica : (R < h->nsm ? h->nsm / R : 1);
+    vr_n = std::min(vr_n, std::min(kMaxVR, h->G));
+    if (vr_n < 2) vr_n = 1;
+  }
+  if (vr_n > 1 && vr_n != h->vr_n) {  // per-range candidate packing (cached per split)
+    for (uint32_t* q : h->vr_pack) cudaFree(q);
+    h->vr_pack.assign(vr_n, nullptr);
+    h->vr_b.assign(vr_n + 1, 0);
+    h->vr_cw.assign(vr_n, 0);
+    split_ranges(h->gn, vr_n, h->vr_b.data());
+    for (int k = 0; k < vr_n; ++k) {
+      std::vector<uint32_t> pk = build_pack(h->gn, h->vr_b[k], h->vr_b[k + 1], &h->vr_cw[k]);
+      CK(h, cudaMalloc(&h->vr_pack[k], pk.size() * 4));
+      CK(h, cudaMemcpy(h->vr_pack[k], pk.data(), pk.size() * 4, cudaMemcpyHostToDevice));
+    }
+    h->vr_n = vr_n;
+  }
+  if (vr_n > 1) {  // the layout holds the largest range of any virtual rank
+    geom_lo = 0;
+    geom_hi = 0;
+    CW = 0;
+    for (int k = 0; k < vr_n; ++k) {
+      geom_hi = std::max(geom_hi, h->vr_b[k + 1] - h->vr_b[k]);
+      CW = std::max(CW, h->vr_cw[k]);
+    }
+  }
   // launch geometry: 8 warps; units = actual-placement warps + candidate warps per GPU
   const int Gc = geom_hi - geom_lo;
   // warps per CTA: the placement phase runs n_units warp units; pick 4..8 warps that divide them
@@ -703,8 +748,9 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   int per_sm = 0;
   CK(h, replay_occupancy(block, sl.total, &per_sm));
   if (per_sm < 1) return fail(h, PROTEAN_ERANGE, "replay kernel does not fit an SM");
-  int grid = (int)std::min<int64_t>(R, (int64_t)h->nsm * per_sm);
-  if (c.max_ctas > 0) grid = std::min(grid, c.max_ctas);
+  int grid = (int)std::min<int64_t>((int64_t)R * vr_n, (int64_t)h->nsm * per_sm);
+  grid -= grid % vr_n;  // every replica's CTAs are resident together (exchange partners)
+  if (c.max_ctas > 0) grid = std::min(grid, std::max(c.max_ctas, vr_n) / vr_n * vr_n);
 
   ReplayParams P;
   std::memset(&P, 0, sizeof(P));
@@ -744,8 +790,44 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   P.seed = c.seed;
   P.price_od = c.price_od_node_hr;
   P.price_spot = c.price_spot_node_hr;
-  P.geom_lo = geom_lo;
-  P.geom_hi = geom_hi;
+  P.geom_lo = vr_n > 1 ? 0 : geom_lo;
+  P.geom_hi = vr_n > 1 ? h->G : geom_hi;
+  P.vr_n = vr_n;
+  if (vr_n > 1) {
+    for (int k = 0; k < vr_n; ++k) {
+      P.vr_lo[k] = h->vr_b[k];
+      P.vr_hi[k] = h->vr_b[k + 1];
+      P.vr_cw[k] = h->vr_cw[k];
+      P.vr_pack[k] = h->vr_pack[k];
+    }
+    const XLayout X{vr_n, R, N};
+    const size_t stride = al(X.bytes());  // 16-byte key pairs: every rank's buffer 256-aligned
+    const size_t need = stride * (size_t)vr_n;
+    if (h->vxl.n != X.n || h->vxl.Rcap != X.Rcap || h->vxl.Ncap != X.Ncap || h->vx_bytes < need) {
+      int rc = ensure(h, &h->d_vxbuf, &h->vx_bytes, need, st);
+      if (rc) return rc;
+      CK(h, cudaMemsetAsync(h->d_vxbuf, 0, need, st));  // flags restart with the sequence
+      std::vector<char*> peers(vr_n);
+      for (int k = 0; k < vr_n; ++k) peers[k] = static_cast<char*>(h->d_vxbuf) + stride * k;
+      void* dp = h->d_vpeer;
+      size_t have = h->d_vpeer ? sizeof(char*) * kMaxVR : 0;
+      rc = ensure(h, &dp, &have, sizeof(char*) * kMaxVR, st);
+      if (rc) return rc;
+      h->d_vpeer = static_cast<char**>(dp);
+      CK(h, cudaMemcpyAsync(h->d_vpeer, peers.data(), sizeof(char*) * vr_n, cudaMemcpyHostToDevice, st));
+      CK(h, cudaStreamSynchronize(st));  // peers lives on this stack frame
+      h->vxl = X;
+      h->vseq = 0;
+    }
+    P.xl = X;
+    P.xpeer = h->d_vpeer;
+    P.xrank = 0;
+    P.xseq = h->vseq;
+    P.xtimeout_ns = 30ull * 1000000000ull;
+    if (const char* ev = std::getenv("PROTEAN_XCHG_TIMEOUT_S"))
+      P.xtimeout_ns = (uint64_t)std::max(1, std::atoi(ev)) * 1000000000ull;
+    CK(h, cudaMemsetAsync(out->counters, 0, sizeof(int64_t) * 10 * (size_t)R, st));  // 8, 9 accumulate
+  }
   if (modeG && !std::getenv("PROTEAN_XCHG_OFF")) {  // debug knob: score the range, no exchange
     P.xl = h->xl;
     P.xpeer = h->d_xpeer;
@@ -792,6 +874,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   CK(h, cudaStreamSynchronize(st));
   herr = herr2[0];
   if (modeG) h->xseq += (uint32_t)E;
+  if (vr_n > 1) h->vseq += (uint32_t)E;
   if (herr2[1]) {
     h->poisoned = true;
     return fail(h, PROTEAN_ENCCL, "mode G exchange: a peer rank did not publish within 30 s");

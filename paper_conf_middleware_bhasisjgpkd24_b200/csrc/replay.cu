@@ -85,6 +85,8 @@ struct CtaState {
   int64_t nlog;
   int nb, cursor, all_avail, bad;
   int task, adone;
+  int glo, ghi, cw, xrank;  // this CTA's candidate geometry range, its candidate warps per GPU and
+                            // its rank in the key exchange (virtual ranks: several CTAs per replica)
   int wtot;
   unsigned long long cold;  // N3 cold starts of the replica          // window entries copied this epoch (incl. alignment padding)
   unsigned long long cnt[10];
@@ -639,7 +641,20 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
 #endif
   const SmemLayout& SL = P.sl;
   const int tid = threadIdx.x, NT = blockDim.x, lane = tid & 31, warp = tid >> 5, NW = NT >> 5;
-  const int N = P.N, S = SL.S, Gc = SL.Gc, CW = SL.CW;
+  const int N = P.N, S = SL.S, Gc = SL.Gc;  // Gc: key stride (the largest range of any CTA)
+  // virtual ranks (P.vr_n > 1): CTA b serves replica b / vr_n and scores geometry range b % vr_n,
+  // exchanging min-loc keys with the replica's other CTAs exactly as mode G ranks do
+  const int vrn = P.vr_n > 1 ? P.vr_n : 1;
+  const int vr = (int)(blockIdx.x % (unsigned)vrn);
+  const int glo = vrn > 1 ? P.vr_lo[vr] : P.geom_lo, ghi = vrn > 1 ? P.vr_hi[vr] : P.geom_hi;
+  const int cwr = vrn > 1 ? P.vr_cw[vr] : SL.CW;
+  const uint32_t* pack_src = vrn > 1 ? P.vr_pack[vr] : P.pack;
+  if (tid == 0) {
+    cs.glo = glo;
+    cs.ghi = ghi;
+    cs.cw = cwr;
+    cs.xrank = vrn > 1 ? vr : P.xrank;
+  }
 
   Ctx c;
   int32_t* tabw = reinterpret_cast<int32_t*>(smem + SL.tab);
@@ -647,7 +662,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
   for (int i = tid; i < P.tl.words; i += NT) tabw[i] = P.tab[i];
   uint32_t* packs = reinterpret_cast<uint32_t*>(smem + SL.pack);
 #pragma unroll 1
-  for (int i = tid; i < CW * 32; i += NT) packs[i] = P.pack[i];
+  for (int i = tid; i < cwr * 32; i += NT) packs[i] = pack_src[i];
   const uint32_t mbar = (uint32_t)__cvta_generic_to_shared(&s_mbar);
   if (tid == 0) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mbar) : "memory");
@@ -696,12 +711,12 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
   __syncthreads();
   int sum_slots = 0;  // slot-evals per batch per decidable GPU
 #pragma unroll 1
-  for (int j = P.geom_lo; j < P.geom_hi; ++j) sum_slots += T.gn[j];
+  for (int j = glo; j < ghi; ++j) sum_slots += T.gn[j];
   const int n_aunits = (N + kAG - 1) / kAG;  // actual-placement warp units: kAG GPUs x 8 slice lanes
   const uint32_t* sarr = c.sarr;
 
 #pragma unroll 1
-  for (int r = blockIdx.x; r < P.R; r += gridDim.x) {
+  for (int r = (int)(blockIdx.x / (unsigned)vrn); r < P.R; r += (int)(gridDim.x / (unsigned)vrn)) {
     const uint64_t replica = (uint64_t)(P.base + r);
     uint32_t* ghist = P.hist + (size_t)r * 2 * kNB;
 
@@ -1101,7 +1116,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
       // One loop body serves both kinds (a single inlined copy of Place).
       // dynamic task queue: [actual units][candidate units][accounting of batch rank rk];
       // accounting waits (rarely) for the actual units, whose warps publish via cs.adone
-      const int n_units = n_aunits + (P.policy == 0 ? N * CW : 0);
+      const int n_units = n_aunits + (P.policy == 0 ? N * cs.cw : 0);
       const int n_tasks = n_units + nb;
       for (;;) {
         int u = 0;
@@ -1202,8 +1217,9 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
           valid = (lane >> 3) < kAG && g < N;
           j = valid ? c.gu8[0 * c.N + g] : 0;
         } else {
-          const int cu = u - n_aunits, w = cu % CW;
-          g = cu / CW;
+          const int cw = cs.cw;
+          const int cu = u - n_aunits, w = cu % cw;
+          g = cu / cw;
           const uint32_t pk = c.pack[w * 32 + lane];
           const int jr = pk & 0xFF;
           s = (pk >> 8) & 0xFF;
@@ -1213,7 +1229,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
           j = valid ? jr : 0;
           if (!c.gu8[5 * c.N + g]) {  // undecidable at T: no candidates scored (O5.4)
             if (valid && lane == gbase) {
-              c.keys[g * Gc + (j - P.geom_lo)] = -1;
+              c.keys[g * Gc + (j - cs.glo)] = -1;
               if (P.cand_keys) P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = -1;
             }
             continue;  // warp-uniform: the whole unit belongs to g
@@ -1256,7 +1272,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
           if (valid && lane == gbase) {
             const int64_t key = make_key(misses, tail, j == c.gu8[0 * c.N + g] ? 0 : j + 1);
             if (j == c.gu8[0 * c.N + g]) c.gi[7 * c.N + g] = key;
-            c.keys[g * Gc + (j - P.geom_lo)] = key;
+            c.keys[g * Gc + (j - cs.glo)] = key;
             if (P.cand_keys) P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = key;
           }
           continue;
@@ -1355,7 +1371,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
         } else if (valid && lane == gbase) {
           const int64_t key = make_key(acc0, acc1, j == c.gu8[0 * c.N + g] ? 0 : j + 1);
           if (j == c.gu8[0 * c.N + g]) c.gi[7 * c.N + g] = key;
-          c.keys[g * Gc + (j - P.geom_lo)] = key;
+          c.keys[g * Gc + (j - cs.glo)] = key;
           if (P.cand_keys) P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = key;
         }
       }
@@ -1382,13 +1398,13 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
               int best;
               if (P.policy == 0) {  // S8: argmin over the candidate keys
 #pragma unroll 1
-                for (int v = 0; v < Gc; ++v) kb = c.keys[g * Gc + v] < kb ? c.keys[g * Gc + v] : kb;
+                for (int v = 0; v < cs.ghi - cs.glo; ++v) kb = c.keys[g * Gc + v] < kb ? c.keys[g * Gc + v] : kb;
                 c.gi[6 * c.N + g] = kb;
                 kc = c.gi[7 * c.N + g];
                 const int tag = (int)(kb & 255);
                 best = tag == 0 ? cur : tag - 1;
                 atomicAdd(&cs.cnt[8], (unsigned long long)(c.g_off[g + 1] - c.g_off[g]) * (unsigned long long)sum_slots);
-                atomicAdd(&cs.cnt[9], (unsigned long long)Gc);
+                atomicAdd(&cs.cnt[9], (unsigned long long)(cs.ghi - cs.glo));
               } else {  // policy 2: Alg 2's own heuristic (N1)
                 if constexpr (kAlg2) best = alg2_final_geometry(P, c, g, c.bats, c.gl);
                 else best = cur;  // unreachable: policy 2 launches replay_kernel<true, *>
@@ -1407,7 +1423,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
             if (P.decisions) P.decisions[((size_t)r * P.E + e) * N + g] = dec_out;
             if (P.policy != 0 && P.cand_keys) {
 #pragma unroll 1
-              for (int j = P.geom_lo; j < P.geom_hi; ++j)
+              for (int j = cs.glo; j < cs.ghi; ++j)
                 P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = -1;
             }
           }
@@ -1456,12 +1472,12 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
           int64_t kb = kForever;
           if (c.gu8[5 * c.N + g]) {
 #pragma unroll 1
-            for (int v = 0; v < Gc; ++v) kb = c.keys[g * Gc + v] < kb ? c.keys[g * Gc + v] : kb;
+            for (int v = 0; v < cs.ghi - cs.glo; ++v) kb = c.keys[g * Gc + v] < kb ? c.keys[g * Gc + v] : kb;
           }
           c.gi[6 * c.N + g] = kb;
         }
         if (P.xl.n > 1)
-          exchange_keys(P.xl, P.xpeer, P.xrank, P.err, P.xtimeout_ns, c.gi, N, r,
+          exchange_keys(P.xl, P.xpeer, cs.xrank, P.err, P.xtimeout_ns, c.gi, N, r,
                         (uint32_t)(P.xseq + (uint32_t)e), tid, NT);
       }
 #pragma unroll 1
@@ -1475,7 +1491,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
             const int tag = (int)(kb & 255);
             best = tag == 0 ? cur : tag - 1;
             atomicAdd(&cs.cnt[8], (unsigned long long)(c.g_off[g + 1] - c.g_off[g]) * (unsigned long long)sum_slots);
-            atomicAdd(&cs.cnt[9], (unsigned long long)Gc);
+            atomicAdd(&cs.cnt[9], (unsigned long long)(cs.ghi - cs.glo));
           } else {  // policy 2: Alg 2's own heuristic (N1)
             if constexpr (kAlg2) best = alg2_final_geometry(P, c, g, c.bats, c.gl);
             else best = cur;  // unreachable: policy 2 launches replay_kernel<true, *>
@@ -1492,7 +1508,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
         if (P.decisions) P.decisions[((size_t)r * P.E + e) * N + g] = dec_out;
         if (P.policy != 0 && P.cand_keys) {
 #pragma unroll 1
-          for (int j = P.geom_lo; j < P.geom_hi; ++j)
+          for (int j = cs.glo; j < cs.ghi; ++j)
             P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = -1;
         }
       }
@@ -1590,7 +1606,12 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
         memt += c.gi[11 * c.N + g];
       }
 #pragma unroll 1
-      for (int i = 0; i < 10; ++i) P.counters[(size_t)r * 10 + i] = (int64_t)cs.cnt[i];
+      for (int i = 0; i < 10; ++i) {
+        if (vrn > 1 && i >= 8)  // slot-evals and candidates: this CTA's range only (zeroed by the host)
+          atomicAdd(reinterpret_cast<unsigned long long*>(&P.counters[(size_t)r * 10 + i]), cs.cnt[i]);
+        else
+          P.counters[(size_t)r * 10 + i] = (int64_t)cs.cnt[i];
+      }
       P.accum[(size_t)r * 4 + 0] = busy;
       P.accum[(size_t)r * 4 + 1] = memt;
       P.accum[(size_t)r * 4 + 2] = od;

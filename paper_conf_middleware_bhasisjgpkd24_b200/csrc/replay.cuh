@@ -25,6 +25,7 @@ constexpr int kZA = 8;            // lanes per actual-placement group (one per s
 constexpr int kAG = PROTEAN_AGPU;  // simulated GPUs per actual-placement warp unit (1, 2 or 4)
 constexpr int kMaxStreams = 2 * PROTEAN_MAX_MODELS;
 constexpr int kPoolCap = 128;     // N3: containers per (sim-GPU, model) (reading R22)
+constexpr int kMaxVR = 16;        // virtual ranks: CTAs per replica splitting the geometry range
 constexpr int64_t kForever = INT64_MAX;
 
 // One batch of the current epoch (40 B).  info = n | model << 16 | strict << 24.
@@ -128,6 +129,10 @@ struct ReplayParams {
   int xrank;
   uint32_t xseq;           // sequence number of epoch 0 of this call
   uint64_t xtimeout_ns;    // a source flag not seen within this time fails the call (ENCCL)
+  // virtual ranks (vr_n > 1): CTA b serves replica b / vr_n, geometry range b % vr_n
+  int vr_n;
+  int vr_lo[kMaxVR], vr_hi[kMaxVR], vr_cw[kMaxVR];
+  const uint32_t* vr_pack[kMaxVR];
 };
 
 struct ScoreParams {

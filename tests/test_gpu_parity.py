@@ -266,3 +266,16 @@ def test_long_jobs_wide_times(oracle, seed):
     for N in (1, 3):
         g = gpu_replay(prof, tr, n_gpus=N)
         compare(g, oracle_replay(oracle, prof, tr, n_gpus=N), 3)
+
+
+@pytest.mark.parametrize("k", [1, 2, 3, 7, 16])
+def test_ctas_per_replica_identical(oracle, k):
+    """Virtual ranks (several CTAs per replica, each scoring a geometry range, min-loc keys
+    exchanged in device memory every epoch) reproduce the oracle for every split, incl. off (1);
+    the 37-set and two replicas per launch."""
+    prof = synth_profiles().with_geometry_set(1 if k >= 7 else 0)
+    tr = tick_trace(mix_b_params(2, seed=8, seconds=12))
+    cfg = dict(n_gpus=8, ctas_per_replica=k)
+    g = gpu_replay(prof, tr, **cfg)
+    o = oracle_replay(oracle, prof, tr, n_gpus=8)
+    compare(g, o, tr.n_replicas)
