@@ -793,6 +793,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   P.geom_lo = vr_n > 1 ? 0 : geom_lo;
   P.geom_hi = vr_n > 1 ? h->G : geom_hi;
   P.vr_n = vr_n;
+  P.few = R < h->nsm;
   if (vr_n > 1) {
     for (int k = 0; k < vr_n; ++k) {
       P.vr_lo[k] = h->vr_b[k];

@@ -417,6 +417,7 @@ struct SliceLane {        // per-lane constants of one placement unit
   int s, p, Z;
 };
 
+template <int kPL>
 __device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, const SliceLane& K,
                                                 const LaneList& L, int& n, int64_t& ls,
                                                 int64_t t, int m, bool strict, int max_live,
@@ -428,20 +429,38 @@ __device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, const
   int64_t fs = 0;
   bool fut = false;
   if (active) {
+    // residents in groups of kPL: the group's loads are issued together (the compaction only
+    // writes indices below the group, so no store can clobber an element not yet loaded)
+    // kPL = 1 for the many-replica launch (its lists are short, and a wider group costs it
+    // registers: measured 181 -> 191 ms); 4 for few-replica launches of long-list workloads
+    // (Mix-B-shaped 1 h replay: 485 -> 418 ms per 600 s)
     int k = 0;
 #pragma unroll 1
-    for (int i = 0; i < n; ++i) {
-      const int64_t ei = L.E(i);
-      if (ei <= t) continue;  // ended: can never matter again (stable compaction)
-      const int64_t si = L.S(i);
-      const uint32_t mi = L.M(i);
-      if (k != i) L.put(k, si, ei, mi);
-      ++k;
-      if (!((mi >> 22) & 1)) be += mi & 0xFFFF;
-      if (ei > t0) {
-        used += mi & 0xFFFF;
-        fs += fbr_p[((mi >> 16) & 63) * kNProf];
-        fut |= si > t0;
+    for (int i0 = 0; i0 < n; i0 += kPL) {
+      int64_t e_[kPL], s_[kPL];
+      uint32_t m_[kPL];
+#pragma unroll
+      for (int u = 0; u < kPL; ++u) {
+        const int i = i0 + u < n ? i0 + u : i0;
+        e_[u] = L.E(i);
+        s_[u] = L.S(i);
+        m_[u] = L.M(i);
+      }
+#pragma unroll
+      for (int u = 0; u < kPL; ++u) {
+        const int i = i0 + u;
+        const int64_t ei = e_[u];
+        if (i >= n || ei <= t) continue;  // ended: can never matter again (stable compaction)
+        const int64_t si = s_[u];
+        const uint32_t mi = m_[u];
+        if (k != i) L.put(k, si, ei, mi);
+        ++k;
+        if (!((mi >> 22) & 1)) be += mi & 0xFFFF;
+        if (ei > t0) {
+          used += mi & 0xFFFF;
+          fs += fbr_p[((mi >> 16) & 63) * kNProf];
+          fut |= si > t0;
+        }
       }
     }
     n = k;
@@ -625,7 +644,7 @@ __device__ __forceinline__ int alg2_final_geometry(const ReplayParams& P, const 
 
 // kAlg2: the policy-2 instance (N1).  A separate instance keeps Alg 2's code out of the search
 // kernel's register allocation (measured: a shared instance costs the search path 1.5%).
-template <bool kAlg2, bool kN3>
+template <bool kAlg2, bool kN3, int kPL>
 __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kernel(ReplayParams P) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ CtaState cs;
@@ -1298,7 +1317,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
             }
           }
           int64_t st, en;
-          const SliceOut so = place_group(T, active && has, K, L, n, ls, t, m, strict,
+          const SliceOut so = place_group<kPL>(T, active && has, K, L, n, ls, t, m, strict,
                                           P.max_live, &st, &en);
           const bool placed = !so.drop_overflow && so.kmin != ~0ull;
           const int wl = (gbase + (int)(so.kmin & 7)) & 31;
@@ -1407,7 +1426,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
                 atomicAdd(&cs.cnt[9], (unsigned long long)(cs.ghi - cs.glo));
               } else {  // policy 2: Alg 2's own heuristic (N1)
                 if constexpr (kAlg2) best = alg2_final_geometry(P, c, g, c.bats, c.gl);
-                else best = cur;  // unreachable: policy 2 launches replay_kernel<true, *>
+                else best = cur;  // unreachable: policy 2 launches replay_kernel<true, *, *>
               }
               dec_out = (uint8_t)best;
               c.gu8[6 * c.N + g] = (uint8_t)best;
@@ -1494,7 +1513,7 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
             atomicAdd(&cs.cnt[9], (unsigned long long)(cs.ghi - cs.glo));
           } else {  // policy 2: Alg 2's own heuristic (N1)
             if constexpr (kAlg2) best = alg2_final_geometry(P, c, g, c.bats, c.gl);
-            else best = cur;  // unreachable: policy 2 launches replay_kernel<true, *>
+            else best = cur;  // unreachable: policy 2 launches replay_kernel<true, *, *>
           }
           dec_out = (uint8_t)best;
           c.gu8[6 * c.N + g] = (uint8_t)best;
@@ -1692,8 +1711,9 @@ static cudaError_t raise_dyn_smem_once() {
   int optin = 0;
   e = cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
   if (e != cudaSuccess) return e;
-  for (auto k : {replay_kernel<false, false>, replay_kernel<true, false>, replay_kernel<false, true>,
-                 replay_kernel<true, true>}) {
+  for (auto k : {replay_kernel<false, false, 1>, replay_kernel<true, false, 1>, replay_kernel<false, true, 1>,
+                 replay_kernel<true, true, 1>, replay_kernel<false, false, 4>, replay_kernel<true, false, 4>,
+                 replay_kernel<false, true, 4>, replay_kernel<true, true, 4>}) {
     cudaFuncAttributes a;
     e = cudaFuncGetAttributes(&a, k);
     if (e != cudaSuccess) return e;
@@ -1707,8 +1727,9 @@ static cudaError_t raise_dyn_smem_once() {
 cudaError_t preload_kernels() {
   cudaFuncAttributes a;
   cudaError_t e = cudaSuccess;
-  for (auto k : {replay_kernel<false, false>, replay_kernel<true, false>, replay_kernel<false, true>,
-                 replay_kernel<true, true>})
+  for (auto k : {replay_kernel<false, false, 1>, replay_kernel<true, false, 1>, replay_kernel<false, true, 1>,
+                 replay_kernel<true, true, 1>, replay_kernel<false, false, 4>, replay_kernel<true, false, 4>,
+                 replay_kernel<false, true, 4>, replay_kernel<true, true, 4>})
     if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, k);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, prepass_kernel);
   if (e == cudaSuccess) e = preload_partition_kernels();
@@ -1720,13 +1741,16 @@ cudaError_t launch_replay(const ReplayParams& P, int grid, int block, cudaStream
   cudaError_t e = raise_dyn_smem_once();
   if (e != cudaSuccess) return e;
   const bool n3 = P.cold_us > 0;  // cold_us = 0: warm containers, no pool work (reading Q15)
+  const bool wide = P.few;        // few replicas: long-list workloads get the 4-wide prune
+  void (*k)(ReplayParams) = nullptr;
   if (P.policy == 2) {
-    if (n3) replay_kernel<true, true><<<grid, block, P.sl.total, st>>>(P);
-    else replay_kernel<true, false><<<grid, block, P.sl.total, st>>>(P);
+    if (n3) k = wide ? replay_kernel<true, true, 4> : replay_kernel<true, true, 1>;
+    else k = wide ? replay_kernel<true, false, 4> : replay_kernel<true, false, 1>;
   } else {
-    if (n3) replay_kernel<false, true><<<grid, block, P.sl.total, st>>>(P);
-    else replay_kernel<false, false><<<grid, block, P.sl.total, st>>>(P);
+    if (n3) k = wide ? replay_kernel<false, true, 4> : replay_kernel<false, true, 1>;
+    else k = wide ? replay_kernel<false, false, 4> : replay_kernel<false, false, 1>;
   }
+  k<<<grid, block, P.sl.total, st>>>(P);
   return cudaGetLastError();
 }
 
@@ -1735,8 +1759,9 @@ cudaError_t replay_occupancy(int block, size_t smem, int* blocks_per_sm) {
   cudaError_t e = raise_dyn_smem_once();
   if (e != cudaSuccess) return e;
   int lo = 1 << 30;
-  for (auto k : {replay_kernel<false, false>, replay_kernel<true, false>, replay_kernel<false, true>,
-                 replay_kernel<true, true>}) {
+  for (auto k : {replay_kernel<false, false, 1>, replay_kernel<true, false, 1>, replay_kernel<false, true, 1>,
+                 replay_kernel<true, true, 1>, replay_kernel<false, false, 4>, replay_kernel<true, false, 4>,
+                 replay_kernel<false, true, 4>, replay_kernel<true, true, 4>}) {
     int a = 0;
     if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, k, block, smem);
     lo = a < lo ? a : lo;

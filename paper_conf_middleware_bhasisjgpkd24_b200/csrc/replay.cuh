@@ -131,6 +131,7 @@ struct ReplayParams {
   uint64_t xtimeout_ns;    // a source flag not seen within this time fails the call (ENCCL)
   // virtual ranks (vr_n > 1): CTA b serves replica b / vr_n, geometry range b % vr_n
   int vr_n;
+  bool few;                // fewer replicas than SMs (the long-list kernel instances)
   int vr_lo[kMaxVR], vr_hi[kMaxVR], vr_cw[kMaxVR];
   const uint32_t* vr_pack[kMaxVR];
 };

@@ -6,6 +6,11 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
+import paper_conf_middleware_bhasisjgpkd24_b200._abi as A  # noqa: E402
+
+if os.environ.get("PROTEAN_LIB"):  # a library variant (experiments)
+    A._lib = None
+    A.load(os.path.abspath(os.environ["PROTEAN_LIB"]))
 import paper_conf_middleware_bhasisjgpkd24_b200 as pkg  # noqa: E402
 from protean_inputs import mix_b_params, synth_profiles, tick_trace  # noqa: E402
 
