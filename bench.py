@@ -296,14 +296,19 @@ def run_ours(args):
         alg_bytes = 4.0 * n_req
         achieved = alg_bytes / (k_ms / 1e3) / 1e9
         part_bytes = 10.0 * n_req
-        traffic = None
+        traffic, issue = None, None
         prof_path = os.path.join(ROOT, "profiles", "ncu_summary.json")
         if os.path.exists(prof_path):
             try:
                 ps = json.load(open(prof_path))
                 traffic = ps["dram_bytes_per_request"] * n_req
+                # the kernel is bound by instruction issue, not HBM: the committed ncu
+                # capture's issue-slot utilisation is the other half of the picture
+                issue = {"issue_slots_busy_pct": ps.get("issue_active_pct"),
+                         "warp_instructions_per_request": ps["warp_instructions"] / ps["requests"],
+                         "source": ps.get("report")}
             except Exception:
-                traffic = None
+                traffic, issue = None, None
         line = {
             "metric": metric, "value": value, "unit": unit, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
@@ -320,7 +325,7 @@ def run_ours(args):
             "geom_candidates_per_s": geom_c * args.steps / sec,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
-                         "kernel": "replay_kernel", "kernel_ms": k_ms, "launch": launch,
+                         "kernel": "replay_kernel", "kernel_ms": k_ms, "launch": launch, "issue": issue,
                          "algorithmic_bytes_per_request": 4.0,
                          "partition": {"ms": p_ms, "algorithmic_bytes_per_request": 10.0,
                                        "achieved_GBps": part_bytes / (p_ms / 1e3) / 1e9,
