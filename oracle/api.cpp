@@ -549,4 +549,89 @@ int orc_sweep(const orc_tables* t, int32_t R, int32_t N, int32_t max_live, int32
   return ORC_OK;
 }
 
+int orc_form_dispatch(const orc_tables* t, int32_t R, int32_t N, int64_t W, int64_t trace_len,
+                     const uint32_t* arrival, const uint8_t* meta, const int64_t* replica_off,
+                     int32_t e_lo, int32_t e_hi, const int64_t* avail, uint32_t* b_ready,
+                     uint32_t* b_req_off, int32_t* b_n, int32_t* b_model, int32_t* b_strict,
+                     int32_t* b_gpu, int32_t* batch_off, int64_t* n_rows, uint32_t* members,
+                     int64_t members_cap) {
+  Tables tb;
+  int rc = build_tables(t, &tb);
+  if (rc) return rc;
+  if (R < 1 || N < 1 || W <= 0 || trace_len <= 0 || !n_rows || !batch_off) return ORC_EINVAL;
+  if (N > 255) return ORC_ERANGE;
+  const int64_t E = num_epochs(tb, trace_len, W);
+  if (e_lo < 0 || e_hi > E || e_lo > e_hi) return ORC_EINVAL;
+  if (!arrival || !meta || !replica_off || replica_off[0] != 0) return ORC_EINVAL;
+  for (int r = 0; r < R; ++r) {
+    if (replica_off[r + 1] < replica_off[r]) return ORC_EINVAL;
+    for (int64_t i = replica_off[r]; i < replica_off[r + 1]; ++i) {
+      if (i > replica_off[r] && arrival[i] < arrival[i - 1]) return ORC_EINVAL;
+      if ((int64_t)arrival[i] >= trace_len) return ORC_EINVAL;
+      if ((meta[i] & 63) >= tb.M || (meta[i] & 0x40)) return ORC_EINVAL;
+    }
+  }
+  if (trace_len - 1 + [&] { int64_t m = 0; for (int q = 0; q < tb.M; ++q) m = std::max<int64_t>(m, tb.tmo[q]); return m; }() >
+      (int64_t)0xFFFFFFFFLL)
+    return ORC_ERANGE;
+  const int Ew = e_hi - e_lo;
+  // per replica: batches in id order (O3), then dispatch from epoch 0 (O5.2, reading Q18)
+  struct Row { int e, gpu; const Batch* b; };
+  std::vector<std::vector<Batch>> all(R);
+  std::vector<std::vector<Row>> rows(R);
+  for (int r = 0; r < R; ++r) {
+    const int64_t off = replica_off[r];
+    all[r] = form_batches(tb, arrival + off, meta + off, replica_off[r + 1] - off);
+    int cursor = 0;
+    for (const Batch& b : all[r]) {
+      const int64_t e = b.ready / W;  // half-open epochs (Q31)
+      if (e >= e_hi) break;
+      int chosen = -1;
+      for (int i = 0; i < N; ++i) {
+        const int n = (cursor + i) % N;
+        const bool ok = !avail || (avail[((int64_t)r * N + n) * 2] <= b.ready &&
+                                   b.ready < avail[((int64_t)r * N + n) * 2 + 1]);
+        if (ok) { chosen = n; break; }
+      }
+      if (chosen < 0) continue;  // dispatch drop: not emitted
+      cursor = (chosen + 1) % N;
+      if (e >= e_lo) rows[r].push_back({(int)(e - e_lo), chosen, &b});
+    }
+    std::stable_sort(rows[r].begin(), rows[r].end(), [](const Row& a, const Row& b) {
+      return a.e != b.e ? a.e < b.e : a.gpu < b.gpu;  // (epoch, gpu), id order kept within
+    });
+  }
+  int64_t total = 0, nmem = 0;
+  for (int r = 0; r < R; ++r) {
+    total += (int64_t)rows[r].size();
+    for (const Row& w : rows[r]) nmem += w.b->n;
+  }
+  const int64_t cap = *n_rows;
+  *n_rows = total;
+  if (total > cap || nmem > members_cap) return ORC_ERANGE;
+  int64_t x = 0, m = 0;
+  batch_off[0] = 0;
+  for (int r = 0; r < R; ++r) {
+    size_t k = 0;
+    for (int e = 0; e < Ew; ++e) {
+      for (int g = 0; g < N; ++g) {
+        while (k < rows[r].size() && rows[r][k].e == e && rows[r][k].gpu == g) {
+          const Batch& b = *rows[r][k].b;
+          b_ready[x] = (uint32_t)b.ready;
+          b_req_off[x] = (uint32_t)m;
+          b_n[x] = b.n;
+          b_model[x] = b.model;
+          b_strict[x] = b.strict ? 1 : 0;
+          b_gpu[x] = g;
+          for (uint32_t a : b.arr) members[m++] = a;
+          ++x;
+          ++k;
+        }
+        batch_off[((int64_t)r * Ew + e) * N + g + 1] = (int32_t)x;
+      }
+    }
+  }
+  return ORC_OK;
+}
+
 }  // extern "C"

@@ -109,6 +109,18 @@ int orc_score_epoch(const orc_tables *t, int32_t R, int32_t N, int32_t epoch, in
                     int64_t *p_start, int64_t *p_end, int32_t *p_slice, int32_t *p_dropped,
                     int64_t *counters, int64_t *accum);
 
+/* O3 batch formation + O5.2 round-robin dispatch for epochs [e_lo, e_hi) (the form_batches
+ * helper of SURVEY §8(b)): rows ordered by (replica, epoch, gpu, batch id), batch_off CSR over
+ * (replica, epoch - e_lo, gpu); avail [R][N][2] {from, until} or NULL (always available); dispatch
+ * drops are not emitted.  members: every row's member arrivals, contiguous and ascending, at
+ * req_off.  *n_rows: capacity in, rows out (ERANGE if too small, *n_rows = rows needed). */
+int orc_form_dispatch(const orc_tables *t, int32_t R, int32_t N, int64_t W, int64_t trace_len,
+                     const uint32_t *arrival, const uint8_t *meta, const int64_t *replica_off,
+                     int32_t e_lo, int32_t e_hi, const int64_t *avail, uint32_t *b_ready,
+                     uint32_t *b_req_off, int32_t *b_n, int32_t *b_model, int32_t *b_strict,
+                     int32_t *b_gpu, int32_t *batch_off, int64_t *n_rows, uint32_t *members,
+                     int64_t members_cap);
+
 /* N4a exhaustive assignment sweep (readings R18-R21): per (replica, gpu) and geometry j in
  * [geom_lo, geom_hi) the min key over every assignment of the GPU's batches (<= max_batches <= 8)
  * to j's slices, scheduled from idle with the slice forced; assign = slice of batch x in bits

@@ -116,6 +116,8 @@ def lib():
         L.orc_replay.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p]
         L.orc_score_epoch.argtypes = ([C.c_void_p] + [C.c_int32] * 4 + [C.c_int64] * 2 +
                                       [C.c_void_p] * 8 + [C.c_int32] * 2 + [C.c_void_p] * 8)
+        L.orc_form_dispatch.argtypes = ([C.c_void_p, C.c_int32, C.c_int32, C.c_int64, C.c_int64] + [C.c_void_p] * 3 +
+                                       [C.c_int32, C.c_int32] + [C.c_void_p] * 10 + [C.c_int64])
         L.orc_sweep.argtypes = ([C.c_void_p] + [C.c_int32] * 4 + [C.c_void_p] * 8 + [C.c_int32] * 2 +
                                 [C.c_void_p] * 4)
         _lib = L
@@ -366,3 +368,31 @@ def sweep(prof, *, R, N, batches, batch_off, arrival, cur_geom, geom_lo=0, geom_
         raise OracleError(rc)
     out["n_assign"] = int(out["n_assign"][0])
     return out
+
+
+def form_dispatch(prof, trace, *, N, e_lo, e_hi, avail=None, W=1_000_000):
+    """O3 + O5.2 for epochs [e_lo, e_hi) (orc_form_dispatch); rows as a dict of arrays."""
+    T = OTables(prof)
+    R = trace.n_replicas
+    arr = np.ascontiguousarray(trace.arrival_us, np.uint32)
+    meta = np.ascontiguousarray(trace.meta, np.uint8)
+    off = np.ascontiguousarray(trace.replica_off, np.int64)
+    if arr.shape[0] == 0:
+        arr, meta = np.zeros(1, np.uint32), np.zeros(1, np.uint8)
+    cap = max(1, int(arr.shape[0]))
+    out = dict(ready=np.zeros(cap, np.uint32), req_off=np.zeros(cap, np.uint32), n=np.zeros(cap, np.int32),
+               model=np.zeros(cap, np.int32), strict=np.zeros(cap, np.int32), gpu=np.zeros(cap, np.int32))
+    boff = np.zeros(R * (e_hi - e_lo) * N + 1, np.int32)
+    members = np.zeros(cap, np.uint32)
+    nrows = np.array([cap], np.int64)
+    av = None if avail is None else np.ascontiguousarray(avail, np.int64)
+    rc = lib().orc_form_dispatch(T.ref, R, N, W, int(trace.trace_len_us), _p(arr), _p(meta), _p(off), e_lo, e_hi,
+                                _p(av), _p(out["ready"]), _p(out["req_off"]), _p(out["n"]), _p(out["model"]),
+                                _p(out["strict"]), _p(out["gpu"]), _p(boff), _p(nrows), _p(members), cap)
+    if rc:
+        raise OracleError(rc)
+    k = int(nrows[0])
+    res = {kk: v[:k] for kk, v in out.items()}
+    res["batch_off"] = boff
+    res["members"] = members
+    return res
