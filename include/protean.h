@@ -285,6 +285,29 @@ int protean_last_timings(const protean_handle *h, float *prepass_ms, float *repl
 void protean_replay_cfg_defaults(protean_replay_cfg *cfg);
 
 /* ---------------------------------------------------------------------------------------------
+ * 3a. Batch formation + dispatch helper (SURVEY §8(b) protean_form_batches) for callers of
+ *     protean_score_epoch: O3 batch formation (a batch of model m closes at B_m requests or at its
+ *     first arrival + T_m, reading Q14) and O5.2 batch-level round-robin dispatch over the
+ *     sim-GPUs available at the batch's ready time (reading Q18; cursor from epoch 0) for
+ *     epochs [e_lo, e_hi) (a batch belongs to epoch ready / W, Q31).  Uses n_replicas, n_gpus,
+ *     trace_len_us, epoch_len_us, arrival_us, meta, replica_off of cfg (device); the trace is
+ *     validated as by protean_replay_traces.
+ *       avail_windows  device int64 [R][N][2] {from, until}: GPU n is available at t iff
+ *                      from <= t < until; NULL = always available.  Dispatch drops are not emitted.
+ *       batches        device, *n_batches rows of capacity; rows ordered by (replica, epoch, gpu,
+ *                      batch id); gpu = the sim-GPU; req_off indexes `members`
+ *       batch_off      device int32 [R * (e_hi - e_lo) * N + 1] CSR over (replica, epoch - e_lo, gpu)
+ *       n_batches      host: capacity in, rows out (PROTEAN_ERANGE if too small; *n_batches then
+ *                      holds the rows needed)
+ *       members        device uint32, members_cap >= requests + 4 per replica: the member arrivals
+ *                      of every batch, contiguous and ascending (a stream-sorted copy of the
+ *                      trace; its layout is otherwise unspecified)
+ *     Synchronous.  Host-side scan between the count and write passes; not a bench path.        */
+int protean_form_batches(protean_handle *h, const protean_replay_cfg *cfg, int32_t e_lo, int32_t e_hi,
+                         const int64_t *avail_windows, protean_batch *batches, int32_t *batch_off,
+                         int64_t *n_batches, uint32_t *members, int64_t members_cap, void *stream);
+
+/* ---------------------------------------------------------------------------------------------
  * 3b. Exhaustive assignment sweep (N4a): the paper's "Oracle" scheme, "ideal GPU configurations
  *     ... obtained through multiple offline ... scheduling sweeps".  For every
  *     (replica, sim-GPU) with b <= max_batches dispatched batches of one epoch and every geometry j

@@ -135,6 +135,8 @@ def load(path: str = LIB_PATH, require_cuda: bool = True):
     L.protean_num_epochs.argtypes = [C.c_void_p, C.c_int64, C.c_int64, C.c_void_p]
     L.protean_score_epoch.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
     L.protean_sweep_assignments.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
+    L.protean_form_batches.argtypes = [C.c_void_p, C.c_void_p, C.c_int32, C.c_int32, C.c_void_p, C.c_void_p,
+                                       C.c_void_p, C.c_void_p, C.c_void_p, C.c_int64, C.c_void_p]
     L.protean_replay_traces.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
     L.protean_replay_cfg_defaults.argtypes = [C.c_void_p]
     L.protean_replay_cfg_defaults.restype = None

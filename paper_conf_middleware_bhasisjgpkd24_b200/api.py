@@ -301,6 +301,39 @@ class Handle:
         out["placement"] = out["placement"][:nb]
         return out
 
+    def form_batches(self, arrival_us, meta, replica_off, *, trace_len_us: int, n_gpus: int, e_lo: int,
+                     e_hi: int, avail=None, epoch_len_us: int = 1_000_000, stream=None):
+        """protean_form_batches on device tensors: rows (uint8 [n, 16] protean_batch), batch_off
+        (int32 CSR over (replica, epoch - e_lo, gpu)) and members (uint32 as int32)."""
+        torch = _torch()
+        dev = torch.device("cuda", self.device)
+        R = int(replica_off.shape[0]) - 1
+        cf = A.ReplayCfg()
+        self._lib.protean_replay_cfg_defaults(C.byref(cf))
+        cf.n_replicas, cf.n_gpus = R, int(n_gpus)
+        cf.trace_len_us, cf.epoch_len_us = int(trace_len_us), int(epoch_len_us)
+        cf.arrival_us = arrival_us.data_ptr() if arrival_us.numel() else replica_off.data_ptr()
+        cf.meta = meta.data_ptr() if meta.numel() else replica_off.data_ptr()
+        cf.replica_off = replica_off.data_ptr()
+        n_req = int(arrival_us.numel())
+        mcap = n_req + 4 * R
+        members = torch.zeros(max(mcap, 1), dtype=torch.int32, device=dev)
+        boff = torch.zeros(R * (e_hi - e_lo) * int(n_gpus) + 1, dtype=torch.int32, device=dev)
+        st = stream if stream is not None else torch.cuda.current_stream(self.device)
+        cap = C.c_int64(0)  # first call sizes the rows
+        rc = self._lib.protean_form_batches(self._h, C.byref(cf), int(e_lo), int(e_hi),
+                                            avail.data_ptr() if avail is not None else None, None,
+                                            boff.data_ptr(), C.byref(cap), members.data_ptr(), mcap,
+                                            C.c_void_p(st.cuda_stream))
+        if rc not in (A.OK, A.ERANGE) or (rc == A.ERANGE and cap.value == 0):
+            _check(self._h, rc)
+        rows = torch.zeros((max(cap.value, 1), 16), dtype=torch.uint8, device=dev)
+        _check(self._h, self._lib.protean_form_batches(self._h, C.byref(cf), int(e_lo), int(e_hi),
+                                                       avail.data_ptr() if avail is not None else None,
+                                                       rows.data_ptr(), boff.data_ptr(), C.byref(cap),
+                                                       members.data_ptr(), mcap, C.c_void_p(st.cuda_stream)))
+        return dict(rows=rows[: cap.value], batch_off=boff, members=members, n=cap.value)
+
     def sweep_assignments(self, *, n_replicas, n_gpus, batches, batch_off, arrival_us, cur_geom,
                           geom_lo=0, geom_hi=None, max_live=64, max_batches=8, want_sweep_keys=True,
                           out=None, stream=None):

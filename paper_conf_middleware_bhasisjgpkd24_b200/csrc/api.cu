@@ -306,6 +306,7 @@ int xchg_finish(protean_handle* h) {
   // replay kernel in this process spins on the exchange
   CK(h, preload_kernels());
   CK(h, preload_sweep_kernel());
+  CK(h, preload_form_kernel());
   CK(h, cudaMalloc(&h->d_xpeer, sizeof(char*) * h->xpeer.size()));
   CK(h, cudaMemcpy(h->d_xpeer, h->xpeer.data(), sizeof(char*) * h->xpeer.size(), cudaMemcpyHostToDevice));
   h->x_ready = true;
@@ -1006,6 +1007,143 @@ int protean_sweep_assignments(protean_handle* h, const protean_sweep_in* in, pro
   CK(h, cudaStreamSynchronize(st));
   if (errs[0]) return fail(h, PROTEAN_EINVAL, "invalid batch / offsets / cur_geom");
   if (errs[1]) return fail(h, PROTEAN_ERANGE, "more than max_batches batches on a GPU");
+  return PROTEAN_OK;
+}
+
+int protean_form_batches(protean_handle* h, const protean_replay_cfg* cfg, int32_t e_lo, int32_t e_hi,
+                         const int64_t* avail_windows, protean_batch* batches, int32_t* batch_off,
+                         int64_t* n_batches, uint32_t* members, int64_t members_cap, void* stream) {
+  if (!h) return PROTEAN_EINVAL;
+  if (h->poisoned) return PROTEAN_ESTATE;
+  if (!cfg || !n_batches || !batch_off || !members) return fail(h, PROTEAN_EINVAL, "null pointer");
+  const protean_replay_cfg& c = *cfg;
+  if (c.n_replicas < 1 || c.n_gpus < 1) return fail(h, PROTEAN_EINVAL, "sizes");
+  if (c.n_gpus > 255) return fail(h, PROTEAN_ERANGE, "n_gpus > 255");
+  if (c.epoch_len_us <= 0 || c.trace_len_us <= 0) return fail(h, PROTEAN_EINVAL, "W / trace_len");
+  if (c.trace_len_us - 1 + h->maxT > (int64_t)0xFFFFFFFFLL)
+    return fail(h, PROTEAN_ERANGE, "ready times exceed uint32 us");
+  if (!c.arrival_us || !c.meta || !c.replica_off) return fail(h, PROTEAN_EINVAL, "null trace");
+  const int64_t W = c.epoch_len_us;
+  const int64_t E = (c.trace_len_us + W - 1) / W + ((int64_t)h->maxT + W - 1) / W;
+  if (e_lo < 0 || e_hi > E || e_lo > e_hi) return fail(h, PROTEAN_EINVAL, "epoch range");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  CK(h, cudaSetDevice(h->device));
+  const int R = c.n_replicas, N = c.n_gpus, S = 2 * h->M, Ew = e_hi - e_lo;
+  std::vector<int64_t> roff(R + 1);
+  CK(h, cudaMemcpyAsync(roff.data(), c.replica_off, sizeof(int64_t) * (R + 1), cudaMemcpyDeviceToHost, st));
+  CK(h, cudaStreamSynchronize(st));
+  if (roff[0] != 0) return fail(h, PROTEAN_EINVAL, "replica_off[0] != 0");
+  for (int r = 0; r < R; ++r)
+    if (roff[r + 1] < roff[r]) return fail(h, PROTEAN_EINVAL, "replica_off not monotone");
+  // the trace-level stream partition of protean_replay_traces (prepass, P1 count + validate, P2
+  // runs, P3 stable scatter): the stream-sorted copy is the members array
+  {
+    void* p = h->d_eoff;
+    int rc = ensure(h, &p, &h->eoff_bytes, sizeof(int64_t) * (size_t)R * (size_t)(E + 1), st);
+    h->d_eoff = static_cast<int64_t*>(p);
+    if (rc) return rc;
+  }
+  unsigned long long* d_wmax = static_cast<unsigned long long*>(h->d_small);
+  int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 64);
+  CK(h, cudaMemsetAsync(h->d_small, 0, 256, st));
+  CK(h, launch_prepass(c.arrival_us, c.replica_off, R, E, W, h->maxT, h->d_eoff, d_wmax, d_err, st));
+  std::vector<int64_t> saoff(R + 1);
+  saoff[0] = 0;
+  for (int r = 0; r < R; ++r) saoff[r + 1] = saoff[r] + ((roff[r + 1] - roff[r] + 3) & ~(int64_t)3);
+  if (members_cap < saoff[R]) return fail(h, PROTEAN_ERANGE, "members capacity < requests + 4 per replica");
+  {
+    int rc = ensure(h, &h->d_cnt, &h->cnt_bytes, std::max<size_t>(4, sizeof(uint32_t) * (size_t)R * E * S), st);
+    if (!rc) rc = ensure(h, &h->d_sidx, &h->sidx_bytes, std::max<size_t>(4, sizeof(uint32_t) * (size_t)R * (E + 1) * S), st);
+    if (!rc) rc = ensure(h, &h->d_sa, &h->sa_bytes, std::max<size_t>(16, sizeof(uint32_t) * (size_t)saoff[R]), st);
+    if (!rc) rc = ensure(h, &h->d_saoff, &h->saoff_bytes, sizeof(int64_t) * (size_t)(R + 1), st);
+    if (rc) return rc;
+  }
+  CK(h, cudaMemcpyAsync(h->d_saoff, saoff.data(), sizeof(int64_t) * (R + 1), cudaMemcpyHostToDevice, st));
+  PartitionArgs PA;
+  PA.arr = c.arrival_us;
+  PA.meta = c.meta;
+  PA.roff = c.replica_off;
+  PA.eoff = h->d_eoff;
+  PA.saoff = static_cast<const int64_t*>(h->d_saoff);
+  PA.R = R;
+  PA.S = S;
+  PA.M = h->M;
+  PA.E = E;
+  PA.tlm1 = (uint32_t)(c.trace_len_us - 1);
+  PA.vec = ((reinterpret_cast<uintptr_t>(c.arrival_us) & 15u) == 0) &&
+           ((reinterpret_cast<uintptr_t>(c.meta) & 15u) == 0);
+  PA.cnt = static_cast<uint32_t*>(h->d_cnt);
+  PA.sidx = static_cast<uint32_t*>(h->d_sidx);
+  PA.sa = static_cast<uint32_t*>(h->d_sa);
+  PA.err = d_err;
+  CK(h, launch_partition_count(PA, st));
+  int herr = 0;
+  CK(h, cudaMemcpyAsync(&herr, d_err, 4, cudaMemcpyDeviceToHost, st));
+  CK(h, cudaStreamSynchronize(st));
+  if (herr) return fail(h, PROTEAN_EINVAL, "arrivals not sorted or beyond the trace");
+  CK(h, launch_partition_rest(PA, st));
+  // pass 0: rows per (replica, epoch, GPU) cell
+  const size_t cells = (size_t)R * Ew * N;
+  void* dc = nullptr;
+  size_t dc_have = 0;
+  {
+    int rc = ensure(h, &dc, &dc_have, std::max<size_t>(4, sizeof(int32_t) * cells), st);
+    if (rc) return rc;
+  }
+  CK(h, cudaMemsetAsync(dc, 0, std::max<size_t>(4, sizeof(int32_t) * cells), st));
+  FormParams F;
+  std::memset(&F, 0, sizeof(F));
+  F.sa = static_cast<const uint32_t*>(h->d_sa);
+  F.saoff = static_cast<const int64_t*>(h->d_saoff);
+  F.sidx = static_cast<const uint32_t*>(h->d_sidx);
+  F.bsz = h->d_tab + h->tl.o_bsz;
+  F.tmo = h->d_tab + h->tl.o_tmo;
+  F.avail = avail_windows;
+  F.R = R;
+  F.N = N;
+  F.S = S;
+  F.e_lo = e_lo;
+  F.e_hi = e_hi;
+  F.E = E;
+  F.W = W;
+  F.cnt = static_cast<int32_t*>(dc);
+  F.pass = 0;
+  CK(h, launch_form(F, st));
+  std::vector<int32_t> cnt(cells);
+  if (cells) CK(h, cudaMemcpyAsync(cnt.data(), dc, sizeof(int32_t) * cells, cudaMemcpyDeviceToHost, st));
+  CK(h, cudaMemcpyAsync(&herr, d_err, 4, cudaMemcpyDeviceToHost, st));
+  CK(h, cudaStreamSynchronize(st));
+  if (herr) {
+    cudaFreeAsync(dc, st);
+    return fail(h, PROTEAN_EINVAL, "invalid request (model id or arrival >= trace_len)");
+  }
+  std::vector<int32_t> off(cells + 1);
+  off[0] = 0;
+  int64_t total = 0;
+  for (size_t i = 0; i < cells; ++i) {
+    total += cnt[i];
+    if (total > INT32_MAX) {
+      cudaFreeAsync(dc, st);
+      return fail(h, PROTEAN_ERANGE, "more than 2^31 rows");
+    }
+    off[i + 1] = (int32_t)total;
+  }
+  const int64_t cap = *n_batches;
+  *n_batches = total;
+  if (total > cap || (total > 0 && !batches)) {
+    cudaFreeAsync(dc, st);
+    return fail(h, PROTEAN_ERANGE, "batches capacity too small (n_batches holds the rows needed)");
+  }
+  CK(h, cudaMemcpyAsync(batch_off, off.data(), sizeof(int32_t) * (cells + 1), cudaMemcpyHostToDevice, st));
+  CK(h, cudaMemsetAsync(dc, 0, std::max<size_t>(4, sizeof(int32_t) * cells), st));
+  // pass 1: the rows, in (replica, epoch, GPU, batch id) order
+  F.pass = 1;
+  F.off = batch_off;
+  F.rows = batches;
+  CK(h, launch_form(F, st));
+  if (saoff[R]) CK(h, cudaMemcpyAsync(members, h->d_sa, sizeof(uint32_t) * (size_t)saoff[R], cudaMemcpyDeviceToDevice, st));
+  CK(h, cudaStreamSynchronize(st));  // off lives on this stack frame
+  cudaFreeAsync(dc, st);
   return PROTEAN_OK;
 }
 

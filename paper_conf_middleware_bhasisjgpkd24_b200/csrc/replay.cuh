@@ -154,6 +154,23 @@ struct ScoreParams {
   int* err;                   // err[0] EINVAL, err[1] ERANGE
 };
 
+// protean_form_batches (form.cu): batch formation + round-robin dispatch on the stream-sorted copy
+struct FormParams {
+  const uint32_t* sa;      // stream-sorted arrivals (partition.cu), replica r at sa + saoff[r]
+  const int64_t* saoff;
+  const uint32_t* sidx;    // [R][E+1][S] stream run starts per epoch (row E = stream ends)
+  const int32_t* bsz;      // [M] batch sizes, [M] timeouts (the staged table)
+  const int32_t* tmo;
+  const int64_t* avail;    // [R][N][2] {from, until} or NULL
+  int R, N, S, e_lo, e_hi, pass;
+  int64_t E, W;
+  int32_t* cnt;            // [R][e_hi - e_lo][N] rows per cell (pass 0) / fill (pass 1, zeroed)
+  const int32_t* off;      // pass 1: first row of every cell (the caller's batch_off)
+  protean_batch* rows;
+};
+cudaError_t launch_form(const FormParams& P, cudaStream_t st);
+cudaError_t preload_form_kernel();
+
 // N4a exhaustive assignment sweep (sweep.cu)
 struct SweepParams {
   const int32_t* tab;
