@@ -316,6 +316,73 @@ int xchg_finish(protean_handle* h) {
 
 }  // namespace
 
+// The trace-level stream partition shared by protean_replay_traces and protean_form_batches
+// (partition.cu): prepass (epoch offsets, largest window, sortedness), P1 count + validate, then
+// P2 run indices and the P3 stable scatter into the stream-sorted copy (h->d_sa at h->d_saoff).
+// Request-level faults found by P3 are left in err[0] for the caller to report after its kernels.
+// timing: record the prepass / partition events read by protean_last_timings.
+int partition_trace(protean_handle* h, const protean_replay_cfg& c, const std::vector<int64_t>& roff,
+                    int64_t E, cudaStream_t st, bool timing, unsigned long long* wmax_out) {
+  const int R = c.n_replicas, S = 2 * h->M;
+  const int64_t W = c.epoch_len_us;
+  {
+    void* p = h->d_eoff;
+    int rc = ensure(h, &p, &h->eoff_bytes, sizeof(int64_t) * (size_t)R * (size_t)(E + 1), st);
+    h->d_eoff = static_cast<int64_t*>(p);
+    if (rc) return rc;
+  }
+  unsigned long long* d_wmax = static_cast<unsigned long long*>(h->d_small);
+  int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 64);
+  CK(h, cudaMemsetAsync(h->d_small, 0, 256, st));
+  if (timing) CK(h, cudaEventRecord(h->ev[0], st));
+  CK(h, launch_prepass(c.arrival_us, c.replica_off, R, E, W, h->maxT, h->d_eoff, d_wmax, d_err, st));
+  std::vector<int64_t> saoff(R + 1);
+  saoff[0] = 0;
+  for (int r = 0; r < R; ++r) saoff[r + 1] = saoff[r] + ((roff[r + 1] - roff[r] + 3) & ~(int64_t)3);
+  {
+    int rc = ensure(h, &h->d_cnt, &h->cnt_bytes, std::max<size_t>(4, sizeof(uint32_t) * (size_t)R * E * S), st);
+    if (!rc) rc = ensure(h, &h->d_sidx, &h->sidx_bytes, std::max<size_t>(4, sizeof(uint32_t) * (size_t)R * (E + 1) * S), st);
+    if (!rc) rc = ensure(h, &h->d_sa, &h->sa_bytes, std::max<size_t>(16, sizeof(uint32_t) * (size_t)saoff[R]), st);
+    if (!rc) rc = ensure(h, &h->d_saoff, &h->saoff_bytes, sizeof(int64_t) * (size_t)(R + 1), st);
+    if (rc) return rc;
+  }
+  CK(h, cudaMemcpyAsync(h->d_saoff, saoff.data(), sizeof(int64_t) * (R + 1), cudaMemcpyHostToDevice, st));
+  PartitionArgs PA;
+  PA.arr = c.arrival_us;
+  PA.meta = c.meta;
+  PA.roff = c.replica_off;
+  PA.eoff = h->d_eoff;
+  PA.saoff = static_cast<const int64_t*>(h->d_saoff);
+  PA.R = R;
+  PA.S = S;
+  PA.M = h->M;
+  PA.E = E;
+  PA.tlm1 = (uint32_t)(c.trace_len_us - 1);  // trace_len - 1 + maxT <= 2^32 - 1 (checked by callers)
+  PA.vec = ((reinterpret_cast<uintptr_t>(c.arrival_us) & 15u) == 0) &&
+           ((reinterpret_cast<uintptr_t>(c.meta) & 15u) == 0);
+  PA.cnt = static_cast<uint32_t*>(h->d_cnt);
+  PA.sidx = static_cast<uint32_t*>(h->d_sidx);
+  PA.sa = static_cast<uint32_t*>(h->d_sa);
+  PA.err = d_err;
+  CK(h, launch_partition_count(PA, st));
+  if (timing) CK(h, cudaEventRecord(h->ev[1], st));
+  unsigned long long wmax = 0;
+  int herr = 0;
+  CK(h, cudaMemcpyAsync(&wmax, d_wmax, 8, cudaMemcpyDeviceToHost, st));
+  CK(h, cudaMemcpyAsync(&herr, d_err, 4, cudaMemcpyDeviceToHost, st));  // also keeps saoff alive
+  CK(h, cudaStreamSynchronize(st));
+  // the prepass guarantees that the epoch ranges tile every replica (else the scatter could leave
+  // it); request-level validation happens in the scatter pass and is reported by the caller
+  if (herr) return fail(h, PROTEAN_EINVAL, "arrivals not sorted or beyond the trace");
+  if (wmax >= (1ull << 25)) return fail(h, PROTEAN_ERANGE, "epoch window >= 2^25 requests");
+  // P2 + P3: run indices and the stable scatter (only on a validated trace)
+  if (timing) CK(h, cudaEventRecord(h->ev[4], st));
+  CK(h, launch_partition_rest(PA, st));
+  if (timing) CK(h, cudaEventRecord(h->ev[5], st));
+  *wmax_out = wmax;
+  return PROTEAN_OK;
+}
+
 extern "C" {
 
 const char* protean_strerror(int code) {
@@ -618,65 +685,16 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   const int64_t E = (c.trace_len_us + W - 1) / W + ((int64_t)h->maxT + W - 1) / W;
   const int64_t H = E * W;
 
-  // prepass: per (replica, epoch) request offsets, largest epoch window
-  const size_t eoff_need = sizeof(int64_t) * (size_t)R * (size_t)(E + 1);
-  {
-    void* p = h->d_eoff;
-    int rc = ensure(h, &p, &h->eoff_bytes, eoff_need, st);
-    h->d_eoff = static_cast<int64_t*>(p);
-    if (rc) return rc;
-  }
-  unsigned long long* d_wmax = static_cast<unsigned long long*>(h->d_small);
-  int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 64);
-  CK(h, cudaMemsetAsync(h->d_small, 0, 256, st));
-  CK(h, cudaEventRecord(h->ev[0], st));
-  CK(h, launch_prepass(c.arrival_us, c.replica_off, R, E, W, h->maxT, h->d_eoff, d_wmax, d_err, st));
+  // the trace-level stream partition: prepass, P1 count + validate, P2 runs, P3 stable scatter
   const int kWarps = PROTEAN_WARPS;  // replay CTA warps (replay.cuh)
-  // stream partition, P1 (count + validate every request)
   const int S = 2 * h->M;
-  std::vector<int64_t> saoff(R + 1);
-  saoff[0] = 0;
-  for (int r = 0; r < R; ++r) saoff[r + 1] = saoff[r] + ((roff[r + 1] - roff[r] + 3) & ~(int64_t)3);
+  unsigned long long wmax = 0;
+  int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 64);
   {
-    int rc = ensure(h, &h->d_cnt, &h->cnt_bytes, std::max<size_t>(4, sizeof(uint32_t) * (size_t)R * E * S), st);
-    if (!rc) rc = ensure(h, &h->d_sidx, &h->sidx_bytes, std::max<size_t>(4, sizeof(uint32_t) * (size_t)R * (E + 1) * S), st);
-    if (!rc) rc = ensure(h, &h->d_sa, &h->sa_bytes, std::max<size_t>(16, sizeof(uint32_t) * (size_t)saoff[R]), st);
-    if (!rc) rc = ensure(h, &h->d_saoff, &h->saoff_bytes, sizeof(int64_t) * (size_t)(R + 1), st);
+    int rc = partition_trace(h, c, roff, E, st, true, &wmax);
     if (rc) return rc;
   }
-  CK(h, cudaMemcpyAsync(h->d_saoff, saoff.data(), sizeof(int64_t) * (R + 1), cudaMemcpyHostToDevice, st));
-  PartitionArgs PA;
-  PA.arr = c.arrival_us;
-  PA.meta = c.meta;
-  PA.roff = c.replica_off;
-  PA.eoff = h->d_eoff;
-  PA.saoff = static_cast<const int64_t*>(h->d_saoff);
-  PA.R = R;
-  PA.S = S;
-  PA.M = h->M;
-  PA.E = E;
-  PA.tlm1 = (uint32_t)(c.trace_len_us - 1);  // trace_len - 1 + maxT <= 2^32 - 1 (checked above)
-  PA.vec = ((reinterpret_cast<uintptr_t>(c.arrival_us) & 15u) == 0) &&
-           ((reinterpret_cast<uintptr_t>(c.meta) & 15u) == 0);
-  PA.cnt = static_cast<uint32_t*>(h->d_cnt);
-  PA.sidx = static_cast<uint32_t*>(h->d_sidx);
-  PA.sa = static_cast<uint32_t*>(h->d_sa);
-  PA.err = d_err;
-  CK(h, launch_partition_count(PA, st));
-  CK(h, cudaEventRecord(h->ev[1], st));
-  unsigned long long wmax = 0;
   int herr = 0;
-  CK(h, cudaMemcpyAsync(&wmax, d_wmax, 8, cudaMemcpyDeviceToHost, st));
-  CK(h, cudaMemcpyAsync(&herr, d_err, 4, cudaMemcpyDeviceToHost, st));
-  CK(h, cudaStreamSynchronize(st));
-  // the prepass guarantees that the epoch ranges tile every replica (else the scatter could leave
-  // it); request-level validation happens in the scatter pass and is reported after the replay
-  if (herr) return fail(h, PROTEAN_EINVAL, "arrivals not sorted or beyond the trace");
-  if (wmax >= (1ull << 25)) return fail(h, PROTEAN_ERANGE, "epoch window >= 2^25 requests");
-  // P2 + P3: run indices and the stable scatter (only on a validated trace)
-  CK(h, cudaEventRecord(h->ev[4], st));
-  CK(h, launch_partition_rest(PA, st));
-  CK(h, cudaEventRecord(h->ev[5], st));
   // window capacity: the largest window (requests in [eW - maxT, (e+1)W)) + per-stream alignment
   const int WCAP = (int)std::max<unsigned long long>(wmax, 1) + 8 * S;
 
@@ -759,9 +777,9 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   P.tl = h->tl;
   P.pack = d_pack;
   P.maxT = h->maxT;
-  P.sa = PA.sa;
-  P.saoff = PA.saoff;
-  P.sidx = PA.sidx;
+  P.sa = static_cast<const uint32_t*>(h->d_sa);
+  P.saoff = static_cast<const int64_t*>(h->d_saoff);
+  P.sidx = static_cast<const uint32_t*>(h->d_sidx);
   P.R = R;
   P.N = N;
   P.base = c.replica_base;
@@ -1035,53 +1053,18 @@ int protean_form_batches(protean_handle* h, const protean_replay_cfg* cfg, int32
   if (roff[0] != 0) return fail(h, PROTEAN_EINVAL, "replica_off[0] != 0");
   for (int r = 0; r < R; ++r)
     if (roff[r + 1] < roff[r]) return fail(h, PROTEAN_EINVAL, "replica_off not monotone");
-  // the trace-level stream partition of protean_replay_traces (prepass, P1 count + validate, P2
-  // runs, P3 stable scatter): the stream-sorted copy is the members array
-  {
-    void* p = h->d_eoff;
-    int rc = ensure(h, &p, &h->eoff_bytes, sizeof(int64_t) * (size_t)R * (size_t)(E + 1), st);
-    h->d_eoff = static_cast<int64_t*>(p);
-    if (rc) return rc;
-  }
-  unsigned long long* d_wmax = static_cast<unsigned long long*>(h->d_small);
+  // the trace-level stream partition of protean_replay_traces: the stream-sorted copy is the
+  // members array
+  int64_t sa_len = 0;
+  for (int r = 0; r < R; ++r) sa_len += (roff[r + 1] - roff[r] + 3) & ~(int64_t)3;
+  if (members_cap < sa_len) return fail(h, PROTEAN_ERANGE, "members capacity < requests + 4 per replica");
   int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 64);
-  CK(h, cudaMemsetAsync(h->d_small, 0, 256, st));
-  CK(h, launch_prepass(c.arrival_us, c.replica_off, R, E, W, h->maxT, h->d_eoff, d_wmax, d_err, st));
-  std::vector<int64_t> saoff(R + 1);
-  saoff[0] = 0;
-  for (int r = 0; r < R; ++r) saoff[r + 1] = saoff[r] + ((roff[r + 1] - roff[r] + 3) & ~(int64_t)3);
-  if (members_cap < saoff[R]) return fail(h, PROTEAN_ERANGE, "members capacity < requests + 4 per replica");
   {
-    int rc = ensure(h, &h->d_cnt, &h->cnt_bytes, std::max<size_t>(4, sizeof(uint32_t) * (size_t)R * E * S), st);
-    if (!rc) rc = ensure(h, &h->d_sidx, &h->sidx_bytes, std::max<size_t>(4, sizeof(uint32_t) * (size_t)R * (E + 1) * S), st);
-    if (!rc) rc = ensure(h, &h->d_sa, &h->sa_bytes, std::max<size_t>(16, sizeof(uint32_t) * (size_t)saoff[R]), st);
-    if (!rc) rc = ensure(h, &h->d_saoff, &h->saoff_bytes, sizeof(int64_t) * (size_t)(R + 1), st);
+    unsigned long long wmax = 0;
+    int rc = partition_trace(h, c, roff, E, st, false, &wmax);
     if (rc) return rc;
   }
-  CK(h, cudaMemcpyAsync(h->d_saoff, saoff.data(), sizeof(int64_t) * (R + 1), cudaMemcpyHostToDevice, st));
-  PartitionArgs PA;
-  PA.arr = c.arrival_us;
-  PA.meta = c.meta;
-  PA.roff = c.replica_off;
-  PA.eoff = h->d_eoff;
-  PA.saoff = static_cast<const int64_t*>(h->d_saoff);
-  PA.R = R;
-  PA.S = S;
-  PA.M = h->M;
-  PA.E = E;
-  PA.tlm1 = (uint32_t)(c.trace_len_us - 1);
-  PA.vec = ((reinterpret_cast<uintptr_t>(c.arrival_us) & 15u) == 0) &&
-           ((reinterpret_cast<uintptr_t>(c.meta) & 15u) == 0);
-  PA.cnt = static_cast<uint32_t*>(h->d_cnt);
-  PA.sidx = static_cast<uint32_t*>(h->d_sidx);
-  PA.sa = static_cast<uint32_t*>(h->d_sa);
-  PA.err = d_err;
-  CK(h, launch_partition_count(PA, st));
   int herr = 0;
-  CK(h, cudaMemcpyAsync(&herr, d_err, 4, cudaMemcpyDeviceToHost, st));
-  CK(h, cudaStreamSynchronize(st));
-  if (herr) return fail(h, PROTEAN_EINVAL, "arrivals not sorted or beyond the trace");
-  CK(h, launch_partition_rest(PA, st));
   // pass 0: rows per (replica, epoch, GPU) cell
   const size_t cells = (size_t)R * Ew * N;
   void* dc = nullptr;
@@ -1141,7 +1124,7 @@ int protean_form_batches(protean_handle* h, const protean_replay_cfg* cfg, int32
   F.off = batch_off;
   F.rows = batches;
   CK(h, launch_form(F, st));
-  if (saoff[R]) CK(h, cudaMemcpyAsync(members, h->d_sa, sizeof(uint32_t) * (size_t)saoff[R], cudaMemcpyDeviceToDevice, st));
+  if (sa_len) CK(h, cudaMemcpyAsync(members, h->d_sa, sizeof(uint32_t) * (size_t)sa_len, cudaMemcpyDeviceToDevice, st));
   CK(h, cudaStreamSynchronize(st));  // off lives on this stack frame
   cudaFreeAsync(dc, st);
   return PROTEAN_OK;

@@ -24,7 +24,7 @@ __global__ void __launch_bounds__(kFormThreads) form_kernel(FormParams P) {
   const uint32_t* sa = P.sa + P.saoff[r];
   const uint32_t* s0 = P.sidx + (size_t)r * (P.E + 1) * S;            // stream starts (epoch 0)
   const uint32_t* s1 = P.sidx + ((size_t)r * (P.E + 1) + P.E) * S;    // stream ends
-  int cur[kMaxStreams], nn[kMaxStreams];
+  int cur[kMaxStreams] = {}, nn[kMaxStreams] = {};
   int64_t rd[kMaxStreams];  // the stream's next batch: ready time (INT64_MAX: exhausted), size
   auto next = [&](int k) {
     const int i = cur[k], end = (int)s1[k];
