@@ -1,16 +1,21 @@
-// replay.cu — the fused B200 epoch engine (sm_100a): one CTA per trace replica, persistent
-// over its E epochs.  Per epoch (O5):
+// replay.cu — the fused B200 epoch engine (sm_100a): one CTA per trace replica (or k CTAs per
+// replica, "virtual ranks", when replicas are fewer than SMs), persistent over its E epochs.  Per
+// epoch (O5):
 //   A  VM events + pending installs (thread per simulated GPU)            O11, O5.3
-//   B  stream partition of the epoch's request window in shared memory   O3
+//   B  the epoch's stream runs TMA-copied (cp.async.bulk) from the        O3
+//      stream-sorted trace copy (partition.cu) into shared memory
 //   C  batch formation, warp per (model, class) stream; id-order ranks   O3
 //   D  round-robin dispatch (closed form when every GPU is available)    Q18
 //   E  placement units, lane per MIG slice: a lane group = one geometry  O6 + O8 (Alg 1, Eq 1/2,
 //      (actual state, or a candidate replayed from idle); group shuffles  the "Oracle" P:L485)
-//      give BE memory, live count and the min-loc of the slice keys
-//   F  per-request accounting: SLO hits, run-length histogram updates    O7
-//   G  argmin + Alg 2 hysteresis + ~30% cap                              O9, O10
-// The request stream (5 B/request) is read from HBM once with coalesced loads (a second, L2-hot
-// read scatters it); everything else lives in shared memory, registers and L1-resident scratch.
+//      give BE memory, live count and the min-loc of the slice keys;
+//      N3 container pools ahead of each actual placement                 R22-R27
+//   F  per-request accounting: SLO hits, log-linear histogram updates    O7
+//   G  argmin (or Alg 2's heuristic, policy 2) + hysteresis + ~30% cap   O9, O10
+//      with the mode-G / virtual-rank min-loc exchange when ranks > 1    S8
+// The caller's trace (5 B/request) is read from HBM once by the partition passes and the
+// stream-sorted copy (4 B/request) once by this kernel; everything else lives in shared memory,
+// registers and L1-resident scratch.
 #include <cuda_runtime.h>
 #include <mutex>
 
