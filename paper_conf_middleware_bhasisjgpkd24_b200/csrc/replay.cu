@@ -29,6 +29,9 @@
 #ifndef PROTEAN_WARP_G
 #define PROTEAN_WARP_G 1
 #endif
+#ifndef PROTEAN_FEW_AG
+#define PROTEAN_FEW_AG 1  // GPUs per actual-placement warp in the few-replica instances
+#endif
 #ifndef PROTEAN_MINB
 #define PROTEAN_MINB 3
 #endif
@@ -736,7 +739,10 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
   int sum_slots = 0;  // slot-evals per batch per decidable GPU
 #pragma unroll 1
   for (int j = glo; j < ghi; ++j) sum_slots += T.gn[j];
-  const int n_aunits = (N + kAG - 1) / kAG;  // actual-placement warp units: kAG GPUs x 8 slice lanes
+  // actual-placement warp units: AG GPUs x 8 slice lanes.  Few-replica launches (long lists, slow
+  // paths common) give each GPU its own warp, so one GPU's slow path never serialises another's
+  constexpr int AG = kPL == 4 ? PROTEAN_FEW_AG : kAG;
+  const int n_aunits = (N + AG - 1) / AG;
   const uint32_t* sarr = c.sarr;
 
 #pragma unroll 1
@@ -1234,11 +1240,11 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
         int g, s, Z, gbase, j;
         bool valid;
         if (actual) {
-          g = u * kAG + (lane >> 3);
+          g = u * AG + (lane >> 3);
           s = lane & 7;
           Z = kZA;
           gbase = lane & ~7;
-          valid = (lane >> 3) < kAG && g < N;
+          valid = (lane >> 3) < AG && g < N;
           j = valid ? c.gu8[0 * c.N + g] : 0;
         } else {
           const int cw = cs.cw;
