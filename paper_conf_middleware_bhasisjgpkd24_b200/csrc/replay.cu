@@ -741,7 +741,8 @@ __global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kerne
   for (int j = glo; j < ghi; ++j) sum_slots += T.gn[j];
   // actual-placement warp units: AG GPUs x 8 slice lanes.  Few-replica launches (long lists, slow
   // paths common) give each GPU its own warp, so one GPU's slow path never serialises another's
-  constexpr int AG = kPL == 4 ? PROTEAN_FEW_AG : kAG;
+  // (up to 16 sim-GPUs; beyond, 64-GPU configs keep 4 per warp: more units than warps cost more)
+  const int AG = (kPL == 4 && N <= 16) ? PROTEAN_FEW_AG : kAG;
   const int n_aunits = (N + AG - 1) / AG;
   const uint32_t* sarr = c.sarr;
 
