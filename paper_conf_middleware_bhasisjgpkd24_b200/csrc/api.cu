@@ -748,7 +748,10 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   // most evenly (prefer more warps on ties)
   const int n_units = (N + kAG - 1) / kAG + (c.policy == 0 ? N * CW : 0);
   (void)n_units;
-  const int block = 32 * kWarps;  // measured on B200: 8 warps x 3 CTAs/SM beat 6 x 4
+  // measured on B200: 8 warps x 3 CTAs/SM beat 6 x 4 for many replicas; with fewer replicas than
+  // SMs one 16-warp CTA per SM runs a replica's actual and candidate chains side by side
+  const bool few_r = (int64_t)R < (int64_t)h->nsm;
+  const int block = 32 * (few_r ? PROTEAN_FEW_WARPS : kWarps);
   SmemLayout sl;
   sl.init(h->tl.words, h->M, N, Gc, CW, 0, 0);
   const size_t fixed = sl.total;
@@ -765,7 +768,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   sl.init(h->tl.words, h->M, N, Gc, CW, BS, WS);
   if (sl.total > 227 * 1024) return fail(h, PROTEAN_ERANGE, "shared memory layout too large");
   int per_sm = 0;
-  CK(h, replay_occupancy(block, sl.total, &per_sm));
+  CK(h, replay_occupancy(block, sl.total, few_r, &per_sm));
   if (per_sm < 1) return fail(h, PROTEAN_ERANGE, "replay kernel does not fit an SM");
   int grid = (int)std::min<int64_t>((int64_t)R * vr_n, (int64_t)h->nsm * per_sm);
   grid -= grid % vr_n;  // every replica's CTAs are resident together (exchange partners)
@@ -812,7 +815,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   P.geom_lo = vr_n > 1 ? 0 : geom_lo;
   P.geom_hi = vr_n > 1 ? h->G : geom_hi;
   P.vr_n = vr_n;
-  P.few = R < h->nsm;
+  P.few = few_r;
   if (vr_n > 1) {
     for (int k = 0; k < vr_n; ++k) {
       P.vr_lo[k] = h->vr_b[k];

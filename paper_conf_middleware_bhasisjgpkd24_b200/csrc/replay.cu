@@ -29,6 +29,9 @@
 #ifndef PROTEAN_WARP_G
 #define PROTEAN_WARP_G 1
 #endif
+#ifndef PROTEAN_FEW_WARPS
+#define PROTEAN_FEW_WARPS 16  // warps per CTA in the few-replica instances
+#endif
 #ifndef PROTEAN_FEW_AG
 #define PROTEAN_FEW_AG 1  // GPUs per actual-placement warp in the few-replica instances
 #endif
@@ -652,8 +655,11 @@ __device__ __forceinline__ int alg2_final_geometry(const ReplayParams& P, const 
 
 // kAlg2: the policy-2 instance (N1).  A separate instance keeps Alg 2's code out of the search
 // kernel's register allocation (measured: a shared instance costs the search path 1.5%).
+// kPL = 4 marks the few-replica instances: 16 warps, one CTA per SM (actual-placement chains and
+// candidate chains of a replica run side by side); kPL = 1: 8 warps, 3 CTAs per SM.
 template <bool kAlg2, bool kN3, int kPL>
-__global__ void __launch_bounds__(32 * PROTEAN_WARPS, PROTEAN_MINB) replay_kernel(ReplayParams P) {
+__global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTEAN_WARPS,
+                                  kPL == 4 ? 1 : PROTEAN_MINB) replay_kernel(ReplayParams P) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ CtaState cs;
   __shared__ uint32_t s_hist[2 * kNB];  // 2 classes x 3328 buckets (u32 < 2^32 per replica)
@@ -1766,17 +1772,25 @@ cudaError_t launch_replay(const ReplayParams& P, int grid, int block, cudaStream
   return cudaGetLastError();
 }
 
-// Both instances share the launch shape (same registers cap, same static shared memory).
-cudaError_t replay_occupancy(int block, size_t smem, int* blocks_per_sm) {
+// Occupancy of the instances a launch of this shape would use (few: the kPL = 4 instances).
+cudaError_t replay_occupancy(int block, size_t smem, bool few, int* blocks_per_sm) {
   cudaError_t e = raise_dyn_smem_once();
   if (e != cudaSuccess) return e;
   int lo = 1 << 30;
-  for (auto k : {replay_kernel<false, false, 1>, replay_kernel<true, false, 1>, replay_kernel<false, true, 1>,
-                 replay_kernel<true, true, 1>, replay_kernel<false, false, 4>, replay_kernel<true, false, 4>,
-                 replay_kernel<false, true, 4>, replay_kernel<true, true, 4>}) {
-    int a = 0;
-    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, k, block, smem);
-    lo = a < lo ? a : lo;
+  if (few) {
+    for (auto k : {replay_kernel<false, false, 4>, replay_kernel<true, false, 4>, replay_kernel<false, true, 4>,
+                   replay_kernel<true, true, 4>}) {
+      int a = 0;
+      if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, k, block, smem);
+      lo = a < lo ? a : lo;
+    }
+  } else {
+    for (auto k : {replay_kernel<false, false, 1>, replay_kernel<true, false, 1>, replay_kernel<false, true, 1>,
+                   replay_kernel<true, true, 1>}) {
+      int a = 0;
+      if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, k, block, smem);
+      lo = a < lo ? a : lo;
+    }
   }
   *blocks_per_sm = lo;
   return e;

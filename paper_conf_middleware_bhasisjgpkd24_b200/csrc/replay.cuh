@@ -15,7 +15,10 @@ __device__ __forceinline__ void inc_shared(uint32_t saddr) {
 }
 
 #ifndef PROTEAN_WARPS
-#define PROTEAN_WARPS 8  // warps per replay CTA
+#define PROTEAN_WARPS 8  // warps per replay CTA (many-replica launches)
+#endif
+#ifndef PROTEAN_FEW_WARPS
+#define PROTEAN_FEW_WARPS 16  // warps per replay CTA when replicas are fewer than SMs
 #endif
 constexpr int kNSeg = PROTEAN_WARPS;  // warps per CTA (stream-partition segments)
 constexpr int kZA = 8;            // lanes per actual-placement group (one per slice position)
@@ -214,7 +217,7 @@ cudaError_t launch_prepass(const uint32_t* arr, const int64_t* roff, int R, int6
                            int64_t maxT, int64_t* eoff, unsigned long long* wmax, int* err,
                            cudaStream_t st);
 cudaError_t launch_replay(const ReplayParams& P, int grid, int block, cudaStream_t st);
-cudaError_t replay_occupancy(int block, size_t smem, int* blocks_per_sm);
+cudaError_t replay_occupancy(int block, size_t smem, bool few, int* blocks_per_sm);
 cudaError_t preload_kernels();
 cudaError_t launch_score(const ScoreParams& P, int block, cudaStream_t st);
 size_t score_smem_bytes(const TabLayout& tl, int N, int Gc);
