@@ -750,7 +750,9 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   (void)n_units;
   // measured on B200: 8 warps x 3 CTAs/SM beat 6 x 4 for many replicas; with fewer replicas than
   // SMs one 16-warp CTA per SM runs a replica's actual and candidate chains side by side
-  const bool few_r = (int64_t)R < (int64_t)h->nsm;
+  bool few_r = (int64_t)R < (int64_t)h->nsm;
+  if (const char* ev = std::getenv("PROTEAN_FEW"))  // experiment knob: force the instance family
+    few_r = std::atoi(ev) != 0;
   const int block = 32 * (few_r ? PROTEAN_FEW_WARPS : kWarps);
   SmemLayout sl;
   sl.init(h->tl.words, h->M, N, Gc, CW, 0, 0);
