@@ -73,19 +73,27 @@ __device__ __forceinline__ bool key_less(int64_t k1, uint32_t i1, int64_t k2, ui
 template <int kB, typename TT>
 __device__ __forceinline__ void place_at(const int X, const SwShared& sh, const int32_t (&qv)[kB], int (&sl)[kB],
                                          TT (&st)[kB], TT (&en)[kB], int max_live, int64_t tb,
-                                         const uint32_t* arrival, int64_t& misses, int64_t& tail) {
+                                         const uint32_t* arrival, int64_t& misses, int64_t& tail,
+                                         int live_in = -1) {
   // sl[y] of an earlier batch is its slice if it was placed, else kOff (matches no slice), and
   // en[y] = 0 if it was not placed (never > t >= 0): one compare per test instead of two.
   constexpr int kOff = 15;
   const SwBatch& b = sh.b[X];
   const int s = sl[X];
   const TT t = (TT)(b.ready - tb);
-  int live = 0;
+  int live = live_in;  // residents live at t, GPU-wide: the same for every slice of batch X
   TT ls = 0;
+  if (live < 0) {
+    live = 0;
+#pragma unroll
+    for (int y = 0; y < kB; ++y) {
+      if (y >= X) break;
+      live += en[y] > t ? 1 : 0;
+    }
+  }
 #pragma unroll
   for (int y = 0; y < kB; ++y) {
     if (y >= X) break;
-    live += en[y] > t ? 1 : 0;
     if (sl[y] == s && st[y] > ls) ls = st[y];  // FIFO: the slice's last start
   }
   const int32_t Ms = sh.cap[s];
@@ -176,11 +184,20 @@ __device__ __forceinline__ void sweep_range(const SwShared& sh, const uint32_t* 
         const uint32_t idx = p + (uint32_t)s1 * wK;
         if (key_less(key, idx, best, bidx)) { best = key; bidx = idx; }
       } else {
+        int live2 = 0;  // the last batch's live count does not depend on its own slice
+        {
+          const TT t2r = (TT)(sh.b[K + 1].ready - tb);
+#pragma unroll
+          for (int y = 0; y < kB; ++y) {
+            if (y > K) break;
+            live2 += en[y] > t2r ? 1 : 0;
+          }
+        }
 #pragma unroll 1
         for (int s2 = 0; s2 < S; ++s2) {
           sl[K + 1] = s2;
           int64_t m2 = m1, t2 = t1;
-          place_at<kB, TT>(K + 1, sh, qv, sl, st, en, max_live, tb, arrival, m2, t2);
+          place_at<kB, TT>(K + 1, sh, qv, sl, st, en, max_live, tb, arrival, m2, t2, live2);
           const int64_t key = make_key(m2, t2, 0);
           const uint32_t idx = p + (uint32_t)s1 * wK + (uint32_t)s2 * wK1;
           if (key_less(key, idx, best, bidx)) { best = key; bidx = idx; }
