@@ -4,7 +4,12 @@
  * What this library computes is the "PROTEAN epoch model" (PEM): the paper's slowdown model
  * (Eq 1 / Eq 2), Job Distribution (Alg 1), the GPU Reconfigurator's decision step (Alg 2,
  * hysteresis + ~30% cap) and cost-aware procurement, driven by an exhaustive per-epoch search
- * over MIG geometries (the paper's "Oracle" scheme run online).  Paper citations are
+ * over MIG geometries (the paper's "Oracle" scheme run online) or by Alg 2's own heuristic
+ * (policy 2), optionally with the Autoscaler's container pools and cold starts; plus the
+ * exhaustive assignment sweep (section 3b) and a batch formation / dispatch helper (3a).
+ * Entry points: protean_load_profiles, protean_score_epoch, protean_replay_traces,
+ * protean_form_batches, protean_sweep_assignments, the mode-G exchange set-up (section 4) and
+ * small helpers (errors, geometries, epochs, timings, defaults).  Paper citations are
  * "P:L<n>" = line n of PAPER.md (Bhasi et al., "Towards SLO-Compliant and Cost-Effective
  * Serverless Computing on Emerging GPU Architectures", MIDDLEWARE '24).  Every reading of a
  * silent / ambiguous passage is listed in DESIGN.md §3 (Q1..Q39 follow SURVEY.md §8(c)).
@@ -15,8 +20,8 @@
  * converted to double once, from integer accumulators.
  *
  * Ownership: the caller owns every input and output buffer.  The library owns only the handle,
- * its device copy of the tables, its scratch memory and (mode G) its NCCL communicator; all are
- * released by protean_free().  The library never frees or reallocates caller memory.
+ * its device copy of the tables, its scratch memory and (mode G / virtual ranks) its exchange
+ * buffers; all are released by protean_free().  The library never frees or reallocates caller memory.
  *
  * Pointers: every pointer inside protean_epoch_in / protean_epoch_out / protean_replay_cfg /
  * protean_replay_out is a DEVICE pointer (cudaMalloc'd or torch CUDA tensor data) on the
@@ -50,7 +55,7 @@ enum {
   PROTEAN_ECUDA = -4,   /* a CUDA runtime call failed (handle poisoned) */
   PROTEAN_ENCCL = -5,   /* a cross-rank exchange failed or timed out (handle poisoned) */
   PROTEAN_ESTATE = -6,  /* handle poisoned, or bad call order */
-  PROTEAN_EUNSUP = -7   /* valid request this build does not implement (e.g. policy = Alg 2) */
+  PROTEAN_EUNSUP = -7   /* valid request this build does not implement (reserved) */
 };
 
 /* MIG slice profiles of the A100-40GB, T2, in ascending-resource order (the order
