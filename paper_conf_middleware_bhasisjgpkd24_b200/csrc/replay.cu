@@ -1676,30 +1676,41 @@ extern "C" int protean_debug_phase_cycles(unsigned long long* out) {
 #endif
 
 // Prepass: eoff[r][e] = first request of replica r with arrival >= e*W (e = 0..E), and the
-// largest request window any epoch needs: [lower_bound(eW - maxT), eoff[e+1]).
+// largest request window any epoch needs: [lower_bound(eW - maxT), eoff[e+1]).  A warp covers 32
+// consecutive epochs of one replica and owns the first 31 (lane 31 only computes its lower bound
+// for lane 30, and is owned again by the next warp's lane 0): eoff[e+1] comes from the next lane,
+// and when maxT <= W the window start lies in [eoff[e-1], eoff[e]] (the previous lane's bound), so
+// a lane runs one full-range binary search and one over about an epoch's requests.  On a sorted
+// trace the bounds equal the full-range searches; an unsorted one is flagged (next < here) here or
+// by the scatter pass, as before.
 __global__ void prepass_kernel(const uint32_t* arr, const int64_t* roff, int R, int64_t E,
                                int64_t W, int64_t maxT, int64_t* eoff, unsigned long long* wmax,
                                int* err) {
-  const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx >= (int64_t)R * (E + 1)) return;
-  const int r = (int)(idx / (E + 1));
-  const int64_t e = idx - (int64_t)r * (E + 1);
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t wpr = (E + 31) / 31;  // warps per replica: epochs 0..E, 31 owned per warp
+  if (gw >= (int64_t)R * wpr) return;  // warp-uniform
+  const int r = (int)(gw / wpr);
+  const int64_t e = (gw - (int64_t)r * wpr) * 31 + lane;
   const int64_t lo0 = roff[r], hi0 = roff[r + 1];
-  auto lower = [&](int64_t v) {
-    int64_t lo = lo0, hi = hi0;
+  auto lower = [&](int64_t v, int64_t lo, int64_t hi) {
     while (lo < hi) {
       const int64_t mid = (lo + hi) >> 1;
       if ((int64_t)arr[mid] >= v) hi = mid; else lo = mid + 1;
     }
     return lo;
   };
-  const int64_t here = lower(e * W);
-  eoff[idx] = here;
-  if (e < E) {
+  const bool live = e <= E;
+  const int64_t here = live ? lower(e * W, lo0, hi0) : hi0;
+  const int64_t next = __shfl_down_sync(0xffffffffu, here, 1);
+  const int64_t prev = __shfl_up_sync(0xffffffffu, here, 1);
+  if (lane == 31 || !live) return;
+  eoff[(size_t)r * (E + 1) + e] = here;
+  if (e < E) {  // lane + 1 <= 31 holds epoch e + 1 <= E
     const int64_t a = e * W - maxT;
-    const int64_t next = lower((e + 1) * W);
     if (next < here) atomicOr(err, 1);  // arrivals not sorted
-    const int64_t w = next - lower(a < 0 ? 0 : a);
+    const int64_t from = (lane > 0 && maxT <= W) ? prev : lo0;  // (e-1)W <= a <= eW
+    const int64_t w = next - lower(a < 0 ? 0 : a, from, here);
     if (w > 0) atomicMax(wmax, (unsigned long long)w);
   } else if (here != hi0) {
     atomicOr(err, 1);                   // an arrival at or beyond E*W >= trace_len
@@ -1709,7 +1720,7 @@ __global__ void prepass_kernel(const uint32_t* arr, const int64_t* roff, int R, 
 cudaError_t launch_prepass(const uint32_t* arr, const int64_t* roff, int R, int64_t E, int64_t W,
                            int64_t maxT, int64_t* eoff, unsigned long long* wmax, int* err,
                            cudaStream_t st) {
-  const int64_t total = (int64_t)R * (E + 1);
+  const int64_t total = (int64_t)R * ((E + 31) / 31) * 32;  // threads: one warp per 31 epochs
   const int bs = 256;
   prepass_kernel<<<(unsigned)((total + bs - 1) / bs), bs, 0, st>>>(arr, roff, R, E, W, maxT, eoff, wmax, err);
   return cudaGetLastError();
