@@ -6,11 +6,16 @@ Mix A (Wiki-shaped 5000 rps vision trace, 50/50 strict/BE, 22-model synthetic pr
 12 candidate geometries, geometry search policy, on-demand VMs.  One step = one full
 protean_replay_traces over all replicas of this rank (every epoch of every replica: batch
 formation, dispatch, actual placement, per-request accounting, candidate scoring, argmin,
-hysteresis/cap, finalize).  Weak scaling: each rank replays its own 4096 replicas (global replica
-ids rank*4096 + i), no data-path collective.  Inputs are generated in HBM before timing (61 GB per
-rank, far larger than the 126 MB L2, so no L2 flush is needed between steps).
+hysteresis/cap, finalize).  Strong scaling, mode R: the 4096 replicas are sharded across the N
+ranks (rank k replays the contiguous global range parallel.replica_range(4096, N, k), "sharded
+across 8xB200"), no data-path collective.  Inputs are generated in HBM before timing (61 GB at
+N = 1, far larger than the 126 MB L2, so no L2 flush is needed between steps).
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--replicas R]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--replicas R_total]
+  python bench.py --path c1|c2|c4   (single-replica latency lines: score_epoch C1, replay C2 / C4)
+
+--gpus N > 1 without a torchrun environment re-launches itself through torch.distributed.run
+(one process per GPU, rendezvous on 127.0.0.1).
 """
 from __future__ import annotations
 
@@ -140,7 +145,7 @@ def time_oracle(prof, tr, cores: int, policy: int = 0, cold_us: int = 0, keepali
     out = O.replay(prof, tr, N=8, nthreads=cores, policy=policy, cold_us=cold_us, keepalive_epochs=keepalive)
     dt = time.perf_counter() - t0
     c = out["counters"]
-    return dt, int(c[:, 8].sum()), int((c[:, 0] + c[:, 4]).sum()), int(c[:, 9].sum())
+    return dt, int(c[:, 8].sum()), int((c[:, 0] + c[:, 4]).sum()), int(c[:, 9].sum()), out["stats"]
 
 
 def run_reference(args):
@@ -156,7 +161,7 @@ def run_reference(args):
         time_oracle(prof, tr, cores, pol, args.cold_start_us, args.keepalive_epochs)
     dts, slots, reqs = [], 0, 0
     for _ in range(args.steps):
-        dt, s, q, _g = time_oracle(prof, tr, cores, pol, args.cold_start_us, args.keepalive_epochs)
+        dt, s, q, _g, _st = time_oracle(prof, tr, cores, pol, args.cold_start_us, args.keepalive_epochs)
         dts.append(dt)
         slots, reqs = s, q
     tot = sum(dts)
@@ -165,12 +170,14 @@ def run_reference(args):
     sample = f"{n_rep} replicas x {args.seconds} s of the config-5 workload (Mix A, 8 sim-GPUs, G=12)"
     line = {"impl": "reference", "metric": metric, "value": val, "unit": unit, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int64",
             "data": "synthetic",
-            "config": {"workload": f"C5 (configs[4]) sample: Mix A, 8 sim-GPUs, 600 s, G=12, {args.policy} policy",
-                       "replicas": n_rep, "seconds": args.seconds},
+            "config": {"workload": "C5 (configs[4]): Mix A Wiki-shaped 5000 rps, 22-model table, "
+                                   f"8 sim-GPUs, 600 s, 12 geometries, {args.policy} policy, on-demand VMs",
+                       "replicas_total": args.replicas, "seconds": args.seconds, "sample_replicas": n_rep},
             "simulated_requests_per_s": reqs * args.steps / tot,
-            "cpu_baseline": {"value": val, "unit": unit, "cores": cores, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": val, "unit": unit, "cores": cores, "kind": "oracle", "sample": sample,
+                             "cpu_model": cpu_info()["model"]},
             "e2e": {"value": val, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
@@ -179,10 +186,49 @@ def run_reference(args):
 # ------------------------------------------------------------------------------------------------
 # our arm
 # ------------------------------------------------------------------------------------------------
+def cpu_info():
+    """CPU model, logical CPUs and physical cores of this host (lscpu)."""
+    info = {"model": None, "logical": os.cpu_count(), "physical_cores": None}
+    try:
+        txt = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        kv = {ln.split(":", 1)[0].strip(): ln.split(":", 1)[1].strip() for ln in txt.splitlines() if ":" in ln}
+        info["model"] = kv.get("Model name")
+        cps, sock = kv.get("Core(s) per socket"), kv.get("Socket(s)")
+        if cps and sock and cps.isdigit() and sock.isdigit():
+            info["physical_cores"] = int(cps) * int(sock)
+    except Exception:
+        pass
+    return info
+
+
+def host_mem_available() -> int:
+    """MemAvailable of this host in bytes (Linux), else a conservative 64 GB."""
+    try:
+        for ln in open("/proc/meminfo"):
+            if ln.startswith("MemAvailable:"):
+                return int(ln.split()[1]) * 1024
+    except Exception:
+        pass
+    return 64 << 30
+
+
+def ncu_summary():
+    """The committed ncu summary of this round (profiles/ncu_summary.json), or None."""
+    path = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        return json.load(open(path))
+    except Exception:
+        return None
+
+
+ALG_BYTES_PER_REQUEST = 5.0  # SURVEY §8(d) d.3: u32 arrival + u8 meta, read once
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
     import paper_conf_middleware_bhasisjgpkd24_b200 as pkg
+    from paper_conf_middleware_bhasisjgpkd24_b200.parallel import replica_range
     from tools import tracegen
 
     world, rank, local = dist_setup()
@@ -192,8 +238,10 @@ def run_ours(args):
         dist.init_process_group("nccl", device_id=dev)
 
     prof = synth_profiles()
-    R, S, N = args.replicas, args.seconds, 8
-    gp = mix_a_params(R, seed=1, seconds=S, replica_base=rank * R)
+    R_total, S, N = args.replicas, args.seconds, 8
+    lo, hi = replica_range(R_total, world, rank)
+    R = hi - lo
+    gp = mix_a_params(R, seed=1, seconds=S, replica_base=lo)
     arr, meta, roff = tracegen.generate_on_device(gp, local)
     n_req = int(arr.shape[0])
     h = pkg.load_profiles(prof, device=local)
@@ -202,7 +250,7 @@ def run_ours(args):
     stream = torch.cuda.current_stream(dev)
     pol = POLICIES[args.policy]
     metric, unit = metric_of(args.policy)
-    cfg = dict(n_gpus=N, replica_base=rank * R, policy=pol, cold_start_us=args.cold_start_us,
+    cfg = dict(n_gpus=N, replica_base=lo, policy=pol, cold_start_us=args.cold_start_us,
                keepalive_epochs=args.keepalive_epochs)
 
     def step():
@@ -233,103 +281,150 @@ def run_ours(args):
     tot_ms = sum(step_ms)
     c = out["counters"].sum(0).cpu().numpy()
     slot, geom_c, reqs = int(c[8]), int(c[9]), int(c[0] + c[4])
+    met, s_arr = int(c[1]), int(c[0])
     if world > 1:
         t = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         tot_ms = float(t.item())
-        s = torch.tensor([slot, geom_c, reqs, n_req], dtype=torch.int64, device=dev)
+        s = torch.tensor([slot, geom_c, reqs, n_req, met, s_arr], dtype=torch.int64, device=dev)
         dist.all_reduce(s)
-        slot, geom_c, reqs, n_req_all = [int(x) for x in s.tolist()]
+        slot, geom_c, reqs, n_req_all, met, s_arr = [int(x) for x in s.tolist()]
     else:
         n_req_all = n_req
     sec = tot_ms / 1e3
     value = (slot if pol == 0 else reqs) * args.steps / sec
 
-    # e2e: the public call on HOST buffers (pinned), H2D + replay + D2H inside the timed region
+    # e2e: the C-ABI host-buffer call (protean_replay_traces_host) on pinned host copies of this
+    # rank's trace; every H2D / D2H is inside the timed region (host wall clock around the call)
     e2e = None
-    if rank == 0 and args.e2e_replicas > 0:
-        Re = min(args.e2e_replicas, R)
-        hi = int(roff[Re].item())
-        h_arr = torch.empty(hi, dtype=torch.int32, pin_memory=True)
-        h_meta = torch.empty(hi, dtype=torch.uint8, pin_memory=True)
-        h_off = torch.empty(Re + 1, dtype=torch.int64, pin_memory=True)
-        h_arr.copy_(arr[:hi])
-        h_meta.copy_(meta[:hi])
+    if args.e2e_replicas != 0:
+        Re = R if args.e2e_replicas < 0 else min(args.e2e_replicas, R)
+        avail = host_mem_available() // max(1, int(os.environ.get("LOCAL_WORLD_SIZE", world)))
+        offs_h = roff.cpu()
+        while Re > 1 and int(offs_h[Re]) * 5 > 0.4 * avail:  # page-locked trace copy within host RAM
+            Re //= 2
+        n_e = int(offs_h[Re])
+        h_arr = torch.empty(max(n_e, 1), dtype=torch.int32).pin_memory()
+        h_meta = torch.empty(max(n_e, 1), dtype=torch.uint8).pin_memory()
+        h_off = torch.empty(Re + 1, dtype=torch.int64).pin_memory()
+        h_arr[:n_e].copy_(arr[:n_e])
+        h_meta[:n_e].copy_(meta[:n_e])
         h_off.copy_(roff[:Re + 1])
-        ks = max(1, min(args.steps, 3))
-        kw = dict(trace_len_us=gp.trace_len_us, chunks=args.e2e_chunks, **cfg)
-        res = h.replay_traces_pinned(h_arr, h_meta, h_off, **kw)  # warm-up (and the pinned outputs)
+        res = h.alloc_host_out(Re, E, N)
         res_bytes = sum(t.numel() * t.element_size() for t in res.values())
+        kw = dict(trace_len_us=gp.trace_len_us, chunks=args.e2e_chunks, out_host=res, **cfg)
+        h.replay_traces_pinned(h_arr[:n_e], h_meta[:n_e], h_off, **kw)  # warm-up
+        ks = max(1, min(args.steps, 3))
+        if world > 1:
+            dist.barrier()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         for _ in range(ks):
-            h.replay_traces_pinned(h_arr, h_meta, h_off, out_host=res, **kw)
-        ems = (time.perf_counter() - t0) * 1e3  # host wall: every copy and the replay inside
+            h.replay_traces_pinned(h_arr[:n_e], h_meta[:n_e], h_off, **kw)
+        ems = (time.perf_counter() - t0) * 1e3
         pc = res["counters"]
         es = int(pc[:, 8].sum()) if pol == 0 else int((pc[:, 0] + pc[:, 4]).sum())
+        if world > 1:
+            t = torch.tensor([ems], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ems = float(t.item())
+            q = torch.tensor([es, n_e, Re], dtype=torch.int64, device=dev)
+            dist.all_reduce(q)
+            es, n_e_all, Re_all = [int(x) for x in q.tolist()]
+        else:
+            n_e_all, Re_all = n_e, Re
         e2e = {"value": es * ks / (ems / 1e3), "unit": unit,
-               "h2d_bytes_per_step": int(hi * 5 + (Re + 1) * 8), "d2h_bytes_per_step": int(res_bytes),
-               "sample": f"{Re} of {R} replicas through Handle.replay_traces_pinned from pinned host memory "
-                         f"({args.e2e_chunks} chunks: H2D of chunk k+1 overlaps the replay of chunk k)"}
+               "h2d_bytes_per_step": int(n_e_all * 5 + (Re_all + world) * 8),
+               "d2h_bytes_per_step": int(res_bytes) * world,
+               "ms_per_step": ems / ks,
+               "sample": f"{Re_all} of {R_total} replicas ({'all' if Re_all == R_total else 'a subset'}) through the "
+                         f"C-ABI host-buffer call protean_replay_traces_host from pinned host memory "
+                         f"({args.e2e_chunks} chunks: H2D of chunk k+1 and D2H of chunk k-1 overlap the replay of "
+                         f"chunk k); host wall clock, max over ranks"}
+        del h_arr, h_meta
 
-    cpu = None
+    cpu, h5 = None, None
     if rank == 0 and world == 1 and args.cpu_sample > 0:
+        ci = cpu_info()
         cores = os.cpu_count() or 1
         n_rep = min(args.cpu_sample, R)
-        tr = oracle_sample(n_rep, S, base=0)
-        dt, s_cpu, q_cpu, passes = 0.0, 0, 0, 0
+        tr = oracle_sample(n_rep, S, base=lo)
+        dt, s_cpu, q_cpu, passes, st = 0.0, 0, 0, 0, None
         while passes < 1 or (dt < 10.0 and passes < 40):  # ~10 s of oracle work on the host cores
-            d, s1, q1, _ = time_oracle(prof, tr, cores, pol, args.cold_start_us, args.keepalive_epochs)
+            d, s1, q1, _, st1 = time_oracle(prof, tr, cores, pol, args.cold_start_us, args.keepalive_epochs)
             dt, s_cpu, q_cpu, passes = dt + d, s_cpu + s1, q_cpu + q1, passes + 1
+            st = st1
+        # one host thread on a smaller sample of the same workload
+        tr1 = tr.subset(range(min(2, n_rep)))
+        d1, s11, q11, _, _ = time_oracle(prof, tr1, 1, pol, args.cold_start_us, args.keepalive_epochs)
         cpu = {"value": (s_cpu if pol == 0 else q_cpu) / dt, "unit": unit, "cores": cores, "kind": "oracle",
-               "sample": f"{n_rep} replicas x {S} s of this workload (numpy-generated), replayed "
-                         f"{passes}x: {dt:.1f} s wall on {cores} threads",
-               "simulated_requests_per_s": q_cpu / dt}
+               "sample": f"{n_rep} replicas x {S} s of this workload (numpy-generated, global ids {lo}..), "
+                         f"replayed {passes}x: {dt:.1f} s wall on {cores} threads",
+               "simulated_requests_per_s": q_cpu / dt,
+               "cpu_model": ci["model"], "logical_cpus": ci["logical"], "physical_cores": ci["physical_cores"],
+               "one_thread": {"value": (s11 if pol == 0 else q11) / d1, "unit": unit,
+                              "simulated_requests_per_s": q11 / d1,
+                              "sample": f"{min(2, n_rep)} replicas x {S} s, 1 thread, {d1:.1f} s"}}
+        if pol == 0 and st is not None:
+            # the search is not vacuous on this workload (oracle counters, same sample)
+            ss = st.sum(0)
+            h5 = {"best_ne_current_frac": float(ss[1] / max(ss[0], 1)),
+                  "fbr_sum_over_1e6_frac": float(ss[2] / max(ss[3], 1)),
+                  "source": f"CPU oracle on the cpu_baseline sample ({n_rep} replicas)",
+                  "threshold": 0.01}
+            h5["ok"] = h5["best_ne_current_frac"] >= 0.01 and h5["fbr_sum_over_1e6_frac"] >= 0.01
+            if not h5["ok"]:
+                print("WARNING: search near-vacuous on this workload (h5 self-check below 1%): "
+                      + json.dumps(h5), file=sys.stderr, flush=True)
 
     if rank == 0:
         peak, peak_kind = peaks()
         k_ms = statistics.mean(kern_ms)
         p_ms = statistics.mean(pre_ms)
-        # replay_kernel reads the stream-sorted arrivals once (4 B/request; its per-epoch run
-        # indices add 4 B per stream per replica-epoch, < 1%); the partition passes before it read
-        # meta (1 B), then arrivals + meta (5 B) and write the sorted arrivals (4 B) per request
-        alg_bytes = 4.0 * n_req
+        # 5 algorithmic bytes per request (u32 arrival + u8 meta, read once);
+        # rank 0's replay_kernel launch processes rank 0's requests
+        alg_bytes = ALG_BYTES_PER_REQUEST * n_req
         achieved = alg_bytes / (k_ms / 1e3) / 1e9
-        part_bytes = 10.0 * n_req
-        traffic, issue = None, None
-        prof_path = os.path.join(ROOT, "profiles", "ncu_summary.json")
-        if os.path.exists(prof_path):
-            try:
-                ps = json.load(open(prof_path))
-                traffic = ps["dram_bytes_per_request"] * n_req
-                # the kernel is bound by instruction issue, not HBM: the committed ncu
-                # capture's issue-slot utilisation is the other half of the picture
-                issue = {"issue_slots_busy_pct": ps.get("issue_active_pct"),
-                         "warp_instructions_per_request": ps["warp_instructions"] / ps["requests"],
-                         "source": ps.get("report")}
-            except Exception:
-                traffic, issue = None, None
+        step_ach = ALG_BYTES_PER_REQUEST * n_req_all / (sec / args.steps) / 1e9
+        ns = ncu_summary()
+        traffic, issue, passes_b = None, None, None
+        if ns:
+            rk = ns.get("kernels", {}).get("replay_kernel")
+            if rk:
+                traffic = rk["dram_bytes_per_request"] * n_req
+                issue = {"issue_slots_busy_pct": rk.get("issue_active_pct"),
+                         "warp_instructions_per_request": rk.get("warp_instructions_per_request"),
+                         "eligible_warps_per_scheduler": rk.get("eligible_warps_per_scheduler"),
+                         "source": ns.get("report")}
+            passes_b = {k: v.get("dram_bytes_per_request") for k, v in ns.get("kernels", {}).items()}
+        design_b = sum(v for v in (passes_b or {}).values() if v) if passes_b else None
         line = {
             "metric": metric, "value": value, "unit": unit, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+            "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
             "config": {"workload": "C5 (configs[4]): Mix A Wiki-shaped 5000 rps, 22-model table, "
                                    f"8 sim-GPUs, 600 s, 12 geometries, {args.policy} policy, on-demand VMs"
                                    + (f", N3 cold starts {args.cold_start_us} us / keep-alive "
                                       f"{args.keepalive_epochs} epochs" if args.cold_start_us else ""),
-                       "replicas_per_rank": R, "seconds": S, "sim_gpus": N, "geometries": h.n_geoms,
-                       "requests_per_rank": n_req, "l2_flush": "inputs (5 B/request, "
-                       f"{5.0 * n_req / 1e9:.1f} GB per rank) exceed the 126 MB L2"},
+                       "replicas_total": R_total, "replicas_per_rank": R, "seconds": S, "sim_gpus": N,
+                       "geometries": h.n_geoms, "requests_total": n_req_all, "parallelism": f"mode R x{world}",
+                       "l2_flush": "inputs (5 B/request, "
+                       f"{5.0 * n_req / 1e9:.1f} GB on rank 0) exceed the 126 MB L2"},
             "simulated_requests_per_s": reqs * args.steps / sec,
+            "strict_slo_compliance": met / max(s_arr, 1),
             "cold_starts_per_step": int(out["cold_starts"].sum().item()) * world if args.cold_start_us else None,
             "geom_candidates_per_s": geom_c * args.steps / sec,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
-                         "kernel": "replay_kernel", "kernel_ms": k_ms, "launch": launch, "issue": issue,
-                         "algorithmic_bytes_per_request": 4.0,
-                         "partition": {"ms": p_ms, "algorithmic_bytes_per_request": 10.0,
-                                       "achieved_GBps": part_bytes / (p_ms / 1e3) / 1e9,
-                                       "frac": part_bytes / (p_ms / 1e3) / 1e9 / peak}},
+                         "kernel": "replay_kernel", "kernel_ms": k_ms, "launch": launch,
+                         "algorithmic_bytes_per_request": ALG_BYTES_PER_REQUEST,
+                         "step": {"achieved": step_ach, "frac": step_ach / peak,
+                                  "note": "5 B x all requests / step time, per GPU"},
+                         "design_dram_bytes_per_request": passes_b,
+                         "traffic_ratio": (design_b / ALG_BYTES_PER_REQUEST) if design_b else None,
+                         "issue": issue,
+                         "passes_before_replay_ms": p_ms},
+            "search_self_check": h5,
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": 5 * args.steps * world, "clocks": clocks,
         }
         print(json.dumps(line), flush=True)
@@ -344,19 +439,6 @@ def run_ours(args):
 # ------------------------------------------------------------------------------------------------
 SWEEP_METRIC = "assignments scored/s (exhaustive sweep, N4a)"
 SWEEP_UNIT = "assignments/s"
-
-
-def sweep_alg_ops(batch_off: np.ndarray, sizes) -> int:
-    """Algorithmic integer work of the sweep: the assignment tree of a GPU-epoch with
-    b batches on S slices has S^(x+1) nodes at depth x (batch x placed after x earlier ones), each
-    12 + 8 x integer ops (live bound, FIFO and memory scans over the x earlier batches, Eq 1, key);
-    a prefix-sharing enumeration does exactly this work."""
-    b = np.diff(np.asarray(batch_off, np.int64))
-    tot = 0
-    for s in sizes:
-        for x in range(int(b.max(initial=0))):
-            tot += int(((b > x) * (s ** (x + 1)) * (12 + 8 * x)).sum())
-    return tot
 
 
 def run_sweep(args):
@@ -417,9 +499,14 @@ def run_sweep(args):
     sec = tot_ms / 1e3
     value = n_assign / sec
     if rank == 0:
-        sizes = [int((g != 255).sum()) for g in h.geometries()]
-        ops = sweep_alg_ops(off, sizes) * args.steps * world
-        peak_ops = 148 * 4 * 32 * 1.965e9  # thread-instructions/s: 1 warp-instr/clk per SMSP at max clock
+        # issue-slot roofline: warp-instructions per assignment from the committed ncu capture
+        # (profiles/ncu_summary.json, kernels.sweep_kernel) x assignments / live time, against the
+        # issue peak 148 SMs x 4 schedulers x 1 warp-instruction/clk at the sampled SM clock
+        ns = ncu_summary()
+        sk = (ns or {}).get("kernels", {}).get("sweep_kernel")
+        clk_mhz = clocks.get("sm_mhz") or 1965.0
+        peak_wi = 148 * 4 * clk_mhz * 1e6
+        wi = sk["warp_instructions_per_assignment"] * n_assign / sec if sk else None
         # e2e: host buffers -> H2D -> sweep -> D2H of the keys, per step
         h_rows = torch.from_numpy(rows.copy()).pin_memory()
         h_off = torch.from_numpy(off.copy()).pin_memory()
@@ -466,10 +553,14 @@ def run_sweep(args):
                                    "vision requests per sim-GPU-epoch, <= 8 batches), 22-model table, 12 geometries",
                        "replicas_per_rank": R, "sim_gpus": N, "batches_per_rank": int(off[-1]),
                        "l2_flush": "none needed: the sweep is ALU-bound (inputs 21 MB, each read once per step)"},
-            "roofline": {"bound": "alu", "achieved": ops / sec, "peak": peak_ops, "unit": "int-ops/s",
-                         "frac": ops / sec / peak_ops, "traffic": None, "peak_kind":
-                         "derived: 148 SMs x 4 schedulers x 32 lanes x 1 instruction/clk x 1965 MHz",
-                         "kernel": "sweep_kernel", "alg_ops_per_step": ops // (args.steps * world)},
+            "roofline": {"bound": "alu", "achieved": wi, "peak": peak_wi, "unit": "warp-instr/s",
+                         "frac": (wi / peak_wi) if wi else None, "traffic": None,
+                         "peak_kind": f"derived: 148 SMs x 4 schedulers x 1 warp-instruction/clk x {clk_mhz:.0f} MHz "
+                                      "(sampled SM clock); achieved = ncu warp-instructions per assignment "
+                                      "(profiles/ncu_summary.json) x assignments / device time",
+                         "issue_slots_busy_pct_ncu": sk.get("issue_active_pct") if sk else None,
+                         "active_threads_per_warp_ncu": sk.get("active_threads_per_warp") if sk else None,
+                         "kernel": "sweep_kernel"},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": args.steps * world, "clocks": clocks,
         }
         print(json.dumps(line), flush=True)
@@ -479,29 +570,189 @@ def run_sweep(args):
     return 0
 
 
+# ------------------------------------------------------------------------------------------------
+# single-replica latency paths (C1 score_epoch latency, C2 / C4 per-epoch latency)
+# ------------------------------------------------------------------------------------------------
+def run_c1(args):
+    """C1: protean_score_epoch latency (median of 100 device-timed calls) on config 1's batches."""
+    import torch
+    import paper_conf_middleware_bhasisjgpkd24_b200 as pkg
+    from paper_conf_middleware_bhasisjgpkd24_b200 import _abi as A
+    from protean_inputs import c1_profiles, c1_trace
+    world, rank, local = dist_setup()
+    if rank != 0:
+        return 0
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(local)
+    lines = []
+    for gs in (0, 1):
+        prof = c1_profiles().with_geometry_set(gs)
+        tr = c1_trace()
+        h = pkg.load_profiles(prof, device=local)
+        arr = torch.from_numpy(np.ascontiguousarray(tr.arrival_us).view(np.int32)).to(dev)
+        meta = torch.from_numpy(np.ascontiguousarray(tr.meta)).to(dev)
+        off = torch.from_numpy(np.ascontiguousarray(tr.replica_off, np.int64)).to(dev)
+        fb = h.form_batches(arr, meta, off, trace_len_us=tr.trace_len_us, n_gpus=1, e_lo=0, e_hi=1)
+        st0 = A.GpuState()
+        st0.geom, st0.target, st0.has_vm, st0.vm_type = 2, 255, 1, 1
+        pristine = torch.from_numpy(np.frombuffer(bytes(st0), np.uint8).copy()).to(dev)
+        state = pristine.clone()
+        stream = torch.cuda.current_stream(dev)
+        boff = fb["batch_off"][:2].contiguous()
+        rows = fb["rows"].reshape(-1)
+
+        def call(out=None):
+            state.copy_(pristine)
+            return h.score_epoch(n_replicas=1, n_gpus=1, epoch=0, batches=rows, batch_off=boff,
+                                 arrival_us=fb["members"], state=state, stream=stream, sync=False)
+        for _ in range(max(args.warmup, 3)):
+            o = call()
+        torch.cuda.synchronize()
+        h.score_epoch_status()
+        ts = []
+        for _ in range(100):
+            state.copy_(pristine)
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            o = h.score_epoch(n_replicas=1, n_gpus=1, epoch=0, batches=rows, batch_off=boff,
+                              arrival_us=fb["members"], state=state, stream=stream, sync=False)
+            b.record(stream)
+            ts.append((a, b))
+        torch.cuda.synchronize()
+        h.score_epoch_status()
+        us = sorted(1e3 * a.elapsed_time(b) for a, b in ts)
+        c = o["counters"].cpu().numpy()[0]
+        lines.append({"geometries": h.n_geoms, "batches": fb["n"], "median_us": us[50], "min_us": us[0],
+                      "slot_evals_per_call": int(c[8]), "slot_evals_per_s": float(c[8]) / (us[50] * 1e-6)})
+    line = {"metric": "protean_score_epoch latency (C1)", "value": lines[0]["median_us"], "unit": "us",
+            "n_gpus": 1, "steps": 100, "warmup": max(args.warmup, 3), "ms_per_step": lines[0]["median_us"] / 1e3,
+            "higher_is_better": False, "scaling": "none", "vs_baseline": None, "dtype": "int64",
+            "data": "synthetic",
+            "config": {"workload": "C1 (configs[0]): 1 sim-GPU, 3 models, 200-request 1 s Poisson trace; one "
+                                   "epoch's dispatched batches (protean_form_batches) scored from a fresh state",
+                       "per_geometry_set": lines},
+            "gpu_launches": 1}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def run_single(args, name):
+    """C2 (8 sim-GPUs, 22 models, 1 h Mix B, G = 12) or C4 (64 sim-GPUs, Mix B x 8, G = 37):
+    one replica replayed on one B200 (virtual ranks: the replica's CTAs split the geometry range);
+    per-epoch latency = replay device time / E."""
+    import torch
+    import paper_conf_middleware_bhasisjgpkd24_b200 as pkg
+    from protean_inputs import mix_b_params
+    from tools import tracegen
+    world, rank, local = dist_setup()
+    if rank != 0:
+        return 0
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(local)
+    seconds = args.seconds if args.seconds != 600 else 3600
+    if name == "c2":
+        gp, N, gs = mix_b_params(1, seed=2, seconds=seconds), 8, 0
+    else:
+        gp, N, gs = mix_b_params(1, seed=4, seconds=seconds, scale=8.0), 64, 1
+    prof = synth_profiles().with_geometry_set(gs)
+    arr, meta, roff = tracegen.generate_on_device(gp, local)
+    h = pkg.load_profiles(prof, device=local)
+    E = h.num_epochs(gp.trace_len_us)
+    out = h.alloc_replay_out(1, E, N)
+    stream = torch.cuda.current_stream(dev)
+    for _ in range(max(1, args.warmup)):
+        h.replay_traces(arr, meta, roff, trace_len_us=gp.trace_len_us, out=out, stream=stream, n_gpus=N)
+    torch.cuda.synchronize()
+    ts, ks = [], []
+    for _ in range(args.steps):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        h.replay_traces(arr, meta, roff, trace_len_us=gp.trace_len_us, out=out, stream=stream, n_gpus=N)
+        b.record(stream)
+        torch.cuda.synchronize()
+        ts.append(a.elapsed_time(b))
+        ks.append(h.last_timings()[1])
+    c = out["counters"].cpu().numpy()[0]
+    ms = statistics.median(ts)
+    cpu = None
+    if args.cpu_sample > 0:
+        from oracle import oracle as O
+        from protean_inputs import tick_trace
+        O.build()
+        secs = min(seconds, 600)
+        gq = mix_b_params(1, seed=2 if name == "c2" else 4, seconds=secs, scale=1.0 if name == "c2" else 8.0)
+        trq = tick_trace(gq)
+        t0 = time.perf_counter()
+        oo = O.replay(prof, trq, N=N, nthreads=1)
+        dq = time.perf_counter() - t0
+        Eq = oo["decisions"].shape[1]
+        cpu = {"value": 1e6 * dq / Eq, "unit": "us per epoch", "cores": 1, "kind": "oracle",
+               "sample": f"first {secs} s of the same trace, 1 thread (a single replica is inherently "
+                         f"sequential), {dq:.1f} s", "cpu_model": cpu_info()["model"]}
+    line = {"metric": f"per-epoch replay latency ({name.upper()})", "value": 1e3 * ms / E, "unit": "us per epoch",
+            "n_gpus": 1, "steps": args.steps, "warmup": max(1, args.warmup), "ms_per_step": ms,
+            "higher_is_better": False, "scaling": "none", "vs_baseline": None, "dtype": "int64",
+            "data": "synthetic",
+            "config": {"workload": ("C2 (configs[1]): 8 sim-GPUs, 22 models, Mix B bursty" if name == "c2" else
+                                    "C4 (configs[3]): 64 sim-GPUs, Mix B x 8, 37 geometries") + f", {seconds} s, 1 replica",
+                       "epochs": E, "requests": int(c[0] + c[4]), "launch": h.last_timings()[2]},
+            "replay_kernel_ms": statistics.median(ks),
+            "slot_evals_per_s": float(c[8]) / (ms / 1e3),
+            "simulated_requests_per_s": float(c[0] + c[4]) / (ms / 1e3),
+            "strict_slo_compliance": float(c[1]) / max(float(c[0]), 1.0),
+            "cpu_baseline": cpu, "gpu_launches": 5 * args.steps}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def relaunch(args) -> int:
+    """--gpus N > 1 outside torchrun: one process per GPU through torch.distributed.run."""
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--replicas", type=int, default=4096, help="replicas per rank")
+    ap.add_argument("--replicas", type=int, default=4096, help="replicas in total (sharded over the ranks)")
     ap.add_argument("--seconds", type=int, default=600)
-    ap.add_argument("--e2e-replicas", type=int, default=512)
-    ap.add_argument("--e2e-chunks", type=int, default=4)
+    ap.add_argument("--e2e-replicas", type=int, default=-1,
+                    help="replicas per rank through the host-buffer call (-1 = all of the rank's, 0 = skip)")
+    ap.add_argument("--e2e-chunks", type=int, default=8)
     ap.add_argument("--cpu-sample", type=int, default=64, help="replicas timed on the CPU oracle")
-    ap.add_argument("--path", default="replay", choices=["replay", "sweep"],
-                    help="replay = protean_replay_traces (headline); sweep = protean_sweep_assignments (N4a)")
+    ap.add_argument("--path", default="replay", choices=["replay", "sweep", "c1", "c2", "c4"],
+                    help="replay = protean_replay_traces on C5 (headline); sweep = protean_sweep_assignments "
+                         "(N4a); c1 = score_epoch latency; c2 / c4 = single-replica per-epoch latency")
     ap.add_argument("--cold-start-us", type=int, default=0,
                     help="N3 container cold start (0 = warm containers, the paper's headline setting)")
     ap.add_argument("--keepalive-epochs", type=int, default=600, help="N3 delayed termination (epochs)")
     ap.add_argument("--policy", default="search", choices=sorted(POLICIES),
                     help="search = the geometry search (headline); alg2 = Alg 2's own heuristic (N1)")
     args = ap.parse_args()
+    if args.gpus < 1:
+        ap.error("--gpus must be >= 1")
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        return relaunch(args)
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world != args.gpus:
+        print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}", file=sys.stderr)
+        return 2
     if args.impl == "reference":
         return run_reference(args)
     if args.path == "sweep":
         return run_sweep(args)
+    if args.path == "c1":
+        return run_c1(args)
+    if args.path in ("c2", "c4"):
+        return run_single(args, args.path)
     return run_ours(args)
 
 

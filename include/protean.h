@@ -120,8 +120,14 @@ int protean_num_epochs(const protean_handle *h, int64_t trace_len_us, int64_t ep
  *    placement, which advances `state`); and if the GPU is decidable at T (has_vm and
  *    recfg_end <= T) every candidate geometry j in [geom_lo, geom_hi) replays the same batch list
  *    from an idle GPU and is scored by key = misses<<40 | BE_tail<<8 | tag, tag 0 = current
- *    geometry, else j+1 (O8).  Enqueued on `stream` (cudaStream_t; NULL = legacy default); returns
- *    after the stream completes, because the in-kernel validation verdict is read back.         */
+ *    geometry, else j+1 (O8); each node-epoch's VM cost price(vm_type) x W is reported (T3,
+ *    P:L173-179; cost projection P:L333; reading Q35: reported, not keyed).
+ *    Enqueue-only: validation runs in the kernel and the call returns once the work is enqueued on
+ *    `stream` (cudaStream_t; NULL = legacy default); outputs (and `state`) are valid after a sync of
+ *    that stream.  The kernel's validation verdict (EINVAL: bad state / batch / offsets; ERANGE:
+ *    n_live > max_live) is latched in a device word of the handle: protean_score_epoch_status()
+ *    reads it after the caller's sync.  An invalid CTA (replica) writes none of its outputs and
+ *    leaves its states untouched.  Host-detectable argument errors are still returned directly. */
 typedef struct {           /* 16 B */
   uint32_t ready_us;       /* batch ready time (O3): last member's arrival if full, else first + T_m */
   uint32_t req_off;        /* index of the batch's first member in arrival_us */
@@ -144,10 +150,15 @@ typedef struct {           /* one simulated GPU's carried state; caller-allocate
   uint8_t wait_ctr;        /* Alg 2 wait_ctr — not modified by score_epoch */
   uint8_t n_live;          /* residents in live[] (<= max_live) */
   uint8_t has_vm;          /* 1 = the node holds a VM at the decision time */
-  uint8_t vm_type, pad[2];
+  uint8_t vm_type;         /* billing type of the node's VM this epoch: 0 none, 1 on-demand, 2 spot */
+  uint8_t pad[2];
   int64_t recfg_start_us, recfg_end_us;  /* reconfiguration window [start, end), 0/0 = none */
   int64_t last_start_us[PROTEAN_MAX_SLICES];   /* FIFO: latest start on each slice */
   int64_t busy_until_us[PROTEAN_MAX_SLICES];   /* busy-time union bookkeeping (O6e) */
+  int64_t busy_us[PROTEAN_MAX_SLICES];         /* ACCUMULATED busy us of each slice instance: the
+                                                  union of its batches' [start, end) clipped to
+                                                  [0, H) (O6e, "percentage non-idle time");
+                                                  cleared with the state on a reconfiguration install */
   protean_resident live[PROTEAN_MAX_LIVE];
 } protean_gpu_state;
 
@@ -168,6 +179,8 @@ typedef struct {
   const uint32_t *arrival_us;          /* member arrivals referenced by req_off */
   protean_gpu_state *state;            /* [R*N] in/out */
   int32_t geom_lo, geom_hi;            /* candidate range; [0, G) = all */
+  double price_od_node_hr;             /* USD per node-hour of an on-demand VM (T3 / 8, Q27), >= 0 */
+  double price_spot_node_hr;           /* USD per node-hour of a spot VM, >= 0 */
 } protean_epoch_in;
 
 typedef struct {
@@ -176,10 +189,17 @@ typedef struct {
   protean_placement *placement; /* [n_batches] actual placement, same order as batches */
   int64_t *counters;          /* [R][10] ACCUMULATED (+=): see protean_replay_out.counters */
   int64_t *accum;             /* [R][4] ACCUMULATED, or NULL: busy_w, mem_num (see replay) */
+  double *cost_usd;           /* [R*N] node-epoch VM cost, or NULL: has_vm ? price(vm_type) * W /
+                                 3.6e9 : 0, evaluated as (price * (double)W) / 3.6e9 */
 } protean_epoch_out;
 
 int protean_score_epoch(protean_handle *h, const protean_epoch_in *in, protean_epoch_out *out,
                         void *stream);
+
+/* Verdict of the score_epoch calls enqueued since the last status call (host; synchronises the
+ * handle's device): PROTEAN_OK, or EINVAL / ERANGE if any enqueued kernel rejected its input (the
+ * detail goes to protean_last_error).  Clears the latched word. */
+int protean_score_epoch_status(protean_handle *h);
 
 /* ---------------------------------------------------------------------------------------------
  * 3. Trace replay, epoch by epoch, of many independent replicas (the north-star path, §8(a)
@@ -285,6 +305,21 @@ int protean_replay_traces(protean_handle *h, const protean_replay_cfg *cfg,
  * and kept by the handle for the next call. */
 int protean_last_timings(const protean_handle *h, float *prepass_ms, float *replay_ms,
                          int32_t *launch);
+
+/* ---------------------------------------------------------------------------------------------
+ * 3c. End-to-end replay from HOST buffers: the computation of protean_replay_traces (mode R), with
+ *     cfg->arrival_us, cfg->meta, cfg->replica_off and every output pointer of `out` being HOST
+ *     pointers (cand_keys and batch_log must be NULL).  The replicas are cut into `chunks`
+ *     contiguous ranges (1..R); chunk k+1's trace is copied host -> device on an internal copy
+ *     stream while chunk k replays on `stream`, and chunk k's outputs are copied back on an
+ *     internal return stream while chunk k+1 replays (two device staging slots owned by the
+ *     handle, grown on demand).  Replicas keep their global ids (replica_base + r), so the outputs
+ *     equal one device call over all replicas.  Host trace and output buffers should be
+ *     page-locked (cudaHostAlloc / cudaHostRegister) for the copies to overlap; pageable memory is
+ *     correct but serialises.  protean_last_timings then reports the device time summed over the
+ *     chunks.  Synchronous.  Errors as protean_replay_traces; EINVAL for shard_mode != 0.       */
+int protean_replay_traces_host(protean_handle *h, const protean_replay_cfg *cfg,
+                               protean_replay_out *out, int32_t chunks, void *stream);
 
 /* Fill a replay config with the defaults listed above (host). */
 void protean_replay_cfg_defaults(protean_replay_cfg *cfg);

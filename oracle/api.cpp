@@ -88,6 +88,7 @@ void state_in(const orc_state* s, GpuState* S) {
   for (int i = 0; i < kMaxSlices; ++i) {
     S->last_start[i] = s->last_start[i];
     S->busy_until[i] = s->busy_until[i];
+    S->busy_us[i] = s->busy_us[i];
   }
   S->res.clear();
   for (int i = 0; i < s->n_res; ++i) {
@@ -107,6 +108,7 @@ void state_out(const GpuState& S, orc_state* s) {
   for (int i = 0; i < kMaxSlices; ++i) {
     s->last_start[i] = S.last_start[i];
     s->busy_until[i] = S.busy_until[i];
+    s->busy_us[i] = S.busy_us[i];
   }
   s->n_res = (int32_t)S.res.size();
   for (size_t i = 0; i < S.res.size() && i < 64; ++i) {
@@ -342,6 +344,8 @@ int orc_replay(const orc_tables* t, const orc_replay_in* in, orc_replay_out* out
         std::copy(ro.cand_keys.begin(), ro.cand_keys.end(), out->cand_keys + (int64_t)r * E * N * G);
       if (out->n_batches) out->n_batches[r] = ro.n_batches;
       if (out->cold_starts) out->cold_starts[r] = ro.cold_starts;
+      if (out->stats)
+        for (int i = 0; i < 4; ++i) out->stats[r * 4 + i] = ro.stats[i];
       if (ro.pool_overflow) overflow = true;
       if (out->log) {
         for (size_t i = 0; i < ro.log.size() && (int64_t)i < out->log_cap; ++i) {
@@ -376,7 +380,8 @@ int orc_score_epoch(const orc_tables* t, int32_t R, int32_t N, int32_t epoch, in
                     const int32_t* batch_off, const uint32_t* arrival, orc_state* state,
                     int32_t geom_lo, int32_t geom_hi, int64_t* best_key, int64_t* cand_key,
                     int64_t* p_start, int64_t* p_end, int32_t* p_slice, int32_t* p_dropped,
-                    int64_t* counters, int64_t* accum) {
+                    int64_t* counters, int64_t* accum, double price_od, double price_spot,
+                    double* cost) {
   Tables tb;
   int rc = build_tables(t, &tb);
   if (rc) return rc;
@@ -387,6 +392,7 @@ int orc_score_epoch(const orc_tables* t, int32_t R, int32_t N, int32_t epoch, in
   if (geom_lo < 0 || geom_hi > G || geom_lo >= geom_hi) return ORC_EINVAL;
   if (!batch_off || !state || !best_key || !counters) return ORC_EINVAL;
   if (batch_off[0] != 0) return ORC_EINVAL;
+  if (!(price_od >= 0) || !(price_spot >= 0)) return ORC_EINVAL;
   const int64_t eW = (int64_t)epoch * W, T = eW + W;
   for (int x = 0; x < R * N; ++x) {
     if (batch_off[x + 1] < batch_off[x]) return ORC_EINVAL;
@@ -394,6 +400,7 @@ int orc_score_epoch(const orc_tables* t, int32_t R, int32_t N, int32_t epoch, in
     if (s.geom < 0 || s.geom >= G) return ORC_EINVAL;
     if (s.target != -1 && (s.target < 0 || s.target >= G)) return ORC_EINVAL;
     if (s.n_res < 0) return ORC_EINVAL;
+    if (s.vm_type < 0 || s.vm_type > 2) return ORC_EINVAL;
     if (s.n_res > max_live) return ORC_ERANGE;
     for (int i = 0; i < s.n_res; ++i)
       if (s.res[i].slice < 0 || s.res[i].slice >= (int)tb.geoms[s.geom].size() ||
@@ -452,6 +459,12 @@ int orc_score_epoch(const orc_tables* t, int32_t R, int32_t N, int32_t epoch, in
         accum[4 * r + 1] += acc.mem_num;
       }
       const bool decidable = st.has_vm && st.recfg_end <= T;
+      // node-epoch VM cost (T3 P:L173-179, cost projection P:L333, reading Q35): the node's
+      // price for its billing type over the epoch, price [$/h] * W [us] / 3.6e9 [us/h]
+      if (cost) {
+        const double price = !st.has_vm ? 0.0 : st.vm_type == 1 ? price_od : st.vm_type == 2 ? price_spot : 0.0;
+        cost[x] = (price * (double)W) / 3.6e9;
+      }
       best_key[x] = -1;
       for (int j = geom_lo; j < geom_hi; ++j) {
         int64_t key = -1;

@@ -340,6 +340,12 @@ struct Replay {
               const Batch& b = batches[x];
               PlaceOut po = place(tb, tb.geoms[j], C, b.ready, b.model, b.strict, cfg.max_live,
                                   nullptr, H);
+              if (po.dropped != 3)  // h5 self-check: co-location pressure on the scored slices
+                for (size_t s = 0; s < tb.geoms[j].size(); ++s)
+                  if (po.feasible[s]) {
+                    out->stats[3] += 1;
+                    if (po.s_F[s] > kPpm) out->stats[2] += 1;
+                  }
               if (b.strict) {
                 if (po.dropped) {
                   misses += b.n;
@@ -363,6 +369,8 @@ struct Replay {
           }
           const int tag = (int)(key_best[n] & 255);
           best[n] = tag == 0 ? cur : tag - 1;
+          out->stats[0] += 1;
+          if (tag != 0) out->stats[1] += 1;
           out->decisions[(size_t)e * N + n] = (uint8_t)best[n];
           // Alg 2 lines 24-30, reading Q22
           if (best[n] != cur) {

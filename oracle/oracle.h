@@ -28,8 +28,9 @@ typedef struct { int64_t start, end; int32_t mem, slice, model, strict; } orc_re
 typedef struct {
   int32_t geom, target, wait_ctr, has_vm;
   int64_t recfg_start, recfg_end;
-  int64_t last_start[7], busy_until[7];
-  int32_t n_res, pad;
+  int64_t last_start[7], busy_until[7], busy_us[7];
+  int32_t vm_type;                /* 0 none, 1 on-demand, 2 spot (billing type this epoch) */
+  int32_t n_res;
   orc_res res[64];
 } orc_state;
 
@@ -96,6 +97,10 @@ typedef struct {
   int64_t log_cap;
   int64_t *n_batches;  /* [R] or NULL */
   int64_t *cold_starts; /* [R] or NULL (N3) */
+  int64_t *stats;       /* [R][4] or NULL: workload self-checks, not a method output:
+                           0 decidable GPU-epochs scored, 1 of them with best != current geometry,
+                           2 candidate (batch, feasible slice) evaluations with Eq 1's F > 10^6,
+                           3 candidate (batch, feasible slice) evaluations */
 } orc_replay_out;
 
 int orc_replay(const orc_tables *t, const orc_replay_in *in, orc_replay_out *out);
@@ -107,7 +112,8 @@ int orc_score_epoch(const orc_tables *t, int32_t R, int32_t N, int32_t epoch, in
                     const int32_t *batch_off, const uint32_t *arrival, orc_state *state,
                     int32_t geom_lo, int32_t geom_hi, int64_t *best_key, int64_t *cand_key,
                     int64_t *p_start, int64_t *p_end, int32_t *p_slice, int32_t *p_dropped,
-                    int64_t *counters, int64_t *accum);
+                    int64_t *counters, int64_t *accum, double price_od, double price_spot,
+                    double *cost);
 
 /* O3 batch formation + O5.2 round-robin dispatch for epochs [e_lo, e_hi) (the form_batches
  * helper of SURVEY §8(b)): rows ordered by (replica, epoch, gpu, batch id), batch_off CSR over

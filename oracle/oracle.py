@@ -38,8 +38,8 @@ class Res(C.Structure):
 class State(C.Structure):
     _fields_ = [("geom", C.c_int32), ("target", C.c_int32), ("wait_ctr", C.c_int32),
                 ("has_vm", C.c_int32), ("recfg_start", C.c_int64), ("recfg_end", C.c_int64),
-                ("last_start", C.c_int64 * 7), ("busy_until", C.c_int64 * 7),
-                ("n_res", C.c_int32), ("pad", C.c_int32), ("res", Res * 64)]
+                ("last_start", C.c_int64 * 7), ("busy_until", C.c_int64 * 7), ("busy_us", C.c_int64 * 7),
+                ("vm_type", C.c_int32), ("n_res", C.c_int32), ("res", Res * 64)]
 
 
 class ReplayIn(C.Structure):
@@ -66,7 +66,8 @@ class ReplayOut(C.Structure):
     _fields_ = [("counters", C.c_void_p), ("accum", C.c_void_p), ("hist", C.c_void_p),
                 ("p50_p99", C.c_void_p), ("cost", C.c_void_p), ("util", C.c_void_p),
                 ("decisions", C.c_void_p), ("cand_keys", C.c_void_p), ("log", C.c_void_p),
-                ("log_cap", C.c_int64), ("n_batches", C.c_void_p), ("cold_starts", C.c_void_p)]
+                ("log_cap", C.c_int64), ("n_batches", C.c_void_p), ("cold_starts", C.c_void_p),
+                ("stats", C.c_void_p)]
 
 
 BATCH_REC_DTYPE = np.dtype([("ready", "<u4"), ("epoch", "<u4"), ("n", "<i4"), ("model", "<i4"),
@@ -115,7 +116,8 @@ def lib():
         L.orc_table_geometries.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p]
         L.orc_replay.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p]
         L.orc_score_epoch.argtypes = ([C.c_void_p] + [C.c_int32] * 4 + [C.c_int64] * 2 +
-                                      [C.c_void_p] * 8 + [C.c_int32] * 2 + [C.c_void_p] * 8)
+                                      [C.c_void_p] * 8 + [C.c_int32] * 2 + [C.c_void_p] * 8 +
+                                      [C.c_double, C.c_double, C.c_void_p])
         L.orc_form_dispatch.argtypes = ([C.c_void_p, C.c_int32, C.c_int32, C.c_int64, C.c_int64] + [C.c_void_p] * 3 +
                                        [C.c_int32, C.c_int32] + [C.c_void_p] * 10 + [C.c_int64])
         L.orc_sweep.argtypes = ([C.c_void_p] + [C.c_int32] * 4 + [C.c_void_p] * 8 + [C.c_int32] * 2 +
@@ -291,7 +293,7 @@ def replay(prof, trace, *, nthreads=1, want_keys=False, want_log=False, log_cap=
                hist=np.zeros((R, 2, NB), np.uint32), p50_p99=np.zeros((R, 2, 2), np.int64),
                cost=np.zeros(R, np.float64), util=np.zeros((R, 2), np.float64),
                decisions=np.zeros((R, E, N), np.uint8), n_batches=np.zeros(R, np.int64),
-               cold_starts=np.zeros(R, np.int64))
+               cold_starts=np.zeros(R, np.int64), stats=np.zeros((R, 4), np.int64))
     if want_keys:
         out["cand_keys"] = np.zeros((R, E, N, G), np.int64)
     if want_log:
@@ -300,7 +302,8 @@ def replay(prof, trace, *, nthreads=1, want_keys=False, want_log=False, log_cap=
         out["log"] = np.zeros((R, log_cap), BATCH_REC_DTYPE)
     ro = ReplayOut(_p(out["counters"]), _p(out["accum"]), _p(out["hist"]), _p(out["p50_p99"]),
                    _p(out["cost"]), _p(out["util"]), _p(out["decisions"]), _p(out.get("cand_keys")),
-                   _p(out.get("log")), int(log_cap or 0), _p(out["n_batches"]), _p(out["cold_starts"]))
+                   _p(out.get("log")), int(log_cap or 0), _p(out["n_batches"]), _p(out["cold_starts"]),
+                   _p(out["stats"]))
     rc = lib().orc_replay(T.ref, C.byref(rin), C.byref(ro))
     if rc:
         raise OracleError(rc)
@@ -309,7 +312,7 @@ def replay(prof, trace, *, nthreads=1, want_keys=False, want_log=False, log_cap=
 
 
 def score_epoch(prof, *, R, N, epoch, batches, batch_off, arrival, states, geom_lo=0, geom_hi=None,
-                W=1_000_000, H=1 << 62, max_live=64):
+                W=1_000_000, H=1 << 62, max_live=64, price_od=32.7726 / 8, price_spot=9.8318 / 8):
     """batches: dict of arrays ready, req_off, n, model, strict (ordered by (replica, gpu, id));
     states: ctypes array of State (modified in place)."""
     T = OTables(prof)
@@ -327,12 +330,14 @@ def score_epoch(prof, *, R, N, epoch, batches, batch_off, arrival, states, geom_
     out = dict(best_key=np.zeros(R * N, np.int64), cand_key=np.zeros(R * N * max(nc, 0), np.int64),
                start=np.zeros(max(nb, 1), np.int64), end=np.zeros(max(nb, 1), np.int64),
                slice=np.zeros(max(nb, 1), np.int32), dropped=np.zeros(max(nb, 1), np.int32),
-               counters=np.zeros((R, 10), np.int64), accum=np.zeros((R, 4), np.int64))
-    rc = lib().orc_score_epoch(T.ref, R, N, epoch, max_live, W, H, _p(arrs["ready"]), _p(arrs["req_off"]),
+               counters=np.zeros((R, 10), np.int64), accum=np.zeros((R, 4), np.int64),
+               cost=np.zeros(R * N, np.float64))
+    rc = lib().orc_score_epoch(T.ref, R, N, epoch, max_live, C.c_int64(W), C.c_int64(H), _p(arrs["ready"]), _p(arrs["req_off"]),
                                _p(arrs["n"]), _p(arrs["model"]), _p(arrs["strict"]), _p(boff),
                                _p(arrival), C.addressof(states), geom_lo, geom_hi, _p(out["best_key"]),
                                _p(out["cand_key"]), _p(out["start"]), _p(out["end"]), _p(out["slice"]),
-                               _p(out["dropped"]), _p(out["counters"]), _p(out["accum"]))
+                               _p(out["dropped"]), _p(out["counters"]), _p(out["accum"]),
+                               C.c_double(price_od), C.c_double(price_spot), _p(out["cost"]))
     if rc:
         raise OracleError(rc)
     for k in ("start", "end", "slice", "dropped"):

@@ -54,6 +54,7 @@ struct GpuState {
   std::vector<Resident> res;
   int64_t last_start[kMaxSlices] = {0};
   int64_t busy_until[kMaxSlices] = {0};
+  int64_t busy_us[kMaxSlices] = {0};  // O6e: busy union of each slice instance, clipped to [0, H)
 };
 
 struct PlaceOut {
@@ -65,6 +66,7 @@ struct PlaceOut {
   bool eligible[kMaxSlices] = {false};
   int64_t s_start[kMaxSlices] = {0};
   int64_t s_end[kMaxSlices] = {0};
+  int64_t s_F[kMaxSlices] = {0};   // Eq 1's F (ppm) at each feasible slice's start (diagnostic)
 };
 
 // Accounting hooks of the actual placement (O6e): busy union + memory-time, clipped to [0,H).
@@ -136,6 +138,7 @@ struct ReplayOut {
   std::vector<int64_t> cand_keys;       // [E][N][G]
   std::vector<BatchRec> log;
   int64_t n_batches = 0;
+  int64_t stats[4] = {0, 0, 0, 0};      // h5 workload self-checks (oracle.h orc_replay_out.stats)
 };
 int64_t num_epochs(const Tables& tb, int64_t trace_len, int64_t W);
 void replay_replica(const Tables& tb, const ReplayCfg& cfg, uint64_t replica_id,

@@ -69,6 +69,7 @@ PlaceOut place(const Tables& tb, const std::vector<int>& geom, GpuState& S, int6
       if (r.slice == s && r.start <= start && start < r.end) F += tb.fbr_at(r.model, p);
 
     o.s_start[s] = start;
+    o.s_F[s] = F;
     o.s_end[s] = start + exec_us(tb.solo_at(m, p), F);
   }
 
@@ -139,7 +140,10 @@ PlaceOut place(const Tables& tb, const std::vector<int>& geom, GpuState& S, int6
     const int p = geom[chosen];
     int64_t lo = std::max(o.start, S.busy_until[chosen]);
     int64_t hi = std::min(o.end, H);
-    if (hi > lo) acc->busy_w += (int64_t)kCompute[p] * (hi - lo);
+    if (hi > lo) {
+      acc->busy_w += (int64_t)kCompute[p] * (hi - lo);
+      S.busy_us[chosen] += hi - lo;
+    }
     int64_t mhi = std::min(o.end, H);
     if (mhi > o.start) acc->mem_num += (int64_t)q * (mhi - o.start);
   }

@@ -45,7 +45,7 @@ class GpuState(C.Structure):     # protean_gpu_state
                 ("has_vm", C.c_uint8), ("vm_type", C.c_uint8), ("pad", C.c_uint8 * 2),
                 ("recfg_start_us", C.c_int64), ("recfg_end_us", C.c_int64),
                 ("last_start_us", C.c_int64 * 7), ("busy_until_us", C.c_int64 * 7),
-                ("live", Resident * MAX_LIVE)]
+                ("busy_us", C.c_int64 * 7), ("live", Resident * MAX_LIVE)]
 
 
 class Placement(C.Structure):    # protean_placement, 24 B
@@ -57,12 +57,13 @@ class EpochIn(C.Structure):
     _fields_ = [("n_replicas", C.c_int32), ("n_gpus", C.c_int32), ("epoch", C.c_int32),
                 ("max_live", C.c_int32), ("epoch_len_us", C.c_int64), ("horizon_us", C.c_int64),
                 ("batches", C.c_void_p), ("batch_off", C.c_void_p), ("arrival_us", C.c_void_p),
-                ("state", C.c_void_p), ("geom_lo", C.c_int32), ("geom_hi", C.c_int32)]
+                ("state", C.c_void_p), ("geom_lo", C.c_int32), ("geom_hi", C.c_int32),
+                ("price_od_node_hr", C.c_double), ("price_spot_node_hr", C.c_double)]
 
 
 class EpochOut(C.Structure):
     _fields_ = [("best_key", C.c_void_p), ("cand_key", C.c_void_p), ("placement", C.c_void_p),
-                ("counters", C.c_void_p), ("accum", C.c_void_p)]
+                ("counters", C.c_void_p), ("accum", C.c_void_p), ("cost_usd", C.c_void_p)]
 
 
 class ReplayCfg(C.Structure):
@@ -108,8 +109,8 @@ assert C.sizeof(Batch) == 16 and C.sizeof(Resident) == 24 and C.sizeof(Placement
 assert C.sizeof(BatchRec) == 32
 
 EXPORTS = ["protean_load_profiles", "protean_free", "protean_strerror", "protean_last_error",
-           "protean_get_geometries", "protean_num_epochs", "protean_score_epoch",
-           "protean_replay_traces", "protean_replay_cfg_defaults", "protean_last_timings",
+           "protean_get_geometries", "protean_num_epochs", "protean_score_epoch", "protean_score_epoch_status",
+           "protean_replay_traces", "protean_replay_traces_host", "protean_replay_cfg_defaults", "protean_last_timings",
            "protean_geometry_split", "protean_xchg_export", "protean_xchg_import", "protean_xchg_attach"]
 IPC_HANDLE_BYTES = 64
 
@@ -134,10 +135,12 @@ def load(path: str = LIB_PATH, require_cuda: bool = True):
     L.protean_get_geometries.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p]
     L.protean_num_epochs.argtypes = [C.c_void_p, C.c_int64, C.c_int64, C.c_void_p]
     L.protean_score_epoch.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
+    L.protean_score_epoch_status.argtypes = [C.c_void_p]
     L.protean_sweep_assignments.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
     L.protean_form_batches.argtypes = [C.c_void_p, C.c_void_p, C.c_int32, C.c_int32, C.c_void_p, C.c_void_p,
                                        C.c_void_p, C.c_void_p, C.c_void_p, C.c_int64, C.c_void_p]
     L.protean_replay_traces.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
+    L.protean_replay_traces_host.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_int32, C.c_void_p]
     L.protean_replay_cfg_defaults.argtypes = [C.c_void_p]
     L.protean_replay_cfg_defaults.restype = None
     L.protean_last_timings.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]

@@ -147,6 +147,50 @@ class Handle:
         out["log_cap"] = int(log_cap)
         return out
 
+    def _cfg(self, R: int, trace_len_us: int, c: dict, arrival_ptr: int, meta_ptr: int, off_ptr: int):
+        cf = A.ReplayCfg()
+        self._lib.protean_replay_cfg_defaults(C.byref(cf))
+        cf.n_replicas, cf.n_gpus = R, int(c["n_gpus"])
+        cf.replica_base = int(c["replica_base"])
+        cf.trace_len_us = int(trace_len_us)
+        cf.epoch_len_us = int(c["epoch_len_us"])
+        cf.arrival_us, cf.meta, cf.replica_off = arrival_ptr, meta_ptr, off_ptr
+        for k in ("policy", "wait_limit", "reconfig_cap_pct", "init_geom", "max_live", "vm_policy",
+                  "reconfig_us", "rev_interval_us", "notice_us", "seed", "shard_mode", "rank", "nranks",
+                  "max_ctas", "ewma_alpha_pm", "t_low_milli", "t_high_milli", "cold_start_us",
+                  "keepalive_epochs", "prewarm", "ctas_per_replica"):
+            setattr(cf, k, int(c[k]))
+        for k in ("p_rev", "price_od_node_hr", "price_spot_node_hr"):
+            setattr(cf, k, float(c[k]))
+        return cf
+
+    @staticmethod
+    def _check_out(out: dict, R: int, E: int, N: int, G: int, device=None):
+        """The C ABI cannot check caller buffer sizes: assert every output's shape (and device)."""
+        want = dict(counters=(R, 10), accum=(R, 4), hist=(R, 2, A.NBUCKETS), p50_p99=(R, 2, 2), cost=(R,),
+                    util=(R, 2), n_batches=(R,), cold_starts=(R,), decisions=(R, E, N), cand_keys=(R, E, N, G))
+        for k, shp in want.items():
+            if k not in out:
+                continue
+            t = out[k]
+            assert tuple(t.shape) == shp, f"out[{k!r}] has shape {tuple(t.shape)}, expected {shp}"
+            assert t.is_contiguous(), f"out[{k!r}] is not contiguous"
+            if device is not None:
+                assert t.is_cuda and t.device.index == device, f"out[{k!r}] is not on cuda:{device}"
+            else:
+                assert not t.is_cuda, f"out[{k!r}] must be a host tensor"
+        if "log" in out:
+            assert out["log"].shape[0] == R and out["log"].shape[1] >= out.get("log_cap", 0)
+
+    def _out_struct(self, out: dict):
+        return A.ReplayOut(out["counters"].data_ptr(), out["accum"].data_ptr(), out["hist"].data_ptr(),
+                           out["p50_p99"].data_ptr(), out["cost"].data_ptr(), out["util"].data_ptr(),
+                           out["decisions"].data_ptr() if "decisions" in out else None,
+                           out["cand_keys"].data_ptr() if "cand_keys" in out else None,
+                           out["log"].data_ptr() if "log" in out else None, out.get("log_cap", 0),
+                           out["n_batches"].data_ptr() if "n_batches" in out else None,
+                           out["cold_starts"].data_ptr() if "cold_starts" in out else None)
+
     def replay_traces(self, arrival_us, meta, replica_off, *, trace_len_us: int, out=None,
                       want_decisions=True, want_cand_keys=False, log_cap=0, stream=None, **cfg):
         """protean_replay_traces on device tensors (arrival uint32/int32, meta uint8, off int64)."""
@@ -159,32 +203,13 @@ class Handle:
         if out is None:
             out = self.alloc_replay_out(R, E, N, decisions=want_decisions, cand_keys=want_cand_keys,
                                         log_cap=log_cap)
+        self._check_out(out, R, E, N, self.n_geoms, device=self.device)
         assert arrival_us.element_size() == 4 and meta.element_size() == 1 and replica_off.element_size() == 8
         for t in (arrival_us, meta, replica_off):
-            assert t.is_cuda and t.is_contiguous()
-        cf = A.ReplayCfg()
-        self._lib.protean_replay_cfg_defaults(C.byref(cf))
-        cf.n_replicas, cf.n_gpus = R, N
-        cf.replica_base = int(c["replica_base"])
-        cf.trace_len_us = int(trace_len_us)
-        cf.epoch_len_us = int(c["epoch_len_us"])
-        cf.arrival_us = arrival_us.data_ptr() if arrival_us.numel() else replica_off.data_ptr()
-        cf.meta = meta.data_ptr() if meta.numel() else replica_off.data_ptr()
-        cf.replica_off = replica_off.data_ptr()
-        for k in ("policy", "wait_limit", "reconfig_cap_pct", "init_geom", "max_live", "vm_policy",
-                  "reconfig_us", "rev_interval_us", "notice_us", "seed", "shard_mode", "rank", "nranks",
-                  "max_ctas", "ewma_alpha_pm", "t_low_milli", "t_high_milli", "cold_start_us",
-                  "keepalive_epochs", "prewarm", "ctas_per_replica"):
-            setattr(cf, k, int(c[k]))
-        for k in ("p_rev", "price_od_node_hr", "price_spot_node_hr"):
-            setattr(cf, k, float(c[k]))
-        o = A.ReplayOut(out["counters"].data_ptr(), out["accum"].data_ptr(), out["hist"].data_ptr(),
-                        out["p50_p99"].data_ptr(), out["cost"].data_ptr(), out["util"].data_ptr(),
-                        out["decisions"].data_ptr() if "decisions" in out else None,
-                        out["cand_keys"].data_ptr() if "cand_keys" in out else None,
-                        out["log"].data_ptr() if "log" in out else None, out.get("log_cap", 0),
-                        out["n_batches"].data_ptr(),
-                        out["cold_starts"].data_ptr() if "cold_starts" in out else None)
+            assert t.is_cuda and t.is_contiguous() and t.device.index == self.device
+        cf = self._cfg(R, trace_len_us, c, arrival_us.data_ptr() if arrival_us.numel() else replica_off.data_ptr(),
+                       meta.data_ptr() if meta.numel() else replica_off.data_ptr(), replica_off.data_ptr())
+        o = self._out_struct(out)
         st = stream if stream is not None else torch.cuda.current_stream(self.device)
         _check(self._h, self._lib.protean_replay_traces(self._h, C.byref(cf), C.byref(o),
                                                         C.c_void_p(st.cuda_stream)))
@@ -192,7 +217,8 @@ class Handle:
         return out
 
     def replay_traces_host(self, trace, *, pinned=None, stream=None, **cfg):
-        """End-to-end public call on HOST buffers: H2D of the trace, the replay, D2H of results."""
+        """A Trace (numpy) through the device call: H2D of the trace, the replay, D2H of results.
+        (Test convenience; the C-ABI host-buffer entry point is replay_traces_pinned.)"""
         torch = _torch()
         dev = torch.device("cuda", self.device)
         arr = torch.from_numpy(np.ascontiguousarray(trace.arrival_us).view(np.int32))
@@ -205,78 +231,53 @@ class Handle:
         out = self.replay_traces(d[0], d[1], d[2], trace_len_us=trace.trace_len_us, stream=stream, **cfg)
         return {k: (v.cpu().numpy() if hasattr(v, "cpu") else v) for k, v in out.items()}
 
-    def replay_traces_pinned(self, arrival_h, meta_h, off_h, *, trace_len_us: int, chunks: int = 4,
-                             out_host=None, stream=None, copy_stream=None, **cfg):
-        """End-to-end replay from PINNED host tensors with the PCIe transfers overlapped: the
-        replicas are cut into `chunks` contiguous ranges; chunk k+1's trace is copied host->device
-        on a copy stream while chunk k replays, and each chunk's results are copied back as soon as
-        it finishes.  Replicas are independent and keep their global ids (replica_base + r), so the
-        outputs equal one call over all replicas.  arrival_h int32/uint32 [n], meta_h uint8 [n],
-        off_h int64 [R+1] (host, pinned).  Returns pinned host output tensors."""
+    def alloc_host_out(self, R: int, E: int, N: int, *, decisions=True):
+        """Page-locked host output tensors for replay_traces_pinned."""
         torch = _torch()
-        dev = torch.device("cuda", self.device)
+        d = self.alloc_replay_out(1, 1, 1, decisions=False)
+        out = {k: torch.empty((R,) + tuple(v.shape[1:]), dtype=v.dtype).pin_memory() for k, v in d.items()
+               if hasattr(v, "shape")}
+        if decisions:
+            out["decisions"] = torch.empty((R, E, N), dtype=torch.uint8).pin_memory()
+        return out
+
+    def replay_traces_pinned(self, arrival_h, meta_h, off_h, *, trace_len_us: int, chunks: int = 4,
+                             out_host=None, stream=None, **cfg):
+        """protean_replay_traces_host (include/protean.h 3c): the end-to-end call on HOST tensors
+        (arrival int32/uint32 [n], meta uint8 [n], off int64 [R+1]; page-locked for overlap).  The
+        library cuts the replicas into `chunks` ranges and overlaps chunk k+1's H2D and chunk k-1's
+        D2H with chunk k's replay.  Returns the host output tensors (out_host, allocated pinned if
+        None)."""
+        torch = _torch()
         c = dict(_REPLAY_DEFAULTS)
         c.update(cfg)
         R = int(off_h.shape[0]) - 1
         N = int(c["n_gpus"])
         E = self.num_epochs(trace_len_us, c["epoch_len_us"])
-        base = int(c.pop("replica_base", 0))
-        st = stream if stream is not None else torch.cuda.current_stream(self.device)
-        cs = copy_stream if copy_stream is not None else torch.cuda.Stream(self.device)
-        offs = off_h.numpy()
-        chunks = max(1, min(int(chunks), R))  # every chunk holds at least one replica
-        bounds = [round(k * R / chunks) for k in range(chunks + 1)]
-        cap = max(int(offs[bounds[k + 1]] - offs[bounds[k]]) for k in range(chunks))
-        rcap = max(bounds[k + 1] - bounds[k] for k in range(chunks))
-        bufs = [(torch.empty(max(cap, 1), dtype=torch.int32, device=dev),
-                 torch.empty(max(cap, 1), dtype=torch.uint8, device=dev),
-                 torch.empty(rcap + 1, dtype=torch.int64, device=dev)) for _ in range(2)]
-        off_rel = [torch.from_numpy(offs[bounds[k]:bounds[k + 1] + 1] - offs[bounds[k]]).pin_memory()
-                   for k in range(chunks)]
-        dout = self.alloc_replay_out(R, E, N, decisions=True)
+        for t in (arrival_h, meta_h, off_h):
+            assert not t.is_cuda and t.is_contiguous()
+        assert arrival_h.element_size() == 4 and meta_h.element_size() == 1 and off_h.element_size() == 8
         if out_host is None:
-            out_host = {k: torch.empty(v.shape, dtype=v.dtype).pin_memory() for k, v in dout.items()
-                        if hasattr(v, "shape")}
-        ready = [torch.cuda.Event() for _ in range(chunks)]
-        freed = [torch.cuda.Event() for _ in range(chunks)]
-
-        def h2d(k):
-            b = bufs[k % 2]
-            if k >= 2:
-                cs.wait_event(freed[k - 2])  # the replay that used this buffer has finished
-            lo, hi = int(offs[bounds[k]]), int(offs[bounds[k + 1]])
-            with torch.cuda.stream(cs):
-                b[0][: hi - lo].copy_(arrival_h[lo:hi], non_blocking=True)
-                b[1][: hi - lo].copy_(meta_h[lo:hi], non_blocking=True)
-                b[2][: bounds[k + 1] - bounds[k] + 1].copy_(off_rel[k], non_blocking=True)
-            ready[k].record(cs)
-
-        h2d(0)
-        for k in range(chunks):
-            if k + 1 < chunks:
-                h2d(k + 1)  # overlaps chunk k's replay
-            st.wait_event(ready[k])
-            r0, r1 = bounds[k], bounds[k + 1]
-            b = bufs[k % 2]
-            n = int(offs[r1] - offs[r0])
-            view = {kk: v[r0:r1] for kk, v in dout.items() if hasattr(v, "shape")}
-            view["log_cap"] = 0
-            self.replay_traces(b[0][:max(n, 1)], b[1][:max(n, 1)], b[2][: r1 - r0 + 1], trace_len_us=trace_len_us,
-                               out=view, stream=st, replica_base=base + r0, **c)
-            freed[k].record(st)
-            with torch.cuda.stream(st):
-                for kk, v in view.items():
-                    if hasattr(v, "shape"):
-                        out_host[kk][r0:r1].copy_(v, non_blocking=True)
-        st.synchronize()
+            out_host = self.alloc_host_out(R, E, N)
+        self._check_out(out_host, R, E, N, self.n_geoms, device=None)
+        assert "cand_keys" not in out_host and "log" not in out_host
+        cf = self._cfg(R, trace_len_us, c, arrival_h.data_ptr() if arrival_h.numel() else off_h.data_ptr(),
+                       meta_h.data_ptr() if meta_h.numel() else off_h.data_ptr(), off_h.data_ptr())
+        o = self._out_struct(out_host)
+        st = stream if stream is not None else torch.cuda.current_stream(self.device)
+        _check(self._h, self._lib.protean_replay_traces_host(self._h, C.byref(cf), C.byref(o), int(chunks),
+                                                             C.c_void_p(st.cuda_stream)))
         return out_host
 
     # -------------------------------------------------------------------------------- score_epoch
     def score_epoch(self, *, n_replicas, n_gpus, epoch, batches, batch_off, arrival_us, state,
                     geom_lo=0, geom_hi=None, epoch_len_us=1_000_000, horizon_us=1 << 62, max_live=64,
-                    counters=None, accum=None, want_cand_keys=True, stream=None):
+                    counters=None, accum=None, want_cand_keys=True, price_od_node_hr=32.7726 / 8,
+                    price_spot_node_hr=9.8318 / 8, stream=None, sync=True):
         """protean_score_epoch.  batches: uint8 device tensor of protean_batch rows (16 B each);
-        state: uint8 device tensor of protean_gpu_state rows (modified in place)."""
+        state: uint8 device tensor of protean_gpu_state rows (modified in place).  The C call only
+        enqueues; with sync=True (default) the stream is synchronised and
+        protean_score_epoch_status raises the kernel's validation verdict, if any."""
         torch = _torch()
         dev = torch.device("cuda", self.device)
         geom_hi = self.n_geoms if geom_hi is None else geom_hi
@@ -286,20 +287,30 @@ class Handle:
         out = dict(best_key=torch.zeros(R * N, dtype=torch.int64, device=dev),
                    placement=torch.zeros((max(nb, 1), 24), dtype=torch.uint8, device=dev),
                    counters=counters if counters is not None else torch.zeros((R, 10), dtype=torch.int64, device=dev),
-                   accum=accum if accum is not None else torch.zeros((R, 4), dtype=torch.int64, device=dev))
+                   accum=accum if accum is not None else torch.zeros((R, 4), dtype=torch.int64, device=dev),
+                   cost=torch.zeros(R * N, dtype=torch.float64, device=dev))
         if want_cand_keys:
             out["cand_key"] = torch.zeros(R * N * max(nc, 1), dtype=torch.int64, device=dev)
         ei = A.EpochIn(R, N, int(epoch), int(max_live), int(epoch_len_us), int(horizon_us),
                        batches.data_ptr() if nb else out["placement"].data_ptr(), batch_off.data_ptr(),
                        arrival_us.data_ptr() if arrival_us.numel() else batch_off.data_ptr(),
-                       state.data_ptr(), int(geom_lo), int(geom_hi))
+                       state.data_ptr(), int(geom_lo), int(geom_hi), float(price_od_node_hr),
+                       float(price_spot_node_hr))
         eo = A.EpochOut(out["best_key"].data_ptr(), out["cand_key"].data_ptr() if want_cand_keys else None,
-                        out["placement"].data_ptr(), out["counters"].data_ptr(), out["accum"].data_ptr())
+                        out["placement"].data_ptr(), out["counters"].data_ptr(), out["accum"].data_ptr(),
+                        out["cost"].data_ptr())
         st = stream if stream is not None else torch.cuda.current_stream(self.device)
         _check(self._h, self._lib.protean_score_epoch(self._h, C.byref(ei), C.byref(eo),
                                                       C.c_void_p(st.cuda_stream)))
+        if sync:
+            st.synchronize()
+            self.score_epoch_status()
         out["placement"] = out["placement"][:nb]
         return out
+
+    def score_epoch_status(self):
+        """protean_score_epoch_status: raise the latched verdict of enqueued score_epoch calls."""
+        _check(self._h, self._lib.protean_score_epoch_status(self._h))
 
     def form_batches(self, arrival_us, meta, replica_off, *, trace_len_us: int, n_gpus: int, e_lo: int,
                      e_hi: int, avail=None, epoch_len_us: int = 1_000_000, stream=None):

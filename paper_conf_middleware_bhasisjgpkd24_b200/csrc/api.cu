@@ -38,7 +38,7 @@ struct protean_handle {
   size_t sa_bytes = 0;
   void* d_saoff = nullptr;
   size_t saoff_bytes = 0;
-  void* d_small = nullptr;  // wmax (8 B) + err (16 B)
+  void* d_small = nullptr;  // wmax (8 B) + err (16 B) at 64; score_epoch's latched verdict (8 B) at 256
   uint32_t* d_pack = nullptr;  // candidate lane packing for the full geometry range
   int CW = 0;
   // [0,1] prepass + partition count, [4,5] partition scan + scatter, [2,3] replay kernel
@@ -67,6 +67,11 @@ struct protean_handle {
   std::vector<char*> xpeer;              // every rank's buffer in this process
   std::vector<char> x_opened;            // 1 = opened through cudaIpcOpenMemHandle
   char** d_xpeer = nullptr;              // device copy of xpeer
+  // protean_replay_traces_host: double-buffered device staging of trace chunks and outputs
+  void* d_hb[2] = {nullptr, nullptr};
+  size_t hb_bytes[2] = {0, 0};
+  cudaStream_t hs_copy = nullptr, hs_back = nullptr;
+  cudaEvent_t hev[3][2] = {{nullptr, nullptr}, {nullptr, nullptr}, {nullptr, nullptr}};
 };
 
 namespace {
@@ -486,7 +491,8 @@ int protean_load_profiles(const protean_profiles* p, protean_handle** out) {
   if (e == cudaSuccess) e = cudaMalloc(&h->d_tab, sizeof(int32_t) * h->words.size());
   if (e == cudaSuccess)
     e = cudaMemcpy(h->d_tab, h->words.data(), sizeof(int32_t) * h->words.size(), cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMalloc(&h->d_small, 256);
+  if (e == cudaSuccess) e = cudaMalloc(&h->d_small, 512);
+  if (e == cudaSuccess) e = cudaMemset(h->d_small, 0, 512);  // [256, 264): score_epoch's latched verdict
   for (int i = 0; i < 6 && e == cudaSuccess; ++i) e = cudaEventCreate(&h->ev[i]);
   if (e == cudaSuccess) e = cudaMalloc(&h->d_pack, pack.size() * 4);
   if (e == cudaSuccess) e = cudaMemcpy(h->d_pack, pack.data(), pack.size() * 4, cudaMemcpyHostToDevice);
@@ -516,6 +522,13 @@ void protean_free(protean_handle* h) {
   xchg_release(h);
   for (int i = 0; i < 6; ++i)
     if (h->ev[i]) cudaEventDestroy(h->ev[i]);
+  for (int b = 0; b < 2; ++b) {
+    if (h->d_hb[b]) cudaFree(h->d_hb[b]);
+    for (int k = 0; k < 3; ++k)
+      if (h->hev[k][b]) cudaEventDestroy(h->hev[k][b]);
+  }
+  if (h->hs_copy) cudaStreamDestroy(h->hs_copy);
+  if (h->hs_back) cudaStreamDestroy(h->hs_back);
   delete h;
 }
 
@@ -933,20 +946,18 @@ int protean_score_epoch(protean_handle* h, const protean_epoch_in* in, protean_e
     return fail(h, PROTEAN_EINVAL, "geometry range");
   if (!in->batch_off || !in->state || !out->best_key || !out->counters || !out->placement)
     return fail(h, PROTEAN_EINVAL, "null pointer");
+  if (!(in->price_od_node_hr >= 0) || !(in->price_spot_node_hr >= 0)) return fail(h, PROTEAN_EINVAL, "price");
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   CK(h, cudaSetDevice(h->device));
   const int R = in->n_replicas, N = in->n_gpus, Gc = in->geom_hi - in->geom_lo;
-  int32_t b0 = 0;
-  CK(h, cudaMemcpyAsync(&b0, in->batch_off, 4, cudaMemcpyDeviceToHost, st));
-  CK(h, cudaStreamSynchronize(st));
-  if (b0 != 0) return fail(h, PROTEAN_EINVAL, "batch_off[0] != 0");
+  // enqueue-only: batch_off[0], the states and the batches are validated in the kernel, whose
+  // verdict is latched in the handle's device word (protean_score_epoch_status)
   const size_t need = sizeof(protean_resident) * (size_t)R * N * Gc * in->max_live;
   {
     int rc = ensure(h, &h->d_scratch, &h->scratch_bytes, std::max<size_t>(need, 256), st);
     if (rc) return rc;
   }
-  int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 64);
-  CK(h, cudaMemsetAsync(d_err, 0, 16, st));
+  int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 256);
   ScoreParams P;
   std::memset(&P, 0, sizeof(P));
   P.tab = h->d_tab;
@@ -968,16 +979,28 @@ int protean_score_epoch(protean_handle* h, const protean_epoch_in* in, protean_e
   P.placement = out->placement;
   P.counters = out->counters;
   P.accum = out->accum;
+  P.cost = out->cost_usd;
+  P.price_od = in->price_od_node_hr;
+  P.price_spot = in->price_spot_node_hr;
   P.scratch = static_cast<protean_resident*>(h->d_scratch);
   P.err = d_err;
   const int nl = N * (1 + Gc);
   int block = std::max(128, std::min(256, ((nl + 31) / 32) * 32));
   CK(h, launch_score(P, block, st));
+  return PROTEAN_OK;
+}
+
+int protean_score_epoch_status(protean_handle* h) {
+  if (!h) return PROTEAN_EINVAL;
+  if (h->poisoned) return PROTEAN_ESTATE;
+  CK(h, cudaSetDevice(h->device));
+  CK(h, cudaDeviceSynchronize());
   int errs[2] = {0, 0};
-  CK(h, cudaMemcpyAsync(errs, d_err, 8, cudaMemcpyDeviceToHost, st));
-  CK(h, cudaStreamSynchronize(st));
-  if (errs[0]) return fail(h, PROTEAN_EINVAL, "invalid state / batch");
-  if (errs[1]) return fail(h, PROTEAN_ERANGE, "n_live > max_live");
+  int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 256);
+  CK(h, cudaMemcpy(errs, d_err, 8, cudaMemcpyDeviceToHost));
+  CK(h, cudaMemset(d_err, 0, 8));
+  if (errs[0]) return fail(h, PROTEAN_EINVAL, "score_epoch: invalid state / batch / batch_off");
+  if (errs[1]) return fail(h, PROTEAN_ERANGE, "score_epoch: n_live > max_live");
   return PROTEAN_OK;
 }
 
@@ -1132,6 +1155,143 @@ int protean_form_batches(protean_handle* h, const protean_replay_cfg* cfg, int32
   if (sa_len) CK(h, cudaMemcpyAsync(members, h->d_sa, sizeof(uint32_t) * (size_t)sa_len, cudaMemcpyDeviceToDevice, st));
   CK(h, cudaStreamSynchronize(st));  // off lives on this stack frame
   cudaFreeAsync(dc, st);
+  return PROTEAN_OK;
+}
+
+
+// End-to-end replay from HOST buffers (include/protean.h section 3c).  Chunk k's trace bytes go
+// host -> device on the handle's copy stream while chunk k-1 replays on `stream`; chunk k's outputs
+// go device -> host on the handle's return stream while chunk k+1 replays.  Two staging slots,
+// each [trace arrivals | meta | relative offsets | per-replica outputs], alternate between chunks.
+int protean_replay_traces_host(protean_handle* h, const protean_replay_cfg* cfg, protean_replay_out* out,
+                               int32_t chunks, void* stream) {
+  if (!h) return PROTEAN_EINVAL;
+  if (h->poisoned) return PROTEAN_ESTATE;
+  if (!cfg || !out) return fail(h, PROTEAN_EINVAL, "null cfg/out");
+  const protean_replay_cfg& c = *cfg;
+  if (c.n_replicas < 1 || c.n_gpus < 1 || c.epoch_len_us <= 0 || c.trace_len_us <= 0)
+    return fail(h, PROTEAN_EINVAL, "sizes");
+  if (c.shard_mode != 0) return fail(h, PROTEAN_EINVAL, "host replay is mode R only");
+  if (!c.arrival_us || !c.meta || !c.replica_off) return fail(h, PROTEAN_EINVAL, "null trace");
+  if (!out->counters || !out->accum || !out->hist || !out->p50_p99_us || !out->cost_usd || !out->util)
+    return fail(h, PROTEAN_EINVAL, "null output");
+  if (out->cand_keys || out->batch_log) return fail(h, PROTEAN_EINVAL, "host replay: cand_keys / batch_log unsupported");
+  const int R = c.n_replicas, N = c.n_gpus;
+  const int64_t* roff = c.replica_off;  // host
+  if (roff[0] != 0) return fail(h, PROTEAN_EINVAL, "replica_off[0] != 0");
+  for (int r = 0; r < R; ++r)
+    if (roff[r + 1] < roff[r]) return fail(h, PROTEAN_EINVAL, "replica_off not monotone");
+  const int64_t W = c.epoch_len_us;
+  const int64_t E = (c.trace_len_us + W - 1) / W + ((int64_t)h->maxT + W - 1) / W;
+  const int K = std::max(1, std::min<int>(chunks < 1 ? 1 : chunks, R));
+  std::vector<int> bnd(K + 1);
+  for (int k = 0; k <= K; ++k) bnd[k] = (int)(((int64_t)k * R) / K);
+  int64_t cap = 1;
+  int rcap = 1;
+  for (int k = 0; k < K; ++k) {
+    cap = std::max<int64_t>(cap, roff[bnd[k + 1]] - roff[bnd[k]]);
+    rcap = std::max(rcap, bnd[k + 1] - bnd[k]);
+  }
+  // staging slot layout (256-byte aligned pieces)
+  size_t o = 0;
+  const size_t o_arr = o; o += al((size_t)cap * 4);
+  const size_t o_meta = o; o += al((size_t)cap);
+  const size_t o_off = o; o += al((size_t)(rcap + 1) * 8);
+  const size_t o_cnt = o; o += al((size_t)rcap * 10 * 8);
+  const size_t o_acc = o; o += al((size_t)rcap * 4 * 8);
+  const size_t o_hist = o; o += al((size_t)rcap * 2 * PROTEAN_NBUCKETS * 4);
+  const size_t o_pct = o; o += al((size_t)rcap * 4 * 8);
+  const size_t o_cost = o; o += al((size_t)rcap * 8);
+  const size_t o_util = o; o += al((size_t)rcap * 2 * 8);
+  const size_t o_dec = o; o += al(out->decisions ? (size_t)rcap * E * N : 0);
+  const size_t o_nb = o; o += al((size_t)rcap * 8);
+  const size_t o_cold = o; o += al((size_t)rcap * 8);
+  const size_t slot = o;
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  CK(h, cudaSetDevice(h->device));
+  if (!h->hs_copy) CK(h, cudaStreamCreateWithFlags(&h->hs_copy, cudaStreamNonBlocking));
+  if (!h->hs_back) CK(h, cudaStreamCreateWithFlags(&h->hs_back, cudaStreamNonBlocking));
+  for (int k = 0; k < 3; ++k)
+    for (int b = 0; b < 2; ++b)
+      if (!h->hev[k][b]) CK(h, cudaEventCreateWithFlags(&h->hev[k][b], cudaEventDisableTiming));
+  for (int b = 0; b < 2; ++b) {
+    int rc = ensure(h, &h->d_hb[b], &h->hb_bytes[b], slot, st);
+    if (rc) return rc;
+  }
+  CK(h, cudaStreamSynchronize(st));  // the staging slots are allocated before the copy stream uses them
+  // hev[0][b]: slot b's trace is on the device; hev[1][b]: slot b's replay finished;
+  // hev[2][b]: slot b's outputs are back on the host (the slot may be refilled)
+  std::vector<std::vector<int64_t>> rel(K);
+  auto h2d = [&](int k) -> int {
+    const int b = k & 1;
+    char* d = static_cast<char*>(h->d_hb[b]);
+    if (k >= 2) CK(h, cudaStreamWaitEvent(h->hs_copy, h->hev[2][b], 0));
+    const int64_t lo = roff[bnd[k]], n = roff[bnd[k + 1]] - lo;
+    rel[k].resize(bnd[k + 1] - bnd[k] + 1);
+    for (int r = bnd[k]; r <= bnd[k + 1]; ++r) rel[k][r - bnd[k]] = roff[r] - lo;
+    if (n > 0) {
+      CK(h, cudaMemcpyAsync(d + o_arr, c.arrival_us + lo, (size_t)n * 4, cudaMemcpyHostToDevice, h->hs_copy));
+      CK(h, cudaMemcpyAsync(d + o_meta, c.meta + lo, (size_t)n, cudaMemcpyHostToDevice, h->hs_copy));
+    }
+    CK(h, cudaMemcpyAsync(d + o_off, rel[k].data(), rel[k].size() * 8, cudaMemcpyHostToDevice, h->hs_copy));
+    CK(h, cudaEventRecord(h->hev[0][b], h->hs_copy));
+    return PROTEAN_OK;
+  };
+  int rc = h2d(0);
+  if (rc) return rc;
+  float t_pre = 0.f, t_rep = 0.f;
+  for (int k = 0; k < K; ++k) {
+    const int b = k & 1;
+    if (k + 1 < K) {
+      rc = h2d(k + 1);  // overlaps chunk k's replay
+      if (rc) return rc;
+    }
+    char* d = static_cast<char*>(h->d_hb[b]);
+    const int r0 = bnd[k], rn = bnd[k + 1] - bnd[k];
+    protean_replay_cfg cc = c;
+    cc.n_replicas = rn;
+    cc.replica_base = c.replica_base + r0;
+    cc.arrival_us = reinterpret_cast<const uint32_t*>(d + o_arr);
+    cc.meta = reinterpret_cast<const uint8_t*>(d + o_meta);
+    cc.replica_off = reinterpret_cast<const int64_t*>(d + o_off);
+    protean_replay_out oo;
+    std::memset(&oo, 0, sizeof(oo));
+    oo.counters = reinterpret_cast<int64_t*>(d + o_cnt);
+    oo.accum = reinterpret_cast<int64_t*>(d + o_acc);
+    oo.hist = reinterpret_cast<uint32_t*>(d + o_hist);
+    oo.p50_p99_us = reinterpret_cast<int64_t*>(d + o_pct);
+    oo.cost_usd = reinterpret_cast<double*>(d + o_cost);
+    oo.util = reinterpret_cast<double*>(d + o_util);
+    oo.decisions = out->decisions ? reinterpret_cast<uint8_t*>(d + o_dec) : nullptr;
+    oo.n_batches = reinterpret_cast<int64_t*>(d + o_nb);
+    oo.cold_starts = reinterpret_cast<int64_t*>(d + o_cold);
+    CK(h, cudaStreamWaitEvent(st, h->hev[0][b], 0));
+    rc = protean_replay_traces(h, &cc, &oo, stream);
+    if (rc) return rc;
+    t_pre += h->t_prepass;
+    t_rep += h->t_replay;
+    CK(h, cudaEventRecord(h->hev[1][b], st));
+    CK(h, cudaStreamWaitEvent(h->hs_back, h->hev[1][b], 0));
+    auto back = [&](void* dst, size_t off, size_t bytes) -> int {
+      if (dst && bytes) CK(h, cudaMemcpyAsync(dst, d + off, bytes, cudaMemcpyDeviceToHost, h->hs_back));
+      return PROTEAN_OK;
+    };
+    const size_t n = (size_t)rn;
+    if ((rc = back(out->counters + (size_t)r0 * 10, o_cnt, n * 80))) return rc;
+    if ((rc = back(out->accum + (size_t)r0 * 4, o_acc, n * 32))) return rc;
+    if ((rc = back(out->hist + (size_t)r0 * 2 * PROTEAN_NBUCKETS, o_hist, n * 2 * PROTEAN_NBUCKETS * 4))) return rc;
+    if ((rc = back(out->p50_p99_us + (size_t)r0 * 4, o_pct, n * 32))) return rc;
+    if ((rc = back(out->cost_usd + r0, o_cost, n * 8))) return rc;
+    if ((rc = back(out->util + (size_t)r0 * 2, o_util, n * 16))) return rc;
+    if (out->decisions && (rc = back(out->decisions + (size_t)r0 * E * N, o_dec, n * E * N))) return rc;
+    if (out->n_batches && (rc = back(out->n_batches + r0, o_nb, n * 8))) return rc;
+    if (out->cold_starts && (rc = back(out->cold_starts + r0, o_cold, n * 8))) return rc;
+    CK(h, cudaEventRecord(h->hev[2][b], h->hs_back));
+  }
+  CK(h, cudaStreamSynchronize(h->hs_back));
+  CK(h, cudaStreamSynchronize(h->hs_copy));
+  h->t_prepass = t_pre;
+  h->t_replay = t_rep;
   return PROTEAN_OK;
 }
 

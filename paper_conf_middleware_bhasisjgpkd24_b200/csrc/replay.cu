@@ -1779,6 +1779,23 @@ cudaError_t launch_replay(const ReplayParams& P, int grid, int block, cudaStream
     if (n3) k = wide ? replay_kernel<false, true, 4> : replay_kernel<false, true, 1>;
     else k = wide ? replay_kernel<false, false, 4> : replay_kernel<false, false, 1>;
   }
+  if (P.vr_n > 1) {
+    // virtual ranks: the CTAs of a replica spin on each other's exchange flags, so the whole grid
+    // must be co-resident; a cooperative launch guarantees it or fails at launch (instead of a
+    // 30 s exchange timeout under MPS or concurrent work).  Mode G ranks (separate launches that
+    // must run side by side) keep the plain launch and the timeout.
+    cudaLaunchConfig_t lc = {};
+    lc.gridDim = dim3((unsigned)grid);
+    lc.blockDim = dim3((unsigned)block);
+    lc.dynamicSmemBytes = P.sl.total;
+    lc.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeCooperative;
+    at[0].val.cooperative = 1;
+    lc.attrs = at;
+    lc.numAttrs = 1;
+    return cudaLaunchKernelEx(&lc, k, P);
+  }
   k<<<grid, block, P.sl.total, st>>>(P);
   return cudaGetLastError();
 }

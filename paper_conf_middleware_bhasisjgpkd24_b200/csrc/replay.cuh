@@ -153,8 +153,10 @@ struct ScoreParams {
   protean_placement* placement;
   int64_t* counters;
   int64_t* accum;
+  double* cost;               // [R*N] node-epoch VM cost, or NULL
+  double price_od, price_spot;
   protean_resident* scratch;  // [R][N*(Gc)][max_live]
-  int* err;                   // err[0] EINVAL, err[1] ERANGE
+  int* err;                   // err[0] EINVAL, err[1] ERANGE (latched until protean_score_epoch_status)
 };
 
 // protean_form_batches (form.cu): batch formation + round-robin dispatch on the stream-sorted copy

@@ -26,7 +26,7 @@ __global__ void __launch_bounds__(256) score_kernel(ScoreParams P) {
     const int x = r * N + g;
     protean_gpu_state& st = P.state[x];
     bool inval = st.geom >= T.G || (st.target != 0xFF && st.target >= T.G) ||
-                 P.batch_off[x + 1] < P.batch_off[x];
+                 P.batch_off[x + 1] < P.batch_off[x] || P.batch_off[0] != 0 || st.vm_type > 2;
     const bool range = st.n_live > P.max_live;
     if (!inval && !range) {
       for (int i = 0; i < st.n_live; ++i)
@@ -55,9 +55,13 @@ __global__ void __launch_bounds__(256) score_kernel(ScoreParams P) {
       st.target = 0xFF;
       st.wait_ctr = 0;
       st.n_live = 0;
-      for (int s = 0; s < kMaxSl; ++s) st.last_start_us[s] = st.busy_until_us[s] = 0;
+      for (int s = 0; s < kMaxSl; ++s) st.last_start_us[s] = st.busy_until_us[s] = st.busy_us[s] = 0;
     }
     dec[g] = (st.has_vm && st.recfg_end_us <= Tend) ? 1 : 0;
+    if (P.cost) {  // node-epoch VM cost: price(vm_type) * W / 3.6e9 (T3 P:L173-179, Q35)
+      const double price = !st.has_vm ? 0.0 : st.vm_type == 1 ? P.price_od : st.vm_type == 2 ? P.price_spot : 0.0;
+      P.cost[r * N + g] = __ddiv_rn(__dmul_rn(price, (double)P.W), 3.6e9);
+    }
   }
   __syncthreads();
 
@@ -73,9 +77,13 @@ __global__ void __launch_bounds__(256) score_kernel(ScoreParams P) {
       Rows rows{st.live};
       const int geom = st.geom;
       int n = st.n_live;
-      int64_t ls[kMaxSl], bu[kMaxSl];
+      int64_t ls[kMaxSl], bu[kMaxSl], bs[kMaxSl];
 #pragma unroll
-      for (int s = 0; s < kMaxSl; ++s) { ls[s] = st.last_start_us[s]; bu[s] = st.busy_until_us[s]; }
+      for (int s = 0; s < kMaxSl; ++s) {
+        ls[s] = st.last_start_us[s];
+        bu[s] = st.busy_until_us[s];
+        bs[s] = st.busy_us[s];
+      }
       for (int b = b0; b < b1; ++b) {
         const protean_batch& bt = P.batches[b];
         const PlaceRes pr = place_lane(T, geom, rows, n, ls, bt.ready_us, bt.model, bt.strict != 0,
@@ -105,7 +113,10 @@ __global__ void __launch_bounds__(256) score_kernel(ScoreParams P) {
           if (s == pr.slice) {
             const int64_t lo = pr.start > bu[s] ? pr.start : bu[s];
             const int64_t hi = pr.end < P.H ? pr.end : P.H;
-            if (hi > lo) busy += (unsigned long long)((int64_t)prof_compute(p) * (hi - lo));
+            if (hi > lo) {
+              busy += (unsigned long long)((int64_t)prof_compute(p) * (hi - lo));
+              bs[s] += hi - lo;
+            }
             if (pr.end > bu[s]) bu[s] = pr.end;
           }
         }
@@ -114,7 +125,11 @@ __global__ void __launch_bounds__(256) score_kernel(ScoreParams P) {
       }
       st.n_live = (uint8_t)n;
 #pragma unroll
-      for (int s = 0; s < kMaxSl; ++s) { st.last_start_us[s] = ls[s]; st.busy_until_us[s] = bu[s]; }
+      for (int s = 0; s < kMaxSl; ++s) {
+        st.last_start_us[s] = ls[s];
+        st.busy_until_us[s] = bu[s];
+        st.busy_us[s] = bs[s];
+      }
     } else {
       const int j = P.geom_lo + v - 1;
       int64_t key = -1;

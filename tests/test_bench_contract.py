@@ -40,3 +40,16 @@ def test_our_arm_line(extra):
     assert r["bound"] in ("hbm", "alu") and 0 < r["frac"] < 1 and r["peak"] > 0
     assert d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] > 0
     assert d["gpu_launches"] > 0 and "sm_mhz" in d["clocks"]
+
+
+def test_gpus_flag_relaunches_one_process_per_rank():
+    """--gpus N outside torchrun re-launches bench.py through torch.distributed.run (ADVICE r1:
+    the flag used to be parsed and ignored); the reference arm prints one line from rank 0 with
+    n_gpus = N.  A WORLD_SIZE that contradicts --gpus fails loudly."""
+    d = _run(["--impl", "reference", "--gpus", "2", "--replicas", "2", "--seconds", "5", "--steps", "1",
+              "--warmup", "0"])
+    assert d["impl"] == "reference" and d["n_gpus"] == 2
+    env = dict(os.environ, WORLD_SIZE="3", RANK="0", LOCAL_RANK="0")
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--gpus", "2"],
+                         capture_output=True, text=True, timeout=300, cwd=ROOT, env=env)
+    assert out.returncode != 0 and "WORLD_SIZE" in out.stderr

@@ -193,6 +193,7 @@ def test_score_epoch_fuzz(oracle, seed):
         for t in np.sort(rng.integers(eW - 400_000, eW, size=int(rng.integers(0, 5)))):
             oracle.place(prof, s, int(t), int(rng.integers(0, M)), int(rng.integers(0, 2)))
         s.has_vm = int(rng.random() < 0.85)
+        s.vm_type = int(rng.integers(0, 3))
         if rng.random() < 0.3:
             s.target = int(rng.integers(0, G))
             s.recfg_start = eW - 500_000
@@ -200,9 +201,11 @@ def test_score_epoch_fuzz(oracle, seed):
         ostates[x] = s
         gs = gstates[x]
         gs.geom, gs.target, gs.n_live, gs.has_vm = s.geom, 255 if s.target < 0 else s.target, s.n_res, s.has_vm
+        gs.vm_type = s.vm_type
         gs.recfg_start_us, gs.recfg_end_us = s.recfg_start, s.recfg_end
         for i in range(7):
             gs.last_start_us[i], gs.busy_until_us[i] = s.last_start[i], s.busy_until[i]
+            gs.busy_us[i] = s.busy_us[i]
         for i in range(s.n_res):
             rr = s.res[i]
             gs.live[i] = A.Resident(rr.start, rr.end, rr.mem, rr.slice, rr.model, rr.strict, 0)
@@ -235,6 +238,7 @@ def test_score_epoch_fuzz(oracle, seed):
     assert g["cand_key"].cpu().tolist() == o["cand_key"].tolist()
     assert g["counters"].cpu().numpy().tolist() == o["counters"].tolist()
     assert g["accum"].cpu().numpy()[:, :2].tolist() == o["accum"][:, :2].tolist()
+    assert g["cost"].cpu().numpy().tolist() == o["cost"].tolist()  # bit-equal doubles
     pl = g["placement"].cpu().numpy()
     for i in range(nb):
         p = A.Placement.from_buffer_copy(pl[i].tobytes())
@@ -250,6 +254,7 @@ def test_score_epoch_fuzz(oracle, seed):
                 (b.start, b.end, b.mem, b.slice, b.model, b.strict)
         assert list(st[x].last_start_us) == list(ostates[x].last_start)
         assert list(st[x].busy_until_us) == list(ostates[x].busy_until)
+        assert list(st[x].busy_us) == list(ostates[x].busy_us)
 
 
 @pytest.mark.parametrize("seed", range(3))

@@ -95,3 +95,50 @@ def test_unaligned_device_buffers(oracle, shift):
     ref = gpu_replay(prof, tr, n_gpus=3)
     for k in ("counters", "hist", "cand_keys"):
         assert np.array_equal(g[k], ref[k]), k
+
+
+def test_score_epoch_enqueue_only_verdict(oracle):
+    """protean_score_epoch only enqueues: an invalid state (geometry >= G) or batch_off[0] != 0 is
+    latched in the handle's device word and raised by protean_score_epoch_status after the sync
+    (SURVEY.md §8(b) "score_epoch enqueues on stream and returns"); the oracle rejects the same
+    input with the same code; a valid call afterwards reports OK (the word is cleared)."""
+    import torch
+    import paper_conf_middleware_bhasisjgpkd24_b200 as pkg
+    from paper_conf_middleware_bhasisjgpkd24_b200 import _abi as A
+    from helpers import w1
+    _, P, _ = w1()
+    dev = torch.device("cuda", 0)
+    h = pkg.load_profiles(P)
+    rows = np.zeros((4, 16), np.uint8)
+    for i, (rd, off, m, s) in enumerate([(5000, 0, 1, 0), (10000, 2, 0, 1), (30000, 4, 1, 0), (45000, 6, 0, 1)]):
+        rows[i] = np.frombuffer(bytes(A.Batch(rd, off, 2, m, s, 0)), np.uint8)
+    arr = torch.tensor(np.array([0, 5000, 0, 10000, 20000, 30000, 40000, 45000], np.int32), device=dev)
+
+    def call(geom, off0):
+        st = A.GpuState()
+        st.geom, st.target, st.has_vm, st.vm_type = geom, 255, 1, 1
+        t_state = torch.from_numpy(np.frombuffer(bytes(st), np.uint8).copy()).to(dev)
+        t_off = torch.tensor([off0, 4], dtype=torch.int32, device=dev)
+        out = h.score_epoch(n_replicas=1, n_gpus=1, epoch=0, batches=torch.from_numpy(rows.reshape(-1)).to(dev),
+                            batch_off=t_off, arrival_us=arr, state=t_state, sync=False)
+        torch.cuda.synchronize()
+        try:
+            h.score_epoch_status()
+        except pkg.ProteanError as e:
+            return e.code, out
+        return 0, out
+
+    code, _ = call(h.n_geoms, 0)
+    assert code == A.EINVAL
+    code, _ = call(2, 1)
+    assert code == A.EINVAL
+    code, out = call(2, 0)
+    assert code == 0
+    assert out["cand_key"].cpu().tolist() == [56320001, 64000002, 78080000]  # W1 golden
+    assert out["cost"].cpu().tolist() == [(32.7726 / 8 * 1e6) / 3.6e9]
+    ostate = (oracle.State * 1)()
+    ostate[0].geom, ostate[0].target, ostate[0].has_vm = P.geoms.shape[0], -1, 1
+    with pytest.raises(oracle.OracleError) as ei:
+        oracle.score_epoch(P, R=1, N=1, epoch=0, batches=dict(ready=[5000], req_off=[0], n=[2], model=[1], strict=[0]),
+                           batch_off=[0, 1], arrival=np.array([0, 5000], np.uint32), states=ostate)
+    assert ei.value.code == A.EINVAL

@@ -366,6 +366,28 @@ def test_score_epoch_matches_w1(oracle):
     assert [[s, a, b] for s, a, b in zip(out["slice"], out["start"], out["end"])] == ex["actual_placement_j2"]
     assert out["counters"][0, 8] == ex["slot_evals_epoch0"] and out["counters"][0, 9] == 3
     assert states[0].n_res == 4  # all four batches stay resident (every end > the epoch start)
+    # per-slice busy union (O6e): 1g [5000,305000), 2g [30000,230000), 4g [10000,165000) (W1)
+    assert list(states[0].busy_us) == [300_000, 200_000, 155_000, 0, 0, 0, 0]
+    assert out["accum"][0, 0] == g["expected"]["accum_busy_weighted"]
+
+
+def test_score_epoch_node_cost_closed_form(oracle):
+    """Node-epoch VM cost = price(vm_type) x W (T3; cost projection P:L333; Q27 per-node
+    price = T3 / 8): 8 nodes x 3600 one-second epochs on-demand sum to T3's AWS $32.7726 per hour,
+    all spot to $9.8318 (the "70% lower cost" ratio 0.300001); no VM -> 0."""
+    g, P, tr = w1()
+    per = {}
+    for vm, has in ((1, 1), (2, 1), (1, 0), (0, 1)):
+        states = (oracle.State * 1)()
+        states[0].geom, states[0].target, states[0].has_vm, states[0].vm_type = 2, -1, has, vm
+        out = oracle.score_epoch(P, R=1, N=1, epoch=0, batches=dict(ready=[], req_off=[], n=[], model=[], strict=[]),
+                                 batch_off=[0, 0], arrival=np.zeros(0, np.uint32), states=states,
+                                 price_od=32.7726 / 8, price_spot=9.8318 / 8)
+        per[(vm, has)] = float(out["cost"][0])
+    assert per[(1, 0)] == 0.0 and per[(0, 1)] == 0.0
+    assert 8 * 3600 * per[(1, 1)] == pytest.approx(32.7726, rel=1e-12)
+    assert 8 * 3600 * per[(2, 1)] == pytest.approx(9.8318, rel=1e-12)
+    assert per[(2, 1)] / per[(1, 1)] == pytest.approx(0.300001, abs=5e-7)
 
 
 # ---------------------------------------------------------------- hysteresis (T6) + cap (T7)
@@ -602,3 +624,14 @@ def test_utilisation_across_reconfiguration(oracle):
     assert out["accum"][0, 0] == u["busy_weighted"]
     assert out["accum"][0, 1] == u["mem_time"]
     assert out["util"][0].tolist() == pytest.approx(u["util"], rel=1e-12)
+
+
+def test_w1_workload_self_check_stats(oracle):
+    """The h5 self-check counters on W1, hand-counted: 2 decidable GPU-epochs, 1 with
+    best != current (epoch 0: (7g) vs (4g,2g,1g)); 24 (batch, feasible slice) candidate evaluations,
+    9 with Eq 1's F > 10^6: (7g) a1 1.3, b2 2.1, a2 2.6; (4g,3g) a1@3g 1.3, b2@3g 1.6, b2@4g 1.3,
+    a2@3g 2.1 (a2@4g is exactly 1.0); (4g,2g,1g) b2@4g 1.3, a2@2g 1.3 (the 1g starts wait until b1
+    ends at 305,000 and run alone)."""
+    _, P, tr = w1()
+    out = oracle.replay(P, tr, N=1, init_geom=2)
+    assert out["stats"][0].tolist() == [2, 1, 9, 24]

@@ -1,17 +1,19 @@
-"""Stall-reason breakdown per kernel phase of an ncu report (source page, cuda,sass view)."""
+"""Stall-reason breakdown per code region of replay.cu from an ncu report (source page, cuda,sass
+view).  Regions are the kernel's '// ----' phase markers AND every device function definition
+(tools/ncu_regions.regions), so helper bodies above the kernel (place_group, candidate_unit_fast,
+exchange_keys, ...) are attributed to themselves, not to the marker that precedes them."""
 import collections
 import csv
 import os
 import subprocess
 import sys
 
-SRC = os.path.join(os.path.dirname(__file__), "..", "paper_conf_middleware_bhasisjgpkd24_b200", "csrc", "replay.cu")
+sys.path.insert(0, os.path.dirname(__file__))
+from ncu_regions import regions  # noqa: E402
 
 
 def main(rep):
-    src = open(SRC).read().split("\n")
-    marks = [(i + 1, l.split("----")[-1].strip()[:28]) for i, l in enumerate(src)
-             if "// ----------------------------------------------------------------" in l]
+    marks = regions()
     txt = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
                          capture_output=True, text=True).stdout
     hdr, fname = None, None
@@ -29,7 +31,7 @@ def main(rep):
             d = dict(zip(hdr[2:], row[2:]))
             k = fname
             if fname == "replay.cu":
-                k = "helpers"
+                k = "?"
                 for i, name in marks:
                     if int(row[0]) >= i:
                         k = name
@@ -40,7 +42,7 @@ def main(rep):
     for k, c in sorted(agg.items(), key=lambda x: -sum(x[1].values())):
         s = sum(c.values())
         top = ", ".join(f"{n} {100 * v / tot:.1f}" for n, v in c.most_common(4))
-        print(f"{100 * s / tot:5.1f}%  {k:28s} {top}")
+        print(f"{100 * s / tot:5.1f}%  {k:30s} {top}")
 
 
 if __name__ == "__main__":

@@ -33,3 +33,6 @@ ev[1].record()
 torch.cuda.synchronize()
 print(os.path.basename(sys.argv[2]) if len(sys.argv) > 2 else "libprotean.so", "assignments",
       int(out["n_assign"].item()), "ms", round(ev[0].elapsed_time(ev[1]) / reps, 2))
+if os.environ.get("SWEEP_INFO"):
+    import json
+    json.dump({"replicas": R, "assignments": int(out["n_assign"].item())}, open(os.environ["SWEEP_INFO"], "w"))
