@@ -26,14 +26,14 @@ int check_geometry_row(const uint8_t* row, std::vector<int>* g) {
     last = row[i];
     cnt[row[i]]++;
     compute += kCompute[row[i]];
-    mem += kMemMiB[row[i]];
+    mem += kMemEighths[row[i]];
     g->push_back(row[i]);
     ++k;
   }
   if (k == 0) return ORC_EINVAL;
   for (int p = 0; p < kProfiles; ++p)
     if (cnt[p] > kMaxCount[p]) return ORC_EINVAL;
-  if (compute > 7 || mem > 40960) return ORC_EINVAL;
+  if (compute > 7 || mem > 8) return ORC_EINVAL;  // <= 7/7 of the SMs, <= 8/8 of the memory (T2)
   return ORC_OK;
 }
 
@@ -42,12 +42,16 @@ int build_tables(const orc_tables* t, Tables* tb) {
   if (t->M < 1 || t->M > 64) return ORC_EINVAL;
   if (!t->solo || !t->fbr || !t->mem || !t->bsz || !t->slo || !t->tmo) return ORC_EINVAL;
   const int M = t->M;
+  const int32_t gmem = t->gpu_mem_mib == 0 ? kA100Mem : t->gpu_mem_mib;
+  if (gmem < 8 || gmem % 8 != 0 || gmem > (1 << 24)) return ORC_EINVAL;
+  tb->gpu_mem = gmem;
+  for (int p = 0; p < kProfiles; ++p) tb->cap_mem[p] = gmem / 8 * kMemEighths[p];
   for (int i = 0; i < M * kProfiles; ++i) {
     if (t->solo[i] <= 0) return ORC_EINVAL;
     if (t->fbr[i] < 0 || t->fbr[i] > 1000000) return ORC_EINVAL;
   }
   for (int m = 0; m < M; ++m) {
-    if (t->mem[m] < 1 || t->mem[m] > 40960) return ORC_EINVAL;
+    if (t->mem[m] < 1 || t->mem[m] > gmem) return ORC_EINVAL;
     if (t->bsz[m] < 1 || t->bsz[m] > 65535) return ORC_EINVAL;
     if (t->slo[m] <= 0 || t->tmo[m] < 0) return ORC_EINVAL;
   }
@@ -211,7 +215,7 @@ int orc_tick_simulate(const orc_tables* t, int32_t geom, int32_t nb, const int64
   std::vector<TickBatch> bs(nb);
   for (int i = 0; i < nb; ++i) {
     if (slice[i] < 0 || slice[i] >= (int)g.size()) return ORC_EINVAL;
-    if (tb.mem[model[i]] > kMemMiB[g[slice[i]]]) return ORC_EINVAL;
+    if (tb.mem[model[i]] > tb.cap(g[slice[i]])) return ORC_EINVAL;
     if (i > 0 && t_ready[i] < t_ready[i - 1]) return ORC_EINVAL;
     bs[i].t = t_ready[i];
     bs[i].m = model[i];

@@ -295,7 +295,7 @@ struct Replay {
           std::vector<int> chosen;
           for (const std::vector<int>& ss : small_slice_set) {
             int64_t sum_max_mem = 0;
-            for (int p : ss) sum_max_mem += kMemMiB[p];
+            for (int p : ss) sum_max_mem += tb.cap(p);
             if (sum_max_mem * 1000 >= g.pred_mem) {
               chosen = ss;
               found = true;
@@ -420,7 +420,7 @@ struct Replay {
     }
     out->cost = ((double)out->accum[2] * cfg.price_od + (double)out->accum[3] * cfg.price_spot) / 3.6e9;
     out->util[0] = (double)out->accum[0] / (7.0 * (double)N * (double)H);
-    out->util[1] = (double)out->accum[1] / (40960.0 * (double)N * (double)H);
+    out->util[1] = (double)out->accum[1] / ((double)tb.gpu_mem * (double)N * (double)H);
   }
 };
 }  // namespace

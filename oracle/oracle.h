@@ -21,6 +21,8 @@ typedef struct {
   int32_t geometry_set;           /* 0: 12 multiset-maximal, 1: all 37, 2: explicit */
   int32_t n_geoms;
   const uint8_t *geoms;           /* explicit: [G][8] */
+  int32_t gpu_mem_mib;            /* N4c: GPU memory (0 = A100-40GB 40960); profile p holds
+                                     gpu_mem * {1,2,4,4,8}[p] / 8; multiple of 8, <= 2^24 */
 } orc_tables;
 
 typedef struct { int64_t start, end; int32_t mem, slice, model, strict; } orc_res;  /* 32 B */

@@ -27,7 +27,8 @@ def build(force: bool = False) -> str:
 class Tables(C.Structure):
     _fields_ = [("M", C.c_int32), ("solo", C.c_void_p), ("fbr", C.c_void_p), ("mem", C.c_void_p),
                 ("bsz", C.c_void_p), ("slo", C.c_void_p), ("tmo", C.c_void_p),
-                ("geometry_set", C.c_int32), ("n_geoms", C.c_int32), ("geoms", C.c_void_p)]
+                ("geometry_set", C.c_int32), ("n_geoms", C.c_int32), ("geoms", C.c_void_p),
+                ("gpu_mem_mib", C.c_int32)]
 
 
 class Res(C.Structure):
@@ -135,7 +136,7 @@ class OTables:
         self.geoms = None if prof.geoms is None else np.ascontiguousarray(prof.geoms, np.uint8)
         self.s = Tables(int(self.arrs[0].shape[0]), *[a.ctypes.data for a in self.arrs],
                         int(prof.geometry_set), 0 if self.geoms is None else int(self.geoms.shape[0]),
-                        _p(self.geoms))
+                        _p(self.geoms), int(getattr(prof, "gpu_mem_mib", 0)))
 
     @property
     def ref(self):

@@ -20,7 +20,8 @@ namespace pem {
 // ---- T2: profiles 1g,2g,3g,4g,7g in ascending-resource order (reading Q3) ------
 constexpr int kProfiles = 5;
 constexpr int kCompute[kProfiles] = {1, 2, 3, 4, 7};                  // sevenths of the SMs
-constexpr int32_t kMemMiB[kProfiles] = {5120, 10240, 20480, 20480, 40960};  // 5/10/20/20/40 GB
+constexpr int kMemEighths[kProfiles] = {1, 2, 4, 4, 8};               // memory slices of 8 (T2)
+constexpr int32_t kA100Mem = 40960;                                    // A100-40GB: 5/10/20/20/40 GB
 constexpr int kMaxCount[kProfiles] = {7, 3, 2, 1, 1};
 constexpr int kMaxSlices = 7;
 constexpr int64_t kPpm = 1000000;               // FBR 1.0 ("0.2 -> 20%")
@@ -35,6 +36,11 @@ struct Tables {
   std::vector<int32_t> solo, fbr;               // [M*5]
   std::vector<int32_t> mem, bsz, slo, tmo;      // [M]
   std::vector<std::vector<int>> geoms;          // candidate geometries: profile ids ascending
+  // N4c (P:L495 generalizability; NVIDIA MIG tables, not in the paper): the GPU's memory; a
+  // profile holds eighths_p / 8 of it (A100-40GB 40960 MiB -> 5120/10240/20480/20480/40960)
+  int32_t gpu_mem = kA100Mem;
+  int32_t cap_mem[kProfiles] = {5120, 10240, 20480, 20480, 40960};
+  int32_t cap(int p) const { return cap_mem[p]; }
   int32_t solo_at(int m, int p) const { return solo[m * kProfiles + p]; }
   int32_t fbr_at(int m, int p) const { return fbr[m * kProfiles + p]; }
 };

@@ -37,7 +37,7 @@ PlaceOut place(const Tables& tb, const std::vector<int>& geom, GpuState& S, int6
   // (b) completion with Eq 1 evaluated at that start instant (reading Q8, Q9).
   for (int s = 0; s < k; ++s) {
     const int p = geom[s];
-    const int32_t Ms = kMemMiB[p];
+    const int32_t Ms = tb.cap(p);
     if (q > Ms) continue;  // the batch can never fit this slice
     o.feasible[s] = true;
 
@@ -83,7 +83,7 @@ PlaceOut place(const Tables& tb, const std::vector<int>& geom, GpuState& S, int6
       if (!r.strict) be_mem += r.mem;
     int64_t R = be_mem;
     for (int s = 0; s < k; ++s) {
-      const int32_t Ms = kMemMiB[geom[s]];
+      const int32_t Ms = tb.cap(geom[s]);
       if (R >= Ms) {  // tag_value == 1: completely occupied by BE
         o.eligible[s] = false;
         R -= Ms;

@@ -26,7 +26,7 @@ PlaceOut place_forced(const Tables& tb, const std::vector<int>& geom, GpuState& 
     return o;
   }
   const int p = geom[slice];
-  const int32_t Ms = kMemMiB[p];
+  const int32_t Ms = tb.cap(p);
   const int32_t q = tb.mem[m];
   if (q > Ms) {
     o.dropped = 2;

@@ -30,7 +30,7 @@ void tick_simulate(const Tables& tb, const std::vector<int>& geom, std::vector<T
         int h = queue[s].front();
         int64_t used = 0;
         for (int i : running[s]) used += tb.mem[bs[i].m];
-        if (used + tb.mem[bs[h].m] > kMemMiB[p]) break;
+        if (used + tb.mem[bs[h].m] > tb.cap(p)) break;
         int64_t F = tb.fbr_at(bs[h].m, p);
         for (int i : running[s]) F += tb.fbr_at(bs[i].m, p);
         int64_t f = F < kPpm ? kPpm : F;

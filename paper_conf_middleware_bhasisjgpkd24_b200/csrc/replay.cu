@@ -56,6 +56,8 @@ namespace pemgpu {
 
 namespace {
 
+constexpr int kMaxWarps = 32;
+
 // Per-lane resident list, interleaved across lanes (entry i of lane l at i*stride + l) so that a
 // warp walking its lists in lock-step issues coalesced loads.  mm = mem | model << 16 | strict << 22.
 struct LaneList {
@@ -99,6 +101,7 @@ struct CtaState {
   int glo, ghi, cw, xrank;  // this CTA's candidate geometry range, its candidate warps per GPU and
                             // its rank in the key exchange (virtual ranks: several CTAs per replica)
   int wtot;
+  int nact;                 // active streams of the epoch (s_act)
   unsigned long long cold;  // N3 cold starts of the replica          // window entries copied this epoch (incl. alignment padding)
   unsigned long long cnt[10];
 };
@@ -513,6 +516,7 @@ __device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, const
 }
 
 constexpr int kKR = 6;  // batches per GPU-epoch handled by the register fast path
+constexpr int kAK = 4;  // batch ranks per accounting task (phase F)
 
 // Candidate unit, fast path: the GPU-epoch's <= kKR batches fully unrolled, times 32-bit relative to
 // the first batch's ready time tb.  Every lane of a geometry's group keeps the whole placement so
@@ -627,6 +631,31 @@ __device__ __forceinline__ bool candidate_unit_fast(const Tab& T, const SliceLan
 
 }  // namespace
 
+// Fold the per-warp request counters of the epoch (phase F) into the replica's 64-bit counters
+// 0..6 (O7) and clear them; called by all lanes of warp 0 after the phase-E barrier.
+__device__ __forceinline__ void fold_wcnt(CtaState& cs, uint32_t (*wcnt)[5], int NW, int lane) {
+  uint32_t v = 0;
+  if (lane < 5) {
+#pragma unroll 1
+    for (int w = 0; w < NW; ++w) {
+      v += wcnt[w][lane];
+      wcnt[w][lane] = 0;
+    }
+  }
+  const uint32_t sarr = __shfl_sync(0xffffffffu, v, 0), met = __shfl_sync(0xffffffffu, v, 1);
+  const uint32_t sdrop = __shfl_sync(0xffffffffu, v, 2), barr = __shfl_sync(0xffffffffu, v, 3);
+  const uint32_t bdrop = __shfl_sync(0xffffffffu, v, 4);
+  if (lane == 0) {
+    cs.cnt[0] += sarr;
+    cs.cnt[1] += met;
+    cs.cnt[2] += sarr - met - sdrop;
+    cs.cnt[3] += sdrop;
+    cs.cnt[4] += barr;
+    cs.cnt[5] += barr - bdrop;
+    cs.cnt[6] += bdrop;
+  }
+}
+
 // Policy 2 (N1): Alg 2 GPU_Reconfigurator lines 1-23 for decidable GPU g, readings
 // R10-R15 of DESIGN.md.  Returns final_geometry; advances the GPU's EWMA history (gi rows 12, 13).
 __device__ __forceinline__ int alg2_final_geometry(const ReplayParams& P, const Ctx& c, int g,
@@ -664,10 +693,15 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
   __shared__ CtaState cs;
   __shared__ uint32_t s_hist[2 * kNB];  // 2 classes x 3328 buckets (u32 < 2^32 per replica)
   __shared__ uint32_t s_sink;           // target of increments with nothing to count
+  // per-warp request counters of the current epoch (O7): strict arrivals, strict met, strict
+  // dropped, BE arrivals, BE dropped; each warp adds only to its own row (no atomics), warp 0 folds
+  // them into the 64-bit replica counters once per epoch (an epoch holds < 2^25 requests)
+  __shared__ uint32_t s_wcnt[kMaxWarps][5];
   const uint32_t sink = (uint32_t)__cvta_generic_to_shared(&s_sink);
   __shared__ __align__(8) uint64_t s_mbar;  // TMA bulk-copy completion of the epoch's window
   __shared__ int s_base[kMaxStreams], s_tot[kMaxStreams], s_cur[kMaxStreams], s_pend[kMaxStreams];
   __shared__ int s_dst[kMaxStreams], s_alo[kMaxStreams], s_asz[kMaxStreams];
+  __shared__ uint8_t s_act[kMaxStreams];  // streams with requests in this epoch's window (phase C)
 #ifdef PROTEAN_PHASE_TIMING
   unsigned long long ph_acc[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
   long long ph_last = clock64();
@@ -761,6 +795,8 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
 #pragma unroll 1
     for (int i = tid; i < 2 * kNB; i += NT) s_hist[i] = 0;
 #pragma unroll 1
+    for (int i = tid; i < kMaxWarps * 5; i += NT) (&s_wcnt[0][0])[i] = 0;
+#pragma unroll 1
     for (int k = tid; k < S; k += NT) s_cur[k] = (int)P.sidx[(size_t)r * (P.E + 1) * S + k];
 #pragma unroll 1
     for (int g = tid; g < N; g += NT) {
@@ -828,7 +864,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
       const uint32_t* sa_r = P.sa + P.saoff[r];
       if (warp == 0) {
         const uint32_t* s1 = P.sidx + ((size_t)r * (P.E + 1) + e + 1) * S;
-        int carry = 0;
+        int carry = 0, nact = 0;
 #pragma unroll 1
         for (int k0 = 0; k0 < S; k0 += 32) {
           const int k = k0 + lane;
@@ -857,7 +893,11 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
             s_dst[k] = dst;
             s_alo[k] = alo;
             s_asz[k] = asz;
+            s_pend[k] = 0;
           }
+          const unsigned am = __ballot_sync(0xffffffffu, k < S && len > 0);
+          if (k < S && len > 0) s_act[nact + __popc(am & ((1u << lane) - 1u))] = (uint8_t)k;
+          nact += __popc(am);
           carry += __shfl_sync(0xffffffffu, x, 31);
         }
         const bool overflow = carry > P.WCAP;  // cannot happen for a valid trace (host bound)
@@ -865,6 +905,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
           for (int k = lane; k < S; k += 32) s_tot[k] = 0;
           if (lane == 0) atomicOr(P.err, 1);
         }
+        if (lane == 0) cs.nact = overflow ? 0 : nact;
         const int tot = overflow ? 0 : carry;
         if (lane == 0) cs.wtot = tot;
         if (win_smem && tot > 0) {
@@ -910,8 +951,10 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
       // ---------------------------------------------------------------- C: batch formation
       // warp per stream: lanes test 32 consecutive B-sized batches at once (full batches are the
       // common case); a batch closed by the timeout, or still open, is resolved by lane 0.
+      const int nact = cs.nact;
 #pragma unroll 1
-      for (int k = warp; k < S; k += NW) {
+      for (int ka = warp; ka < nact; ka += NW) {
+        const int k = s_act[ka];
         const int m = k >> 1;
         const bool strict = (k & 1) == 0;
         const int B = T.bsz[m];
@@ -1154,7 +1197,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
       // dynamic task queue: [actual units][candidate units][accounting of batch rank rk];
       // accounting waits (rarely) for the actual units, whose warps publish via cs.adone
       const int n_units = n_aunits + (P.policy == 0 ? N * cs.cw : 0);
-      const int n_tasks = n_units + nb;
+      const int n_tasks = n_units + (nb + kAK - 1) / kAK;
       for (;;) {
         int u = 0;
         if (lane == 0) u = atomicAdd(&cs.task, 1);
@@ -1168,78 +1211,89 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
           __device__ ~TaskClock() { if (lane == 0) atomicAdd(&acc[kind], (unsigned long long)(clock64() - t0)); }
         } tclock{tk0, tkind, lane, g_phase_cycles + 10};
 #endif
-        if (u >= n_units) {  // ---- F: accounting (O7) of batch rank u - n_units
+        if (u >= n_units) {  // ---- F: accounting (O7) of batch ranks [kAK t, kAK t + kAK)
+          // acquire the actual units' batch results (slice, start, end, drop): lane 0's acquire
+          // load, then the warp barrier orders it before every lane's reads (PTX memory model:
+          // release/acquire at CTA scope + bar.warp.sync)
           if (lane == 0) {
-            while (*(volatile int*)&cs.adone < n_aunits) __nanosleep(64);
+            const uint32_t fa = (uint32_t)__cvta_generic_to_shared(&cs.adone);
+            for (;;) {
+              int v;
+              asm volatile("ld.acquire.cta.shared::cta.s32 %0, [%1];" : "=r"(v) : "r"(fa) : "memory");
+              if (v >= n_aunits) break;
+              __nanosleep(64);
+            }
           }
           __syncwarp();
-          __threadfence_block();
-          const int rk = u - n_units;
-          const Bat& bt = bats[ord[rk]];
-          const int nreq = bt.info & 0xFFFF, m = (bt.info >> 16) & 0xFF;
-          const bool strict = (bt.info >> 24) & 1;
-          if (lane == 0) {
-            const int64_t row = cs.nlog + rk;
-            if (P.log && row < P.log_cap) {
-              protean_batch_rec rec;
-              rec.ready_us = bt.ready;
-              rec.epoch = (uint32_t)e;
-              rec.n_req = (uint16_t)nreq;
-              rec.model = (uint8_t)m;
-              rec.strict = strict ? 1 : 0;
-              rec.gpu = bt.gpu;
-              rec.slice = bt.slice;
-              rec.dropped = bt.drop;
-              rec.pad = 0;
-              rec.start_us = bt.start;
-              rec.end_us = bt.end;
-              P.log[(size_t)r * P.log_cap + row] = rec;
-            }
-          }
-          int met = 0;  // strict members within the SLO (lane 0's count)
-          if (!bt.drop) {
-            const int64_t slo = T.slo[m];
-            const int cls = strict ? 0 : kNB;
-            const uint32_t* ma = sarr + bt.pos;
-            const int64_t bend = bt.end;
-            const uint32_t hb = (uint32_t)__cvta_generic_to_shared(s_hist + cls);
-            if (bend - (int64_t)ma[0] <= (int64_t)0xFFFFFFFFLL) {
-              // every latency end - a (>= 0, <= end - a_first) fits 32 bits: lat = end - a mod 2^32;
-              // bucket = 128 s + (lat >> s), s = max(0, floor(log2 lat) - 7) (O7, reading Q30)
-              const uint32_t e32 = (uint32_t)bend;
-              const uint32_t slo32 = slo > (int64_t)0xFFFFFFFFLL ? 0xFFFFFFFFu : (uint32_t)slo;
+          const int rk0 = (u - n_units) * kAK, rk1 = min(nb, rk0 + kAK);
+          uint32_t c_sarr = 0, c_met = 0, c_sdrop = 0, c_barr = 0, c_bdrop = 0;  // warp-uniform
 #pragma unroll 1
-              for (int i0 = 0; i0 < nreq; i0 += 32) {
-                const int i = i0 + lane;
-                const bool valid = i < nreq;
-                const uint32_t lat = e32 - ma[valid ? i : 0];
-                const int sh = max(24 - __clz(lat), 0);
-                inc_shared(valid ? hb + 4u * (uint32_t)((sh << 7) + (int)(lat >> sh)) : sink);
-                met += __popc(__ballot_sync(0xffffffffu, valid && lat <= slo32));
-              }
-            } else {  // some latency >= 2^32 us: the saturating 64-bit bucket
-#pragma unroll 1
-              for (int i0 = 0; i0 < nreq; i0 += 32) {
-                const int i = i0 + lane;
-                const bool valid = i < nreq;
-                const int64_t lat = bend - (int64_t)ma[valid ? i : 0];
-                inc_shared(valid ? hb + 4u * (uint32_t)lat_bucket(lat) : sink);
-                met += __popc(__ballot_sync(0xffffffffu, valid && lat <= slo));
+          for (int rk = rk0; rk < rk1; ++rk) {
+            const Bat& bt = bats[ord[rk]];
+            const uint32_t info = bt.info;
+            const int nreq = info & 0xFFFF, m = (info >> 16) & 0xFF;
+            const bool strict = (info >> 24) & 1;
+            const int drop = bt.drop;
+            if (P.log && lane == 0) {
+              const int64_t row = cs.nlog + rk;
+              if (row < P.log_cap) {
+                protean_batch_rec rec;
+                rec.ready_us = bt.ready;
+                rec.epoch = (uint32_t)e;
+                rec.n_req = (uint16_t)nreq;
+                rec.model = (uint8_t)m;
+                rec.strict = strict ? 1 : 0;
+                rec.gpu = bt.gpu;
+                rec.slice = bt.slice;
+                rec.dropped = (uint8_t)drop;
+                rec.pad = 0;
+                rec.start_us = bt.start;
+                rec.end_us = bt.end;
+                P.log[(size_t)r * P.log_cap + row] = rec;
               }
             }
-          }
-          if (lane == 0) {
+            uint32_t met = 0;  // strict members within the SLO
+            if (!drop) {
+              const int64_t slo = T.slo[m];
+              const uint32_t* ma = sarr + bt.pos;
+              const int64_t bend = bt.end;
+              const uint32_t hb = (uint32_t)__cvta_generic_to_shared(s_hist + (strict ? 0 : kNB));
+              if (bend - (int64_t)ma[0] <= (int64_t)0xFFFFFFFFLL) {
+                // every latency end - a (>= 0, <= end - a_first) fits 32 bits: lat = end - a mod 2^32;
+                // bucket = 128 s + (lat >> s), s = max(0, floor(log2 lat) - 7) (O7, reading Q30)
+                const uint32_t e32 = (uint32_t)bend;
+                const uint32_t slo32 = slo > (int64_t)0xFFFFFFFFLL ? 0xFFFFFFFFu : (uint32_t)slo;
+#pragma unroll 4
+                for (int i0 = 0; i0 < nreq; i0 += 32) {
+                  const int i = i0 + lane;
+                  const bool valid = i < nreq;
+                  const uint32_t lat = e32 - ma[valid ? i : 0];
+                  const int sh = max(24 - __clz(lat), 0);
+                  inc_shared(valid ? hb + 4u * (uint32_t)((sh << 7) + (int)(lat >> sh)) : sink);
+                  met += __popc(__ballot_sync(0xffffffffu, valid && lat <= slo32));
+                }
+              } else {  // some latency >= 2^32 us: the saturating 64-bit bucket
+#pragma unroll 1
+                for (int i0 = 0; i0 < nreq; i0 += 32) {
+                  const int i = i0 + lane;
+                  const bool valid = i < nreq;
+                  const int64_t lat = bend - (int64_t)ma[valid ? i : 0];
+                  inc_shared(valid ? hb + 4u * (uint32_t)lat_bucket(lat) : sink);
+                  met += __popc(__ballot_sync(0xffffffffu, valid && lat <= slo));
+                }
+              }
+            }
             if (strict) {
-              atomicAdd(&cs.cnt[0], (unsigned long long)nreq);
-              if (bt.drop) atomicAdd(&cs.cnt[3], (unsigned long long)nreq);
-              else {
-                atomicAdd(&cs.cnt[1], (unsigned long long)met);
-                atomicAdd(&cs.cnt[2], (unsigned long long)(nreq - met));
-              }
+              c_sarr += nreq;
+              if (drop) c_sdrop += nreq; else c_met += met;
             } else {
-              atomicAdd(&cs.cnt[4], (unsigned long long)nreq);
-              atomicAdd(&cs.cnt[bt.drop ? 6 : 5], (unsigned long long)nreq);
+              c_barr += nreq;
+              if (drop) c_bdrop += nreq;
             }
+          }
+          if (lane < 5) {
+            const uint32_t v = lane == 0 ? c_sarr : lane == 1 ? c_met : lane == 2 ? c_sdrop : lane == 3 ? c_barr : c_bdrop;
+            s_wcnt[warp][lane] += v;
           }
           continue;
         }
@@ -1294,11 +1348,16 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
         int64_t ls = actual && valid ? c.a_ls[al] : 0;
         int64_t bu = actual && valid ? c.a_bu[al] : 0;
         const int x0 = valid ? c.g_off[g] : 0, x1 = valid ? c.g_off[g + 1] : 0;
-        int len_max = x1 - x0;
+        int len_max;
+        if (actual) {  // up to AG GPUs per warp: the longest batch list of the warp's GPUs
+          len_max = x1 - x0;
 #pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-          const int o = __shfl_xor_sync(0xffffffffu, len_max, d);
-          len_max = o > len_max ? o : len_max;
+          for (int d = 1; d < 32; d <<= 1) {
+            const int o = __shfl_xor_sync(0xffffffffu, len_max, d);
+            len_max = o > len_max ? o : len_max;
+          }
+        } else {       // one GPU per candidate warp: uniform
+          len_max = c.g_off[g + 1] - c.g_off[g];
         }
         int64_t misses, tail;
         // register fast path (warp-uniform batch range: idle lanes still take part in the shuffles);
@@ -1400,10 +1459,10 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
             c.gi[10 * c.N + g] += bsum;
             c.gi[11 * c.N + g] += msum;
           }
-          __syncwarp();
+          __syncwarp();  // every lane's batch-result stores precede lane 0's release below
           if (lane == 0) {
-            __threadfence_block();
-            atomicAdd(&cs.adone, 1);
+            const uint32_t fa = (uint32_t)__cvta_generic_to_shared(&cs.adone);
+            asm volatile("red.release.cta.shared::cta.add.s32 [%0], 1;" ::"r"(fa) : "memory");
           }
         } else if (valid && lane == gbase) {
           const int64_t key = make_key(acc0, acc1, j == c.gu8[0 * c.N + g] ? 0 : j + 1);
@@ -1428,6 +1487,8 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
           const bool gv = g < N;
           bool want = false;
           int64_t kb = kForever, kc = -1;
+          uint32_t scored_b = 0;  // batches of this GPU scored by every candidate (counters 8, 9)
+          bool scored = false;
           if (gv) {
             uint8_t dec_out = kNoGeom;
             if (P.policy != 1 && c.gu8[5 * c.N + g]) {
@@ -1440,8 +1501,8 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
                 kc = c.gi[7 * c.N + g];
                 const int tag = (int)(kb & 255);
                 best = tag == 0 ? cur : tag - 1;
-                atomicAdd(&cs.cnt[8], (unsigned long long)(c.g_off[g + 1] - c.g_off[g]) * (unsigned long long)sum_slots);
-                atomicAdd(&cs.cnt[9], (unsigned long long)(cs.ghi - cs.glo));
+                scored_b = (uint32_t)(c.g_off[g + 1] - c.g_off[g]);
+                scored = true;
               } else {  // policy 2: Alg 2's own heuristic (N1)
                 if constexpr (kAlg2) best = alg2_final_geometry(P, c, g, c.bats, c.gl);
                 else best = cur;  // unreachable: policy 2 launches replay_kernel<true, *, *>
@@ -1464,6 +1525,15 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
                 P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = -1;
             }
           }
+          {  // counters 8, 9 (O8): slot-evals = sum over scored GPUs of batches x slots of the range
+            const uint32_t tb = __reduce_add_sync(0xffffffffu, scored_b);  // <= nb < 2^25
+            const int nsc = __popc(__ballot_sync(0xffffffffu, scored));
+            if (lane == 0) {
+              cs.cnt[8] += (unsigned long long)tb * (unsigned long long)sum_slots;
+              cs.cnt[9] += (unsigned long long)nsc * (unsigned long long)(cs.ghi - cs.glo);
+            }
+          }
+          fold_wcnt(cs, s_wcnt, NW, lane);
           if (P.policy != 1) {
             const unsigned alive = __ballot_sync(0xffffffffu, gv && has_vm(c, g, Tend));
             const unsigned open = __ballot_sync(0xffffffffu, gv && c.gi[1 * c.N + g] > Tend);
@@ -1551,6 +1621,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
       }
       __syncthreads();
       PH(8);
+      if (warp == 0) fold_wcnt(cs, s_wcnt, NW, lane);
       if (tid == 0) {
         if (P.policy != 1) {
           int alive = 0, open = 0;

@@ -34,6 +34,7 @@ class Profiles:
     geometry_set: int = 0
     geoms: np.ndarray | None = None   # uint8 [G,8] for geometry_set == 2
     names: tuple = ()
+    gpu_mem_mib: int = 0              # N4c: GPU memory (0 = A100-40GB, 40960 MiB)
 
     @property
     def n_models(self) -> int:
