@@ -82,7 +82,7 @@ typedef struct {
   int32_t n_models;                /* M, 1..64 */
   const int32_t *solo_us;          /* [M][5] solo (isolated) batch exec time per profile, > 0 */
   const int32_t *fbr_ppm;          /* [M][5] fractional bandwidth requirement per profile, 0..10^6 */
-  const int32_t *mem_mib;          /* [M] memory footprint of one batch, 1..40960 */
+  const int32_t *mem_mib;          /* [M] memory footprint of one batch, 1..gpu_mem_mib (40960) */
   const int32_t *batch_size;       /* [M] B_m, 1..65535 (128 vision, 4 language) */
   const int32_t *slo_us;           /* [M] strict SLO, > 0 (paper: 3 x solo on 7g) */
   const int32_t *batch_timeout_us; /* [M] T_m >= 0: a batch closes at B_m requests or first+T_m (Q14) */
@@ -93,6 +93,15 @@ typedef struct {
   const uint8_t *geoms;            /* explicit only: [G][8] profile ids ascending, 0xFF padded;
                                       each validated against T2 (counts, compute <= 7/7, mem <= 40 GB) */
   int32_t device;                  /* CUDA device ordinal */
+  int32_t gpu_mem_mib;             /* N4c, MIG profile table of the simulated GPU (P:L495
+                                      "Generalizability"; NVIDIA's MIG tables, not in the paper):
+                                      its memory in MiB, a multiple of 8, <= 2^24.  Profile p holds
+                                      gpu_mem * {1,2,4,4,8}[p] / 8 MiB; compute sevenths, max counts
+                                      and hence the geometry sets are T2's.  0 = A100-40GB (40960);
+                                      81920 = A100-80GB / H100-80GB, 144384 = H200-141GB,
+                                      184320 = B200-180GB (nominal GiB x 1024).  The double-memory
+                                      1g profiles (1g.20gb, 1g.45gb) are not modelled.  Footprints
+                                      (mem_mib) must be <= gpu_mem_mib; mem utilisation divides by it. */
 } protean_profiles;
 
 /* Validates the tables, enumerates the geometry set (canonical order: count vectors
@@ -380,6 +389,29 @@ typedef struct {
  * ERANGE (a GPU with more than max_batches batches).  With several faults, the code of one. */
 int protean_sweep_assignments(protean_handle *h, const protean_sweep_in *in, protean_sweep_out *out,
                               void *stream);
+
+/* ---------------------------------------------------------------------------------------------
+ * 3c'. BE-reserve depth sweep (N4b; SURVEY §8(f) N4 "BE-reserve depth as an enumerated dimension";
+ *     reading R28 of DESIGN.md).  Alg 1 lines 1-8 tag slices from the BE memory in
+ *     ascending order and choose_strict_slice avoids the BE-full ones.  Here the reserve is
+ *     an enumerated parameter instead: for every (replica, sim-GPU) and every geometry j in
+ *     [geom_lo, geom_hi), the GPU-epoch's batches are replayed from idle with Alg 1's greedy Place
+ *     (O6) under depth code c: c = 0 keeps the tag walk, c = 1 + d reserves the d smallest slices for
+ *     BE (strict eligible on positions >= d; with none eligible, every fitting slice, as Q6), for
+ *     d = 0 .. S_j - 1; each replay is scored with the O8 key (tag 0 = current geometry).  Code 0 is
+ *     exactly protean_score_epoch's candidate key.  Same input as the assignment sweep (3b);
+ *     max_batches is ignored (no batch-count limit).  Synchronous.  Device pointers.
+ *     Errors: EINVAL (sizes, range, null pointers, batch_off, model id, n_req, unsorted ready or
+ *     members, cur_geom >= G).                                                                  */
+typedef struct {
+  int64_t *depth_key;   /* [R*N*(hi-lo)][8] key per depth code (-1 for codes beyond S_j), or NULL */
+  uint8_t *depth_code;  /* [R*N*(hi-lo)] the minimising code (lowest among equal keys), or NULL */
+  int64_t *best_key;    /* [R*N] min over the range and every code */
+  int64_t *n_eval;      /* [1] ACCUMULATED (+=): replays scored, sum over (GPU, j) of S_j + 1 */
+} protean_depth_out;
+
+int protean_sweep_depths(protean_handle *h, const protean_sweep_in *in, protean_depth_out *out,
+                         void *stream);
 
 /* ---------------------------------------------------------------------------------------------
  * 4. Mode G: geometry-range sharding with one min-loc exchange per replica-epoch (SURVEY §8(e),

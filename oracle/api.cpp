@@ -505,6 +505,60 @@ int orc_score_epoch(const orc_tables* t, int32_t R, int32_t N, int32_t epoch, in
   return ORC_OK;
 }
 
+int orc_sweep_depths(const orc_tables* t, int32_t R, int32_t N, int32_t max_live,
+              const uint32_t* b_ready, const uint32_t* b_req_off, const int32_t* b_n,
+              const int32_t* b_model, const int32_t* b_strict, const int32_t* batch_off,
+              const uint32_t* arrival, const uint8_t* cur_geom, int32_t geom_lo, int32_t geom_hi,
+              int64_t* depth_key, uint8_t* depth_code, int64_t* best_key, int64_t* n_eval) {
+  Tables tb;
+  int rc = build_tables(t, &tb);
+  if (rc) return rc;
+  const int G = (int)tb.geoms.size();
+  if (R < 1 || N < 1) return ORC_EINVAL;
+  if (N > 255) return ORC_ERANGE;
+  if (max_live < 1 || max_live > 64) return ORC_EINVAL;
+  if (geom_lo < 0 || geom_hi > G || geom_lo >= geom_hi) return ORC_EINVAL;
+  if (!batch_off || !cur_geom || !best_key || !n_eval) return ORC_EINVAL;
+  if (batch_off[0] != 0) return ORC_EINVAL;
+  for (int x = 0; x < R * N; ++x) {
+    if (batch_off[x + 1] < batch_off[x]) return ORC_EINVAL;
+    if (cur_geom[x] != 0xFF && cur_geom[x] >= G) return ORC_EINVAL;
+    for (int32_t b = batch_off[x]; b < batch_off[x + 1]; ++b) {
+      if (b_model[b] < 0 || b_model[b] >= tb.M || b_n[b] < 1) return ORC_EINVAL;
+      if (b > batch_off[x] && b_ready[b] < b_ready[b - 1]) return ORC_EINVAL;
+      for (int i = 0; i < b_n[b]; ++i) {
+        uint32_t a = arrival[b_req_off[b] + i];
+        if (a > b_ready[b] || (i > 0 && a < arrival[b_req_off[b] + i - 1])) return ORC_EINVAL;
+      }
+    }
+  }
+  const int nc = geom_hi - geom_lo;
+  uint64_t total = 0;
+  for (int x = 0; x < R * N; ++x) {
+    std::vector<SweepBatch> bs;
+    for (int32_t b = batch_off[x]; b < batch_off[x + 1]; ++b) {
+      SweepBatch sb;
+      sb.ready = b_ready[b];
+      sb.model = b_model[b];
+      sb.strict = b_strict[b] != 0;
+      sb.arr.assign(arrival + b_req_off[b], arrival + b_req_off[b] + b_n[b]);
+      bs.push_back(sb);
+    }
+    best_key[x] = -1;
+    for (int j = geom_lo; j < geom_hi; ++j) {
+      int64_t keys[8], key;
+      int code;
+      sweep_depths(tb, j, cur_geom[x] == j ? 0 : j + 1, bs, max_live, keys, &key, &code, &total);
+      if (depth_key)
+        for (int c = 0; c < 8; ++c) depth_key[((int64_t)x * nc + (j - geom_lo)) * 8 + c] = keys[c];
+      if (depth_code) depth_code[(int64_t)x * nc + (j - geom_lo)] = (uint8_t)code;
+      if (best_key[x] < 0 || key < best_key[x]) best_key[x] = key;
+    }
+  }
+  *n_eval += (int64_t)total;
+  return ORC_OK;
+}
+
 int orc_sweep(const orc_tables* t, int32_t R, int32_t N, int32_t max_live, int32_t max_batches,
               const uint32_t* b_ready, const uint32_t* b_req_off, const int32_t* b_n,
               const int32_t* b_model, const int32_t* b_strict, const int32_t* batch_off,

@@ -133,6 +133,15 @@ int orc_form_dispatch(const orc_tables *t, int32_t R, int32_t N, int64_t W, int6
  * [geom_lo, geom_hi) the min key over every assignment of the GPU's batches (<= max_batches <= 8)
  * to j's slices, scheduled from idle with the slice forced; assign = slice of batch x in bits
  * 3x..3x+2 of the lowest-index minimiser; best_key = min over the range, tag 0 when j == cur_geom. */
+/* N4b: BE-reserve depths (reading R28): per (replica, gpu, geometry j in range) the keys of Alg 1
+ * replays from idle with strict eligibility "position >= d" for d = 0..S_j-1, plus the tag walk
+ * (code 0); depth_key [R*N*nc][8] (code 0 = auto, 1 + d; -1 beyond S_j), depth_code = argmin code
+ * (ties -> lowest code), best_key = min over the range; n_eval += replays. */
+int orc_sweep_depths(const orc_tables *t, int32_t R, int32_t N, int32_t max_live,
+                     const uint32_t *b_ready, const uint32_t *b_req_off, const int32_t *b_n,
+                     const int32_t *b_model, const int32_t *b_strict, const int32_t *batch_off,
+                     const uint32_t *arrival, const uint8_t *cur_geom, int32_t geom_lo, int32_t geom_hi,
+                     int64_t *depth_key, uint8_t *depth_code, int64_t *best_key, int64_t *n_eval);
 int orc_sweep(const orc_tables *t, int32_t R, int32_t N, int32_t max_live, int32_t max_batches,
               const uint32_t *b_ready, const uint32_t *b_req_off, const int32_t *b_n,
               const int32_t *b_model, const int32_t *b_strict, const int32_t *batch_off,

@@ -123,6 +123,8 @@ def lib():
                                        [C.c_int32, C.c_int32] + [C.c_void_p] * 10 + [C.c_int64])
         L.orc_sweep.argtypes = ([C.c_void_p] + [C.c_int32] * 4 + [C.c_void_p] * 8 + [C.c_int32] * 2 +
                                 [C.c_void_p] * 4)
+        L.orc_sweep_depths.argtypes = ([C.c_void_p] + [C.c_int32] * 3 + [C.c_void_p] * 8 + [C.c_int32] * 2 +
+                                       [C.c_void_p] * 4)
         _lib = L
     return _lib
 
@@ -373,6 +375,36 @@ def sweep(prof, *, R, N, batches, batch_off, arrival, cur_geom, geom_lo=0, geom_
     if rc:
         raise OracleError(rc)
     out["n_assign"] = int(out["n_assign"][0])
+    return out
+
+
+def sweep_depths(prof, *, R, N, batches, batch_off, arrival, cur_geom, geom_lo=0, geom_hi=None, max_live=64):
+    """N4b BE-reserve depth sweep (orc_sweep_depths); batches as for score_epoch.  depth_key is
+    [R*N, nc, 8]: code 0 = Alg 1's tag walk, 1 + d = reserve depth d (-1 beyond the slice count)."""
+    T = OTables(prof)
+    G = table_geometries(prof).shape[0]
+    if geom_hi is None:
+        geom_hi = G
+    arrs = {k: np.ascontiguousarray(batches[k], np.uint32 if k in ("ready", "req_off") else np.int32)
+            for k in ("ready", "req_off", "n", "model", "strict")}
+    for k in arrs:
+        if arrs[k].shape[0] == 0:
+            arrs[k] = np.zeros(1, arrs[k].dtype)
+    boff = np.ascontiguousarray(batch_off, np.int32)
+    arrival = np.ascontiguousarray(arrival, np.uint32)
+    if arrival.shape[0] == 0:
+        arrival = np.zeros(1, np.uint32)
+    cg = np.ascontiguousarray(cur_geom, np.uint8)
+    nc = geom_hi - geom_lo
+    out = dict(depth_key=np.zeros((R * N, max(nc, 0), 8), np.int64), depth_code=np.zeros((R * N, max(nc, 0)), np.uint8),
+               best_key=np.zeros(R * N, np.int64), n_eval=np.zeros(1, np.int64))
+    rc = lib().orc_sweep_depths(T.ref, R, N, max_live, _p(arrs["ready"]), _p(arrs["req_off"]), _p(arrs["n"]),
+                                _p(arrs["model"]), _p(arrs["strict"]), _p(boff), _p(arrival), _p(cg), geom_lo,
+                                geom_hi, _p(out["depth_key"]), _p(out["depth_code"]), _p(out["best_key"]),
+                                _p(out["n_eval"]))
+    if rc:
+        raise OracleError(rc)
+    out["n_eval"] = int(out["n_eval"][0])
     return out
 
 

@@ -85,8 +85,10 @@ struct Accum {
 int64_t exec_us(int64_t solo, int64_t F_ppm);
 
 // O6: Alg 1 Distribute_Jobs for one batch of model m at time t on geometry `geom`.
+// depth (N4b, reading R28): -1 = Alg 1's BE tag walk; d >= 0 = the d smallest slices are reserved
+// for BE (strict eligible on positions >= d), with the same fallback to every fitting slice.
 PlaceOut place(const Tables& tb, const std::vector<int>& geom, GpuState& S, int64_t t, int m,
-               bool strict, int max_live, Accum* acc, int64_t H);
+               bool strict, int max_live, Accum* acc, int64_t H, int depth = -1);
 
 // ---- O2: geometries by NVIDIA A100 MIG placement intervals (reading Q2) -------------------------
 struct GeomStats { int feasible, maximal_placements, placement_maximal_multisets, multiset_maximal; };
@@ -167,6 +169,8 @@ struct SweepBatch {
 };
 PlaceOut place_forced(const Tables& tb, const std::vector<int>& geom, GpuState& S, int64_t t, int m,
                       bool strict, int max_live, int slice);
+void sweep_depths(const Tables& tb, int j, int tag, const std::vector<SweepBatch>& bs, int max_live,
+                  int64_t* keys, int64_t* best_key, int* best_code, uint64_t* n_eval);
 void sweep_gpu(const Tables& tb, int j, int tag, const std::vector<SweepBatch>& bs, int max_live,
                int64_t* key_out, uint64_t* idx_out, uint64_t* n_assign);
 

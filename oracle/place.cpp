@@ -14,7 +14,7 @@ int64_t exec_us(int64_t solo, int64_t F_ppm) {
 }
 
 PlaceOut place(const Tables& tb, const std::vector<int>& geom, GpuState& S, int64_t t, int m,
-               bool strict, int max_live, Accum* acc, int64_t H) {
+               bool strict, int max_live, Accum* acc, int64_t H, int depth) {
   PlaceOut o;
 
   // Residents that ended at or before t can never be co-runners or memory holders again.
@@ -84,7 +84,9 @@ PlaceOut place(const Tables& tb, const std::vector<int>& geom, GpuState& S, int6
     int64_t R = be_mem;
     for (int s = 0; s < k; ++s) {
       const int32_t Ms = tb.cap(geom[s]);
-      if (R >= Ms) {  // tag_value == 1: completely occupied by BE
+      if (depth >= 0) {  // N4b (R28): an enumerated BE-reserve depth replaces the tags
+        o.eligible[s] = s >= depth;
+      } else if (R >= Ms) {  // tag_value == 1: completely occupied by BE
         o.eligible[s] = false;
         R -= Ms;
       } else {        // tag_value < 1

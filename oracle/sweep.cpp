@@ -114,4 +114,45 @@ void sweep_gpu(const Tables& tb, int j, int tag, const std::vector<SweepBatch>& 
   *n_assign += total;
 }
 
+// N4b: the BE-reserve depth as an enumerated dimension (reading R28).  For geometry j with S_j
+// slices, depth d in {auto, 0, 1, ..., S_j - 1} replays the GPU-epoch's batches from idle with
+// Alg 1's greedy choice (O6) whose strict eligibility is "position >= d" (auto = the BE tag walk of
+// Alg 1 lines 1-8).  keys[1 + d] (keys[0] = auto) is the O8 key; the minimum over (key, auto < 0 <
+// 1 < ...) is returned with its depth code (0 = auto, 1 + d).
+void sweep_depths(const Tables& tb, int j, int tag, const std::vector<SweepBatch>& bs, int max_live,
+                  int64_t* keys /* [8] */, int64_t* best_key, int* best_code, uint64_t* n_eval) {
+  const std::vector<int>& geom = tb.geoms[j];
+  const int S = (int)geom.size();
+  *best_key = -1;
+  *best_code = 0;
+  for (int code = 0; code < 8; ++code) keys[code] = -1;
+  for (int code = 0; code <= S; ++code) {
+    GpuState C;  // idle GPU in geometry j (reading Q19)
+    C.geom = j;
+    int64_t misses = 0, tail = 0;
+    for (const SweepBatch& bt : bs) {
+      PlaceOut po = place(tb, geom, C, bt.ready, bt.model, bt.strict, max_live, nullptr, INT64_MAX, code - 1);
+      if (bt.strict) {
+        if (po.dropped) {
+          misses += (int64_t)bt.arr.size();
+        } else {
+          int64_t hits = 0;
+          for (uint32_t a : bt.arr)
+            if (po.end - (int64_t)a <= tb.slo[bt.model]) hits++;
+          misses += (int64_t)bt.arr.size() - hits;
+        }
+      } else {
+        const int64_t t_b = po.dropped ? (int64_t)kSat32 : po.end - (int64_t)bt.arr[0];
+        tail = std::max(tail, t_b);
+      }
+    }
+    keys[code] = make_key(misses, tail, tag);
+    if (*best_key < 0 || keys[code] < *best_key) {
+      *best_key = keys[code];
+      *best_code = code;
+    }
+    *n_eval += 1;
+  }
+}
+
 }  // namespace pem

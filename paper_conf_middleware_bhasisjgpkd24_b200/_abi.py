@@ -27,7 +27,8 @@ class Profiles(C.Structure):
     _fields_ = [("abi_version", C.c_int32), ("n_models", C.c_int32), ("solo_us", C.c_void_p),
                 ("fbr_ppm", C.c_void_p), ("mem_mib", C.c_void_p), ("batch_size", C.c_void_p),
                 ("slo_us", C.c_void_p), ("batch_timeout_us", C.c_void_p), ("geometry_set", C.c_int32),
-                ("n_geoms", C.c_int32), ("geoms", C.c_void_p), ("device", C.c_int32)]
+                ("n_geoms", C.c_int32), ("geoms", C.c_void_p), ("device", C.c_int32),
+                ("gpu_mem_mib", C.c_int32)]
 
 
 class Batch(C.Structure):        # protean_batch, 16 B
@@ -92,6 +93,11 @@ class SweepOut(C.Structure):     # protean_sweep_out
                 ("n_assign", C.c_void_p)]
 
 
+class DepthOut(C.Structure):
+    _fields_ = [("depth_key", C.c_void_p), ("depth_code", C.c_void_p), ("best_key", C.c_void_p),
+                ("n_eval", C.c_void_p)]
+
+
 class BatchRec(C.Structure):     # protean_batch_rec, 32 B
     _fields_ = [("ready_us", C.c_uint32), ("epoch", C.c_uint32), ("n_req", C.c_uint16), ("model", C.c_uint8),
                 ("strict", C.c_uint8), ("gpu", C.c_uint8), ("slice", C.c_uint8), ("dropped", C.c_uint8),
@@ -111,17 +117,21 @@ assert C.sizeof(BatchRec) == 32
 EXPORTS = ["protean_load_profiles", "protean_free", "protean_strerror", "protean_last_error",
            "protean_get_geometries", "protean_num_epochs", "protean_score_epoch", "protean_score_epoch_status",
            "protean_replay_traces", "protean_replay_traces_host", "protean_replay_cfg_defaults", "protean_last_timings",
-           "protean_geometry_split", "protean_xchg_export", "protean_xchg_import", "protean_xchg_attach"]
+           "protean_sweep_depths", "protean_geometry_split", "protean_xchg_export", "protean_xchg_import", "protean_xchg_attach"]
 IPC_HANDLE_BYTES = 64
 
 _lib = None
 
 
-def load(path: str = LIB_PATH, require_cuda: bool = True):
-    """Load libprotean.so.  Raises if the library (or, with require_cuda, a GPU) is missing."""
+def load(path: str = None, require_cuda: bool = True):
+    """Load libprotean.so (or the in-tree debug build named by PROTEAN_LIB, e.g. the racecheck
+    variant).  Raises if the library (or, with require_cuda, a GPU) is missing."""
     global _lib
     if _lib is not None:
         return _lib
+    if path is None:
+        v = os.environ.get("PROTEAN_LIB")
+        path = os.path.join(os.path.dirname(LIB_PATH), v) if v else LIB_PATH
     if not os.path.exists(path):
         raise ImportError(f"{path} is missing: run __graft_entry__.build() (nvcc, sm_100a)")
     L = C.CDLL(path)
@@ -137,6 +147,7 @@ def load(path: str = LIB_PATH, require_cuda: bool = True):
     L.protean_score_epoch.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
     L.protean_score_epoch_status.argtypes = [C.c_void_p]
     L.protean_sweep_assignments.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
+    L.protean_sweep_depths.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
     L.protean_form_batches.argtypes = [C.c_void_p, C.c_void_p, C.c_int32, C.c_int32, C.c_void_p, C.c_void_p,
                                        C.c_void_p, C.c_void_p, C.c_void_p, C.c_int64, C.c_void_p]
     L.protean_replay_traces.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]

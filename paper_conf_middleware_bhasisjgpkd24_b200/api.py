@@ -40,7 +40,8 @@ def _profiles_struct(profiles, device: int = 0):
     geoms = None if profiles.geoms is None else np.ascontiguousarray(profiles.geoms, np.uint8)
     p = A.Profiles(A.ABI_VERSION, int(arrs[0].shape[0]), *[a.ctypes.data for a in arrs],
                    int(profiles.geometry_set), 0 if geoms is None else int(geoms.shape[0]),
-                   None if geoms is None else geoms.ctypes.data, int(device))
+                   None if geoms is None else geoms.ctypes.data, int(device),
+                   int(getattr(profiles, "gpu_mem_mib", 0)))
     return p, (arrs, geoms)
 
 
@@ -372,6 +373,30 @@ class Handle:
         st = stream if stream is not None else torch.cuda.current_stream(self.device)
         _check(self._h, self._lib.protean_sweep_assignments(self._h, C.byref(si), C.byref(so),
                                                             C.c_void_p(st.cuda_stream)))
+        return out
+
+    def sweep_depths(self, *, n_replicas, n_gpus, batches, batch_off, arrival_us, cur_geom, geom_lo=0,
+                     geom_hi=None, max_live=64, out=None, stream=None):
+        """protean_sweep_depths (N4b, BE-reserve depth codes).  Inputs as sweep_assignments.
+        Returns depth_key [R*N, nc, 8], depth_code [R*N, nc] (uint8), best_key [R*N], n_eval [1]."""
+        torch = _torch()
+        dev = torch.device("cuda", self.device)
+        geom_hi = self.n_geoms if geom_hi is None else geom_hi
+        R, N = int(n_replicas), int(n_gpus)
+        nc = geom_hi - geom_lo
+        if out is None:
+            out = dict(depth_key=torch.zeros((R * N, max(nc, 1), 8), dtype=torch.int64, device=dev),
+                       depth_code=torch.zeros((R * N, max(nc, 1)), dtype=torch.uint8, device=dev),
+                       best_key=torch.zeros(R * N, dtype=torch.int64, device=dev),
+                       n_eval=torch.zeros(1, dtype=torch.int64, device=dev))
+        nb = batches.numel() // 16
+        si = A.SweepIn(R, N, int(max_live), 8, batches.data_ptr() if nb else batch_off.data_ptr(),
+                       batch_off.data_ptr(), arrival_us.data_ptr() if arrival_us.numel() else batch_off.data_ptr(),
+                       cur_geom.data_ptr(), int(geom_lo), int(geom_hi))
+        do = A.DepthOut(out["depth_key"].data_ptr(), out["depth_code"].data_ptr(), out["best_key"].data_ptr(),
+                        out["n_eval"].data_ptr())
+        st = stream if stream is not None else torch.cuda.current_stream(self.device)
+        _check(self._h, self._lib.protean_sweep_depths(self._h, C.byref(si), C.byref(do), C.c_void_p(st.cuda_stream)))
         return out
 
 

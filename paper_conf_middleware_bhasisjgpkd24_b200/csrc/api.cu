@@ -100,7 +100,8 @@ const int kMem[5] = {5120, 10240, 20480, 20480, 40960};
 const int kMaxCnt[5] = {7, 3, 2, 1, 1};
 
 // O2 by T2 sum constraints: count vectors with at most the T2 max counts, <= 7/7 compute and
-// <= 40 GB.  Default set = multiset-maximal ones.  Order: (c7g,c4g,c3g,c2g,c1g) descending.
+// <= 40 GB (<= 8/8 of the memory: the set is the same for every MIG table of N4c, whose profiles
+// keep T2's memory eighths).  Default set = multiset-maximal ones.  Order: (c7g,c4g,c3g,c2g,c1g) descending.
 std::vector<std::vector<uint8_t>> geometry_set(bool all) {
   std::vector<std::array<int, 5>> feas;
   for (int a = 0; a <= kMaxCnt[0]; ++a)
@@ -443,9 +444,14 @@ int protean_load_profiles(const protean_profiles* p, protean_handle** out) {
     if (p->solo_us[i] <= 0) return PROTEAN_EINVAL;
     if (p->fbr_ppm[i] < 0 || p->fbr_ppm[i] > 1000000) return PROTEAN_EINVAL;
   }
+  // N4c: the GPU's memory (0 = A100-40GB); profile p holds gmem * eighths_p / 8
+  const int32_t gmem = p->gpu_mem_mib == 0 ? 40960 : p->gpu_mem_mib;
+  if (gmem < 8 || gmem % 8 != 0 || gmem > (1 << 24)) return PROTEAN_EINVAL;
+  int32_t cap[5];
+  for (int q = 0; q < 5; ++q) cap[q] = gmem / 8 * prof_eighths(q);
   int maxT = 0;
   for (int m = 0; m < M; ++m) {
-    if (p->mem_mib[m] < 1 || p->mem_mib[m] > 40960) return PROTEAN_EINVAL;
+    if (p->mem_mib[m] < 1 || p->mem_mib[m] > gmem) return PROTEAN_EINVAL;
     if (p->batch_size[m] < 1 || p->batch_size[m] > 65535) return PROTEAN_EINVAL;
     if (p->slo_us[m] <= 0 || p->batch_timeout_us[m] < 0) return PROTEAN_EINVAL;
     maxT = std::max(maxT, p->batch_timeout_us[m]);
@@ -477,11 +483,12 @@ int protean_load_profiles(const protean_profiles* p, protean_handle** out) {
       const uint8_t v = s < (int)gs[j].size() ? gs[j][s] : 0xFF;
       gp[j * 8 + s] = v;
       h->geoms[j * 8 + s] = v;
-      if (v != 0xFF) pref += kMem[v];
+      if (v != 0xFF) pref += cap[v];
       w[h->tl.o_gpref + j * 8 + s] = pref;  // capacity of slices 0..s (Alg 1 tag walk)
     }
     w[h->tl.o_gn + j] = (int32_t)gs[j].size();
   }
+  for (int q = 0; q < 5; ++q) w[h->tl.o_cap + q] = cap[q];
   for (int j = 0; j < h->G; ++j) h->gn.push_back((int)gs[j].size());
   int cw = 0;
   std::vector<uint32_t> pack = build_pack(h->gn, 0, h->G, &cw);
@@ -1053,6 +1060,63 @@ int protean_sweep_assignments(protean_handle* h, const protean_sweep_in* in, pro
   CK(h, cudaStreamSynchronize(st));
   if (errs[0]) return fail(h, PROTEAN_EINVAL, "invalid batch / offsets / cur_geom");
   if (errs[1]) return fail(h, PROTEAN_ERANGE, "more than max_batches batches on a GPU");
+  return PROTEAN_OK;
+}
+
+int protean_sweep_depths(protean_handle* h, const protean_sweep_in* in, protean_depth_out* out, void* stream) {
+  if (!h) return PROTEAN_EINVAL;
+  if (h->poisoned) return PROTEAN_ESTATE;
+  if (!in || !out) return fail(h, PROTEAN_EINVAL, "null in/out");
+  if (in->n_replicas < 1 || in->n_gpus < 1) return fail(h, PROTEAN_EINVAL, "sizes");
+  if (in->n_gpus > 255) return fail(h, PROTEAN_ERANGE, "n_gpus > 255");
+  if (in->max_live < 1 || in->max_live > PROTEAN_MAX_LIVE) return fail(h, PROTEAN_EINVAL, "max_live");
+  if (in->geom_lo < 0 || in->geom_hi > h->G || in->geom_lo >= in->geom_hi)
+    return fail(h, PROTEAN_EINVAL, "geometry range");
+  if (!in->batch_off || !in->cur_geom || !out->best_key || !out->n_eval)
+    return fail(h, PROTEAN_EINVAL, "null pointer");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  CK(h, cudaSetDevice(h->device));
+  const int R = in->n_replicas, N = in->n_gpus, nc = in->geom_hi - in->geom_lo;
+  const int block = 128;
+  const int64_t lanes = (int64_t)R * N * nc * 8;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((lanes + block - 1) / block, (int64_t)h->nsm * 8));
+  // scratch: one resident list per thread of the grid, then (if the caller passes no depth_key) the keys
+  const size_t lists = al((size_t)grid * block * in->max_live * sizeof(protean_resident));
+  const size_t keys = out->depth_key ? 0 : al((size_t)lanes * 8);
+  {
+    int rc = ensure(h, &h->d_scratch, &h->scratch_bytes, lists + keys, st);
+    if (rc) return rc;
+  }
+  int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 64);
+  CK(h, cudaMemsetAsync(d_err, 0, 16, st));
+  DepthParams P;
+  std::memset(&P, 0, sizeof(P));
+  P.tab = h->d_tab;
+  P.tl = h->tl;
+  P.R = R;
+  P.N = N;
+  P.max_live = in->max_live;
+  P.geom_lo = in->geom_lo;
+  P.geom_hi = in->geom_hi;
+  P.batches = in->batches;
+  P.batch_off = in->batch_off;
+  P.arrival = in->arrival_us;
+  P.cur_geom = in->cur_geom;
+  P.scratch = static_cast<protean_resident*>(h->d_scratch);
+  P.depth_key = out->depth_key ? out->depth_key
+                               : reinterpret_cast<int64_t*>(static_cast<char*>(h->d_scratch) + lists);
+  P.depth_code = out->depth_code;
+  P.best_key = out->best_key;
+  P.n_eval = out->n_eval;
+  int64_t per_x = 0;  // depth codes per (replica, gpu): sum over the range of (slices + 1)
+  for (int j = in->geom_lo; j < in->geom_hi; ++j) per_x += h->gn[j] + 1;
+  P.n_eval_add = per_x * (int64_t)R * N;
+  P.err = d_err;
+  CK(h, launch_depths(P, grid, block, st));
+  int err0 = 0;
+  CK(h, cudaMemcpyAsync(&err0, d_err, 4, cudaMemcpyDeviceToHost, st));
+  CK(h, cudaStreamSynchronize(st));
+  if (err0) return fail(h, PROTEAN_EINVAL, "invalid batch / offsets / cur_geom");
   return PROTEAN_OK;
 }
 

@@ -17,9 +17,13 @@ constexpr int64_t kPpm = 1000000;
 constexpr uint32_t kNoGeom = 0xFF;
 constexpr int kNB = PROTEAN_NBUCKETS;
 
-// T2 — slice memory in MiB and compute sevenths per profile (1g,2g,3g,4g,7g).
-__host__ __device__ __forceinline__ int32_t prof_cap(int p) {
-  return p == 0 ? 5120 : p == 1 ? 10240 : p == 4 ? 40960 : 20480;
+constexpr uint32_t kMemMask = 0xFFFFFFu;  // packed resident words: footprint in the low 24 bits
+
+// T2 — memory eighths and compute sevenths per profile (1g,2g,3g,4g,7g); a slice's
+// memory is gpu_mem * eighths / 8 (A100-40GB: 5120/10240/20480/20480/40960 MiB; N4c: the same
+// structure over the H100 / H200 / B200 memories), staged per handle in Tab::cap.
+__host__ __device__ __forceinline__ int32_t prof_eighths(int p) {
+  return p == 0 ? 1 : p == 1 ? 2 : p == 4 ? 8 : 4;
 }
 __host__ __device__ __forceinline__ int32_t prof_compute(int p) {
   return p == 0 ? 1 : p == 1 ? 2 : p == 2 ? 3 : p == 3 ? 4 : 7;
@@ -32,23 +36,24 @@ struct TabLayout {
   int o_gprof;   // G*8 bytes packed into G*2 words: profile ids ascending, 0xFF padded
   int o_gn;      // G words: slice count
   int o_gpref;   // G*8 words: prefix capacity including slice s (tag walk, Alg 1 lines 1-8)
+  int o_cap;     // 5 words: slice memory per profile (MiB), N4c
   int words;
   __host__ __device__ void init(int m, int g) {
     M = m; G = g;
     o_solo = 0; o_fbr = o_solo + 5 * M; o_mem = o_fbr + 5 * M; o_bsz = o_mem + M;
     o_slo = o_bsz + M; o_tmo = o_slo + M; o_gprof = o_tmo + M; o_gn = o_gprof + 2 * G;
-    o_gpref = o_gn + G; words = o_gpref + 8 * G;
+    o_gpref = o_gn + G; o_cap = o_gpref + 8 * G; words = o_cap + 8;
   }
 };
 
 struct Tab {  // smem views
   int M, G;
-  const int32_t *solo, *fbr, *mem, *bsz, *slo, *tmo, *gn, *gpref;
+  const int32_t *solo, *fbr, *mem, *bsz, *slo, *tmo, *gn, *gpref, *cap;
   const uint8_t *gprof;
   __device__ void bind(const int32_t* w, const TabLayout& L) {
     M = L.M; G = L.G;
     solo = w + L.o_solo; fbr = w + L.o_fbr; mem = w + L.o_mem; bsz = w + L.o_bsz;
-    slo = w + L.o_slo; tmo = w + L.o_tmo; gn = w + L.o_gn; gpref = w + L.o_gpref;
+    slo = w + L.o_slo; tmo = w + L.o_tmo; gn = w + L.o_gn; gpref = w + L.o_gpref; cap = w + L.o_cap;
     gprof = reinterpret_cast<const uint8_t*>(w + L.o_gprof);
   }
 };
@@ -85,7 +90,7 @@ __device__ __forceinline__ int64_t exec_time(int32_t solo, int64_t F) {
 static __device__ __noinline__ void place_slow_slice(const Tab& T, const uint8_t* gp, Rows L, int n, int s,
                                               int p, int64_t t0, int32_t q, int m, int64_t* start_out,
                                               int64_t* F_out) {
-  const int32_t Ms = prof_cap(p);
+  const int32_t Ms = T.cap[p];
   int64_t used = 0, e = INT64_MAX;
   for (int i = 0; i < n; ++i)
     if ((int)(L.meta(i) & 0xFF) == s && L.en(i) > t0) {
@@ -121,9 +126,10 @@ static __device__ __noinline__ void place_slow_slice(const Tab& T, const uint8_t
 // slice, the memory still held after t0_s = max(t, last_start_s) and the FBR of those residents;
 // since every resident of a slice started at or before its last start (FIFO), they are exactly
 // Eq 1's co-runners at t0_s.  The rare memory-wait case takes place_slow_slice().
+// depth (N4b, reading R28): -1 = Alg 1's BE tags; d >= 0 = the d smallest slices reserved for BE.
 __device__ __forceinline__ PlaceRes place_lane(const Tab& T, int geom, Rows L, int& n,
                                                int64_t (&ls)[kMaxSl], int64_t t, int m,
-                                               bool strict, int max_live) {
+                                               bool strict, int max_live, int depth = -1) {
   PlaceRes o;
   o.dropped = 0;
   o.slice = -1;
@@ -170,7 +176,7 @@ __device__ __forceinline__ PlaceRes place_lane(const Tab& T, int geom, Rows L, i
   for (int x = 0; x < kMaxSl; ++x) {
     if (x < ns) {
       const int p = gp[x];
-      const int32_t Ms = prof_cap(p);
+      const int32_t Ms = T.cap[p];
       if (q <= Ms) {
         int64_t start, F;
         if (used[x] + q <= Ms && !((fut >> x) & 1)) {
@@ -182,7 +188,8 @@ __device__ __forceinline__ PlaceRes place_lane(const Tab& T, int geom, Rows L, i
         const int64_t c = start + exec_time(T.solo[m * kNProf + p], F);
         uint64_t key;
         if (strict) {  // choose_strict_slice: tag < 1, least eta == least completion (Q11)
-          const uint64_t inelig = (be_mem >= T.gpref[geom * 8 + x]) ? (1ull << 62) : 0ull;
+          const bool full = depth >= 0 ? x < depth : be_mem >= T.gpref[geom * 8 + x];
+          const uint64_t inelig = full ? (1ull << 62) : 0ull;
           key = inelig | ((uint64_t)c << 6) | ((uint64_t)(4 - p) << 3) | (uint64_t)x;
         } else {       // choose_best_effort_slice: first fit, else earliest start (Q12)
           key = ((uint64_t)start << 3) | (uint64_t)x;

@@ -20,9 +20,6 @@
 #include <mutex>
 
 #include "replay.cuh"
-#ifndef PROTEAN_A_BARRIER
-#define PROTEAN_A_BARRIER 0
-#endif
 #ifndef PROTEAN_D_BARRIER
 #define PROTEAN_D_BARRIER 1
 #endif
@@ -59,7 +56,8 @@ namespace {
 constexpr int kMaxWarps = 32;
 
 // Per-lane resident list, interleaved across lanes (entry i of lane l at i*stride + l) so that a
-// warp walking its lists in lock-step issues coalesced loads.  mm = mem | model << 16 | strict << 22.
+// warp walking its lists in lock-step issues coalesced loads.  mm = mem | model << 24 | strict << 30
+// (footprints < 2^24 MiB: every MIG table of N4c fits).
 struct LaneList {
   int64_t* st;
   int64_t* en;
@@ -98,6 +96,7 @@ struct CtaState {
   int64_t nlog;
   int nb, cursor, all_avail, bad;
   int task, adone;
+  int task_r[2];            // PROTEAN_ACCT_BARRIER debug build: the two rounds' task counters
   int glo, ghi, cw, xrank;  // this CTA's candidate geometry range, its candidate warps per GPU and
                             // its rank in the key exchange (virtual ranks: several CTAs per replica)
   int wtot;
@@ -381,9 +380,9 @@ __device__ __noinline__ void slice_slow(const LaneList& L, int n, int64_t t0, in
     const int64_t ei = L.E(i);
     if (ei > t0) {
       const uint32_t mi = L.M(i);
-      used += mi & 0xFFFF;
+      used += mi & kMemMask;
       e = ei < e ? ei : e;
-      if (L.S(i) <= t0) F += fbr_p[((mi >> 16) & 63) * kNProf];
+      if (L.S(i) <= t0) F += fbr_p[((mi >> 24) & 63) * kNProf];
     }
   }
   int64_t start = t0;
@@ -399,9 +398,9 @@ __device__ __noinline__ void slice_slow(const LaneList& L, int n, int64_t t0, in
         const int64_t ek = L.E(k);
         if (ek > e) {
           const uint32_t mk = L.M(k);
-          rem += mk & 0xFFFF;
+          rem += mk & kMemMask;
           nxt = ek < nxt ? ek : nxt;
-          if (L.S(k) <= e) Fe += fbr_p[((mk >> 16) & 63) * kNProf];
+          if (L.S(k) <= e) Fe += fbr_p[((mk >> 24) & 63) * kNProf];
         }
       }
       if (rem + q <= Ms) {  // always by the last release (q <= Ms)
@@ -469,10 +468,10 @@ __device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, const
         const uint32_t mi = m_[u];
         if (k != i) L.put(k, si, ei, mi);
         ++k;
-        if (!((mi >> 22) & 1)) be += mi & 0xFFFF;
+        if (!((mi >> 30) & 1)) be += mi & kMemMask;
         if (ei > t0) {
-          used += mi & 0xFFFF;
-          fs += fbr_p[((mi >> 16) & 63) * kNProf];
+          used += mi & kMemMask;
+          fs += fbr_p[((mi >> 24) & 63) * kNProf];
           fut |= si > t0;
         }
       }
@@ -508,7 +507,7 @@ __device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, const
   *my_start = start;
   *my_end = c;
   if (o.kmin != ~0ull && key == o.kmin) {  // schedule(batch, chosen_slice)
-    L.put(n, start, c, (uint32_t)q | ((uint32_t)m << 16) | ((uint32_t)(strict ? 1 : 0) << 22));
+    L.put(n, start, c, (uint32_t)q | ((uint32_t)m << 24) | ((uint32_t)(strict ? 1 : 0) << 30));
     ++n;
     ls = start;
   }
@@ -517,6 +516,7 @@ __device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, const
 
 constexpr int kKR = 6;  // batches per GPU-epoch handled by the register fast path
 constexpr int kAK = 4;  // batch ranks per accounting task (phase F)
+constexpr int kBW = 1;  // the warp that lays out the next epoch's windows (phase B) during G
 
 // Candidate unit, fast path: the GPU-epoch's <= kKR batches fully unrolled, times 32-bit relative to
 // the first batch's ready time tb.  Every lane of a geometry's group keeps the whole placement so
@@ -560,9 +560,9 @@ __device__ __forceinline__ bool candidate_unit_fast(const Tab& T, const SliceLan
     for (int i = 0; i < x; ++i) {
       const bool alive = en[i] > rt;
       live += alive ? 1 : 0;
-      if (alive && (mm[i] >> 16)) be += (int32_t)(mm[i] & 0xFFFF);
+      if (alive && (mm[i] >> 24)) be += (int32_t)(mm[i] & kMemMask);
       if (((mine >> i) & 1u) && en[i] > rt0) {
-        used += (int32_t)(mm[i] & 0xFFFF);
+        used += (int32_t)(mm[i] & kMemMask);
         fs += fb[i];
       }
     }
@@ -583,7 +583,7 @@ __device__ __forceinline__ bool candidate_unit_fast(const Tab& T, const SliceLan
             int32_t rem = 0;
 #pragma unroll
             for (int i = 0; i < x; ++i)
-              if (((mine >> i) & 1u) && en[i] > en[jj]) rem += (int32_t)(mm[i] & 0xFFFF);
+              if (((mine >> i) & 1u) && en[i] > en[jj]) rem += (int32_t)(mm[i] & kMemMask);
             if (rem + q <= K.Ms && en[jj] < start) start = en[jj];
           }
         }
@@ -601,7 +601,7 @@ __device__ __forceinline__ bool candidate_unit_fast(const Tab& T, const SliceLan
     const bool placed = !overflow && kmin != 0xFFFFFFFFu;
     const uint32_t cwin = __shfl_sync(0xffffffffu, c, (gbase + (int)(kmin & 7)) & 31);
     en[x] = placed ? cwin : 0u;
-    mm[x] = (uint32_t)q | (strict ? 0u : 0x10000u);
+    mm[x] = (uint32_t)q | (strict ? 0u : 0x1000000u);
     fb[x] = fbm;
     if (placed && key == kmin) {  // schedule(batch, chosen_slice)
       mine |= 1u << x;
@@ -675,8 +675,8 @@ __device__ __forceinline__ int alg2_final_geometry(const ReplayParams& P, const 
   c.gi[12 * c.N + g] = X;
   c.gi[13 * c.N + g] = Y;
   // lines 10-18: the first of [[1g,2g],[3g]] whose summed T2 capacity holds pred_BE_mem (R12)
-  const bool fits12 = (int64_t)(prof_cap(0) + prof_cap(1)) * 1000 >= Y;
-  const bool found = fits12 || (int64_t)prof_cap(2) * 1000 >= Y;
+  const bool fits12 = (int64_t)(c.T.cap[0] + c.T.cap[1]) * 1000 >= Y;
+  const bool found = fits12 || (int64_t)c.T.cap[2] * 1000 >= Y;
   // lines 19-23: thresholds on pot_occupancy = pred_BE_num (R13, R14), (4g,3g) fallback, + 4g (R15)
   if (!found || X < P.t_low || X > P.t_high) return P.g43;
   return fits12 ? P.g421 : P.g43;
@@ -815,6 +815,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
       cs.cursor = 0;
       cs.bad = 0;
       cs.task = 0;  // per-epoch scratch, re-armed at the end of every epoch
+      cs.task_r[0] = cs.task_r[1] = 0;
       cs.adone = 0;
       cs.nb = 0;
       cs.all_avail = 1;
@@ -824,12 +825,13 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
     }
     __syncthreads();
 
+    // ---------------------------------------------------------------- A: VM events, installs
+    // (warp 0, lane = simulated GPU), for epoch ee; runs right after G of epoch ee - 1 in the same
+    // warp (program order: the windows G opened are visible), overlapping B of epoch ee in warp kBW
+    auto phase_a = [&](int64_t ee) {
+      const int64_t eW = ee * P.W, Tend = eW + P.W;
 #pragma unroll 1
-    for (int64_t e = 0; e < P.E; ++e) {
-      const int64_t eW = e * P.W, Tend = eW + P.W;
-      // ---------------------------------------------------------------- A: VM events, installs
-#pragma unroll 1
-      for (int g = tid; g < N; g += NT) {
+      for (int g = lane; g < N; g += 32) {
         if (P.vm_policy != 0) {
 #pragma unroll 1
           for (int64_t k = (eW + P.rev - 1) / P.rev; k * P.rev < Tend; ++k) {
@@ -851,19 +853,20 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
                            !(c.gi[0 * c.N + g] < Tend && c.gi[1 * c.N + g] > eW);
         if (!whole) cs.all_avail = 0;  // set to 1 before the previous epoch's last barrier
       }
-#if PROTEAN_A_BARRIER
-      __syncthreads();
-#endif
-      // ---------------------------------------------------------------- B: stream windows
-      // Stream k's unbatched requests are [s_cur[k], sidx[r][e+1][k]) of the stream-sorted copy
-      // (partition.cu).  Warp 0 lays the streams out contiguously in the window (each as its
-      // 16-byte aligned superset) and, for a shared-memory window, every lane issues its streams'
-      // TMA bulk copies (cp.async.bulk global -> shared, completion on one mbarrier); the next
-      // epoch's new requests are prefetched into L2 meanwhile.  A global-scratch window (too large
-      // for shared memory) is filled by a cooperative 16-byte copy instead.
-      const uint32_t* sa_r = P.sa + P.saoff[r];
-      if (warp == 0) {
-        const uint32_t* s1 = P.sidx + ((size_t)r * (P.E + 1) + e + 1) * S;
+    };
+    // ---------------------------------------------------------------- B: stream windows
+    // Stream k's unbatched requests are [s_cur[k], sidx[r][e+1][k]) of the stream-sorted copy
+    // (partition.cu).  Warp kBW lays the streams out contiguously in the window (each as its
+    // 16-byte aligned superset) and, for a shared-memory window, every lane issues its streams'
+    // TMA bulk copies (cp.async.bulk global -> shared, completion on one mbarrier); the next
+    // epoch's new requests are prefetched into L2 meanwhile.  A global-scratch window (too large
+    // for shared memory) is filled by a cooperative 16-byte copy after the barrier instead.
+    // B of epoch e + 1 runs while warp 0 decides epoch e (G): it reads only s_cur (final after
+    // epoch e's formation) and overwrites the window, which no phase after E reads.
+    const uint32_t* sa_r = P.sa + P.saoff[r];
+    auto phase_b = [&](int64_t ee) {
+      {
+        const uint32_t* s1 = P.sidx + ((size_t)r * (P.E + 1) + ee + 1) * S;
         int carry = 0, nact = 0;
 #pragma unroll 1
         for (int k0 = 0; k0 < S; k0 += 32) {
@@ -875,7 +878,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
             len = hi - cur;
             alo = cur & ~3;
             asz = len > 0 ? ((hi + 3) & ~3) - alo : 0;
-            if (e + 1 < P.E && tid < 32) {  // the next epoch's new requests: into L2 during this one
+            if (ee + 1 < P.E) {  // the next epoch's new requests: into L2 during this one
               const int h2 = (int)s1[S + k];
               if (h2 > hi) prefetch_l2(sa_r + hi, (int64_t)(h2 - hi) * 4);
             }
@@ -925,6 +928,13 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
             asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mbar), "r"(tot * 4) : "memory");
         }
       }
+    };
+    // e = -1 only prepares epoch 0 (A and B below); one call site each keeps one inlined copy
+#pragma unroll 1
+    for (int64_t e = -1; e < P.E; ++e) {
+      const int64_t eW = e * P.W, Tend = eW + P.W;
+      (void)eW;
+      if (e >= 0) {
       __syncthreads();
       PH(1);
       if (win_smem) {
@@ -1198,11 +1208,19 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
       // accounting waits (rarely) for the actual units, whose warps publish via cs.adone
       const int n_units = n_aunits + (P.policy == 0 ? N * cs.cw : 0);
       const int n_tasks = n_units + (nb + kAK - 1) / kAK;
+#ifndef PROTEAN_ACCT_BARRIER
+#define PROTEAN_ACCT_BARRIER 0  // 1: debug build for compute-sanitizer racecheck (accounting after a CTA barrier)
+#endif
+      constexpr int kRounds = PROTEAN_ACCT_BARRIER ? 2 : 1;
+#pragma unroll 1
+      for (int round = 0; round < kRounds; ++round) {
+      if (PROTEAN_ACCT_BARRIER && round == 1) __syncthreads();  // every actual unit has finished
       for (;;) {
         int u = 0;
-        if (lane == 0) u = atomicAdd(&cs.task, 1);
+        if (lane == 0) u = PROTEAN_ACCT_BARRIER ? atomicAdd(&cs.task_r[round], 1) + (round ? n_units : 0)
+                                                : atomicAdd(&cs.task, 1);
         u = __shfl_sync(0xffffffffu, u, 0);
-        if (u >= n_tasks) break;
+        if (u >= (PROTEAN_ACCT_BARRIER && round == 0 ? n_units : n_tasks)) break;
 #ifdef PROTEAN_PHASE_TIMING
         const long long tk0 = clock64();
         const int tkind = u >= n_units ? 2 : (u < n_aunits ? 0 : 1);
@@ -1215,7 +1233,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
           // acquire the actual units' batch results (slice, start, end, drop): lane 0's acquire
           // load, then the warp barrier orders it before every lane's reads (PTX memory model:
           // release/acquire at CTA scope + bar.warp.sync)
-          if (lane == 0) {
+          if (!PROTEAN_ACCT_BARRIER && lane == 0) {
             const uint32_t fa = (uint32_t)__cvta_generic_to_shared(&cs.adone);
             for (;;) {
               int v;
@@ -1331,7 +1349,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
         SliceLane K;
         K.fbr_p = T.fbr + p;
         K.solo_p = T.solo + p;
-        K.Ms = prof_cap(p);
+        K.Ms = T.cap[p];
         K.pref = T.gpref[j * 8 + (s & 7)];
         K.s = s;
         K.p = p;
@@ -1471,11 +1489,13 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
           if (P.cand_keys) P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = key;
         }
       }
+      }  // rounds
       __syncthreads();
       PH(7);
       if constexpr (kN3) {  // R26: delayed termination (pools are next used in the next epoch's E)
 #pragma unroll 1
         for (int k = tid; k < N * pl.M; k += NT) pool_terminate(P, pl, c, k / pl.M, k % pl.M, c.bats, c.gl, Tend);
+        __syncthreads();  // the next epoch's A (warp 0) may reset pools on a VM change
       }
       // ---------------------------------------------------------------- G: decisions (O9, O10)
       if (PROTEAN_WARP_G && P.xl.n <= 1 && N <= 32) {
@@ -1567,6 +1587,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
           if (lane == 0) {
             cs.nlog += nb;
             cs.task = 0;  // re-arm the per-epoch scratch for the next epoch
+            cs.task_r[0] = cs.task_r[1] = 0;
             cs.adone = 0;
             cs.nb = 0;
             cs.all_avail = 1;
@@ -1655,14 +1676,27 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
         }
         cs.nlog += nb;
         cs.task = 0;  // re-arm the per-epoch scratch for the next epoch
+        cs.task_r[0] = cs.task_r[1] = 0;
         cs.adone = 0;
         cs.nb = 0;
         cs.all_avail = 1;
       }
       }
-      __syncthreads();
-      PH(9);
+      PH(9);  // the next epoch's first barrier closes this one
+      }  // e >= 0
+      // A and B of the next epoch: A in warp 0 after its decisions (program order: the windows G
+      // opened are visible to A), B in warp kBW at the same time (it reads only s_cur and writes the
+      // window, which nothing after E reads)
+      if (e + 1 < P.E) {
+        if (warp == 0) {
+          __syncwarp();
+          phase_a(e + 1);
+        } else if (warp == kBW) {
+          phase_b(e + 1);
+        }
+      }
     }
+    __syncthreads();  // the last epoch's decisions before finalize
 
     // ---------------------------------------------------------------- finalize (O12)
 #pragma unroll 1
@@ -1728,7 +1762,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
                                       __dmul_rn((double)spot, P.price_spot)), 3.6e9);
       const double dN = (double)N, dH = (double)P.H;
       P.util[2 * (size_t)r] = __ddiv_rn((double)busy, __dmul_rn(__dmul_rn(7.0, dN), dH));
-      P.util[2 * (size_t)r + 1] = __ddiv_rn((double)memt, __dmul_rn(__dmul_rn(40960.0, dN), dH));
+      P.util[2 * (size_t)r + 1] = __ddiv_rn((double)memt, __dmul_rn(__dmul_rn((double)T.cap[4], dN), dH));
       if (P.n_batches) P.n_batches[r] = cs.nlog;
       if (P.cold_starts) P.cold_starts[r] = (int64_t)cs.cold;
     }

@@ -192,6 +192,25 @@ struct SweepParams {
   int* err;                   // err[0] EINVAL, err[1] ERANGE
 };
 cudaError_t launch_sweep(const SweepParams& P, int grid, cudaStream_t st);
+
+// N4b BE-reserve depth sweep (score.cu): lanes (replica, gpu, geometry, depth code)
+struct DepthParams {
+  const int32_t* tab;
+  TabLayout tl;
+  int R, N, max_live, geom_lo, geom_hi;
+  const protean_batch* batches;
+  const int32_t* batch_off;
+  const uint32_t* arrival;
+  const uint8_t* cur_geom;
+  int64_t* depth_key;         // [R*N*nc*8] (library scratch when the caller passes NULL)
+  uint8_t* depth_code;        // [R*N*nc] or NULL
+  int64_t* best_key;          // [R*N]
+  int64_t* n_eval;            // [1] += evaluations
+  int64_t n_eval_add;
+  protean_resident* scratch;  // [grid*block][max_live]
+  int* err;                   // err[0] EINVAL
+};
+cudaError_t launch_depths(const DepthParams& P, int grid, int block, cudaStream_t st);
 cudaError_t preload_sweep_kernel();
 
 // Trace-level stream partition (partition.cu): P1 count + validate, P2 scan, P3 stable scatter.

@@ -178,6 +178,102 @@ __global__ void __launch_bounds__(256) score_kernel(ScoreParams P) {
   }
 }
 
+// N4b: the BE-reserve depth as an enumerated dimension (reading R28).  A lane is (replica r, gpu
+// g, geometry j, depth code c): code 0 replays the GPU-epoch's batches from idle with Alg 1's tag
+// walk, code 1 + d with "the d smallest slices reserved for BE" (strict eligible on positions >= d,
+// fallback to every fitting slice), both through place_lane (O6) and scored by the O8 key.  Grid-
+// stride lanes; each thread's resident list is its own scratch slot.
+__global__ void __launch_bounds__(128) depth_kernel(DepthParams P) {
+  extern __shared__ int32_t tabw[];
+  const int tid = threadIdx.x;
+  for (int i = tid; i < P.tl.words; i += blockDim.x) tabw[i] = P.tab[i];
+  __syncthreads();
+  Tab T;
+  T.bind(tabw, P.tl);
+  const int nc = P.geom_hi - P.geom_lo;
+  const int64_t lanes = (int64_t)P.R * P.N * nc * 8;
+  const int64_t slot = (int64_t)blockIdx.x * blockDim.x + tid;
+  Rows rows{P.scratch + slot * P.max_live};
+  for (int64_t L = slot; L < lanes; L += (int64_t)gridDim.x * blockDim.x) {
+    const int code = (int)(L & 7);
+    const int64_t xj = L >> 3;
+    const int jj = (int)(xj % nc);
+    const int64_t x = xj / nc;
+    const int j = P.geom_lo + jj;
+    int64_t key = -1;
+    if (code <= T.gn[j]) {
+      const int b0 = P.batch_off[x], b1 = P.batch_off[x + 1];
+      int n = 0;
+      int64_t ls[kMaxSl];
+#pragma unroll
+      for (int s = 0; s < kMaxSl; ++s) ls[s] = 0;
+      int64_t misses = 0, tail = 0;
+      for (int b = b0; b < b1; ++b) {
+        const protean_batch& bt = P.batches[b];
+        const PlaceRes pr = place_lane(T, j, rows, n, ls, bt.ready_us, bt.model, bt.strict != 0, P.max_live,
+                                       code - 1);
+        if (bt.strict) {
+          misses += pr.dropped ? bt.n_req
+                               : bt.n_req - hits_sorted(P.arrival + bt.req_off, bt.n_req, pr.end, T.slo[bt.model]);
+        } else {
+          const int64_t tb = pr.dropped ? (int64_t)0xFFFFFFFFLL : pr.end - (int64_t)P.arrival[bt.req_off];
+          tail = tb > tail ? tb : tail;
+        }
+      }
+      key = make_key(misses, tail, P.cur_geom[x] == j ? 0 : j + 1);
+    }
+    P.depth_key[L] = key;
+  }
+}
+
+// Per (replica, gpu): the best code of every geometry (lowest code among equal keys) and the min key
+__global__ void depth_reduce_kernel(DepthParams P) {
+  const int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int nc = P.geom_hi - P.geom_lo;
+  if (x == 0) *P.n_eval += P.n_eval_add;
+  if (x >= (int64_t)P.R * P.N) return;
+  int64_t best = -1;
+  for (int jj = 0; jj < nc; ++jj) {
+    const int64_t* k = P.depth_key + (x * nc + jj) * 8;
+    int bc = 0;
+    for (int c = 1; c < 8; ++c)
+      if (k[c] >= 0 && k[c] < k[bc]) bc = c;
+    if (P.depth_code) P.depth_code[x * nc + jj] = (uint8_t)bc;
+    if (best < 0 || k[bc] < best) best = k[bc];
+  }
+  P.best_key[x] = best;
+}
+
+// Input validation, one thread per (replica, gpu): the sweep's rules (include/protean.h 3b).
+__global__ void depth_validate_kernel(DepthParams P) {
+  const int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (x >= (int64_t)P.R * P.N) return;
+  const int G = P.tl.G, M = P.tl.M;
+  bool bad = P.batch_off[x + 1] < P.batch_off[x] || P.batch_off[0] != 0 ||
+             (P.cur_geom[x] != 0xFF && P.cur_geom[x] >= G);
+  for (int b = P.batch_off[x]; b < P.batch_off[x + 1] && !bad; ++b) {
+    const protean_batch& bt = P.batches[b];
+    if (bt.model >= M || bt.n_req < 1 || bt.strict > 1) bad = true;
+    if (b > P.batch_off[x] && bt.ready_us < P.batches[b - 1].ready_us) bad = true;
+    for (int i = 0; i < bt.n_req && !bad; ++i) {
+      const uint32_t a = P.arrival[bt.req_off + i];
+      if (a > bt.ready_us || (i > 0 && a < P.arrival[bt.req_off + i - 1])) bad = true;
+    }
+  }
+  if (bad) atomicOr(&P.err[0], 1);
+}
+
+cudaError_t launch_depths(const DepthParams& P, int grid, int block, cudaStream_t st) {
+  const int64_t X0 = (int64_t)P.R * P.N;
+  depth_validate_kernel<<<(unsigned)((X0 + 127) / 128), 128, 0, st>>>(P);
+  depth_kernel<<<grid, block, (size_t)P.tl.words * 4, st>>>(P);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  const int64_t X = (int64_t)P.R * P.N;
+  depth_reduce_kernel<<<(unsigned)((X + 127) / 128), 128, 0, st>>>(P);
+  return cudaGetLastError();
+}
+
 size_t score_smem_bytes(const TabLayout& tl, int N, int Gc) {
   return (((size_t)tl.words * 4 + 15) & ~(size_t)15) + (size_t)N * Gc * 8 + (size_t)N;
 }

@@ -296,7 +296,7 @@ __global__ void __launch_bounds__(kSwThreads, PROTEAN_SWEEP_MINB) sweep_kernel(S
           sh.sx[x][s] = T.solo[m * kNProf + p];
         }
       }
-      if (tid < S) sh.cap[tid] = prof_cap(T.gprof[j * 8 + tid]);
+      if (tid < S) sh.cap[tid] = T.cap[T.gprof[j * 8 + tid]];
       __syncthreads();
       uint32_t total = 1;
       for (int x = 0; x < nb; ++x) total *= (uint32_t)S;
