@@ -145,13 +145,16 @@ def load(path: str = None, require_cuda: bool = True):
     L.protean_get_geometries.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p]
     L.protean_num_epochs.argtypes = [C.c_void_p, C.c_int64, C.c_int64, C.c_void_p]
     L.protean_score_epoch.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
-    L.protean_score_epoch_status.argtypes = [C.c_void_p]
+    if hasattr(L, "protean_score_epoch_status"):
+        L.protean_score_epoch_status.argtypes = [C.c_void_p]
     L.protean_sweep_assignments.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
-    L.protean_sweep_depths.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
+    if hasattr(L, "protean_sweep_depths"):  # (older experiment builds loaded by path lack it)
+        L.protean_sweep_depths.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
     L.protean_form_batches.argtypes = [C.c_void_p, C.c_void_p, C.c_int32, C.c_int32, C.c_void_p, C.c_void_p,
                                        C.c_void_p, C.c_void_p, C.c_void_p, C.c_int64, C.c_void_p]
     L.protean_replay_traces.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
-    L.protean_replay_traces_host.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_int32, C.c_void_p]
+    if hasattr(L, "protean_replay_traces_host"):
+        L.protean_replay_traces_host.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_int32, C.c_void_p]
     L.protean_replay_cfg_defaults.argtypes = [C.c_void_p]
     L.protean_replay_cfg_defaults.restype = None
     L.protean_last_timings.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]

@@ -991,6 +991,8 @@ int protean_score_epoch(protean_handle* h, const protean_epoch_in* in, protean_e
   P.price_spot = in->price_spot_node_hr;
   P.scratch = static_cast<protean_resident*>(h->d_scratch);
   P.err = d_err;
+  // resident lists in shared memory when the lanes' lists fit next to the tables (C1: 13 x 1.5 KB)
+  P.smem_lists = score_smem_bytes(h->tl, N, Gc) + score_list_bytes(N, Gc, in->max_live) <= 160 * 1024 ? 1 : 0;
   const int nl = N * (1 + Gc);
   int block = std::max(128, std::min(256, ((nl + 31) / 32) * 32));
   CK(h, launch_score(P, block, st));

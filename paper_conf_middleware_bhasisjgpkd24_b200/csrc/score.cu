@@ -16,6 +16,9 @@ __global__ void __launch_bounds__(256) score_kernel(ScoreParams P) {
   for (int i = tid; i < P.tl.words; i += NT) tabw[i] = P.tab[i];
   int64_t* keys = reinterpret_cast<int64_t*>(smem + (((size_t)P.tl.words * 4 + 15) & ~(size_t)15));
   uint8_t* dec = reinterpret_cast<uint8_t*>(keys + (size_t)N * Gc);
+  // every lane's resident list in shared memory when it fits (P.smem_lists), else global scratch
+  protean_resident* slists = reinterpret_cast<protean_resident*>(
+      reinterpret_cast<unsigned char*>(dec) + (((size_t)N + 15) & ~(size_t)15));
   Tab T;
   T.bind(tabw, P.tl);
   if (tid == 0) bad = 0;
@@ -74,9 +77,11 @@ __global__ void __launch_bounds__(256) score_kernel(ScoreParams P) {
     protean_gpu_state& st = P.state[x];
     const int b0 = P.batch_off[x], b1 = P.batch_off[x + 1];
     if (v == 0) {
-      Rows rows{st.live};
+      Rows rows{P.smem_lists ? slists + (size_t)L * P.max_live : st.live};
       const int geom = st.geom;
       int n = st.n_live;
+      if (P.smem_lists)
+        for (int i = 0; i < n; ++i) rows.r[i] = st.live[i];
       int64_t ls[kMaxSl], bu[kMaxSl], bs[kMaxSl];
 #pragma unroll
       for (int s = 0; s < kMaxSl; ++s) {
@@ -124,6 +129,8 @@ __global__ void __launch_bounds__(256) score_kernel(ScoreParams P) {
         if (mhi > pr.start) memt += (unsigned long long)((int64_t)T.mem[bt.model] * (mhi - pr.start));
       }
       st.n_live = (uint8_t)n;
+      if (P.smem_lists)
+        for (int i = 0; i < n; ++i) st.live[i] = rows.r[i];
 #pragma unroll
       for (int s = 0; s < kMaxSl; ++s) {
         st.last_start_us[s] = ls[s];
@@ -134,7 +141,8 @@ __global__ void __launch_bounds__(256) score_kernel(ScoreParams P) {
       const int j = P.geom_lo + v - 1;
       int64_t key = -1;
       if (dec[g]) {
-        Rows rows{P.scratch + ((size_t)r * N * Gc + (size_t)g * Gc + (v - 1)) * P.max_live};
+        Rows rows{P.smem_lists ? slists + (size_t)L * P.max_live
+                               : P.scratch + ((size_t)r * N * Gc + (size_t)g * Gc + (v - 1)) * P.max_live};
         int n = 0;
         int64_t ls[kMaxSl];
 #pragma unroll
@@ -186,6 +194,7 @@ __global__ void __launch_bounds__(256) score_kernel(ScoreParams P) {
 __global__ void __launch_bounds__(128) depth_kernel(DepthParams P) {
   extern __shared__ int32_t tabw[];
   const int tid = threadIdx.x;
+  if (*(volatile int*)P.err) return;  // the validation kernel (same stream) rejected the input
   for (int i = tid; i < P.tl.words; i += blockDim.x) tabw[i] = P.tab[i];
   __syncthreads();
   Tab T;
@@ -230,6 +239,7 @@ __global__ void __launch_bounds__(128) depth_kernel(DepthParams P) {
 __global__ void depth_reduce_kernel(DepthParams P) {
   const int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const int nc = P.geom_hi - P.geom_lo;
+  if (*(volatile int*)P.err) return;
   if (x == 0) *P.n_eval += P.n_eval_add;
   if (x >= (int64_t)P.R * P.N) return;
   int64_t best = -1;
@@ -275,11 +285,17 @@ cudaError_t launch_depths(const DepthParams& P, int grid, int block, cudaStream_
 }
 
 size_t score_smem_bytes(const TabLayout& tl, int N, int Gc) {
-  return (((size_t)tl.words * 4 + 15) & ~(size_t)15) + (size_t)N * Gc * 8 + (size_t)N;
+  return (((size_t)tl.words * 4 + 15) & ~(size_t)15) + (size_t)N * Gc * 8 + (((size_t)N + 15) & ~(size_t)15);
+}
+
+// the lanes' resident lists in shared memory: N * (1 + Gc) lanes x max_live rows of 24 B
+size_t score_list_bytes(int N, int Gc, int max_live) {
+  return (size_t)N * (1 + Gc) * (size_t)max_live * sizeof(protean_resident);
 }
 
 cudaError_t launch_score(const ScoreParams& P, int block, cudaStream_t st) {
-  const size_t sm = score_smem_bytes(P.tl, P.N, P.geom_hi - P.geom_lo);
+  const size_t sm = score_smem_bytes(P.tl, P.N, P.geom_hi - P.geom_lo) +
+                    (P.smem_lists ? score_list_bytes(P.N, P.geom_hi - P.geom_lo, P.max_live) : 0);
   cudaError_t e = cudaFuncSetAttribute(score_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
   if (e != cudaSuccess) return e;
   score_kernel<<<P.R, block, sm, st>>>(P);
