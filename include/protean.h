@@ -168,7 +168,8 @@ typedef struct {           /* one simulated GPU's carried state; caller-allocate
                                                   union of its batches' [start, end) clipped to
                                                   [0, H) (O6e, "percentage non-idle time");
                                                   cleared with the state on a reconfiguration install */
-  protean_resident live[PROTEAN_MAX_LIVE];
+  protean_resident live[PROTEAN_MAX_LIVE];  /* the live residents as a set: order unspecified
+                                               (score_epoch writes them back grouped by slice) */
 } protean_gpu_state;
 
 typedef struct {           /* 24 B */

@@ -67,6 +67,9 @@ struct protean_handle {
   std::vector<char*> xpeer;              // every rank's buffer in this process
   std::vector<char> x_opened;            // 1 = opened through cudaIpcOpenMemHandle
   char** d_xpeer = nullptr;              // device copy of xpeer
+  // protean_score_epoch: candidate lane packing of the last geometry range
+  uint32_t* d_sc_pack = nullptr;
+  int sc_lo = -1, sc_hi = -1, sc_cw = 0;
   // protean_replay_traces_host: double-buffered device staging of trace chunks and outputs
   void* d_hb[2] = {nullptr, nullptr};
   size_t hb_bytes[2] = {0, 0};
@@ -301,6 +304,7 @@ int xchg_finish(protean_handle* h) {
     int cw = 0;
     std::vector<uint32_t> pk = build_pack(h->gn, b[h->xrank], b[h->xrank + 1], &cw);
     if (h->d_pack_g) cudaFree(h->d_pack_g);
+  if (h->d_sc_pack) cudaFree(h->d_sc_pack);
     h->d_pack_g = nullptr;
     CK(h, cudaMalloc(&h->d_pack_g, pk.size() * 4));
     CK(h, cudaMemcpy(h->d_pack_g, pk.data(), pk.size() * 4, cudaMemcpyHostToDevice));
@@ -523,6 +527,7 @@ void protean_free(protean_handle* h) {
   if (h->d_small) cudaFree(h->d_small);
   if (h->d_pack) cudaFree(h->d_pack);
   if (h->d_pack_g) cudaFree(h->d_pack_g);
+  if (h->d_sc_pack) cudaFree(h->d_sc_pack);
   for (uint32_t* q : h->vr_pack) cudaFree(q);
   if (h->d_vxbuf) cudaFree(h->d_vxbuf);
   if (h->d_vpeer) cudaFree(h->d_vpeer);
@@ -956,13 +961,23 @@ int protean_score_epoch(protean_handle* h, const protean_epoch_in* in, protean_e
   if (!(in->price_od_node_hr >= 0) || !(in->price_spot_node_hr >= 0)) return fail(h, PROTEAN_EINVAL, "price");
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   CK(h, cudaSetDevice(h->device));
-  const int R = in->n_replicas, N = in->n_gpus, Gc = in->geom_hi - in->geom_lo;
+  const int R = in->n_replicas, N = in->n_gpus;
   // enqueue-only: batch_off[0], the states and the batches are validated in the kernel, whose
   // verdict is latched in the handle's device word (protean_score_epoch_status)
-  const size_t need = sizeof(protean_resident) * (size_t)R * N * Gc * in->max_live;
+  const int block = 256;  // 8 warps: one per actual unit / candidate warp of the lane packing
+  const size_t lb = score_list_bytes(N, block, in->max_live);
   {
-    int rc = ensure(h, &h->d_scratch, &h->scratch_bytes, std::max<size_t>(need, 256), st);
+    int rc = ensure(h, &h->d_scratch, &h->scratch_bytes, std::max<size_t>(lb * (size_t)R, 256), st);
     if (rc) return rc;
+  }
+  if (h->sc_lo != in->geom_lo || h->sc_hi != in->geom_hi) {  // lane packing of the range (cached)
+    std::vector<uint32_t> pk = build_pack(h->gn, in->geom_lo, in->geom_hi, &h->sc_cw);
+    if (h->d_sc_pack) cudaFree(h->d_sc_pack);
+    h->d_sc_pack = nullptr;
+    CK(h, cudaMalloc(&h->d_sc_pack, pk.size() * 4));
+    CK(h, cudaMemcpy(h->d_sc_pack, pk.data(), pk.size() * 4, cudaMemcpyHostToDevice));
+    h->sc_lo = in->geom_lo;
+    h->sc_hi = in->geom_hi;
   }
   int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 256);
   ScoreParams P;
@@ -989,12 +1004,11 @@ int protean_score_epoch(protean_handle* h, const protean_epoch_in* in, protean_e
   P.cost = out->cost_usd;
   P.price_od = in->price_od_node_hr;
   P.price_spot = in->price_spot_node_hr;
-  P.scratch = static_cast<protean_resident*>(h->d_scratch);
+  P.pack = h->d_sc_pack;
+  P.cw = h->sc_cw;
+  P.lists = h->d_scratch;
+  P.list_bytes = lb;
   P.err = d_err;
-  // resident lists in shared memory when the lanes' lists fit next to the tables (C1: 13 x 1.5 KB)
-  P.smem_lists = score_smem_bytes(h->tl, N, Gc) + score_list_bytes(N, Gc, in->max_live) <= 160 * 1024 ? 1 : 0;
-  const int nl = N * (1 + Gc);
-  int block = std::max(128, std::min(256, ((nl + 31) / 32) * 32));
   CK(h, launch_score(P, block, st));
   return PROTEAN_OK;
 }

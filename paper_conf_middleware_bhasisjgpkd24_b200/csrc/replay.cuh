@@ -155,8 +155,10 @@ struct ScoreParams {
   int64_t* accum;
   double* cost;               // [R*N] node-epoch VM cost, or NULL
   double price_od, price_spot;
-  protean_resident* scratch;  // [R][N*(Gc)][max_live]
-  int smem_lists;             // 1: every lane's resident list in shared memory (small N x G)
+  const uint32_t* pack;       // [cw * 32] candidate lane packing of [geom_lo, geom_hi)
+  int cw;                     // candidate warps per GPU
+  void* lists;                // per-CTA lane lists, list_bytes each (score_list_bytes)
+  size_t list_bytes;
   int* err;                   // err[0] EINVAL, err[1] ERANGE (latched until protean_score_epoch_status)
 };
 
@@ -243,6 +245,6 @@ cudaError_t replay_occupancy(int block, size_t smem, bool few, int* blocks_per_s
 cudaError_t preload_kernels();
 cudaError_t launch_score(const ScoreParams& P, int block, cudaStream_t st);
 size_t score_smem_bytes(const TabLayout& tl, int N, int Gc);
-size_t score_list_bytes(int N, int Gc, int max_live);
+size_t score_list_bytes(int N, int block, int max_live);
 
 }  // namespace pemgpu

@@ -1,6 +1,6 @@
 """Stall-reason breakdown per code region of replay.cu from an ncu report (source page, cuda,sass
 view).  Regions are the kernel's '// ----' phase markers AND every device function definition
-(tools/ncu_regions.regions), so helper bodies above the kernel (place_group, candidate_unit_fast,
+(tools/ncu_regions.regions_from the report's embedded source), so helper bodies above the kernel (place_group, candidate_unit_fast,
 exchange_keys, ...) are attributed to themselves, not to the marker that precedes them."""
 import collections
 import csv
@@ -9,11 +9,12 @@ import subprocess
 import sys
 
 sys.path.insert(0, os.path.dirname(__file__))
-from ncu_regions import regions  # noqa: E402
+from ncu_lines import lines  # noqa: E402
+from ncu_regions import region_of, regions_from, source_map  # noqa: E402
 
 
 def main(rep):
-    marks = regions()
+    marks = regions_from(source_map(lines(rep)))
     txt = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
                          capture_output=True, text=True).stdout
     hdr, fname = None, None
@@ -31,10 +32,7 @@ def main(rep):
             d = dict(zip(hdr[2:], row[2:]))
             k = fname
             if fname == "replay.cu":
-                k = "?"
-                for i, name in marks:
-                    if int(row[0]) >= i:
-                        k = name
+                k = region_of(marks, int(row[0]))
             for col, v in d.items():
                 if col.startswith("stall_") and "Not Issued" not in col and v.isdigit():
                     agg[k][col[6:]] += int(v)
