@@ -652,8 +652,26 @@ def run_c1(args):
         h.score_epoch_status()
         us = sorted(1e3 * a.elapsed_time(b) for a, b in ts)
         c = o["counters"].cpu().numpy()[0]
+        # cpu_baseline: the oracle's score_epoch on the same batches (one host thread), median of 20
+        from oracle import oracle as O
+        from paper_conf_middleware_bhasisjgpkd24_b200 import _abi as A2
+        O.build()
+        rws = fb["rows"].cpu().numpy()[: fb["n"]]
+        recs = [A2.Batch.from_buffer_copy(bytes(rws[i])) for i in range(fb["n"])]
+        ob = dict(ready=[b.ready_us for b in recs], req_off=[b.req_off for b in recs], n=[b.n_req for b in recs],
+                  model=[b.model for b in recs], strict=[b.strict for b in recs])
+        members = fb["members"].cpu().numpy().view(np.uint32)
+        cts = []
+        for _ in range(20):
+            ost = (O.State * 1)()
+            ost[0].geom, ost[0].target, ost[0].has_vm, ost[0].vm_type = 2, -1, 1, 1
+            t0 = time.perf_counter()
+            O.score_epoch(prof, R=1, N=1, epoch=0, batches=ob, batch_off=[0, fb["n"]], arrival=members, states=ost)
+            cts.append(1e6 * (time.perf_counter() - t0))
+        cts.sort()
         lines.append({"geometries": h.n_geoms, "batches": fb["n"], "median_us": us[50], "min_us": us[0],
-                      "slot_evals_per_call": int(c[8]), "slot_evals_per_s": float(c[8]) / (us[50] * 1e-6)})
+                      "slot_evals_per_call": int(c[8]), "slot_evals_per_s": float(c[8]) / (us[50] * 1e-6),
+                      "cpu_oracle_median_us_1thread": cts[10]})
     line = {"metric": "protean_score_epoch latency (C1)", "value": lines[0]["median_us"], "unit": "us",
             "n_gpus": 1, "steps": 100, "warmup": max(args.warmup, 3), "ms_per_step": lines[0]["median_us"] / 1e3,
             "higher_is_better": False, "scaling": "none", "vs_baseline": None, "dtype": "int64",
@@ -661,6 +679,9 @@ def run_c1(args):
             "config": {"workload": "C1 (configs[0]): 1 sim-GPU, 3 models, 200-request 1 s Poisson trace; one "
                                    "epoch's dispatched batches (protean_form_batches) scored from a fresh state",
                        "per_geometry_set": lines},
+            "cpu_baseline": {"value": lines[0]["cpu_oracle_median_us_1thread"], "unit": "us", "cores": 1,
+                             "kind": "oracle", "sample": "the same 59 batches through oracle.score_epoch, median of 20",
+                             "cpu_model": cpu_info()["model"]},
             "gpu_launches": 1}
     print(json.dumps(line), flush=True)
     return 0

@@ -9,7 +9,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 PKG = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "paper_conf_middleware_bhasisjgpkd24_b200")
 import paper_conf_middleware_bhasisjgpkd24_b200._abi as A  # noqa: E402
 
-A.LIB_PATH = os.path.join(PKG, "libprotean_phase.so")
+A.LIB_PATH = os.path.join(PKG, os.environ.get("PHASE_LIB", "libprotean_phase.so"))
 import torch  # noqa: E402
 
 import paper_conf_middleware_bhasisjgpkd24_b200 as pkg  # noqa: E402
