@@ -901,7 +901,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   P.sl = sl;
   P.WCAP = WCAP;
   size_t o = 0;
-  P.o_alist = o; o += al((size_t)N * kZA * c.max_live * 20);
+  P.o_alist = o; o += al((size_t)N * kZA * (few_r ? 4 : 1) * c.max_live * 20);  // x4: sub-lanes (few)
   P.o_clist = o; o += al((size_t)block * c.max_live * 20);
   P.o_gbat = o; o += al((size_t)WCAP * sizeof(Bat));
   P.o_gord = o; o += al((size_t)WCAP * 4);

@@ -213,5 +213,148 @@ __device__ __forceinline__ SliceOut place_group(const Tab& T, bool active, const
   return o;
 }
 
+
+// ---- Sub-lanes: one warp per simulated GPU, lane = sub * 8 + s; the 4 lanes (s, sub = 0..3) share
+// slice position s and each keeps a quarter of its resident list (a new resident goes to the
+// shortest).  Long lists (overloaded single-replica workloads) are pruned and summed 4 lanes wide;
+// the per-slice quantities are reduced over the 4 sub-lanes (xor 8, 16), the GPU-wide live count
+// and BE memory over the warp, and the slice min-loc runs within each group of 8 as in
+// place_group.  Same results as place_group: every rule of O6 depends on the resident set only.
+__device__ __forceinline__ int64_t sub_sum(int64_t v) {
+  v += __shfl_xor_sync(0xffffffffu, v, 8);
+  return v + __shfl_xor_sync(0xffffffffu, v, 16);
+}
+__device__ __forceinline__ int64_t sub_min(int64_t v) {
+  int64_t o = __shfl_xor_sync(0xffffffffu, v, 8);
+  v = o < v ? o : v;
+  o = __shfl_xor_sync(0xffffffffu, v, 16);
+  return o < v ? o : v;
+}
+__device__ __forceinline__ int warp_sum32(int v) {
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) v += __shfl_xor_sync(0xffffffffu, v, d);
+  return v;
+}
+
+template <int kPL>
+__device__ __forceinline__ SliceOut place_group_sub(const Tab& T, bool active, const SliceLane& K,
+                                                    const LaneList& L, int& n, int64_t& ls,
+                                                    int64_t t, int m, bool strict, int max_live,
+                                                    int64_t* my_start, int64_t* my_end) {
+  const int lane = threadIdx.x & 31, sub = lane >> 3;
+  const int64_t t0 = t > ls ? t : ls;
+  const int32_t* fbr_p = K.fbr_p;
+  const int s = K.s, p = K.p;
+  int64_t used = 0, fs = 0;
+  int32_t be = 0;
+  bool fut = false;
+  if (active) {  // prune this lane's quarter of the list (as place_group)
+    int k = 0;
+#pragma unroll 1
+    for (int i0 = 0; i0 < n; i0 += kPL) {
+      int64_t e_[kPL], s_[kPL];
+      uint32_t m_[kPL];
+#pragma unroll
+      for (int u = 0; u < kPL; ++u) {
+        const int i = i0 + u < n ? i0 + u : i0;
+        e_[u] = L.E(i);
+        s_[u] = L.S(i);
+        m_[u] = L.M(i);
+      }
+#pragma unroll
+      for (int u = 0; u < kPL; ++u) {
+        const int i = i0 + u;
+        const int64_t ei = e_[u];
+        if (i >= n || ei <= t) continue;
+        const int64_t si = s_[u];
+        const uint32_t mi = m_[u];
+        if (k != i) L.put(k, si, ei, mi);
+        ++k;
+        if (!((mi >> 30) & 1)) be += mi & kMemMask;
+        if (ei > t0) {
+          used += mi & kMemMask;
+          fs += fbr_p[((mi >> 24) & 63) * kNProf];
+          fut |= si > t0;
+        }
+      }
+    }
+    n = k;
+  }
+  const int live = warp_sum32(active ? n : 0);
+  const int be_mem = warp_sum32(be);
+  used = sub_sum(used);
+  fs = sub_sum(fs);
+  fut = sub_sum(fut ? 1 : 0) != 0;
+  SliceOut o;
+  o.drop_overflow = live >= max_live;
+  uint64_t key = ~0ull;
+  int64_t start = 0, c = 0;
+  const int32_t q = T.mem[m];
+  const int32_t Ms = K.Ms;
+  const bool doit = active && !o.drop_overflow && q <= Ms;  // uniform over a slice's 4 lanes
+  const int64_t own_f = fbr_p[m * kNProf];
+  int64_t F = own_f + fs;
+  start = t0;
+  bool slow = doit && !(used + q <= Ms && !fut);
+  if (__any_sync(0xffffffffu, slow)) {
+    // the plain definition over the slice's whole list, 4 lanes wide: the held memory, the next
+    // release and Eq 1's co-runner sum at a tried start (first t0, then releases ascending)
+    int64_t e = t0;
+    bool first = true;
+#pragma unroll 1
+    for (;;) {
+      int64_t rem = 0, nxt = INT64_MAX, Fe = 0;
+      if (slow) {
+#pragma unroll 1
+        for (int k = 0; k < n; ++k) {
+          const int64_t ek = L.E(k);
+          if (ek > e) {
+            const uint32_t mk = L.M(k);
+            rem += mk & kMemMask;
+            nxt = ek < nxt ? ek : nxt;
+            if (L.S(k) <= e) Fe += fbr_p[((mk >> 24) & 63) * kNProf];
+          }
+        }
+      }
+      rem = sub_sum(rem);
+      nxt = sub_min(nxt);
+      Fe = sub_sum(Fe);
+      if (slow) {
+        if (rem + q <= Ms) {  // always by the last release (q <= Ms)
+          start = e;
+          F = own_f + Fe;
+          slow = false;
+        } else {
+          e = nxt;
+        }
+      }
+      first = false;
+      if (!__any_sync(0xffffffffu, slow)) break;
+    }
+    (void)first;
+  }
+  if (doit) {
+    c = start + exec_time(K.solo_p[m * kNProf], F);
+    if (strict) {  // choose_strict_slice: tag < 1 (Alg 1 lines 1-8), least eta == least completion
+      const uint64_t inelig = (be_mem >= K.pref) ? (1ull << 62) : 0ull;
+      key = inelig | ((uint64_t)c << 6) | ((uint64_t)(4 - p) << 3) | (uint64_t)s;
+    } else {       // choose_best_effort_slice: first fit, else earliest start (reading Q12)
+      key = ((uint64_t)start << 3) | (uint64_t)s;
+    }
+  }
+  o.kmin = group_min(key, 8);
+  *my_start = start;
+  *my_end = c;
+  // schedule(batch, chosen_slice): the chosen slice's shortest quarter list (lowest sub on ties)
+  const int64_t pick = sub_min(((int64_t)n << 2) | sub);
+  const bool chosen = o.kmin != ~0ull && key == o.kmin;
+  if (chosen && pick == (((int64_t)n << 2) | sub)) {
+    L.put(n, start, c, (uint32_t)q | ((uint32_t)m << 24) | ((uint32_t)(strict ? 1 : 0) << 30));
+    ++n;
+  }
+  if (chosen) ls = start;
+  return o;
+}
+
 }  // namespace pg
 }  // namespace pemgpu

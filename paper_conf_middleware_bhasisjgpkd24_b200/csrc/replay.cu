@@ -314,7 +314,10 @@ __device__ __forceinline__ void prefetch_l2(const void* p, int64_t bytes) {
   }
 }
 
-constexpr int kKR = 6;  // batches per GPU-epoch handled by the register fast path
+#ifndef PROTEAN_KKR
+#define PROTEAN_KKR 7  // measured: 5 -> 41.2, 6 -> 39.8, 7 -> 39.5, 8 -> 40.1 ms (4096 x 120 s)
+#endif
+constexpr int kKR = PROTEAN_KKR;  // batches per GPU-epoch handled by the register fast path
 constexpr int kAK = 4;  // batch ranks per accounting task (phase F)
 constexpr int kBW = 1;  // the warp that lays out the next epoch's windows (phase B) during G
 
@@ -562,8 +565,10 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
   c.ggl = reinterpret_cast<uint32_t*>(slot + P.o_gglist);
   const bool win_smem = SL.WS > 0;  // the epoch window in shared memory (else global scratch)
   c.sarr = win_smem ? reinterpret_cast<uint32_t*>(smem + SL.sarr) : reinterpret_cast<uint32_t*>(slot + P.o_gsarr);
-  // resident lists: actual lanes [N*8 lanes][max_live], candidate lanes [NT lanes][max_live]
-  const int NA = N * kZA;
+  // resident lists: actual lanes [N*8 lanes][max_live] (x 4 sub-lanes in the few-replica instances
+  // with one GPU per warp), candidate lanes [NT lanes][max_live]
+  const bool subm = kPL == 4 && !kN3 && N <= 16 && PROTEAN_FEW_AG == 1;
+  const int NA = N * kZA * (subm ? 4 : 1);
   LaneList AL;
   AL.stride = NA;
   AL.st = reinterpret_cast<int64_t*>(slot + P.o_alist);
@@ -1119,11 +1124,11 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
         int g, s, Z, gbase, j;
         bool valid;
         if (actual) {
-          g = u * AG + (lane >> 3);
+          g = subm ? u : u * AG + (lane >> 3);
           s = lane & 7;
           Z = kZA;
           gbase = lane & ~7;
-          valid = (lane >> 3) < AG && g < N;
+          valid = subm ? g < N : ((lane >> 3) < AG && g < N);
           j = valid ? c.gu8[0 * c.N + g] : 0;
         } else {
           const int cw = cs.cw;
@@ -1154,15 +1159,17 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
         K.s = s;
         K.p = p;
         K.Z = Z;
-        const int al = actual && valid ? g * kZA + s : 0;  // actual lane id
+        const int al = actual && valid ? g * kZA + s : 0;  // actual slice state id
+        const int sub = subm ? lane >> 3 : 0;                // sub-lane of the slice (subm)
         LaneList L;
         if (actual) {
           L = AL;
-          L.st += al; L.en += al; L.mm += al;
+          const int ll = subm ? (actual && valid ? g * 32 + lane : 0) : al;  // actual list id
+          L.st += ll; L.en += ll; L.mm += ll;
         } else {
           L = CL;
         }
-        int n = actual && valid ? c.a_n[al] : 0;
+        int n = actual && valid ? (subm ? (c.a_n[al] >> (8 * sub)) & 0xFF : c.a_n[al]) : 0;
         int64_t ls = actual && valid ? c.a_ls[al] : 0;
         int64_t bu = actual && valid ? c.a_bu[al] : 0;
         const int x0 = valid ? c.g_off[g] : 0, x1 = valid ? c.g_off[g + 1] : 0;
@@ -1212,8 +1219,9 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
             }
           }
           int64_t st, en;
-          const SliceOut so = place_group<kPL>(T, active && has, K, L, n, ls, t, m, strict,
-                                          P.max_live, &st, &en);
+          const SliceOut so = (subm && actual)
+              ? place_group_sub<kPL>(T, active && has, K, L, n, ls, t, m, strict, P.max_live, &st, &en)
+              : place_group<kPL>(T, active && has, K, L, n, ls, t, m, strict, P.max_live, &st, &en);
           const bool placed = !so.drop_overflow && so.kmin != ~0ull;
           const int wl = (gbase + (int)(so.kmin & 7)) & 31;
           const int64_t cwin = __shfl_sync(0xffffffffu, en, wl);
@@ -1225,18 +1233,22 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
           }
           if (!has) continue;
           if (actual) {
-            if (placed && lane == wl) {  // winner: busy union + memory-time, clipped to [0, H)
+            // winner: busy union + memory-time, clipped to [0, H) (with sub-lanes: the slice's 4
+            // lanes keep busy-until replicated, sub-lane 0 accounts and records)
+            if (placed && (subm ? s == (int)(so.kmin & 7) : lane == wl)) {
               const int64_t lo = st > bu ? st : bu;
               const int64_t hi = en < P.H ? en : P.H;
-              if (hi > lo) acc0 += (int64_t)prof_compute(p) * (hi - lo);
+              if (sub == 0) {
+                if (hi > lo) acc0 += (int64_t)prof_compute(p) * (hi - lo);
+                if (hi > st) acc1 += (int64_t)T.mem[m] * (hi - st);
+                bt->slice = (uint8_t)s;
+                bt->start = st;
+                bt->end = en;
+                bt->drop = 0;
+              }
               if (en > bu) bu = en;
-              if (hi > st) acc1 += (int64_t)T.mem[m] * (hi - st);
-              bt->slice = (uint8_t)s;
-              bt->start = st;
-              bt->end = en;
-              bt->drop = 0;
             }
-            if (!placed && lane == gbase) {
+            if (!placed && lane == gbase && sub == 0) {
               bt->drop = so.drop_overflow ? 3 : 2;
               bt->slice = 0xFF;
               bt->start = bt->end = 0;
@@ -1260,19 +1272,25 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
         if (actual) {
           int64_t mx = 0;
           if (valid) {
-            c.a_n[al] = n;
-            c.a_ls[al] = ls;
-            c.a_bu[al] = bu;
+            if (subm) {  // one count byte per sub-list; ls / bu are replicated over the 4 sub-lanes
+              reinterpret_cast<uint8_t*>(c.a_n + al)[sub] = (uint8_t)n;
+            } else {
+              c.a_n[al] = n;
+            }
+            if (sub == 0) {
+              c.a_ls[al] = ls;
+              c.a_bu[al] = bu;
+            }
 #pragma unroll 1
             for (int i = 0; i < n; ++i) mx = L.E(i) > mx ? L.E(i) : mx;
           }
 #pragma unroll
-          for (int d = 1; d < 8; d <<= 1) {
+          for (int d = 1; d < 32; d <<= 1) {  // AG = 1 with sub-lanes: the whole warp is one GPU
             const int64_t o = __shfl_xor_sync(0xffffffffu, mx, d);
-            mx = o > mx ? o : mx;
+            if (subm || d < 8) mx = o > mx ? o : mx;
           }
           const int64_t bsum = group_sum(acc0, 8), msum = group_sum(acc1, 8);
-          if (valid && s == 0) {
+          if (valid && s == 0 && sub == 0) {
             c.gi[5 * c.N + g] = mx;
             c.gi[10 * c.N + g] += bsum;
             c.gi[11 * c.N + g] += msum;
