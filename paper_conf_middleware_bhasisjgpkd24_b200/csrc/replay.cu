@@ -33,6 +33,9 @@
 #ifndef PROTEAN_FEW_AG
 #define PROTEAN_FEW_AG 1  // GPUs per actual-placement warp in the few-replica instances
 #endif
+#ifndef PROTEAN_FEW_NMAX
+#define PROTEAN_FEW_NMAX 16  // up to this many sim-GPUs the few-replica instances use PROTEAN_FEW_AG
+#endif
 #ifndef PROTEAN_MINB
 #define PROTEAN_MINB 3
 #endif
@@ -378,18 +381,25 @@ __device__ __forceinline__ bool candidate_unit_fast(const Tab& T, const SliceLan
       if (used + q <= K.Ms) {
         start = rt0;
         F += fs;
-      } else {  // memory wait: the earliest release on this slice after which the batch fits
-        start = 0xFFFFFFFFu;
+      } else {  // memory wait: the earliest release on this slice after which the batch fits --
+                // releases after rt0 in ascending order, the held footprint only shrinks, so the
+                // first that fits is the minimum (ends at the last release: q <= Ms).  A rolled
+                // walk (O(x) code per batch, not O(x^2)): the unrolled form cost i-cache space.
+        uint32_t e = rt0;
+#pragma unroll 1
+        for (;;) {
+          uint32_t nxt = 0xFFFFFFFFu;
 #pragma unroll
-        for (int jj = 0; jj < x; ++jj) {
-          if (((mine >> jj) & 1u) && en[jj] > rt0) {
-            int32_t rem = 0;
+          for (int i = 0; i < x; ++i)
+            if (((mine >> i) & 1u) && en[i] > e && en[i] < nxt) nxt = en[i];
+          e = nxt;
+          int32_t rem = 0;
 #pragma unroll
-            for (int i = 0; i < x; ++i)
-              if (((mine >> i) & 1u) && en[i] > en[jj]) rem += (int32_t)(mm[i] & kMemMask);
-            if (rem + q <= K.Ms && en[jj] < start) start = en[jj];
-          }
+          for (int i = 0; i < x; ++i)
+            if (((mine >> i) & 1u) && en[i] > e) rem += (int32_t)(mm[i] & kMemMask);
+          if (rem + q <= K.Ms) break;
         }
+        start = e;
 #pragma unroll
         for (int i = 0; i < x; ++i)
           if (((mine >> i) & 1u) && en[i] > start) F += fb[i];
@@ -567,7 +577,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
   c.sarr = win_smem ? reinterpret_cast<uint32_t*>(smem + SL.sarr) : reinterpret_cast<uint32_t*>(slot + P.o_gsarr);
   // resident lists: actual lanes [N*8 lanes][max_live] (x 4 sub-lanes in the few-replica instances
   // with one GPU per warp), candidate lanes [NT lanes][max_live]
-  const bool subm = kPL == 4 && !kN3 && N <= 16 && PROTEAN_FEW_AG == 1;
+  const bool subm = kPL == 4 && !kN3 && N <= PROTEAN_FEW_NMAX && PROTEAN_FEW_AG == 1;
   const int NA = N * kZA * (subm ? 4 : 1);
   LaneList AL;
   AL.stride = NA;
@@ -587,7 +597,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
   // actual-placement warp units: AG GPUs x 8 slice lanes.  Few-replica launches (long lists, slow
   // paths common) give each GPU its own warp, so one GPU's slow path never serialises another's
   // (up to 16 sim-GPUs; beyond, 64-GPU configs keep 4 per warp: more units than warps cost more)
-  const int AG = (kPL == 4 && N <= 16) ? PROTEAN_FEW_AG : kAG;
+  const int AG = (kPL == 4 && N <= PROTEAN_FEW_NMAX) ? PROTEAN_FEW_AG : kAG;
   const int n_aunits = (N + AG - 1) / AG;
   const uint32_t* sarr = c.sarr;
 
