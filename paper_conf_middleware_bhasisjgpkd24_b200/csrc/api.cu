@@ -331,32 +331,27 @@ int xchg_finish(protean_handle* h) {
 // P2 run indices and the P3 stable scatter into the stream-sorted copy (h->d_sa at h->d_saoff).
 // Request-level faults found by P3 are left in err[0] for the caller to report after its kernels.
 // timing: record the prepass / partition events read by protean_last_timings.
-int partition_trace(protean_handle* h, const protean_replay_cfg& c, const std::vector<int64_t>& roff,
-                    int64_t E, cudaStream_t st, bool timing, unsigned long long* wmax_out) {
+int partition_trace(protean_handle* h, const protean_replay_cfg& c, int64_t E, cudaStream_t st,
+                    bool timing, unsigned long long* wmax_out) {
   const int R = c.n_replicas, S = 2 * h->M;
   const int64_t W = c.epoch_len_us;
   {
     void* p = h->d_eoff;
     int rc = ensure(h, &p, &h->eoff_bytes, sizeof(int64_t) * (size_t)R * (size_t)(E + 1), st);
     h->d_eoff = static_cast<int64_t*>(p);
+    if (!rc) rc = ensure(h, &h->d_cnt, &h->cnt_bytes, std::max<size_t>(4, sizeof(uint32_t) * (size_t)R * E * S), st);
+    if (!rc) rc = ensure(h, &h->d_sidx, &h->sidx_bytes, std::max<size_t>(4, sizeof(uint32_t) * (size_t)R * (E + 1) * S), st);
+    if (!rc) rc = ensure(h, &h->d_saoff, &h->saoff_bytes, sizeof(int64_t) * (size_t)(R + 1), st);
     if (rc) return rc;
   }
   unsigned long long* d_wmax = static_cast<unsigned long long*>(h->d_small);
   int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 64);
   CK(h, cudaMemsetAsync(h->d_small, 0, 256, st));
   if (timing) CK(h, cudaEventRecord(h->ev[0], st));
+  // replica_off is validated and scanned on the device: the call's only host round trip before
+  // the replay is the one below (the window size and the copy's length size the next launches)
+  CK(h, launch_roff_scan(c.replica_off, R, static_cast<int64_t*>(h->d_saoff), d_err, st));
   CK(h, launch_prepass(c.arrival_us, c.replica_off, R, E, W, h->maxT, h->d_eoff, d_wmax, d_err, st));
-  std::vector<int64_t> saoff(R + 1);
-  saoff[0] = 0;
-  for (int r = 0; r < R; ++r) saoff[r + 1] = saoff[r] + ((roff[r + 1] - roff[r] + 3) & ~(int64_t)3);
-  {
-    int rc = ensure(h, &h->d_cnt, &h->cnt_bytes, std::max<size_t>(4, sizeof(uint32_t) * (size_t)R * E * S), st);
-    if (!rc) rc = ensure(h, &h->d_sidx, &h->sidx_bytes, std::max<size_t>(4, sizeof(uint32_t) * (size_t)R * (E + 1) * S), st);
-    if (!rc) rc = ensure(h, &h->d_sa, &h->sa_bytes, std::max<size_t>(16, sizeof(uint32_t) * (size_t)saoff[R]), st);
-    if (!rc) rc = ensure(h, &h->d_saoff, &h->saoff_bytes, sizeof(int64_t) * (size_t)(R + 1), st);
-    if (rc) return rc;
-  }
-  CK(h, cudaMemcpyAsync(h->d_saoff, saoff.data(), sizeof(int64_t) * (R + 1), cudaMemcpyHostToDevice, st));
   PartitionArgs PA;
   PA.arr = c.arrival_us;
   PA.meta = c.meta;
@@ -372,19 +367,27 @@ int partition_trace(protean_handle* h, const protean_replay_cfg& c, const std::v
            ((reinterpret_cast<uintptr_t>(c.meta) & 15u) == 0);
   PA.cnt = static_cast<uint32_t*>(h->d_cnt);
   PA.sidx = static_cast<uint32_t*>(h->d_sidx);
-  PA.sa = static_cast<uint32_t*>(h->d_sa);
+  PA.sa = nullptr;
   PA.err = d_err;
   CK(h, launch_partition_count(PA, st));
   if (timing) CK(h, cudaEventRecord(h->ev[1], st));
   unsigned long long wmax = 0;
   int herr = 0;
+  int64_t sa_len = 0;
   CK(h, cudaMemcpyAsync(&wmax, d_wmax, 8, cudaMemcpyDeviceToHost, st));
-  CK(h, cudaMemcpyAsync(&herr, d_err, 4, cudaMemcpyDeviceToHost, st));  // also keeps saoff alive
+  CK(h, cudaMemcpyAsync(&herr, d_err, 4, cudaMemcpyDeviceToHost, st));
+  CK(h, cudaMemcpyAsync(&sa_len, static_cast<int64_t*>(h->d_saoff) + R, 8, cudaMemcpyDeviceToHost, st));
   CK(h, cudaStreamSynchronize(st));
+  if (herr & 4) return fail(h, PROTEAN_EINVAL, "replica_off: first entry != 0 or not monotone");
   // the prepass guarantees that the epoch ranges tile every replica (else the scatter could leave
   // it); request-level validation happens in the scatter pass and is reported by the caller
   if (herr) return fail(h, PROTEAN_EINVAL, "arrivals not sorted or beyond the trace");
   if (wmax >= (1ull << 25)) return fail(h, PROTEAN_ERANGE, "epoch window >= 2^25 requests");
+  {
+    int rc = ensure(h, &h->d_sa, &h->sa_bytes, std::max<size_t>(16, sizeof(uint32_t) * (size_t)sa_len), st);
+    if (rc) return rc;
+  }
+  PA.sa = static_cast<uint32_t*>(h->d_sa);
   // P2 + P3: run indices and the stable scatter (only on a validated trace)
   if (timing) CK(h, cudaEventRecord(h->ev[4], st));
   CK(h, launch_partition_rest(PA, st));
@@ -699,13 +702,6 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   CK(h, cudaSetDevice(h->device));
   const int R = c.n_replicas, N = c.n_gpus;
-  std::vector<int64_t> roff(R + 1);
-  CK(h, cudaMemcpyAsync(roff.data(), c.replica_off, sizeof(int64_t) * (R + 1), cudaMemcpyDeviceToHost, st));
-  CK(h, cudaStreamSynchronize(st));
-  if (roff[0] != 0) return fail(h, PROTEAN_EINVAL, "replica_off[0] != 0");
-  for (int r = 0; r < R; ++r)
-    if (roff[r + 1] < roff[r]) return fail(h, PROTEAN_EINVAL, "replica_off not monotone");
-
   const int64_t W = c.epoch_len_us;
   const int64_t E = (c.trace_len_us + W - 1) / W + ((int64_t)h->maxT + W - 1) / W;
   const int64_t H = E * W;
@@ -716,7 +712,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   unsigned long long wmax = 0;
   int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 64);
   {
-    int rc = partition_trace(h, c, roff, E, st, true, &wmax);
+    int rc = partition_trace(h, c, E, st, true, &wmax);
     if (rc) return rc;
   }
   int herr = 0;
@@ -797,6 +793,8 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   int per_sm = 0;
   CK(h, replay_occupancy(block, sl.total, few_r, &per_sm));
   if (per_sm < 1) return fail(h, PROTEAN_ERANGE, "replay kernel does not fit an SM");
+  if (const char* ev = std::getenv("PROTEAN_PER_SM"))  // experiment knob: fewer resident CTAs per SM
+    per_sm = std::max(1, std::min(per_sm, std::atoi(ev)));
   int grid = (int)std::min<int64_t>((int64_t)R * vr_n, (int64_t)h->nsm * per_sm);
   grid -= grid % vr_n;  // every replica's CTAs are resident together (exchange partners)
   if (c.max_ctas > 0) grid = std::min(grid, std::max(c.max_ctas, vr_n) / vr_n * vr_n);
@@ -1169,7 +1167,7 @@ int protean_form_batches(protean_handle* h, const protean_replay_cfg* cfg, int32
   int* d_err = reinterpret_cast<int*>(static_cast<char*>(h->d_small) + 64);
   {
     unsigned long long wmax = 0;
-    int rc = partition_trace(h, c, roff, E, st, false, &wmax);
+    int rc = partition_trace(h, c, E, st, false, &wmax);
     if (rc) return rc;
   }
   int herr = 0;

@@ -171,6 +171,7 @@ __global__ void __launch_bounds__(32 * kPW) part_count_kernel(const uint32_t* ar
   __syncthreads();
   const int64_t idx = (int64_t)blockIdx.x * kPW + warp;
   if (idx >= (int64_t)R * E) return;
+  if (*(volatile const int*)err & 4) return;  // replica_off rejected: eoff was not written
   const int r = (int)(idx / E);
   const int64_t e = idx - (int64_t)r * E;
   const int64_t lo = eoff[(size_t)r * (E + 1) + e], hi = eoff[(size_t)r * (E + 1) + e + 1];

@@ -1608,6 +1608,62 @@ extern "C" int protean_debug_phase_cycles(unsigned long long* out) {
 }
 #endif
 
+// replica_off on the device (no host round trip before the prepass): one CTA checks
+// replica_off[0] == 0 and monotone (else err[0] |= 4, and every later pass of the call skips) and
+// writes the stream-sorted copy's per-replica offsets saoff[r] = sum over r' < r of the replica's
+// request count rounded up to 4 (16-byte aligned runs), saoff[R] = the copy's length.
+__global__ void __launch_bounds__(1024) roff_scan_kernel(const int64_t* roff, int R, int64_t* saoff,
+                                                         int* err) {
+  __shared__ int64_t wsum[32];
+  __shared__ int64_t carry;
+  __shared__ int bad;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (tid == 0) {
+    carry = 0;
+    bad = roff[0] != 0;
+    saoff[0] = 0;
+  }
+  __syncthreads();
+#pragma unroll 1
+  for (int r0 = 0; r0 < R; r0 += 1024) {
+    const int r = r0 + tid;
+    int64_t v = 0;
+    if (r < R) {
+      const int64_t n = roff[r + 1] - roff[r];
+      if (n < 0) bad = 1;
+      v = n < 0 ? 0 : (n + 3) & ~(int64_t)3;
+    }
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const int64_t y = __shfl_up_sync(0xffffffffu, v, d);
+      if (lane >= d) v += y;
+    }
+    if (lane == 31) wsum[warp] = v;
+    __syncthreads();
+    if (warp == 0) {
+      int64_t w = wsum[lane];
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const int64_t y = __shfl_up_sync(0xffffffffu, w, d);
+        if (lane >= d) w += y;
+      }
+      wsum[lane] = w;  // inclusive over warps
+    }
+    __syncthreads();
+    const int64_t incl = carry + v + (warp ? wsum[warp - 1] : 0);
+    if (r < R) saoff[r + 1] = incl;
+    __syncthreads();
+    if (tid == 1023) carry = incl;
+    __syncthreads();
+  }
+  if (tid == 0 && bad) atomicOr(err, 4);
+}
+
+cudaError_t launch_roff_scan(const int64_t* roff, int R, int64_t* saoff, int* err, cudaStream_t st) {
+  roff_scan_kernel<<<1, 1024, 0, st>>>(roff, R, saoff, err);
+  return cudaGetLastError();
+}
+
 // Prepass: eoff[r][e] = first request of replica r with arrival >= e*W (e = 0..E), and the
 // largest request window any epoch needs: [lower_bound(eW - maxT), eoff[e+1]).  A warp covers 32
 // consecutive epochs of one replica and owns the first 31 (lane 31 only computes its lower bound
@@ -1619,6 +1675,7 @@ extern "C" int protean_debug_phase_cycles(unsigned long long* out) {
 __global__ void prepass_kernel(const uint32_t* arr, const int64_t* roff, int R, int64_t E,
                                int64_t W, int64_t maxT, int64_t* eoff, unsigned long long* wmax,
                                int* err) {
+  if (*(volatile int*)err & 4) return;  // replica_off rejected by roff_scan_kernel
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t wpr = (E + 31) / 31;  // warps per replica: epochs 0..E, 31 owned per warp

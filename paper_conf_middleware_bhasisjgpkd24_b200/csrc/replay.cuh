@@ -237,6 +237,7 @@ cudaError_t launch_partition_rest(const PartitionArgs& A, cudaStream_t st);
 cudaError_t preload_partition_kernels();
 
 // launchers (replay.cu / score.cu)
+cudaError_t launch_roff_scan(const int64_t* roff, int R, int64_t* saoff, int* err, cudaStream_t st);
 cudaError_t launch_prepass(const uint32_t* arr, const int64_t* roff, int R, int64_t E, int64_t W,
                            int64_t maxT, int64_t* eoff, unsigned long long* wmax, int* err,
                            cudaStream_t st);

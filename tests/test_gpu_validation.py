@@ -11,6 +11,7 @@ import pytest
 
 from gpu_common import compare, gpu_replay, oracle_replay
 from protean_inputs import concat, pack_meta, random_profiles
+from protean_inputs.traces import Trace
 
 pytestmark = pytest.mark.gpu
 
@@ -142,3 +143,46 @@ def test_score_epoch_enqueue_only_verdict(oracle):
         oracle.score_epoch(P, R=1, N=1, epoch=0, batches=dict(ready=[5000], req_off=[0], n=[2], model=[1], strict=[0]),
                            batch_off=[0, 1], arrival=np.array([0, 5000], np.uint32), states=ostate)
     assert ei.value.code == A.EINVAL
+
+
+def test_replica_off_checked_on_device(oracle):
+    """replica_off is validated and scanned on the device (roff_scan_kernel; no host readback
+    before the prepass): replica_off[0] != 0 or a decreasing entry is PROTEAN_EINVAL like the
+    oracle's host check, with nothing else launched on the bad offsets; a valid trace of more
+    replicas than the scan's 1024-wide chunk (empty replicas included) matches the oracle."""
+    import torch
+    import paper_conf_middleware_bhasisjgpkd24_b200 as pkg
+    from paper_conf_middleware_bhasisjgpkd24_b200 import _abi as A
+    rng = np.random.default_rng(21)
+    prof = random_profiles(rng, 3)
+    T = 2_000_000
+    parts = []
+    for r in range(1100):
+        n = 0 if r % 7 == 3 else int(rng.integers(1, 12))
+        a, m, _ = _trace(rng, n=n, M=3, T=T)
+        parts.append((a, m))
+    tr = concat(parts, T)
+    h = pkg.load_profiles(prof)
+    arr = torch.from_numpy(tr.arrival_us.view(np.int32)).cuda()
+    meta = torch.from_numpy(tr.meta).cuda()
+    R = len(parts)
+    out = h.replay_traces(arr, meta, torch.from_numpy(tr.replica_off).cuda(), trace_len_us=T, n_gpus=2)
+    o = oracle_replay(oracle, prof, tr, want_keys=False, want_log=False, n_gpus=2)
+    assert np.array_equal(out["counters"].cpu().numpy(), o["counters"])
+    assert np.array_equal(out["hist"].cpu().numpy().view(np.uint32), o["hist"])
+    for bad in ("first", "decreasing"):
+        off = tr.replica_off.copy()
+        if bad == "first":
+            off[0] = 1
+        else:
+            off[600] = off[599] - 1 if off[599] > 0 else off[601] + 5
+        with pytest.raises(pkg.ProteanError) as ei:
+            h.replay_traces(arr, meta, torch.from_numpy(off).cuda(), trace_len_us=T, n_gpus=2)
+        assert ei.value.code == A.EINVAL
+        with pytest.raises(oracle.OracleError) as eo:
+            oracle_replay(oracle, prof, Trace(tr.arrival_us, tr.meta, off, T),
+                          want_keys=False, want_log=False, n_gpus=2)
+        assert eo.value.code == A.EINVAL
+    # the handle is usable afterwards
+    out2 = h.replay_traces(arr, meta, torch.from_numpy(tr.replica_off).cuda(), trace_len_us=T, n_gpus=2)
+    assert np.array_equal(out2["counters"].cpu().numpy(), o["counters"])
