@@ -24,6 +24,12 @@
 #ifndef PROTEAN_D_BARRIER
 #define PROTEAN_D_BARRIER 1
 #endif
+#ifndef PROTEAN_ACCT_UNROLL
+#define PROTEAN_ACCT_UNROLL 1  // measured (4096 x 120 s): 4 -> 38.2, 2 -> 38.7, 1 -> 37.1 ms (code size)
+#endif
+#ifndef PROTEAN_RANK_UNROLL
+#define PROTEAN_RANK_UNROLL 4  // 1 -> 38.9 ms
+#endif
 #ifndef PROTEAN_WARP_G
 #define PROTEAN_WARP_G 1
 #endif
@@ -320,7 +326,8 @@ __device__ __forceinline__ void prefetch_l2(const void* p, int64_t bytes) {
 #ifndef PROTEAN_KKR
 #define PROTEAN_KKR 7  // measured: 5 -> 41.2, 6 -> 39.8, 7 -> 39.5, 8 -> 40.1 ms (4096 x 120 s)
 #endif
-constexpr int kKR = PROTEAN_KKR;  // batches per GPU-epoch handled by the register fast path
+constexpr int kKR = PROTEAN_KKR;
+constexpr int kAcctUnroll = PROTEAN_ACCT_UNROLL, kRankUnroll = PROTEAN_RANK_UNROLL;  // batches per GPU-epoch handled by the register fast path
 constexpr int kAK = 4;  // batch ranks per accounting task (phase F)
 constexpr int kBW = 1;  // the warp that lays out the next epoch's windows (phase B) during G
 
@@ -890,7 +897,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
       for (int b = tid; b < nb; b += NT) {  // id order (O3): rank by key
         const uint64_t kb = bats[b].key;
         int rank = 0;
-#pragma unroll 4
+#pragma unroll kRankUnroll
         for (int x = 0; x < nb; ++x) rank += (bats[x].key < kb) ? 1 : 0;
         ord[rank] = (uint32_t)b;
         if (avail_all) {
@@ -1096,7 +1103,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
                 // bucket = 128 s + (lat >> s), s = max(0, floor(log2 lat) - 7) (O7, reading Q30)
                 const uint32_t e32 = (uint32_t)bend;
                 const uint32_t slo32 = slo > (int64_t)0xFFFFFFFFLL ? 0xFFFFFFFFu : (uint32_t)slo;
-#pragma unroll 4
+#pragma unroll kAcctUnroll
                 for (int i0 = 0; i0 < nreq; i0 += 32) {
                   const int i = i0 + lane;
                   const bool valid = i < nreq;
