@@ -451,6 +451,13 @@ __device__ __forceinline__ bool candidate_unit_fast(const Tab& T, const SliceLan
 
 }  // namespace
 
+// The n-th (0-based) set bit of m (n < popcount(m)).
+__device__ __forceinline__ int nth_bit64(uint64_t m, int n) {
+  const uint32_t lo = (uint32_t)m;
+  const int pl = __popc(lo);
+  return n < pl ? (int)__fns(lo, 0, n + 1) : 32 + (int)__fns((uint32_t)(m >> 32), 0, n - pl + 1);
+}
+
 // Fold the per-warp request counters of the epoch (phase F) into the replica's 64-bit counters
 // 0..6 (O7) and clear them; called by all lanes of warp 0 after the phase-E barrier.
 __device__ __forceinline__ void fold_wcnt(CtaState& cs, uint32_t (*wcnt)[5], int NW, int lane) {
@@ -917,17 +924,18 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
       // ---------------------------------------------------------------- D: dispatch
       if (avail_all) {
         // done above
-      } else if (N <= 32) {
+      } else if (N <= 64) {
         // availability mask per batch (parallel); then runs of equal masks are dispatched in
         // closed form: inside a run the k-th batch goes to the (i0 + k) mod |A|-th available GPU
+        // (i0: the first available at or after the cursor), exactly the serial round robin (O4)
 #pragma unroll 1
         for (int rk = tid; rk < nb; rk += NT) {
           Bat& bt = bats[ord[rk]];
           const int64_t t = bt.ready;
-          uint32_t m = 0;
+          uint64_t m = 0;
 #pragma unroll 1
           for (int g = 0; g < N; ++g)
-            if (available(c, g, t)) m |= 1u << g;
+            if (available(c, g, t)) m |= 1ull << g;
           bt.key = m;  // the id-order key is no longer needed
         }
         __syncthreads();
@@ -935,17 +943,17 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
           int cur = cs.cursor;
 #pragma unroll 1
           for (int r0 = 0; r0 < nb;) {
-            const uint32_t m = (uint32_t)bats[ord[r0]].key;
+            const uint64_t m = bats[ord[r0]].key;
             int r1 = r0 + 1;
 #pragma unroll 1
             for (;;) {  // end of the run of equal masks
               const int rk = r1 + lane;
-              const unsigned dm = __ballot_sync(0xffffffffu, rk >= nb || (uint32_t)bats[ord[rk]].key != m);
+              const unsigned dm = __ballot_sync(0xffffffffu, rk >= nb || bats[ord[rk]].key != m);
               if (dm) { r1 += __ffs(dm) - 1; break; }
               r1 += 32;
             }
-            const int A = __popc(m);
-            const int i0 = A ? __popc(m & ((1u << cur) - 1u)) % A : 0;  // first available >= cur
+            const int A = __popcll(m);
+            const int i0 = A ? __popcll(m & ((1ull << cur) - 1ull)) % A : 0;  // first available >= cur
 #pragma unroll 1
             for (int rk = r0 + lane; rk < r1; rk += 32) {
               Bat& bt = bats[ord[rk]];
@@ -953,31 +961,51 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
                 bt.gpu = 0xFF;
                 bt.drop = 1;  // dispatch drop
               } else {
-                bt.gpu = (uint8_t)__fns(m, 0, (i0 + (rk - r0)) % A + 1);
+                bt.gpu = (uint8_t)nth_bit64(m, (i0 + (rk - r0)) % A);
               }
             }
-            if (A) cur = ((int)__fns(m, 0, (i0 + (r1 - 1 - r0)) % A + 1) + 1) % N;
+            if (A) cur = (nth_bit64(m, (i0 + (r1 - 1 - r0)) % A) + 1) % N;
             r0 = r1;
           }
           __syncwarp();
-          // lanes = GPUs: per-GPU counts, offsets, and the id-ordered per-GPU lists
-          int mycnt = 0;
+          // per-GPU lists in id order: a warp-stable counting sort over 32 ranks at a time (peers by
+          // match_any; the highest peer lane advances the GPU's running count)
+          if (lane < N) c.g_cnt[lane] = 0;
+          if (lane + 32 < N) c.g_cnt[lane + 32] = 0;
+          __syncwarp();
 #pragma unroll 1
-          for (int rk = 0; rk < nb; ++rk) mycnt += (bats[ord[rk]].gpu == lane) ? 1 : 0;
-          int x = mycnt;
+          for (int rk0 = 0; rk0 < nb; rk0 += 32) {
+            const int rk = rk0 + lane;
+            const int gg = rk < nb ? bats[ord[rk]].gpu : 0xFF;
+            const unsigned peers = __match_any_sync(0xffffffffu, gg);
+            if (gg < N && lane == 31 - __clz(peers)) c.g_cnt[gg] += __popc(peers);
+            __syncwarp();
+          }
+          const int c0 = lane < N ? c.g_cnt[lane] : 0, c1 = lane + 32 < N ? c.g_cnt[lane + 32] : 0;
+          int x0 = c0, x1 = c1;
 #pragma unroll
           for (int d = 1; d < 32; d <<= 1) {
-            const int y = __shfl_up_sync(0xffffffffu, x, d);
-            if (lane >= d) x += y;
+            const int y0 = __shfl_up_sync(0xffffffffu, x0, d), y1 = __shfl_up_sync(0xffffffffu, x1, d);
+            if (lane >= d) { x0 += y0; x1 += y1; }
           }
-          if (lane < N) c.g_off[lane] = x - mycnt;
-          if (lane == N - 1) c.g_off[N] = x;
+          const int t0 = __shfl_sync(0xffffffffu, x0, 31), t1 = __shfl_sync(0xffffffffu, x1, 31);
+          if (lane < N) { c.g_off[lane] = x0 - c0; c.g_cnt[lane] = 0; }
+          if (lane + 32 < N) { c.g_off[lane + 32] = t0 + x1 - c1; c.g_cnt[lane + 32] = 0; }
+          if (lane == 0) c.g_off[N] = t0 + t1;  // dropped batches (gpu 0xFF) are in no list
           __syncwarp();
-          int fill = 0;
 #pragma unroll 1
-          for (int rk = 0; rk < nb; ++rk) {
-            const uint32_t b = ord[rk];
-            if (bats[b].gpu == lane) gl[c.g_off[lane] + fill++] = b;
+          for (int rk0 = 0; rk0 < nb; rk0 += 32) {
+            const int rk = rk0 + lane;
+            const uint32_t b = rk < nb ? ord[rk] : 0u;
+            const int gg = rk < nb ? bats[b].gpu : 0xFF;
+            const unsigned peers = __match_any_sync(0xffffffffu, gg);
+            const int base = gg < N ? c.g_off[gg] + c.g_cnt[gg] : 0;
+            __syncwarp();
+            if (gg < N) {
+              gl[base + __popc(peers & ((1u << lane) - 1u))] = b;
+              if (lane == 31 - __clz(peers)) c.g_cnt[gg] += __popc(peers);
+            }
+            __syncwarp();
           }
           if (lane == 0) cs.cursor = cur;
         }

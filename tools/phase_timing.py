@@ -20,15 +20,19 @@ R = int(sys.argv[1]) if len(sys.argv) > 1 else 444
 S = int(sys.argv[2]) if len(sys.argv) > 2 else 60
 MIX = os.environ.get("PHASE_MIX", "a")
 NG = int(os.environ.get("PHASE_N", "8"))
+GS = 0
 if MIX == "b":
     from protean_inputs import mix_b_params
     gp = mix_b_params(R, seed=2, seconds=S)
+elif MIX == "b8":  # the C4 shape: Mix B x 8, 37 geometries (use PHASE_N=64)
+    from protean_inputs import mix_b_params
+    gp, GS = mix_b_params(R, seed=4, seconds=S, scale=8.0), 1
 else:
     gp = mix_a_params(R, seed=1, seconds=S)
 arr, meta, roff = tracegen.generate_on_device(gp, 0)
 A._lib = None
 L = A.load(A.LIB_PATH)
-h = pkg.load_profiles(synth_profiles())
+h = pkg.load_profiles(synth_profiles().with_geometry_set(GS))
 POL = int(sys.argv[3]) if len(sys.argv) > 3 else 0
 out = h.replay_traces(arr, meta, roff, trace_len_us=gp.trace_len_us, n_gpus=NG, policy=POL)
 torch.cuda.synchronize()
