@@ -56,6 +56,8 @@ struct protean_handle {
   void* d_vxbuf = nullptr;
   size_t vx_bytes = 0;
   char** d_vpeer = nullptr;
+  void* d_vdone = nullptr;  // [R] finalize arrival counters of the split accounting
+  size_t vdone_bytes = 0;
   XLayout vxl{0, 0, 0};
   uint32_t vseq = 0;
   // mode G exchange (protean_xchg_*)
@@ -533,6 +535,7 @@ void protean_free(protean_handle* h) {
   if (h->d_sc_pack) cudaFree(h->d_sc_pack);
   for (uint32_t* q : h->vr_pack) cudaFree(q);
   if (h->d_vxbuf) cudaFree(h->d_vxbuf);
+  if (h->d_vdone) cudaFree(h->d_vdone);
   if (h->d_vpeer) cudaFree(h->d_vpeer);
   xchg_release(h);
   for (int i = 0; i < 6; ++i)
@@ -874,7 +877,16 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
     P.xtimeout_ns = 30ull * 1000000000ull;
     if (const char* ev = std::getenv("PROTEAN_XCHG_TIMEOUT_S"))
       P.xtimeout_ns = (uint64_t)std::max(1, std::atoi(ev)) * 1000000000ull;
-    CK(h, cudaMemsetAsync(out->counters, 0, sizeof(int64_t) * 10 * (size_t)R, st));  // 8, 9 accumulate
+    // the CTAs of a replica split the accounting: counters, histogram and finalize's arrival
+    // counter accumulate
+    CK(h, cudaMemsetAsync(out->counters, 0, sizeof(int64_t) * 10 * (size_t)R, st));
+    CK(h, cudaMemsetAsync(out->hist, 0, sizeof(uint32_t) * 2 * PROTEAN_NBUCKETS * (size_t)R, st));
+    {
+      int rc = ensure(h, &h->d_vdone, &h->vdone_bytes, sizeof(uint32_t) * (size_t)R, st);
+      if (rc) return rc;
+    }
+    CK(h, cudaMemsetAsync(h->d_vdone, 0, sizeof(uint32_t) * (size_t)R, st));
+    P.vr_done = static_cast<uint32_t*>(h->d_vdone);
   }
   if (modeG && !std::getenv("PROTEAN_XCHG_OFF")) {  // debug knob: score the range, no exchange
     P.xl = h->xl;

@@ -542,6 +542,9 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
   const int vr = (int)(blockIdx.x % (unsigned)vrn);
   const int glo = vrn > 1 ? P.vr_lo[vr] : P.geom_lo, ghi = vrn > 1 ? P.vr_hi[vr] : P.geom_hi;
   const int cwr = vrn > 1 ? P.vr_cw[vr] : SL.CW;
+  // the few-replica instances split the replica's accounting over its virtual ranks (the
+  // many-replica instance, where virtual ranks are an explicit request, replicates it)
+  const bool vsplit = kPL == 4 && vrn > 1;
   const uint32_t* pack_src = vrn > 1 ? P.vr_pack[vr] : P.pack;
   if (tid == 0) {
     cs.glo = glo;
@@ -1098,7 +1101,10 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
       // dynamic task queue: [actual units][candidate units][accounting of batch rank rk];
       // accounting waits (rarely) for the actual units, whose warps publish via cs.adone
       const int n_units = n_aunits + (P.policy == 0 ? N * cs.cw : 0);
-      const int n_tasks = n_units + (nb + kAK - 1) / kAK;
+      // split accounting (vsplit): CTA vr takes tasks vr, vr + vrn, ... (counters and the histogram
+      // are summed in finalize); otherwise every CTA takes them all
+      const int ntk = (nb + kAK - 1) / kAK;
+      const int n_tasks = n_units + (vsplit ? (ntk + vrn - 1 - vr) / vrn : ntk);
 #ifndef PROTEAN_ACCT_BARRIER
 #define PROTEAN_ACCT_BARRIER 0  // 1: debug build for compute-sanitizer racecheck (accounting after a CTA barrier)
 #endif
@@ -1134,7 +1140,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
             }
           }
           __syncwarp();
-          const int rk0 = (u - n_units) * kAK, rk1 = min(nb, rk0 + kAK);
+          const int rk0 = (vsplit ? (u - n_units) * vrn + vr : u - n_units) * kAK, rk1 = min(nb, rk0 + kAK);
           uint32_t c_sarr = 0, c_met = 0, c_sdrop = 0, c_barr = 0, c_bdrop = 0;  // warp-uniform
 #pragma unroll 1
           for (int rk = rk0; rk < rk1; ++rk) {
@@ -1605,14 +1611,27 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
     // ---------------------------------------------------------------- finalize (O12)
 #pragma unroll 1
     for (int g = tid; g < N; g += NT) bill_switch(c, g, VM_NONE, P.H, P.H);
+    bool pct_here = true;  // this CTA holds the replica's whole histogram
+    if (vsplit) {  // partial histograms (split accounting): summed in HBM, the last CTA ranks them
 #pragma unroll 1
-    for (int w = tid; w < 2 * kNB; w += NT) ghist[w] = s_hist[w];  // histogram to HBM
-    __syncthreads();
-    if (warp < 2) {  // nearest-rank P50 / P99 per class
+      for (int w = tid; w < 2 * kNB; w += NT)
+        if (s_hist[w]) atomicAdd(ghist + w, s_hist[w]);
+      __threadfence();
+      __syncthreads();
+      if (tid == 0) cs.task = (int)(atomicAdd(P.vr_done + r, 1u) == (unsigned)(vrn - 1));
+      __syncthreads();
+      pct_here = cs.task != 0;
+      __threadfence();
+    } else {
+#pragma unroll 1
+      for (int w = tid; w < 2 * kNB; w += NT) ghist[w] = s_hist[w];  // histogram to HBM
+      __syncthreads();
+    }
+    if (warp < 2 && pct_here) {  // nearest-rank P50 / P99 per class
       const uint32_t* h = ghist + warp * kNB;
       uint32_t n = 0;  // requests per class per replica < 2^32
 #pragma unroll 1
-      for (int b = lane; b < kNB; b += 32) n += h[b];
+      for (int b = lane; b < kNB; b += 32) n += __ldcg(h + b);
 #pragma unroll
       for (int d = 16; d > 0; d >>= 1) n += __shfl_xor_sync(0xffffffffu, n, d);
       int64_t p50 = 0, p99 = 0;
@@ -1622,7 +1641,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
         int f50 = -1, f99 = -1;
 #pragma unroll 1
         for (int b0 = 0; b0 < kNB && f99 < 0; b0 += 32) {
-          uint32_t x = h[b0 + lane];
+          uint32_t x = __ldcg(h + b0 + lane);
 #pragma unroll
           for (int d = 1; d < 32; d <<= 1) {
             const uint32_t y = __shfl_up_sync(0xffffffffu, x, d);
@@ -1653,7 +1672,9 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
       }
 #pragma unroll 1
       for (int i = 0; i < 10; ++i) {
-        if (vrn > 1 && i >= 8)  // slot-evals and candidates: this CTA's range only (zeroed by the host)
+        // virtual ranks: slot-evals / candidates (this CTA's range) and the request counters (its
+        // accounting tasks) are partial sums (zeroed by the host); reconfigurations are replicated
+        if ((vsplit && i != 7) || (vrn > 1 && i >= 8))
           atomicAdd(reinterpret_cast<unsigned long long*>(&P.counters[(size_t)r * 10 + i]), cs.cnt[i]);
         else
           P.counters[(size_t)r * 10 + i] = (int64_t)cs.cnt[i];

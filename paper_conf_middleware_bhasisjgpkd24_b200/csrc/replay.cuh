@@ -137,6 +137,7 @@ struct ReplayParams {
   bool few;                // fewer replicas than SMs (the long-list kernel instances)
   int vr_lo[kMaxVR], vr_hi[kMaxVR], vr_cw[kMaxVR];
   const uint32_t* vr_pack[kMaxVR];
+  uint32_t* vr_done;       // [R] CTAs of the replica past finalize's histogram (zeroed by the host)
 };
 
 struct ScoreParams {
