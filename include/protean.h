@@ -316,6 +316,21 @@ int protean_replay_traces(protean_handle *h, const protean_replay_cfg *cfg,
 int protean_last_timings(const protean_handle *h, float *prepass_ms, float *replay_ms,
                          int32_t *launch);
 
+/* Device time (ms, CUDA events on the call's stream) of the candidate search the last
+ * protean_replay_traces ran ahead of its epoch chain: batch-aligned stream cursors (O3)
+ * and the O8 keys of every (replica, epoch, residue class, geometry) replayed from idle (Alg 1,
+ * P:L251-277; the "Oracle" scheme), used for the epochs whose dispatch is the closed form
+ * of Q18 (every sim-GPU available all epoch).  0 when the call scored every epoch inside
+ * the chain (mode G, virtual ranks, policy != 0, n_gpus > 32, or PROTEAN_PRECAND=0).  The search
+ * holds R*(E+1)*2M uint32 cursors and R*E*N*G int64 keys in handle scratch.  *walk_ms (may be
+ * NULL) = the cursor pass alone.  When the call ran the lean chain (a warp per replica on the
+ * search's id-ordered batch rows; many-replica mode R, policy 0, no container pools, N*G even, no
+ * epoch above 96 batches), protean_last_timings' replay_ms is the chain and *acct_ms (may be NULL)
+ * the per-request accounting pass after it (O7: histograms, SLO hits, P50/P99); else 0.
+ * EINVAL for a NULL handle or search_ms. */
+int protean_last_search_ms(const protean_handle *h, float *search_ms, float *walk_ms,
+                           float *acct_ms);
+
 /* ---------------------------------------------------------------------------------------------
  * 3c. End-to-end replay from HOST buffers: the computation of protean_replay_traces (mode R), with
  *     cfg->arrival_us, cfg->meta, cfg->replica_off and every output pointer of `out` being HOST

@@ -116,7 +116,7 @@ assert C.sizeof(BatchRec) == 32
 
 EXPORTS = ["protean_load_profiles", "protean_free", "protean_strerror", "protean_last_error",
            "protean_get_geometries", "protean_num_epochs", "protean_score_epoch", "protean_score_epoch_status",
-           "protean_replay_traces", "protean_replay_traces_host", "protean_replay_cfg_defaults", "protean_last_timings",
+           "protean_replay_traces", "protean_replay_traces_host", "protean_replay_cfg_defaults", "protean_last_timings", "protean_last_search_ms",
            "protean_sweep_depths", "protean_geometry_split", "protean_xchg_export", "protean_xchg_import", "protean_xchg_attach"]
 IPC_HANDLE_BYTES = 64
 
@@ -158,6 +158,8 @@ def load(path: str = None, require_cuda: bool = True):
     L.protean_replay_cfg_defaults.argtypes = [C.c_void_p]
     L.protean_replay_cfg_defaults.restype = None
     L.protean_last_timings.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
+    if hasattr(L, "protean_last_search_ms"):  # tolerant of older experiment builds
+        L.protean_last_search_ms.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
     L.protean_geometry_split.argtypes = [C.c_void_p, C.c_int32, C.c_void_p]
     L.protean_xchg_export.argtypes = [C.c_void_p, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_void_p]
     L.protean_xchg_import.argtypes = [C.c_void_p, C.c_void_p]

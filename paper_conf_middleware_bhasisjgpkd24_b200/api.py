@@ -127,6 +127,16 @@ class Handle:
         _check(self._h, self._lib.protean_last_timings(self._h, C.byref(a), C.byref(b), launch))
         return a.value, b.value, dict(zip(("grid", "block", "smem", "per_sm"), list(launch)))
 
+    def last_search_ms(self):
+        """(search_ms, walk_ms, acct_ms): device time of the candidate search (cand.cu) the last
+        replay ran ahead of its chain, of its cursor pass alone, and of the accounting pass after
+        the lean chain (chain.cu; 0 when the fused engine ran)."""
+        a, b, d = C.c_float(), C.c_float(), C.c_float()
+        if not hasattr(self._lib, "protean_last_search_ms"):
+            return 0.0, 0.0, 0.0
+        _check(self._h, self._lib.protean_last_search_ms(self._h, C.byref(a), C.byref(b), C.byref(d)))
+        return a.value, b.value, d.value
+
     # -------------------------------------------------------------------------------- replay
     def alloc_replay_out(self, R: int, E: int, N: int, *, decisions=True, cand_keys=False, log_cap=0):
         torch = _torch()

@@ -6,7 +6,7 @@ import subprocess
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-SOURCES = ["api.cu", "replay.cu", "partition.cu", "score.cu", "sweep.cu", "form.cu"]
+SOURCES = ["api.cu", "replay.cu", "partition.cu", "score.cu", "sweep.cu", "form.cu", "cand.cu", "chain.cu"]
 OUT = os.path.join(HERE, "libprotean.so")
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",
               "-Xcompiler", "-fPIC", "-shared", "-cudart", "static"]

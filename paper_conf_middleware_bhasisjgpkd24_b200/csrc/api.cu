@@ -43,7 +43,13 @@ struct protean_handle {
   int CW = 0;
   // [0,1] prepass + partition count, [4,5] partition scan + scatter, [2,3] replay kernel
   cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
-  float t_prepass = 0.f, t_replay = 0.f;
+  float t_prepass = 0.f, t_replay = 0.f, t_search = 0.f;
+  // the candidate search ahead of the chain (cand.cu): batch-aligned cursors, keys, lane order
+  void* d_cand = nullptr;
+  size_t cand_bytes = 0;
+  cudaEvent_t evc[4] = {nullptr, nullptr, nullptr, nullptr};
+  float t_walk = 0.f, t_acct = 0.f;
+  uint8_t* d_gorder = nullptr;
   int last_grid = 0, last_block = 0, last_smem = 0, last_per_sm = 0;
   std::vector<int> gn;  // slice count per geometry
   // mode G: candidate lane packing of the rank's geometry range
@@ -177,6 +183,15 @@ int ensure(protean_handle* h, void** p, size_t* have, size_t need, cudaStream_t 
   *p = nullptr;
   *have = 0;
   cudaError_t e = cudaMallocAsync(p, need, st);
+  if (e != cudaSuccess) {  // give the device pool's idle memory back and retry once
+    cudaGetLastError();
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, h->device) == cudaSuccess) {
+      cudaStreamSynchronize(st);
+      cudaMemPoolTrimTo(pool, 0);
+      e = cudaMallocAsync(p, need, st);
+    }
+  }
   if (e != cudaSuccess) {
     cudaGetLastError();
     *p = nullptr;
@@ -319,6 +334,8 @@ int xchg_finish(protean_handle* h) {
   CK(h, preload_kernels());
   CK(h, preload_sweep_kernel());
   CK(h, preload_form_kernel());
+  CK(h, preload_cand_kernels());
+  CK(h, preload_chain_kernels());
   CK(h, cudaMalloc(&h->d_xpeer, sizeof(char*) * h->xpeer.size()));
   CK(h, cudaMemcpy(h->d_xpeer, h->xpeer.data(), sizeof(char*) * h->xpeer.size(), cudaMemcpyHostToDevice));
   h->x_ready = true;
@@ -510,6 +527,14 @@ int protean_load_profiles(const protean_profiles* p, protean_handle** out) {
   if (e == cudaSuccess) e = cudaMalloc(&h->d_small, 512);
   if (e == cudaSuccess) e = cudaMemset(h->d_small, 0, 512);  // [256, 264): score_epoch's latched verdict
   for (int i = 0; i < 6 && e == cudaSuccess; ++i) e = cudaEventCreate(&h->ev[i]);
+  for (int i = 0; i < 4 && e == cudaSuccess; ++i) e = cudaEventCreate(&h->evc[i]);
+  if (e == cudaSuccess) {  // cand.cu lane order: geometries by slice count, descending
+    std::vector<uint8_t> go(h->G);
+    for (int j = 0; j < h->G; ++j) go[j] = (uint8_t)j;
+    std::stable_sort(go.begin(), go.end(), [&](uint8_t a, uint8_t b) { return h->gn[a] > h->gn[b]; });
+    e = cudaMalloc(&h->d_gorder, h->G);
+    if (e == cudaSuccess) e = cudaMemcpy(h->d_gorder, go.data(), h->G, cudaMemcpyHostToDevice);
+  }
   if (e == cudaSuccess) e = cudaMalloc(&h->d_pack, pack.size() * 4);
   if (e == cudaSuccess) e = cudaMemcpy(h->d_pack, pack.data(), pack.size() * 4, cudaMemcpyHostToDevice);
   if (e != cudaSuccess) {
@@ -531,6 +556,10 @@ void protean_free(protean_handle* h) {
     if (q) cudaFree(q);
   if (h->d_small) cudaFree(h->d_small);
   if (h->d_pack) cudaFree(h->d_pack);
+  if (h->d_gorder) cudaFree(h->d_gorder);
+  if (h->d_cand) cudaFree(h->d_cand);
+  for (cudaEvent_t v : h->evc)
+    if (v) cudaEventDestroy(v);
   if (h->d_pack_g) cudaFree(h->d_pack_g);
   if (h->d_sc_pack) cudaFree(h->d_sc_pack);
   for (uint32_t* q : h->vr_pack) cudaFree(q);
@@ -547,6 +576,14 @@ void protean_free(protean_handle* h) {
   }
   if (h->hs_copy) cudaStreamDestroy(h->hs_copy);
   if (h->hs_back) cudaStreamDestroy(h->hs_back);
+  {  // the stream-ordered allocations go back to the device pool: return it to the device
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, h->device) == cudaSuccess) {
+      cudaDeviceSynchronize();
+      cudaMemPoolTrimTo(pool, 0);
+    }
+    cudaGetLastError();
+  }
   delete h;
 }
 
@@ -635,6 +672,14 @@ int protean_last_timings(const protean_handle* h, float* prepass_ms, float* repl
     launch[2] = h->last_smem;
     launch[3] = h->last_per_sm;
   }
+  return PROTEAN_OK;
+}
+
+int protean_last_search_ms(const protean_handle* h, float* search_ms, float* walk_ms, float* acct_ms) {
+  if (!h || !search_ms) return PROTEAN_EINVAL;
+  *search_ms = h->t_search;
+  if (walk_ms) *walk_ms = h->t_walk;
+  if (acct_ms) *acct_ms = h->t_acct;
   return PROTEAN_OK;
 }
 
@@ -739,7 +784,11 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   // slot-balanced geometry range and exchanging min-loc keys per epoch in device memory (the
   // mode G exchange inside one launch); auto = min(16, G, SMs / R)
   int vr_n = 1;
-  if (!modeG && c.policy == 0 && h->G >= 2 && c.ctas_per_replica != 1) {
+  // PROTEAN_LEAN=2 (test knob): the lean chain whenever it can hold the call (no virtual ranks,
+  // no few-replica instance), so small parity cases exercise it
+  const char* lean_env = std::getenv("PROTEAN_LEAN");
+  const bool lean_force = lean_env && std::atoi(lean_env) == 2;
+  if (!modeG && c.policy == 0 && h->G >= 2 && c.ctas_per_replica != 1 && !lean_force) {
     vr_n = c.ctas_per_replica > 1 ? c.ctas_per_replica : (R < h->nsm ? h->nsm / R : 1);
     vr_n = std::min(vr_n, std::min(kMaxVR, h->G));
     if (vr_n < 2) vr_n = 1;
@@ -778,8 +827,14 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   if (const char* ev = std::getenv("PROTEAN_FEW"))  // experiment knob: force the instance family
     few_r = std::atoi(ev) != 0;
   const int block = 32 * (few_r ? PROTEAN_FEW_WARPS : kWarps);
+  // the candidate search as a data-parallel pass ahead of the chain (cand.cu): mode R, policy 0,
+  // one CTA per replica, the one-warp decision path (N <= 32)
+  bool precand = c.policy == 0 && !modeG && vr_n == 1 && N <= 32;
+  if (const char* ev = std::getenv("PROTEAN_PRECAND"))  // experiment knob: 0 = in-chain candidates only
+    if (std::atoi(ev) == 0) precand = false;
+  const int KS = precand ? N * h->G : 0;
   SmemLayout sl;
-  sl.init(h->tl.words, h->M, N, Gc, CW, 0, 0);
+  sl.init(h->tl.words, h->M, N, Gc, CW, 0, 0, KS);
   const size_t fixed = sl.total;
   int BS = std::min(WCAP, 64);
   size_t budget = 72 * 1024;
@@ -791,7 +846,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   int WS = (with_bats + (size_t)WCAP * 4 <= budget) ? WCAP : 0;  // window all in smem or all in HBM
   if (const char* ev = std::getenv("PROTEAN_WINDOW_SMEM"))  // experiment knob: 0 = window in global scratch
     if (std::atoi(ev) == 0) WS = 0;
-  sl.init(h->tl.words, h->M, N, Gc, CW, BS, WS);
+  sl.init(h->tl.words, h->M, N, Gc, CW, BS, WS, KS);
   if (sl.total > 227 * 1024) return fail(h, PROTEAN_ERANGE, "shared memory layout too large");
   int per_sm = 0;
   CK(h, replay_occupancy(block, sl.total, few_r, &per_sm));
@@ -926,6 +981,124 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   }
   P.scratch = static_cast<char*>(h->d_scratch);
   P.err = d_err;
+  h->t_search = 0.f;
+  h->t_acct = 0.f;
+  // the lean chain (chain.cu): a warp per replica on cand.cu's batch rows and keys, accounting in
+  // its own pass; many-replica calls without container pools (an epoch with more than 96 batches
+  // sends the call back to the fused engine below)
+  bool lean = precand && (!few_r || lean_force) && c.cold_start_us == 0 && (N * h->G) % 2 == 0;
+  if (lean_env && std::atoi(lean_env) == 0) lean = false;  // experiment knob: 0 = the fused engine
+  size_t b_ub = 0, b_br = 0;
+  if (precand) {
+    const size_t b_bs = al((size_t)R * S * (E + 1) * 4), b_kf = al((size_t)R * E * N * h->G * 8);
+    if (lean) {
+      b_ub = al((size_t)R * E * sizeof(UnitBats));
+      b_br = al((size_t)R * E * kUnitBats * 8);
+    }
+    int rc = ensure(h, &h->d_cand, &h->cand_bytes, b_bs + b_kf + b_ub + b_br, st);
+    if (rc == PROTEAN_ENOMEM && lean) {  // without the lean chain's rows: the search alone
+      lean = false;
+      b_ub = b_br = 0;
+      rc = ensure(h, &h->d_cand, &h->cand_bytes, b_bs + b_kf, st);
+    }
+    if (rc == PROTEAN_ENOMEM) {  // no room for the search either: the fused engine scores in-chain
+      precand = lean = false;
+      h->err.clear();
+    } else if (rc) {
+      return rc;
+    }
+  }
+  if (precand) {
+    const size_t b_bs = al((size_t)R * S * (E + 1) * 4), b_kf = al((size_t)R * E * N * h->G * 8);
+    CandParams Q;
+    std::memset(&Q, 0, sizeof(Q));
+    Q.tab = h->d_tab;
+    Q.tl = h->tl;
+    Q.sa = P.sa;
+    Q.saoff = P.saoff;
+    Q.sidx = P.sidx;
+    Q.bstart = static_cast<uint32_t*>(h->d_cand);
+    Q.kfc = reinterpret_cast<int64_t*>(static_cast<char*>(h->d_cand) + b_bs);
+    Q.gorder = h->d_gorder;
+    if (lean) {
+      Q.ub = reinterpret_cast<UnitBats*>(static_cast<char*>(h->d_cand) + b_bs + b_kf);
+      Q.overflow = d_err + 3;
+      P.ub = Q.ub;
+      P.bres = reinterpret_cast<int64_t*>(static_cast<char*>(h->d_cand) + b_bs + b_kf + b_ub);
+      P.ovf = d_err + 3;
+    }
+    Q.R = R;
+    Q.S = S;
+    Q.N = N;
+    Q.max_live = c.max_live;
+    Q.E = E;
+    Q.W = W;
+    size_t ws_off = 0;
+    cand_smem_bytes(h->tl, &ws_off);
+    Q.ws_off = ws_off;
+    int cper = 0;
+    CK(h, cand_occupancy(h->tl, &cper));
+    if (cper < 1) return fail(h, PROTEAN_ERANGE, "candidate kernel does not fit an SM");
+    CK(h, cudaEventRecord(h->evc[0], st));
+    CK(h, launch_walk(Q, st));
+    CK(h, cudaEventRecord(h->evc[2], st));
+    CK(h, launch_cand(Q, h->nsm * cper, st));
+    CK(h, cudaEventRecord(h->evc[1], st));
+    P.kfc = Q.kfc;
+  }
+  ReplayParams PL = P;
+  int cper = 0, cgrid_l = 0;
+  if (lean) {
+    PL.cl.init(N, N * h->G);
+    const size_t sl_a = al((size_t)N * kZA * c.max_live * 20), sl_c = al((size_t)kUnitBats * 32 * 16);
+    PL.o_alist = 0;
+    PL.o_clist = sl_a;
+    PL.slot_bytes = sl_a + sl_c;
+    CK(h, chain_occupancy(PL, &cper));
+    if (cper < 1) return fail(h, PROTEAN_ERANGE, "chain kernel does not fit an SM");
+    const int cgrid = (int)std::min<int64_t>((int64_t)h->nsm * cper, ((int64_t)R + 3) / 4);
+    cgrid_l = cgrid;
+    int rc = ensure(h, &h->d_scratch, &h->scratch_bytes,
+                    std::max(PL.slot_bytes * (size_t)cgrid * 4, P.slot_bytes * (size_t)grid), st);
+    if (rc == PROTEAN_ENOMEM) {  // the fused engine's scratch is smaller: replay there
+      h->err.clear();
+      rc = ensure(h, &h->d_scratch, &h->scratch_bytes, P.slot_bytes * (size_t)grid, st);
+      if (rc) return rc;
+      lean = false;
+    } else if (rc) {
+      return rc;
+    }
+    P.scratch = PL.scratch = static_cast<char*>(h->d_scratch);
+  }
+  if (lean) {
+    const int cgrid = cgrid_l;
+    CK(h, cudaEventRecord(h->ev[2], st));
+    CK(h, launch_chain(PL, cgrid, st));
+    CK(h, cudaEventRecord(h->ev[3], st));
+    CK(h, launch_acct(PL, st));
+    CK(h, cudaEventRecord(h->evc[3], st));
+    int herr3[4] = {0, 0, 0, 0};
+    CK(h, cudaMemcpyAsync(herr3, d_err, 16, cudaMemcpyDeviceToHost, st));
+    CK(h, cudaStreamSynchronize(st));
+    if (!herr3[3]) {  // every epoch fitted the chain's batch rows
+      float a = 0.f, b = 0.f;
+      CK(h, cudaEventElapsedTime(&a, h->ev[0], h->ev[1]));
+      CK(h, cudaEventElapsedTime(&b, h->ev[4], h->ev[5]));
+      h->t_prepass = a + b;
+      CK(h, cudaEventElapsedTime(&h->t_replay, h->ev[2], h->ev[3]));
+      CK(h, cudaEventElapsedTime(&h->t_acct, h->ev[3], h->evc[3]));
+      CK(h, cudaEventElapsedTime(&h->t_search, h->evc[0], h->evc[1]));
+      CK(h, cudaEventElapsedTime(&h->t_walk, h->evc[0], h->evc[2]));
+      h->last_grid = cgrid;
+      h->last_block = 32 * 4;
+      h->last_smem = (int)chain_smem_bytes(PL);
+      h->last_per_sm = cper;
+      if (herr3[0]) return fail(h, PROTEAN_EINVAL, "invalid request (unsorted, model id, or arrival >= trace_len)");
+      return PROTEAN_OK;
+    }
+    // some epoch held more than kUnitBats batches: the fused engine replays the call (its keys
+    // for the epochs cand.cu held are still valid)
+  }
   CK(h, cudaEventRecord(h->ev[2], st));
   CK(h, launch_replay(P, grid, block, st));
   CK(h, cudaEventRecord(h->ev[3], st));
@@ -946,6 +1119,10 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
     h->t_prepass = a + b;  // device time of the prepass and the three partition passes
   }
   CK(h, cudaEventElapsedTime(&h->t_replay, h->ev[2], h->ev[3]));
+  if (precand) {
+    CK(h, cudaEventElapsedTime(&h->t_search, h->evc[0], h->evc[1]));
+    CK(h, cudaEventElapsedTime(&h->t_walk, h->evc[0], h->evc[2]));
+  }
   h->last_grid = grid;
   h->last_block = block;
   h->last_smem = (int)sl.total;

@@ -1,0 +1,791 @@
+// chain.cu — the lean per-replica epoch chain and the per-request accounting pass (sm_100a).
+//
+// With the candidate search (cand.cu) taken out of the chain, what remains sequential per replica
+// is small: per epoch, the VM events and installs (O11, O5.3), the round-robin dispatch of the
+// epoch's id-ordered batches (Q18), the actual Alg 1 placement on the carried GPU state
+// (P:L251-277 under Eq 1 / Eq 2, P:L191 / P:L208), and the decision step (argmin over the
+// candidate keys, hysteresis and the ~30% cap).  One WARP carries one replica
+// (no CTA barriers; a few KB of shared memory per replica), so every replica of config 5 is
+// resident at once instead of three per SM:
+//
+//   chain_kernel  warp per replica.  Per epoch: A (lane = GPU), the epoch's batch rows (cand.cu,
+//                 prefetched one epoch ahead with cp.async), D (closed form when every GPU is
+//                 available, else the plain round robin on lane 0), E (the fused engine's
+//                 lane-per-slice placement units, four GPUs per pass), G (lane = GPU).  The
+//                 candidate keys come from cand.cu for closed-form epochs (rotated by the cursor);
+//                 other epochs are scored here, one lane per (GPU, geometry), Alg 1 from idle in
+//                 64-bit time.  Each batch's outcome goes to HBM for the accounting pass.
+//   acct_kernel   CTA per replica: per-request latencies end - arrival of every placed batch (O7),
+//                 log-linear histograms in shared memory, SLO hits, arrival / drop counters, then
+//                 the nearest-rank P50 / P99 (O12) -- the fused engine's phase F and finalize.
+//
+// Both produce exactly the fused engine's outputs (replay.cu); the host takes this path for mode R,
+// policy 0 or 1, no container pools, N <= 32 (api.cu).
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "replay.cuh"
+#include "place_group.cuh"
+#include "chain_state.cuh"
+
+namespace pemgpu {
+
+namespace {
+
+using namespace pg;
+constexpr int kChainWarps = 4;  // warps (replicas) per chain CTA
+#ifndef PROTEAN_CHAIN_MINB
+#define PROTEAN_CHAIN_MINB 7  // 7 x 4 warps per SM: all 4096 replicas of config 5 resident at once
+#endif
+constexpr int kAcctWarps = 8;  // warps per accounting CTA
+constexpr int kUB = kUnitBats;
+
+__device__ __forceinline__ void cp_async16(const void* dst_smem, const void* src) {
+  const uint32_t d = (uint32_t)__cvta_generic_to_shared(dst_smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+
+// Alg 1 from idle of GPU-epoch batches gl[0..cnt) on geometry j (O8), one lane, 64-bit times: the
+// plain definitions (live residents, BE memory for the tag walk, FIFO start, memory wait, Eq 1
+// co-runners) by scans over the batches placed so far.  Per-lane arrays in global scratch,
+// interleaved by lane.  For the epochs cand.cu did not hold (a GPU unavailable inside the epoch).
+__device__ int64_t score_idle(const Tab& T, int j, int cur, const UnitBats& U, const uint8_t* gl, int cnt,
+                              const uint32_t* sa_r, int max_live, int64_t* en, uint32_t* pk, int32_t* fb) {
+  constexpr int L = 32;  // lane stride of the per-lane arrays
+  const int ns = T.gn[j];
+  int64_t ls[kMaxSl];
+#pragma unroll
+  for (int s = 0; s < kMaxSl; ++s) ls[s] = 0;
+  int64_t misses = 0, tail = 0;
+#pragma unroll 1
+  for (int x = 0; x < cnt; ++x) {
+    const int b = gl[x];
+    const uint32_t info = U.info[b];
+    const int m = (info >> 16) & 0xFF, nreq = info & 0xFFFF;
+    const bool strict = (info >> 24) & 1;
+    const int64_t t = U.ready[b];
+    int live = 0;
+    int32_t be = 0;
+#pragma unroll 1
+    for (int i = 0; i < x; ++i) {
+      if (en[i * L] > t) {
+        ++live;
+        if (pk[i * L] >> 27) be += (int32_t)(pk[i * L] & kMemMask);
+      }
+    }
+    const int32_t q = T.mem[m];
+    uint64_t best = ~0ull;
+    int64_t bst = 0, bend = 0;
+    if (live < max_live) {
+#pragma unroll 1
+      for (int s = 0; s < ns; ++s) {
+        const int p = T.gprof[j * 8 + s];
+        const int32_t Ms = T.cap[p];
+        if (q > Ms) continue;
+        int64_t lss = 0;
+#pragma unroll
+        for (int z = 0; z < kMaxSl; ++z)
+          if (z == s) lss = ls[z];
+        const int64_t t0 = t > lss ? t : lss;
+        int32_t used = 0;
+        int64_t F = T.fbr[m * kNProf + p];
+#pragma unroll 1
+        for (int i = 0; i < x; ++i)
+          if ((int)((pk[i * L] >> 24) & 7) == s && en[i * L] > t0) {
+            used += (int32_t)(pk[i * L] & kMemMask);
+            F += fb[i * L];
+          }
+        int64_t start = t0;
+        if (used + q > Ms) {  // releases after t0 ascending; the first that fits (q <= Ms)
+          int64_t ev = t0;
+#pragma unroll 1
+          for (;;) {
+            int64_t nxt = INT64_MAX;
+            int32_t rem = 0;
+#pragma unroll 1
+            for (int i = 0; i < x; ++i)
+              if ((int)((pk[i * L] >> 24) & 7) == s && en[i * L] > ev && en[i * L] < nxt) nxt = en[i * L];
+            ev = nxt;
+#pragma unroll 1
+            for (int i = 0; i < x; ++i)
+              if ((int)((pk[i * L] >> 24) & 7) == s && en[i * L] > ev) rem += (int32_t)(pk[i * L] & kMemMask);
+            if (rem + q <= Ms) break;
+          }
+          start = ev;
+          F = T.fbr[m * kNProf + p];
+#pragma unroll 1
+          for (int i = 0; i < x; ++i)
+            if ((int)((pk[i * L] >> 24) & 7) == s && en[i * L] > start) F += fb[i * L];
+        }
+        const int64_t c = start + exec_time(T.solo[m * kNProf + p], F);
+        uint64_t key;
+        if (strict) {  // choose_strict_slice (Q11)
+          const uint64_t inelig = (be >= T.gpref[j * 8 + s]) ? (1ull << 62) : 0ull;
+          key = inelig | ((uint64_t)c << 6) | ((uint64_t)(4 - p) << 3) | (uint64_t)s;
+        } else {       // choose_best_effort_slice (Q12)
+          key = ((uint64_t)start << 3) | (uint64_t)s;
+        }
+        if (key < best) {
+          best = key;
+          bst = start;
+          bend = c;
+        }
+      }
+    }
+    const bool placed = best != ~0ull;
+    const int bsl = (int)(best & 7);
+    en[x * L] = placed ? bend : 0;
+    pk[x * L] = (uint32_t)q | ((uint32_t)bsl << 24) | (strict ? 0u : (1u << 27));
+    fb[x * L] = placed ? T.fbr[m * kNProf + T.gprof[j * 8 + bsl]] : 0;
+    if (placed) {
+#pragma unroll
+      for (int z = 0; z < kMaxSl; ++z)
+        if (z == bsl) ls[z] = bst;
+    }
+    const uint32_t* ma = sa_r + U.pos[b];
+    if (strict) {
+      if (!placed) {
+        misses += nreq;
+      } else {
+        const int64_t slo = T.slo[m];
+        if (bend - (int64_t)ma[0] > slo)
+          misses += (bend - (int64_t)ma[nreq - 1] > slo) ? nreq : nreq - hits_in(ma, nreq, bend, slo);
+      }
+    } else {
+      const int64_t tb = placed ? bend - (int64_t)ma[0] : (int64_t)0xFFFFFFFFLL;
+      tail = tb > tail ? tb : tail;
+    }
+  }
+  return make_key(misses, tail, j == cur ? 0 : j + 1);
+}
+
+__global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_kernel(ReplayParams P) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  if (*(volatile const int*)P.ovf) return;  // the host replays the call on the fused engine
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  int32_t* tabw = reinterpret_cast<int32_t*>(smem);
+#pragma unroll 1
+  for (int i = tid; i < P.tl.words; i += blockDim.x) tabw[i] = P.tab[i];
+  __syncthreads();
+  const ChainLayout& CL = P.cl;
+  unsigned char* wb = smem + (((size_t)P.tl.words * 4 + 15) & ~(size_t)15) + (size_t)warp * CL.total;
+  const int N = P.N, G = P.tl.G, KS = CL.KS;
+  const int64_t E = P.E, W = P.W;
+  Ctx c;
+  c.T.bind(tabw, P.tl);
+  c.N = N;
+  c.gu8 = wb + CL.gu8;
+  c.gi = reinterpret_cast<int64_t*>(wb + CL.gi);
+  c.g_cnt = reinterpret_cast<int*>(wb + CL.gcnt);
+  c.g_off = reinterpret_cast<int*>(wb + CL.goff);
+  c.a_n = reinterpret_cast<int*>(wb + CL.a_n);
+  c.a_ls = reinterpret_cast<int64_t*>(wb + CL.a_ls);
+  c.a_bu = reinterpret_cast<int64_t*>(wb + CL.a_bu);
+  const Tab& T = c.T;
+  UnitBats* ubs = reinterpret_cast<UnitBats*>(wb + CL.ub);
+  int64_t* kst = reinterpret_cast<int64_t*>(wb + CL.kst);
+  uint8_t* gl = wb + CL.gl;
+  uint8_t* gpu_of = wb + CL.gpu;
+  int sum_slots = 0;  // slot-evals per batch per decidable GPU (counter 8)
+#pragma unroll 1
+  for (int j = 0; j < G; ++j) sum_slots += T.gn[j];
+  const int n_aunits = (N + kAG - 1) / kAG;
+  const int gw = blockIdx.x * kChainWarps + warp;  // this warp's scratch slot
+  char* slot = P.scratch + (size_t)gw * P.slot_bytes;
+  const int NA = N * kZA;
+  LaneList AL;
+  AL.stride = NA;
+  AL.st = reinterpret_cast<int64_t*>(slot + P.o_alist);
+  AL.en = AL.st + (size_t)NA * P.max_live;
+  AL.mm = reinterpret_cast<uint32_t*>(AL.en + (size_t)NA * P.max_live);
+  int64_t* sc_en = reinterpret_cast<int64_t*>(slot + P.o_clist) + lane;  // score_idle arrays
+  uint32_t* sc_pk = reinterpret_cast<uint32_t*>(slot + P.o_clist + (size_t)kUB * 32 * 8) + lane;
+  int32_t* sc_fb = reinterpret_cast<int32_t*>(slot + P.o_clist + (size_t)kUB * 32 * 12) + lane;
+  constexpr int kUBChunks = (int)(sizeof(UnitBats) / 16);
+
+#pragma unroll 1
+  for (int r = gw; r < P.R; r += gridDim.x * kChainWarps) {
+    const uint64_t replica = (uint64_t)(P.base + r);
+    const UnitBats* ubr = P.ub + (size_t)r * E;
+    const int64_t* kfr = P.kfc ? P.kfc + (size_t)r * E * KS : nullptr;
+    int64_t* bres = P.bres + (size_t)r * E * kUB;
+    const uint32_t* sa_r = P.sa + P.saoff[r];
+    // ---- replica init (as replay.cu)
+#pragma unroll 1
+    for (int g = lane; g < N; g += 32) {
+      reset_gpu_state(c, g, P.init_geom);
+      c.gu8[3 * N + g] = c.gu8[4 * N + g] = (P.vm_policy == 0) ? VM_OD : VM_SPOT;
+      c.gi[0 * N + g] = c.gi[1 * N + g] = 0;
+      c.gi[2 * N + g] = 0;
+      c.gi[3 * N + g] = kForever;
+      c.gi[4 * N + g] = 0;
+      c.gi[8 * N + g] = c.gi[9 * N + g] = c.gi[10 * N + g] = c.gi[11 * N + g] = 0;
+      c.gi[12 * N + g] = c.gi[13 * N + g] = 0;
+    }
+    int cursor = 0;
+    int64_t nlog = 0;
+    unsigned long long n_recfg = 0, n_slot = 0, n_cand = 0;
+#pragma unroll 1
+    for (int i = lane; i < kUBChunks; i += 32)
+      cp_async16(reinterpret_cast<const char*>(&ubs[0]) + 16 * i, reinterpret_cast<const char*>(ubr) + 16 * i);
+    cp_async_commit();
+    cp_async_wait_all();
+    __syncwarp();
+
+#pragma unroll 1
+    for (int64_t e = 0; e < E; ++e) {
+      const int64_t eW = e * W, Tend = eW + W;
+      const UnitBats& U = ubs[e & 1];
+      // the candidate keys of this epoch and the batch rows of the next one, in flight during A-E
+      if (kfr) {
+#pragma unroll 1
+        for (int i = lane; i < KS / 2; i += 32) cp_async16(kst + 2 * i, kfr + (size_t)e * KS + 2 * i);
+      }
+      if (e + 1 < E) {
+#pragma unroll 1
+        for (int i = lane; i < kUBChunks; i += 32)
+          cp_async16(reinterpret_cast<const char*>(&ubs[(e + 1) & 1]) + 16 * i,
+                     reinterpret_cast<const char*>(ubr + e + 1) + 16 * i);
+      }
+      cp_async_commit();
+      // ---- A: VM events, installs, decidability (lane = simulated GPU)
+      bool whole = true;
+#pragma unroll 1
+      for (int g = lane; g < N; g += 32) {
+        if (P.vm_policy != 0) {
+#pragma unroll 1
+          for (int64_t k = (eW + P.rev - 1) / P.rev; k * P.rev < Tend; ++k) {
+            const int64_t tau = k * P.rev;
+            if (k < 1 || tau >= P.H) continue;
+            if (c.gu8[1 * N + g] != kNoGeom && c.gi[1 * N + g] <= tau) reset_gpu_state(c, g, c.gu8[1 * N + g]);
+            vm_event(P, c, replica, g, k, tau);
+          }
+        }
+        if (c.gu8[1 * N + g] != kNoGeom && c.gi[1 * N + g] <= Tend) reset_gpu_state(c, g, c.gu8[1 * N + g]);
+        c.gu8[5 * N + g] = (has_vm(c, g, Tend) && c.gi[1 * N + g] <= Tend) ? 1 : 0;
+        c.gu8[7 * N + g] = 0;
+        c.gu8[6 * N + g] = kNoGeom;
+        c.gi[7 * N + g] = -1;
+        whole &= c.gi[2 * N + g] <= eW && c.gi[3 * N + g] >= Tend &&
+                 !(c.gi[0 * N + g] < Tend && c.gi[1 * N + g] > eW);
+      }
+      const bool avail_all = __all_sync(0xffffffffu, whole);
+      __syncwarp();
+      const int nb = (int)U.nb;
+      const int cur0 = cursor;
+      // ---- D: dispatch (id order = row order)
+      if (avail_all) {  // closed form (Q18): rank b -> GPU (cursor + b) mod N, position b div N
+        const int dq = nb / N, drem = nb - dq * N;
+        auto goff = [&](int g) {
+          const int wrap = cursor + drem - N;
+          int x = g - cursor;
+          x = x < 0 ? 0 : (x > drem ? drem : x);
+          if (wrap > 0) x = min(max(g - cursor, 0), N - cursor) + min(g, wrap);
+          return g * dq + x;
+        };
+#pragma unroll 1
+        for (int b = lane; b < nb; b += 32) {
+          const int q = b / N, g = cursor + (b - q * N);
+          const int gg = g >= N ? g - N : g;
+          gpu_of[b] = (uint8_t)gg;
+          gl[goff(gg) + q] = (uint8_t)b;
+        }
+        for (int g = lane; g <= N; g += 32) c.g_off[g] = goff(g);
+        cursor = (int)((cursor + nb) % N);
+      } else {
+        if (lane == 0) {  // the plain round robin over the GPUs available at the batch's ready time
+          int cu = cursor;
+#pragma unroll 1
+          for (int g = 0; g < N; ++g) c.g_cnt[g] = 0;
+#pragma unroll 1
+          for (int b = 0; b < nb; ++b) {
+            int chosen = -1;
+#pragma unroll 1
+            for (int i = 0; i < N; ++i) {
+              const int g = (cu + i) % N;
+              if (available(c, g, U.ready[b])) { chosen = g; break; }
+            }
+            gpu_of[b] = chosen < 0 ? 0xFF : (uint8_t)chosen;
+            if (chosen >= 0) {
+              c.g_cnt[chosen]++;
+              cu = (chosen + 1) % N;
+            }
+          }
+          int off = 0;
+#pragma unroll 1
+          for (int g = 0; g < N; ++g) {
+            c.g_off[g] = off;
+            off += c.g_cnt[g];
+            c.g_cnt[g] = 0;
+          }
+          c.g_off[N] = off;
+#pragma unroll 1
+          for (int b = 0; b < nb; ++b) {
+            const int g = gpu_of[b];
+            if (g != 0xFF) gl[c.g_off[g] + c.g_cnt[g]++] = (uint8_t)b;
+          }
+          cursor = cu;
+        }
+        cursor = __shfl_sync(0xffffffffu, cursor, 0);
+        __syncwarp();
+#pragma unroll 1
+        for (int b = lane; b < nb; b += 32) {  // no GPU available: dropped (drop code 1)
+          if (gpu_of[b] != 0xFF) continue;
+          bres[(size_t)e * kUB + b] = -1;
+          if (P.log && nlog + b < P.log_cap) {
+            protean_batch_rec rec;
+            const uint32_t info = U.info[b];
+            rec.ready_us = U.ready[b];
+            rec.epoch = (uint32_t)e;
+            rec.n_req = (uint16_t)(info & 0xFFFF);
+            rec.model = (uint8_t)((info >> 16) & 0xFF);
+            rec.strict = (uint8_t)((info >> 24) & 1);
+            rec.gpu = 0xFF;
+            rec.slice = 0xFF;
+            rec.dropped = 1;
+            rec.pad = 0;
+            rec.start_us = rec.end_us = 0;
+            P.log[(size_t)r * P.log_cap + nlog + b] = rec;
+          }
+        }
+      }
+      __syncwarp();
+      // ---- E: actual placement, four GPUs per pass, lane per MIG slice (replay.cu phase E)
+#pragma unroll 1
+      for (int u = 0; u < n_aunits; ++u) {
+        const int g = u * kAG + (lane >> 3), s = lane & 7, gbase = lane & ~7;
+        const bool valid = (lane >> 3) < kAG && g < N;
+        const int j = valid ? c.gu8[0 * N + g] : 0;
+        const bool active = valid && s < T.gn[j];
+        const int p = active ? T.gprof[j * 8 + s] : 0;
+        SliceLane K;
+        K.fbr_p = T.fbr + p;
+        K.solo_p = T.solo + p;
+        K.Ms = T.cap[p];
+        K.pref = T.gpref[j * 8 + (s & 7)];
+        K.s = s;
+        K.p = p;
+        K.Z = kZA;
+        const int al = valid ? g * kZA + s : 0;
+        LaneList Lst = AL;
+        Lst.st += al;
+        Lst.en += al;
+        Lst.mm += al;
+        int n = valid ? c.a_n[al] : 0;
+        int64_t ls = valid ? c.a_ls[al] : 0;
+        int64_t bu = valid ? c.a_bu[al] : 0;
+        const int x0 = valid ? c.g_off[g] : 0, x1 = valid ? c.g_off[g + 1] : 0;
+        int len_max = x1 - x0;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+          const int o = __shfl_xor_sync(0xffffffffu, len_max, d);
+          len_max = o > len_max ? o : len_max;
+        }
+        int64_t acc0 = 0, acc1 = 0;  // busy, memory-time of the slice's winners
+#pragma unroll 1
+        for (int xi = 0; xi < len_max; ++xi) {
+          const bool has = xi < x1 - x0;
+          const int b = has ? gl[x0 + xi] : 0;
+          const uint32_t info = has ? U.info[b] : 0u;
+          const int m = (info >> 16) & 0xFF;
+          const bool strict = (info >> 24) & 1;
+          const int64_t t = has ? (int64_t)U.ready[b] : 0;
+          int64_t st, en;
+          const SliceOut so = place_group<1>(T, active && has, K, Lst, n, ls, t, m, strict, P.max_live, &st, &en);
+          const bool placed = !so.drop_overflow && so.kmin != ~0ull;
+          const int wl = (gbase + (int)(so.kmin & 7)) & 31;
+          if (!has) continue;
+          const bool rec_here = placed ? lane == wl : lane == gbase;
+          if (placed && lane == wl) {  // busy union + memory-time, clipped to [0, H)
+            const int64_t lo = st > bu ? st : bu;
+            const int64_t hi = en < P.H ? en : P.H;
+            if (hi > lo) acc0 += (int64_t)prof_compute(p) * (hi - lo);
+            if (hi > st) acc1 += (int64_t)T.mem[m] * (hi - st);
+            if (en > bu) bu = en;
+          }
+          if (rec_here) {
+            const int drop = placed ? 0 : (so.drop_overflow ? 3 : 2);
+            bres[(size_t)e * kUB + b] = placed ? en : -(int64_t)drop;
+            if (P.log && nlog + b < P.log_cap) {
+              protean_batch_rec rec;
+              rec.ready_us = U.ready[b];
+              rec.epoch = (uint32_t)e;
+              rec.n_req = (uint16_t)(info & 0xFFFF);
+              rec.model = (uint8_t)m;
+              rec.strict = strict ? 1 : 0;
+              rec.gpu = (uint8_t)g;
+              rec.slice = placed ? (uint8_t)s : 0xFF;
+              rec.dropped = (uint8_t)drop;
+              rec.pad = 0;
+              rec.start_us = placed ? st : 0;
+              rec.end_us = placed ? en : 0;
+              P.log[(size_t)r * P.log_cap + nlog + b] = rec;
+            }
+          }
+        }
+        int64_t mx = 0;
+        if (valid) {
+          c.a_n[al] = n;
+          c.a_ls[al] = ls;
+          c.a_bu[al] = bu;
+#pragma unroll 1
+          for (int i = 0; i < n; ++i) mx = Lst.E(i) > mx ? Lst.E(i) : mx;
+        }
+#pragma unroll
+        for (int d = 1; d < 8; d <<= 1) {
+          const int64_t o = __shfl_xor_sync(0xffffffffu, mx, d);
+          mx = o > mx ? o : mx;
+        }
+        const int64_t bsum = group_sum(acc0, 8), msum = group_sum(acc1, 8);
+        if (valid && s == 0) {
+          c.gi[5 * N + g] = mx;
+          c.gi[10 * N + g] += bsum;
+          c.gi[11 * N + g] += msum;
+        }
+        __syncwarp();
+      }
+      cp_async_wait_all();
+      __syncwarp();
+      // ---- candidate keys: cand.cu's (closed form) or scored here
+      const bool pre = P.policy == 0 && kfr && avail_all && kst[0] != INT64_MIN;
+      if (P.policy == 0 && !pre) {
+#pragma unroll 1
+        for (int pi = lane; pi < N * G; pi += 32) {
+          const int g = pi / G, j = pi - g * G;
+          int64_t key = -1;
+          if (c.gu8[5 * N + g])
+            key = score_idle(T, j, c.gu8[0 * N + g], U, gl + c.g_off[g], c.g_off[g + 1] - c.g_off[g], sa_r,
+                             P.max_live, sc_en, sc_pk, sc_fb);
+          kst[pi] = key;  // by GPU
+        }
+        __syncwarp();
+      }
+      // ---- G: decisions (O9, O10), lane = simulated GPU (replay.cu's one-warp path)
+      {
+        const int g = lane;
+        const bool gv = g < N;
+        bool want = false;
+        int64_t kb = kForever, kc = -1;
+        uint32_t scored_b = 0;
+        bool scored = false;
+        if (gv) {
+          uint8_t dec_out = kNoGeom;
+          if (P.policy != 1 && c.gu8[5 * N + g]) {
+            const int cur = c.gu8[0 * N + g];
+            int cl = g;  // keys by GPU (scored here) or by residue class (cand.cu)
+            if (pre) {
+              cl = g - cur0;
+              cl = cl < 0 ? cl + N : cl;
+            }
+            const int64_t* kr = kst + cl * G;
+#pragma unroll 1
+            for (int v = 0; v < G; ++v) {
+              int64_t kv = kr[v];
+              if (v == cur) {
+                if (pre) kv &= ~(int64_t)255;  // tag 0: the current geometry (O8, Q20)
+                kc = kv;
+              }
+              kb = kv < kb ? kv : kb;
+              if (P.cand_keys) P.cand_keys[(((size_t)r * E + e) * N + g) * (size_t)G + v] = kv;
+            }
+            c.gi[6 * N + g] = kb;
+            c.gi[7 * N + g] = kc;
+            const int tag = (int)(kb & 255);
+            const int best = tag == 0 ? cur : tag - 1;
+            scored_b = (uint32_t)(c.g_off[g + 1] - c.g_off[g]);
+            scored = true;
+            dec_out = (uint8_t)best;
+            c.gu8[6 * N + g] = (uint8_t)best;
+            if (best != cur) {  // Alg 2 lines 24-30 (Q22)
+              if (c.gu8[2 * N + g] >= P.wait_limit) want = true;
+              else c.gu8[2 * N + g]++;
+            } else {
+              c.gu8[2 * N + g] = 0;
+            }
+          } else if (P.policy == 0) {
+            c.gi[6 * N + g] = kForever;
+          }
+          if (P.decisions) P.decisions[((size_t)r * E + e) * N + g] = dec_out;
+          if (P.cand_keys && (P.policy != 0 || !c.gu8[5 * N + g])) {
+#pragma unroll 1
+            for (int j = 0; j < G; ++j) P.cand_keys[(((size_t)r * E + e) * N + g) * (size_t)G + j] = -1;
+          }
+        }
+        {  // counters 8, 9: slot-evals = scored GPUs' batches x the slots of the geometry set
+          const uint32_t tb = __reduce_add_sync(0xffffffffu, scored_b);
+          const int nsc = __popc(__ballot_sync(0xffffffffu, scored));
+          n_slot += (unsigned long long)tb * (unsigned long long)sum_slots;
+          n_cand += (unsigned long long)nsc * (unsigned long long)G;
+        }
+        if (P.policy != 1) {  // the ~30% cap: picks by (delta misses desc, GPU asc)
+          const unsigned alive = __ballot_sync(0xffffffffu, gv && has_vm(c, g, Tend));
+          const unsigned open = __ballot_sync(0xffffffffu, gv && c.gi[1 * N + g] > Tend);
+          int cap = P.cap_pct * __popc(alive) / 100;
+          if (cap < 1) cap = 1;
+          int free_slots = cap - __popc(open);
+          const int64_t d = (want && P.policy == 0) ? (kc >> 40) - (kb >> 40) : 0;
+#pragma unroll 1
+          while (free_slots > 0) {
+            const unsigned wm = __ballot_sync(0xffffffffu, want);
+            if (!wm) break;
+            int64_t best_d = want ? d : INT64_MIN;
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+              const int64_t od = __shfl_xor_sync(0xffffffffu, best_d, o);
+              best_d = od > best_d ? od : best_d;
+            }
+            const unsigned tie = __ballot_sync(0xffffffffu, want && d == best_d);
+            const int pick = __ffs(tie) - 1;
+            if (lane == pick) {
+              want = false;
+              const int64_t drain_end = c.gi[5 * N + g] > Tend ? c.gi[5 * N + g] : Tend;
+              c.gi[0 * N + g] = Tend;
+              c.gi[1 * N + g] = drain_end + P.reconfig_us;
+              c.gu8[1 * N + g] = c.gu8[6 * N + g];
+              ++n_recfg;
+            }
+            --free_slots;
+          }
+        }
+      }
+      nlog += nb;
+      __syncwarp();
+    }
+    // ---- finalize (O12): VM bills to H, cost, utilisation, counters 7-9 (0-6: acct_kernel)
+#pragma unroll 1
+    for (int g = lane; g < N; g += 32) bill_switch(c, g, VM_NONE, P.H, P.H);
+    __syncwarp();
+    n_recfg = __reduce_add_sync(0xffffffffu, (unsigned)n_recfg);
+    if (lane == 0) {
+      int64_t od = 0, spot = 0, busy = 0, memt = 0;
+#pragma unroll 1
+      for (int g = 0; g < N; ++g) {
+        od += c.gi[8 * N + g];
+        spot += c.gi[9 * N + g];
+        busy += c.gi[10 * N + g];
+        memt += c.gi[11 * N + g];
+      }
+      P.counters[(size_t)r * 10 + 7] = (int64_t)n_recfg;
+      P.counters[(size_t)r * 10 + 8] = (int64_t)n_slot;
+      P.counters[(size_t)r * 10 + 9] = (int64_t)n_cand;
+      P.accum[(size_t)r * 4 + 0] = busy;
+      P.accum[(size_t)r * 4 + 1] = memt;
+      P.accum[(size_t)r * 4 + 2] = od;
+      P.accum[(size_t)r * 4 + 3] = spot;
+      P.cost[r] = __ddiv_rn(__dadd_rn(__dmul_rn((double)od, P.price_od),
+                                      __dmul_rn((double)spot, P.price_spot)), 3.6e9);
+      const double dN = (double)N, dH = (double)P.H;
+      P.util[2 * (size_t)r] = __ddiv_rn((double)busy, __dmul_rn(__dmul_rn(7.0, dN), dH));
+      P.util[2 * (size_t)r + 1] = __ddiv_rn((double)memt, __dmul_rn(__dmul_rn((double)T.cap[4], dN), dH));
+      if (P.n_batches) P.n_batches[r] = nlog;
+      if (P.cold_starts) P.cold_starts[r] = 0;
+    }
+    __syncwarp();
+  }
+}
+
+// ---------------------------------------------------------------- accounting (O7, O12)
+__global__ void __launch_bounds__(32 * kAcctWarps) acct_kernel(ReplayParams P) {
+  if (*(volatile const int*)P.ovf) return;
+  __shared__ uint32_t s_hist[2 * kNB];
+  __shared__ uint32_t s_sink;
+  __shared__ unsigned long long s_cnt[kAcctWarps][5];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t sink = (uint32_t)__cvta_generic_to_shared(&s_sink);
+  const int64_t E = P.E;
+  const int32_t* tabw = P.tab;
+  const int32_t* slo_t = tabw + P.tl.o_slo;
+#pragma unroll 1
+  for (int r = blockIdx.x; r < P.R; r += gridDim.x) {
+#pragma unroll 1
+    for (int i = tid; i < 2 * kNB; i += blockDim.x) s_hist[i] = 0;
+    __syncthreads();
+    const UnitBats* ubr = P.ub + (size_t)r * E;
+    const int64_t* bres = P.bres + (size_t)r * E * kUB;
+    const uint32_t* sa_r = P.sa + P.saoff[r];
+    unsigned long long c_sarr = 0, c_met = 0, c_sdrop = 0, c_barr = 0, c_bdrop = 0;  // warp-uniform
+#pragma unroll 1
+    for (int64_t e = warp; e < E; e += kAcctWarps) {  // warp per epoch
+      const UnitBats& U = ubr[e];
+      const int nb = (int)U.nb;
+      // the epoch's rows and outcomes, one batch per lane, then the members batch by batch
+#pragma unroll 1
+      for (int b0 = 0; b0 < nb; b0 += 32) {
+        const int bl = b0 + lane;
+        uint32_t info_l = 0, pos_l = 0;
+        int64_t end_l = 0;
+        if (bl < nb) {
+          info_l = U.info[bl];
+          pos_l = U.pos[bl];
+          end_l = bres[(size_t)e * kUB + bl];
+        }
+        const int nbl = min(32, nb - b0);
+        // batch by batch, the next batch's first 128 members in flight while this one is counted
+        uint32_t nxt[4];
+        auto load128 = [&](int k, uint32_t* a) {
+          const uint32_t pos = __shfl_sync(0xffffffffu, pos_l, k);
+          const int nreq = (int)(__shfl_sync(0xffffffffu, info_l, k) & 0xFFFF);
+          const uint32_t* ma = sa_r + pos;
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            const int i = q * 32 + lane;
+            a[q] = i < nreq ? __ldcs(ma + i) : 0u;
+          }
+        };
+        if (nbl > 0) load128(0, nxt);
+#pragma unroll 1
+        for (int k = 0; k < nbl; ++k) {
+          uint32_t cur[4];
+#pragma unroll
+          for (int q = 0; q < 4; ++q) cur[q] = nxt[q];
+          if (k + 1 < nbl) load128(k + 1, nxt);
+          const uint32_t info = __shfl_sync(0xffffffffu, info_l, k);
+          const uint32_t pos = __shfl_sync(0xffffffffu, pos_l, k);
+          const int64_t bend = __shfl_sync(0xffffffffu, end_l, k);
+          const int nreq = info & 0xFFFF, m = (info >> 16) & 0xFF;
+          const bool strict = (info >> 24) & 1;
+          uint32_t met = 0;
+          const bool drop = bend < 0;
+          if (!drop) {
+            const int64_t slo = slo_t[m];
+            const uint32_t* ma = sa_r + pos;
+            const uint32_t hb = (uint32_t)__cvta_generic_to_shared(s_hist + (strict ? 0 : kNB));
+            if (bend - (int64_t)__shfl_sync(0xffffffffu, cur[0], 0) <= (int64_t)0xFFFFFFFFLL) {
+              // latencies fit 32 bits: bucket = 128 s + (lat >> s), s = max(0, floor(log2 lat) - 7)
+              const uint32_t e32 = (uint32_t)bend;
+              const uint32_t slo32 = slo > (int64_t)0xFFFFFFFFLL ? 0xFFFFFFFFu : (uint32_t)slo;
+#pragma unroll
+              for (int q = 0; q < 4; ++q) {
+                const int i = q * 32 + lane;
+                const bool valid = i < nreq;
+                const uint32_t lat = e32 - cur[q];
+                const int sh = max(24 - __clz(lat), 0);
+                inc_shared(valid ? hb + 4u * (uint32_t)((sh << 7) + (int)(lat >> sh)) : sink);
+                met += __popc(__ballot_sync(0xffffffffu, valid && lat <= slo32));
+              }
+#pragma unroll 1
+              for (int i0 = 128; i0 < nreq; i0 += 32) {  // batches above 128 requests
+                const int i = i0 + lane;
+                const bool valid = i < nreq;
+                const uint32_t lat = e32 - ma[valid ? i : 0];
+                const int sh = max(24 - __clz(lat), 0);
+                inc_shared(valid ? hb + 4u * (uint32_t)((sh << 7) + (int)(lat >> sh)) : sink);
+                met += __popc(__ballot_sync(0xffffffffu, valid && lat <= slo32));
+              }
+            } else {  // some latency >= 2^32 us: the saturating 64-bit bucket
+#pragma unroll 1
+              for (int i0 = 0; i0 < nreq; i0 += 32) {
+                const int i = i0 + lane;
+                const bool valid = i < nreq;
+                const int64_t lat = bend - (int64_t)ma[valid ? i : 0];
+                inc_shared(valid ? hb + 4u * (uint32_t)lat_bucket(lat) : sink);
+                met += __popc(__ballot_sync(0xffffffffu, valid && lat <= slo));
+              }
+            }
+          }
+          if (strict) {
+            c_sarr += nreq;
+            if (drop) c_sdrop += nreq; else c_met += met;
+          } else {
+            c_barr += nreq;
+            if (drop) c_bdrop += nreq;
+          }
+        }
+      }
+    }
+    if (lane == 0) {
+      s_cnt[warp][0] = c_sarr;
+      s_cnt[warp][1] = c_met;
+      s_cnt[warp][2] = c_sdrop;
+      s_cnt[warp][3] = c_barr;
+      s_cnt[warp][4] = c_bdrop;
+    }
+    __syncthreads();
+    uint32_t* ghist = P.hist + (size_t)r * 2 * kNB;
+#pragma unroll 1
+    for (int w = tid; w < 2 * kNB; w += blockDim.x) ghist[w] = s_hist[w];
+    if (tid == 0) {  // counters 0-6 (fold_wcnt's formulas)
+      unsigned long long v[5] = {0, 0, 0, 0, 0};
+#pragma unroll 1
+      for (int w = 0; w < kAcctWarps; ++w)
+        for (int i = 0; i < 5; ++i) v[i] += s_cnt[w][i];
+      int64_t* cn = P.counters + (size_t)r * 10;
+      cn[0] = (int64_t)v[0];
+      cn[1] = (int64_t)v[1];
+      cn[2] = (int64_t)(v[0] - v[1] - v[2]);
+      cn[3] = (int64_t)v[2];
+      cn[4] = (int64_t)v[3];
+      cn[5] = (int64_t)(v[3] - v[4]);
+      cn[6] = (int64_t)v[4];
+    }
+    if (warp < 2) {  // nearest-rank P50 / P99 per class (O12), from the shared histogram
+      const uint32_t* h = s_hist + warp * kNB;
+      uint32_t n = 0;
+#pragma unroll 1
+      for (int b = lane; b < kNB; b += 32) n += h[b];
+#pragma unroll
+      for (int d = 16; d > 0; d >>= 1) n += __shfl_xor_sync(0xffffffffu, n, d);
+      int64_t p50 = 0, p99 = 0;
+      if (n) {
+        const uint64_t r50 = (50 * (uint64_t)n + 99) / 100, r99 = (99 * (uint64_t)n + 99) / 100;
+        uint64_t cum = 0;
+        int f50 = -1, f99 = -1;
+#pragma unroll 1
+        for (int b0 = 0; b0 < kNB && f99 < 0; b0 += 32) {
+          uint32_t x = h[b0 + lane];
+#pragma unroll
+          for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, d);
+            if (lane >= d) x += y;
+          }
+          const unsigned m50 = __ballot_sync(0xffffffffu, cum + x >= r50);
+          const unsigned m99 = __ballot_sync(0xffffffffu, cum + x >= r99);
+          if (f50 < 0 && m50) f50 = b0 + __ffs(m50) - 1;
+          if (f99 < 0 && m99) f99 = b0 + __ffs(m99) - 1;
+          cum += __shfl_sync(0xffffffffu, x, 31);
+        }
+        p50 = (int64_t)bucket_lower_edge(f50);
+        p99 = (int64_t)bucket_lower_edge(f99);
+      }
+      if (lane == 0) {
+        P.pct[(size_t)r * 4 + warp * 2] = p50;
+        P.pct[(size_t)r * 4 + warp * 2 + 1] = p99;
+      }
+    }
+    __syncthreads();
+  }
+}
+
+}  // namespace
+
+size_t chain_smem_bytes(const ReplayParams& P) {
+  return (((size_t)P.tl.words * 4 + 15) & ~(size_t)15) + P.cl.total * kChainWarps;
+}
+
+cudaError_t chain_occupancy(const ReplayParams& P, int* per_sm) {
+  const size_t smem = chain_smem_bytes(P);
+  cudaError_t e = cudaFuncSetAttribute(chain_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, chain_kernel, 32 * kChainWarps, smem);
+}
+
+cudaError_t launch_chain(const ReplayParams& P, int grid, cudaStream_t st) {
+  chain_kernel<<<grid, 32 * kChainWarps, chain_smem_bytes(P), st>>>(P);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_acct(const ReplayParams& P, cudaStream_t st) {
+  acct_kernel<<<P.R, 32 * kAcctWarps, 0, st>>>(P);
+  return cudaGetLastError();
+}
+
+cudaError_t preload_chain_kernels() {
+  cudaFuncAttributes a;
+  cudaError_t e = cudaFuncGetAttributes(&a, chain_kernel);
+  if (e != cudaSuccess) return e;
+  return cudaFuncGetAttributes(&a, acct_kernel);
+}
+
+}  // namespace pemgpu

@@ -21,6 +21,7 @@
 
 #include "replay.cuh"
 #include "place_group.cuh"
+#include "chain_state.cuh"
 #ifndef PROTEAN_D_BARRIER
 #define PROTEAN_D_BARRIER 1
 #endif
@@ -66,25 +67,6 @@ namespace {
 using namespace pg;
 constexpr int kMaxWarps = 32;
 
-struct Ctx {
-  Tab T;
-  const uint32_t* pack;
-  int N;
-  uint8_t* gu8;   // [8][N]: geom, target, ctr, vm, bill, dec, best, want
-  int64_t* gi;    // [12][N]: rs, re, from, until, since, maxend, kbest, kcur, od, spot, busy, mem
-  int *g_cnt, *g_off;
-  int* a_n;
-  int64_t *a_ls, *a_bu;
-  int64_t* keys;
-  Bat *sb, *gb;
-  uint32_t *sord, *gord, *sgl, *ggl, *sarr;
-  int BS;
-  // per-epoch generic views (shared or global memory)
-  Bat* bats;
-  uint32_t *ord, *gl;
-  __device__ __forceinline__ Bat& bat_w(int i) const { return i < BS ? sb[i] : gb[i]; }
-};
-
 struct CtaState {
   int64_t nlog;
   int nb, cursor, all_avail, bad;
@@ -97,8 +79,6 @@ struct CtaState {
   unsigned long long cold;  // N3 cold starts of the replica          // window entries copied this epoch (incl. alignment padding)
   unsigned long long cnt[10];
 };
-
-enum { VM_NONE = 0, VM_OD = 1, VM_SPOT = 2 };
 
 // ------------------------------------------------------------------ mode G exchange (S8, §8(e))
 __device__ __forceinline__ uint64_t global_ns() {
@@ -157,80 +137,6 @@ static __device__ __noinline__ void exchange_keys(XLayout X, char* const* xpeer,
     gi[7 * N + g] = kc;
   }
   __syncthreads();
-}
-
-__device__ __forceinline__ int64_t clip_h(int64_t x, int64_t H) { return x < H ? x : H; }
-
-__device__ void bill_switch(const Ctx& c, int g, int type, int64_t at, int64_t H) {
-  const int64_t d = clip_h(at, H) - clip_h(c.gi[4 * c.N + g], H);
-  if (c.gu8[4 * c.N + g] == VM_OD) c.gi[8 * c.N + g] += d;
-  if (c.gu8[4 * c.N + g] == VM_SPOT) c.gi[9 * c.N + g] += d;
-  c.gu8[4 * c.N + g] = (uint8_t)type;
-  c.gi[4 * c.N + g] = at;
-}
-
-__device__ void reset_gpu_state(const Ctx& c, int g, int geom) {
-  c.gu8[0 * c.N + g] = (uint8_t)geom;
-  c.gu8[1 * c.N + g] = kNoGeom;
-  c.gu8[2 * c.N + g] = 0;
-#pragma unroll 1
-  for (int s = 0; s < kZA; ++s) {
-    c.a_n[g * kZA + s] = 0;
-    c.a_ls[g * kZA + s] = 0;
-    c.a_bu[g * kZA + s] = 0;
-  }
-}
-
-__device__ __forceinline__ bool has_vm(const Ctx& c, int g, int64_t t) {
-  return c.gi[2 * c.N + g] <= t && t < c.gi[3 * c.N + g];
-}
-__device__ __forceinline__ bool available(const Ctx& c, int g, int64_t t) {
-  return has_vm(c, g, t) && !(c.gi[0 * c.N + g] <= t && t < c.gi[1 * c.N + g]);
-}
-
-// O11: one revocation boundary tau = k * T_rev for node g (draws specified in DESIGN.md §3).
-// Returns true when the node changes VM under Spot Only (its containers go with it, reading R27).
-__device__ __forceinline__ bool vm_event(const ReplayParams& P, const Ctx& c, uint64_t replica, int g,
-                                      int64_t k, int64_t tau) {
-  const uint64_t x = (replica << 32) ^ ((uint64_t)g << 20) ^ ((uint64_t)k << 2);
-  const uint64_t d0 = smix(P.seed ^ smix(x ^ 0ull)) >> 11;
-  const uint64_t d1 = smix(P.seed ^ smix(x ^ 1ull)) >> 11;
-  const bool revoked = d0 < P.thr, spot_ok = d1 >= P.thr;
-  if (P.vm_policy == 1) {  // PROTEAN: retry spot, else on-demand; seamless redirect
-    if (c.gu8[3 * c.N + g] == VM_SPOT) {
-      if (revoked && !spot_ok) {
-        c.gu8[3 * c.N + g] = VM_OD;
-        bill_switch(c, g, VM_OD, tau + P.notice, P.H);
-      }
-    } else if (c.gu8[3 * c.N + g] == VM_OD) {
-      if (spot_ok) {
-        c.gu8[3 * c.N + g] = VM_SPOT;
-        bill_switch(c, g, VM_SPOT, tau, P.H);
-      }
-    }
-  } else if (P.vm_policy == 2) {  // Spot Only
-    if (c.gu8[3 * c.N + g] == VM_SPOT) {
-      if (revoked && !spot_ok) {
-        c.gu8[3 * c.N + g] = VM_NONE;
-        c.gi[3 * c.N + g] = tau;
-        bill_switch(c, g, VM_NONE, tau + P.notice, P.H);
-        c.gu8[1 * c.N + g] = kNoGeom;
-        c.gi[0 * c.N + g] = c.gi[1 * c.N + g] = 0;
-        return true;
-      }
-    } else if (c.gu8[3 * c.N + g] == VM_NONE) {
-      if (spot_ok) {
-        c.gu8[3 * c.N + g] = VM_SPOT;
-        c.gi[2 * c.N + g] = tau;
-        c.gi[3 * c.N + g] = kForever;
-        bill_switch(c, g, VM_SPOT, tau, P.H);
-        reset_gpu_state(c, g, P.init_geom);
-        c.gi[0 * c.N + g] = c.gi[1 * c.N + g] = 0;
-        return true;
-      }
-    }
-  }
-  return false;
 }
 
 // ---- N3: the Autoscaler's container pools (readings R22-R27).  Per CTA slot
@@ -696,7 +602,15 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
     // B of epoch e + 1 runs while warp 0 decides epoch e (G): it reads only s_cur (final after
     // epoch e's formation) and overwrites the window, which no phase after E reads.
     const uint32_t* sa_r = P.sa + P.saoff[r];
+    int64_t* kst = reinterpret_cast<int64_t*>(smem + SL.kst);  // [2][N*G] precomputed keys (cand.cu)
     auto phase_b = [&](int64_t ee) {
+      if (P.kfc) {  // the epoch's candidate keys by residue class; G of epoch ee - 1 reads the other half
+        const int KS = SL.KS;
+        const int64_t* src = P.kfc + ((size_t)r * P.E + ee) * KS;
+        int64_t* dst = kst + (ee & 1) * KS;
+#pragma unroll 1
+        for (int i = lane; i < KS; i += 32) dst[i] = __ldg(src + i);
+      }
       {
         const uint32_t* s1 = P.sidx + ((size_t)r * (P.E + 1) + ee + 1) * S;
         int carry = 0, nact = 0;
@@ -1100,7 +1014,9 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
       // One loop body serves both kinds (a single inlined copy of Place).
       // dynamic task queue: [actual units][candidate units][accounting of batch rank rk];
       // accounting waits (rarely) for the actual units, whose warps publish via cs.adone
-      const int n_units = n_aunits + (P.policy == 0 ? N * cs.cw : 0);
+      // closed-form dispatch + keys held by cand.cu: the candidate units are done (G reads kst)
+      const bool pre = P.kfc && avail_all && kst[(e & 1) * SL.KS] != INT64_MIN;
+      const int n_units = n_aunits + (P.policy == 0 && !pre ? N * cs.cw : 0);
       // split accounting (vsplit): CTA vr takes tasks vr, vr + vrn, ... (counters and the histogram
       // are summed in finalize); otherwise every CTA takes them all
       const int ntk = (nb + kAK - 1) / kAK;
@@ -1424,7 +1340,27 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
             if (P.policy != 1 && c.gu8[5 * c.N + g]) {
               const int cur = c.gu8[0 * c.N + g];
               int best;
-              if (P.policy == 0) {  // S8: argmin over the candidate keys
+              if (P.policy == 0 && pre) {  // S8 over the keys of g's residue class (cand.cu)
+                int cl = g - cursor;
+                cl = cl < 0 ? cl + N : cl;
+                const int64_t* kr = kst + (e & 1) * SL.KS + cl * T.G;
+#pragma unroll 1
+                for (int v = 0; v < T.G; ++v) {
+                  int64_t kv = kr[v];
+                  if (v == cur) {
+                    kv &= ~(int64_t)255;  // tag 0: the current geometry (O8, Q20)
+                    kc = kv;
+                  }
+                  kb = kv < kb ? kv : kb;
+                  if (P.cand_keys) P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + v] = kv;
+                }
+                c.gi[6 * c.N + g] = kb;
+                c.gi[7 * c.N + g] = kc;
+                const int tag = (int)(kb & 255);
+                best = tag == 0 ? cur : tag - 1;
+                scored_b = (uint32_t)(c.g_off[g + 1] - c.g_off[g]);
+                scored = true;
+              } else if (P.policy == 0) {  // S8: argmin over the candidate keys
 #pragma unroll 1
                 for (int v = 0; v < cs.ghi - cs.glo; ++v) kb = c.keys[g * Gc + v] < kb ? c.keys[g * Gc + v] : kb;
                 c.gi[6 * c.N + g] = kb;
@@ -1449,7 +1385,7 @@ __global__ void __launch_bounds__(kPL == 4 ? 32 * PROTEAN_FEW_WARPS : 32 * PROTE
               c.gi[6 * c.N + g] = kForever;
             }
             if (P.decisions) P.decisions[((size_t)r * P.E + e) * N + g] = dec_out;
-            if (P.policy != 0 && P.cand_keys) {
+            if ((P.policy != 0 || (pre && !c.gu8[5 * c.N + g])) && P.cand_keys) {  // nothing scored
 #pragma unroll 1
               for (int j = cs.glo; j < cs.ghi; ++j)
                 P.cand_keys[(((size_t)r * P.E + e) * N + g) * (size_t)T.G + j] = -1;

@@ -39,6 +39,14 @@ struct Bat {
   int64_t start, end;
 };
 
+constexpr int kUnitBats = 64;  // batches held per (replica, epoch) unit (config 5: ~38 per epoch)
+struct UnitBats {              // 784 B, 16-byte aligned: one cp.async run
+  uint32_t nb, pad[3];         // batch count (> kUnitBats: not held, the call takes the fused path)
+  uint32_t ready[kUnitBats];
+  uint32_t info[kUnitBats];    // n | model << 16 | strict << 24
+  uint32_t pos[kUnitBats];     // first member in the replica's stream-sorted copy
+};
+
 // Candidate lane packing (host-built, P.pack): per candidate warp w of a GPU and lane l, the
 // geometry (0xFF idle), the slice position, the group size Z (power of two >= slice count) and the
 // lane of the group's slice 0, packed as j | s << 8 | Z << 16 | base << 24.
@@ -49,9 +57,10 @@ struct SmemLayout {
   int N, Gc, CW;    // simulated GPUs, candidate geometries in range, candidate warps per GPU
   int BS, WS;       // batches / window entries held in smem
   size_t tab, pack;
-  size_t g_u8, g_i64, g_i32, a_n, a_ls, a_bu, keys, bats, ord, glist, sarr, total;
-  __host__ void init(int words, int M, int n_gpus, int gc, int cw, int bs, int ws) {
-    S = 2 * M; N = n_gpus; Gc = gc; CW = cw; BS = bs; WS = ws;
+  int KS;           // precomputed candidate keys staged per epoch (cand.cu): N * G, 0 = off
+  size_t g_u8, g_i64, g_i32, a_n, a_ls, a_bu, keys, kst, bats, ord, glist, sarr, total;
+  __host__ void init(int words, int M, int n_gpus, int gc, int cw, int bs, int ws, int ks = 0) {
+    S = 2 * M; N = n_gpus; Gc = gc; CW = cw; BS = bs; WS = ws; KS = ks;
     size_t o = 0;
     auto take = [&](size_t bytes) { size_t r = o; o += (bytes + 15) & ~(size_t)15; return r; };
     tab = take((size_t)words * 4);
@@ -64,6 +73,7 @@ struct SmemLayout {
     a_ls = take((size_t)N * kZA * 8);
     a_bu = take((size_t)N * kZA * 8);
     keys = take((size_t)N * Gc * 8);
+    kst = take((size_t)2 * KS * 8);             // [epoch parity][class][geometry]
     bats = take((size_t)BS * sizeof(Bat));
     ord = take((size_t)BS * 4);
     glist = take((size_t)BS * 4);
@@ -85,6 +95,29 @@ struct XLayout {
   __host__ __device__ size_t bytes() const { return flag_off(n, 0); }
 };
 
+// Per-warp shared-memory layout of the lean chain (chain.cu), byte offsets from the warp's base.
+struct ChainLayout {
+  int N, KS;
+  size_t gu8, gi, gcnt, goff, a_n, a_ls, a_bu, kst, ub, gl, gpu, total;
+  __host__ void init(int n, int ks) {
+    N = n; KS = ks;
+    size_t o = 0;
+    auto take = [&](size_t bytes) { size_t r = o; o += (bytes + 15) & ~(size_t)15; return r; };
+    ub = take(2 * sizeof(UnitBats));             // this epoch's rows and the next one's (cp.async)
+    kst = take((size_t)KS * 8);                  // keys: by residue class (cand.cu) or by GPU
+    gu8 = take((size_t)N * 8);
+    gi = take((size_t)N * 14 * 8);
+    gcnt = take((size_t)N * 4);
+    goff = take((size_t)(N + 1) * 4);
+    a_n = take((size_t)N * kZA * 4);
+    a_ls = take((size_t)N * kZA * 8);
+    a_bu = take((size_t)N * kZA * 8);
+    gl = take(kUnitBats);
+    gpu = take(kUnitBats);
+    total = o;
+  }
+};
+
 struct ReplayParams {
   // tables
   const int32_t* tab;
@@ -95,6 +128,13 @@ struct ReplayParams {
   const uint32_t* sa;      // arrivals, per replica stream-major, replica r at sa + saoff[r]
   const int64_t* saoff;    // [R+1] 16-byte aligned replica offsets into sa
   const uint32_t* sidx;    // [R][E+1][S] first request of stream k with arrival >= e*W (replica-relative)
+  const int64_t* kfc;      // [R][E][N][G] candidate keys by residue class (cand.cu), or NULL
+  // lean chain (chain.cu): the epochs' id-ordered batch rows (cand.cu) and each batch's outcome
+  // for the accounting pass: end (us) if placed, else -drop (1 no GPU, 2 no slice, 3 max_live)
+  const UnitBats* ub;
+  int64_t* bres;           // [R][E][kUnitBats]
+  ChainLayout cl;
+  const int* ovf;          // set by cand.cu when an epoch outgrew kUnitBats: the chain does nothing
   int R, N;
   int64_t base, trace_len, W, E, H;
   // policy
@@ -236,6 +276,35 @@ struct PartitionArgs {
 cudaError_t launch_partition_count(const PartitionArgs& A, cudaStream_t st);
 cudaError_t launch_partition_rest(const PartitionArgs& A, cudaStream_t st);
 cudaError_t preload_partition_kernels();
+
+// The candidate search ahead of the chain (cand.cu): batch-aligned stream cursors, then the keys
+// of every (replica, epoch, residue class, geometry) from idle, and every epoch's id-ordered
+// batch rows (UnitBats) for the lean chain and the accounting pass (chain.cu).
+struct CandParams {
+  const int32_t* tab;      // device table block (global)
+  TabLayout tl;
+  const uint32_t* sa;
+  const int64_t* saoff;
+  const uint32_t* sidx;    // [R][E+1][S]
+  uint32_t* bstart;        // [R][S][E+1] the chain's stream cursor at the start of each epoch
+  int64_t* kfc;            // [R][E][N][G]; [..][0][0] = INT64_MIN: unit not held, chain scores it
+  UnitBats* ub;            // [R][E] id-ordered batch rows, or NULL (fused chain: it forms its own)
+  int* overflow;           // set when some unit holds more than kUnitBats batches
+  const uint8_t* gorder;   // [G] geometries by slice count, descending (lane order)
+  int R, S, N, max_live;
+  int64_t E, W;
+  size_t ws_off;
+};
+cudaError_t launch_walk(const CandParams& P, cudaStream_t st);
+cudaError_t launch_cand(const CandParams& P, int grid, cudaStream_t st);
+cudaError_t cand_occupancy(const TabLayout& tl, int* per_sm);
+size_t cand_smem_bytes(const TabLayout& tl, size_t* ws_off);
+cudaError_t preload_cand_kernels();
+cudaError_t launch_chain(const ReplayParams& P, int grid, cudaStream_t st);
+cudaError_t launch_acct(const ReplayParams& P, cudaStream_t st);
+cudaError_t chain_occupancy(const ReplayParams& P, int* per_sm);
+size_t chain_smem_bytes(const ReplayParams& P);
+cudaError_t preload_chain_kernels();
 
 // launchers (replay.cu / score.cu)
 cudaError_t launch_roff_scan(const int64_t* roff, int R, int64_t* saoff, int* err, cudaStream_t st);

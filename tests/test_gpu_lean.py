@@ -1,0 +1,97 @@
+"""The lean replay path (csrc/cand.cu + csrc/chain.cu) vs the CPU oracle.  -m gpu.
+
+The lean path (a data-parallel candidate search ahead of a warp-per-replica chain, accounting in
+its own pass) serves many-replica mode-R calls; PROTEAN_LEAN=2 makes small cases take it too.  Each
+test asserts the path was taken (the accounting pass reports a time) and compares every output
+element by element with the oracle: closed-form epochs scored by cand.cu, epochs with an
+unavailable GPU scored in the chain, units cand.cu cannot hold (a class above 12 batches,
+completions 2^25 us past the epoch start), and calls with an epoch above 96 batches, which go back
+to the fused engine."""
+import numpy as np
+import pytest
+
+from gpu_common import GPU_LOG_DTYPE, compare, oracle_replay
+from protean_inputs import mix_a_params, mix_b_params, random_profiles, synth_profiles, tick_trace, uniform_trace
+
+pytestmark = pytest.mark.gpu
+
+
+def lean_replay(monkeypatch, prof, trace, *, expect_lean=True, **cfg):
+    import paper_conf_middleware_bhasisjgpkd24_b200 as pkg
+    monkeypatch.setenv("PROTEAN_LEAN", "2")
+    h = pkg.load_profiles(prof, device=0)
+    log_cap = max(1, int(np.max(np.diff(trace.replica_off))))
+    out = h.replay_traces_host(trace, want_cand_keys=True, log_cap=log_cap, **cfg)
+    search, walk, acct = h.last_search_ms()
+    h.close()
+    assert search > 0, "the candidate search did not run"
+    assert (acct > 0) == expect_lean, f"lean chain {'not ' if expect_lean else ''}taken (acct {acct} ms)"
+    out["log"] = out["log"].reshape(trace.n_replicas, log_cap, 32).view(GPU_LOG_DTYPE).reshape(
+        trace.n_replicas, log_cap)
+    out["hist"] = out["hist"].view(np.uint32)
+    return out
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_lean_fuzz(oracle, monkeypatch, seed):
+    rng = np.random.default_rng(700 + seed)
+    M = int(rng.integers(1, 7))
+    gset = int(rng.integers(0, 2))
+    prof = random_profiles(rng, M).with_geometry_set(gset)
+    N = int(rng.choice([2, 4, 8])) if gset else int(rng.choice([1, 2, 3, 8]))  # N * G even
+    R = int(rng.integers(1, 6))
+    tr = uniform_trace(rng, R, M, int(rng.integers(2, 12)) * 1_000_000, int(rng.integers(5, 600)))
+    cfg = dict(n_gpus=N, init_geom=int(rng.integers(0, 12)), max_live=int(rng.choice([2, 8, 64])),
+               wait_limit=int(rng.integers(0, 4)), reconfig_us=int(rng.integers(0, 3_000_000)),
+               vm_policy=int(seed % 3), p_rev=float(rng.choice([0.0, 0.354, 0.708, 1.0])),
+               rev_interval_us=2_000_000, notice_us=300_000, seed=seed)
+    tr.replica_base = int(rng.integers(0, 100))
+    g = lean_replay(monkeypatch, prof, tr, **cfg)
+    compare(g, oracle_replay(oracle, prof, tr, **cfg), R)
+
+
+@pytest.mark.parametrize("n_gpus", [8, 5])
+def test_lean_mix_a(oracle, monkeypatch, n_gpus):
+    """Config-5-shaped replicas (Mix A, 12 geometries): nearly every epoch closed-form."""
+    gp = mix_a_params(3, seed=11, seconds=40)
+    tr = tick_trace(gp)
+    P = synth_profiles()
+    g = lean_replay(monkeypatch, P, tr, n_gpus=n_gpus)
+    compare(g, oracle_replay(oracle, P, tr, n_gpus=n_gpus), 3)
+
+
+def test_lean_reconfig_heavy(oracle, monkeypatch):
+    """Short epochs and long reconfigurations: many epochs with an unavailable GPU (in-chain keys),
+    batches dropped for want of an available GPU, spot revocations."""
+    rng = np.random.default_rng(5)
+    prof = random_profiles(rng, 4, small_time=True)
+    tr = uniform_trace(rng, 4, 4, 3_000_000, 900)
+    cfg = dict(n_gpus=4, epoch_len_us=50_000, wait_limit=0, reconfig_us=120_000, vm_policy=2,
+               p_rev=0.5, rev_interval_us=200_000, notice_us=30_000, seed=3)
+    g = lean_replay(monkeypatch, prof, tr, **cfg)
+    compare(g, oracle_replay(oracle, prof, tr, **cfg), 4)
+
+
+def test_lean_units_not_held(oracle, monkeypatch):
+    """Units cand.cu does not hold: a residue class above 12 batches (one sim-GPU, dense tiny
+    batches) and completions beyond 2^25 us past the epoch start (solo times x 400)."""
+    rng = np.random.default_rng(9)
+    prof = random_profiles(rng, 3, max_batch=2)
+    tr = uniform_trace(rng, 2, 3, 4_000_000, 160)
+    g = lean_replay(monkeypatch, prof, tr, n_gpus=1)
+    compare(g, oracle_replay(oracle, prof, tr, n_gpus=1), 2)
+    slow = random_profiles(np.random.default_rng(10), 3)
+    slow.solo_us[:] = np.minimum(slow.solo_us.astype(np.int64) * 400, 2**31 - 1).astype(slow.solo_us.dtype)
+    tr2 = uniform_trace(np.random.default_rng(11), 2, 3, 3_000_000, 60)
+    g = lean_replay(monkeypatch, slow, tr2, n_gpus=2)
+    compare(g, oracle_replay(oracle, slow, tr2, n_gpus=2), 2)
+
+
+def test_lean_overflow_falls_back(oracle, monkeypatch):
+    """An epoch above 96 batches (Mix B x 8 on 8 sim-GPUs): the call goes back to the fused
+    engine, with identical results."""
+    gp = mix_b_params(1, seed=4, seconds=6, scale=8.0)
+    tr = tick_trace(gp)
+    P = synth_profiles()
+    g = lean_replay(monkeypatch, P, tr, expect_lean=False, n_gpus=8)
+    compare(g, oracle_replay(oracle, P, tr, n_gpus=8), 1)

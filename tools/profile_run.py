@@ -25,7 +25,7 @@ torch.cuda.synchronize()
 import json
 c = out["counters"].sum(0).cpu().tolist()
 info = {"replicas": a.replicas, "seconds": a.seconds, "requests": int(arr.shape[0]),
-        "slot_evals": int(c[8]), "geom_candidates": int(c[9]), "timings": h.last_timings()[:2],
+        "slot_evals": int(c[8]), "geom_candidates": int(c[9]), "timings": h.last_timings()[:2], "search_ms": h.last_search_ms(),
         "launch": h.last_timings()[2]}
 print(json.dumps(info))
 os.makedirs("gpurun_out", exist_ok=True)
