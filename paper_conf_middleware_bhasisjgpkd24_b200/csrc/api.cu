@@ -1050,7 +1050,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   int cper = 0, cgrid_l = 0;
   if (lean) {
     PL.cl.init(N, N * h->G);
-    const size_t sl_a = al((size_t)N * kZA * c.max_live * 20), sl_c = al((size_t)kUnitBats * 32 * 16);
+    const size_t sl_a = al((size_t)N * kZA * c.max_live * 20), sl_c = al((size_t)kUnitBats * 32 * 16 + 2 * kMaxSl * 32 * 4);
     PL.o_alist = 0;
     PL.o_clist = sl_a;
     PL.slot_bytes = sl_a + sl_c;

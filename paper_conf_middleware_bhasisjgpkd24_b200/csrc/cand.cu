@@ -191,11 +191,26 @@ __global__ void __launch_bounds__(32 * kCandWarps) cand_kernel(CandParams P) {
   uint8_t* gord = smem + ((P.tl.words * 4 + 15) & ~15);  // geometry order (slice count desc)
 #pragma unroll 1
   for (int i = tid; i < P.tl.G; i += blockDim.x) gord[i] = P.gorder[i];
+  // fitm[j][m]: the slice positions of geometry j whose memory holds model m's footprint
+  uint8_t* fitm = gord + ((P.tl.G + 15) & ~15);
+  {
+    Tab T0;
+    T0.bind(tabw, P.tl);
+    __syncthreads();  // the table is staged
+#pragma unroll 1
+    for (int i = tid; i < P.tl.G * P.tl.M; i += blockDim.x) {
+      const int j = i / P.tl.M, m = i % P.tl.M;
+      uint32_t f = 0;
+      for (int s = 0; s < T0.gn[j]; ++s)
+        if (T0.mem[m] <= T0.cap[T0.gprof[j * 8 + s]]) f |= 1u << s;
+      fitm[i] = (uint8_t)f;
+    }
+  }
   WarpSmem& ws = reinterpret_cast<WarpSmem*>(smem + P.ws_off)[warp];
   __syncthreads();
   Tab T;
   T.bind(tabw, P.tl);
-  const int S = P.S, N = P.N, G = P.tl.G;
+  const int S = P.S, N = P.N, G = P.tl.G, M = P.tl.M;
   const int64_t E = P.E, W = P.W;
   const int64_t n_units = (int64_t)P.R * E;
   const int npairs = N * G;
@@ -371,12 +386,13 @@ __global__ void __launch_bounds__(32 * kCandWarps) cand_kernel(CandParams P) {
         // strict = inelig << 31 | c << 6 | (4 - p) << 3 | s, best-effort = start << 3 | s
         uint32_t best = 0xFFFFFFFFu;
         uint32_t bst = 0, bc = 0;
-        const int nsx = __popc(alive) < P.max_live ? ns : 0;  // reading Q39: no room, no slice
+        // the slices of j that hold the batch's footprint (q <= Ms), none without room (Q39)
+        uint32_t fit = __popc(alive) < P.max_live ? (uint32_t)fitm[j * M + m] : 0u;
+        const uint32_t sflag = strict ? 0xFFFFFFFFu : 0u;
 #pragma unroll 1
-        for (int s = 0; s < nsx; ++s) {
+        for (; fit; fit &= fit - 1) {
+          const int s = __ffs(fit) - 1;
           const int p = gp[s];
-          const int32_t Ms = T.cap[p];
-          if (q > Ms) continue;
           const uint32_t lss = ws.ls[s][lane];
           const uint32_t t0 = rt > lss ? rt : lss;
           const uint32_t set = ws.msk[s][lane] & alive;
@@ -391,24 +407,27 @@ __global__ void __launch_bounds__(32 * kCandWarps) cand_kernel(CandParams P) {
             }
           }
           uint32_t start = t0;
-          if (used + q > Ms) {
+          if (used + q > T.cap[p]) {
             F = (uint32_t)fbr_m[p];
-            start = mem_wait(ws, lane, set, t0, q, Ms, &F);
+            start = mem_wait(ws, lane, set, t0, q, T.cap[p], &F);
           }
-          // Eq 1: exec = floor(solo * max(F, 10^6) / 10^6) = solo when F <= 10^6
+          // Eq 1: exec = floor(solo * max(F, 10^6) / 10^6) = solo when F <= 10^6.  Completions at or
+          // past 2^25 us clamp to 2^25 - 1 in the key (a clamped slice can only win when every
+          // slice clamps, and then the unit goes to the chain: checked once per batch below)
           const int32_t so = solo_m[p];
           const int64_t ex = F <= (uint32_t)kPpm ? (int64_t)so : exec_time(so, F);
-          const uint32_t cc = start + (uint32_t)ex;
-          wide |= (ex | (int64_t)cc) >= (1 << 25);  // start < 2^25 (a release or rt), so no wrap
-          const uint32_t key = strict  // choose_strict_slice (Alg 1 lines 1-8; Q11) / BE (Q12)
-              ? ((be >= gpref[s]) ? 0x80000000u : 0u) | (cc << 6) | ((uint32_t)(4 - p) << 3) | (uint32_t)s
-              : (start << 3) | (uint32_t)s;
+          const uint32_t cc = ex >= (1 << 25) ? (1u << 25) : min(start + (uint32_t)ex, 1u << 25);
+          const uint32_t ks = ((be >= gpref[s]) ? 0x80000000u : 0u) | (min(cc, (1u << 25) - 1u) << 6) |
+                              ((uint32_t)(4 - p) << 3) | (uint32_t)s;   // choose_strict_slice (Q11)
+          const uint32_t kb = (start << 3) | (uint32_t)s;               // choose_best_effort_slice (Q12)
+          const uint32_t key = (ks & sflag) | (kb & ~sflag);
           if (key < best) {
             best = key;
             bst = start;
             bc = cc;
           }
         }
+        wide |= best != 0xFFFFFFFFu && bc >= (1u << 25) - 1u;  // ends and keys are held in 25 bits
         const int bsl = best & 7;
         const bool placed = best != 0xFFFFFFFFu;
         ws.en[x][lane] = placed ? bc : 0u;
@@ -447,7 +466,8 @@ __global__ void __launch_bounds__(32 * kCandWarps) cand_kernel(CandParams P) {
 }  // namespace
 
 size_t cand_smem_bytes(const TabLayout& tl, size_t* ws_off) {
-  const size_t o = (((size_t)tl.words * 4 + 15) & ~(size_t)15) + (((size_t)tl.G + 15) & ~(size_t)15);
+  const size_t o = (((size_t)tl.words * 4 + 15) & ~(size_t)15) + (((size_t)tl.G + 15) & ~(size_t)15) +
+                   (((size_t)tl.G * tl.M + 15) & ~(size_t)15);
   *ws_off = o;
   return o + sizeof(WarpSmem) * kCandWarps;
 }

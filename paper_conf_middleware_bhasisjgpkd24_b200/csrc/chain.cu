@@ -161,6 +161,134 @@ __device__ int64_t score_idle(const Tab& T, int j, int cur, const UnitBats& U, c
   return make_key(misses, tail, j == cur ? 0 : j + 1);
 }
 
+// The same Alg 1 from idle in 32-bit time relative to eW with per-slice bit masks of the batches
+// placed so far (cand.cu's lane, its state in global scratch instead of shared memory).  Returns
+// false when a completion is 2^25 us past eW or the GPU holds more than 32 batches: the caller
+// then takes score_idle.
+__device__ bool score_idle32(const Tab& T, int j, int cur, const UnitBats& U, const uint8_t* gl, int cnt,
+                             const uint32_t* sa_r, int max_live, uint32_t eW32, int64_t eW, uint32_t* en,
+                             uint32_t* pk, int32_t* fb, uint32_t* lsm, int64_t* key_out) {
+  constexpr int L = 32;
+  if (cnt > 32) return false;
+  const int ns = T.gn[j];
+  const uint8_t* gp = T.gprof + j * 8;
+  const int32_t* gpref = T.gpref + j * 8;
+#pragma unroll 1
+  for (int s = 0; s < ns; ++s) {
+    lsm[(2 * s) * L] = 0;      // last start
+    lsm[(2 * s + 1) * L] = 0;  // batches placed on the slice
+  }
+  uint32_t alive = 0;
+  int be = 0;
+  bool wide = false;
+  int64_t misses = 0, tail = 0;
+#pragma unroll 1
+  for (int x = 0; x < cnt; ++x) {
+    const int b = gl[x];
+    const uint32_t info = U.info[b];
+    const int m = (info >> 16) & 0xFF, nreq = info & 0xFFFF;
+    const bool strict = (info >> 24) & 1;
+    const uint32_t rt = U.ready[b] - eW32;
+#pragma unroll 1
+    for (uint32_t a = alive; a; a &= a - 1) {
+      const int i = __ffs(a) - 1;
+      if (en[i * L] <= rt) {
+        alive &= ~(1u << i);
+        if (pk[i * L] >> 27) be -= (int)(pk[i * L] & kMemMask);
+      }
+    }
+    const int32_t q = T.mem[m];
+    const int32_t* fbr_m = T.fbr + m * kNProf;
+    const int32_t* solo_m = T.solo + m * kNProf;
+    uint32_t best = 0xFFFFFFFFu, bst = 0, bc = 0;
+    const int nsx = __popc(alive) < max_live ? ns : 0;
+#pragma unroll 1
+    for (int s = 0; s < nsx; ++s) {
+      const int p = gp[s];
+      const int32_t Ms = T.cap[p];
+      if (q > Ms) continue;
+      const uint32_t lss = lsm[(2 * s) * L];
+      const uint32_t t0 = rt > lss ? rt : lss;
+      const uint32_t set = lsm[(2 * s + 1) * L] & alive;
+      int32_t used = 0;
+      uint32_t F = (uint32_t)fbr_m[p];
+#pragma unroll 1
+      for (uint32_t a = set; a; a &= a - 1) {
+        const int i = __ffs(a) - 1;
+        if (en[i * L] > t0) {
+          used += (int32_t)(pk[i * L] & kMemMask);
+          F += (uint32_t)fb[i * L];
+        }
+      }
+      uint32_t start = t0;
+      if (used + q > Ms) {  // releases after t0 ascending; the first that fits
+        uint32_t ev = t0;
+#pragma unroll 1
+        for (;;) {
+          uint32_t nxt = 0xFFFFFFFFu;
+          for (uint32_t a = set; a; a &= a - 1) {
+            const uint32_t e = en[(__ffs(a) - 1) * L];
+            if (e > ev && e < nxt) nxt = e;
+          }
+          ev = nxt;
+          int32_t rem = 0;
+          for (uint32_t a = set; a; a &= a - 1) {
+            const int i = __ffs(a) - 1;
+            if (en[i * L] > ev) rem += (int32_t)(pk[i * L] & kMemMask);
+          }
+          if (rem + q <= Ms) break;
+        }
+        start = ev;
+        F = (uint32_t)fbr_m[p];
+        for (uint32_t a = set; a; a &= a - 1) {
+          const int i = __ffs(a) - 1;
+          if (en[i * L] > start) F += (uint32_t)fb[i * L];
+        }
+      }
+      const int32_t so = solo_m[p];
+      const int64_t ex = F <= (uint32_t)kPpm ? (int64_t)so : exec_time(so, F);
+      const uint32_t cc = start + (uint32_t)ex;
+      wide |= (ex | (int64_t)cc) >= (1 << 25);
+      const uint32_t key = strict
+          ? ((be >= gpref[s]) ? 0x80000000u : 0u) | (cc << 6) | ((uint32_t)(4 - p) << 3) | (uint32_t)s
+          : (start << 3) | (uint32_t)s;
+      if (key < best) {
+        best = key;
+        bst = start;
+        bc = cc;
+      }
+    }
+    if (wide) return false;
+    const bool placed = best != 0xFFFFFFFFu;
+    const int bsl = best & 7;
+    en[x * L] = placed ? bc : 0u;
+    pk[x * L] = (uint32_t)q | (strict ? 0u : (1u << 27));
+    fb[x * L] = fbr_m[gp[bsl]];
+    if (placed) {
+      lsm[(2 * bsl) * L] = bst;
+      lsm[(2 * bsl + 1) * L] |= 1u << x;
+      alive |= 1u << x;
+      if (!strict) be += q;
+    }
+    const int64_t cw = eW + (int64_t)bc;
+    const uint32_t* ma = sa_r + U.pos[b];
+    if (strict) {
+      if (!placed) {
+        misses += nreq;
+      } else {
+        const int64_t slo = T.slo[m];
+        if (cw - (int64_t)ma[0] > slo)
+          misses += (cw - (int64_t)ma[nreq - 1] > slo) ? nreq : nreq - hits_in(ma, nreq, cw, slo);
+      }
+    } else {
+      const int64_t tb = placed ? cw - (int64_t)ma[0] : (int64_t)0xFFFFFFFFLL;
+      tail = tb > tail ? tb : tail;
+    }
+  }
+  *key_out = make_key(misses, tail, j == cur ? 0 : j + 1);
+  return true;
+}
+
 __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_kernel(ReplayParams P) {
   extern __shared__ __align__(16) unsigned char smem[];
   if (*(volatile const int*)P.ovf) return;  // the host replays the call on the fused engine
@@ -203,6 +331,8 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
   int64_t* sc_en = reinterpret_cast<int64_t*>(slot + P.o_clist) + lane;  // score_idle arrays
   uint32_t* sc_pk = reinterpret_cast<uint32_t*>(slot + P.o_clist + (size_t)kUB * 32 * 8) + lane;
   int32_t* sc_fb = reinterpret_cast<int32_t*>(slot + P.o_clist + (size_t)kUB * 32 * 12) + lane;
+  uint32_t* sc_ls = reinterpret_cast<uint32_t*>(slot + P.o_clist + (size_t)kUB * 32 * 16) + lane;
+  uint32_t* sc_en32 = reinterpret_cast<uint32_t*>(slot + P.o_clist) + lane;  // score_idle32's ends
   constexpr int kUBChunks = (int)(sizeof(UnitBats) / 16);
 
 #pragma unroll 1
@@ -295,40 +425,41 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
         for (int g = lane; g <= N; g += 32) c.g_off[g] = goff(g);
         cursor = (int)((cursor + nb) % N);
       } else {
-        if (lane == 0) {  // the plain round robin over the GPUs available at the batch's ready time
-          int cu = cursor;
+        // round robin over the GPUs available at each batch's ready time (lane = GPU): a ballot
+        // of availability, the first available GPU at or after the cursor
+        const unsigned nmask = N == 32 ? 0xffffffffu : ((1u << N) - 1u);
+        int cu = cursor;
 #pragma unroll 1
-          for (int g = 0; g < N; ++g) c.g_cnt[g] = 0;
-#pragma unroll 1
-          for (int b = 0; b < nb; ++b) {
-            int chosen = -1;
-#pragma unroll 1
-            for (int i = 0; i < N; ++i) {
-              const int g = (cu + i) % N;
-              if (available(c, g, U.ready[b])) { chosen = g; break; }
-            }
-            gpu_of[b] = chosen < 0 ? 0xFF : (uint8_t)chosen;
-            if (chosen >= 0) {
-              c.g_cnt[chosen]++;
-              cu = (chosen + 1) % N;
-            }
+        for (int b = 0; b < nb; ++b) {
+          const unsigned av = __ballot_sync(0xffffffffu, lane < N && available(c, lane, U.ready[b])) & nmask;
+          int chosen = -1;
+          if (av) {
+            const unsigned hi = av & ~((1u << cu) - 1u);  // GPUs cu..N-1
+            chosen = hi ? __ffs(hi) - 1 : __ffs(av) - 1;
+            cu = chosen + 1 == N ? 0 : chosen + 1;
           }
-          int off = 0;
-#pragma unroll 1
-          for (int g = 0; g < N; ++g) {
-            c.g_off[g] = off;
-            off += c.g_cnt[g];
-            c.g_cnt[g] = 0;
-          }
-          c.g_off[N] = off;
-#pragma unroll 1
-          for (int b = 0; b < nb; ++b) {
-            const int g = gpu_of[b];
-            if (g != 0xFF) gl[c.g_off[g] + c.g_cnt[g]++] = (uint8_t)b;
-          }
-          cursor = cu;
+          if (lane == 0) gpu_of[b] = chosen < 0 ? 0xFF : (uint8_t)chosen;
         }
-        cursor = __shfl_sync(0xffffffffu, cursor, 0);
+        cursor = cu;
+        __syncwarp();
+        {  // per-GPU lists in id order: counts, exclusive scan over lanes, fill
+          int cntg = 0;
+          if (lane < N)
+            for (int b = 0; b < nb; ++b) cntg += gpu_of[b] == lane ? 1 : 0;
+          int x = cntg;
+#pragma unroll
+          for (int d = 1; d < 32; d <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, x, d);
+            if (lane >= d) x += y;
+          }
+          if (lane < N) {
+            int o = x - cntg;
+            c.g_off[lane] = o;
+            for (int b = 0; b < nb; ++b)
+              if (gpu_of[b] == lane) gl[o++] = (uint8_t)b;
+          }
+          if (lane == N - 1) c.g_off[N] = x;
+        }
         __syncwarp();
 #pragma unroll 1
         for (int b = lane; b < nb; b += 32) {  // no GPU available: dropped (drop code 1)
@@ -455,9 +586,12 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
         for (int pi = lane; pi < N * G; pi += 32) {
           const int g = pi / G, j = pi - g * G;
           int64_t key = -1;
-          if (c.gu8[5 * N + g])
-            key = score_idle(T, j, c.gu8[0 * N + g], U, gl + c.g_off[g], c.g_off[g + 1] - c.g_off[g], sa_r,
-                             P.max_live, sc_en, sc_pk, sc_fb);
+          if (c.gu8[5 * N + g]) {
+            const int cur = c.gu8[0 * N + g], x0 = c.g_off[g], cnt = c.g_off[g + 1] - x0;
+            if (!score_idle32(T, j, cur, U, gl + x0, cnt, sa_r, P.max_live, (uint32_t)eW, eW,
+                              sc_en32, sc_pk, sc_fb, sc_ls, &key))
+              key = score_idle(T, j, cur, U, gl + x0, cnt, sa_r, P.max_live, sc_en, sc_pk, sc_fb);
+          }
           kst[pi] = key;  // by GPU
         }
         __syncwarp();
@@ -587,7 +721,10 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
 }
 
 // ---------------------------------------------------------------- accounting (O7, O12)
-__global__ void __launch_bounds__(32 * kAcctWarps) acct_kernel(ReplayParams P) {
+#ifndef PROTEAN_ACCT_MINB
+#define PROTEAN_ACCT_MINB 4  // measured (4096 x 120 s): 4 -> 4.08, 6 -> 4.13, 8 -> 4.27 ms (issue-bound)
+#endif
+__global__ void __launch_bounds__(32 * kAcctWarps, PROTEAN_ACCT_MINB) acct_kernel(ReplayParams P) {
   if (*(volatile const int*)P.ovf) return;
   __shared__ uint32_t s_hist[2 * kNB];
   __shared__ uint32_t s_sink;
