@@ -22,7 +22,9 @@ METRICS = ["dram__bytes_read.sum", "dram__bytes_write.sum", "smsp__inst_executed
            "sm__warps_active.avg.pct_of_peak_sustained_active", "gpu__time_duration.sum",
            "sm__cycles_elapsed.avg.per_second", "smsp__thread_inst_executed_per_inst_executed.ratio"]
 SHORT = {"replay_kernel": "replay_kernel", "prepass_kernel": "prepass", "part_count": "part_count",
-         "part_scan": "part_scan", "part_scatter": "part_scatter", "sweep_kernel": "sweep_kernel"}
+         "part_scan": "part_scan", "part_scatter": "part_scatter", "sweep_kernel": "sweep_kernel",
+         "walk_kernel": "walk_kernel", "cand_kernel": "cand_kernel", "chain_kernel": "chain_kernel",
+         "acct_kernel": "acct_kernel"}
 
 
 def run(a):
@@ -84,7 +86,7 @@ def parse(a):
                      "warps_active_pct": m.get("sm__warps_active.avg.pct_of_peak_sustained_active"),
                      "active_threads_per_warp": m.get("smsp__thread_inst_executed_per_inst_executed.ratio"),
                      "sm_clock_hz": m.get("sm__cycles_elapsed.avg.per_second")}
-        if key == "replay_kernel" and info.get("slot_evals"):
+        if key in ("replay_kernel", "cand_kernel") and info.get("slot_evals"):
             kern[key]["warp_instructions_per_slot_eval"] = m.get("smsp__inst_executed.sum", 0) / info["slot_evals"]
     out = {"report": f"{a.round}: ncu --metrics (per-kernel) of tools/profile_run.py --replicas "
                      f"{info['replicas']} --seconds {info['seconds']} (config-5 shape)",

@@ -25,6 +25,13 @@ def main(which: str):
         prof, tr = c1_profiles(), c1_trace()
         compare(gpu_replay(prof, tr, n_gpus=1), oracle_replay(O, prof, tr, n_gpus=1), 1)
         print("c1 replay ok")
+    elif which == "lean":  # the lean path (cand.cu + chain.cu), forced on small Mix A replicas
+        os.environ["PROTEAN_LEAN"] = "2"
+        from protean_inputs import mix_a_params
+        prof = synth_profiles()
+        tr = tick_trace(mix_a_params(3, seed=11, seconds=12))
+        compare(gpu_replay(prof, tr, n_gpus=8), oracle_replay(O, prof, tr, n_gpus=8), 3)
+        print("lean replay ok")
     elif which in ("c2", "c2many"):
         prof = synth_profiles()
         R = 1 if which == "c2" else 8
