@@ -35,7 +35,7 @@ namespace pemgpu {
 namespace {
 
 constexpr int kBC = kUnitBats;  // batches per (replica, epoch) unit held in shared memory
-constexpr int kKC = 12;        // batches per residue class held per lane (<= 32: bit masks)
+constexpr int kKC = 10;        // batches per residue class held per lane (config 5: ~5)
 constexpr int kCandWarps = 8;  // warps per CTA
 
 // ---------------------------------------------------------------- walk
@@ -118,16 +118,21 @@ __global__ void __launch_bounds__(256) walk_kernel(CandParams P) {
 
 // ---------------------------------------------------------------- candidates
 struct WarpSmem {
-  uint64_t key[kBC];
+  union {                  // the rank keys are dead once the epoch is in id order
+    uint64_t key[kBC];
+    struct {
+      uint32_t en[kKC][32];  // per lane: end of each placed batch, relative to eW (0: dropped)
+      uint32_t pk[kKC][32];  //           footprint | best-effort << 27
+      int32_t fb[kKC][32];   //           FBR of the batch on its slice's profile
+    };
+  };
   uint32_t ready[kBC], info[kBC], pos[kBC], afirst[kBC], alast[kBC];
   uint8_t ord[kBC];
-  uint32_t en[kKC][32];  // per lane: end of each placed batch, relative to eW (0: dropped)
-  uint32_t pk[kKC][32];  //           footprint | best-effort << 27
-  int32_t fb[kKC][32];   //           FBR of the batch on its slice's profile
   uint32_t ls[kMaxSl][32];   //       last start per slice position (FIFO), relative to eW
-  uint32_t msk[kMaxSl][32];  //       batches placed on each slice position
+  uint16_t msk[kMaxSl][32];  //       batches placed on each slice position
   int nb, bad;
 };
+static_assert(kKC <= 16, "16-bit slice masks");
 
 // Memory wait of Alg 1 on one slice (the batch does not fit at t0): releases after t0 in ascending
 // order, the footprint still held only shrinks, so the first that fits is the minimum of the plain
@@ -435,7 +440,7 @@ __global__ void __launch_bounds__(32 * kCandWarps) cand_kernel(CandParams P) {
         ws.fb[x][lane] = fbr_m[gp[bsl]];
         if (placed) {
           ws.ls[bsl][lane] = bst;
-          ws.msk[bsl][lane] |= 1u << x;
+          ws.msk[bsl][lane] |= (uint16_t)(1u << x);
           alive |= 1u << x;
           if (!strict) be += q;
         }
