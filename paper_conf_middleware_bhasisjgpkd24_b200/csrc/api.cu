@@ -986,7 +986,8 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   // the lean chain (chain.cu): a warp per replica on cand.cu's batch rows and keys, accounting in
   // its own pass; many-replica calls without container pools (an epoch with more than 96 batches
   // sends the call back to the fused engine below)
-  bool lean = precand && (!few_r || lean_force) && c.cold_start_us == 0 && (N * h->G) % 2 == 0;
+  bool lean = precand && (!few_r || lean_force) && c.cold_start_us == 0 && (N * h->G) % 2 == 0 &&
+              c.max_live <= 64;  // the chain's resident slots: 64-bit masks
   if (lean_env && std::atoi(lean_env) == 0) lean = false;  // experiment knob: 0 = the fused engine
   size_t b_ub = 0, b_br = 0;
   if (precand) {
@@ -1049,8 +1050,8 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   ReplayParams PL = P;
   int cper = 0, cgrid_l = 0;
   if (lean) {
-    PL.cl.init(N, N * h->G);
-    const size_t sl_a = al((size_t)N * kZA * c.max_live * 20), sl_c = al((size_t)kUnitBats * 32 * 16 + 2 * kMaxSl * 32 * 4);
+    PL.cl.init(N, N * h->G, h->G, h->M);
+    const size_t sl_a = al((size_t)64 * 32 * 16), sl_c = al((size_t)kUnitBats * 32 * 16 + 2 * kMaxSl * 32 * 4);
     PL.o_alist = 0;
     PL.o_clist = sl_a;
     PL.slot_bytes = sl_a + sl_c;

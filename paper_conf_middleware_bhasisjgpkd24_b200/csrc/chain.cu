@@ -298,6 +298,20 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
   for (int i = tid; i < P.tl.words; i += blockDim.x) tabw[i] = P.tab[i];
   __syncthreads();
   const ChainLayout& CL = P.cl;
+  {
+    uint8_t* fw = smem + (((size_t)P.tl.words * 4 + 15) & ~(size_t)15) + (size_t)kChainWarps * CL.total;
+    Tab T0;
+    T0.bind(tabw, P.tl);
+#pragma unroll 1
+    for (int i = tid; i < P.tl.G * P.tl.M; i += blockDim.x) {
+      const int j = i / P.tl.M, m = i % P.tl.M;
+      uint32_t f = 0;
+      for (int s = 0; s < T0.gn[j]; ++s)
+        if (T0.mem[m] <= T0.cap[T0.gprof[j * 8 + s]]) f |= 1u << s;
+      fw[i] = (uint8_t)f;
+    }
+    __syncthreads();
+  }
   unsigned char* wb = smem + (((size_t)P.tl.words * 4 + 15) & ~(size_t)15) + (size_t)warp * CL.total;
   const int N = P.N, G = P.tl.G, KS = CL.KS;
   const int64_t E = P.E, W = P.W;
@@ -319,15 +333,14 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
   int sum_slots = 0;  // slot-evals per batch per decidable GPU (counter 8)
 #pragma unroll 1
   for (int j = 0; j < G; ++j) sum_slots += T.gn[j];
-  const int n_aunits = (N + kAG - 1) / kAG;
   const int gw = blockIdx.x * kChainWarps + warp;  // this warp's scratch slot
   char* slot = P.scratch + (size_t)gw * P.slot_bytes;
-  const int NA = N * kZA;
-  LaneList AL;
-  AL.stride = NA;
-  AL.st = reinterpret_cast<int64_t*>(slot + P.o_alist);
-  AL.en = AL.st + (size_t)NA * P.max_live;
-  AL.mm = reinterpret_cast<uint32_t*>(AL.en + (size_t)NA * P.max_live);
+  // the actual residents of GPU lane: 64 slots, lane-interleaved (slot i of lane l at i * 32 + l)
+  int64_t* ga_en = reinterpret_cast<int64_t*>(slot + P.o_alist) + lane;
+  uint32_t* ga_pk = reinterpret_cast<uint32_t*>(slot + P.o_alist + 64 * 32 * 8) + lane;
+  int32_t* ga_fb = reinterpret_cast<int32_t*>(slot + P.o_alist + 64 * 32 * 12) + lane;
+  // fitm[j][m]: the slice positions of geometry j that hold model m's footprint (CTA-wide table)
+  const uint8_t* fitm = smem + (((size_t)P.tl.words * 4 + 15) & ~(size_t)15) + (size_t)kChainWarps * CL.total;
   int64_t* sc_en = reinterpret_cast<int64_t*>(slot + P.o_clist) + lane;  // score_idle arrays
   uint32_t* sc_pk = reinterpret_cast<uint32_t*>(slot + P.o_clist + (size_t)kUB * 32 * 8) + lane;
   int32_t* sc_fb = reinterpret_cast<int32_t*>(slot + P.o_clist + (size_t)kUB * 32 * 12) + lane;
@@ -483,100 +496,146 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
         }
       }
       __syncwarp();
-      // ---- E: actual placement, four GPUs per pass, lane per MIG slice (replay.cu phase E)
+      // ---- E: actual placement (O6, Alg 1), lane = simulated GPU, its batches in id order.
+      // The carried residents of a GPU live in 64 slots (max_live <= 64): an alive mask, per-slice
+      // masks, and per slot the end, footprint | best-effort flag and the FBR on its slice's
+      // profile.  Per-slice FIFO keeps every resident's start <= the slice's last start <= t0, so
+      // Eq 1's co-runners at any tried start are the slice's residents that end after it.
+      if (lane < N) {
+        const int g = lane, j = c.gu8[0 * N + g];
+        uint64_t* alive_p = reinterpret_cast<uint64_t*>(c.a_n + g * kZA);
+        uint64_t alive = *alive_p;
+        uint64_t* msk = reinterpret_cast<uint64_t*>(wb + CL.msk) + g * kZA;
+        int64_t* lsg = c.a_ls + g * kZA;
+        int64_t* bug = c.a_bu + g * kZA;
+        const uint8_t* gp = T.gprof + j * 8;
+        const int32_t* gpref = T.gpref + j * 8;
+        int64_t acc0 = 0, acc1 = 0;  // busy, memory-time of the placed batches
+        const int x0 = c.g_off[g], cnt = c.g_off[g + 1] - x0;
 #pragma unroll 1
-      for (int u = 0; u < n_aunits; ++u) {
-        const int g = u * kAG + (lane >> 3), s = lane & 7, gbase = lane & ~7;
-        const bool valid = (lane >> 3) < kAG && g < N;
-        const int j = valid ? c.gu8[0 * N + g] : 0;
-        const bool active = valid && s < T.gn[j];
-        const int p = active ? T.gprof[j * 8 + s] : 0;
-        SliceLane K;
-        K.fbr_p = T.fbr + p;
-        K.solo_p = T.solo + p;
-        K.Ms = T.cap[p];
-        K.pref = T.gpref[j * 8 + (s & 7)];
-        K.s = s;
-        K.p = p;
-        K.Z = kZA;
-        const int al = valid ? g * kZA + s : 0;
-        LaneList Lst = AL;
-        Lst.st += al;
-        Lst.en += al;
-        Lst.mm += al;
-        int n = valid ? c.a_n[al] : 0;
-        int64_t ls = valid ? c.a_ls[al] : 0;
-        int64_t bu = valid ? c.a_bu[al] : 0;
-        const int x0 = valid ? c.g_off[g] : 0, x1 = valid ? c.g_off[g + 1] : 0;
-        int len_max = x1 - x0;
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-          const int o = __shfl_xor_sync(0xffffffffu, len_max, d);
-          len_max = o > len_max ? o : len_max;
-        }
-        int64_t acc0 = 0, acc1 = 0;  // busy, memory-time of the slice's winners
-#pragma unroll 1
-        for (int xi = 0; xi < len_max; ++xi) {
-          const bool has = xi < x1 - x0;
-          const int b = has ? gl[x0 + xi] : 0;
-          const uint32_t info = has ? U.info[b] : 0u;
+        for (int xi = 0; xi < cnt; ++xi) {
+          const int b = gl[x0 + xi];
+          const uint32_t info = U.info[b];
           const int m = (info >> 16) & 0xFF;
           const bool strict = (info >> 24) & 1;
-          const int64_t t = has ? (int64_t)U.ready[b] : 0;
-          int64_t st, en;
-          const SliceOut so = place_group<1>(T, active && has, K, Lst, n, ls, t, m, strict, P.max_live, &st, &en);
-          const bool placed = !so.drop_overflow && so.kmin != ~0ull;
-          const int wl = (gbase + (int)(so.kmin & 7)) & 31;
-          if (!has) continue;
-          const bool rec_here = placed ? lane == wl : lane == gbase;
-          if (placed && lane == wl) {  // busy union + memory-time, clipped to [0, H)
-            const int64_t lo = st > bu ? st : bu;
-            const int64_t hi = en < P.H ? en : P.H;
-            if (hi > lo) acc0 += (int64_t)prof_compute(p) * (hi - lo);
-            if (hi > st) acc1 += (int64_t)T.mem[m] * (hi - st);
-            if (en > bu) bu = en;
-          }
-          if (rec_here) {
-            const int drop = placed ? 0 : (so.drop_overflow ? 3 : 2);
-            bres[(size_t)e * kUB + b] = placed ? en : -(int64_t)drop;
-            if (P.log && nlog + b < P.log_cap) {
-              protean_batch_rec rec;
-              rec.ready_us = U.ready[b];
-              rec.epoch = (uint32_t)e;
-              rec.n_req = (uint16_t)(info & 0xFFFF);
-              rec.model = (uint8_t)m;
-              rec.strict = strict ? 1 : 0;
-              rec.gpu = (uint8_t)g;
-              rec.slice = placed ? (uint8_t)s : 0xFF;
-              rec.dropped = (uint8_t)drop;
-              rec.pad = 0;
-              rec.start_us = placed ? st : 0;
-              rec.end_us = placed ? en : 0;
-              P.log[(size_t)r * P.log_cap + nlog + b] = rec;
+          const int64_t t = (int64_t)U.ready[b];
+          const int32_t q = T.mem[m];
+          int be = 0;  // best-effort footprint still running at t (Alg 1's tag walk)
+#pragma unroll 1
+          for (uint64_t a = alive; a; a &= a - 1) {  // residents ended by t never matter again
+            const int i = __ffsll((long long)a) - 1;
+            if (ga_en[i * 32] <= t) {
+              alive &= ~(1ull << i);
+            } else {
+              const uint32_t pki = ga_pk[i * 32];
+              if (pki >> 27) be += (int)(pki & kMemMask);
             }
           }
-        }
-        int64_t mx = 0;
-        if (valid) {
-          c.a_n[al] = n;
-          c.a_ls[al] = ls;
-          c.a_bu[al] = bu;
+          const bool overflow = __popcll(alive) >= P.max_live;  // reading Q39
+          uint64_t best = ~0ull;
+          int64_t bst = 0, bend = 0;
+          uint32_t fit = overflow ? 0u : (uint32_t)fitm[j * CL.M + m];
 #pragma unroll 1
-          for (int i = 0; i < n; ++i) mx = Lst.E(i) > mx ? Lst.E(i) : mx;
-        }
+          for (; fit; fit &= fit - 1) {
+            const int s = __ffs(fit) - 1;
+            const int p = gp[s];
+            const int32_t Ms = T.cap[p];
+            const int64_t t0 = t > lsg[s] ? t : lsg[s];
+            const uint64_t set = msk[s] & alive;
+            int32_t used = 0;
+            int64_t F = T.fbr[m * kNProf + p];
+#pragma unroll 1
+            for (uint64_t a = set; a; a &= a - 1) {
+              const int i = __ffsll((long long)a) - 1;
+              if (ga_en[i * 32] > t0) {
+                used += (int32_t)(ga_pk[i * 32] & kMemMask);
+                F += ga_fb[i * 32];
+              }
+            }
+            int64_t start = t0;
+            if (used + q > Ms) {  // the earliest release after which the batch fits (q <= Ms)
+              int64_t ev = t0;
+#pragma unroll 1
+              for (;;) {
+                int64_t nxt = INT64_MAX;
+                int32_t rem = 0;
+                for (uint64_t a = set; a; a &= a - 1) {
+                  const int64_t ei = ga_en[(__ffsll((long long)a) - 1) * 32];
+                  if (ei > ev && ei < nxt) nxt = ei;
+                }
+                ev = nxt;
+                for (uint64_t a = set; a; a &= a - 1) {
+                  const int i = __ffsll((long long)a) - 1;
+                  if (ga_en[i * 32] > ev) rem += (int32_t)(ga_pk[i * 32] & kMemMask);
+                }
+                if (rem + q <= Ms) break;
+              }
+              start = ev;
+              F = T.fbr[m * kNProf + p];
+              for (uint64_t a = set; a; a &= a - 1) {
+                const int i = __ffsll((long long)a) - 1;
+                if (ga_en[i * 32] > start) F += ga_fb[i * 32];
+              }
+            }
+            const int64_t cc = start + exec_time(T.solo[m * kNProf + p], F);
+            const uint64_t key = strict  // choose_strict_slice (Q11) / choose_best_effort_slice (Q12)
+                ? ((be >= gpref[s]) ? (1ull << 62) : 0ull) | ((uint64_t)cc << 6) | ((uint64_t)(4 - p) << 3) | (uint64_t)s
+                : ((uint64_t)start << 3) | (uint64_t)s;
+            if (key < best) {
+              best = key;
+              bst = start;
+              bend = cc;
+            }
+          }
+          const bool placed = best != ~0ull;
+          const int s = (int)(best & 7);
+          if (placed) {  // schedule(batch, slice): a free slot, the slice's FIFO, the busy union
+            const int i = __ffsll((long long)~alive) - 1;
+            const int p = gp[s];
+            ga_en[i * 32] = bend;
+            ga_pk[i * 32] = (uint32_t)q | (strict ? 0u : (1u << 27));
+            ga_fb[i * 32] = T.fbr[m * kNProf + p];
+            alive |= 1ull << i;
 #pragma unroll
-        for (int d = 1; d < 8; d <<= 1) {
-          const int64_t o = __shfl_xor_sync(0xffffffffu, mx, d);
-          mx = o > mx ? o : mx;
+            for (int z = 0; z < kZA; ++z) msk[z] &= ~(1ull << i);
+            msk[s] |= 1ull << i;
+            lsg[s] = bst;
+            const int64_t bu = bug[s];
+            const int64_t lo = bst > bu ? bst : bu;
+            const int64_t hi = bend < P.H ? bend : P.H;
+            if (hi > lo) acc0 += (int64_t)prof_compute(p) * (hi - lo);
+            if (hi > bst) acc1 += (int64_t)q * (hi - bst);
+            if (bend > bu) bug[s] = bend;
+          }
+          const int drop = placed ? 0 : (overflow ? 3 : 2);
+          bres[(size_t)e * kUB + b] = placed ? bend : -(int64_t)drop;
+          if (P.log && nlog + b < P.log_cap) {
+            protean_batch_rec rec;
+            rec.ready_us = U.ready[b];
+            rec.epoch = (uint32_t)e;
+            rec.n_req = (uint16_t)(info & 0xFFFF);
+            rec.model = (uint8_t)m;
+            rec.strict = strict ? 1 : 0;
+            rec.gpu = (uint8_t)g;
+            rec.slice = placed ? (uint8_t)s : 0xFF;
+            rec.dropped = (uint8_t)drop;
+            rec.pad = 0;
+            rec.start_us = placed ? bst : 0;
+            rec.end_us = placed ? bend : 0;
+            P.log[(size_t)r * P.log_cap + nlog + b] = rec;
+          }
         }
-        const int64_t bsum = group_sum(acc0, 8), msum = group_sum(acc1, 8);
-        if (valid && s == 0) {
-          c.gi[5 * N + g] = mx;
-          c.gi[10 * N + g] += bsum;
-          c.gi[11 * N + g] += msum;
+        *alive_p = alive;
+        int64_t mx = 0;  // the latest end among the GPU's residents (drain end of a reconfiguration)
+        for (uint64_t a = alive; a; a &= a - 1) {
+          const int64_t ei = ga_en[(__ffsll((long long)a) - 1) * 32];
+          mx = ei > mx ? ei : mx;
         }
-        __syncwarp();
+        c.gi[5 * N + g] = mx;
+        c.gi[10 * N + g] += acc0;
+        c.gi[11 * N + g] += acc1;
       }
+      __syncwarp();
       cp_async_wait_all();
       __syncwarp();
       // ---- candidate keys: cand.cu's (closed form) or scored here
@@ -898,7 +957,7 @@ __global__ void __launch_bounds__(32 * kAcctWarps, PROTEAN_ACCT_MINB) acct_kerne
 }  // namespace
 
 size_t chain_smem_bytes(const ReplayParams& P) {
-  return (((size_t)P.tl.words * 4 + 15) & ~(size_t)15) + P.cl.total * kChainWarps;
+  return (((size_t)P.tl.words * 4 + 15) & ~(size_t)15) + P.cl.total * kChainWarps + P.cl.fitm;
 }
 
 cudaError_t chain_occupancy(const ReplayParams& P, int* per_sm) {

@@ -98,9 +98,10 @@ struct XLayout {
 // Per-warp shared-memory layout of the lean chain (chain.cu), byte offsets from the warp's base.
 struct ChainLayout {
   int N, KS;
-  size_t gu8, gi, gcnt, goff, a_n, a_ls, a_bu, kst, ub, gl, gpu, total;
-  __host__ void init(int n, int ks) {
-    N = n; KS = ks;
+  int G, M;
+  size_t gu8, gi, gcnt, goff, a_n, a_ls, a_bu, msk, kst, ub, gl, gpu, total, fitm;
+  __host__ void init(int n, int ks, int g, int m) {
+    N = n; KS = ks; G = g; M = m;
     size_t o = 0;
     auto take = [&](size_t bytes) { size_t r = o; o += (bytes + 15) & ~(size_t)15; return r; };
     ub = take(2 * sizeof(UnitBats));             // this epoch's rows and the next one's (cp.async)
@@ -112,9 +113,11 @@ struct ChainLayout {
     a_n = take((size_t)N * kZA * 4);
     a_ls = take((size_t)N * kZA * 8);
     a_bu = take((size_t)N * kZA * 8);
+    msk = take((size_t)N * kZA * 8);             // per (GPU, slice): resident slots on the slice
     gl = take(kUnitBats);
     gpu = take(kUnitBats);
     total = o;
+    fitm = ((size_t)G * M + 15) & ~(size_t)15;   // per CTA: [G][M] slices of j that hold model m
   }
 };
 
