@@ -357,6 +357,12 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
     const uint32_t* sa_r = P.sa + P.saoff[r];
     // ---- replica init (as replay.cu)
 #pragma unroll 1
+    for (int i = lane; i < N * kZA; i += 32) reinterpret_cast<uint64_t*>(wb + CL.msk)[i] = 0;
+#pragma unroll 1
+    for (int i = lane; i < 64; i += 32)  // every slot's packed word names slice 0 (no stale bits)
+      for (int g = 0; g < N; ++g)
+        reinterpret_cast<uint32_t*>(slot + P.o_alist + 64 * 32 * 8)[i * 32 + g] = 0;
+#pragma unroll 1
     for (int g = lane; g < N; g += 32) {
       reset_gpu_state(c, g, P.init_geom);
       c.gu8[3 * N + g] = c.gu8[4 * N + g] = (P.vm_policy == 0) ? VM_OD : VM_SPOT;
@@ -592,12 +598,13 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
           if (placed) {  // schedule(batch, slice): a free slot, the slice's FIFO, the busy union
             const int i = __ffsll((long long)~alive) - 1;
             const int p = gp[s];
+            // a slot's bit sits only in the mask of the slice its packed word names (masks are
+            // zeroed at replica start; a reset clears alive, not the masks)
+            msk[(ga_pk[i * 32] >> 24) & 7] &= ~(1ull << i);
             ga_en[i * 32] = bend;
-            ga_pk[i * 32] = (uint32_t)q | (strict ? 0u : (1u << 27));
+            ga_pk[i * 32] = (uint32_t)q | ((uint32_t)s << 24) | (strict ? 0u : (1u << 27));
             ga_fb[i * 32] = T.fbr[m * kNProf + p];
             alive |= 1ull << i;
-#pragma unroll
-            for (int z = 0; z < kZA; ++z) msk[z] &= ~(1ull << i);
             msk[s] |= 1ull << i;
             lsg[s] = bst;
             const int64_t bu = bug[s];
