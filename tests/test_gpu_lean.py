@@ -4,8 +4,8 @@ The lean path (a data-parallel candidate search ahead of a warp-per-replica chai
 its own pass) serves many-replica mode-R calls; PROTEAN_LEAN=2 makes small cases take it too.  Each
 test asserts the path was taken (the accounting pass reports a time) and compares every output
 element by element with the oracle: closed-form epochs scored by cand.cu, epochs with an
-unavailable GPU scored in the chain, units cand.cu cannot hold (a class above 12 batches,
-completions 2^25 us past the epoch start), and calls with an epoch above 96 batches, which go back
+unavailable GPU scored in the chain, units cand.cu cannot hold (a class above 10 batches,
+completions 2^25 us past the epoch start), and calls with an epoch above 64 batches, which go back
 to the fused engine."""
 import numpy as np
 import pytest
@@ -73,7 +73,7 @@ def test_lean_reconfig_heavy(oracle, monkeypatch):
 
 
 def test_lean_units_not_held(oracle, monkeypatch):
-    """Units cand.cu does not hold: a residue class above 12 batches (one sim-GPU, dense tiny
+    """Units cand.cu does not hold: a residue class above 10 batches (one sim-GPU, dense tiny
     batches) and completions beyond 2^25 us past the epoch start (solo times x 400)."""
     rng = np.random.default_rng(9)
     prof = random_profiles(rng, 3, max_batch=2)
@@ -88,10 +88,22 @@ def test_lean_units_not_held(oracle, monkeypatch):
 
 
 def test_lean_overflow_falls_back(oracle, monkeypatch):
-    """An epoch above 96 batches (Mix B x 8 on 8 sim-GPUs): the call goes back to the fused
+    """An epoch above 64 batches (Mix B x 8 on 8 sim-GPUs): the call goes back to the fused
     engine, with identical results."""
     gp = mix_b_params(1, seed=4, seconds=6, scale=8.0)
     tr = tick_trace(gp)
     P = synth_profiles()
     g = lean_replay(monkeypatch, P, tr, expect_lean=False, n_gpus=8)
     compare(g, oracle_replay(oracle, P, tr, n_gpus=8), 1)
+
+
+@pytest.mark.parametrize("W", [5_000, 40_000_000])
+def test_lean_epoch_length_extremes(oracle, monkeypatch, W):
+    """Epochs of 5 ms (most batches straddle epochs: the cursor walk's epoch fill) and of 40 s
+    (ready times up to 2^25 us past the epoch start: every unit falls back from 32-bit time)."""
+    rng = np.random.default_rng(31 + W % 7)
+    prof = random_profiles(rng, 3, small_time=W < 100_000)
+    tr = uniform_trace(rng, 3, 3, 80_000_000 if W > 1_000_000 else 400_000, 60 if W > 1_000_000 else 300)
+    cfg = dict(n_gpus=4, epoch_len_us=W, reconfig_us=W // 2, wait_limit=1)
+    g = lean_replay(monkeypatch, prof, tr, **cfg)
+    compare(g, oracle_replay(oracle, prof, tr, **cfg), 3)
