@@ -107,3 +107,19 @@ def test_lean_epoch_length_extremes(oracle, monkeypatch, W):
     cfg = dict(n_gpus=4, epoch_len_us=W, reconfig_us=W // 2, wait_limit=1)
     g = lean_replay(monkeypatch, prof, tr, **cfg)
     compare(g, oracle_replay(oracle, prof, tr, **cfg), 3)
+
+
+@pytest.mark.parametrize("case", ["arrivals_and_ready_at_epoch_starts", "fbr_sum_exactly_one",
+                                  "ready_exactly_at_reconfiguration_end", "revocation_at_and_inside_epochs",
+                                  "epochs_shorter_than_batch_timeouts"])
+def test_lean_targeted_edges(oracle, monkeypatch, case):
+    """tests/test_gpu_edges.py's targeted edges (each asserts its edge occurs) on the lean path."""
+    import test_gpu_edges as edges
+    monkeypatch.setenv("PROTEAN_LEAN", "2")
+    fn = getattr(edges, "test_" + case)
+    if case == "revocation_at_and_inside_epochs":
+        fn(oracle, 2.5, 2)
+    elif case == "epochs_shorter_than_batch_timeouts":
+        fn(oracle, 0)
+    else:
+        fn(oracle)
