@@ -167,7 +167,8 @@ __device__ int64_t score_idle(const Tab& T, int j, int cur, const UnitBats& U, c
 // then takes score_idle.
 __device__ bool score_idle32(const Tab& T, int j, int cur, const UnitBats& U, const uint8_t* gl, int cnt,
                              const uint32_t* sa_r, int max_live, uint32_t eW32, int64_t eW, uint32_t* en,
-                             uint32_t* pk, int32_t* fb, uint32_t* lsm, int64_t* key_out) {
+                             uint32_t* pk, int32_t* fb, uint32_t* lsm, const uint8_t* fitm, int M,
+                             int64_t* key_out) {
   constexpr int L = 32;
   if (cnt > 32) return false;
   const int ns = T.gn[j];
@@ -201,12 +202,12 @@ __device__ bool score_idle32(const Tab& T, int j, int cur, const UnitBats& U, co
     const int32_t* fbr_m = T.fbr + m * kNProf;
     const int32_t* solo_m = T.solo + m * kNProf;
     uint32_t best = 0xFFFFFFFFu, bst = 0, bc = 0;
-    const int nsx = __popc(alive) < max_live ? ns : 0;
+    const uint32_t sflag = strict ? 0xFFFFFFFFu : 0u;
 #pragma unroll 1
-    for (int s = 0; s < nsx; ++s) {
+    for (uint32_t fit = __popc(alive) < max_live ? (uint32_t)fitm[j * M + m] : 0u; fit; fit &= fit - 1) {
+      const int s = __ffs(fit) - 1;
       const int p = gp[s];
       const int32_t Ms = T.cap[p];
-      if (q > Ms) continue;
       const uint32_t lss = lsm[(2 * s) * L];
       const uint32_t t0 = rt > lss ? rt : lss;
       const uint32_t set = lsm[(2 * s + 1) * L] & alive;
@@ -245,19 +246,21 @@ __device__ bool score_idle32(const Tab& T, int j, int cur, const UnitBats& U, co
           if (en[i * L] > start) F += (uint32_t)fb[i * L];
         }
       }
+      // completions clamp to 2^25 - 1 in the key; a clamped winner sends the GPU to score_idle
       const int32_t so = solo_m[p];
       const int64_t ex = F <= (uint32_t)kPpm ? (int64_t)so : exec_time(so, F);
-      const uint32_t cc = start + (uint32_t)ex;
-      wide |= (ex | (int64_t)cc) >= (1 << 25);
-      const uint32_t key = strict
-          ? ((be >= gpref[s]) ? 0x80000000u : 0u) | (cc << 6) | ((uint32_t)(4 - p) << 3) | (uint32_t)s
-          : (start << 3) | (uint32_t)s;
+      const uint32_t cc = ex >= (1 << 25) ? (1u << 25) : min(start + (uint32_t)ex, 1u << 25);
+      const uint32_t ks = ((be >= gpref[s]) ? 0x80000000u : 0u) | (min(cc, (1u << 25) - 1u) << 6) |
+                          ((uint32_t)(4 - p) << 3) | (uint32_t)s;
+      const uint32_t kb = (start << 3) | (uint32_t)s;
+      const uint32_t key = (ks & sflag) | (kb & ~sflag);
       if (key < best) {
         best = key;
         bst = start;
         bc = cc;
       }
     }
+    wide |= best != 0xFFFFFFFFu && bc >= (1u << 25) - 1u;
     if (wide) return false;
     const bool placed = best != 0xFFFFFFFFu;
     const int bsl = best & 7;
@@ -655,7 +658,7 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
           if (c.gu8[5 * N + g]) {
             const int cur = c.gu8[0 * N + g], x0 = c.g_off[g], cnt = c.g_off[g + 1] - x0;
             if (!score_idle32(T, j, cur, U, gl + x0, cnt, sa_r, P.max_live, (uint32_t)eW, eW,
-                              sc_en32, sc_pk, sc_fb, sc_ls, &key))
+                              sc_en32, sc_pk, sc_fb, sc_ls, fitm, CL.M, &key))
               key = score_idle(T, j, cur, U, gl + x0, cnt, sa_r, P.max_live, sc_en, sc_pk, sc_fb);
           }
           kst[pi] = key;  // by GPU
