@@ -210,7 +210,16 @@ __global__ void __launch_bounds__(32 * kCandWarps) cand_kernel(CandParams P) {
         if (T0.mem[m] <= T0.cap[T0.gprof[j * 8 + s]]) f |= 1u << s;
       fitm[i] = (uint8_t)f;
     }
+#pragma unroll 1
+    for (int i = tid; i < P.tl.G * kNProf; i += blockDim.x) {  // pmask[j][p]: slices of profile p
+      const int j = i / kNProf, pp = i % kNProf;
+      uint32_t f = 0;
+      for (int s = 0; s < T0.gn[j]; ++s)
+        if (T0.gprof[j * 8 + s] == pp) f |= 1u << s;
+      fitm[P.tl.G * P.tl.M + i] = (uint8_t)f;
+    }
   }
+  const uint8_t* pmask = fitm + P.tl.G * P.tl.M;
   WarpSmem& ws = reinterpret_cast<WarpSmem*>(smem + P.ws_off)[warp];
   __syncthreads();
   Tab T;
@@ -375,13 +384,16 @@ __global__ void __launch_bounds__(32 * kCandWarps) cand_kernel(CandParams P) {
         const bool strict = (info >> 24) & 1;
         const uint32_t rt = ws.ready[b] - (uint32_t)eW;  // ready - eW in [0, W); ready order
         // residents that ended by rt never matter again (ready times ascend along the class)
+        uint32_t occ = 0;  // slices with a resident still running at rt
 #pragma unroll 1
         for (uint32_t a = alive; a; a &= a - 1) {
           const int i = __ffs(a) - 1;
+          const uint32_t pki = ws.pk[i][lane];
           if (ws.en[i][lane] <= rt) {
             alive &= ~(1u << i);
-            const uint32_t pki = ws.pk[i][lane];
             if (pki >> 27) be -= (int)(pki & kMemMask);
+          } else {
+            occ |= 1u << ((pki >> 24) & 7);
           }
         }
         const int32_t q = T.mem[m];
@@ -393,6 +405,27 @@ __global__ void __launch_bounds__(32 * kCandWarps) cand_kernel(CandParams P) {
         uint32_t bst = 0, bc = 0;
         // the slices of j that hold the batch's footprint (q <= Ms), none without room (Q39)
         uint32_t fit = __popc(alive) < P.max_live ? (uint32_t)fitm[j * M + m] : 0u;
+        // An idle slice (no resident running at rt; its last start is below rt) starts the batch
+        // at rt alone: exec = solo (F = its own FBR <= 10^6), so idle slices of one profile tie on
+        // completion and differ only in the tag bit and the position.  Only the lowest of them --
+        // and, for a strict batch, the lowest one past the tag walk's threshold (pref[s] > be,
+        // pref ascending in s) -- can hold the minimum key: the rest are dropped unevaluated.
+        if (const uint32_t idle = fit & ~occ) {
+          uint32_t elig = 0;
+          if (strict) {
+#pragma unroll 1
+            for (int s = 0; s < kMaxSl && !elig; ++s)
+              if (s < ns && gpref[s] > be) elig = ~((1u << s) - 1u);
+          }
+          uint32_t keep = 0;
+#pragma unroll
+          for (int pp = 0; pp < kNProf; ++pp) {
+            const uint32_t ip = idle & pmask[j * kNProf + pp];
+            const uint32_t ie = ip & elig;
+            keep |= (ip & (0u - ip)) | (ie & (0u - ie));
+          }
+          fit = (fit & occ) | keep;
+        }
         const uint32_t sflag = strict ? 0xFFFFFFFFu : 0u;
 #pragma unroll 1
         for (; fit; fit &= fit - 1) {
@@ -436,7 +469,7 @@ __global__ void __launch_bounds__(32 * kCandWarps) cand_kernel(CandParams P) {
         const int bsl = best & 7;
         const bool placed = best != 0xFFFFFFFFu;
         ws.en[x][lane] = placed ? bc : 0u;
-        ws.pk[x][lane] = (uint32_t)q | (strict ? 0u : (1u << 27));
+        ws.pk[x][lane] = (uint32_t)q | ((uint32_t)bsl << 24) | (strict ? 0u : (1u << 27));
         ws.fb[x][lane] = fbr_m[gp[bsl]];
         if (placed) {
           ws.ls[bsl][lane] = bst;
@@ -472,7 +505,7 @@ __global__ void __launch_bounds__(32 * kCandWarps) cand_kernel(CandParams P) {
 
 size_t cand_smem_bytes(const TabLayout& tl, size_t* ws_off) {
   const size_t o = (((size_t)tl.words * 4 + 15) & ~(size_t)15) + (((size_t)tl.G + 15) & ~(size_t)15) +
-                   (((size_t)tl.G * tl.M + 15) & ~(size_t)15);
+                   (((size_t)tl.G * tl.M + (size_t)tl.G * kNProf + 15) & ~(size_t)15);
   *ws_off = o;
   return o + sizeof(WarpSmem) * kCandWarps;
 }
