@@ -8,23 +8,28 @@
 // when the chain reaches the epoch -- decides which GPU a class lands on.  The search is therefore
 // a data-parallel pass over (replica, epoch) units ahead of the chain:
 //
-//   walk_kernel   thread per (replica, stream): O3 batch formation (reading Q14) is a
+//   walk_kernel   warp per (replica, stream): O3 batch formation (reading Q14) is a
 //                 greedy chain along the stream -- close at B requests or at the first arrival + T
 //                 -- whose batches have non-decreasing ready times, so the chain kernel's stream
 //                 cursor at the start of epoch e is the first batch start whose ready time is
-//                 >= eW.  Records it as bstart[r][k][e] (e = 0..E).
-//   cand_kernel   warp per (replica, epoch): forms the epoch's batches from bstart (lanes over
-//                 streams), ranks them into id order (ready, strict first, model, position), and
-//                 scores every (residue class, geometry) pair with one lane each -- Alg 1 (P:L251-
-//                 277) under Eq 1 / Eq 2 over the class's batches from idle, the
-//                 lane walking its geometry's slices itself (no shuffles) -- then the O8 key
-//                 (misses << 40 | BE tail << 8 | tag j + 1; the chain re-tags the GPU's current
-//                 geometry with 0).  Writes kfc[r][e][class][j].  A unit it cannot hold (more
-//                 than kBC batches, more than kKC in a class, a completion 2^32 us past eW) is
-//                 marked with kfc[r][e][0][0] = INT64_MIN and the chain scores that epoch itself.
+//                 >= eW (DESIGN F1).  Lanes test 32 consecutive full batches per load round.
+//                 Records bstart[r][k][e] (e = 0..E).
+//   cand_kernel   warp per (replica, epoch): forms the epoch's batches from bstart (the warp on one
+//                 active stream at a time, 32 batches per round), ranks them into id order (ready,
+//                 strict first, model, position), writes the rows (UnitBats) for the chain and the
+//                 accounting pass, and scores every (residue class, geometry) pair with one lane
+//                 each -- Alg 1 under Eq 1 / Eq 2 over the class's
+//                 batches from idle in 32-bit time relative to eW, the lane walking its geometry's
+//                 fitting slices itself (bit masks of the batches placed per slice, dominated idle
+//                 slices dropped) -- then the O8 key (misses << 40 | BE tail << 8 | tag j + 1; the
+//                 chain re-tags the GPU's current geometry with 0).  Writes kfc[r][e][class][j].  A
+//                 unit it cannot hold (more than kBC = 64 batches: the whole call goes back to the
+//                 fused engine; more than kKC = 10 in a class, or a completion 2^25 us past eW: that
+//                 epoch is scored in the chain) is marked with kfc[r][e][0][0] = INT64_MIN.
 //
-// The chain (replay.cu) uses the keys for every epoch whose dispatch is the closed form; an epoch
-// with a GPU unavailable inside it (reconfiguration window, VM change) keeps its in-kernel units.
+// The chain (chain.cu, or the fused replay.cu) uses the keys for every epoch whose dispatch is the
+// closed form; an epoch with a GPU unavailable inside it (reconfiguration window, VM change) is
+// scored in the chain.
 #include <cuda_runtime.h>
 #include <stdint.h>
 

@@ -10,17 +10,19 @@
 //
 //   chain_kernel  warp per replica.  Per epoch: A (lane = GPU), the epoch's batch rows (cand.cu,
 //                 prefetched one epoch ahead with cp.async), D (closed form when every GPU is
-//                 available, else the plain round robin on lane 0), E (the fused engine's
-//                 lane-per-slice placement units, four GPUs per pass), G (lane = GPU).  The
-//                 candidate keys come from cand.cu for closed-form epochs (rotated by the cursor);
-//                 other epochs are scored here, one lane per (GPU, geometry), Alg 1 from idle in
-//                 64-bit time.  Each batch's outcome goes to HBM for the accounting pass.
+//                 available, else a ballot over availability per batch), E (lane = GPU: Alg 1 over
+//                 the GPU's 64 resident slots -- alive and per-slice masks; the per-slice FIFO keeps
+//                 every resident's start <= t0, so only ends, footprints and co-runner FBRs are
+//                 stored), G (lane = GPU).  The candidate keys come from cand.cu for closed-form
+//                 epochs (rotated by the cursor); other epochs are scored here, one lane per (GPU,
+//                 geometry), Alg 1 from idle (32-bit time, 64-bit fallback).  Each batch's outcome
+//                 goes to HBM for the accounting pass.
 //   acct_kernel   CTA per replica: per-request latencies end - arrival of every placed batch (O7),
 //                 log-linear histograms in shared memory, SLO hits, arrival / drop counters, then
 //                 the nearest-rank P50 / P99 (O12) -- the fused engine's phase F and finalize.
 //
 // Both produce exactly the fused engine's outputs (replay.cu); the host takes this path for mode R,
-// policy 0 or 1, no container pools, N <= 32 (api.cu).
+// policy 0, no container pools, N <= 32, N * G even, max_live <= 64 (api.cu).
 #include <cuda_runtime.h>
 #include <stdint.h>
 
