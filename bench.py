@@ -443,7 +443,9 @@ def run_ours(args):
                          "passes_before_replay_ms": p_ms},
             "search_self_check": h5,
             "cpu_baseline": cpu, "e2e": e2e,
-            "gpu_launches": (5 + (2 if s_ms > 0 else 0) + (1 if lean else 0)) * args.steps * world,
+            # per step: roff_scan, prepass, P1, P2, P3 (5) + walk, cand (search) + chain, acct
+            # (lean) or the fused replay_kernel -- as the committed ncu launch list shows
+            "gpu_launches": (5 + (2 if s_ms > 0 else 0) + (2 if lean else 1)) * args.steps * world,
             "clocks": clocks,
         }
         print(json.dumps(line), flush=True)
@@ -770,7 +772,7 @@ def run_single(args, name):
             "slot_evals_per_s": float(c[8]) / (ms / 1e3),
             "simulated_requests_per_s": float(c[0] + c[4]) / (ms / 1e3),
             "strict_slo_compliance": float(c[1]) / max(float(c[0]), 1.0),
-            "cpu_baseline": cpu, "gpu_launches": 5 * args.steps}
+            "cpu_baseline": cpu, "gpu_launches": 6 * args.steps}  # partition (5) + the fused replay_kernel
     print(json.dumps(line), flush=True)
     return 0
 
