@@ -341,9 +341,8 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
   const int gw = blockIdx.x * kChainWarps + warp;  // this warp's scratch slot
   char* slot = P.scratch + (size_t)gw * P.slot_bytes;
   // the actual residents of GPU lane: 64 slots, lane-interleaved (slot i of lane l at i * 32 + l)
-  int64_t* ga_en = reinterpret_cast<int64_t*>(slot + P.o_alist) + lane;
-  uint32_t* ga_pk = reinterpret_cast<uint32_t*>(slot + P.o_alist + 64 * 32 * 8) + lane;
-  int32_t* ga_fb = reinterpret_cast<int32_t*>(slot + P.o_alist + 64 * 32 * 12) + lane;
+  // ga[i * 32]: end; ga[(64 + i) * 32]: packed word | co-runner FBR << 32 (one live base pointer)
+  int64_t* ga = reinterpret_cast<int64_t*>(slot + P.o_alist) + lane;
   // fitm[j][m]: the slice positions of geometry j that hold model m's footprint (CTA-wide table)
   const uint8_t* fitm = smem + (((size_t)P.tl.words * 4 + 15) & ~(size_t)15) + (size_t)kChainWarps * CL.total;
   int64_t* sc_en = reinterpret_cast<int64_t*>(slot + P.o_clist) + lane;  // score_idle arrays
@@ -366,7 +365,7 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
 #pragma unroll 1
     for (int i = lane; i < 64; i += 32)  // every slot's packed word names slice 0 (no stale bits)
       for (int g = 0; g < N; ++g)
-        reinterpret_cast<uint32_t*>(slot + P.o_alist + 64 * 32 * 8)[i * 32 + g] = 0;
+        reinterpret_cast<int64_t*>(slot + P.o_alist)[(64 + i) * 32 + g] = 0;
 #pragma unroll 1
     for (int g = lane; g < N; g += 32) {
       reset_gpu_state(c, g, P.init_geom);
@@ -535,10 +534,10 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
 #pragma unroll 1
           for (uint64_t a = alive; a; a &= a - 1) {  // residents ended by t never matter again
             const int i = __ffsll((long long)a) - 1;
-            if (ga_en[i * 32] <= t) {
+            if (ga[i * 32] <= t) {
               alive &= ~(1ull << i);
             } else {
-              const uint32_t pki = ga_pk[i * 32];
+              const uint32_t pki = (uint32_t)ga[(64 + i) * 32];
               if (pki >> 27) be += (int)(pki & kMemMask);
             }
           }
@@ -558,9 +557,10 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
 #pragma unroll 1
             for (uint64_t a = set; a; a &= a - 1) {
               const int i = __ffsll((long long)a) - 1;
-              if (ga_en[i * 32] > t0) {
-                used += (int32_t)(ga_pk[i * 32] & kMemMask);
-                F += ga_fb[i * 32];
+              if (ga[i * 32] > t0) {
+                const uint64_t pf = (uint64_t)ga[(64 + i) * 32];
+                used += (int32_t)((uint32_t)pf & kMemMask);
+                F += (int32_t)(pf >> 32);
               }
             }
             int64_t start = t0;
@@ -571,13 +571,13 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
                 int64_t nxt = INT64_MAX;
                 int32_t rem = 0;
                 for (uint64_t a = set; a; a &= a - 1) {
-                  const int64_t ei = ga_en[(__ffsll((long long)a) - 1) * 32];
+                  const int64_t ei = ga[(__ffsll((long long)a) - 1) * 32];
                   if (ei > ev && ei < nxt) nxt = ei;
                 }
                 ev = nxt;
                 for (uint64_t a = set; a; a &= a - 1) {
                   const int i = __ffsll((long long)a) - 1;
-                  if (ga_en[i * 32] > ev) rem += (int32_t)(ga_pk[i * 32] & kMemMask);
+                  if (ga[i * 32] > ev) rem += (int32_t)((uint32_t)ga[(64 + i) * 32] & kMemMask);
                 }
                 if (rem + q <= Ms) break;
               }
@@ -585,7 +585,7 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
               F = T.fbr[m * kNProf + p];
               for (uint64_t a = set; a; a &= a - 1) {
                 const int i = __ffsll((long long)a) - 1;
-                if (ga_en[i * 32] > start) F += ga_fb[i * 32];
+                if (ga[i * 32] > start) F += (int32_t)((uint64_t)ga[(64 + i) * 32] >> 32);
               }
             }
             const int64_t cc = start + exec_time(T.solo[m * kNProf + p], F);
@@ -605,10 +605,10 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
             const int p = gp[s];
             // a slot's bit sits only in the mask of the slice its packed word names (masks are
             // zeroed at replica start; a reset clears alive, not the masks)
-            msk[(ga_pk[i * 32] >> 24) & 7] &= ~(1ull << i);
-            ga_en[i * 32] = bend;
-            ga_pk[i * 32] = (uint32_t)q | ((uint32_t)s << 24) | (strict ? 0u : (1u << 27));
-            ga_fb[i * 32] = T.fbr[m * kNProf + p];
+            msk[((uint32_t)ga[(64 + i) * 32] >> 24) & 7] &= ~(1ull << i);
+            ga[i * 32] = bend;
+            ga[(64 + i) * 32] = (int64_t)((uint64_t)((uint32_t)q | ((uint32_t)s << 24) | (strict ? 0u : (1u << 27))) |
+                                          ((uint64_t)(uint32_t)T.fbr[m * kNProf + p] << 32));
             alive |= 1ull << i;
             msk[s] |= 1ull << i;
             lsg[s] = bst;
@@ -640,7 +640,7 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
         *alive_p = alive;
         int64_t mx = 0;  // the latest end among the GPU's residents (drain end of a reconfiguration)
         for (uint64_t a = alive; a; a &= a - 1) {
-          const int64_t ei = ga_en[(__ffsll((long long)a) - 1) * 32];
+          const int64_t ei = ga[(__ffsll((long long)a) - 1) * 32];
           mx = ei > mx ? ei : mx;
         }
         c.gi[5 * N + g] = mx;
