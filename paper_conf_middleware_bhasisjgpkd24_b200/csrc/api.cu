@@ -829,10 +829,12 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   const int block = 32 * (few_r ? PROTEAN_FEW_WARPS : kWarps);
   // the candidate search as a data-parallel pass ahead of the chain (cand.cu): mode R, policy 0,
   // one CTA per replica, the one-warp decision path (N <= 32)
-  bool precand = c.policy == 0 && !modeG && vr_n == 1 && N <= 32;
+  // (policy 2 runs the search pass for its batch rows only, and only to feed the lean chain)
+  bool precand = (c.policy == 0 || c.policy == 2) && !modeG && vr_n == 1 && N <= 32;
+  const bool keys = c.policy == 0;
   if (const char* ev = std::getenv("PROTEAN_PRECAND"))  // experiment knob: 0 = in-chain candidates only
     if (std::atoi(ev) == 0) precand = false;
-  const int KS = precand ? N * h->G : 0;
+  const int KS = precand && keys ? N * h->G : 0;
   SmemLayout sl;
   sl.init(h->tl.words, h->M, N, Gc, CW, 0, 0, KS);
   const size_t fixed = sl.total;
@@ -989,15 +991,16 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   bool lean = precand && (!few_r || lean_force) && c.cold_start_us == 0 && (N * h->G) % 2 == 0 &&
               c.max_live <= 64;  // the chain's resident slots: 64-bit masks
   if (lean_env && std::atoi(lean_env) == 0) lean = false;  // experiment knob: 0 = the fused engine
+  if (!keys && !lean) precand = false;  // Alg 2 on the fused engine forms its own batches
   size_t b_ub = 0, b_br = 0;
   if (precand) {
-    const size_t b_bs = al((size_t)R * S * (E + 1) * 4), b_kf = al((size_t)R * E * N * h->G * 8);
+    const size_t b_bs = al((size_t)R * S * (E + 1) * 4), b_kf = keys ? al((size_t)R * E * N * h->G * 8) : 0;
     if (lean) {
       b_ub = al((size_t)R * E * sizeof(UnitBats));
       b_br = al((size_t)R * E * kUnitBats * 8);
     }
     int rc = ensure(h, &h->d_cand, &h->cand_bytes, b_bs + b_kf + b_ub + b_br, st);
-    if (rc == PROTEAN_ENOMEM && lean) {  // without the lean chain's rows: the search alone
+    if (rc == PROTEAN_ENOMEM && lean && keys) {  // without the lean chain's rows: the search alone
       lean = false;
       b_ub = b_br = 0;
       rc = ensure(h, &h->d_cand, &h->cand_bytes, b_bs + b_kf, st);
@@ -1010,7 +1013,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
     }
   }
   if (precand) {
-    const size_t b_bs = al((size_t)R * S * (E + 1) * 4), b_kf = al((size_t)R * E * N * h->G * 8);
+    const size_t b_bs = al((size_t)R * S * (E + 1) * 4), b_kf = keys ? al((size_t)R * E * N * h->G * 8) : 0;
     CandParams Q;
     std::memset(&Q, 0, sizeof(Q));
     Q.tab = h->d_tab;
@@ -1019,7 +1022,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
     Q.saoff = P.saoff;
     Q.sidx = P.sidx;
     Q.bstart = static_cast<uint32_t*>(h->d_cand);
-    Q.kfc = reinterpret_cast<int64_t*>(static_cast<char*>(h->d_cand) + b_bs);
+    Q.kfc = keys ? reinterpret_cast<int64_t*>(static_cast<char*>(h->d_cand) + b_bs) : nullptr;
     Q.gorder = h->d_gorder;
     if (lean) {
       Q.ub = reinterpret_cast<UnitBats*>(static_cast<char*>(h->d_cand) + b_bs + b_kf);

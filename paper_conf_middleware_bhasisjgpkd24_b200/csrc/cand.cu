@@ -241,7 +241,7 @@ __global__ void __launch_bounds__(32 * kCandWarps) cand_kernel(CandParams P) {
     const int64_t eW = e * W;
     const int64_t sbase = P.saoff[r];
     const uint32_t* sa = P.sa + sbase;
-    int64_t* kout = P.kfc + (size_t)u * N * G;
+    int64_t* kout = P.kfc ? P.kfc + (size_t)u * N * G : nullptr;  // NULL: rows only (policy 2)
     if (lane == 0) {
       ws.nb = 0;
       ws.bad = 0;
@@ -338,7 +338,7 @@ __global__ void __launch_bounds__(32 * kCandWarps) cand_kernel(CandParams P) {
     if (ubu && lane == 0) ubu->nb = (uint32_t)nb;
     if (nb > kBC) {  // the chain scores this epoch itself (the lean chain cannot hold it)
       if (lane == 0) {
-        kout[0] = INT64_MIN;
+        if (kout) kout[0] = INT64_MIN;
         if (P.overflow) atomicOr(P.overflow, 1);
       }
       __syncwarp();
@@ -359,6 +359,7 @@ __global__ void __launch_bounds__(32 * kCandWarps) cand_kernel(CandParams P) {
       }
     }
     __syncwarp();
+    if (!kout) continue;  // rows only: no candidate keys (Alg 2's heuristic decides, policy 2)
     // ---- candidates: lane per (residue class c, geometry j), Alg 1 from idle
     bool bad = false, wide = false;
 #pragma unroll 1

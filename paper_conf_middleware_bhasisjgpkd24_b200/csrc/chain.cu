@@ -22,7 +22,8 @@
 //                 the nearest-rank P50 / P99 (O12) -- the fused engine's phase F and finalize.
 //
 // Both produce exactly the fused engine's outputs (replay.cu); the host takes this path for mode R,
-// policy 0, no container pools, N <= 32, N * G even, max_live <= 64 (api.cu).
+// policy 0 (keys from cand.cu) or 2 (Alg 2's heuristic in G; cand.cu forms rows only), no container
+// pools, N <= 32, N * G even, max_live <= 64 (api.cu).
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -679,28 +680,50 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
           uint8_t dec_out = kNoGeom;
           if (P.policy != 1 && c.gu8[5 * N + g]) {
             const int cur = c.gu8[0 * N + g];
-            int cl = g;  // keys by GPU (scored here) or by residue class (cand.cu)
-            if (pre) {
-              cl = g - cur0;
-              cl = cl < 0 ? cl + N : cl;
-            }
-            const int64_t* kr = kst + cl * G;
-#pragma unroll 1
-            for (int v = 0; v < G; ++v) {
-              int64_t kv = kr[v];
-              if (v == cur) {
-                if (pre) kv &= ~(int64_t)255;  // tag 0: the current geometry (O8, Q20)
-                kc = kv;
+            int best;
+            if (P.policy == 0) {  // S8: argmin over the candidate keys
+              int cl = g;  // keys by GPU (scored here) or by residue class (cand.cu)
+              if (pre) {
+                cl = g - cur0;
+                cl = cl < 0 ? cl + N : cl;
               }
-              kb = kv < kb ? kv : kb;
-              if (P.cand_keys) P.cand_keys[(((size_t)r * E + e) * N + g) * (size_t)G + v] = kv;
+              const int64_t* kr = kst + cl * G;
+#pragma unroll 1
+              for (int v = 0; v < G; ++v) {
+                int64_t kv = kr[v];
+                if (v == cur) {
+                  if (pre) kv &= ~(int64_t)255;  // tag 0: the current geometry (O8, Q20)
+                  kc = kv;
+                }
+                kb = kv < kb ? kv : kb;
+                if (P.cand_keys) P.cand_keys[(((size_t)r * E + e) * N + g) * (size_t)G + v] = kv;
+              }
+              c.gi[6 * N + g] = kb;
+              c.gi[7 * N + g] = kc;
+              const int tag = (int)(kb & 255);
+              best = tag == 0 ? cur : tag - 1;
+              scored_b = (uint32_t)(c.g_off[g + 1] - c.g_off[g]);
+              scored = true;
+            } else {  // policy 2: Alg 2's own heuristic (N1, readings R10-R15)
+              int64_t be_num = 0, be_mem = 0;  // line 2: the BE batches dispatched to g (R10)
+#pragma unroll 1
+              for (int x = c.g_off[g]; x < c.g_off[g + 1]; ++x) {
+                const uint32_t info = U.info[gl[x]];
+                if ((info >> 24) & 1u) continue;
+                be_num += 1;
+                be_mem += T.mem[(info >> 16) & 0xFFu];  // footprint per batch (Q36)
+              }
+              const int64_t a = P.ewma_a;  // lines 8-9: EWMA in milli-units (R11)
+              const int64_t X = (a * 1000 * be_num + (1000 - a) * c.gi[12 * N + g]) / 1000;
+              const int64_t Y = (a * 1000 * be_mem + (1000 - a) * c.gi[13 * N + g]) / 1000;
+              c.gi[12 * N + g] = X;
+              c.gi[13 * N + g] = Y;
+              // lines 10-18: the first of [[1g,2g],[3g]] whose summed capacity holds pred_BE_mem
+              const bool fits12 = (int64_t)(T.cap[0] + T.cap[1]) * 1000 >= Y;
+              const bool found = fits12 || (int64_t)T.cap[2] * 1000 >= Y;
+              // lines 19-23: thresholds on pred_BE_num (R13, R14), (4g,3g) fallback, + 4g (R15)
+              best = (!found || X < P.t_low || X > P.t_high) ? P.g43 : (fits12 ? P.g421 : P.g43);
             }
-            c.gi[6 * N + g] = kb;
-            c.gi[7 * N + g] = kc;
-            const int tag = (int)(kb & 255);
-            const int best = tag == 0 ? cur : tag - 1;
-            scored_b = (uint32_t)(c.g_off[g + 1] - c.g_off[g]);
-            scored = true;
             dec_out = (uint8_t)best;
             c.gu8[6 * N + g] = (uint8_t)best;
             if (best != cur) {  // Alg 2 lines 24-30 (Q22)

@@ -123,3 +123,22 @@ def test_lean_targeted_edges(oracle, monkeypatch, case):
         fn(oracle, 0)
     else:
         fn(oracle)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_lean_alg2_policy(oracle, monkeypatch, seed):
+    """Alg 2's own heuristic (policy 2, N1) on the lean path: the search pass forms and ranks the
+    epoch's batches without scoring candidates; the chain's decision step runs the heuristic."""
+    rng = np.random.default_rng(950 + seed)
+    if seed < 2:
+        gp = mix_a_params(2, seed=20 + seed, seconds=30)
+        tr, P, N = tick_trace(gp), synth_profiles(), 8
+    else:
+        M = int(rng.integers(2, 6))
+        P = random_profiles(rng, M)
+        tr = uniform_trace(rng, 3, M, 8_000_000, 200)  # <= 64 batches per epoch: the lean chain
+        N = int(rng.choice([2, 4]))
+    cfg = dict(n_gpus=N, policy=2, wait_limit=int(rng.integers(0, 3)), ewma_alpha_pm=int(rng.integers(100, 900)),
+               t_low_milli=int(rng.integers(0, 2000)), t_high_milli=int(rng.integers(2000, 8000)))
+    g = lean_replay(monkeypatch, P, tr, **cfg)
+    compare(g, oracle_replay(oracle, P, tr, **cfg), tr.n_replicas)
