@@ -986,9 +986,9 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
   h->t_search = 0.f;
   h->t_acct = 0.f;
   // the lean chain (chain.cu): a warp per replica on cand.cu's batch rows and keys, accounting in
-  // its own pass; many-replica calls without container pools (an epoch with more than 96 batches
-  // sends the call back to the fused engine below)
-  bool lean = precand && (!few_r || lean_force) && c.cold_start_us == 0 && (N * h->G) % 2 == 0 &&
+  // its own pass; many-replica calls, container pools (N3) included (an epoch with more than 64
+  // batches sends the call back to the fused engine below)
+  bool lean = precand && (!few_r || lean_force) && (N * h->G) % 2 == 0 &&
               c.max_live <= 64;  // the chain's resident slots: 64-bit masks
   if (lean_env && std::atoi(lean_env) == 0) lean = false;  // experiment knob: 0 = the fused engine
   if (!keys && !lean) precand = false;  // Alg 2 on the fused engine forms its own batches
@@ -1057,7 +1057,8 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
     const size_t sl_a = al((size_t)64 * 32 * 16), sl_c = al((size_t)kUnitBats * 32 * 16 + 2 * kMaxSl * 32 * 4);
     PL.o_alist = 0;
     PL.o_clist = sl_a;
-    PL.slot_bytes = sl_a + sl_c;
+    PL.o_pool = sl_a + sl_c;  // N3 pools: busy-until [N][M][kPoolCap] int64, size + counter [N][M] int32
+    PL.slot_bytes = sl_a + sl_c + (c.cold_start_us > 0 ? al((size_t)N * h->M * (kPoolCap * 8 + 8)) : 0);
     CK(h, chain_occupancy(PL, &cper));
     if (cper < 1) return fail(h, PROTEAN_ERANGE, "chain kernel does not fit an SM");
     const int cgrid = (int)std::min<int64_t>((int64_t)h->nsm * cper, ((int64_t)R + 3) / 4);
@@ -1085,6 +1086,7 @@ int protean_replay_traces(protean_handle* h, const protean_replay_cfg* cfg, prot
     CK(h, cudaMemcpyAsync(herr3, d_err, 16, cudaMemcpyDeviceToHost, st));
     CK(h, cudaStreamSynchronize(st));
     if (!herr3[3]) {  // every epoch fitted the chain's batch rows
+      if (herr3[2]) return fail(h, PROTEAN_ERANGE, "a container pool outgrew 128 containers (N3)");
       float a = 0.f, b = 0.f;
       CK(h, cudaEventElapsedTime(&a, h->ev[0], h->ev[1]));
       CK(h, cudaEventElapsedTime(&b, h->ev[4], h->ev[5]));

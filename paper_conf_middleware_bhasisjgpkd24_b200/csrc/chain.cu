@@ -295,6 +295,64 @@ __device__ bool score_idle32(const Tab& T, int j, int cur, const UnitBats& U, co
   return true;
 }
 
+// ---- N3 container pools on the lean chain (readings R22-R27), lane = sim-GPU:
+// per (GPU, model) busy-until [kPoolCap] int64, size and surplus counter int32, in the warp's slot.
+struct LanePools {
+  int64_t* bu;
+  int32_t* sz;
+  int32_t* ctr;
+  int M;
+  __device__ __forceinline__ size_t pm(int g, int m) const { return (size_t)g * M + m; }
+};
+__device__ __forceinline__ void lane_pool_reset(const ReplayParams& P, const LanePools& pl, int g) {  // R22
+  for (int m = 0; m < pl.M; ++m) {
+    for (int i = 0; i < P.prewarm; ++i) pl.bu[pl.pm(g, m) * kPoolCap + i] = 0;
+    pl.sz[pl.pm(g, m)] = P.prewarm;
+    pl.ctr[pl.pm(g, m)] = 0;
+  }
+}
+// R23: the first container of (g, m) idle at t, else a new one after a cold start (t + cold_us).
+__device__ __forceinline__ int lane_pool_acquire(const ReplayParams& P, const LanePools& pl, int g, int m,
+                                                 int64_t t, int64_t* t_eff, unsigned long long* cold) {
+  const size_t k = pl.pm(g, m);
+  const int64_t* b = pl.bu + k * kPoolCap;
+  const int n = pl.sz[k];
+  *t_eff = t;
+#pragma unroll 1
+  for (int i = 0; i < n; ++i)
+    if (b[i] <= t) return i;
+  *t_eff = t + P.cold_us;  // reactive scale-up
+  *cold += 1;
+  if (n >= kPoolCap) {
+    atomicOr(&P.err[2], 1);
+    return -1;
+  }
+  pl.bu[k * kPoolCap + n] = t;
+  pl.sz[k] = n + 1;
+  return n;
+}
+// R26: pools larger than the epoch's batch count for keepalive epochs in a row terminate their
+// surplus containers idle at T (stable compaction).
+__device__ __forceinline__ void lane_pool_terminate(const ReplayParams& P, const LanePools& pl, int g, int m,
+                                                    int need, int64_t T) {
+  const size_t k = pl.pm(g, m);
+  const int n = pl.sz[k];
+  int surplus = n - need;
+  if (surplus <= 0) {
+    pl.ctr[k] = 0;
+    return;
+  }
+  if (++pl.ctr[k] < P.keepalive) return;
+  int64_t* b = pl.bu + k * kPoolCap;
+  int w = 0;
+  for (int i = 0; i < n; ++i) {
+    if (surplus > 0 && b[i] <= T) { --surplus; continue; }
+    b[w++] = b[i];
+  }
+  pl.sz[k] = w;
+  pl.ctr[k] = 0;
+}
+
 __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_kernel(ReplayParams P) {
   extern __shared__ __align__(16) unsigned char smem[];
   if (*(volatile const int*)P.ovf) return;  // the host replays the call on the fused engine
@@ -344,6 +402,12 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
   // the actual residents of GPU lane: 64 slots, lane-interleaved (slot i of lane l at i * 32 + l)
   // ga[i * 32]: end; ga[(64 + i) * 32]: packed word | co-runner FBR << 32 (one live base pointer)
   int64_t* ga = reinterpret_cast<int64_t*>(slot + P.o_alist) + lane;
+  const bool n3 = P.cold_us > 0;  // N3: container pools ahead of each actual placement
+  LanePools pl;
+  pl.M = P.tl.M;
+  pl.bu = reinterpret_cast<int64_t*>(slot + P.o_pool);
+  pl.sz = reinterpret_cast<int32_t*>(slot + P.o_pool + (size_t)N * pl.M * kPoolCap * 8);
+  pl.ctr = pl.sz + (size_t)N * pl.M;
   // fitm[j][m]: the slice positions of geometry j that hold model m's footprint (CTA-wide table)
   const uint8_t* fitm = smem + (((size_t)P.tl.words * 4 + 15) & ~(size_t)15) + (size_t)kChainWarps * CL.total;
   int64_t* sc_en = reinterpret_cast<int64_t*>(slot + P.o_clist) + lane;  // score_idle arrays
@@ -377,8 +441,10 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
       c.gi[4 * N + g] = 0;
       c.gi[8 * N + g] = c.gi[9 * N + g] = c.gi[10 * N + g] = c.gi[11 * N + g] = 0;
       c.gi[12 * N + g] = c.gi[13 * N + g] = 0;
+      if (n3) lane_pool_reset(P, pl, g);
     }
     int cursor = 0;
+    unsigned long long n_cold = 0;  // this lane's GPU's cold starts (N3)
     int64_t nlog = 0;
     unsigned long long n_recfg = 0, n_slot = 0, n_cand = 0;
 #pragma unroll 1
@@ -414,7 +480,8 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
             const int64_t tau = k * P.rev;
             if (k < 1 || tau >= P.H) continue;
             if (c.gu8[1 * N + g] != kNoGeom && c.gi[1 * N + g] <= tau) reset_gpu_state(c, g, c.gu8[1 * N + g]);
-            vm_event(P, c, replica, g, k, tau);
+            const bool lost = vm_event(P, c, replica, g, k, tau);
+            if (n3 && lost) lane_pool_reset(P, pl, g);  // its containers go with the VM (R27)
           }
         }
         if (c.gu8[1 * N + g] != kNoGeom && c.gi[1 * N + g] <= Tend) reset_gpu_state(c, g, c.gu8[1 * N + g]);
@@ -529,7 +596,13 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
           const uint32_t info = U.info[b];
           const int m = (info >> 16) & 0xFF;
           const bool strict = (info >> 24) & 1;
-          const int64_t t = (int64_t)U.ready[b];
+          int64_t t = (int64_t)U.ready[b];
+          int ci = -1;  // N3: the batch's container (R23; acquisition on the actual placement, R25)
+          if (n3) {
+            int64_t te;
+            ci = lane_pool_acquire(P, pl, g, m, t, &te, &n_cold);
+            t = te;
+          }
           const int32_t q = T.mem[m];
           int be = 0;  // best-effort footprint still running at t (Alg 1's tag walk)
 #pragma unroll 1
@@ -620,6 +693,7 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
             if (hi > bst) acc1 += (int64_t)q * (hi - bst);
             if (bend > bu) bug[s] = bend;
           }
+          if (n3 && ci >= 0) pl.bu[pl.pm(g, m) * kPoolCap + ci] = placed ? bend : t;  // R24
           const int drop = placed ? 0 : (overflow ? 3 : 2);
           bres[(size_t)e * kUB + b] = placed ? bend : -(int64_t)drop;
           if (P.log && nlog + b < P.log_cap) {
@@ -648,11 +722,26 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
         c.gi[10 * N + g] += acc0;
         c.gi[11 * N + g] += acc1;
       }
+      if (n3) {  // R26: delayed termination, every (GPU, model) of the epoch
+#pragma unroll 1
+        for (int g = lane; g < N; g += 32) {
+          const int x0 = c.g_off[g], cnt = c.g_off[g + 1] - x0;
+#pragma unroll 1
+          for (int m = 0; m < pl.M; ++m) {
+            int need = 0;
+            for (int x = 0; x < cnt; ++x) need += ((U.info[gl[x0 + x]] >> 16) & 0xFF) == (uint32_t)m ? 1 : 0;
+            lane_pool_terminate(P, pl, g, m, need, Tend);
+          }
+        }
+      }
       __syncwarp();
       cp_async_wait_all();
       __syncwarp();
-      // ---- candidate keys: cand.cu's (closed form) or scored here
-      const bool pre = P.policy == 0 && kfr && avail_all && kst[0] != INT64_MIN;
+      // ---- candidate keys: cand.cu's (closed form) or scored here.  The sentinel is read by
+      // lane 0 and broadcast: when it is set, the scoring below overwrites kst[0], and a lane
+      // still behind (ITS gives no lockstep after a __syncwarp) would otherwise read the key.
+      const bool pre = P.policy == 0 && kfr && avail_all &&
+                       __shfl_sync(0xffffffffu, (int)(kst[0] != INT64_MIN), 0) != 0;
       if (P.policy == 0 && !pre) {
 #pragma unroll 1
         for (int pi = lane; pi < N * G; pi += 32) {
@@ -786,6 +875,7 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
     for (int g = lane; g < N; g += 32) bill_switch(c, g, VM_NONE, P.H, P.H);
     __syncwarp();
     n_recfg = __reduce_add_sync(0xffffffffu, (unsigned)n_recfg);
+    n_cold = __reduce_add_sync(0xffffffffu, (unsigned)n_cold);
     if (lane == 0) {
       int64_t od = 0, spot = 0, busy = 0, memt = 0;
 #pragma unroll 1
@@ -808,7 +898,7 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
       P.util[2 * (size_t)r] = __ddiv_rn((double)busy, __dmul_rn(__dmul_rn(7.0, dN), dH));
       P.util[2 * (size_t)r + 1] = __ddiv_rn((double)memt, __dmul_rn(__dmul_rn((double)T.cap[4], dN), dH));
       if (P.n_batches) P.n_batches[r] = nlog;
-      if (P.cold_starts) P.cold_starts[r] = 0;
+      if (P.cold_starts) P.cold_starts[r] = (int64_t)n_cold;
     }
     __syncwarp();
   }

@@ -142,3 +142,35 @@ def test_lean_alg2_policy(oracle, monkeypatch, seed):
                t_low_milli=int(rng.integers(0, 2000)), t_high_milli=int(rng.integers(2000, 8000)))
     g = lean_replay(monkeypatch, P, tr, **cfg)
     compare(g, oracle_replay(oracle, P, tr, **cfg), tr.n_replicas)
+
+
+def test_lean_unheld_epoch_sentinel_race(oracle, monkeypatch):
+    """Regression: an epoch with every GPU available whose unit cand.cu did not hold (the
+    kfc[r][e][0][0] sentinel) makes the chain score it and overwrite kst[0]; a lane behind the
+    others used to read the key instead of the sentinel, take the other branch and deadlock the
+    warp in the reconfiguration cap's collectives.  The sentinel is now read once and broadcast."""
+    rng = np.random.default_rng(1301)
+    M = int(rng.integers(2, 6))
+    P = random_profiles(rng, M)
+    tr = uniform_trace(rng, 3, M, 8_000_000, 200)
+    N = int(rng.choice([2, 4]))
+    g = lean_replay(monkeypatch, P, tr, n_gpus=N)
+    compare(g, oracle_replay(oracle, P, tr, n_gpus=N), 3)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_lean_container_pools(oracle, monkeypatch, seed):
+    """N3 container pools (cold starts, keep-alive, pre-warm, readings R22-R27)
+    on the lean chain, lane = sim-GPU, with spot revocations taking a VM's containers (R27)."""
+    rng = np.random.default_rng(1300 + seed)
+    M = int(rng.integers(2, 6))
+    P = random_profiles(rng, M)
+    tr = uniform_trace(rng, 3, M, 8_000_000, 200)
+    N = int(rng.choice([2, 4]))
+    cfg = dict(n_gpus=N, cold_start_us=int(rng.integers(100_000, 3_000_000)),
+               keepalive_epochs=int(rng.integers(1, 5)), prewarm=int(rng.integers(0, 3)),
+               vm_policy=int(seed % 3), p_rev=0.5, rev_interval_us=2_000_000, notice_us=200_000, seed=seed)
+    g = lean_replay(monkeypatch, P, tr, **cfg)
+    o = oracle_replay(oracle, P, tr, **cfg)
+    assert int(np.sum(o["cold_starts"])) > 0
+    compare(g, o, 3)
