@@ -353,6 +353,9 @@ __device__ __forceinline__ void lane_pool_terminate(const ReplayParams& P, const
   pl.ctr[k] = 0;
 }
 
+// kN3: container pools (cold_us > 0).  A template argument so that the pool-free instantiation
+// carries none of the pool code (the runtime flag alone cost config 5's chain 13.4 -> 16.2 ms).
+template <bool kN3>
 __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_kernel(ReplayParams P) {
   extern __shared__ __align__(16) unsigned char smem[];
   if (*(volatile const int*)P.ovf) return;  // the host replays the call on the fused engine
@@ -402,7 +405,7 @@ __global__ void __launch_bounds__(32 * kChainWarps, PROTEAN_CHAIN_MINB) chain_ke
   // the actual residents of GPU lane: 64 slots, lane-interleaved (slot i of lane l at i * 32 + l)
   // ga[i * 32]: end; ga[(64 + i) * 32]: packed word | co-runner FBR << 32 (one live base pointer)
   int64_t* ga = reinterpret_cast<int64_t*>(slot + P.o_alist) + lane;
-  const bool n3 = P.cold_us > 0;  // N3: container pools ahead of each actual placement
+  constexpr bool n3 = kN3;  // N3: container pools ahead of each actual placement
   LanePools pl;
   pl.M = P.tl.M;
   pl.bu = reinterpret_cast<int64_t*>(slot + P.o_pool);
@@ -1087,13 +1090,17 @@ size_t chain_smem_bytes(const ReplayParams& P) {
 
 cudaError_t chain_occupancy(const ReplayParams& P, int* per_sm) {
   const size_t smem = chain_smem_bytes(P);
-  cudaError_t e = cudaFuncSetAttribute(chain_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  auto k = P.cold_us > 0 ? chain_kernel<true> : chain_kernel<false>;
+  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, chain_kernel, 32 * kChainWarps, smem);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, k, 32 * kChainWarps, smem);
 }
 
 cudaError_t launch_chain(const ReplayParams& P, int grid, cudaStream_t st) {
-  chain_kernel<<<grid, 32 * kChainWarps, chain_smem_bytes(P), st>>>(P);
+  if (P.cold_us > 0)
+    chain_kernel<true><<<grid, 32 * kChainWarps, chain_smem_bytes(P), st>>>(P);
+  else
+    chain_kernel<false><<<grid, 32 * kChainWarps, chain_smem_bytes(P), st>>>(P);
   return cudaGetLastError();
 }
 
@@ -1104,7 +1111,8 @@ cudaError_t launch_acct(const ReplayParams& P, cudaStream_t st) {
 
 cudaError_t preload_chain_kernels() {
   cudaFuncAttributes a;
-  cudaError_t e = cudaFuncGetAttributes(&a, chain_kernel);
+  cudaError_t e = cudaFuncGetAttributes(&a, chain_kernel<false>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, chain_kernel<true>);
   if (e != cudaSuccess) return e;
   return cudaFuncGetAttributes(&a, acct_kernel);
 }
