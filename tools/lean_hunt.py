@@ -2,7 +2,8 @@
 printing each seed before it runs (a hang names its seed) and every mismatch."""
 import os, sys, numpy as np
 sys.path.insert(0, os.getcwd()); sys.path.insert(0, os.path.join(os.getcwd(), "tests"))
-os.environ["PROTEAN_LEAN"] = "2"
+os.environ["PROTEAN_LEAN"] = os.environ.get("LEANV", "2")  # 0: the fused engine, "": auto
+if not os.environ["PROTEAN_LEAN"]: del os.environ["PROTEAN_LEAN"]
 from oracle import oracle as O; O.build()
 from gpu_common import compare, oracle_replay, GPU_LOG_DTYPE
 from test_gpu_lean import wide_case
