@@ -192,7 +192,11 @@ __device__ __forceinline__ int64_t key_of(int64_t misses, int64_t tail, int tag)
   return (misses << 40) | (tail << 8) | (int64_t)tag;
 }
 
+#ifdef PROTEAN_CAND_MINB  // experiment knob: minimum resident CTAs per SM (register cap)
+__global__ void __launch_bounds__(32 * kCandWarps, PROTEAN_CAND_MINB) cand_kernel(CandParams P) {
+#else
 __global__ void __launch_bounds__(32 * kCandWarps) cand_kernel(CandParams P) {
+#endif
   extern __shared__ __align__(16) unsigned char smem[];
   int32_t* tabw = reinterpret_cast<int32_t*>(smem);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;

@@ -28,4 +28,4 @@ for _ in range(4):
     ts.append(h.last_timings()[1])
 c = out["counters"].sum(0).cpu().tolist()
 print(json.dumps({"lib": os.path.basename(sys.argv[1]), "env": {k: v for k, v in os.environ.items() if k.startswith("PROTEAN")},
-                  "kernel_ms": [round(t, 3) for t in ts[1:]], "launch": h.last_timings()[2], "slot_evals": c[8]}))
+                  "kernel_ms": [round(t, 3) for t in ts[1:]], "search_walk_acct_ms": [round(t, 3) for t in h.last_search_ms()], "launch": h.last_timings()[2], "slot_evals": c[8]}))
