@@ -40,6 +40,7 @@ namespace pemgpu {
 namespace {
 
 constexpr int kBC = kUnitBats;  // batches per (replica, epoch) unit held in shared memory
+static_assert(kBC <= 64, "the id-order rank: two batches per lane");
 constexpr int kKC = 10;        // batches per residue class held per lane (config 5: ~5)
 constexpr int kCandWarps = 8;  // warps per CTA
 
@@ -349,17 +350,26 @@ __global__ void __launch_bounds__(32 * kCandWarps) cand_kernel(CandParams P) {
       continue;
     }
     // ---- id order (O3): rank by key
-#pragma unroll 1
-    for (int b = lane; b < nb; b += 32) {
-      const uint64_t kb = ws.key[b];
-      int rank = 0;
+    {  // nb <= kBC = 64: lane ranks batches lane and lane + 32 in one pass over the keys
+      const int b0 = lane, b1 = lane + 32;
+      const uint64_t k0 = b0 < nb ? ws.key[b0] : ~0ull, k1 = b1 < nb ? ws.key[b1] : ~0ull;
+      int r0 = 0, r1 = 0;
 #pragma unroll 4
-      for (int x = 0; x < nb; ++x) rank += ws.key[x] < kb ? 1 : 0;
-      ws.ord[rank] = (uint8_t)b;
-      if (ubu) {  // the epoch's batches in id order for the lean chain / accounting
-        ubu->ready[rank] = ws.ready[b];
-        ubu->info[rank] = ws.info[b];
-        ubu->pos[rank] = ws.pos[b];
+      for (int x = 0; x < nb; ++x) {
+        const uint64_t kx = ws.key[x];
+        r0 += kx < k0 ? 1 : 0;
+        r1 += kx < k1 ? 1 : 0;
+      }
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int b = h ? b1 : b0, rank = h ? r1 : r0;
+        if (b >= nb) continue;
+        ws.ord[rank] = (uint8_t)b;
+        if (ubu) {  // the epoch's batches in id order for the lean chain / accounting
+          ubu->ready[rank] = ws.ready[b];
+          ubu->info[rank] = ws.info[b];
+          ubu->pos[rank] = ws.pos[b];
+        }
       }
     }
     __syncwarp();
